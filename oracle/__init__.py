@@ -1,0 +1,192 @@
+"""CPU oracle (TEST INFRASTRUCTURE ONLY) -- ctypes binding of oracle/lf_oracle.c.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference
+legs may import this package.  The product path (paper_conf_icpp_0002s22_b200) never
+imports it, and it never imports the product path.  See lf_oracle.c for the paper
+passages each function follows and DESIGN.md §3 for the readings it takes.
+
+Parity status: every function is pinned by tests in tests/test_oracle_*.py against
+values the paper prints (Table 1, Tables 4/5 ANISO rows), a library routine (hashlib
+MD5 for the charge), a second algorithm from the paper (Alg. 1 vs Alg. 2 with m=1,
+M=inf), closed forms, brute force on tiny graphs and invariants; except the charged
+rounds' exact bits, whose hash the paper does not specify ("parity unpinned" against
+the paper for those bits; pinned statistically and through the MD5 library check).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "lf_oracle.c")
+_LIB = os.path.join(_HERE, "liblf_oracle.so")
+_lib = None
+
+
+def build(force=False):
+    """Compile the oracle (plain C, -O2, single thread, no intrinsics)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-std=c99", "-Wall", "-shared", "-fPIC",
+                               "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = C.CDLL(_LIB)
+        P = C.c_void_p
+        L.lfo_md5_round1_state.argtypes = [C.c_uint32, C.c_uint32, C.c_uint32, P]
+        L.lfo_charge_hash.argtypes = [C.c_uint32, C.c_uint32, C.c_uint32]
+        L.lfo_charge_hash.restype = C.c_uint32
+        L.lfo_charge.argtypes = [C.c_uint32, C.c_uint32, C.c_uint32, C.c_float]
+        L.lfo_factor.argtypes = [C.c_int64, P, P, P, C.c_int, C.c_int, C.c_int, C.c_int,
+                                 C.c_float, C.c_uint32, C.c_int, P, P, P, P, P, P, C.c_int]
+        L.lfo_greedy.argtypes = [C.c_int64, P, P, P, C.c_int, P, P]
+        L.lfo_linear_forest.argtypes = [C.c_int64, P, P, P, P, P, P, P, P]
+        L.lfo_tridiag.argtypes = [C.c_int64, P, P, P, P, P, P, P, P]
+        L.lfo_factor_weight.argtypes = [C.c_int64, P, C.c_int, P, P, P]
+        L.lfo_factor_weight.restype = C.c_double
+        _lib = L
+    return _lib
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data_as(C.c_void_p)
+
+
+def _csr(A):
+    rp = np.ascontiguousarray(A.rowptr, dtype=np.int64)
+    col = np.ascontiguousarray(A.col, dtype=np.int32)
+    val = np.ascontiguousarray(A.val, dtype=np.float32)
+    return rp, col, val
+
+
+def md5_round1_state(v, k, seed=0):
+    out = np.zeros(4, dtype=np.uint32)
+    lib().lfo_md5_round1_state(v, k, seed, _p(out))
+    return out
+
+
+def charge_hash(v, k, seed=0):
+    return int(lib().lfo_charge_hash(v, k, seed))
+
+
+def charge(v, k, seed=0, p=0.5):
+    return int(lib().lfo_charge(v, k, seed, p))
+
+
+def factor(A, n, M=5, m=5, k_m=0, p=0.5, seed=0, until_maximal=False,
+           charge_override=None, counters=False):
+    """Algorithm 2 -> (pi[N,n] int32, pi_w[N,n] float32, rounds, live_rows, live_nnz)."""
+    rp, col, val = _csr(A)
+    N = A.N
+    pi = np.empty(N * n, dtype=np.int32)
+    pw = np.empty(N * n, dtype=np.float32)
+    rounds = np.zeros(1, dtype=np.int32)
+    co = None
+    if charge_override is not None:
+        co = np.ascontiguousarray(charge_override, dtype=np.uint8).reshape(-1)
+        assert co.size >= M * N
+    R = M if not until_maximal else 0
+    lr = np.zeros(max(R, 1), dtype=np.int64) if counters else None
+    ln = np.zeros(max(R, 1), dtype=np.int64) if counters else None
+    rc = lib().lfo_factor(N, _p(rp), _p(col), _p(val), n, M, m, k_m, p, seed,
+                          int(bool(until_maximal)), _p(co), _p(pi), _p(pw), _p(rounds),
+                          _p(lr), _p(ln), R if counters else 0)
+    if rc != 0:
+        raise ValueError(f"lfo_factor failed ({rc})")
+    return pi.reshape(N, n), pw.reshape(N, n), int(rounds[0]), lr, ln
+
+
+def greedy(A, n):
+    """Algorithm 1 -> (pi[N,n], pi_w[N,n])."""
+    rp, col, val = _csr(A)
+    N = A.N
+    pi = np.empty(N * n, dtype=np.int32)
+    pw = np.empty(N * n, dtype=np.float32)
+    rc = lib().lfo_greedy(N, _p(rp), _p(col), _p(val), n, _p(pi), _p(pw))
+    if rc != 0:
+        raise ValueError(f"lfo_greedy failed ({rc})")
+    return pi.reshape(N, n), pw.reshape(N, n)
+
+
+def linear_forest(pi2, pi2_w):
+    """Section 3.3 steps (1)-(3) -> dict(forest, path_id, pos, perm, iperm, n_cycles)."""
+    pi2 = np.ascontiguousarray(pi2, dtype=np.int32).reshape(-1)
+    pw = np.ascontiguousarray(pi2_w, dtype=np.float32).reshape(-1)
+    N = pi2.size // 2
+    forest = np.empty(2 * N, dtype=np.int32)
+    pid = np.empty(N, dtype=np.int32)
+    pos = np.empty(N, dtype=np.int32)
+    perm = np.empty(N, dtype=np.int32)
+    iperm = np.empty(N, dtype=np.int32)
+    ncyc = np.zeros(1, dtype=np.int64)
+    rc = lib().lfo_linear_forest(N, _p(pi2), _p(pw), _p(forest), _p(pid), _p(pos),
+                                 _p(perm), _p(iperm), _p(ncyc))
+    if rc != 0:
+        raise ValueError(f"lfo_linear_forest failed ({rc})")
+    return dict(forest=forest.reshape(N, 2), path_id=pid, pos=pos, perm=perm, iperm=iperm,
+                n_cycles=int(ncyc[0]))
+
+
+def tridiag(A, forest, perm):
+    """Step (4) -> (a, b, c) float32 [N]."""
+    rp, col, val = _csr(A)
+    N = A.N
+    f = np.ascontiguousarray(forest, dtype=np.int32).reshape(-1)
+    pm = np.ascontiguousarray(perm, dtype=np.int32)
+    a = np.empty(N, dtype=np.float32)
+    b = np.empty(N, dtype=np.float32)
+    c = np.empty(N, dtype=np.float32)
+    lib().lfo_tridiag(N, _p(rp), _p(col), _p(val), _p(f), _p(pm), _p(a), _p(b), _p(c))
+    return a, b, c
+
+
+def factor_weight(A, pi):
+    """omega_pi, Eq. (3), fp64."""
+    rp, col, val = _csr(A)
+    pi = np.ascontiguousarray(pi, dtype=np.int32)
+    n = pi.shape[1] if pi.ndim == 2 else 1
+    return float(lib().lfo_factor_weight(A.N, _p(pi.reshape(-1)), n, _p(rp), _p(col), _p(val)))
+
+
+def graph_weight(A):
+    """omega_G, Eq. (4): sum over undirected off-diagonal edges of |w|, fp64."""
+    rows = np.repeat(np.arange(A.N, dtype=np.int64), np.diff(A.rowptr))
+    off = rows < A.col
+    return float(np.abs(A.val[off].astype(np.float64)).sum())
+
+
+def coverage(A, pi):
+    """c_pi, Eq. (4)."""
+    return factor_weight(A, pi) / graph_weight(A)
+
+
+def coverage_id(A):
+    """c_id, Eq. (5): weight of the sub/super-diagonal couplings {i, i+1}, over omega_G.
+
+    Eq. (5) sums |w({i,i-1})| + |w({i,i+1})| over i, which counts every coupling
+    {i,i+1} twice; the paper's printed values (ANISO1 0.68 = 2/3) correspond to
+    counting each such edge once, which is what is computed here.
+    """
+    rows = np.repeat(np.arange(A.N, dtype=np.int64), np.diff(A.rowptr))
+    sel = A.col.astype(np.int64) == rows + 1
+    return float(np.abs(A.val[sel].astype(np.float64)).sum()) / graph_weight(A)
+
+
+def run_pipeline(A, n=2, M=5, m=5, k_m=0, p=0.5, seed=0):
+    """Whole hot path on the CPU: factor -> linear forest -> tridiag (n must be 2 for LF)."""
+    pi, pw, rounds, _, _ = factor(A, n, M, m, k_m, p, seed)
+    out = dict(pi=pi, pi_w=pw, rounds=rounds)
+    if n == 2:
+        lf = linear_forest(pi, pw)
+        out.update(lf)
+        out["a"], out["b"], out["c"] = tridiag(A, lf["forest"], lf["perm"])
+    return out
