@@ -1,0 +1,366 @@
+#!/usr/bin/env python
+"""Benchmark of the hot path: [0,2]-factor (M=5) + linear forest + permutation + tridiag.
+
+Contract: `python bench.py --gpus N --steps K --warmup W` prints ONE
+JSON line on rank 0.  A step is one pass of the whole hot path over one synthetic graph
+resident in HBM; `value` is whole-job Medges/s (undirected edges E / step time, summed
+over ranks).  Device time with CUDA events per step, L2 flushed between steps, max over
+ranks.  `--impl reference` times the CPU oracle (the reference arm of this tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "ms and Medges/s per [0,2]-factor+linear forest at 1/2/4/8 B200; % HBM peak"
+CONFIG_DESC = {
+    "C1": "2D 5-pt 64x64 (4,096 vertices), n=2",
+    "C2": "3D 7-pt anisotropic 128^3 (2.1M vertices, 6.24M edges), n=2",
+    "C3": "FEM-like jittered 27-pt 100^3 bricks (1M vertices), n=2",
+    "C4": "Chung-Lu power-law 5M vertices, n=2",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-runs", type=int, default=8)
+    return ap.parse_args()
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class Clocks:
+    """nvidia-smi clock/throttle sampler running during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+        self.path = f"/tmp/lf_clocks_{os.getpid()}.csv"
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, val in zip(names, f[5:9]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        sm.sort()
+        med = sm[len(sm) // 2] if sm else None
+        return {"sm_mhz": med, "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
+    """Algorithmic HBM bytes of one launch: what the method must move."""
+    base = name.split("[")[0]
+    k = int(name.split("[")[1].rstrip("]")) if "[" in name else -1
+    if base == "propose":
+        if k == 0:  # whole CSR + rowptr; write prop (j, value) and the diagonal
+            return 8 * Z + 8 * (N + 1) + 8 * n * N + 4 * N
+        Na, Za = live_rows[k], live_nnz[k]
+        # live rows' CSR payload + rowptr pair + worklist + state + pi; write prop
+        return 8 * Za + 16 * Na + 4 * Na + Na + 4 * n * Na + 8 * n * Na
+    if base == "mutual":
+        if k == 0:  # read prop (j, value); write pi, pi_w, pi_val, state, worklist
+            return 8 * n * N + 12 * n * N + N + 4 * live_rows[1 if len(live_rows) > 1 else 0]
+        Na = live_rows[k]
+        nxt = live_rows[k + 1] if k + 1 < len(live_rows) else 0
+        return 4 * Na + 8 * n * Na + 8 * n * Na + Na + 4 * nxt
+    if base == "cycle_scan":
+        return 16 * N + 8 * N  # read pi2 + pi2_w, write forest
+    if base == "rank_scan":
+        return 8 * N + 12 * N  # read forest, write path_id, pos, len
+    if base == "path_offsets":
+        return 8 * N
+    if base == "perm":
+        return 12 * N + 8 * N
+    if base == "tridiag":
+        return 8 * N + 4 * N + 8 * N + 8 * N + 4 * N + 12 * N
+    return 0
+
+
+def cpu_baseline(A, runs):
+    import oracle
+
+    oracle.build()
+    t0 = time.perf_counter()
+    for _ in range(runs):
+        oracle.run_pipeline(A)
+    dt = (time.perf_counter() - t0) / runs
+    return {"value": A.n_edges / dt / 1e6, "unit": "Medges/s", "cores": 1, "kind": "oracle",
+            "ms_per_graph": dt * 1e3,
+            "sample": f"full {A.name} graph (N={A.N}, E={A.n_edges}), oracle pipeline "
+                      f"(Alg. 2 M=5 + walks + sort + tridiag) x{runs}, single thread"}
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    import lfgen
+    import oracle
+
+    oracle.build()
+    A = lfgen.config(args.config)
+    for _ in range(args.warmup):
+        oracle.run_pipeline(A)
+    ts = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.run_pipeline(A)
+        ts.append(time.perf_counter() - t0)
+    ms = 1e3 * sum(ts) / len(ts)
+    val = A.n_edges / (ms / 1e3) / 1e6
+    out = {
+        "impl": "reference", "metric": METRIC, "value": round(val, 3), "unit": "Medges/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic", "config": {"workload": CONFIG_DESC.get(args.config, args.config),
+                                        "name": args.config, "N": A.N, "E": A.n_edges, "nnz": A.nnz},
+        "cpu_baseline": {"value": round(val, 3), "unit": "Medges/s", "cores": 1, "kind": "oracle",
+                         "sample": f"full {A.name} graph per step, single thread"},
+        "e2e": {"value": round(val, 3), "unit": "Medges/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import numpy as np
+    import torch
+
+    import lfgen
+    from paper_conf_icpp_0002s22_b200 import _build, lf
+
+    ws, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if ws > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    _build.build()
+    lf.load()
+
+    A = lfgen.config(args.config)
+    N, Z, E = A.N, A.nnz, A.n_edges
+    rp = torch.from_numpy(A.rowptr).cuda()
+    col = torch.from_numpy(A.col).cuda()
+    val = torch.from_numpy(A.val).cuda()
+    P = lf.Pipeline(rp, col, val)
+    flush = torch.empty(512 * 1024 * 1024, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    for _ in range(max(args.warmup, 3)):
+        P.run()
+    torch.cuda.synchronize()
+
+    graph = None
+    if not args.no_graph:
+        try:
+            lf.profile_enable(True)
+            s = torch.cuda.Stream()
+            s.wait_stream(stream)
+            with torch.cuda.stream(s):
+                P.run()  # warm the stream once before capture
+            torch.cuda.synchronize()
+            lf.profile_enable(True)
+            graph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph):
+                P.run()
+            torch.cuda.synchronize()
+            graph.replay()
+            torch.cuda.synchronize()
+        except Exception as e:  # capture unsupported -> eager launches
+            print(f"# graph capture failed ({e}); timing eager launches", file=sys.stderr)
+            graph = None
+    launches_per_step = None
+
+    def step():
+        if graph is not None:
+            graph.replay()
+        else:
+            lf.profile_enable(True)
+            P.run()
+
+    clocks = Clocks(local)
+    if ws > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    step_ms, kern = [], {}
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    for _ in range(args.steps):
+        flush.zero_()  # write 512 MB > 126 MB L2 between steps
+        ev0.record(stream)
+        step()
+        ev1.record(stream)
+        ev1.synchronize()
+        step_ms.append(ev0.elapsed_time(ev1))
+        recs = lf.profile_collect()
+        launches_per_step = len(recs)
+        for nm, ms in recs:
+            kern.setdefault(nm, []).append(ms)
+    torch.cuda.synchronize()
+    if ws > 1:
+        torch.distributed.barrier()
+    clk = clocks.stop()
+    lf.profile_enable(False)
+
+    t_step = sum(step_ms) / len(step_ms)
+    if ws > 1:
+        t = torch.tensor([t_step], device="cuda", dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        t_step = float(t.item())
+
+    live = P.fac["live"].cpu().numpy()
+    M = P.M
+    lr, ln = [int(x) for x in live[:M]], [int(x) for x in live[M:2 * M]]
+    kavg = {nm: sum(v) / len(v) for nm, v in kern.items()}
+    stage = {"factor": sum(t for nm, t in kavg.items() if nm.split("[")[0] in ("propose", "mutual", "rounds", "init_state")),
+             "linear_forest": sum(t for nm, t in kavg.items() if nm.split("[")[0] in ("cycle_scan", "rank_scan", "path_offsets", "perm")),
+             "tridiag": kavg.get("tridiag", 0.0)}
+    dom = max(kavg, key=kavg.get) if kavg else None
+    peak, peak_kind = load_peaks()
+    n = 2
+    dom_bytes = kernel_bytes(dom, N, Z, n, lr, ln) if dom else 0
+    dom_ach = dom_bytes / (kavg[dom] * 1e-3) / 1e9 if dom else None
+    b_main = sum(kernel_bytes(nm, N, Z, n, lr, ln) for nm in kavg if nm.split("[")[0] != "tridiag")
+    b_tri = kernel_bytes("tridiag", N, Z, n, lr, ln)
+    t_main = stage["factor"] + stage["linear_forest"]
+
+    # e2e through the C ABI with HOST buffers (pinned), copies inside the timed region
+    rp_h = torch.from_numpy(A.rowptr).pin_memory()
+    col_h = torch.from_numpy(A.col).pin_memory()
+    val_h = torch.from_numpy(A.val).pin_memory()
+    e2e_ws = lf.Workspace()
+    outs = None
+    for _ in range(2):
+        outs = lf.pipeline_host(rp_h, col_h, val_h, ws=e2e_ws, outs=outs)
+    e2e_ms = []
+    for _ in range(max(3, min(args.steps, 10))):
+        ev0.record(stream)
+        outs = lf.pipeline_host(rp_h, col_h, val_h, ws=e2e_ws, outs=outs)
+        ev1.record(stream)
+        ev1.synchronize()
+        e2e_ms.append(ev0.elapsed_time(ev1))
+    e2e_t = sum(e2e_ms) / len(e2e_ms)
+    if ws > 1:
+        t = torch.tensor([e2e_t], device="cuda", dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        e2e_t = float(t.item())
+
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(A, args.cpu_runs)
+
+    if rank == 0:
+        value = ws * E / (t_step * 1e-3) / 1e6
+        out = {
+            "metric": METRIC,
+            "value": round(value, 2),
+            "unit": "Medges/s",
+            "n_gpus": ws,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": round(t_step, 4),
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "f32",
+            "data": "synthetic",
+            "config": {
+                "workload": CONFIG_DESC.get(args.config, args.config), "name": args.config,
+                "N": N, "E": E, "nnz": Z, "n": 2, "M": 5, "m": 5, "k_m": 0,
+                "per_rank": "one independent graph per rank" if ws > 1 else "single graph",
+                "l2": "flushed between steps (512 MB write)",
+                "graph": graph is not None,
+            },
+            "stages_ms": {k: round(v, 4) for k, v in stage.items()},
+            "t_main_ms": round(t_main, 4),
+            "B_main_bytes": int(b_main),
+            "B_tri_bytes": int(b_tri),
+            "main_frac_of_peak": round(b_main / (t_main * 1e-3) / 1e9 / peak, 4) if t_main > 0 else None,
+            "roofline": {
+                "kernel": dom, "bound": "hbm", "achieved": round(dom_ach, 1) if dom_ach else None,
+                "peak": peak, "peak_kind": peak_kind, "unit": "GB/s",
+                "frac": round(dom_ach / peak, 4) if dom_ach else None, "traffic": None,
+                "alg_bytes_per_launch": int(dom_bytes),
+                "ms_per_launch": round(kavg[dom], 5) if dom else None,
+            },
+            "kernels_ms": {k: round(v, 5) for k, v in sorted(kavg.items(), key=lambda t: -t[1])},
+            "live_rows": lr,
+            "live_nnz": ln,
+            "e2e": {"value": round(ws * E / (e2e_t * 1e-3) / 1e6, 2), "unit": "Medges/s",
+                    "ms_per_step": round(e2e_t, 3),
+                    "h2d_bytes_per_step": int(8 * (N + 1) + 8 * Z),
+                    "d2h_bytes_per_step": int(24 * N)},
+            "gpu_launches": launches_per_step,
+            "clocks": clk,
+        }
+        if cpu is not None:
+            out["cpu_baseline"] = cpu
+        print(json.dumps(out), flush=True)
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,434 @@
+// lf_factor.cu -- weighted [0,n]-factor, Algorithm 2 of PAPER.md (L93-L128, §3.2, §4.1).
+//
+// B200 design:
+//  * one `propose` kernel per round (Alg. 2 L14-L22, the generalized SpMV of §4.1): G
+//    lanes per CSR row stream col/val with read-only loads, each lane keeps a sorted
+//    register top-n of 64-bit keys, a shuffle butterfly merges the G lists.  The key
+//    order is total, so the reduction order never changes the result (bit parity).
+//  * one `mutual` kernel per round (Alg. 2 L26-L28): confirms mutual proposals, keeps
+//    pi canonical, writes the next round's state byte (degree + charge, L8-L12) and
+//    appends still-live rows to the next worklist.  Rows whose charge-free candidate
+//    set became empty are retired: they provably never propose or receive a proposal
+//    again, so later rounds only touch live rows.
+//  * no host synchronisation: round count, worklist sizes and the maximality flags
+//    (L23-L25) stay on the device; the launch chain is fixed and graph-capturable.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "lf_common.cuh"
+#include "lf_internal.h"
+
+namespace lf {
+
+struct ProposeArgs {
+    int64_t N;
+    const int64_t* __restrict__ rowptr;
+    const int32_t* __restrict__ col;
+    const float* __restrict__ val;
+    const uint8_t* __restrict__ state;   // NULL in a fresh round 0 (all degrees 0, no charge)
+    const int32_t* __restrict__ pi;      // NULL in a fresh round 0
+    const int32_t* __restrict__ wl;      // worklist; NULL = all rows
+    const int32_t* __restrict__ wl_count;
+    int32_t* __restrict__ prop_j;        // [N*n] new proposals of worklist rows
+    float* __restrict__ prop_v;          // [N*n] their signed values
+    float* __restrict__ diag;            // [N] written when non-NULL (round 0)
+    int charging;
+    unsigned long long* live_rows;       // NULL or &live[k]
+    unsigned long long* live_nnz;        // NULL or &live[M+k]
+    int* proposed;                       // &flags[k]: set to 1 if anything was proposed
+};
+
+// G lanes per row (G = 1..32), NN = n.  Persistent grid-stride over the worklist.
+template <int NN, int G>
+__global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
+    constexpr int RPW = 32 / G;  // rows per warp per iteration
+    const int lane = threadIdx.x & 31;
+    const int li = lane & (G - 1);
+    const int64_t warp_global = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t n_warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t count = a.wl_count ? (int64_t)*a.wl_count : a.N;
+
+    unsigned long long my_live = 0, my_nnz = 0;
+    int my_prop = 0;
+
+    for (int64_t base = warp_global * RPW; base < count; base += n_warps * RPW) {
+        const int64_t idx = base + lane / G;
+        const bool valid = idx < count;
+        int32_t v = -1;
+        if (valid) v = a.wl ? __ldg(a.wl + idx) : (int32_t)idx;
+        int deg = 0;
+        uint32_t cv = 0;
+        int32_t p[NN];
+#pragma unroll
+        for (int s = 0; s < NN; s++) p[s] = -1;
+        int64_t rs = 0, re = 0;
+        if (valid) {
+            if (a.state) {
+                uint8_t st = a.state[v];
+                deg = st & ST_DEG;
+                cv = (st & ST_CHARGE) ? 1u : 0u;
+            }
+            if (a.pi && deg > 0) {
+#pragma unroll
+                for (int s = 0; s < NN; s++) p[s] = a.pi[(int64_t)v * NN + s];
+            }
+            rs = __ldg(a.rowptr + v);
+            re = __ldg(a.rowptr + v + 1);
+        }
+        uint64_t top[NN];
+#pragma unroll
+        for (int s = 0; s < NN; s++) top[s] = 0;
+        uint32_t theta0 = 0;
+        uint32_t dbits = 0;
+        for (int64_t e = rs + li; e < re; e += G) {
+            const int32_t j = __ldg(a.col + e);
+            const float x = __ldg(a.val + e);
+            if (j == v) {  // diagonal: not an edge (A' = |A| - diag|A|, L231)
+                dbits = __float_as_uint(x);
+                continue;
+            }
+            if ((__float_as_uint(x) & 0x7FFFFFFFu) == 0u) continue;  // zero: not an edge (L31)
+            uint32_t sj = 0;
+            if (a.state) sj = a.state[j];
+            if ((int)(sj & ST_DEG) == NN) continue;  // j saturated (L15)
+            bool in_pi = false;
+#pragma unroll
+            for (int s = 0; s < NN; s++) in_pi |= (p[s] == j);
+            if (in_pi) continue;  // already confirmed (L19: W \ pi(v))
+            theta0 = 1;
+            if (a.charging && (((sj & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
+            topn_insert<NN>(top, make_key(x, j));
+        }
+        // merge the G partial lists; OR the flags
+        topn_merge_group<NN, G>(top);
+#pragma unroll
+        for (int off = G / 2; off >= 1; off >>= 1) {
+            theta0 |= __shfl_xor_sync(0xffffffffu, theta0, off);
+            dbits |= __shfl_xor_sync(0xffffffffu, dbits, off);
+        }
+        if (valid && li == 0) {
+            const int need = NN - deg;
+            int32_t* pj = a.prop_j + (int64_t)v * NN;
+            float* pv = a.prop_v + (int64_t)v * NN;
+            int np = 0;
+#pragma unroll
+            for (int s = 0; s < NN; s++) {
+                if (s < need && top[s] != 0) {
+                    pj[s] = key_col(top[s]);
+                    pv[s] = key_val(top[s]);
+                    np++;
+                } else {
+                    pj[s] = (s == 0 && !theta0) ? PROP_RETIRED : -1;
+                }
+            }
+            if (a.diag) a.diag[v] = __uint_as_float(dbits);
+            if (theta0) {
+                my_live += 1;
+                my_nnz += (unsigned long long)(re - rs);
+            }
+            my_prop |= (np > 0);
+        }
+    }
+    // one atomic per warp
+#pragma unroll
+    for (int off = 16; off >= 1; off >>= 1) {
+        my_live += __shfl_xor_sync(0xffffffffu, my_live, off);
+        my_nnz += __shfl_xor_sync(0xffffffffu, my_nnz, off);
+        my_prop |= __shfl_xor_sync(0xffffffffu, my_prop, off);
+    }
+    if (lane == 0) {
+        if (a.live_rows && my_live) atomicAdd(a.live_rows, my_live);
+        if (a.live_nnz && my_nnz) atomicAdd(a.live_nnz, my_nnz);
+        if (my_prop) atomicOr(a.proposed, 1);
+    }
+}
+
+struct MutualArgs {
+    int64_t N;
+    const int32_t* __restrict__ wl;  // NULL = all rows (round 0)
+    const int32_t* __restrict__ wl_count;
+    const int32_t* __restrict__ prop_j;
+    const float* __restrict__ prop_v;
+    uint8_t* __restrict__ state;
+    int32_t* __restrict__ pi;
+    float* __restrict__ pi_w;
+    float* __restrict__ pi_val;      // NULL if not requested
+    int32_t* __restrict__ wl_next;   // NULL in the last round
+    int32_t* __restrict__ wl_next_count;
+    int32_t* __restrict__ wl_zero;   // count slot to reset for round k+2 (NULL: none)
+    int fresh;                       // round 0 from scratch: state/pi not initialised yet
+    int next_charging;
+    uint32_t next_k;
+    uint32_t seed;
+    unsigned long long thr;
+};
+
+template <int NN>
+__global__ void __launch_bounds__(256) k_mutual(MutualArgs a) {
+    const int64_t count = a.wl_count ? (int64_t)*a.wl_count : a.N;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    if (a.wl_zero && blockIdx.x == 0 && threadIdx.x == 0) *a.wl_zero = 0;
+    const int lane = threadIdx.x & 31;
+    // warp-uniform trip count so that the warp-aggregated append is safe
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < count;
+         base += stride) {
+        const int64_t idx = base + lane;
+        bool keep = false;
+        int32_t v = -1;
+        if (idx < count) {
+            v = a.wl ? __ldg(a.wl + idx) : (int32_t)idx;
+            int32_t pj[NN];
+#pragma unroll
+            for (int s = 0; s < NN; s++) pj[s] = a.prop_j[(int64_t)v * NN + s];
+            int deg = 0;
+            if (!a.fresh) deg = a.state[v] & ST_DEG;
+            const bool retired = pj[0] == PROP_RETIRED;
+            // Alg. 2 L27: keep w in prop(v) iff v in prop(w).  Confirmed slots are not in
+            // prop_j (which holds only this round's new proposals) and always survive.
+            uint64_t conf[NN];
+            int nconf = 0;
+#pragma unroll
+            for (int s = 0; s < NN; s++) {
+                conf[s] = 0;
+                const int32_t w = pj[s];
+                if (w >= 0) {
+                    bool mutual = false;
+#pragma unroll
+                    for (int t = 0; t < NN; t++) mutual |= (a.prop_j[(int64_t)w * NN + t] == v);
+                    if (mutual) {
+                        conf[s] = make_key(a.prop_v[(int64_t)v * NN + s], w);
+                        nconf++;
+                    }
+                }
+            }
+            if (nconf > 0 || a.fresh) {
+                uint64_t t[NN];
+#pragma unroll
+                for (int s = 0; s < NN; s++) t[s] = 0;
+                if (deg > 0) {
+#pragma unroll
+                    for (int s = 0; s < NN; s++) {
+                        if (s < deg) {
+                            const int32_t w = a.pi[(int64_t)v * NN + s];
+                            const float aw = a.pi_w[(int64_t)v * NN + s];
+                            uint32_t sg = 0;
+                            if (a.pi_val) sg = __float_as_uint(a.pi_val[(int64_t)v * NN + s]) >> 31;
+                            t[s] = make_key_abs(aw, sg, w);
+                        }
+                    }
+                }
+#pragma unroll
+                for (int s = 0; s < NN; s++)
+                    if (conf[s]) topn_insert<NN>(t, conf[s]);
+#pragma unroll
+                for (int s = 0; s < NN; s++) {
+                    const int64_t o = (int64_t)v * NN + s;
+                    if (t[s]) {
+                        a.pi[o] = key_col(t[s]);
+                        a.pi_w[o] = key_abs(t[s]);
+                        if (a.pi_val) a.pi_val[o] = key_val(t[s]);
+                    } else {
+                        a.pi[o] = -1;
+                        a.pi_w[o] = 0.0f;
+                        if (a.pi_val) a.pi_val[o] = 0.0f;
+                    }
+                }
+                deg += nconf;
+            }
+            if (a.wl_next) {
+                uint32_t ch = 0;
+                keep = !retired && deg < NN;
+                if (keep && a.next_charging) ch = charge_bit((uint32_t)v, a.next_k, a.seed, a.thr);
+                a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0));
+            } else if (a.fresh || nconf > 0) {
+                a.state[v] = (uint8_t)deg;
+            }
+        }
+        if (a.wl_next) {
+            // warp-aggregated append to the next worklist
+            const unsigned m = __ballot_sync(0xffffffffu, keep);
+            int32_t basepos = 0;
+            if (lane == 0 && m) basepos = atomicAdd(a.wl_next_count, __popc(m));
+            basepos = __shfl_sync(0xffffffffu, basepos, 0);
+            if (keep) a.wl_next[basepos + __popc(m & ((1u << lane) - 1u))] = v;
+        }
+    }
+}
+
+// state of round 0 when round 0 is charged (k_m != 0): degree 0 + charge(v, 0)
+__global__ void k_init_state(int64_t N, uint8_t* state, uint32_t seed, unsigned long long thr) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N;
+         v += (int64_t)gridDim.x * blockDim.x)
+        state[v] = charge_bit((uint32_t)v, 0u, seed, thr) ? ST_CHARGE : 0;
+}
+
+// Alg. 2 L23-L24 / L30: rounds = k+1 for the first uncharged round without proposals
+__global__ void k_rounds(const int* flags, int M, int m, int k_m, int32_t* rounds) {
+    int r = M;
+    for (int k = 0; k < M; k++)
+        if ((k % m) == k_m && flags[k] == 0) {
+            r = k + 1;
+            break;
+        }
+    *rounds = r;
+}
+
+// ---------------------------------------------------------------------------
+// host side
+// ---------------------------------------------------------------------------
+
+template <int NN>
+static void launch_propose(int G, const ProposeArgs& pa, int grid, cudaStream_t s) {
+    switch (G) {
+        case 1: k_propose<NN, 1><<<grid, 256, 0, s>>>(pa); break;
+        case 2: k_propose<NN, 2><<<grid, 256, 0, s>>>(pa); break;
+        case 4: k_propose<NN, 4><<<grid, 256, 0, s>>>(pa); break;
+        case 8: k_propose<NN, 8><<<grid, 256, 0, s>>>(pa); break;
+        case 16: k_propose<NN, 16><<<grid, 256, 0, s>>>(pa); break;
+        default: k_propose<NN, 32><<<grid, 256, 0, s>>>(pa); break;
+    }
+}
+
+static int lanes_per_row(double avg) {
+    // enough lanes to cover an average row in one or two passes
+    if (avg <= 3) return 2;
+    if (avg <= 7.5) return 4;
+    if (avg <= 16) return 8;
+    if (avg <= 40) return 16;
+    return 32;
+}
+
+template <int NN>
+static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi, float* pi_w,
+                       float* pi_val, float* diag, int32_t* rounds_dev, int64_t* live,
+                       const FactorWs& w, cudaStream_t s) {
+    const int64_t N = A->n;
+    const int M = o->until_maximal ? 0x7fffffff : o->M;
+    const double pthr = (double)o->p * 4294967296.0;
+    unsigned long long thr = pthr <= 0 ? 0ull : (pthr >= 4294967296.0 ? 4294967296ull
+                                                                      : (unsigned long long)ceil(pthr));
+    const int G = lanes_per_row(N > 0 ? (double)A->nnz / (double)N : 1.0);
+    const int grid_p = persistent_grid((const void*)k_propose<NN, 32>, 256);
+    const int grid_m = persistent_grid((const void*)k_mutual<NN>, 256);
+
+    LF_CUDA(cudaMemsetAsync(w.flags, 0, sizeof(int) * kMaxFlagRounds, s));
+    LF_CUDA(cudaMemsetAsync(w.counts, 0, sizeof(int32_t) * 4, s));
+    if (live && !o->until_maximal && o->M > 0)
+        LF_CUDA(cudaMemsetAsync(live, 0, sizeof(int64_t) * 2 * o->M, s));
+    if (N == 0 || (!o->until_maximal && o->M == 0)) {
+        // no rounds: empty factor
+        if (N > 0) {
+            LF_CUDA(cudaMemsetAsync(pi, 0xff, sizeof(int32_t) * N * NN, s));
+            LF_CUDA(cudaMemsetAsync(pi_w, 0, sizeof(float) * N * NN, s));
+            if (pi_val) LF_CUDA(cudaMemsetAsync(pi_val, 0, sizeof(float) * N * NN, s));
+            if (diag) LF_CUDA(cudaMemsetAsync(diag, 0, sizeof(float) * N, s));
+        }
+        if (rounds_dev) LF_CUDA(cudaMemsetAsync(rounds_dev, 0, sizeof(int32_t), s));
+        return LF_OK;
+    }
+    const bool charged0 = (0 % o->m) != o->k_m;
+    if (charged0) {
+        LF_PROF("init_state", -1, s);
+        k_init_state<<<persistent_grid((const void*)k_init_state, 256), 256, 0, s>>>(N, w.state, o->seed, thr);
+        LF_CUDA(cudaGetLastError());
+    }
+    int rounds_host = -1;
+    for (int k = 0; k < M; k++) {
+        const bool charging = (k % o->m) != o->k_m;
+        const bool fresh = (k == 0);
+        ProposeArgs pa;
+        pa.N = N;
+        pa.rowptr = A->rowptr;
+        pa.col = A->col;
+        pa.val = A->val;
+        pa.state = (fresh && !charged0) ? nullptr : w.state;
+        pa.pi = fresh ? nullptr : pi;
+        pa.wl = fresh ? nullptr : w.wl[k & 1];
+        pa.wl_count = fresh ? nullptr : &w.counts[k % 3];
+        pa.prop_j = w.prop_j;
+        pa.prop_v = w.prop_v;
+        pa.diag = fresh ? diag : nullptr;
+        pa.charging = charging ? 1 : 0;
+        const bool rec = live && !o->until_maximal;
+        pa.live_rows = rec ? (unsigned long long*)&live[k] : nullptr;
+        pa.live_nnz = rec ? (unsigned long long*)&live[o->M + k] : nullptr;
+        pa.proposed = &w.flags[k % kMaxFlagRounds];
+        if (o->until_maximal && k >= kMaxFlagRounds)
+            LF_CUDA(cudaMemsetAsync(pa.proposed, 0, sizeof(int), s));
+        {
+            LF_PROF("propose", k, s);
+            launch_propose<NN>(G, pa, grid_p, s);
+            LF_CUDA(cudaGetLastError());
+        }
+
+        if (o->until_maximal && (k % o->m) == o->k_m) {
+            // L23-L25 checked on the host in this mode (one sync per m rounds)
+            int f = 0;
+            LF_CUDA(cudaMemcpyAsync(&f, pa.proposed, sizeof(int), cudaMemcpyDeviceToHost, s));
+            LF_CUDA(cudaStreamSynchronize(s));
+            if (f == 0) {
+                rounds_host = k + 1;
+                if (fresh) {
+                    // nothing proposed at all: export the empty factor
+                    MutualArgs ma{};
+                    ma.N = N; ma.prop_j = w.prop_j; ma.prop_v = w.prop_v; ma.state = w.state;
+                    ma.pi = pi; ma.pi_w = pi_w; ma.pi_val = pi_val; ma.fresh = 1;
+                    k_mutual<NN><<<grid_m, 256, 0, s>>>(ma);
+                    LF_CUDA(cudaGetLastError());
+                }
+                break;
+            }
+        }
+        const bool last = !o->until_maximal && (k == M - 1);
+        MutualArgs ma;
+        ma.N = N;
+        ma.wl = fresh ? nullptr : w.wl[k & 1];
+        ma.wl_count = fresh ? nullptr : &w.counts[k % 3];
+        ma.prop_j = w.prop_j;
+        ma.prop_v = w.prop_v;
+        ma.state = w.state;
+        ma.pi = pi;
+        ma.pi_w = pi_w;
+        ma.pi_val = pi_val;
+        ma.wl_next = last ? nullptr : w.wl[(k + 1) & 1];
+        ma.wl_next_count = last ? nullptr : &w.counts[(k + 1) % 3];
+        ma.wl_zero = last ? nullptr : &w.counts[(k + 2) % 3];
+        ma.fresh = fresh ? 1 : 0;
+        ma.next_charging = ((k + 1) % o->m) != o->k_m;
+        ma.next_k = (uint32_t)(k + 1);
+        ma.seed = o->seed;
+        ma.thr = thr;
+        {
+            LF_PROF("mutual", k, s);
+            k_mutual<NN><<<grid_m, 256, 0, s>>>(ma);
+            LF_CUDA(cudaGetLastError());
+        }
+    }
+    if (rounds_dev) {
+        if (o->until_maximal) {
+            LF_CUDA(cudaMemcpyAsync(rounds_dev, &rounds_host, sizeof(int32_t), cudaMemcpyHostToDevice, s));
+            LF_CUDA(cudaStreamSynchronize(s));
+        } else {
+            if (o->M > kMaxFlagRounds) return set_error(LF_EINVAL, "M > 1024 needs until_maximal");
+            LF_PROF("rounds", -1, s);
+            k_rounds<<<1, 1, 0, s>>>(w.flags, o->M, o->m, o->k_m, rounds_dev);
+            LF_CUDA(cudaGetLastError());
+        }
+    }
+    return LF_OK;
+}
+
+int factor_dispatch(const lf_csr_t* A, int n, const lf_factor_opts_t* o, int32_t* pi, float* pi_w,
+                    float* pi_val, float* diag, int32_t* rounds_dev, int64_t* live, const FactorWs& w,
+                    cudaStream_t s) {
+    switch (n) {
+        case 1: return factor_impl<1>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
+        case 2: return factor_impl<2>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
+        case 3: return factor_impl<3>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
+        case 4: return factor_impl<4>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
+        default: return set_error(LF_EINVAL, "n must be in [1,4]");
+    }
+}
+
+}  // namespace lf

@@ -1,0 +1,90 @@
+// lf_internal.h -- host-side internals shared by the translation units of liblf.so.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+
+#include "../../include/lf.h"
+
+namespace lf {
+
+constexpr int kMaxFlagRounds = 1024;  // maximality flags kept on the device (ring)
+
+// error state (thread-local message, lf_api.cu)
+int set_error(int code, const char* msg);
+int set_cuda_error(cudaError_t e, const char* where);
+
+#define LF_CUDA(call)                                                     \
+    do {                                                                  \
+        cudaError_t e_ = (call);                                          \
+        if (e_ != cudaSuccess) return ::lf::set_cuda_error(e_, #call);    \
+    } while (0)
+
+// optional per-kernel event timing (lf_profile_enable / lf_profile_collect)
+void prof_begin(const char* name, int k, cudaStream_t s);
+void prof_end(cudaStream_t s);
+struct ProfScope {
+    cudaStream_t s;
+    ProfScope(const char* name, int k, cudaStream_t st) : s(st) { prof_begin(name, k, s); }
+    ~ProfScope() { prof_end(s); }
+};
+#define LF_PROF(name, k, s) ::lf::ProfScope lf_prof_scope_(name, k, s)
+
+// grid of a persistent kernel: resident blocks per SM x SM count (cached per kernel)
+int persistent_grid(const void* kernel, int block, size_t smem = 0);
+int sm_count();
+
+// 256-byte aligned bump allocator over a caller workspace
+struct Carve {
+    char* base;
+    size_t cap;
+    size_t off = 0;
+    Carve(void* b, size_t c) : base((char*)b), cap(c) {}
+    template <class T>
+    T* take(size_t n) {
+        off = (off + 255) & ~(size_t)255;
+        T* p = (T*)(base ? base + off : nullptr);
+        off += n * sizeof(T);
+        return p;
+    }
+    bool ok() const { return off <= cap; }
+};
+
+struct FactorWs {
+    uint8_t* state;     // [N]
+    int32_t* prop_j;    // [N*n]
+    float* prop_v;      // [N*n]
+    int32_t* wl[2];     // [N] each
+    int32_t* counts;    // [4]
+    int* flags;         // [kMaxFlagRounds]
+};
+size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w);
+
+int factor_dispatch(const lf_csr_t* A, int n, const lf_factor_opts_t* o, int32_t* pi, float* pi_w,
+                    float* pi_val, float* diag, int32_t* rounds_dev, int64_t* live,
+                    const FactorWs& w, cudaStream_t s);
+
+struct ForestWs {
+    int32_t* q[2];       // [2N] stride neighbours, ping-pong
+    uint64_t* mk[2];     // [2N] min edge key per direction (cycle scan), ping-pong
+    int32_t* r[2];       // [2N] positions (rank scan), ping-pong
+    uint64_t* ekey;      // [2N] key of the edge in each slot of pi2
+    int32_t* len;        // [N] path length at the path-ID vertex, else 0
+    int32_t* off;        // [N] exclusive scan of len
+    int* ctl;            // [256] per-step "not done" counters, cycle count
+    void* scan_tmp;      // CUB temp storage
+    size_t scan_tmp_bytes;
+};
+size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w);
+
+int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
+               int32_t* pos, int32_t* perm, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
+               cudaStream_t s);
+
+int tridiag_run(int64_t N, const int32_t* forest, const int32_t* iperm, const int32_t* pi2,
+                const float* pi2_val, const float* diag, float* a, float* b, float* c,
+                cudaStream_t s);
+
+}  // namespace lf

@@ -1,0 +1,270 @@
+"""Thin Python binding of liblf.so (include/lf.h): argument marshalling only.
+
+Every step of the path runs in the library's CUDA kernels.  torch tensors serve only as
+device memory; the current torch CUDA stream is passed through.  There is no CPU
+fallback: if liblf.so is missing or no CUDA device is present, calls raise.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from dataclasses import dataclass
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "liblf.so")
+
+LF_OK = 0
+ERRORS = {-1: "LF_EINVAL", -2: "LF_ENOMEM", -3: "LF_ECUDA", -4: "LF_ENCCL", -5: "LF_EINPUT"}
+
+# every symbol include/lf.h declares (checked by tests/test_abi.py)
+EXPORTS = (
+    "lf_factor_opts_default", "lf_factor_workspace_size", "lf_factor",
+    "lf_linear_forest_workspace_size", "lf_linear_forest", "lf_tridiag",
+    "lf_pipeline_workspace_size", "lf_pipeline_host", "lf_validate_csr",
+    "lf_last_error", "lf_version", "lf_profile_enable", "lf_profile_collect",
+)
+
+
+class LFError(RuntimeError):
+    pass
+
+
+class CSRDesc(C.Structure):
+    _fields_ = [("n", C.c_int64), ("nnz", C.c_int64), ("rowptr", C.c_void_p),
+                ("col", C.c_void_p), ("val", C.c_void_p)]
+
+
+class FactorOpts(C.Structure):
+    _fields_ = [("M", C.c_int32), ("m", C.c_int32), ("k_m", C.c_int32), ("p", C.c_float),
+                ("seed", C.c_uint32), ("until_maximal", C.c_int32)]
+
+
+_lib = None
+
+
+def load(path: str = LIB_PATH):
+    """Load liblf.so (raises if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise LFError(f"{path} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
+    L = C.CDLL(path)
+    P, I64, I32 = C.c_void_p, C.c_int64, C.c_int
+    L.lf_factor_opts_default.argtypes = [P]
+    L.lf_factor_workspace_size.argtypes = [I64, I32]
+    L.lf_factor_workspace_size.restype = C.c_size_t
+    L.lf_factor.argtypes = [P, I32, P, P, P, P, P, P, P, P, C.c_size_t, P]
+    L.lf_linear_forest_workspace_size.argtypes = [I64]
+    L.lf_linear_forest_workspace_size.restype = C.c_size_t
+    L.lf_linear_forest.argtypes = [I64, P, P, P, P, P, P, P, P, P, C.c_size_t, P]
+    L.lf_tridiag.argtypes = [I64, P, P, P, P, P, P, P, P, P]
+    L.lf_pipeline_workspace_size.argtypes = [I64, I64]
+    L.lf_pipeline_workspace_size.restype = C.c_size_t
+    L.lf_pipeline_host.argtypes = [P, P, P, P, P, P, P, P, P, C.c_size_t, P]
+    L.lf_validate_csr.argtypes = [P, P, C.c_size_t, P]
+    L.lf_profile_enable.argtypes = [I32]
+    L.lf_profile_collect.argtypes = [P, I32, P, I32]
+    L.lf_last_error.restype = C.c_char_p
+    L.lf_version.restype = C.c_char_p
+    for name in ("lf_factor", "lf_linear_forest", "lf_tridiag", "lf_pipeline_host", "lf_validate_csr",
+                 "lf_factor_opts_default"):
+        getattr(L, name).restype = C.c_int if name != "lf_factor_opts_default" else None
+    _lib = L
+    return L
+
+
+def _check(rc):
+    if rc != LF_OK:
+        msg = load().lf_last_error().decode()
+        raise LFError(f"{ERRORS.get(rc, rc)}: {msg}")
+
+
+def _torch():
+    import torch
+
+    if not torch.cuda.is_available():
+        raise LFError("liblf needs a CUDA device (no CPU fallback)")
+    return torch
+
+
+def _ptr(t):
+    return None if t is None else C.c_void_p(t.data_ptr())
+
+
+def _stream():
+    torch = _torch()
+    return C.c_void_p(torch.cuda.current_stream().cuda_stream)
+
+
+def _csr_desc(rowptr, col, val):
+    N = rowptr.numel() - 1
+    return CSRDesc(N, col.numel(), rowptr.data_ptr(), col.data_ptr(), val.data_ptr())
+
+
+def opts(M=5, m=5, k_m=0, p=0.5, seed=0, until_maximal=False) -> FactorOpts:
+    return FactorOpts(M, m, k_m, p, seed, 1 if until_maximal else 0)
+
+
+class Workspace:
+    """Grow-only device scratch buffer (torch uint8 tensor)."""
+
+    def __init__(self):
+        self.buf = None
+
+    def get(self, nbytes: int):
+        torch = _torch()
+        if self.buf is None or self.buf.numel() < nbytes:
+            self.buf = torch.empty(max(nbytes, 256), dtype=torch.uint8, device="cuda")
+        return self.buf
+
+
+_ws = Workspace()
+
+
+def factor(rowptr, col, val, n=2, *, M=5, m=5, k_m=0, p=0.5, seed=0, until_maximal=False,
+           want_val=True, want_diag=True, live=False, ws=None, out=None):
+    """lf_factor on device CSR tensors -> dict(pi[N,n], pi_w, pi_val, diag, rounds, live)."""
+    torch = _torch()
+    L = load()
+    N = rowptr.numel() - 1
+    dev = rowptr.device
+    if out is None:
+        out = dict(
+            pi=torch.empty((N, n), dtype=torch.int32, device=dev),
+            pi_w=torch.empty((N, n), dtype=torch.float32, device=dev),
+            pi_val=torch.empty((N, n), dtype=torch.float32, device=dev) if want_val else None,
+            diag=torch.empty(N, dtype=torch.float32, device=dev) if want_diag else None,
+            rounds=torch.zeros(1, dtype=torch.int32, device=dev),
+            live=torch.zeros(2 * max(M, 1), dtype=torch.int64, device=dev) if live else None,
+        )
+    A = _csr_desc(rowptr, col, val)
+    o = opts(M, m, k_m, p, seed, until_maximal)
+    nb = L.lf_factor_workspace_size(N, n)
+    buf = (ws or _ws).get(nb)
+    _check(L.lf_factor(C.byref(A), n, C.byref(o), _ptr(out["pi"]), _ptr(out["pi_w"]),
+                       _ptr(out["pi_val"]), _ptr(out["diag"]), _ptr(out["rounds"]),
+                       _ptr(out["live"]), _ptr(buf), nb, _stream()))
+    return out
+
+
+def linear_forest(pi2, pi2_w, *, ws=None, out=None, n_cycles=True):
+    """lf_linear_forest -> dict(forest[N,2], path_id, pos, perm, iperm, n_cycles)."""
+    torch = _torch()
+    L = load()
+    N = pi2.shape[0]
+    dev = pi2.device
+    if out is None:
+        out = dict(
+            forest=torch.empty((N, 2), dtype=torch.int32, device=dev),
+            path_id=torch.empty(N, dtype=torch.int32, device=dev),
+            pos=torch.empty(N, dtype=torch.int32, device=dev),
+            perm=torch.empty(N, dtype=torch.int32, device=dev),
+            iperm=torch.empty(N, dtype=torch.int32, device=dev),
+            n_cycles=torch.zeros(1, dtype=torch.int64, device=dev) if n_cycles else None,
+        )
+    nb = L.lf_linear_forest_workspace_size(N)
+    buf = (ws or _ws).get(nb)
+    _check(L.lf_linear_forest(N, _ptr(pi2), _ptr(pi2_w), _ptr(out["forest"]), _ptr(out["path_id"]),
+                              _ptr(out["pos"]), _ptr(out["perm"]), _ptr(out["iperm"]),
+                              _ptr(out["n_cycles"]), _ptr(buf), nb, _stream()))
+    return out
+
+
+def tridiag(forest, iperm, pi2, pi2_val, diag, *, out=None):
+    """lf_tridiag -> (a, b, c) device float32 [N]."""
+    torch = _torch()
+    L = load()
+    N = forest.shape[0]
+    if out is None:
+        out = tuple(torch.empty(N, dtype=torch.float32, device=forest.device) for _ in range(3))
+    a, b, c = out
+    _check(L.lf_tridiag(N, _ptr(forest), _ptr(iperm), _ptr(pi2), _ptr(pi2_val), _ptr(diag),
+                        _ptr(a), _ptr(b), _ptr(c), _stream()))
+    return a, b, c
+
+
+@dataclass
+class Pipeline:
+    """Preallocated device buffers for the whole hot path on one graph (n=2)."""
+
+    rowptr: object
+    col: object
+    val: object
+    M: int = 5
+    m: int = 5
+    k_m: int = 0
+    p: float = 0.5
+    seed: int = 0
+
+    def __post_init__(self):
+        torch = _torch()
+        N = self.rowptr.numel() - 1
+        self.N = N
+        self.ws_f = Workspace()
+        self.ws_l = Workspace()
+        self.fac = None
+        self.lf = None
+        self.tri = tuple(torch.empty(N, dtype=torch.float32, device="cuda") for _ in range(3))
+
+    def run_factor(self):
+        self.fac = factor(self.rowptr, self.col, self.val, 2, M=self.M, m=self.m, k_m=self.k_m,
+                          p=self.p, seed=self.seed, ws=self.ws_f, out=self.fac, live=True)
+        return self.fac
+
+    def run_forest(self):
+        self.lf = linear_forest(self.fac["pi"], self.fac["pi_w"], ws=self.ws_l, out=self.lf)
+        return self.lf
+
+    def run_tridiag(self):
+        return tridiag(self.lf["forest"], self.lf["iperm"], self.fac["pi"], self.fac["pi_val"],
+                       self.fac["diag"], out=self.tri)
+
+    def run(self):
+        self.run_factor()
+        self.run_forest()
+        self.run_tridiag()
+        return self
+
+
+def pipeline_host(rowptr_h, col_h, val_h, *, M=5, m=5, k_m=0, p=0.5, seed=0, ws=None, outs=None):
+    """lf_pipeline_host with HOST (pinned) torch CPU tensors -> (perm, path_id, pos, a, b, c)."""
+    torch = _torch()
+    L = load()
+    N = rowptr_h.numel() - 1
+    if outs is None:
+        mk = lambda dt: torch.empty(N, dtype=dt, pin_memory=True)  # noqa: E731
+        outs = (mk(torch.int32), mk(torch.int32), mk(torch.int32), mk(torch.float32),
+                mk(torch.float32), mk(torch.float32))
+    A = _csr_desc(rowptr_h, col_h, val_h)
+    o = opts(M, m, k_m, p, seed)
+    nb = L.lf_pipeline_workspace_size(N, col_h.numel())
+    buf = (ws or _ws).get(nb)
+    _check(L.lf_pipeline_host(C.byref(A), C.byref(o), *[_ptr(t) for t in outs], _ptr(buf), nb,
+                              _stream()))
+    return outs
+
+
+def validate(rowptr, col, val):
+    L = load()
+    A = _csr_desc(rowptr, col, val)
+    buf = _ws.get(256)
+    _check(L.lf_validate_csr(C.byref(A), _ptr(buf), 256, _stream()))
+
+
+def profile_enable(on: bool = True):
+    load().lf_profile_enable(1 if on else 0)
+
+
+def profile_collect(cap: int = 4096):
+    """-> list of (kernel name, ms) for the launches recorded since profile_enable(True)."""
+    L = load()
+    stride = 40
+    names = C.create_string_buffer(stride * cap)
+    ms = (C.c_float * cap)()
+    n = L.lf_profile_collect(names, stride, ms, cap)
+    out = []
+    for i in range(n):
+        nm = names.raw[i * stride:(i + 1) * stride].split(b"\0", 1)[0].decode()
+        out.append((nm, float(ms[i])))
+    return out

@@ -1,0 +1,77 @@
+"""The C-ABI library builds, loads and exports every symbol include/lf.h declares.
+
+CPU only: no call here reaches a CUDA API (argument checks fail before any launch).
+"""
+import ctypes as C
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_icpp_0002s22_b200 import _build, lf
+
+    _build.build()
+    return lf.load()
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "lf.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(lf_[a-z_]+)\s*\(", src)))
+
+
+def test_exports_every_declared_symbol(lib):
+    from paper_conf_icpp_0002s22_b200 import lf
+
+    names = _declared()
+    assert set(names) == set(lf.EXPORTS)
+    for n in names:
+        assert hasattr(lib, n), n
+
+
+def test_version_and_defaults(lib):
+    from paper_conf_icpp_0002s22_b200 import lf
+
+    assert b"sm_100a" in lib.lf_version()
+    o = lf.FactorOpts()
+    lib.lf_factor_opts_default(C.byref(o))
+    assert (o.M, o.m, o.k_m, o.p, o.seed, o.until_maximal) == (5, 5, 0, 0.5, 0, 0)
+
+
+def test_workspace_size_grows_with_n(lib):
+    s1 = lib.lf_factor_workspace_size(1000, 1)
+    s4 = lib.lf_factor_workspace_size(1000, 4)
+    assert 0 < s1 < s4
+    assert lib.lf_factor_workspace_size(1000, 5) == 0
+
+
+def test_invalid_arguments_rejected_before_launch(lib):
+    from paper_conf_icpp_0002s22_b200 import lf
+
+    A = lf.CSRDesc(10, 0, 1, None, None)
+    o = lf.FactorOpts(5, 5, 0, 0.5, 0, 0)
+    assert lib.lf_factor(C.byref(A), 5, C.byref(o), None, None, None, None, None, None, None, 0, None) == -1
+    assert b"n must be" in lib.lf_last_error()
+    assert lib.lf_factor(None, 2, None, None, None, None, None, None, None, None, 0, None) == -1
+    A = lf.CSRDesc(2 ** 31, 0, 1, None, None)
+    assert lib.lf_factor(C.byref(A), 2, None, 1, 1, None, None, None, None, None, 0, None) == -1
+    o = lf.FactorOpts(5, 5, 7, 0.5, 0, 1)  # until_maximal with k_m >= m
+    A = lf.CSRDesc(10, 0, 1, None, None)
+    assert lib.lf_factor(C.byref(A), 2, C.byref(o), 1, 1, None, None, None, None, None, 0, None) == -1
+    assert lib.lf_linear_forest(-1, None, None, None, None, None, None, None, None, None, 0, None) == -1
+    assert lib.lf_tridiag(5, None, None, None, None, None, None, None, None, None) == -1
+
+
+def test_product_package_does_not_import_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_icpp_0002s22_b200")
+    for dp, _, fs in os.walk(pkg):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                txt = open(os.path.join(dp, f)).read()
+                assert "import oracle" not in txt and "from oracle" not in txt, f
+                assert "lf_oracle" not in txt, f
