@@ -263,6 +263,18 @@ __global__ void k_init_state(int64_t N, uint8_t* state, uint32_t seed, unsigned 
         state[v] = charge_bit((uint32_t)v, 0u, seed, thr) ? ST_CHARGE : 0;
 }
 
+// diagonal only (M = 0: no round streams the rows)
+__global__ void k_diag(int64_t N, const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+                       const float* __restrict__ val, float* diag) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        float d = 0.0f;
+        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; e++)
+            if (col[e] == (int32_t)v) d = val[e];
+        diag[v] = d;
+    }
+}
+
 // Alg. 2 L23-L24 / L30: rounds = k+1 for the first uncharged round without proposals
 __global__ void k_rounds(const int* flags, int M, int m, int k_m, int32_t* rounds) {
     int r = M;
@@ -322,7 +334,11 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_CUDA(cudaMemsetAsync(pi, 0xff, sizeof(int32_t) * N * NN, s));
             LF_CUDA(cudaMemsetAsync(pi_w, 0, sizeof(float) * N * NN, s));
             if (pi_val) LF_CUDA(cudaMemsetAsync(pi_val, 0, sizeof(float) * N * NN, s));
-            if (diag) LF_CUDA(cudaMemsetAsync(diag, 0, sizeof(float) * N, s));
+            if (diag) {
+                LF_PROF("diag", -1, s);
+                k_diag<<<persistent_grid((const void*)k_diag, 256), 256, 0, s>>>(N, A->rowptr, A->col, A->val, diag);
+                LF_CUDA(cudaGetLastError());
+            }
         }
         if (rounds_dev) LF_CUDA(cudaMemsetAsync(rounds_dev, 0, sizeof(int32_t), s));
         return LF_OK;

@@ -275,9 +275,15 @@ __global__ void k_perm(int64_t N, const int32_t* __restrict__ path_id, const int
 }
 
 static size_t scan_temp_bytes(int64_t N) {
+    // CUB's decoupled look-back scan needs one tile descriptor per tile (~1-2k items) plus
+    // padding.  The query below can fail (it reports a pending CUDA error of an unrelated
+    // earlier call), so the workspace uses a bound that covers it: 16 B per 64 items.
+    const size_t bound = 16 * ((size_t)(N > 0 ? N : 1) / 64 + 256) + 4096;
     size_t b = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, b, (const int32_t*)nullptr, (int32_t*)nullptr, (int)(N > 0 ? N : 1));
-    return b;
+    cudaError_t e = cub::DeviceScan::ExclusiveSum(nullptr, b, (const int32_t*)nullptr, (int32_t*)nullptr,
+                                                  (int)(N > 0 ? N : 1));
+    if (e != cudaSuccess) return bound;
+    return b > bound ? b : bound;
 }
 
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
