@@ -76,6 +76,12 @@ class Clocks:
         except Exception:
             self.proc = None
 
+    def n_samples(self):
+        try:
+            return sum(1 for _ in open(self.path))
+        except OSError:
+            return 0
+
     def stop(self):
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
@@ -207,6 +213,8 @@ def main():
     flush = torch.empty(512 * 1024 * 1024, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
 
+    clocks = Clocks(local)
+    clocks.start()
     for _ in range(max(args.warmup, 3)):
         P.run()
     torch.cuda.synchronize()
@@ -239,11 +247,15 @@ def main():
             lf.profile_enable(True)
             P.run()
 
-    clocks = Clocks(local)
+    # keep the GPU busy until the clock sampler is producing samples (bounded)
+    t_end = time.time() + 5.0
+    while clocks.n_samples() < 3 and time.time() < t_end:
+        for _ in range(10):
+            step()
+        torch.cuda.synchronize()
     if ws > 1:
         torch.distributed.barrier()
     torch.cuda.synchronize()
-    clocks.start()
     step_ms, kern = [], {}
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
@@ -261,6 +273,10 @@ def main():
     torch.cuda.synchronize()
     if ws > 1:
         torch.distributed.barrier()
+    t_end = time.time() + 1.0
+    n0 = clocks.n_samples()
+    while clocks.n_samples() < n0 + 2 and time.time() < t_end:
+        time.sleep(0.05)
     clk = clocks.stop()
     lf.profile_enable(False)
 

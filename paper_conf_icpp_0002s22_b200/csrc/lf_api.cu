@@ -39,6 +39,15 @@ static bool g_prof = false;
 static std::vector<ProfRec> g_recs;
 static std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_pool;
 
+// inside a stream capture a plain record only orders streams; an "external" record
+// becomes an event-record node that fires on every graph replay
+static void record_event(cudaEvent_t e, cudaStream_t s) {
+    cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(s, &st);
+    if (st == cudaStreamCaptureStatusActive) cudaEventRecordWithFlags(e, s, cudaEventRecordExternal);
+    else cudaEventRecord(e, s);
+}
+
 void prof_begin(const char* name, int k, cudaStream_t s) {
     if (!g_prof) return;
     std::lock_guard<std::mutex> lk(g_prof_mu);
@@ -55,13 +64,13 @@ void prof_begin(const char* name, int k, cudaStream_t s) {
     r.a = g_pool[i].first;
     r.b = g_pool[i].second;
     g_recs.push_back(r);
-    cudaEventRecord(r.a, s);
+    record_event(r.a, s);
 }
 
 void prof_end(cudaStream_t s) {
     if (!g_prof) return;
     std::lock_guard<std::mutex> lk(g_prof_mu);
-    if (!g_recs.empty()) cudaEventRecord(g_recs.back().b, s);
+    if (!g_recs.empty()) record_event(g_recs.back().b, s);
 }
 
 int sm_count() {
