@@ -1,22 +1,29 @@
 // lf_forest.cu -- linear forest from a [0,2]-factor (§3.3,
 // Algorithm 3, §4.2, §4.3).
 //
-// Both scans are the paper's bidirectional pointer-jumping scan (no orientation, no
-// random-access iterator), run as ONE cooperative persistent kernel each instead of
-// ceil(log2 N) launches: the grid iterates stride-doubling steps separated by grid-wide
-// barriers over ping-pong buffers (L249) and leaves as soon as every vertex is done,
-// i.e. after ceil(log2 L_max)+O(1) steps for the longest component L_max rather than
-// ceil(log2 N).
-//   cycle scan (step (1), L225, L245-L247): per direction the stride pointer and the
-//     minimum edge key seen.  A path vertex is done when both pointers are path-end
-//     markers -(e+1) (L245).  A cycle vertex is done when its two windows share the
-//     cycle's weakest edge (equal minima) or both pointers coincide: then the union of
-//     its windows is the whole cycle.  Every cycle vertex then knows the weakest edge;
-//     its two endpoints drop it.
-//   rank scan (step (2), Alg. 3): per direction the pointer and the position sum r.
-//     l(v) = smaller end ID, p(v) = r toward that end (L223).
-//   permutation (step (3)): path length at the path-ID vertex, exclusive scan (CUB),
-//     new(v) = off[l(v)] + p(v) - 1 -- the same order as sorting by (l, p) (L297).
+// The paper runs its bidirectional scan (stride-doubling pointer jumping over the
+// unoriented doubly-linked list, end markers -(e+1), ping-pong buffers) as ceil(log2 N)
+// global launches over all N vertices, twice (cycles, then positions).  On B200 the same
+// scan runs hierarchically:
+//
+//   1. block-local scan (k_lf_local1): a CTA loads 2048 consecutive vertices into shared
+//      memory and runs the bidirectional scan on the links that stay inside the block
+//      (a link to another block is an "exit" and ends the local walk like a path end).
+//      Every vertex learns the local terminal it reaches in each direction, the local
+//      distance and the minimum edge key on the way; cycles that lie inside the block are
+//      complete.  Only "boundary" vertices (with a link leaving the block) go on.
+//   2. reduced scan (k_red_scan, one cooperative kernel): the same bidirectional scan on
+//      the reduced graph whose nodes are boundary vertices and whose links are either a
+//      cross-block edge or a whole local segment (weighted by its length and minimum
+//      key).  It leaves as soon as every node is done.
+//   3. expand (k_lf_local2 / k_lf_local3): the block-local scan is recomputed from the
+//      input (cheaper than storing it) and combined with the reduced results of the two
+//      terminals of each local segment.
+//
+// Step (1) (cycles) and step (2) (positions) each take one local + one reduced pass; the
+// forest is written between them by the fused kernel k_lf_local2, which also runs the
+// step-(2) local scan on the freshly broken forest while it is still in shared memory.
+// Step (3) is a CUB exclusive scan of path lengths plus a scatter.
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
@@ -31,235 +38,468 @@ namespace cg = cooperative_groups;
 namespace lf {
 
 constexpr uint64_t KEY_INF = ~0ull;
-constexpr int kCtlCycle = 0;    // ctl[0..63]  per-step not-done counts of the cycle scan
-constexpr int kCtlRank = 64;    // ctl[64..127] rank scan
+constexpr int LB = 2048;          // vertices per block-local tile
+constexpr int LT = 512;           // threads per tile CTA
+constexpr int VPT = LB / LT;      // vertices per thread
+constexpr int kCtlRed1 = 0;       // ctl[0..63]   per-step not-done counts, reduced scan 1
+constexpr int kCtlRed2 = 64;      // ctl[64..127] reduced scan 2
+constexpr int kCtlCnt1 = 128;     // boundary list sizes
+constexpr int kCtlCnt2 = 129;
 constexpr int kMaxSteps = 62;
 
-__device__ __forceinline__ int block_reduce_add(int x, int* sh) {
-    // sh: 32 ints of shared memory
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-#pragma unroll
-    for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
-    if (lane == 0) sh[wid] = x;
-    __syncthreads();
-    int t = 0;
-    if (threadIdx.x < 32) {
-        t = (threadIdx.x < (blockDim.x >> 5)) ? sh[threadIdx.x] : 0;
-#pragma unroll
-        for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
-    }
-    __syncthreads();
-    return t;  // valid in thread 0
-}
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 
-// key of the edge {u,x} for the weakest-edge search: minimise (|w| bits, -rank), where
-// rank orders edges by (min, max) lexicographically: rank = 2*min + c, c = 1 iff max is
-// the larger of min's two higher neighbours (DESIGN.md §3 reading c9).
-__device__ __forceinline__ uint64_t edge_key(const int2* __restrict__ nb, int32_t v, int32_t w,
-                                             float wabs, int2 nbv) {
+// Global key of edge {v,w} for the weakest-edge search, minimised: (|w| bits, -rank), rank
+// = 2*min + c orders edges by (min, max) lexicographically (c = 1 iff max is the larger of
+// min's two higher neighbours).  Realises reading c9 (ties -> larger (min,max) is weaker).
+__device__ __forceinline__ uint64_t edge_key(int32_t v, int32_t w, float wabs, int2 nb_min) {
     const int32_t u = v < w ? v : w;
     const int32_t x = v < w ? w : v;
-    const int2 nu = (u == v) ? nbv : nb[u];
-    const int32_t y = (nu.x == x) ? nu.y : nu.x;  // u's other neighbour
+    const int32_t y = (nb_min.x == x) ? nb_min.y : nb_min.x;  // min endpoint's other neighbour
     const uint32_t c = (y > u && y < x) ? 1u : 0u;
     const uint32_t rank = 2u * (uint32_t)u + c;
     return ((uint64_t)__float_as_uint(wabs) << 32) | (uint64_t)(0xFFFFFFFFu - rank);
 }
 
-__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+// shared-memory state of one tile
+struct TileSmem {
+    int2 nb[LB];          // global neighbours (slot order), -1 = none
+    short2 P[LB];         // local stride pointer per direction, or marker -(t+1), t local
+    short2 R[LB];         // local edges covered per direction
+    ulonglong2 K[LB];     // min edge key per direction (cycle pass only)
+};
 
-struct CycleArgs {
+__device__ __forceinline__ bool is_local(int32_t x, int32_t b0) {
+    return x >= b0 && x < b0 + LB;
+}
+
+// Bidirectional scan inside the tile (Alg. 3 / its min variant restricted to local links).
+// On return (after a __syncthreads) s.P/s.R/s.K hold, for every local vertex and each
+// direction, either a terminal marker -(t+1) with the local distance and min key to t, or
+// (both directions non-negative) a completed local cycle whose min key is min(K.x, K.y).
+// WITH_KEYS: also carry min keys (cycle pass).  ek[k] = keys of the own vertices' slots.
+template <bool WITH_KEYS>
+__device__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT]) {
+    const int tid = threadIdx.x;
+    // init: stride-1 local neighbours; a missing or non-local neighbour ends the walk
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const int2 nb = s.nb[u];
+        short2 p;
+        short2 r;
+        const bool l0 = nb.x >= 0 && is_local(nb.x, b0);
+        const bool l1 = nb.y >= 0 && is_local(nb.y, b0);
+        p.x = l0 ? (short)(nb.x - b0) : (short)(-(u + 1));
+        p.y = l1 ? (short)(nb.y - b0) : (short)(-(u + 1));
+        r.x = l0 ? 1 : 0;
+        r.y = l1 ? 1 : 0;
+        s.P[u] = p;
+        s.R[u] = r;
+        if (WITH_KEYS) {
+            ulonglong2 kk;
+            kk.x = l0 ? ek[k].x : KEY_INF;
+            kk.y = l1 ? ek[k].y : KEY_INF;
+            s.K[u] = kk;
+        }
+    }
+    __syncthreads();
+    for (int step = 0; step < 16; step++) {
+        short2 np[VPT], nr[VPT];
+        ulonglong2 nk[VPT];
+        int notdone = 0;
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int u = tid + k * LT;
+            const short2 p = s.P[u];
+            short2 r = s.R[u];
+            short2 q = p;
+            ulonglong2 kk;
+            if (WITH_KEYS) kk = s.K[u];
+            if (p.x >= 0) {
+                const short2 pw = s.P[p.x];
+                const short2 rw = s.R[p.x];
+                if (pw.x != u) {
+                    q.x = pw.x; r.x = (short)(r.x + rw.x);
+                    if (WITH_KEYS) kk.x = umin64(kk.x, s.K[p.x].x);
+                } else if (pw.y != u) {
+                    q.x = pw.y; r.x = (short)(r.x + rw.y);
+                    if (WITH_KEYS) kk.x = umin64(kk.x, s.K[p.x].y);
+                }
+            }
+            if (p.y >= 0) {
+                const short2 pw = s.P[p.y];
+                const short2 rw = s.R[p.y];
+                if (pw.x != u) {
+                    q.y = pw.x; r.y = (short)(r.y + rw.x);
+                    if (WITH_KEYS) kk.y = umin64(kk.y, s.K[p.y].x);
+                } else if (pw.y != u) {
+                    q.y = pw.y; r.y = (short)(r.y + rw.y);
+                    if (WITH_KEYS) kk.y = umin64(kk.y, s.K[p.y].y);
+                }
+            }
+            np[k] = q;
+            nr[k] = r;
+            if (WITH_KEYS) nk[k] = kk;
+            const bool path_done = q.x < 0 && q.y < 0;
+            bool cyc_done = false;
+            if (WITH_KEYS) cyc_done = q.x >= 0 && q.y >= 0 && (kk.x == kk.y || q.x == q.y);
+            notdone |= !(path_done || cyc_done);
+        }
+        __syncthreads();
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int u = tid + k * LT;
+            s.P[u] = np[k];
+            s.R[u] = nr[k];
+            if (WITH_KEYS) s.K[u] = nk[k];
+        }
+        if (!__syncthreads_or(notdone)) break;
+    }
+}
+
+// the slot of local terminal t (t not the walk's start) that leaves its segment: the
+// one that is not a local link (a remote neighbour or none)
+__device__ __forceinline__ int outward_slot(int2 nbt, int32_t b0) {
+    const bool l0 = nbt.x >= 0 && is_local(nbt.x, b0);
+    return l0 ? 1 : 0;
+}
+
+__device__ __forceinline__ void list_append(int32_t* list, int* count, int32_t g, bool take) {
+    const unsigned m = __ballot_sync(0xffffffffu, take);
+    const int lane = threadIdx.x & 31;
+    int base = 0;
+    if (lane == 0 && m) base = atomicAdd(count, __popc(m));
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (take) list[base + __popc(m & ((1u << lane) - 1u))] = g;
+}
+
+struct ForestArgs {
     int64_t N;
-    const int2* __restrict__ pi2;     // [N] slots as int2
+    const int2* __restrict__ pi2;
     const float2* __restrict__ pi2_w;
-    int2* q0;
-    int2* q1;
-    ulonglong2* m0;
-    ulonglong2* m1;
-    ulonglong2* ekey;                 // [N] key of each slot's edge
     int2* forest;
+    // reduced graph, pass 1 (cycles)
+    int2* rq1[2];
+    ulonglong2* rk1[2];
+    uint64_t* cyc_k;       // [N] weakest key of the global cycle through a boundary vertex
+    int32_t* list1;
+    // reduced graph, pass 2 (positions)
+    int2* rq2[2];
+    int2* rr2[2];
+    int2* end2;            // [N] path ends per direction of a boundary vertex
+    int2* dist2;           // [N] distances to them
+    int32_t* list2;
     int* ctl;
-    unsigned long long* n_cycles;     // may be NULL
+    int32_t* path_id;
+    int32_t* pos;
+    int32_t* len;
+    unsigned long long* n_cycles;
     int max_steps;
 };
 
-__global__ void __launch_bounds__(256) k_cycle_scan(CycleArgs a) {
+// keys of the own vertices' slots (global; a remote min endpoint needs one gather)
+__device__ __forceinline__ void slot_keys(const ForestArgs& a, const TileSmem& s, int32_t b0,
+                                         ulonglong2 (&ek)[VPT]) {
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        const int2 nb = s.nb[u];
+        ek[k].x = KEY_INF;
+        ek[k].y = KEY_INF;
+        if (g >= a.N) continue;
+        const float2 w = a.pi2_w[g];
+        if (nb.x >= 0) {
+            const int32_t mn = g < nb.x ? g : nb.x;
+            const int2 nbm = is_local(mn, b0) ? s.nb[mn - b0] : a.pi2[mn];
+            ek[k].x = edge_key(g, nb.x, w.x, nbm);
+        }
+        if (nb.y >= 0) {
+            const int32_t mn = g < nb.y ? g : nb.y;
+            const int2 nbm = is_local(mn, b0) ? s.nb[mn - b0] : a.pi2[mn];
+            ek[k].y = edge_key(g, nb.y, w.y, nbm);
+        }
+    }
+}
+
+__device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem& s, int32_t b0, int64_t N) {
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int64_t g = (int64_t)b0 + u;
+        s.nb[u] = g < N ? src[g] : make_int2(-1, -1);
+    }
+    __syncthreads();
+}
+
+// reduced-graph direction of boundary vertex g through its slot i:
+//   none -> end marker at g (distance 0); remote -> the neighbour (distance 1);
+//   local -> the segment's other terminal t: t itself if t continues in another block,
+//   else an end marker at t (distance = local length, key = segment min key).
+__device__ __forceinline__ void reduced_dir(const TileSmem& s, int32_t b0, int32_t g, int2 nb, int i,
+                                            short2 p, short2 r, int32_t& q, int32_t& d) {
+    const int32_t x = i ? nb.y : nb.x;
+    if (x < 0) { q = -(g + 1); d = 0; return; }
+    if (!is_local(x, b0)) { q = x; d = 1; return; }
+    const int t = -((i ? p.y : p.x) + 1);
+    const int2 nbt = s.nb[t];
+    const int so = outward_slot(nbt, b0);
+    const int32_t xo = so ? nbt.y : nbt.x;
+    q = xo >= 0 ? (b0 + t) : -(b0 + t + 1);
+    d = i ? r.y : r.x;
+}
+
+// Pass 1, local part: emit the reduced-graph records of boundary vertices.
+__global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
+    const int32_t b0 = blockIdx.x * LB;
+    load_tile(a.pi2, s, b0, a.N);
+    ulonglong2 ek[VPT];
+    slot_keys(a, s, b0, ek);
+    tile_scan<true>(s, b0, ek);
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        const int2 nb = s.nb[u];
+        const bool r0 = nb.x >= 0 && !is_local(nb.x, b0);
+        const bool r1 = nb.y >= 0 && !is_local(nb.y, b0);
+        const bool boundary = g < a.N && (r0 || r1);
+        if (boundary) {
+            const short2 p = s.P[u];
+            const short2 r = s.R[u];
+            const ulonglong2 kk = s.K[u];
+            int32_t q0, q1, d0, d1;
+            reduced_dir(s, b0, g, nb, 0, p, r, q0, d0);
+            reduced_dir(s, b0, g, nb, 1, p, r, q1, d1);
+            // key of each reduced link: the remote edge's key, or the segment's min key
+            ulonglong2 rk;
+            rk.x = (nb.x < 0) ? KEY_INF : (r0 ? ek[k].x : kk.x);
+            rk.y = (nb.y < 0) ? KEY_INF : (r1 ? ek[k].y : kk.y);
+            const int2 q = make_int2(q0, q1);
+            a.rq1[0][g] = q; a.rq1[1][g] = q;
+            a.rk1[0][g] = rk; a.rk1[1][g] = rk;
+        }
+        list_append(a.list1, &a.ctl[kCtlCnt1], g, boundary);
+    }
+}
+
+// Reduced bidirectional scan over a boundary list (one cooperative kernel).
+//   MIN: min-scan of edge keys; epilogue writes cyc_k (INF unless on a global cycle).
+//   ADD: position scan with weighted hops; epilogue writes end2 / dist2.
+template <bool MIN>
+__global__ void __launch_bounds__(256) k_red_scan(ForestArgs a) {
     __shared__ int sh[32];
     cg::grid_group grid = cg::this_grid();
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    // init (Alg. 3 L1-L4 analogue): stride-1 neighbours or end markers, edge keys
-    for (int64_t v = t0; v < a.N; v += stride) {
-        const int2 nb = a.pi2[v];
-        const float2 wv = a.pi2_w[v];
-        ulonglong2 k;
-        k.x = nb.x >= 0 ? edge_key(a.pi2, (int32_t)v, nb.x, wv.x, nb) : KEY_INF;
-        k.y = nb.y >= 0 ? edge_key(a.pi2, (int32_t)v, nb.y, wv.y, nb) : KEY_INF;
-        a.ekey[v] = k;
-        int2 q;
-        q.x = nb.x >= 0 ? nb.x : -(int32_t)(v + 1);
-        q.y = nb.y >= 0 ? nb.y : -(int32_t)(v + 1);
-        a.q0[v] = q;
-        a.m0[v] = k;
-        a.q1[v] = q;   // a vertex final from the start must be final in both buffers
-        a.m1[v] = k;
-    }
-    grid.sync();
+    const int32_t* list = MIN ? a.list1 : a.list2;
+    const int cnt = *(volatile int*)&a.ctl[MIN ? kCtlCnt1 : kCtlCnt2];
+    int* ctl = a.ctl + (MIN ? kCtlRed1 : kCtlRed2);
+    const int stride = gridDim.x * blockDim.x;
+    const int t0 = blockIdx.x * blockDim.x + threadIdx.x;
     int step = 0;
     for (; step < a.max_steps; step++) {
-        const int2* qs = (step & 1) ? a.q1 : a.q0;
-        const ulonglong2* ms = (step & 1) ? a.m1 : a.m0;
-        int2* qd = (step & 1) ? a.q0 : a.q1;
-        ulonglong2* md = (step & 1) ? a.m0 : a.m1;
+        const int2* qs = MIN ? a.rq1[step & 1] : a.rq2[step & 1];
+        int2* qd = MIN ? a.rq1[(step & 1) ^ 1] : a.rq2[(step & 1) ^ 1];
+        const ulonglong2* ks = a.rk1[step & 1];
+        ulonglong2* kd = a.rk1[(step & 1) ^ 1];
+        const int2* rs = a.rr2[step & 1];
+        int2* rd = a.rr2[(step & 1) ^ 1];
         int notdone = 0;
-        for (int64_t v = t0; v < a.N; v += stride) {
+        for (int idx = t0; idx < cnt; idx += stride) {
+            const int32_t v = list[idx];
             const int2 q = qs[v];
-            if (q.x < 0 && q.y < 0) {
-                // path vertex, final: make sure the other buffer holds the same values
+            if (q.x < 0 && q.y < 0) {  // final: keep both buffers equal
                 const int2 qo = qd[v];
                 if (qo.x != q.x || qo.y != q.y) {
                     qd[v] = q;
-                    md[v] = ms[v];
+                    if (MIN) kd[v] = ks[v]; else rd[v] = rs[v];
                 }
                 continue;
             }
-            ulonglong2 m = ms[v];
             int2 nq = q;
-            ulonglong2 nm = m;
-            if (q.x >= 0) {  // Alg. 3 L12-L20 with the min operator
-                const int2 qw = qs[q.x];
-                const ulonglong2 mw = ms[q.x];
-                if (qw.x != (int32_t)v) { nq.x = qw.x; nm.x = umin64(m.x, mw.x); }
-                else if (qw.y != (int32_t)v) { nq.x = qw.y; nm.x = umin64(m.x, mw.y); }
-            }
-            if (q.y >= 0) {
-                const int2 qw = qs[q.y];
-                const ulonglong2 mw = ms[q.y];
-                if (qw.x != (int32_t)v) { nq.y = qw.x; nm.y = umin64(m.y, mw.x); }
-                else if (qw.y != (int32_t)v) { nq.y = qw.y; nm.y = umin64(m.y, mw.y); }
+            ulonglong2 nk = make_ulonglong2(0, 0);
+            int2 nr = make_int2(0, 0);
+            if (MIN) nk = ks[v]; else nr = rs[v];
+#pragma unroll
+            for (int i = 0; i < 2; i++) {
+                const int32_t w = i ? q.y : q.x;
+                if (w < 0) continue;
+                const int2 qw = qs[w];
+                int j = -1;
+                if (qw.x != v) j = 0;
+                else if (qw.y != v) j = 1;
+                if (j < 0) continue;  // stall (reading c13)
+                const int32_t tgt = j ? qw.y : qw.x;
+                if (i) nq.y = tgt; else nq.x = tgt;
+                if (MIN) {
+                    const ulonglong2 kw = ks[w];
+                    const uint64_t kv = j ? kw.y : kw.x;
+                    if (i) nk.y = umin64(nk.y, kv); else nk.x = umin64(nk.x, kv);
+                } else {
+                    const int2 rw = rs[w];
+                    const int32_t dv = j ? rw.y : rw.x;
+                    if (i) nr.y += dv; else nr.x += dv;
+                }
             }
             qd[v] = nq;
-            md[v] = nm;
+            if (MIN) kd[v] = nk; else rd[v] = nr;
             const bool path_done = nq.x < 0 && nq.y < 0;
-            const bool cyc_done = nq.x >= 0 && nq.y >= 0 && (nm.x == nm.y || nq.x == nq.y);
+            bool cyc_done = false;
+            if (MIN) cyc_done = nq.x >= 0 && nq.y >= 0 && (nk.x == nk.y || nq.x == nq.y);
             notdone += (path_done || cyc_done) ? 0 : 1;
         }
-        const int tot = block_reduce_add(notdone, sh);
-        if (threadIdx.x == 0 && tot) atomicAdd(&a.ctl[kCtlCycle + step], tot);
+        // block reduction of notdone, one atomic per block
+#pragma unroll
+        for (int o = 16; o; o >>= 1) notdone += __shfl_xor_sync(0xffffffffu, notdone, o);
+        if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = notdone;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int tot = 0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); w++) tot += sh[w];
+            if (tot) atomicAdd(&ctl[step], tot);
+        }
         grid.sync();
-        if (*(volatile int*)&a.ctl[kCtlCycle + step] == 0) { step++; break; }
+        if (*(volatile int*)&ctl[step] == 0) { step++; break; }
     }
-    // results are in the buffer written by the last step
-    const int2* qf = (step & 1) ? a.q1 : a.q0;
-    const ulonglong2* mf = (step & 1) ? a.m1 : a.m0;
+    // results are in the buffer written by the last executed step
+    const int fb = step & 1;
+    for (int idx = t0; idx < cnt; idx += stride) {
+        const int32_t v = list[idx];
+        if (MIN) {
+            const int2 q = a.rq1[fb][v];
+            const ulonglong2 k = a.rk1[fb][v];
+            a.cyc_k[v] = (q.x >= 0 && q.y >= 0) ? umin64(k.x, k.y) : KEY_INF;
+        } else {
+            const int2 q = a.rq2[fb][v];
+            a.end2[v] = make_int2(-(q.x + 1), -(q.y + 1));
+            a.dist2[v] = a.rr2[fb][v];
+        }
+    }
+}
+
+// Pass 1 expand (break cycles, write the forest) fused with pass 2's local part.
+__global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
+    const int32_t b0 = blockIdx.x * LB;
+    load_tile(a.pi2, s, b0, a.N);
+    ulonglong2 ek[VPT];
+    slot_keys(a, s, b0, ek);
+    tile_scan<true>(s, b0, ek);
+    // weakest edge of the cycle through each own vertex (INF: not on a cycle)
+    int2 f[VPT];
     unsigned long long ncyc = 0;
-    for (int64_t v = t0; v < a.N; v += stride) {
-        int2 f = a.pi2[v];
-        const int2 q = qf[v];
-        if (q.x >= 0 && q.y >= 0) {  // on a cycle (L245): drop the weakest edge
-            const ulonglong2 m = mf[v];
-            const uint64_t kmin = umin64(m.x, m.y);
-            const ulonglong2 ek = a.ekey[v];
-            if (ek.x == kmin) {
-                f.x = f.y;
-                f.y = -1;
-                if ((int32_t)v < a.pi2[v].x) ncyc++;
-            } else if (ek.y == kmin) {
-                if ((int32_t)v < f.y) ncyc++;
-                f.y = -1;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        const int2 nb = s.nb[u];
+        f[k] = nb;
+        if (g >= a.N) continue;
+        const short2 p = s.P[u];
+        uint64_t kstar = KEY_INF;
+        if (p.x >= 0 && p.y >= 0) {  // local cycle
+            const ulonglong2 kk = s.K[u];
+            kstar = umin64(kk.x, kk.y);
+        } else {
+            // a segment: its cycle status is that of a terminal that continues in another
+            // block (a segment ending in a path end is on a path)
+#pragma unroll
+            for (int i = 0; i < 2; i++) {
+                const int t = -((i ? p.y : p.x) + 1);
+                const int2 nbt = s.nb[t];
+                const int so = (t == u) ? i : outward_slot(nbt, b0);
+                const int32_t xo = so ? nbt.y : nbt.x;
+                if (xo >= 0 && kstar == KEY_INF) kstar = a.cyc_k[b0 + t];
             }
         }
-        a.forest[v] = f;
+        if (kstar != KEY_INF) {
+            if (ek[k].x == kstar) {
+                if (g < nb.x) ncyc++;
+                f[k].x = f[k].y;
+                f[k].y = -1;
+            } else if (ek[k].y == kstar) {
+                if (g < nb.y) ncyc++;
+                f[k].y = -1;
+            }
+        }
+        a.forest[g] = f[k];
     }
     if (a.n_cycles) {
 #pragma unroll
         for (int o = 16; o; o >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o);
         if ((threadIdx.x & 31) == 0 && ncyc) atomicAdd(a.n_cycles, ncyc);
     }
+    __syncthreads();
+    // pass 2 local scan on the broken forest (still in shared memory)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) s.nb[threadIdx.x + k * LT] = f[k];
+    __syncthreads();
+    tile_scan<false>(s, b0, ek);
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        const int2 nb = s.nb[u];
+        const bool r0 = nb.x >= 0 && !is_local(nb.x, b0);
+        const bool r1 = nb.y >= 0 && !is_local(nb.y, b0);
+        const bool boundary = g < a.N && (r0 || r1);
+        if (boundary) {
+            const short2 p = s.P[u];
+            const short2 r = s.R[u];
+            int32_t q0, q1, d0, d1;
+            reduced_dir(s, b0, g, nb, 0, p, r, q0, d0);
+            reduced_dir(s, b0, g, nb, 1, p, r, q1, d1);
+            const int2 q = make_int2(q0, q1);
+            const int2 d = make_int2(d0, d1);
+            a.rq2[0][g] = q; a.rq2[1][g] = q;
+            a.rr2[0][g] = d; a.rr2[1][g] = d;
+        }
+        list_append(a.list2, &a.ctl[kCtlCnt2], g, boundary);
+    }
 }
 
-struct RankArgs {
-    int64_t N;
-    const int2* __restrict__ forest;
-    int2* q0;
-    int2* q1;
-    int2* r0;
-    int2* r1;
-    int32_t* path_id;
-    int32_t* pos;
-    int32_t* len;
-    int* ctl;
-    int max_steps;
-};
-
-__global__ void __launch_bounds__(256) k_rank_scan(RankArgs a) {
-    __shared__ int sh[32];
-    cg::grid_group grid = cg::this_grid();
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    for (int64_t v = t0; v < a.N; v += stride) {  // Alg. 3 L1-L4
-        const int2 f = a.forest[v];
-        int2 q;
-        q.x = f.x >= 0 ? f.x : -(int32_t)(v + 1);
-        q.y = f.y >= 0 ? f.y : -(int32_t)(v + 1);
-        const int2 one = make_int2(1, 1);
-        a.q0[v] = q;
-        a.r0[v] = one;
-        a.q1[v] = q;
-        a.r1[v] = one;
-    }
-    grid.sync();
-    int step = 0;
-    for (; step < a.max_steps; step++) {  // Alg. 3 L5-L26
-        const int2* qs = (step & 1) ? a.q1 : a.q0;
-        const int2* rs = (step & 1) ? a.r1 : a.r0;
-        int2* qd = (step & 1) ? a.q0 : a.q1;
-        int2* rd = (step & 1) ? a.r0 : a.r1;
-        int notdone = 0;
-        for (int64_t v = t0; v < a.N; v += stride) {
-            const int2 q = qs[v];
-            if (q.x < 0 && q.y < 0) {
-                const int2 qo = qd[v];
-                if (qo.x != q.x || qo.y != q.y) {
-                    qd[v] = q;
-                    rd[v] = rs[v];
-                }
-                continue;
+// Pass 2 expand: path ID, position and (at the path-ID vertex) the path length.
+__global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
+    const int32_t b0 = blockIdx.x * LB;
+    load_tile(a.forest, s, b0, a.N);
+    ulonglong2 ek[VPT];
+    tile_scan<false>(s, b0, ek);
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        if (g >= a.N) continue;
+        const short2 p = s.P[u];
+        const short2 r = s.R[u];
+        int32_t E[2], D[2];
+#pragma unroll
+        for (int i = 0; i < 2; i++) {
+            const int t = -((i ? p.y : p.x) + 1);  // local terminal in direction i
+            const int32_t d = i ? r.y : r.x;
+            const int2 nbt = s.nb[t];
+            // the outward slot of t: slot i itself when t == u (the walk never left u)
+            const int so = (t == u) ? i : outward_slot(nbt, b0);
+            const int32_t xo = so ? nbt.y : nbt.x;
+            if (xo >= 0) {  // continues in another block: reduced result of t
+                const int2 e = a.end2[b0 + t];
+                const int2 dd = a.dist2[b0 + t];
+                E[i] = so ? e.y : e.x;
+                D[i] = d + (so ? dd.y : dd.x);
+            } else {
+                E[i] = b0 + t;
+                D[i] = d;
             }
-            const int2 r = rs[v];
-            int2 nq = q, nr = r;
-            if (q.x >= 0) {
-                const int2 qw = qs[q.x];
-                const int2 rw = rs[q.x];
-                if (qw.x != (int32_t)v) { nq.x = qw.x; nr.x = r.x + rw.x; }       // L16-L18
-                else if (qw.y != (int32_t)v) { nq.x = qw.y; nr.x = r.x + rw.y; }
-            }
-            if (q.y >= 0) {
-                const int2 qw = qs[q.y];
-                const int2 rw = rs[q.y];
-                if (qw.x != (int32_t)v) { nq.y = qw.x; nr.y = r.y + rw.x; }
-                else if (qw.y != (int32_t)v) { nq.y = qw.y; nr.y = r.y + rw.y; }
-            }
-            qd[v] = nq;
-            rd[v] = nr;
-            notdone += (nq.x < 0 && nq.y < 0) ? 0 : 1;
         }
-        const int tot = block_reduce_add(notdone, sh);
-        if (threadIdx.x == 0 && tot) atomicAdd(&a.ctl[kCtlRank + step], tot);
-        grid.sync();
-        if (*(volatile int*)&a.ctl[kCtlRank + step] == 0) { step++; break; }
-    }
-    const int2* qf = (step & 1) ? a.q1 : a.q0;
-    const int2* rf = (step & 1) ? a.r1 : a.r0;
-    for (int64_t v = t0; v < a.N; v += stride) {  // Alg. 3 L27-L33 with l = min end (L223)
-        const int2 q = qf[v];
-        const int2 r = rf[v];
-        const int32_t e0 = -(q.x + 1), e1 = -(q.y + 1);
-        int32_t l, p;
-        if (e0 <= e1) { l = e0; p = r.x; } else { l = e1; p = r.y; }
-        a.path_id[v] = l;
-        a.pos[v] = p;
-        a.len[v] = (l == (int32_t)v) ? (r.x + r.y - 1) : 0;
+        int32_t l, pp;
+        if (E[0] <= E[1]) { l = E[0]; pp = D[0] + 1; } else { l = E[1]; pp = D[1] + 1; }
+        a.path_id[g] = l;
+        a.pos[g] = pp;
+        a.len[g] = (l == g) ? (D[0] + D[1] + 1) : 0;
     }
 }
 
@@ -289,14 +529,17 @@ static size_t scan_temp_bytes(int64_t N) {
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     ForestWs t;
     const size_t n = (size_t)(N > 0 ? N : 1);
-    t.q[0] = c.take<int32_t>(2 * n);
-    t.q[1] = c.take<int32_t>(2 * n);
-    t.mk[0] = c.take<uint64_t>(2 * n);
-    t.mk[1] = c.take<uint64_t>(2 * n);
-    // the rank scan reuses the min-key buffers for r (8 bytes per vertex each)
-    t.r[0] = (int32_t*)t.mk[0];
-    t.r[1] = (int32_t*)t.mk[1];
-    t.ekey = c.take<uint64_t>(2 * n);
+    for (int i = 0; i < 2; i++) {
+        t.rq1[i] = c.take<int2>(n);
+        t.rk1[i] = c.take<ulonglong2>(n);
+        t.rq2[i] = c.take<int2>(n);
+        t.rr2[i] = c.take<int2>(n);
+    }
+    t.cyc_k = c.take<uint64_t>(n);
+    t.end2 = c.take<int2>(n);
+    t.dist2 = c.take<int2>(n);
+    t.list1 = c.take<int32_t>(n);
+    t.list2 = c.take<int32_t>(n);
     t.len = c.take<int32_t>(n);
     t.off = c.take<int32_t>(n);
     t.ctl = c.take<int>(256);
@@ -309,7 +552,15 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
 static int max_steps_for(int64_t N) {
     int s = 0;
     while (s < 40 && ((int64_t)1 << s) < N) s++;
-    return s + 3;  // ceil(log2 N) + margin for cycle detection and the final copy
+    return s + 3;  // ceil(log2 N) + margin for cycle detection
+}
+
+template <class K>
+static int coop_launch(K kernel, int block, ForestArgs& a, cudaStream_t s) {
+    const int grid = persistent_grid((const void*)kernel, block);
+    void* args[] = {&a};
+    LF_CUDA(cudaLaunchCooperativeKernel((const void*)kernel, grid, block, args, 0, s));
+    return LF_OK;
 }
 
 int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
@@ -319,45 +570,63 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         if (n_cycles) LF_CUDA(cudaMemsetAsync(n_cycles, 0, sizeof(int64_t), s));
         return LF_OK;
     }
+    static bool attr_done = false;
+    const int smem = (int)sizeof(TileSmem);
+    if (!attr_done) {
+        LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local1, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local2, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local3, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        attr_done = true;
+    }
     LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
     if (n_cycles) LF_CUDA(cudaMemsetAsync(n_cycles, 0, sizeof(int64_t), s));
-    const int steps = max_steps_for(N) < kMaxSteps ? max_steps_for(N) : kMaxSteps;
+    ForestArgs a;
+    a.N = N;
+    a.pi2 = (const int2*)pi2;
+    a.pi2_w = (const float2*)pi2_w;
+    a.forest = (int2*)forest;
+    for (int i = 0; i < 2; i++) {
+        a.rq1[i] = w.rq1[i];
+        a.rk1[i] = w.rk1[i];
+        a.rq2[i] = w.rq2[i];
+        a.rr2[i] = w.rr2[i];
+    }
+    a.cyc_k = w.cyc_k;
+    a.list1 = w.list1;
+    a.end2 = w.end2;
+    a.dist2 = w.dist2;
+    a.list2 = w.list2;
+    a.ctl = w.ctl;
+    a.path_id = path_id;
+    a.pos = pos;
+    a.len = w.len;
+    a.n_cycles = (unsigned long long*)n_cycles;
+    a.max_steps = max_steps_for(N) < kMaxSteps ? max_steps_for(N) : kMaxSteps;
+    const int tiles = (int)((N + LB - 1) / LB);
     {
-        CycleArgs a;
-        a.N = N;
-        a.pi2 = (const int2*)pi2;
-        a.pi2_w = (const float2*)pi2_w;
-        a.q0 = (int2*)w.q[0];
-        a.q1 = (int2*)w.q[1];
-        a.m0 = (ulonglong2*)w.mk[0];
-        a.m1 = (ulonglong2*)w.mk[1];
-        a.ekey = (ulonglong2*)w.ekey;
-        a.forest = (int2*)forest;
-        a.ctl = w.ctl;
-        a.n_cycles = (unsigned long long*)n_cycles;
-        a.max_steps = steps;
-        const int grid = persistent_grid((const void*)k_cycle_scan, 256);
-        void* args[] = {&a};
-        LF_PROF("cycle_scan", -1, s);
-        LF_CUDA(cudaLaunchCooperativeKernel((const void*)k_cycle_scan, grid, 256, args, 0, s));
+        LF_PROF("lf_local1", -1, s);
+        k_lf_local1<<<tiles, LT, smem, s>>>(a);
+        LF_CUDA(cudaGetLastError());
     }
     {
-        RankArgs a;
-        a.N = N;
-        a.forest = (const int2*)forest;
-        a.q0 = (int2*)w.q[0];
-        a.q1 = (int2*)w.q[1];
-        a.r0 = (int2*)w.r[0];
-        a.r1 = (int2*)w.r[1];
-        a.path_id = path_id;
-        a.pos = pos;
-        a.len = w.len;
-        a.ctl = w.ctl;
-        a.max_steps = steps;
-        const int grid = persistent_grid((const void*)k_rank_scan, 256);
-        void* args[] = {&a};
-        LF_PROF("rank_scan", -1, s);
-        LF_CUDA(cudaLaunchCooperativeKernel((const void*)k_rank_scan, grid, 256, args, 0, s));
+        LF_PROF("red_scan_cycles", -1, s);
+        int rc = coop_launch(k_red_scan<true>, 256, a, s);
+        if (rc) return rc;
+    }
+    {
+        LF_PROF("lf_local2", -1, s);
+        k_lf_local2<<<tiles, LT, smem, s>>>(a);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("red_scan_ranks", -1, s);
+        int rc = coop_launch(k_red_scan<false>, 256, a, s);
+        if (rc) return rc;
+    }
+    {
+        LF_PROF("lf_local3", -1, s);
+        k_lf_local3<<<tiles, LT, smem, s>>>(a);
+        LF_CUDA(cudaGetLastError());
     }
     {
         LF_PROF("path_offsets", -1, s);

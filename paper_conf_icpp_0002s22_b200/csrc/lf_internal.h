@@ -67,14 +67,19 @@ int factor_dispatch(const lf_csr_t* A, int n, const lf_factor_opts_t* o, int32_t
                     const FactorWs& w, cudaStream_t s);
 
 struct ForestWs {
-    int32_t* q[2];       // [2N] stride neighbours, ping-pong
-    uint64_t* mk[2];     // [2N] min edge key per direction (cycle scan), ping-pong
-    int32_t* r[2];       // [2N] positions (rank scan), ping-pong
-    uint64_t* ekey;      // [2N] key of the edge in each slot of pi2
-    int32_t* len;        // [N] path length at the path-ID vertex, else 0
-    int32_t* off;        // [N] exclusive scan of len
-    int* ctl;            // [256] per-step "not done" counters, cycle count
-    void* scan_tmp;      // CUB temp storage
+    int2* rq1[2];          // reduced graph, cycle pass: stride pointers (ping-pong)
+    ulonglong2* rk1[2];    //   min edge keys
+    int2* rq2[2];          // reduced graph, rank pass: stride pointers
+    int2* rr2[2];          //   distances
+    uint64_t* cyc_k;       // [N] weakest edge key of the global cycle through a boundary vertex
+    int2* end2;            // [N] path ends per direction of a boundary vertex
+    int2* dist2;           // [N] distances to them
+    int32_t* list1;        // boundary vertices, cycle pass
+    int32_t* list2;        // boundary vertices, rank pass
+    int32_t* len;          // [N] path length at the path-ID vertex, else 0
+    int32_t* off;          // [N] exclusive scan of len
+    int* ctl;              // [256] per-step counters, list sizes
+    void* scan_tmp;        // CUB temp storage
     size_t scan_tmp_bytes;
 };
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w);
