@@ -16,9 +16,9 @@
 //      the reduced graph whose nodes are boundary vertices and whose links are either a
 //      cross-block edge or a whole local segment (weighted by its length and minimum
 //      key).  It leaves as soon as every node is done.
-//   3. expand (k_lf_local2 / k_lf_local3): the block-local scan is recomputed from the
-//      input (cheaper than storing it) and combined with the reduced results of the two
-//      terminals of each local segment.
+//   3. expand (k_lf_local2 / k_lf_local3): the stored local result of each vertex (its
+//      two local terminals and distances, 4-8 bytes) is combined with the reduced results
+//      of those terminals.
 //
 // Step (1) (cycles) and step (2) (positions) each take one local + one reduced pass; the
 // forest is written between them by the fused kernel k_lf_local2, which also runs the
@@ -65,94 +65,102 @@ __device__ __forceinline__ uint64_t edge_key(int32_t v, int32_t w, float wabs, i
 struct TileSmem {
     int2 nb[LB];          // global neighbours (slot order), -1 = none
     short2 P[LB];         // local stride pointer per direction, or marker -(t+1), t local
-    short2 R[LB];         // local edges covered per direction
-    ulonglong2 K[LB];     // min edge key per direction (cycle pass only)
+    short2 R[LB];         // local edges covered per direction (rank pass)
+    uint64_t K0[LB];      // min edge key, direction 0 (cycle pass)
+    uint64_t K1[LB];      // min edge key, direction 1
 };
 
 __device__ __forceinline__ bool is_local(int32_t x, int32_t b0) {
     return x >= b0 && x < b0 + LB;
 }
 
-// Bidirectional scan inside the tile (Alg. 3 / its min variant restricted to local links).
-// On return (after a __syncthreads) s.P/s.R/s.K hold, for every local vertex and each
-// direction, either a terminal marker -(t+1) with the local distance and min key to t, or
-// (both directions non-negative) a completed local cycle whose min key is min(K.x, K.y).
-// WITH_KEYS: also carry min keys (cycle pass).  ek[k] = keys of the own vertices' slots.
-template <bool WITH_KEYS>
-__device__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT]) {
+// Bidirectional scan inside the tile (Alg. 3, or its min variant when MINK, restricted
+// to local links: a missing or non-local neighbour ends the walk like a path end).
+// Each thread keeps its own vertices' state in registers and publishes it to shared
+// memory for its neighbours; vertices whose both pointers are terminal markers are final
+// and drop out (markers are absorbing, so their published state stays valid).  Cycle
+// vertices keep stepping until the whole tile is done (their neighbours read them).
+// On return P[k] holds, per direction, a terminal marker -(t+1) (t local) or, on a
+// completed local cycle, non-negative pointers; R[k] the local distances (rank pass);
+// K[k] the min edge keys (cycle pass).  ek: keys of the own vertices' slots.
+template <bool MINK>
+__device__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
+                          int2 (&R)[VPT], ulonglong2 (&K)[VPT]) {
     const int tid = threadIdx.x;
-    // init: stride-1 local neighbours; a missing or non-local neighbour ends the walk
+    bool fin[VPT];
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = tid + k * LT;
         const int2 nb = s.nb[u];
-        short2 p;
-        short2 r;
         const bool l0 = nb.x >= 0 && is_local(nb.x, b0);
         const bool l1 = nb.y >= 0 && is_local(nb.y, b0);
-        p.x = l0 ? (short)(nb.x - b0) : (short)(-(u + 1));
-        p.y = l1 ? (short)(nb.y - b0) : (short)(-(u + 1));
-        r.x = l0 ? 1 : 0;
-        r.y = l1 ? 1 : 0;
-        s.P[u] = p;
-        s.R[u] = r;
-        if (WITH_KEYS) {
-            ulonglong2 kk;
-            kk.x = l0 ? ek[k].x : KEY_INF;
-            kk.y = l1 ? ek[k].y : KEY_INF;
-            s.K[u] = kk;
+        P[k] = make_int2(l0 ? nb.x - b0 : -(u + 1), l1 ? nb.y - b0 : -(u + 1));
+        fin[k] = !l0 && !l1;
+        s.P[u] = make_short2((short)P[k].x, (short)P[k].y);
+        if (MINK) {
+            K[k].x = l0 ? ek[k].x : KEY_INF;
+            K[k].y = l1 ? ek[k].y : KEY_INF;
+            s.K0[u] = K[k].x;
+            s.K1[u] = K[k].y;
+        } else {
+            R[k] = make_int2(l0 ? 1 : 0, l1 ? 1 : 0);
+            s.R[u] = make_short2((short)R[k].x, (short)R[k].y);
         }
     }
-    __syncthreads();
+    int notdone = 0;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) notdone |= !fin[k];
+    if (!__syncthreads_or(notdone)) return;
     for (int step = 0; step < 16; step++) {
-        short2 np[VPT], nr[VPT];
-        ulonglong2 nk[VPT];
-        int notdone = 0;
+        int2 nP[VPT], nR[VPT];
+        ulonglong2 nK[VPT];
 #pragma unroll
         for (int k = 0; k < VPT; k++) {
             const int u = tid + k * LT;
-            const short2 p = s.P[u];
-            short2 r = s.R[u];
-            short2 q = p;
-            ulonglong2 kk;
-            if (WITH_KEYS) kk = s.K[u];
-            if (p.x >= 0) {
-                const short2 pw = s.P[p.x];
-                const short2 rw = s.R[p.x];
-                if (pw.x != u) {
-                    q.x = pw.x; r.x = (short)(r.x + rw.x);
-                    if (WITH_KEYS) kk.x = umin64(kk.x, s.K[p.x].x);
-                } else if (pw.y != u) {
-                    q.x = pw.y; r.x = (short)(r.x + rw.y);
-                    if (WITH_KEYS) kk.x = umin64(kk.x, s.K[p.x].y);
+            nP[k] = P[k];
+            if (MINK) nK[k] = K[k]; else nR[k] = R[k];
+            if (fin[k]) continue;
+#pragma unroll
+            for (int i = 0; i < 2; i++) {
+                const int w = i ? P[k].y : P[k].x;
+                if (w < 0) continue;
+                const short2 pw = s.P[w];
+                int j = -1;
+                if (pw.x != u) j = 0;
+                else if (pw.y != u) j = 1;
+                if (j < 0) continue;  // stall (reading c13)
+                const int tgt = j ? pw.y : pw.x;
+                if (i) nP[k].y = tgt; else nP[k].x = tgt;
+                if (MINK) {
+                    const uint64_t kv = j ? s.K1[w] : s.K0[w];
+                    if (i) nK[k].y = umin64(nK[k].y, kv); else nK[k].x = umin64(nK[k].x, kv);
+                } else {
+                    const short2 rw = s.R[w];
+                    const int dv = j ? rw.y : rw.x;
+                    if (i) nR[k].y += dv; else nR[k].x += dv;
                 }
             }
-            if (p.y >= 0) {
-                const short2 pw = s.P[p.y];
-                const short2 rw = s.R[p.y];
-                if (pw.x != u) {
-                    q.y = pw.x; r.y = (short)(r.y + rw.x);
-                    if (WITH_KEYS) kk.y = umin64(kk.y, s.K[p.y].x);
-                } else if (pw.y != u) {
-                    q.y = pw.y; r.y = (short)(r.y + rw.y);
-                    if (WITH_KEYS) kk.y = umin64(kk.y, s.K[p.y].y);
-                }
-            }
-            np[k] = q;
-            nr[k] = r;
-            if (WITH_KEYS) nk[k] = kk;
-            const bool path_done = q.x < 0 && q.y < 0;
-            bool cyc_done = false;
-            if (WITH_KEYS) cyc_done = q.x >= 0 && q.y >= 0 && (kk.x == kk.y || q.x == q.y);
-            notdone |= !(path_done || cyc_done);
         }
         __syncthreads();
+        notdone = 0;
 #pragma unroll
         for (int k = 0; k < VPT; k++) {
+            if (fin[k]) continue;
             const int u = tid + k * LT;
-            s.P[u] = np[k];
-            s.R[u] = nr[k];
-            if (WITH_KEYS) s.K[u] = nk[k];
+            P[k] = nP[k];
+            s.P[u] = make_short2((short)P[k].x, (short)P[k].y);
+            if (MINK) {
+                K[k] = nK[k];
+                s.K0[u] = K[k].x;
+                s.K1[u] = K[k].y;
+            } else {
+                R[k] = nR[k];
+                s.R[u] = make_short2((short)R[k].x, (short)R[k].y);
+            }
+            fin[k] = P[k].x < 0 && P[k].y < 0;
+            bool cyc_done = false;
+            if (MINK) cyc_done = P[k].x >= 0 && P[k].y >= 0 && (K[k].x == K[k].y || P[k].x == P[k].y);
+            notdone |= !(fin[k] || cyc_done);
         }
         if (!__syncthreads_or(notdone)) break;
     }
@@ -179,6 +187,10 @@ struct ForestArgs {
     const int2* __restrict__ pi2;
     const float2* __restrict__ pi2_w;
     int2* forest;
+    // per-vertex local results (written by the local pass, read by the expand pass)
+    short2* loc1;          // [N] local terminal markers of the cycle pass (>= 0: local cycle)
+    uint64_t* kst;         // [N] weakest key of a local cycle (written on local cycles only)
+    int2* loc2;            // [N] (terminal markers as shorts packed, local distances)
     // reduced graph, pass 1 (cycles)
     int2* rq1[2];
     ulonglong2* rk1[2];
@@ -236,9 +248,9 @@ __device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem
 // reduced-graph direction of boundary vertex g through its slot i:
 //   none -> end marker at g (distance 0); remote -> the neighbour (distance 1);
 //   local -> the segment's other terminal t: t itself if t continues in another block,
-//   else an end marker at t (distance = local length, key = segment min key).
+//   else an end marker at t (distance = local length).
 __device__ __forceinline__ void reduced_dir(const TileSmem& s, int32_t b0, int32_t g, int2 nb, int i,
-                                            short2 p, short2 r, int32_t& q, int32_t& d) {
+                                            int2 p, int2 r, int32_t& q, int32_t& d) {
     const int32_t x = i ? nb.y : nb.x;
     if (x < 0) { q = -(g + 1); d = 0; return; }
     if (!is_local(x, b0)) { q = x; d = 1; return; }
@@ -250,7 +262,8 @@ __device__ __forceinline__ void reduced_dir(const TileSmem& s, int32_t b0, int32
     d = i ? r.y : r.x;
 }
 
-// Pass 1, local part: emit the reduced-graph records of boundary vertices.
+// Pass 1, local part: local min-scan; store the local results; emit the reduced-graph
+// records of boundary vertices.
 __global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
@@ -258,7 +271,9 @@ __global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
     load_tile(a.pi2, s, b0, a.N);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
-    tile_scan<true>(s, b0, ek);
+    int2 P[VPT], R[VPT];
+    ulonglong2 K[VPT];
+    tile_scan<true>(s, b0, ek, P, R, K);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -267,17 +282,18 @@ __global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
         const bool r0 = nb.x >= 0 && !is_local(nb.x, b0);
         const bool r1 = nb.y >= 0 && !is_local(nb.y, b0);
         const bool boundary = g < a.N && (r0 || r1);
+        if (g < a.N) {
+            a.loc1[g] = make_short2((short)P[k].x, (short)P[k].y);
+            if (P[k].x >= 0 && P[k].y >= 0) a.kst[g] = umin64(K[k].x, K[k].y);
+        }
         if (boundary) {
-            const short2 p = s.P[u];
-            const short2 r = s.R[u];
-            const ulonglong2 kk = s.K[u];
             int32_t q0, q1, d0, d1;
-            reduced_dir(s, b0, g, nb, 0, p, r, q0, d0);
-            reduced_dir(s, b0, g, nb, 1, p, r, q1, d1);
+            reduced_dir(s, b0, g, nb, 0, P[k], R[k], q0, d0);
+            reduced_dir(s, b0, g, nb, 1, P[k], R[k], q1, d1);
             // key of each reduced link: the remote edge's key, or the segment's min key
             ulonglong2 rk;
-            rk.x = (nb.x < 0) ? KEY_INF : (r0 ? ek[k].x : kk.x);
-            rk.y = (nb.y < 0) ? KEY_INF : (r1 ? ek[k].y : kk.y);
+            rk.x = (nb.x < 0) ? KEY_INF : (r0 ? ek[k].x : K[k].x);
+            rk.y = (nb.y < 0) ? KEY_INF : (r1 ? ek[k].y : K[k].y);
             const int2 q = make_int2(q0, q1);
             a.rq1[0][g] = q; a.rq1[1][g] = q;
             a.rk1[0][g] = rk; a.rk1[1][g] = rk;
@@ -387,7 +403,6 @@ __global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
     load_tile(a.pi2, s, b0, a.N);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
-    tile_scan<true>(s, b0, ek);
     // weakest edge of the cycle through each own vertex (INF: not on a cycle)
     int2 f[VPT];
     unsigned long long ncyc = 0;
@@ -398,11 +413,10 @@ __global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
         const int2 nb = s.nb[u];
         f[k] = nb;
         if (g >= a.N) continue;
-        const short2 p = s.P[u];
+        const short2 p = a.loc1[g];
         uint64_t kstar = KEY_INF;
         if (p.x >= 0 && p.y >= 0) {  // local cycle
-            const ulonglong2 kk = s.K[u];
-            kstar = umin64(kk.x, kk.y);
+            kstar = a.kst[g];
         } else {
             // a segment: its cycle status is that of a terminal that continues in another
             // block (a segment ending in a path end is on a path)
@@ -437,7 +451,9 @@ __global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
 #pragma unroll
     for (int k = 0; k < VPT; k++) s.nb[threadIdx.x + k * LT] = f[k];
     __syncthreads();
-    tile_scan<false>(s, b0, ek);
+    int2 P[VPT], R[VPT];
+    ulonglong2 K[VPT];
+    tile_scan<false>(s, b0, ek, P, R, K);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -446,12 +462,16 @@ __global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
         const bool r0 = nb.x >= 0 && !is_local(nb.x, b0);
         const bool r1 = nb.y >= 0 && !is_local(nb.y, b0);
         const bool boundary = g < a.N && (r0 || r1);
+        if (g < a.N) {
+            // terminal markers (16 bits each) and local distances (16 bits each)
+            const uint32_t pp = ((uint32_t)(uint16_t)(short)P[k].x) | ((uint32_t)(uint16_t)(short)P[k].y << 16);
+            const uint32_t rr = ((uint32_t)(uint16_t)R[k].x) | ((uint32_t)(uint16_t)R[k].y << 16);
+            a.loc2[g] = make_int2((int)pp, (int)rr);
+        }
         if (boundary) {
-            const short2 p = s.P[u];
-            const short2 r = s.R[u];
             int32_t q0, q1, d0, d1;
-            reduced_dir(s, b0, g, nb, 0, p, r, q0, d0);
-            reduced_dir(s, b0, g, nb, 1, p, r, q1, d1);
+            reduced_dir(s, b0, g, nb, 0, P[k], R[k], q0, d0);
+            reduced_dir(s, b0, g, nb, 1, P[k], R[k], q1, d1);
             const int2 q = make_int2(q0, q1);
             const int2 d = make_int2(d0, d1);
             a.rq2[0][g] = q; a.rq2[1][g] = q;
@@ -467,20 +487,19 @@ __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = blockIdx.x * LB;
     load_tile(a.forest, s, b0, a.N);
-    ulonglong2 ek[VPT];
-    tile_scan<false>(s, b0, ek);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
         const int32_t g = b0 + u;
         if (g >= a.N) continue;
-        const short2 p = s.P[u];
-        const short2 r = s.R[u];
+        const int2 lc = a.loc2[g];
+        const int px = (short)(lc.x & 0xffff), py = (short)((uint32_t)lc.x >> 16);
+        const int rx = lc.y & 0xffff, ry = (int)((uint32_t)lc.y >> 16);
         int32_t E[2], D[2];
 #pragma unroll
         for (int i = 0; i < 2; i++) {
-            const int t = -((i ? p.y : p.x) + 1);  // local terminal in direction i
-            const int32_t d = i ? r.y : r.x;
+            const int t = -((i ? py : px) + 1);  // local terminal in direction i
+            const int32_t d = i ? ry : rx;
             const int2 nbt = s.nb[t];
             // the outward slot of t: slot i itself when t == u (the walk never left u)
             const int so = (t == u) ? i : outward_slot(nbt, b0);
@@ -536,6 +555,9 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
         t.rr2[i] = c.take<int2>(n);
     }
     t.cyc_k = c.take<uint64_t>(n);
+    t.loc1 = c.take<short2>(n);
+    t.kst = c.take<uint64_t>(n);
+    t.loc2 = c.take<int2>(n);
     t.end2 = c.take<int2>(n);
     t.dist2 = c.take<int2>(n);
     t.list1 = c.take<int32_t>(n);
@@ -592,6 +614,9 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         a.rr2[i] = w.rr2[i];
     }
     a.cyc_k = w.cyc_k;
+    a.loc1 = w.loc1;
+    a.kst = w.kst;
+    a.loc2 = w.loc2;
     a.list1 = w.list1;
     a.end2 = w.end2;
     a.dist2 = w.dist2;

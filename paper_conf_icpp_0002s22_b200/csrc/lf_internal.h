@@ -71,6 +71,9 @@ struct ForestWs {
     ulonglong2* rk1[2];    //   min edge keys
     int2* rq2[2];          // reduced graph, rank pass: stride pointers
     int2* rr2[2];          //   distances
+    short2* loc1;          // [N] local results of the cycle pass
+    uint64_t* kst;         // [N] weakest key of a local cycle
+    int2* loc2;            // [N] local results of the rank pass
     uint64_t* cyc_k;       // [N] weakest edge key of the global cycle through a boundary vertex
     int2* end2;            // [N] path ends per direction of a boundary vertex
     int2* dist2;           // [N] distances to them
