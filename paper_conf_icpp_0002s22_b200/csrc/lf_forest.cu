@@ -64,10 +64,16 @@ __device__ __forceinline__ uint64_t edge_key(int32_t v, int32_t w, float wabs, i
 // shared-memory state of one tile
 struct TileSmem {
     int2 nb[LB];          // global neighbours (slot order), -1 = none
-    short2 P[LB];         // local stride pointer per direction, or marker -(t+1), t local
-    short2 R[LB];         // local edges covered per direction (rank pass)
+    float2 w[LB];         // |w| per slot (cycle pass)
+    short2 P[LB];         // stride pointer per direction (vertex or splitter node), or marker
+    short2 R[LB];         // edges covered per direction (rank pass)
     uint64_t K0[LB];      // min edge key, direction 0 (cycle pass)
     uint64_t K1[LB];      // min edge key, direction 1
+    short sidx[LB];       // splitter node index of a vertex, -1 if not a splitter
+    short spl[LB];        // local vertex of each splitter node
+    short2 recS[LB];      // per face: (node << 1 | start slot) of the walk that visited it
+    short2 recD[LB];      // per face: distance to that node
+    int nspl;             // number of splitter nodes
 };
 
 __device__ __forceinline__ bool is_local(int32_t x, int32_t b0) {
@@ -85,12 +91,13 @@ __device__ __forceinline__ bool is_local(int32_t x, int32_t b0) {
 // K[k] the min edge keys (cycle pass).  ek: keys of the own vertices' slots.
 template <bool MINK>
 __device__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
-                          int2 (&R)[VPT], ulonglong2 (&K)[VPT]) {
+                          int2 (&R)[VPT], ulonglong2 (&K)[VPT], const bool (&skip)[VPT]) {
     const int tid = threadIdx.x;
     bool fin[VPT];
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = tid + k * LT;
+        if (skip[k]) { fin[k] = true; continue; }
         const int2 nb = s.nb[u];
         const bool l0 = nb.x >= 0 && is_local(nb.x, b0);
         const bool l1 = nb.y >= 0 && is_local(nb.y, b0);
@@ -166,6 +173,186 @@ __device__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
     }
 }
 
+constexpr int kSplitShift = 28;  // splitter density 1/16 from the top 4 bits of a hash
+
+__device__ __forceinline__ bool hashed_splitter(int32_t g) {
+    return (((uint32_t)g * 0x9E3779B1u) >> kSplitShift) == 0u;
+}
+
+// Block-local ranking by a ruling set.  Same outputs as tile_scan, but
+// O(1) work per vertex: splitters (segment terminals plus hashed vertices, density 1/16)
+// walk sequentially through shared memory to the next splitter in each direction,
+// recording (node, distance) in every vertex they pass; the bidirectional scan then runs
+// on the splitter nodes only; every vertex combines its record with its node's result.
+// Cycles without a splitter are left unvisited and fall back to tile_scan (cycle pass
+// only -- a forest has none).
+template <bool MINK>
+__device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
+                          int2 (&R)[VPT], ulonglong2 (&K)[VPT]) {
+    const int tid = threadIdx.x;
+    if (tid == 0) s.nspl = 0;
+    __syncthreads();
+    // 1. splitters: terminals of the local structure (a slot that is missing or remote) and
+    //    hashed vertices; node numbering by a shared counter (order does not matter)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const int2 nb = s.nb[u];
+        const bool l0 = nb.x >= 0 && is_local(nb.x, b0);
+        const bool l1 = nb.y >= 0 && is_local(nb.y, b0);
+        const bool sp = !l0 || !l1 || hashed_splitter(b0 + u);
+        short id = -1;
+        if (sp) id = (short)atomicAdd(&s.nspl, 1);
+        s.sidx[u] = id;
+        if (sp) s.spl[id] = (short)u;
+        s.recS[u] = make_short2(-1, -1);
+    }
+    __syncthreads();
+    const int C = s.nspl;
+    // 2. walks: one per (node, slot), sequential through non-splitters
+    for (int wk = tid; wk < 2 * C; wk += LT) {
+        const int i = wk >> 1, f = wk & 1;
+        const int su = s.spl[i];
+        const int2 nbs = s.nb[su];
+        const int32_t x = f ? nbs.y : nbs.x;
+        short ptr = (short)(-(i + 1));
+        int dist = 0;
+        uint64_t km = KEY_INF;
+        if (x >= 0 && is_local(x, b0)) {
+            int prev = su, cur = x - b0, d = 1;
+            if (MINK) {
+                const float2 ws = s.w[su];
+                const int mn = su < cur ? su : cur;
+                km = edge_key(b0 + su, x, f ? ws.y : ws.x, s.nb[mn]);
+            }
+            while (s.sidx[cur] < 0) {
+                const int2 nbc = s.nb[cur];
+                const int face = (nbc.x == b0 + prev) ? 0 : 1;
+                if (face == 0) { s.recS[cur].x = (short)((i << 1) | f); s.recD[cur].x = (short)d; }
+                else { s.recS[cur].y = (short)((i << 1) | f); s.recD[cur].y = (short)d; }
+                const int nxt = (face ? nbc.x : nbc.y) - b0;  // local (else cur were a splitter)
+                if (MINK) {
+                    const float2 wc = s.w[cur];
+                    const int mn = cur < nxt ? cur : nxt;
+                    km = umin64(km, edge_key(b0 + cur, b0 + nxt, face ? wc.x : wc.y, s.nb[mn]));
+                }
+                prev = cur;
+                cur = nxt;
+                d++;
+            }
+            ptr = s.sidx[cur];
+            dist = d;
+        }
+        if (f) { s.P[i].y = ptr; s.R[i].y = (short)dist; s.K1[i] = km; }
+        else { s.P[i].x = ptr; s.R[i].x = (short)dist; s.K0[i] = km; }
+    }
+    __syncthreads();
+    // 3. bidirectional scan over the splitter nodes (node arrays in s.P/s.R/s.K*)
+    for (int step = 0; step < 16; step++) {
+        int notdone = 0;
+        short2 nP[VPT], nR[VPT];
+        uint64_t nk0[VPT], nk1[VPT];
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int i = tid + k * LT;
+            if (i >= C) continue;
+            const short2 p = s.P[i];
+            short2 q = p, r = s.R[i];
+            uint64_t k0 = 0, k1 = 0;
+            if (MINK) { k0 = s.K0[i]; k1 = s.K1[i]; }
+#pragma unroll
+            for (int dd = 0; dd < 2; dd++) {
+                const int w = dd ? p.y : p.x;
+                if (w < 0) continue;
+                const short2 pw = s.P[w];
+                int j = -1;
+                if (pw.x != i) j = 0;
+                else if (pw.y != i) j = 1;
+                if (j < 0) continue;  // stall (reading c13)
+                const short tgt = j ? pw.y : pw.x;
+                if (dd) q.y = tgt; else q.x = tgt;
+                if (MINK) {
+                    const uint64_t kv = j ? s.K1[w] : s.K0[w];
+                    if (dd) k1 = umin64(k1, kv); else k0 = umin64(k0, kv);
+                } else {
+                    const short2 rw = s.R[w];
+                    const short dv = j ? rw.y : rw.x;
+                    if (dd) r.y = (short)(r.y + dv); else r.x = (short)(r.x + dv);
+                }
+            }
+            nP[k] = q;
+            nR[k] = r;
+            nk0[k] = k0;
+            nk1[k] = k1;
+            const bool path_done = q.x < 0 && q.y < 0;
+            bool cyc_done = false;
+            if (MINK) cyc_done = q.x >= 0 && q.y >= 0 && (k0 == k1 || q.x == q.y);
+            notdone |= !(path_done || cyc_done);
+        }
+        __syncthreads();
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int i = tid + k * LT;
+            if (i >= C) continue;
+            s.P[i] = nP[k];
+            if (MINK) { s.K0[i] = nk0[k]; s.K1[i] = nk1[k]; } else s.R[i] = nR[k];
+        }
+        if (!__syncthreads_or(notdone)) break;
+    }
+    // 4. expand: every vertex from its node (splitter) or its walk records
+    bool unvisited[VPT];
+    int any_unvisited = 0;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        unvisited[k] = false;
+        const int id = s.sidx[u];
+        if (id >= 0) {
+            const short2 p = s.P[id];
+            P[k] = make_int2(p.x >= 0 ? p.x : -(s.spl[-(p.x + 1)] + 1), p.y >= 0 ? p.y : -(s.spl[-(p.y + 1)] + 1));
+            if (MINK) { K[k].x = s.K0[id]; K[k].y = s.K1[id]; }
+            else { const short2 r = s.R[id]; R[k] = make_int2(r.x, r.y); }
+            continue;
+        }
+        const short2 rs = s.recS[u];
+        if (rs.x < 0 && rs.y < 0) { unvisited[k] = true; any_unvisited = 1; continue; }
+        const short2 rd = s.recD[u];
+#pragma unroll
+        for (int f = 0; f < 2; f++) {
+            const int rec = f ? rs.y : rs.x;
+            const int i = rec >> 1, f0 = rec & 1;
+            const short2 p = s.P[i];
+            const int away = f0 ^ 1;  // node i's direction that leads away from u
+            const int pa = away ? p.y : p.x;
+            if (pa >= 0) {  // node on a cycle: the cycle's weakest key is min(K0,K1)
+                if (f) P[k].y = 0; else P[k].x = 0;
+                if (MINK) { K[k].x = s.K0[i]; K[k].y = s.K1[i]; }
+                continue;
+            }
+            const int t = s.spl[-(pa + 1)];
+            const int dd = (f ? rd.y : rd.x) + (MINK ? 0 : (away ? s.R[i].y : s.R[i].x));
+            if (f) { P[k].y = -(t + 1); R[k].y = dd; } else { P[k].x = -(t + 1); R[k].x = dd; }
+        }
+        // a vertex on a cycle: make both pointers non-negative (cycle flag)
+        if (P[k].x >= 0 || P[k].y >= 0) { P[k].x = 0; P[k].y = 0; }
+    }
+    if (MINK) {
+        if (__syncthreads_or(any_unvisited)) {
+            // splitter-free local cycles: the pointer-jumping scan on them alone
+            bool skip[VPT];
+#pragma unroll
+            for (int k = 0; k < VPT; k++) skip[k] = !unvisited[k];
+            int2 P2[VPT], R2[VPT];
+            ulonglong2 K2[VPT];
+            tile_scan<true>(s, b0, ek, P2, R2, K2, skip);
+#pragma unroll
+            for (int k = 0; k < VPT; k++)
+                if (unvisited[k]) { P[k] = P2[k]; K[k] = K2[k]; }
+        }
+    }
+    __syncthreads();
+}
+
 // the slot of local terminal t (t not the walk's start) that leaves its segment: the
 // one that is not a local link (a remote neighbour or none)
 __device__ __forceinline__ int outward_slot(int2 nbt, int32_t b0) {
@@ -211,7 +398,7 @@ struct ForestArgs {
 };
 
 // keys of the own vertices' slots (global; a remote min endpoint needs one gather)
-__device__ __forceinline__ void slot_keys(const ForestArgs& a, const TileSmem& s, int32_t b0,
+__device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int32_t b0,
                                          ulonglong2 (&ek)[VPT]) {
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
@@ -220,8 +407,9 @@ __device__ __forceinline__ void slot_keys(const ForestArgs& a, const TileSmem& s
         const int2 nb = s.nb[u];
         ek[k].x = KEY_INF;
         ek[k].y = KEY_INF;
-        if (g >= a.N) continue;
+        if (g >= a.N) { s.w[u] = make_float2(0.f, 0.f); continue; }
         const float2 w = a.pi2_w[g];
+        s.w[u] = w;
         if (nb.x >= 0) {
             const int32_t mn = g < nb.x ? g : nb.x;
             const int2 nbm = is_local(mn, b0) ? s.nb[mn - b0] : a.pi2[mn];
@@ -273,7 +461,7 @@ __global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
     slot_keys(a, s, b0, ek);
     int2 P[VPT], R[VPT];
     ulonglong2 K[VPT];
-    tile_scan<true>(s, b0, ek, P, R, K);
+    tile_rank<true>(s, b0, ek, P, R, K);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -453,7 +641,7 @@ __global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
     __syncthreads();
     int2 P[VPT], R[VPT];
     ulonglong2 K[VPT];
-    tile_scan<false>(s, b0, ek, P, R, K);
+    tile_rank<false>(s, b0, ek, P, R, K);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
