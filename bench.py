@@ -286,6 +286,7 @@ def main():
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         t_step = float(t.item())
 
+    fstats = lf.forest_stats(N, P.ws_l)
     live = P.fac["live"].cpu().numpy()
     M = P.M
     lr, ln = [int(x) for x in live[:M]], [int(x) for x in live[M:2 * M]]
@@ -362,6 +363,7 @@ def main():
                 "ms_per_launch": round(kavg[dom], 5) if dom else None,
             },
             "kernels_ms": {k: round(v, 5) for k, v in sorted(kavg.items(), key=lambda t: -t[1])},
+            "forest_stats": fstats,
             "live_rows": lr,
             "live_nnz": ln,
             "e2e": {"value": round(ws * E / (e2e_t * 1e-3) / 1e6, 2), "unit": "Medges/s",

@@ -228,6 +228,15 @@ int lf_linear_forest(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t*
     return forest_run(N, pi2, pi2_w, forest, path_id, pos, perm, iperm, n_cycles, w, (cudaStream_t)stream);
 }
 
+int lf_forest_stats(int64_t N, void* ws, size_t ws_bytes, int32_t* out, int cap) {
+    g_err[0] = 0;
+    Carve c(ws, ws_bytes);
+    ForestWs w;
+    forest_ws_carve(c, N, &w);
+    if (!ws || !c.ok()) return set_error(LF_ENOMEM, "lf_forest_stats: workspace too small");
+    return forest_stats(w, out, cap);
+}
+
 int lf_tridiag(int64_t N, const int32_t* forest, const int32_t* iperm, const int32_t* pi2,
                const float* pi2_val, const float* diag, float* a, float* b, float* c, void* stream) {
     g_err[0] = 0;

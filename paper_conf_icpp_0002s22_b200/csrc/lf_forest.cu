@@ -46,6 +46,9 @@ constexpr int kCtlRed2 = 64;      // ctl[64..127] reduced scan 2
 constexpr int kCtlCnt1 = 128;     // boundary list sizes
 constexpr int kCtlCnt2 = 129;
 constexpr int kMaxSteps = 62;
+constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
+// ctl[192] splitter nodes (cycle pass), [193] unvisited vertices (fallback), [194] tiles
+// that needed the fallback, [195] splitter nodes (rank pass), [196] max node-scan steps
 
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 
@@ -188,7 +191,7 @@ __device__ __forceinline__ bool hashed_splitter(int32_t g) {
 // only -- a forest has none).
 template <bool MINK>
 __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
-                          int2 (&R)[VPT], ulonglong2 (&K)[VPT]) {
+                          int2 (&R)[VPT], ulonglong2 (&K)[VPT], int* stats) {
     const int tid = threadIdx.x;
     if (tid == 0) s.nspl = 0;
     __syncthreads();
@@ -209,6 +212,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
     }
     __syncthreads();
     const int C = s.nspl;
+    if (tid == 0 && stats) atomicAdd(&stats[MINK ? 0 : 3], C);
     // 2. walks: one per (node, slot), sequential through non-splitters
     for (int wk = tid; wk < 2 * C; wk += LT) {
         const int i = wk >> 1, f = wk & 1;
@@ -297,7 +301,10 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
             s.P[i] = nP[k];
             if (MINK) { s.K0[i] = nk0[k]; s.K1[i] = nk1[k]; } else s.R[i] = nR[k];
         }
-        if (!__syncthreads_or(notdone)) break;
+        if (!__syncthreads_or(notdone)) {
+            if (tid == 0 && stats) atomicMax(&stats[4], step + 1);
+            break;
+        }
     }
     // 4. expand: every vertex from its node (splitter) or its walk records
     bool unvisited[VPT];
@@ -337,7 +344,14 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         if (P[k].x >= 0 || P[k].y >= 0) { P[k].x = 0; P[k].y = 0; }
     }
     if (MINK) {
+        if (stats) {
+            int nu = 0;
+#pragma unroll
+            for (int k = 0; k < VPT; k++) nu += unvisited[k];
+            if (nu) atomicAdd(&stats[1], nu);
+        }
         if (__syncthreads_or(any_unvisited)) {
+            if (tid == 0 && stats) atomicAdd(&stats[2], 1);
             // splitter-free local cycles: the pointer-jumping scan on them alone
             bool skip[VPT];
 #pragma unroll
@@ -461,7 +475,7 @@ __global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
     slot_keys(a, s, b0, ek);
     int2 P[VPT], R[VPT];
     ulonglong2 K[VPT];
-    tile_rank<true>(s, b0, ek, P, R, K);
+    tile_rank<true>(s, b0, ek, P, R, K, a.ctl + kCtlStat);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -641,7 +655,7 @@ __global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
     __syncthreads();
     int2 P[VPT], R[VPT];
     ulonglong2 K[VPT];
-    tile_rank<false>(s, b0, ek, P, R, K);
+    tile_rank<false>(s, b0, ek, P, R, K, a.ctl + kCtlStat);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -851,6 +865,23 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         k_perm<<<persistent_grid((const void*)k_perm, 256), 256, 0, s>>>(N, path_id, pos, w.off, perm, iperm);
         LF_CUDA(cudaGetLastError());
     }
+    return LF_OK;
+}
+
+int forest_stats(const ForestWs& w, int32_t* out, int cap) {
+    int h[256];
+    LF_CUDA(cudaMemcpy(h, w.ctl, sizeof(h), cudaMemcpyDeviceToHost));
+    // [0] boundary vertices cycle pass, [1] rank pass, [2] reduced steps cycle, [3] rank,
+    // [4] splitter nodes cycle pass, [5] unvisited, [6] fallback tiles, [7] nodes rank pass,
+    // [8] max node-scan steps
+    int steps1 = 0, steps2 = 0;
+    for (int i = 0; i < 64; i++) {
+        if (h[kCtlRed1 + i]) steps1 = i + 2;
+        if (h[kCtlRed2 + i]) steps2 = i + 2;
+    }
+    int v[9] = {h[kCtlCnt1], h[kCtlCnt2], steps1, steps2, h[kCtlStat], h[kCtlStat + 1], h[kCtlStat + 2],
+                h[kCtlStat + 3], h[kCtlStat + 4]};
+    for (int i = 0; i < cap && i < 9; i++) out[i] = v[i];
     return LF_OK;
 }
 

@@ -91,6 +91,8 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
                int32_t* pos, int32_t* perm, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
                cudaStream_t s);
 
+int forest_stats(const ForestWs& w, int32_t* out, int cap);
+
 int tridiag_run(int64_t N, const int32_t* forest, const int32_t* iperm, const int32_t* pi2,
                 const float* pi2_val, const float* diag, float* a, float* b, float* c,
                 cudaStream_t s);

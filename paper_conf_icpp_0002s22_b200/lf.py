@@ -22,6 +22,7 @@ EXPORTS = (
     "lf_linear_forest_workspace_size", "lf_linear_forest", "lf_tridiag",
     "lf_pipeline_workspace_size", "lf_pipeline_host", "lf_validate_csr",
     "lf_last_error", "lf_version", "lf_profile_enable", "lf_profile_collect",
+    "lf_forest_stats",
 )
 
 
@@ -63,6 +64,7 @@ def load(path: str = LIB_PATH):
     L.lf_pipeline_workspace_size.restype = C.c_size_t
     L.lf_pipeline_host.argtypes = [P, P, P, P, P, P, P, P, P, C.c_size_t, P]
     L.lf_validate_csr.argtypes = [P, P, C.c_size_t, P]
+    L.lf_forest_stats.argtypes = [I64, P, C.c_size_t, P, I32]
     L.lf_profile_enable.argtypes = [I32]
     L.lf_profile_collect.argtypes = [P, I32, P, I32]
     L.lf_last_error.restype = C.c_char_p
@@ -268,3 +270,18 @@ def profile_collect(cap: int = 4096):
         nm = names.raw[i * stride:(i + 1) * stride].split(b"\0", 1)[0].decode()
         out.append((nm, float(ms[i])))
     return out
+
+
+FOREST_STATS = ("boundary_cycle_pass", "boundary_rank_pass", "reduced_steps_cycle",
+                "reduced_steps_rank", "splitters_cycle_pass", "unvisited", "fallback_tiles",
+                "splitters_rank_pass", "max_node_scan_steps")
+
+
+def forest_stats(N, ws):
+    """Diagnostics of the last linear_forest run that used workspace `ws` (a Workspace)."""
+    import numpy as np
+
+    L = load()
+    out = np.zeros(16, dtype=np.int32)
+    _check(L.lf_forest_stats(N, _ptr(ws.buf), ws.buf.numel(), C.c_void_p(out.ctypes.data), 16))
+    return dict(zip(FOREST_STATS, (int(x) for x in out[:len(FOREST_STATS)])))
