@@ -504,52 +504,62 @@ __global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
     }
 }
 
-// Reduced bidirectional scan over a boundary list (one cooperative kernel).
-//   MIN: min-scan of edge keys; epilogue writes cyc_k (INF unless on a global cycle).
-//   ADD: position scan with weighted hops; epilogue writes end2 / dist2.
+// One step of the reduced bidirectional scan for the list entries t0, t0+stride, ...
+// Nodes are processed in batches of RB so that each thread keeps several independent
+// L2 gathers in flight.  Returns the number of entries not yet done.
+constexpr int RB = 4;
+
 template <bool MIN>
-__global__ void __launch_bounds__(256) k_red_scan(ForestArgs a) {
-    __shared__ int sh[32];
-    cg::grid_group grid = cg::this_grid();
-    const int32_t* list = MIN ? a.list1 : a.list2;
-    const int cnt = *(volatile int*)&a.ctl[MIN ? kCtlCnt1 : kCtlCnt2];
-    int* ctl = a.ctl + (MIN ? kCtlRed1 : kCtlRed2);
-    const int stride = gridDim.x * blockDim.x;
-    const int t0 = blockIdx.x * blockDim.x + threadIdx.x;
-    int step = 0;
-    for (; step < a.max_steps; step++) {
-        const int2* qs = MIN ? a.rq1[step & 1] : a.rq2[step & 1];
-        int2* qd = MIN ? a.rq1[(step & 1) ^ 1] : a.rq2[(step & 1) ^ 1];
-        const ulonglong2* ks = a.rk1[step & 1];
-        ulonglong2* kd = a.rk1[(step & 1) ^ 1];
-        const int2* rs = a.rr2[step & 1];
-        int2* rd = a.rr2[(step & 1) ^ 1];
-        int notdone = 0;
-        for (int idx = t0; idx < cnt; idx += stride) {
-            const int32_t v = list[idx];
-            const int2 q = qs[v];
-            if (q.x < 0 && q.y < 0) {  // final: keep both buffers equal
-                const int2 qo = qd[v];
-                if (qo.x != q.x || qo.y != q.y) {
-                    qd[v] = q;
-                    if (MIN) kd[v] = ks[v]; else rd[v] = rs[v];
+__device__ __forceinline__ int red_step(const ForestArgs& a, const int32_t* __restrict__ list, int cnt,
+                                        int step, int t0, int stride) {
+    const int2* __restrict__ qs = MIN ? a.rq1[step & 1] : a.rq2[step & 1];
+    int2* __restrict__ qd = MIN ? a.rq1[(step & 1) ^ 1] : a.rq2[(step & 1) ^ 1];
+    const ulonglong2* __restrict__ ks = a.rk1[step & 1];
+    ulonglong2* __restrict__ kd = a.rk1[(step & 1) ^ 1];
+    const int2* __restrict__ rs = a.rr2[step & 1];
+    int2* __restrict__ rd = a.rr2[(step & 1) ^ 1];
+    int notdone = 0;
+    for (int base = t0; base < cnt; base += stride * RB) {
+        int32_t v[RB];
+        int2 q[RB];
+#pragma unroll
+        for (int b = 0; b < RB; b++) {
+            const int idx = base + b * stride;
+            v[b] = idx < cnt ? list[idx] : -1;
+        }
+#pragma unroll
+        for (int b = 0; b < RB; b++) q[b] = v[b] >= 0 ? qs[v[b]] : make_int2(-1, -1);
+        int2 qw[RB][2];
+#pragma unroll
+        for (int b = 0; b < RB; b++) {
+            qw[b][0] = q[b].x >= 0 ? qs[q[b].x] : make_int2(0, 0);
+            qw[b][1] = q[b].y >= 0 ? qs[q[b].y] : make_int2(0, 0);
+        }
+#pragma unroll
+        for (int b = 0; b < RB; b++) {
+            if (v[b] < 0) continue;
+            if (q[b].x < 0 && q[b].y < 0) {  // final: keep both buffers equal
+                const int2 qo = qd[v[b]];
+                if (qo.x != q[b].x || qo.y != q[b].y) {
+                    qd[v[b]] = q[b];
+                    if (MIN) kd[v[b]] = ks[v[b]]; else rd[v[b]] = rs[v[b]];
                 }
                 continue;
             }
-            int2 nq = q;
+            int2 nq = q[b];
             ulonglong2 nk = make_ulonglong2(0, 0);
             int2 nr = make_int2(0, 0);
-            if (MIN) nk = ks[v]; else nr = rs[v];
+            if (MIN) nk = ks[v[b]]; else nr = rs[v[b]];
 #pragma unroll
             for (int i = 0; i < 2; i++) {
-                const int32_t w = i ? q.y : q.x;
+                const int32_t w = i ? q[b].y : q[b].x;
                 if (w < 0) continue;
-                const int2 qw = qs[w];
+                const int2 qww = qw[b][i];
                 int j = -1;
-                if (qw.x != v) j = 0;
-                else if (qw.y != v) j = 1;
+                if (qww.x != v[b]) j = 0;
+                else if (qww.y != v[b]) j = 1;
                 if (j < 0) continue;  // stall (reading c13)
-                const int32_t tgt = j ? qw.y : qw.x;
+                const int32_t tgt = j ? qww.y : qww.x;
                 if (i) nq.y = tgt; else nq.x = tgt;
                 if (MIN) {
                     const ulonglong2 kw = ks[w];
@@ -561,13 +571,66 @@ __global__ void __launch_bounds__(256) k_red_scan(ForestArgs a) {
                     if (i) nr.y += dv; else nr.x += dv;
                 }
             }
-            qd[v] = nq;
-            if (MIN) kd[v] = nk; else rd[v] = nr;
+            qd[v[b]] = nq;
+            if (MIN) kd[v[b]] = nk; else rd[v[b]] = nr;
             const bool path_done = nq.x < 0 && nq.y < 0;
             bool cyc_done = false;
             if (MIN) cyc_done = nq.x >= 0 && nq.y >= 0 && (nk.x == nk.y || nq.x == nq.y);
             notdone += (path_done || cyc_done) ? 0 : 1;
         }
+    }
+    return notdone;
+}
+
+template <bool MIN>
+__device__ __forceinline__ void red_epilogue(const ForestArgs& a, const int32_t* list, int cnt, int fb,
+                                             int t0, int stride) {
+    for (int idx = t0; idx < cnt; idx += stride) {
+        const int32_t v = list[idx];
+        if (MIN) {
+            const int2 q = a.rq1[fb][v];
+            const ulonglong2 k = a.rk1[fb][v];
+            a.cyc_k[v] = (q.x >= 0 && q.y >= 0) ? umin64(k.x, k.y) : KEY_INF;
+        } else {
+            const int2 q = a.rq2[fb][v];
+            a.end2[v] = make_int2(-(q.x + 1), -(q.y + 1));
+            a.dist2[v] = a.rr2[fb][v];
+        }
+    }
+}
+
+constexpr int RT = 1024;                    // reduced-scan block size
+constexpr int kRedSmall = RT * RB * 2;      // lists up to this size run in one CTA
+
+// Reduced bidirectional scan over a boundary list (one cooperative kernel).
+//   MIN: min-scan of edge keys; epilogue writes cyc_k (INF unless on a global cycle).
+//   ADD: position scan with weighted hops; epilogue writes end2 / dist2.
+// Small lists run in block 0 alone with block barriers (a grid barrier costs more than
+// the work); large ones use the whole grid with grid barriers.  Both leave as soon as
+// every node is done.
+template <bool MIN>
+__global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
+    __shared__ int sh[32];
+    const int32_t* list = MIN ? a.list1 : a.list2;
+    const int cnt = *(volatile int*)&a.ctl[MIN ? kCtlCnt1 : kCtlCnt2];
+    int* ctl = a.ctl + (MIN ? kCtlRed1 : kCtlRed2);
+    int step = 0;
+    if (cnt <= kRedSmall) {
+        if (blockIdx.x != 0) return;
+        for (; step < a.max_steps; step++) {
+            const int nd = red_step<MIN>(a, list, cnt, step, threadIdx.x, blockDim.x);
+            const int any = __syncthreads_or(nd);
+            if (threadIdx.x == 0 && any) ctl[step] = 1;  // diagnostics: steps taken
+            if (!any) { step++; break; }
+        }
+        red_epilogue<MIN>(a, list, cnt, step & 1, threadIdx.x, blockDim.x);
+        return;
+    }
+    cg::grid_group grid = cg::this_grid();
+    const int stride = gridDim.x * blockDim.x;
+    const int t0 = blockIdx.x * blockDim.x + threadIdx.x;
+    for (; step < a.max_steps; step++) {
+        int notdone = red_step<MIN>(a, list, cnt, step, t0, stride);
         // block reduction of notdone, one atomic per block
 #pragma unroll
         for (int o = 16; o; o >>= 1) notdone += __shfl_xor_sync(0xffffffffu, notdone, o);
@@ -581,20 +644,7 @@ __global__ void __launch_bounds__(256) k_red_scan(ForestArgs a) {
         grid.sync();
         if (*(volatile int*)&ctl[step] == 0) { step++; break; }
     }
-    // results are in the buffer written by the last executed step
-    const int fb = step & 1;
-    for (int idx = t0; idx < cnt; idx += stride) {
-        const int32_t v = list[idx];
-        if (MIN) {
-            const int2 q = a.rq1[fb][v];
-            const ulonglong2 k = a.rk1[fb][v];
-            a.cyc_k[v] = (q.x >= 0 && q.y >= 0) ? umin64(k.x, k.y) : KEY_INF;
-        } else {
-            const int2 q = a.rq2[fb][v];
-            a.end2[v] = make_int2(-(q.x + 1), -(q.y + 1));
-            a.dist2[v] = a.rr2[fb][v];
-        }
-    }
+    red_epilogue<MIN>(a, list, cnt, step & 1, t0, stride);
 }
 
 // Pass 1 expand (break cycles, write the forest) fused with pass 2's local part.
@@ -837,7 +887,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("red_scan_cycles", -1, s);
-        int rc = coop_launch(k_red_scan<true>, 256, a, s);
+        int rc = coop_launch(k_red_scan<true>, RT, a, s);
         if (rc) return rc;
     }
     {
@@ -847,7 +897,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("red_scan_ranks", -1, s);
-        int rc = coop_launch(k_red_scan<false>, 256, a, s);
+        int rc = coop_launch(k_red_scan<false>, RT, a, s);
         if (rc) return rc;
     }
     {
