@@ -600,32 +600,127 @@ __device__ __forceinline__ void red_epilogue(const ForestArgs& a, const int32_t*
 }
 
 constexpr int RT = 1024;                    // reduced-scan block size
-constexpr int kRedSmall = RT * RB * 2;      // lists up to this size run in one CTA
+constexpr int kRedSmall = 4 * RT;           // lists up to this size run in one CTA, in smem
+constexpr int RNPT = kRedSmall / RT;
+
+// smem image of a small reduced graph (pointers are compact node indices or end markers)
+struct RedSmem {
+    int2 q[kRedSmall];
+    ulonglong2 k[kRedSmall];  // MIN: min keys; ADD: distances in .x/.y low words
+};
+
+// The whole reduced scan inside one CTA: load the list's nodes into shared memory with
+// compact indices (cidx maps vertex -> index), run the bidirectional scan there with
+// block barriers, write the results.  Used when the boundary list is small.
+template <bool MIN>
+__device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt, int* ctl, RedSmem& S) {
+    const int tid = threadIdx.x;
+    int32_t* cidx = MIN ? (int32_t*)a.end2 : (int32_t*)a.dist2;  // [N] scratch, unused yet
+    int32_t v[RNPT];
+#pragma unroll
+    for (int k = 0; k < RNPT; k++) {
+        const int idx = tid + k * RT;
+        v[k] = idx < cnt ? list[idx] : -1;
+        if (v[k] >= 0) cidx[v[k]] = idx;
+    }
+    __syncthreads();
+    int2 q[RNPT];
+    ulonglong2 kk[RNPT];
+    bool fin[RNPT];
+#pragma unroll
+    for (int k = 0; k < RNPT; k++) {
+        fin[k] = true;
+        if (v[k] < 0) continue;
+        int2 g = MIN ? a.rq1[0][v[k]] : a.rq2[0][v[k]];
+        q[k].x = g.x >= 0 ? cidx[g.x] : g.x;
+        q[k].y = g.y >= 0 ? cidx[g.y] : g.y;
+        if (MIN) kk[k] = a.rk1[0][v[k]];
+        else { const int2 r = a.rr2[0][v[k]]; kk[k] = make_ulonglong2((uint64_t)(uint32_t)r.x, (uint64_t)(uint32_t)r.y); }
+        fin[k] = q[k].x < 0 && q[k].y < 0;
+        S.q[tid + k * RT] = q[k];
+        S.k[tid + k * RT] = kk[k];
+    }
+    int step = 0;
+    int notdone = 0;
+#pragma unroll
+    for (int k = 0; k < RNPT; k++) notdone |= !fin[k];
+    if (__syncthreads_or(notdone)) {
+        for (; step < a.max_steps; step++) {
+            int2 nq[RNPT];
+            ulonglong2 nk[RNPT];
+#pragma unroll
+            for (int k = 0; k < RNPT; k++) {
+                if (fin[k]) continue;
+                const int me = tid + k * RT;
+                nq[k] = q[k];
+                nk[k] = kk[k];
+#pragma unroll
+                for (int i = 0; i < 2; i++) {
+                    const int w = i ? q[k].y : q[k].x;
+                    if (w < 0) continue;
+                    const int2 qw = S.q[w];
+                    int j = -1;
+                    if (qw.x != me) j = 0;
+                    else if (qw.y != me) j = 1;
+                    if (j < 0) continue;  // stall (reading c13)
+                    const int tgt = j ? qw.y : qw.x;
+                    if (i) nq[k].y = tgt; else nq[k].x = tgt;
+                    const ulonglong2 kw = S.k[w];
+                    const uint64_t kv = j ? kw.y : kw.x;
+                    if (MIN) { if (i) nk[k].y = umin64(nk[k].y, kv); else nk[k].x = umin64(nk[k].x, kv); }
+                    else { if (i) nk[k].y += kv; else nk[k].x += kv; }
+                }
+            }
+            __syncthreads();
+            notdone = 0;
+#pragma unroll
+            for (int k = 0; k < RNPT; k++) {
+                if (fin[k]) continue;
+                const int me = tid + k * RT;
+                q[k] = nq[k];
+                kk[k] = nk[k];
+                S.q[me] = q[k];
+                S.k[me] = kk[k];
+                fin[k] = q[k].x < 0 && q[k].y < 0;
+                bool cyc_done = false;
+                if (MIN) cyc_done = q[k].x >= 0 && q[k].y >= 0 && (kk[k].x == kk[k].y || q[k].x == q[k].y);
+                notdone |= !(fin[k] || cyc_done);
+            }
+            const int any = __syncthreads_or(notdone);
+            if (tid == 0) ctl[step] = 1;  // diagnostics: steps taken
+            if (!any) break;
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < RNPT; k++) {
+        if (v[k] < 0) continue;
+        if (MIN) {
+            a.cyc_k[v[k]] = (q[k].x >= 0 && q[k].y >= 0) ? umin64(kk[k].x, kk[k].y) : KEY_INF;
+        } else {
+            a.end2[v[k]] = make_int2(-(q[k].x + 1), -(q[k].y + 1));
+            a.dist2[v[k]] = make_int2((int)kk[k].x, (int)kk[k].y);
+        }
+    }
+}
 
 // Reduced bidirectional scan over a boundary list (one cooperative kernel).
 //   MIN: min-scan of edge keys; epilogue writes cyc_k (INF unless on a global cycle).
 //   ADD: position scan with weighted hops; epilogue writes end2 / dist2.
-// Small lists run in block 0 alone with block barriers (a grid barrier costs more than
-// the work); large ones use the whole grid with grid barriers.  Both leave as soon as
-// every node is done.
+// Small lists run in block 0 alone, in shared memory (a grid barrier costs more than the
+// work); large ones use the whole grid with grid barriers.  Both leave as soon as every
+// node is done.
 template <bool MIN>
 __global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
     __shared__ int sh[32];
+    extern __shared__ __align__(16) unsigned char red_smem[];
     const int32_t* list = MIN ? a.list1 : a.list2;
     const int cnt = *(volatile int*)&a.ctl[MIN ? kCtlCnt1 : kCtlCnt2];
     int* ctl = a.ctl + (MIN ? kCtlRed1 : kCtlRed2);
-    int step = 0;
     if (cnt <= kRedSmall) {
-        if (blockIdx.x != 0) return;
-        for (; step < a.max_steps; step++) {
-            const int nd = red_step<MIN>(a, list, cnt, step, threadIdx.x, blockDim.x);
-            const int any = __syncthreads_or(nd);
-            if (threadIdx.x == 0 && any) ctl[step] = 1;  // diagnostics: steps taken
-            if (!any) { step++; break; }
-        }
-        red_epilogue<MIN>(a, list, cnt, step & 1, threadIdx.x, blockDim.x);
+        if (blockIdx.x == 0) red_scan_small<MIN>(a, list, cnt, ctl, *reinterpret_cast<RedSmem*>(red_smem));
         return;
     }
+    int step = 0;
     cg::grid_group grid = cg::this_grid();
     const int stride = gridDim.x * blockDim.x;
     const int t0 = blockIdx.x * blockDim.x + threadIdx.x;
@@ -830,10 +925,10 @@ static int max_steps_for(int64_t N) {
 }
 
 template <class K>
-static int coop_launch(K kernel, int block, ForestArgs& a, cudaStream_t s) {
-    const int grid = persistent_grid((const void*)kernel, block);
+static int coop_launch(K kernel, int block, ForestArgs& a, cudaStream_t s, size_t smem = 0) {
+    const int grid = persistent_grid((const void*)kernel, block, smem);
     void* args[] = {&a};
-    LF_CUDA(cudaLaunchCooperativeKernel((const void*)kernel, grid, block, args, 0, s));
+    LF_CUDA(cudaLaunchCooperativeKernel((const void*)kernel, grid, block, args, smem, s));
     return LF_OK;
 }
 
@@ -850,6 +945,10 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local1, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
         LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local2, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
         LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local3, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sizeof(RedSmem)));
+        LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sizeof(RedSmem)));
         attr_done = true;
     }
     LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
@@ -887,7 +986,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("red_scan_cycles", -1, s);
-        int rc = coop_launch(k_red_scan<true>, RT, a, s);
+        int rc = coop_launch(k_red_scan<true>, RT, a, s, sizeof(RedSmem));
         if (rc) return rc;
     }
     {
@@ -897,7 +996,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("red_scan_ranks", -1, s);
-        int rc = coop_launch(k_red_scan<false>, RT, a, s);
+        int rc = coop_launch(k_red_scan<false>, RT, a, s, sizeof(RedSmem));
         if (rc) return rc;
     }
     {
