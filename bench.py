@@ -125,14 +125,16 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
         Na = live_rows[k]
         nxt = live_rows[k + 1] if k + 1 < len(live_rows) else 0
         return 4 * Na + 8 * n * Na + 8 * n * Na + Na + 4 * nxt
-    if base == "cycle_scan":
-        return 16 * N + 8 * N  # read pi2 + pi2_w, write forest
-    if base == "rank_scan":
-        return 8 * N + 12 * N  # read forest, write path_id, pos, len
-    if base == "path_offsets":
-        return 8 * N
+    # linear forest: B_LF = 40N attributed to the kernel that moves it;
+    # block-local intermediates (loc1/loc2, boundary records) are implementation traffic
+    if base == "lf_local1":
+        return 16 * N  # read pi2 + pi2_w
+    if base == "lf_local2":
+        return 8 * N  # write forest
+    if base == "lf_local3":
+        return 8 * N  # write path_id, pos
     if base == "perm":
-        return 12 * N + 8 * N
+        return 8 * N  # write perm, iperm
     if base == "tridiag":
         return 8 * N + 4 * N + 8 * N + 8 * N + 4 * N + 12 * N
     return 0
@@ -219,32 +221,37 @@ def main():
         P.run()
     torch.cuda.synchronize()
 
-    graph = None
+    def capture(prof):
+        lf.profile_enable(prof)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            P.run()
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        return g
+
+    graph = graph_prof = None
     if not args.no_graph:
         try:
-            lf.profile_enable(True)
             s = torch.cuda.Stream()
             s.wait_stream(stream)
             with torch.cuda.stream(s):
-                P.run()  # warm the stream once before capture
+                P.run()  # warm a side stream once before capture
             torch.cuda.synchronize()
-            lf.profile_enable(True)
-            graph = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(graph):
-                P.run()
-            torch.cuda.synchronize()
-            graph.replay()
-            torch.cuda.synchronize()
+            graph = capture(False)       # the timed step: no instrumentation
+            graph_prof = capture(True)   # same launches + event records per kernel
+            lf.profile_enable(False)
         except Exception as e:  # capture unsupported -> eager launches
             print(f"# graph capture failed ({e}); timing eager launches", file=sys.stderr)
-            graph = None
+            graph = graph_prof = None
     launches_per_step = None
 
-    def step():
+    def step(prof=False):
         if graph is not None:
-            graph.replay()
+            (graph_prof if prof else graph).replay()
         else:
-            lf.profile_enable(True)
+            lf.profile_enable(prof)
             P.run()
 
     # keep the GPU busy until the clock sampler is producing samples (bounded)
@@ -256,9 +263,10 @@ def main():
     if ws > 1:
         torch.distributed.barrier()
     torch.cuda.synchronize()
-    step_ms, kern = [], {}
+    step_ms, prof_step_ms, kern = [], [], {}
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
+    # timed region: K steps of the plain graph (L2 flushed before each)
     for _ in range(args.steps):
         flush.zero_()  # write 512 MB > 126 MB L2 between steps
         ev0.record(stream)
@@ -266,6 +274,14 @@ def main():
         ev1.record(stream)
         ev1.synchronize()
         step_ms.append(ev0.elapsed_time(ev1))
+    # per-kernel breakdown: K steps of the instrumented graph, same conditions
+    for _ in range(args.steps):
+        flush.zero_()
+        ev0.record(stream)
+        step(prof=True)
+        ev1.record(stream)
+        ev1.synchronize()
+        prof_step_ms.append(ev0.elapsed_time(ev1))
         recs = lf.profile_collect()
         launches_per_step = len(recs)
         for nm, ms in recs:
@@ -291,8 +307,9 @@ def main():
     M = P.M
     lr, ln = [int(x) for x in live[:M]], [int(x) for x in live[M:2 * M]]
     kavg = {nm: sum(v) / len(v) for nm, v in kern.items()}
-    stage = {"factor": sum(t for nm, t in kavg.items() if nm.split("[")[0] in ("propose", "mutual", "rounds", "init_state")),
-             "linear_forest": sum(t for nm, t in kavg.items() if nm.split("[")[0] in ("cycle_scan", "rank_scan", "path_offsets", "perm")),
+    FACTOR_K = ("propose", "mutual", "rounds", "init_state", "diag", "rounds_fused")
+    stage = {"factor": sum(t for nm, t in kavg.items() if nm.split("[")[0] in FACTOR_K),
+             "linear_forest": sum(t for nm, t in kavg.items() if nm.split("[")[0] not in FACTOR_K + ("tridiag",)),
              "tridiag": kavg.get("tridiag", 0.0)}
     dom = max(kavg, key=kavg.get) if kavg else None
     peak, peak_kind = load_peaks()
@@ -351,6 +368,7 @@ def main():
                 "graph": graph is not None,
             },
             "stages_ms": {k: round(v, 4) for k, v in stage.items()},
+            "instrumented_ms_per_step": round(sum(prof_step_ms) / len(prof_step_ms), 4),
             "t_main_ms": round(t_main, 4),
             "B_main_bytes": int(b_main),
             "B_tri_bytes": int(b_tri),
