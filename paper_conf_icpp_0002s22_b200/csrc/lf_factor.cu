@@ -144,6 +144,116 @@ __global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
     }
 }
 
+// Round 0 (every row proposes; Alg. 2 L14-L22 at k = 0) as a tiled streaming kernel: a
+// CTA takes PT/G consecutive rows, stages their col/val range into shared memory with
+// coalesced 16-byte loads, and scans each row from shared memory with G lanes (G = 1:
+// thread per row).  A tile whose entry span exceeds ETILE (a hub row) is scanned from
+// global memory instead.  Same per-row semantics and outputs as k_propose.
+constexpr int PT = 256;
+constexpr int ETILE = 4096;
+
+template <int NN, int G>
+__global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
+    constexpr int R = PT / G;
+    __shared__ __align__(16) int32_t scol[ETILE];
+    __shared__ __align__(16) float sval[ETILE];
+    __shared__ int64_t srp[R + 1];
+    const int tid = threadIdx.x;
+    const int64_t r0 = (int64_t)blockIdx.x * R;
+    for (int i = tid; i <= R; i += PT) {
+        const int64_t r = r0 + i < a.N ? r0 + i : a.N;
+        srp[i] = __ldg(a.rowptr + r);
+    }
+    __syncthreads();
+    const int64_t e0 = srp[0], e1 = srp[R];
+    const int64_t a0 = e0 & ~(int64_t)3;
+    const bool staged = (e1 - a0) <= ETILE;
+    if (staged) {
+        const int64_t v1 = e1 & ~(int64_t)3;
+        const int nvec = (int)((v1 - a0) >> 2);
+        const int4* c4 = reinterpret_cast<const int4*>(a.col + a0);
+        const float4* f4 = reinterpret_cast<const float4*>(a.val + a0);
+        for (int i = tid; i < nvec; i += PT) {
+            reinterpret_cast<int4*>(scol)[i] = __ldg(c4 + i);
+            reinterpret_cast<float4*>(sval)[i] = __ldg(f4 + i);
+        }
+        for (int64_t e = v1 + tid; e < e1; e += PT) {
+            scol[e - a0] = __ldg(a.col + e);
+            sval[e - a0] = __ldg(a.val + e);
+        }
+    }
+    __syncthreads();
+    const int lr = tid / G, li = tid % G;
+    const int64_t row = r0 + lr;
+    const bool valid = row < a.N;
+    const int32_t v = (int32_t)row;
+    const int64_t rs = srp[lr], re = valid ? srp[lr + 1] : rs;
+    uint32_t cv = 0;
+    if (valid && a.state) cv = (a.state[v] & ST_CHARGE) ? 1u : 0u;
+    uint64_t top[NN];
+#pragma unroll
+    for (int s = 0; s < NN; s++) top[s] = 0;
+    uint32_t theta0 = 0, dbits = 0;
+    for (int64_t e = rs + li; e < re; e += G) {
+        int32_t j;
+        float x;
+        if (staged) { j = scol[e - a0]; x = sval[e - a0]; }
+        else { j = __ldg(a.col + e); x = __ldg(a.val + e); }
+        if (j == v) { dbits = __float_as_uint(x); continue; }          // diagonal (L231)
+        if ((__float_as_uint(x) & 0x7FFFFFFFu) == 0u) continue;       // zero (L31)
+        theta0 = 1;                      // round 0: nothing saturated, nothing confirmed
+        if (a.charging && ((((a.state[j] & ST_CHARGE) ? 1u : 0u)) == cv)) continue;  // L17
+        topn_insert<NN>(top, make_key(x, j));
+    }
+    if (G > 1) {
+        topn_merge_group<NN, G>(top);
+#pragma unroll
+        for (int off = G / 2; off >= 1; off >>= 1) {
+            theta0 |= __shfl_xor_sync(0xffffffffu, theta0, off);
+            dbits |= __shfl_xor_sync(0xffffffffu, dbits, off);
+        }
+    }
+    unsigned long long my_live = 0, my_nnz = 0;
+    int my_prop = 0;
+    if (valid && li == 0) {
+        int32_t pj[NN];
+        float pv[NN];
+        int np = 0;
+#pragma unroll
+        for (int s = 0; s < NN; s++) {
+            if (top[s] != 0) { pj[s] = key_col(top[s]); pv[s] = key_val(top[s]); np++; }
+            else { pj[s] = (s == 0 && !theta0) ? PROP_RETIRED : -1; pv[s] = 0.0f; }
+        }
+        if (NN == 2) {
+            reinterpret_cast<int2*>(a.prop_j)[v] = make_int2(pj[0], pj[1]);
+            reinterpret_cast<float2*>(a.prop_v)[v] = make_float2(pv[0], pv[1]);
+        } else if (NN == 4) {
+            reinterpret_cast<int4*>(a.prop_j)[v] = make_int4(pj[0], pj[NN > 1 ? 1 : 0], pj[NN > 2 ? 2 : 0], pj[NN > 3 ? 3 : 0]);
+            reinterpret_cast<float4*>(a.prop_v)[v] = make_float4(pv[0], pv[NN > 1 ? 1 : 0], pv[NN > 2 ? 2 : 0], pv[NN > 3 ? 3 : 0]);
+        } else {
+#pragma unroll
+            for (int s = 0; s < NN; s++) {
+                a.prop_j[(int64_t)v * NN + s] = pj[s];
+                a.prop_v[(int64_t)v * NN + s] = pv[s];
+            }
+        }
+        if (a.diag) a.diag[v] = __uint_as_float(dbits);
+        if (theta0) { my_live = 1; my_nnz = (unsigned long long)(re - rs); }
+        my_prop = np > 0;
+    }
+#pragma unroll
+    for (int off = 16; off >= 1; off >>= 1) {
+        my_live += __shfl_xor_sync(0xffffffffu, my_live, off);
+        my_nnz += __shfl_xor_sync(0xffffffffu, my_nnz, off);
+        my_prop |= __shfl_xor_sync(0xffffffffu, my_prop, off);
+    }
+    if ((tid & 31) == 0) {
+        if (a.live_rows && my_live) atomicAdd(a.live_rows, my_live);
+        if (a.live_nnz && my_nnz) atomicAdd(a.live_nnz, my_nnz);
+        if (my_prop) atomicOr(a.proposed, 1);
+    }
+}
+
 struct MutualArgs {
     int64_t N;
     const int32_t* __restrict__ wl;  // NULL = all rows (round 0)
@@ -302,6 +412,26 @@ static void launch_propose(int G, const ProposeArgs& pa, int grid, cudaStream_t 
     }
 }
 
+template <int NN>
+static void launch_propose_tile(int G, const ProposeArgs& pa, int64_t N, cudaStream_t s) {
+    const int R = PT / G;
+    const int grid = (int)((N + R - 1) / R);
+    switch (G) {
+        case 1: k_propose_tile<NN, 1><<<grid, PT, 0, s>>>(pa); break;
+        case 2: k_propose_tile<NN, 2><<<grid, PT, 0, s>>>(pa); break;
+        case 4: k_propose_tile<NN, 4><<<grid, PT, 0, s>>>(pa); break;
+        default: k_propose_tile<NN, 8><<<grid, PT, 0, s>>>(pa); break;
+    }
+}
+
+// lanes per row of the staged round-0 kernel (thread per row for sparse rows)
+static int tile_lanes(double avg) {
+    if (avg <= 12) return 1;
+    if (avg <= 24) return 2;
+    if (avg <= 48) return 4;
+    return 8;
+}
+
 static int lanes_per_row(double avg) {
     // enough lanes to cover an average row in one or two passes
     if (avg <= 3) return 2;
@@ -374,7 +504,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_CUDA(cudaMemsetAsync(pa.proposed, 0, sizeof(int), s));
         {
             LF_PROF("propose", k, s);
-            launch_propose<NN>(G, pa, grid_p, s);
+            if (fresh) launch_propose_tile<NN>(tile_lanes(N > 0 ? (double)A->nnz / (double)N : 1.0), pa, N, s);
+            else launch_propose<NN>(G, pa, grid_p, s);
             LF_CUDA(cudaGetLastError());
         }
 
