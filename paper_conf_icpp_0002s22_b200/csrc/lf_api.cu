@@ -109,6 +109,8 @@ size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w) {
     t.wl[1] = c.take<int32_t>(nn);
     t.counts = c.take<int32_t>(4);
     t.flags = c.take<int>(kMaxFlagRounds);
+    t.long_rows = c.take<int32_t>(nn);
+    t.long_count = c.take<int32_t>(kMaxFlagRounds);
     if (w) *w = t;
     return c.off;
 }
@@ -161,7 +163,7 @@ const char* lf_last_error(void) { return g_err; }
 int lf_profile_enable(int on) {
     std::lock_guard<std::mutex> lk(g_prof_mu);
     g_prof = on != 0;
-    g_recs.clear();
+    if (g_prof) g_recs.clear();  // turning off keeps the records for lf_profile_collect
     return LF_OK;
 }
 

@@ -37,7 +37,21 @@ struct ProposeArgs {
     unsigned long long* live_rows;       // NULL or &live[k]
     unsigned long long* live_nnz;        // NULL or &live[M+k]
     int* proposed;                       // &flags[k]: set to 1 if anything was proposed
+    int64_t defer_len;                   // rows with more entries go to the long-row list
+    int32_t* defer_list;                 // long rows of this round (processed warp-per-row)
+    int32_t* defer_count;
 };
+
+// append the rows flagged by lanes of this warp to the long-row list
+__device__ __forceinline__ void defer_append(const ProposeArgs& a, bool take, int32_t v) {
+    const unsigned m = __ballot_sync(0xffffffffu, take);
+    if (!m) return;
+    const int lane = threadIdx.x & 31;
+    int base = 0;
+    if (lane == 0) base = atomicAdd(a.defer_count, __popc(m));
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (take) a.defer_list[base + __popc(m & ((1u << lane) - 1u))] = v;
+}
 
 // G lanes per row (G = 1..32), NN = n.  Persistent grid-stride over the worklist.
 template <int NN, int G>
@@ -76,6 +90,9 @@ __global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
             rs = __ldg(a.rowptr + v);
             re = __ldg(a.rowptr + v + 1);
         }
+        const bool deferred = valid && (re - rs) > a.defer_len;
+        defer_append(a, deferred && li == 0, v);
+        if (deferred) re = rs;
         uint64_t top[NN];
 #pragma unroll
         for (int s = 0; s < NN; s++) top[s] = 0;
@@ -107,7 +124,7 @@ __global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
             theta0 |= __shfl_xor_sync(0xffffffffu, theta0, off);
             dbits |= __shfl_xor_sync(0xffffffffu, dbits, off);
         }
-        if (valid && li == 0) {
+        if (valid && !deferred && li == 0) {
             const int need = NN - deg;
             int32_t* pj = a.prop_j + (int64_t)v * NN;
             float* pv = a.prop_v + (int64_t)v * NN;
@@ -187,7 +204,11 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
     const int64_t row = r0 + lr;
     const bool valid = row < a.N;
     const int32_t v = (int32_t)row;
-    const int64_t rs = srp[lr], re = valid ? srp[lr + 1] : rs;
+    const int64_t rs = srp[lr];
+    int64_t re = valid ? srp[lr + 1] : rs;
+    const bool deferred = valid && (re - rs) > a.defer_len;
+    defer_append(a, deferred && li == 0, v);
+    if (deferred) re = rs;
     uint32_t cv = 0;
     if (valid && a.state) cv = (a.state[v] & ST_CHARGE) ? 1u : 0u;
     uint64_t top[NN];
@@ -215,7 +236,7 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
     }
     unsigned long long my_live = 0, my_nnz = 0;
     int my_prop = 0;
-    if (valid && li == 0) {
+    if (valid && !deferred && li == 0) {
         int32_t pj[NN];
         float pv[NN];
         int np = 0;
@@ -455,6 +476,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
     const int grid_m = persistent_grid((const void*)k_mutual<NN>, 256);
 
     LF_CUDA(cudaMemsetAsync(w.flags, 0, sizeof(int) * kMaxFlagRounds, s));
+    LF_CUDA(cudaMemsetAsync(w.long_count, 0, sizeof(int32_t) * kMaxFlagRounds, s));
     LF_CUDA(cudaMemsetAsync(w.counts, 0, sizeof(int32_t) * 4, s));
     if (live && !o->until_maximal && o->M > 0)
         LF_CUDA(cudaMemsetAsync(live, 0, sizeof(int64_t) * 2 * o->M, s));
@@ -500,12 +522,32 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         pa.live_rows = rec ? (unsigned long long*)&live[k] : nullptr;
         pa.live_nnz = rec ? (unsigned long long*)&live[o->M + k] : nullptr;
         pa.proposed = &w.flags[k % kMaxFlagRounds];
-        if (o->until_maximal && k >= kMaxFlagRounds)
+        pa.defer_list = w.long_rows;
+        pa.defer_count = &w.long_count[k % kMaxFlagRounds];
+        if (o->until_maximal && k >= kMaxFlagRounds) {
             LF_CUDA(cudaMemsetAsync(pa.proposed, 0, sizeof(int), s));
+            LF_CUDA(cudaMemsetAsync(pa.defer_count, 0, sizeof(int32_t), s));
+        }
         {
             LF_PROF("propose", k, s);
-            if (fresh) launch_propose_tile<NN>(tile_lanes(N > 0 ? (double)A->nnz / (double)N : 1.0), pa, N, s);
-            else launch_propose<NN>(G, pa, grid_p, s);
+            if (fresh) {
+                const int Gt = tile_lanes(N > 0 ? (double)A->nnz / (double)N : 1.0);
+                pa.defer_len = 32 * Gt;
+                launch_propose_tile<NN>(Gt, pa, N, s);
+            } else {
+                pa.defer_len = 32 * G;
+                launch_propose<NN>(G, pa, grid_p, s);
+            }
+            LF_CUDA(cudaGetLastError());
+        }
+        {
+            // long rows of this round: one warp per row
+            LF_PROF("propose_long", k, s);
+            ProposeArgs pl = pa;
+            pl.wl = w.long_rows;
+            pl.wl_count = pa.defer_count;
+            pl.defer_len = INT64_MAX;
+            k_propose<NN, 32><<<grid_p, 256, 0, s>>>(pl);
             LF_CUDA(cudaGetLastError());
         }
 

@@ -59,6 +59,8 @@ struct FactorWs {
     int32_t* wl[2];     // [N] each
     int32_t* counts;    // [4]
     int* flags;         // [kMaxFlagRounds]
+    int32_t* long_rows; // [N] rows deferred to the warp-per-row pass of a round
+    int32_t* long_count;// [kMaxFlagRounds]
 };
 size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w);
 
