@@ -125,6 +125,10 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
         Na = live_rows[k]
         nxt = live_rows[k + 1] if k + 1 < len(live_rows) else 0
         return 4 * Na + 8 * n * Na + 8 * n * Na + Na + 4 * nxt
+    if base == "rounds_fused":  # rounds 1..M-1: live rows' propose + mutual traffic
+        return sum(kernel_bytes(f"propose[{kk}]", N, Z, n, live_rows, live_nnz)
+                   + kernel_bytes(f"mutual[{kk}]", N, Z, n, live_rows, live_nnz)
+                   for kk in range(1, len(live_rows)))
     # linear forest: B_LF = 40N attributed to the kernel that moves it;
     # block-local intermediates (loc1/loc2, boundary records) are implementation traffic
     if base == "lf_local1":
@@ -307,7 +311,8 @@ def main():
     M = P.M
     lr, ln = [int(x) for x in live[:M]], [int(x) for x in live[M:2 * M]]
     kavg = {nm: sum(v) / len(v) for nm, v in kern.items()}
-    FACTOR_K = ("propose", "mutual", "rounds", "init_state", "diag", "rounds_fused")
+    FACTOR_K = ("propose", "mutual", "rounds", "init_state", "diag", "rounds_fused", "finalize",
+                "propose_long")
     stage = {"factor": sum(t for nm, t in kavg.items() if nm.split("[")[0] in FACTOR_K),
              "linear_forest": sum(t for nm, t in kavg.items() if nm.split("[")[0] not in FACTOR_K + ("tridiag",)),
              "tridiag": kavg.get("tridiag", 0.0)}

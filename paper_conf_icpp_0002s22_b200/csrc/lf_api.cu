@@ -111,6 +111,7 @@ size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w) {
     t.flags = c.take<int>(kMaxFlagRounds);
     t.long_rows = c.take<int32_t>(nn);
     t.long_count = c.take<int32_t>(kMaxFlagRounds);
+    t.live_part = c.take<unsigned long long>((size_t)kMaxFlagRounds * 128);
     if (w) *w = t;
     return c.off;
 }

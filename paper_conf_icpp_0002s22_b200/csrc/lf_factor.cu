@@ -12,12 +12,17 @@
 //    again, so later rounds only touch live rows.
 //  * no host synchronisation: round count, worklist sizes and the maximality flags
 //    (L23-L25) stay on the device; the launch chain is fixed and graph-capturable.
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
 #include <cstdint>
 
 #include "lf_common.cuh"
 #include "lf_internal.h"
+
+#include <cstring>
+
+namespace cg = cooperative_groups;
 
 namespace lf {
 
@@ -34,8 +39,8 @@ struct ProposeArgs {
     float* __restrict__ prop_v;          // [N*n] their signed values
     float* __restrict__ diag;            // [N] written when non-NULL (round 0)
     int charging;
-    unsigned long long* live_rows;       // NULL or &live[k]
-    unsigned long long* live_nnz;        // NULL or &live[M+k]
+    unsigned long long* live_rows;       // NULL or 64 partial-sum slots of round k
+    unsigned long long* live_nnz;        // NULL or 64 partial-sum slots of round k
     int* proposed;                       // &flags[k]: set to 1 if anything was proposed
     int64_t defer_len;                   // rows with more entries go to the long-row list
     int32_t* defer_list;                 // long rows of this round (processed warp-per-row)
@@ -55,7 +60,7 @@ __device__ __forceinline__ void defer_append(const ProposeArgs& a, bool take, in
 
 // G lanes per row (G = 1..32), NN = n.  Persistent grid-stride over the worklist.
 template <int NN, int G>
-__global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
+__device__ __forceinline__ void propose_phase(const ProposeArgs& a) {
     constexpr int RPW = 32 / G;  // rows per warp per iteration
     const int lane = threadIdx.x & 31;
     const int li = lane & (G - 1);
@@ -155,10 +160,16 @@ __global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
         my_prop |= __shfl_xor_sync(0xffffffffu, my_prop, off);
     }
     if (lane == 0) {
-        if (a.live_rows && my_live) atomicAdd(a.live_rows, my_live);
-        if (a.live_nnz && my_nnz) atomicAdd(a.live_nnz, my_nnz);
-        if (my_prop) atomicOr(a.proposed, 1);
+        const int slot = (int)(warp_global & 63);
+        if (a.live_rows && my_live) atomicAdd(a.live_rows + slot, my_live);
+        if (a.live_nnz && my_nnz) atomicAdd(a.live_nnz + slot, my_nnz);
+        if (my_prop && *(volatile int*)a.proposed == 0) atomicOr(a.proposed, 1);
     }
+}
+
+template <int NN, int G>
+__global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
+    propose_phase<NN, G>(a);
 }
 
 // Round 0 (every row proposes; Alg. 2 L14-L22 at k = 0) as a tiled streaming kernel: a
@@ -268,10 +279,21 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
         my_nnz += __shfl_xor_sync(0xffffffffu, my_nnz, off);
         my_prop |= __shfl_xor_sync(0xffffffffu, my_prop, off);
     }
+    __shared__ unsigned long long red[3][PT / 32];
     if ((tid & 31) == 0) {
-        if (a.live_rows && my_live) atomicAdd(a.live_rows, my_live);
-        if (a.live_nnz && my_nnz) atomicAdd(a.live_nnz, my_nnz);
-        if (my_prop) atomicOr(a.proposed, 1);
+        red[0][tid >> 5] = my_live;
+        red[1][tid >> 5] = my_nnz;
+        red[2][tid >> 5] = (unsigned long long)my_prop;
+    }
+    __syncthreads();
+    if (tid == 0) {
+        unsigned long long l = 0, z = 0, pr = 0;
+#pragma unroll
+        for (int w = 0; w < PT / 32; w++) { l += red[0][w]; z += red[1][w]; pr |= red[2][w]; }
+        // counters spread over 64 slots (one L2 atomic per CTA), summed by k_finalize
+        if (a.live_rows && l) atomicAdd(a.live_rows + (blockIdx.x & 63), l);
+        if (a.live_nnz && z) atomicAdd(a.live_nnz + (blockIdx.x & 63), z);
+        if (pr && *(volatile int*)a.proposed == 0) atomicOr(a.proposed, 1);
     }
 }
 
@@ -296,7 +318,7 @@ struct MutualArgs {
 };
 
 template <int NN>
-__global__ void __launch_bounds__(256) k_mutual(MutualArgs a) {
+__device__ __forceinline__ void mutual_phase(const MutualArgs& a) {
     const int64_t count = a.wl_count ? (int64_t)*a.wl_count : a.N;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     if (a.wl_zero && blockIdx.x == 0 && threadIdx.x == 0) *a.wl_zero = 0;
@@ -387,6 +409,67 @@ __global__ void __launch_bounds__(256) k_mutual(MutualArgs a) {
     }
 }
 
+template <int NN>
+__global__ void __launch_bounds__(256) k_mutual(MutualArgs a) {
+    mutual_phase<NN>(a);
+}
+
+// Rounds 1..M-1 in one cooperative persistent kernel: after round 0 only the live rows
+// (2-40% of them) remain, and separate launches would be latency-bound.  Per round:
+// propose over the worklist | long rows warp-per-row | mutual, separated by grid barriers.
+struct FusedArgs {
+    ProposeArgs pa;      // round-independent fields (CSR, state, pi, prop, live slots base)
+    MutualArgs ma;
+    int32_t* wl[2];
+    int32_t* counts;     // [3] worklist sizes (ring)
+    int* flags;
+    int32_t* long_rows;
+    int32_t* long_count;
+    unsigned long long* live_part;
+    int M, m, k_m;
+    int G;
+};
+
+template <int NN, int G>
+__global__ void __launch_bounds__(256) k_rounds_fused(FusedArgs f) {
+    cg::grid_group grid = cg::this_grid();
+    for (int k = 1; k < f.M; k++) {
+        ProposeArgs pa = f.pa;
+        pa.wl = f.wl[k & 1];
+        pa.wl_count = &f.counts[k % 3];
+        pa.charging = (k % f.m) != f.k_m;
+        pa.proposed = &f.flags[k];
+        pa.defer_count = &f.long_count[k];
+        pa.defer_len = 32 * G;
+        if (f.live_part) {
+            pa.live_rows = f.live_part + (size_t)k * 128;
+            pa.live_nnz = f.live_part + (size_t)k * 128 + 64;
+        }
+        propose_phase<NN, G>(pa);
+        grid.sync();
+        if (*(volatile int32_t*)pa.defer_count > 0) {
+            ProposeArgs pl = pa;
+            pl.wl = f.long_rows;
+            pl.wl_count = pa.defer_count;
+            pl.defer_len = INT64_MAX;
+            propose_phase<NN, 32>(pl);
+            grid.sync();
+        }
+        MutualArgs ma = f.ma;
+        const bool last = k == f.M - 1;
+        ma.wl = f.wl[k & 1];
+        ma.wl_count = &f.counts[k % 3];
+        ma.wl_next = last ? nullptr : f.wl[(k + 1) & 1];
+        ma.wl_next_count = last ? nullptr : &f.counts[(k + 1) % 3];
+        ma.wl_zero = last ? nullptr : &f.counts[(k + 2) % 3];
+        ma.fresh = 0;
+        ma.next_charging = ((k + 1) % f.m) != f.k_m;
+        ma.next_k = (uint32_t)(k + 1);
+        mutual_phase<NN>(ma);
+        if (!last) grid.sync();
+    }
+}
+
 // state of round 0 when round 0 is charged (k_m != 0): degree 0 + charge(v, 0)
 __global__ void k_init_state(int64_t N, uint8_t* state, uint32_t seed, unsigned long long thr) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N;
@@ -406,15 +489,27 @@ __global__ void k_diag(int64_t N, const int64_t* __restrict__ rowptr, const int3
     }
 }
 
-// Alg. 2 L23-L24 / L30: rounds = k+1 for the first uncharged round without proposals
-__global__ void k_rounds(const int* flags, int M, int m, int k_m, int32_t* rounds) {
-    int r = M;
-    for (int k = 0; k < M; k++)
-        if ((k % m) == k_m && flags[k] == 0) {
-            r = k + 1;
-            break;
+// Alg. 2 L23-L24 / L30: rounds = k+1 for the first uncharged round without proposals;
+// also sums the live-row counter slots into live[k], live[M+k]
+__global__ void k_finalize(const int* flags, int M, int m, int k_m, int32_t* rounds,
+                           const unsigned long long* part, int64_t* live) {
+    if (threadIdx.x == 0 && rounds) {
+        int r = M;
+        for (int k = 0; k < M; k++)
+            if ((k % m) == k_m && flags[k] == 0) {
+                r = k + 1;
+                break;
+            }
+        *rounds = r;
+    }
+    if (live) {
+        for (int i = threadIdx.x; i < 2 * M; i += blockDim.x) {
+            const int k = i % M, which = i / M;
+            unsigned long long t = 0;
+            for (int j = 0; j < 64; j++) t += part[(size_t)k * 128 + which * 64 + j];
+            live[i] = (int64_t)t;
         }
-    *rounds = r;
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -479,7 +574,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
     LF_CUDA(cudaMemsetAsync(w.long_count, 0, sizeof(int32_t) * kMaxFlagRounds, s));
     LF_CUDA(cudaMemsetAsync(w.counts, 0, sizeof(int32_t) * 4, s));
     if (live && !o->until_maximal && o->M > 0)
-        LF_CUDA(cudaMemsetAsync(live, 0, sizeof(int64_t) * 2 * o->M, s));
+        LF_CUDA(cudaMemsetAsync(w.live_part, 0, sizeof(unsigned long long) * 128 * o->M, s));
     if (N == 0 || (!o->until_maximal && o->M == 0)) {
         // no rounds: empty factor
         if (N > 0) {
@@ -502,7 +597,10 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         LF_CUDA(cudaGetLastError());
     }
     int rounds_host = -1;
-    for (int k = 0; k < M; k++) {
+    // rounds 1..M-1 in one cooperative kernel unless the host must check maximality
+    const bool fuse = !o->until_maximal && o->M > 1;
+    const int M_loop = fuse ? 1 : M;
+    for (int k = 0; k < M_loop; k++) {
         const bool charging = (k % o->m) != o->k_m;
         const bool fresh = (k == 0);
         ProposeArgs pa;
@@ -519,8 +617,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         pa.diag = fresh ? diag : nullptr;
         pa.charging = charging ? 1 : 0;
         const bool rec = live && !o->until_maximal;
-        pa.live_rows = rec ? (unsigned long long*)&live[k] : nullptr;
-        pa.live_nnz = rec ? (unsigned long long*)&live[o->M + k] : nullptr;
+        pa.live_rows = rec ? w.live_part + (size_t)k * 128 : nullptr;
+        pa.live_nnz = rec ? w.live_part + (size_t)k * 128 + 64 : nullptr;
         pa.proposed = &w.flags[k % kMaxFlagRounds];
         pa.defer_list = w.long_rows;
         pa.defer_count = &w.long_count[k % kMaxFlagRounds];
@@ -571,6 +669,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         }
         const bool last = !o->until_maximal && (k == M - 1);
         MutualArgs ma;
+        ma.wl_zero = nullptr;
         ma.N = N;
         ma.wl = fresh ? nullptr : w.wl[k & 1];
         ma.wl_count = fresh ? nullptr : &w.counts[k % 3];
@@ -594,16 +693,63 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_CUDA(cudaGetLastError());
         }
     }
-    if (rounds_dev) {
-        if (o->until_maximal) {
+    if (fuse) {
+        FusedArgs f;
+        memset(&f, 0, sizeof(f));
+        ProposeArgs& pa = f.pa;
+        pa.N = N;
+        pa.rowptr = A->rowptr;
+        pa.col = A->col;
+        pa.val = A->val;
+        pa.state = w.state;
+        pa.pi = pi;
+        pa.prop_j = w.prop_j;
+        pa.prop_v = w.prop_v;
+        pa.diag = nullptr;
+        pa.defer_list = w.long_rows;
+        MutualArgs& ma = f.ma;
+        ma.N = N;
+        ma.prop_j = w.prop_j;
+        ma.prop_v = w.prop_v;
+        ma.state = w.state;
+        ma.pi = pi;
+        ma.pi_w = pi_w;
+        ma.pi_val = pi_val;
+        ma.seed = o->seed;
+        ma.thr = thr;
+        f.wl[0] = w.wl[0];
+        f.wl[1] = w.wl[1];
+        f.counts = w.counts;
+        f.flags = w.flags;
+        f.long_rows = w.long_rows;
+        f.long_count = w.long_count;
+        f.live_part = (live && !o->until_maximal) ? w.live_part : nullptr;
+        f.M = o->M;
+        f.m = o->m;
+        f.k_m = o->k_m;
+        f.G = G;
+        LF_PROF("rounds_fused", -1, s);
+        void* args[] = {&f};
+        const void* kfn;
+        switch (G) {
+            case 2: kfn = (const void*)k_rounds_fused<NN, 2>; break;
+            case 4: kfn = (const void*)k_rounds_fused<NN, 4>; break;
+            case 8: kfn = (const void*)k_rounds_fused<NN, 8>; break;
+            case 16: kfn = (const void*)k_rounds_fused<NN, 16>; break;
+            default: kfn = (const void*)k_rounds_fused<NN, 32>; break;
+        }
+        const int grid = persistent_grid(kfn, 256);
+        LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, 256, args, 0, s));
+    }
+    if (o->until_maximal) {
+        if (rounds_dev) {
             LF_CUDA(cudaMemcpyAsync(rounds_dev, &rounds_host, sizeof(int32_t), cudaMemcpyHostToDevice, s));
             LF_CUDA(cudaStreamSynchronize(s));
-        } else {
-            if (o->M > kMaxFlagRounds) return set_error(LF_EINVAL, "M > 1024 needs until_maximal");
-            LF_PROF("rounds", -1, s);
-            k_rounds<<<1, 1, 0, s>>>(w.flags, o->M, o->m, o->k_m, rounds_dev);
-            LF_CUDA(cudaGetLastError());
         }
+    } else if (rounds_dev || live) {
+        LF_PROF("finalize", -1, s);
+        k_finalize<<<1, 32, 0, s>>>(w.flags, o->M, o->m, o->k_m, rounds_dev, w.live_part, live);
+        LF_CUDA(cudaGetLastError());
     }
     return LF_OK;
 }

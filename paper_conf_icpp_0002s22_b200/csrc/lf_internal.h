@@ -61,6 +61,7 @@ struct FactorWs {
     int* flags;         // [kMaxFlagRounds]
     int32_t* long_rows; // [N] rows deferred to the warp-per-row pass of a round
     int32_t* long_count;// [kMaxFlagRounds]
+    unsigned long long* live_part;  // [kMaxFlagRounds][2][64] live-row counter slots
 };
 size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w);
 
