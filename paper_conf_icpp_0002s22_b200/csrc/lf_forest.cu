@@ -52,6 +52,24 @@ constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
 
 __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
 
+// optional per-phase cycle accounting of the tile kernels (build with -DLF_PHASE_TIMING;
+// accumulated into ctl[208 + phase], read with lf_forest_stats' extended slots)
+#ifdef LF_PHASE_TIMING
+#define LF_PHASE(ctl, i)                                                              \
+    do {                                                                              \
+        __syncthreads();                                                              \
+        if (threadIdx.x == 0) {                                                       \
+            const long long t_ = clock64();                                           \
+            atomicAdd((unsigned long long*)&(ctl)[208 + 2 * (i)], (unsigned long long)(t_ - ph_t)); \
+            ph_t = t_;                                                                \
+        }                                                                             \
+    } while (0)
+#define LF_PHASE_INIT long long ph_t = clock64()
+#else
+#define LF_PHASE(ctl, i) do { } while (0)
+#define LF_PHASE_INIT do { } while (0)
+#endif
+
 // Global key of edge {v,w} for the weakest-edge search, minimised: (|w| bits, -rank), rank
 // = 2*min + c orders edges by (min, max) lexicographically (c = 1 iff max is the larger of
 // min's two higher neighbours).  Realises reading c9 (ties -> larger (min,max) is weaker).
@@ -193,6 +211,7 @@ template <bool MINK>
 __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
                           int2 (&R)[VPT], ulonglong2 (&K)[VPT], int* stats) {
     const int tid = threadIdx.x;
+    LF_PHASE_INIT;
     if (tid == 0) s.nspl = 0;
     __syncthreads();
     // 1. splitters: terminals of the local structure (a slot that is missing or remote) and
@@ -210,7 +229,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         if (sp) s.spl[id] = (short)u;
         s.recS[u] = make_short2(-1, -1);
     }
-    __syncthreads();
+    LF_PHASE(stats - kCtlStat, 3);
     const int C = s.nspl;
     if (tid == 0 && stats) atomicAdd(&stats[MINK ? 0 : 3], C);
     // 2. walks: one per (node, slot), sequential through non-splitters
@@ -250,7 +269,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         if (f) { s.P[i].y = ptr; s.R[i].y = (short)dist; s.K1[i] = km; }
         else { s.P[i].x = ptr; s.R[i].x = (short)dist; s.K0[i] = km; }
     }
-    __syncthreads();
+    LF_PHASE(stats - kCtlStat, 4);
     // 3. bidirectional scan over the splitter nodes (node arrays in s.P/s.R/s.K*)
     for (int step = 0; step < 16; step++) {
         int notdone = 0;
@@ -306,6 +325,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
             break;
         }
     }
+    LF_PHASE(stats - kCtlStat, 5);
     // 4. expand: every vertex from its node (splitter) or its walk records
     bool unvisited[VPT];
     int any_unvisited = 0;
@@ -343,6 +363,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         // a vertex on a cycle: make both pointers non-negative (cycle flag)
         if (P[k].x >= 0 || P[k].y >= 0) { P[k].x = 0; P[k].y = 0; }
     }
+    LF_PHASE(stats - kCtlStat, 6);
     if (MINK) {
         if (stats) {
             int nu = 0;
@@ -365,6 +386,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         }
     }
     __syncthreads();
+    LF_PHASE(stats - kCtlStat, 7);
 }
 
 // the slot of local terminal t (t not the walk's start) that leaves its segment: the
@@ -470,12 +492,16 @@ __global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = blockIdx.x * LB;
+    LF_PHASE_INIT;
     load_tile(a.pi2, s, b0, a.N);
+    LF_PHASE(a.ctl, 0);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
+    LF_PHASE(a.ctl, 1);
     int2 P[VPT], R[VPT];
     ulonglong2 K[VPT];
     tile_rank<true>(s, b0, ek, P, R, K, a.ctl + kCtlStat);
+    LF_PHASE(a.ctl, 2);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -1031,6 +1057,9 @@ int forest_stats(const ForestWs& w, int32_t* out, int cap) {
     int v[9] = {h[kCtlCnt1], h[kCtlCnt2], steps1, steps2, h[kCtlStat], h[kCtlStat + 1], h[kCtlStat + 2],
                 h[kCtlStat + 3], h[kCtlStat + 4]};
     for (int i = 0; i < cap && i < 9; i++) out[i] = v[i];
+    // [16..31]: per-phase cycle sums (units of 1024 cycles; LF_PHASE_TIMING builds only)
+    const unsigned long long* ph = reinterpret_cast<const unsigned long long*>(h + 208);
+    for (int i = 0; i < 16 && 16 + i < cap; i++) out[16 + i] = (int)(ph[i] >> 10);
     return LF_OK;
 }
 

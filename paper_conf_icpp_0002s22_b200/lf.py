@@ -282,6 +282,9 @@ def forest_stats(N, ws):
     import numpy as np
 
     L = load()
-    out = np.zeros(16, dtype=np.int32)
-    _check(L.lf_forest_stats(N, _ptr(ws.buf), ws.buf.numel(), C.c_void_p(out.ctypes.data), 16))
-    return dict(zip(FOREST_STATS, (int(x) for x in out[:len(FOREST_STATS)])))
+    out = np.zeros(32, dtype=np.int32)
+    _check(L.lf_forest_stats(N, _ptr(ws.buf), ws.buf.numel(), C.c_void_p(out.ctypes.data), 32))
+    d = dict(zip(FOREST_STATS, (int(x) for x in out[:len(FOREST_STATS)])))
+    if out[16:].any():  # LF_PHASE_TIMING build: per-phase kcycles summed over tiles
+        d["phase_kcycles"] = [int(x) for x in out[16:24]]
+    return d
