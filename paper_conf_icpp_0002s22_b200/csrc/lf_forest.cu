@@ -111,7 +111,7 @@ __device__ __forceinline__ bool is_local(int32_t x, int32_t b0) {
 // completed local cycle, non-negative pointers; R[k] the local distances (rank pass);
 // K[k] the min edge keys (cycle pass).  ek: keys of the own vertices' slots.
 template <bool MINK>
-__device__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
+__device__ __noinline__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
                           int2 (&R)[VPT], ulonglong2 (&K)[VPT], const bool (&skip)[VPT]) {
     const int tid = threadIdx.x;
     bool fin[VPT];
@@ -194,7 +194,7 @@ __device__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
     }
 }
 
-constexpr int kSplitShift = 28;  // splitter density 1/16 from the top 4 bits of a hash
+constexpr int kSplitShift = 29;  // splitter density 1/8 from the top 3 bits of a hash
 
 __device__ __forceinline__ bool hashed_splitter(int32_t g) {
     return (((uint32_t)g * 0x9E3779B1u) >> kSplitShift) == 0u;
@@ -488,7 +488,7 @@ __device__ __forceinline__ void reduced_dir(const TileSmem& s, int32_t b0, int32
 
 // Pass 1, local part: local min-scan; store the local results; emit the reduced-graph
 // records of boundary vertices.
-__global__ void __launch_bounds__(LT) k_lf_local1(ForestArgs a) {
+__global__ void __launch_bounds__(LT, 2) k_lf_local1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = blockIdx.x * LB;
@@ -769,7 +769,7 @@ __global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
 }
 
 // Pass 1 expand (break cycles, write the forest) fused with pass 2's local part.
-__global__ void __launch_bounds__(LT) k_lf_local2(ForestArgs a) {
+__global__ void __launch_bounds__(LT, 2) k_lf_local2(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = blockIdx.x * LB;
