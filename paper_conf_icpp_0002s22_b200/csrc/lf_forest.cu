@@ -66,7 +66,7 @@ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < 
     } while (0)
 #define LF_PHASE_INIT long long ph_t = clock64()
 #else
-#define LF_PHASE(ctl, i) do { } while (0)
+#define LF_PHASE(ctl, i) __syncthreads()  // a phase boundary is always a block barrier
 #define LF_PHASE_INIT do { } while (0)
 #endif
 
@@ -336,7 +336,10 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         const int id = s.sidx[u];
         if (id >= 0) {
             const short2 p = s.P[id];
-            P[k] = make_int2(p.x >= 0 ? p.x : -(s.spl[-(p.x + 1)] + 1), p.y >= 0 ? p.y : -(s.spl[-(p.y + 1)] + 1));
+            P[k].x = p.x;
+            P[k].y = p.y;
+            if (p.x < 0) P[k].x = -(s.spl[-(p.x + 1)] + 1);
+            if (p.y < 0) P[k].y = -(s.spl[-(p.y + 1)] + 1);
             if (MINK) { K[k].x = s.K0[id]; K[k].y = s.K1[id]; }
             else { const short2 r = s.R[id]; R[k] = make_int2(r.x, r.y); }
             continue;

@@ -11,7 +11,7 @@ import os
 from dataclasses import dataclass
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "liblf.so")
+LIB_PATH = os.environ.get("LF_LIB_PATH", os.path.join(HERE, "liblf.so"))
 
 LF_OK = 0
 ERRORS = {-1: "LF_EINVAL", -2: "LF_ENOMEM", -3: "LF_ECUDA", -4: "LF_ENCCL", -5: "LF_EINPUT"}
