@@ -180,11 +180,23 @@ __global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
 constexpr int PT = 256;
 constexpr int ETILE = 4096;
 
-template <int NN, int G>
+// sorted-descending top-NN insertion with an early exit: most candidates lose against
+// the current last slot, so the common path is one 64-bit compare
+template <int NN>
+__device__ __forceinline__ void topn_insert_fast(uint64_t (&t)[NN], uint64_t x) {
+    if (x <= t[NN - 1]) return;
+#pragma unroll
+    for (int i = NN - 1; i > 0; i--) {
+        if (x > t[i - 1]) t[i] = t[i - 1];
+        else { t[i] = x; return; }
+    }
+    t[0] = x;
+}
+
+template <int NN, int G, bool CHARGED>
 __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
     constexpr int R = PT / G;
-    __shared__ __align__(16) int32_t scol[ETILE];
-    __shared__ __align__(16) float sval[ETILE];
+    __shared__ __align__(16) int2 sent[ETILE];  // interleaved (col, value bits)
     __shared__ int64_t srp[R + 1];
     const int tid = threadIdx.x;
     const int64_t r0 = (int64_t)blockIdx.x * R;
@@ -200,15 +212,16 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
         const int64_t v1 = e1 & ~(int64_t)3;
         const int nvec = (int)((v1 - a0) >> 2);
         const int4* c4 = reinterpret_cast<const int4*>(a.col + a0);
-        const float4* f4 = reinterpret_cast<const float4*>(a.val + a0);
+        const int4* f4 = reinterpret_cast<const int4*>(a.val + a0);
         for (int i = tid; i < nvec; i += PT) {
-            reinterpret_cast<int4*>(scol)[i] = __ldg(c4 + i);
-            reinterpret_cast<float4*>(sval)[i] = __ldg(f4 + i);
+            const int4 c = __ldg(c4 + i);
+            const int4 f = __ldg(f4 + i);
+            int4* d = reinterpret_cast<int4*>(sent + 4 * i);
+            d[0] = make_int4(c.x, f.x, c.y, f.y);
+            d[1] = make_int4(c.z, f.z, c.w, f.w);
         }
-        for (int64_t e = v1 + tid; e < e1; e += PT) {
-            scol[e - a0] = __ldg(a.col + e);
-            sval[e - a0] = __ldg(a.val + e);
-        }
+        for (int64_t e = v1 + tid; e < e1; e += PT)
+            sent[e - a0] = make_int2(__ldg(a.col + e), __float_as_int(__ldg(a.val + e)));
     }
     __syncthreads();
     const int lr = tid / G, li = tid % G;
@@ -221,21 +234,35 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
     defer_append(a, deferred && li == 0, v);
     if (deferred) re = rs;
     uint32_t cv = 0;
-    if (valid && a.state) cv = (a.state[v] & ST_CHARGE) ? 1u : 0u;
+    if (CHARGED && valid) cv = (a.state[v] & ST_CHARGE) ? 1u : 0u;
     uint64_t top[NN];
 #pragma unroll
     for (int s = 0; s < NN; s++) top[s] = 0;
     uint32_t theta0 = 0, dbits = 0;
-    for (int64_t e = rs + li; e < re; e += G) {
-        int32_t j;
-        float x;
-        if (staged) { j = scol[e - a0]; x = sval[e - a0]; }
-        else { j = __ldg(a.col + e); x = __ldg(a.val + e); }
-        if (j == v) { dbits = __float_as_uint(x); continue; }          // diagonal (L231)
-        if ((__float_as_uint(x) & 0x7FFFFFFFu) == 0u) continue;       // zero (L31)
-        theta0 = 1;                      // round 0: nothing saturated, nothing confirmed
-        if (a.charging && ((((a.state[j] & ST_CHARGE) ? 1u : 0u)) == cv)) continue;  // L17
-        topn_insert<NN>(top, make_key(x, j));
+    if (staged) {
+        const int hi = (int)(re - a0);
+        for (int e = (int)(rs - a0) + li; e < hi; e += G) {
+            const int2 ent = sent[e];
+            const int32_t j = ent.x;
+            const uint32_t xb = (uint32_t)ent.y;
+            if (j == v) { dbits = xb; continue; }                        // diagonal (L231)
+            const uint32_t ab = xb & 0x7FFFFFFFu;
+            if (ab == 0u) continue;                                      // zero (L31)
+            theta0 = 1;                 // round 0: nothing saturated, nothing confirmed
+            if (CHARGED && (((a.state[j] & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
+            topn_insert_fast<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
+        }
+    } else {
+        for (int64_t e = rs + li; e < re; e += G) {
+            const int32_t j = __ldg(a.col + e);
+            const uint32_t xb = __float_as_uint(__ldg(a.val + e));
+            if (j == v) { dbits = xb; continue; }
+            const uint32_t ab = xb & 0x7FFFFFFFu;
+            if (ab == 0u) continue;
+            theta0 = 1;
+            if (CHARGED && (((a.state[j] & ST_CHARGE) ? 1u : 0u) == cv)) continue;
+            topn_insert_fast<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
+        }
     }
     if (G > 1) {
         topn_merge_group<NN, G>(top);
@@ -257,8 +284,8 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
             else { pj[s] = (s == 0 && !theta0) ? PROP_RETIRED : -1; pv[s] = 0.0f; }
         }
         if (NN == 2) {
-            reinterpret_cast<int2*>(a.prop_j)[v] = make_int2(pj[0], pj[1]);
-            reinterpret_cast<float2*>(a.prop_v)[v] = make_float2(pv[0], pv[1]);
+            reinterpret_cast<int2*>(a.prop_j)[v] = make_int2(pj[0], pj[NN > 1 ? 1 : 0]);
+            reinterpret_cast<float2*>(a.prop_v)[v] = make_float2(pv[0], pv[NN > 1 ? 1 : 0]);
         } else if (NN == 4) {
             reinterpret_cast<int4*>(a.prop_j)[v] = make_int4(pj[0], pj[NN > 1 ? 1 : 0], pj[NN > 2 ? 2 : 0], pj[NN > 3 ? 3 : 0]);
             reinterpret_cast<float4*>(a.prop_v)[v] = make_float4(pv[0], pv[NN > 1 ? 1 : 0], pv[NN > 2 ? 2 : 0], pv[NN > 3 ? 3 : 0]);
@@ -532,11 +559,20 @@ template <int NN>
 static void launch_propose_tile(int G, const ProposeArgs& pa, int64_t N, cudaStream_t s) {
     const int R = PT / G;
     const int grid = (int)((N + R - 1) / R);
-    switch (G) {
-        case 1: k_propose_tile<NN, 1><<<grid, PT, 0, s>>>(pa); break;
-        case 2: k_propose_tile<NN, 2><<<grid, PT, 0, s>>>(pa); break;
-        case 4: k_propose_tile<NN, 4><<<grid, PT, 0, s>>>(pa); break;
-        default: k_propose_tile<NN, 8><<<grid, PT, 0, s>>>(pa); break;
+    if (pa.charging) {
+        switch (G) {
+            case 1: k_propose_tile<NN, 1, true><<<grid, PT, 0, s>>>(pa); break;
+            case 2: k_propose_tile<NN, 2, true><<<grid, PT, 0, s>>>(pa); break;
+            case 4: k_propose_tile<NN, 4, true><<<grid, PT, 0, s>>>(pa); break;
+            default: k_propose_tile<NN, 8, true><<<grid, PT, 0, s>>>(pa); break;
+        }
+    } else {
+        switch (G) {
+            case 1: k_propose_tile<NN, 1, false><<<grid, PT, 0, s>>>(pa); break;
+            case 2: k_propose_tile<NN, 2, false><<<grid, PT, 0, s>>>(pa); break;
+            case 4: k_propose_tile<NN, 4, false><<<grid, PT, 0, s>>>(pa); break;
+            default: k_propose_tile<NN, 8, false><<<grid, PT, 0, s>>>(pa); break;
+        }
     }
 }
 
