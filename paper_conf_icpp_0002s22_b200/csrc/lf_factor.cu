@@ -193,8 +193,16 @@ __device__ __forceinline__ void topn_insert_fast(uint64_t (&t)[NN], uint64_t x) 
     t[0] = x;
 }
 
+#ifndef LF_TILE_MINB
+#define LF_TILE_MINB 4
+#endif
+#ifdef LF_BRANCHFREE
+#define TOPN_INS topn_insert
+#else
+#define TOPN_INS topn_insert_fast
+#endif
 template <int NN, int G, bool CHARGED>
-__global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
+__global__ void __launch_bounds__(PT, LF_TILE_MINB) k_propose_tile(ProposeArgs a) {
     constexpr int R = PT / G;
     __shared__ __align__(16) int2 sent[ETILE];  // interleaved (col, value bits)
     __shared__ int64_t srp[R + 1];
@@ -250,7 +258,7 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
             if (ab == 0u) continue;                                      // zero (L31)
             theta0 = 1;                 // round 0: nothing saturated, nothing confirmed
             if (CHARGED && (((a.state[j] & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
-            topn_insert_fast<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
+            TOPN_INS<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
         }
     } else {
         for (int64_t e = rs + li; e < re; e += G) {
@@ -261,7 +269,7 @@ __global__ void __launch_bounds__(PT) k_propose_tile(ProposeArgs a) {
             if (ab == 0u) continue;
             theta0 = 1;
             if (CHARGED && (((a.state[j] & ST_CHARGE) ? 1u : 0u) == cv)) continue;
-            topn_insert_fast<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
+            TOPN_INS<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
         }
     }
     if (G > 1) {

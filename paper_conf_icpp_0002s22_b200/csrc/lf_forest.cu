@@ -38,8 +38,17 @@ namespace cg = cooperative_groups;
 namespace lf {
 
 constexpr uint64_t KEY_INF = ~0ull;
-constexpr int LB = 2048;          // vertices per block-local tile
-constexpr int LT = 512;           // threads per tile CTA
+#ifndef LF_LB
+#define LF_LB 2048
+#endif
+#ifndef LF_LT
+#define LF_LT 512
+#endif
+#ifndef LF_LMINB
+#define LF_LMINB 2
+#endif
+constexpr int LB = LF_LB;         // vertices per block-local tile
+constexpr int LT = LF_LT;         // threads per tile CTA
 constexpr int VPT = LB / LT;      // vertices per thread
 constexpr int kCtlRed1 = 0;       // ctl[0..63]   per-step not-done counts, reduced scan 1
 constexpr int kCtlRed2 = 64;      // ctl[64..127] reduced scan 2
@@ -491,7 +500,7 @@ __device__ __forceinline__ void reduced_dir(const TileSmem& s, int32_t b0, int32
 
 // Pass 1, local part: local min-scan; store the local results; emit the reduced-graph
 // records of boundary vertices.
-__global__ void __launch_bounds__(LT, 2) k_lf_local1(ForestArgs a) {
+__global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = blockIdx.x * LB;
@@ -772,7 +781,7 @@ __global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
 }
 
 // Pass 1 expand (break cycles, write the forest) fused with pass 2's local part.
-__global__ void __launch_bounds__(LT, 2) k_lf_local2(ForestArgs a) {
+__global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = blockIdx.x * LB;
