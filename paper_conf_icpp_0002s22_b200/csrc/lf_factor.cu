@@ -193,8 +193,10 @@ __device__ __forceinline__ void topn_insert_fast(uint64_t (&t)[NN], uint64_t x) 
     t[0] = x;
 }
 
-#ifndef LF_TILE_MINB
-#define LF_TILE_MINB 4
+#if defined(LF_TILE_MINB) && LF_TILE_MINB > 0
+#define LF_TILE_BOUNDS __launch_bounds__(PT, LF_TILE_MINB)
+#else
+#define LF_TILE_BOUNDS __launch_bounds__(PT)
 #endif
 #ifdef LF_BRANCHFREE
 #define TOPN_INS topn_insert
@@ -202,7 +204,7 @@ __device__ __forceinline__ void topn_insert_fast(uint64_t (&t)[NN], uint64_t x) 
 #define TOPN_INS topn_insert_fast
 #endif
 template <int NN, int G, bool CHARGED>
-__global__ void __launch_bounds__(PT, LF_TILE_MINB) k_propose_tile(ProposeArgs a) {
+__global__ void LF_TILE_BOUNDS k_propose_tile(ProposeArgs a) {
     constexpr int R = PT / G;
     __shared__ __align__(16) int2 sent[ETILE];  // interleaved (col, value bits)
     __shared__ int64_t srp[R + 1];
