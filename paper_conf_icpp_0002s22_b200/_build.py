@@ -13,8 +13,9 @@ OBJ = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "liblf.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+NCCL_DIR = os.environ.get("LF_NCCL_DIR", "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl")
 FLAGS = [*os.environ.get("LF_EXTRA_FLAGS", "").split(), "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "--expt-relaxed-constexpr",
-         "-Xptxas", "-v", "-I", os.path.join(ROOT, "include")]
+         "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"), "-I", os.path.join(NCCL_DIR, "include")]
 
 
 def sources():
@@ -51,7 +52,9 @@ def build(force=False, verbose=False):
     with ThreadPoolExecutor(max_workers=os.cpu_count() or 4) as ex:
         objs = list(ex.map(comp, sources()))
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs]
+    nccl_lib = os.path.join(NCCL_DIR, "lib")
+    cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-L", nccl_lib, "-l:libnccl.so.2",
+           "-Xlinker", "-rpath=" + nccl_lib]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stderr}")

@@ -16,6 +16,8 @@ namespace lf {
 
 static thread_local char g_err[512] = "";
 
+void g_err_clear() { g_err[0] = 0; }
+
 int set_error(int code, const char* msg) {
     snprintf(g_err, sizeof(g_err), "%s", msg);
     return code;

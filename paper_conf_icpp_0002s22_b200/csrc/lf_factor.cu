@@ -27,7 +27,8 @@ namespace cg = cooperative_groups;
 namespace lf {
 
 struct ProposeArgs {
-    int64_t N;
+    int64_t N;                           // CSR rows (this partition's own rows)
+    int64_t row_base;                    // vertex id of CSR row r is row_base + r
     const int64_t* __restrict__ rowptr;
     const int32_t* __restrict__ col;
     const float* __restrict__ val;
@@ -75,7 +76,8 @@ __device__ __forceinline__ void propose_phase(const ProposeArgs& a) {
         const int64_t idx = base + lane / G;
         const bool valid = idx < count;
         int32_t v = -1;
-        if (valid) v = a.wl ? __ldg(a.wl + idx) : (int32_t)idx;
+        if (valid) v = a.wl ? __ldg(a.wl + idx) : (int32_t)(a.row_base + idx);
+        const int64_t row = (int64_t)v - a.row_base;
         int deg = 0;
         uint32_t cv = 0;
         int32_t p[NN];
@@ -92,8 +94,8 @@ __device__ __forceinline__ void propose_phase(const ProposeArgs& a) {
 #pragma unroll
                 for (int s = 0; s < NN; s++) p[s] = a.pi[(int64_t)v * NN + s];
             }
-            rs = __ldg(a.rowptr + v);
-            re = __ldg(a.rowptr + v + 1);
+            rs = __ldg(a.rowptr + row);
+            re = __ldg(a.rowptr + row + 1);
         }
         const bool deferred = valid && (re - rs) > a.defer_len;
         defer_append(a, deferred && li == 0, v);
@@ -237,7 +239,7 @@ __global__ void LF_TILE_BOUNDS k_propose_tile(ProposeArgs a) {
     const int lr = tid / G, li = tid % G;
     const int64_t row = r0 + lr;
     const bool valid = row < a.N;
-    const int32_t v = (int32_t)row;
+    const int32_t v = (int32_t)(a.row_base + row);
     const int64_t rs = srp[lr];
     int64_t re = valid ? srp[lr + 1] : rs;
     const bool deferred = valid && (re - rs) > a.defer_len;
@@ -335,7 +337,9 @@ __global__ void LF_TILE_BOUNDS k_propose_tile(ProposeArgs a) {
 }
 
 struct MutualArgs {
-    int64_t N;
+    int64_t N;                       // rows in all-rows mode (round 0)
+    int64_t row_base;                // vertex of row r in all-rows mode: row_base + r
+    int64_t gid_off;                 // global id of an own vertex v: v + gid_off (charges)
     const int32_t* __restrict__ wl;  // NULL = all rows (round 0)
     const int32_t* __restrict__ wl_count;
     const int32_t* __restrict__ prop_j;
@@ -367,7 +371,7 @@ __device__ __forceinline__ void mutual_phase(const MutualArgs& a) {
         bool keep = false;
         int32_t v = -1;
         if (idx < count) {
-            v = a.wl ? __ldg(a.wl + idx) : (int32_t)idx;
+            v = a.wl ? __ldg(a.wl + idx) : (int32_t)(a.row_base + idx);
             int32_t pj[NN];
 #pragma unroll
             for (int s = 0; s < NN; s++) pj[s] = a.prop_j[(int64_t)v * NN + s];
@@ -429,7 +433,7 @@ __device__ __forceinline__ void mutual_phase(const MutualArgs& a) {
             if (a.wl_next) {
                 uint32_t ch = 0;
                 keep = !retired && deg < NN;
-                if (keep && a.next_charging) ch = charge_bit((uint32_t)v, a.next_k, a.seed, a.thr);
+                if (keep && a.next_charging) ch = charge_bit((uint32_t)(v + a.gid_off), a.next_k, a.seed, a.thr);
                 a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0));
             } else if (a.fresh || nconf > 0) {
                 a.state[v] = (uint8_t)deg;
@@ -508,20 +512,24 @@ __global__ void __launch_bounds__(256) k_rounds_fused(FusedArgs f) {
 }
 
 // state of round 0 when round 0 is charged (k_m != 0): degree 0 + charge(v, 0)
-__global__ void k_init_state(int64_t N, uint8_t* state, uint32_t seed, unsigned long long thr) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N;
-         v += (int64_t)gridDim.x * blockDim.x)
-        state[v] = charge_bit((uint32_t)v, 0u, seed, thr) ? ST_CHARGE : 0;
+__global__ void k_init_state(int64_t NL, uint8_t* state, uint32_t seed, unsigned long long thr,
+                             const int32_t* __restrict__ l2g) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < NL;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t g = l2g ? (uint32_t)l2g[v] : (uint32_t)v;
+        state[v] = charge_bit(g, 0u, seed, thr) ? ST_CHARGE : 0;
+    }
 }
 
 // diagonal only (M = 0: no round streams the rows)
 __global__ void k_diag(int64_t N, const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
-                       const float* __restrict__ val, float* diag) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N;
-         v += (int64_t)gridDim.x * blockDim.x) {
+                       const float* __restrict__ val, float* diag, int64_t row_base) {
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < N;
+         r += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t v = (int32_t)(row_base + r);
         float d = 0.0f;
-        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; e++)
-            if (col[e] == (int32_t)v) d = val[e];
+        for (int64_t e = rowptr[r]; e < rowptr[r + 1]; e++)
+            if (col[e] == v) d = val[e];
         diag[v] = d;
     }
 }
@@ -606,8 +614,12 @@ static int lanes_per_row(double avg) {
 template <int NN>
 static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi, float* pi_w,
                        float* pi_val, float* diag, int32_t* rounds_dev, int64_t* live,
-                       const FactorWs& w, cudaStream_t s) {
-    const int64_t N = A->n;
+                       const FactorWs& w, cudaStream_t s, const PartCtx* part) {
+    const int64_t N = A->n;                        // CSR rows
+    const int64_t NL = part ? part->NL : N;        // vertex-indexed array length
+    const int64_t row_base = part ? part->row_base : 0;
+    const int64_t gid_off = part ? part->gid_off : 0;
+    if (part && o->until_maximal) return set_error(LF_EINVAL, "partitioned factor: until_maximal unsupported");
     const int M = o->until_maximal ? 0x7fffffff : o->M;
     const double pthr = (double)o->p * 4294967296.0;
     unsigned long long thr = pthr <= 0 ? 0ull : (pthr >= 4294967296.0 ? 4294967296ull
@@ -623,15 +635,16 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         LF_CUDA(cudaMemsetAsync(w.live_part, 0, sizeof(unsigned long long) * 128 * o->M, s));
     if (N == 0 || (!o->until_maximal && o->M == 0)) {
         // no rounds: empty factor
-        if (N > 0) {
-            LF_CUDA(cudaMemsetAsync(pi, 0xff, sizeof(int32_t) * N * NN, s));
-            LF_CUDA(cudaMemsetAsync(pi_w, 0, sizeof(float) * N * NN, s));
-            if (pi_val) LF_CUDA(cudaMemsetAsync(pi_val, 0, sizeof(float) * N * NN, s));
-            if (diag) {
-                LF_PROF("diag", -1, s);
-                k_diag<<<persistent_grid((const void*)k_diag, 256), 256, 0, s>>>(N, A->rowptr, A->col, A->val, diag);
-                LF_CUDA(cudaGetLastError());
-            }
+        if (NL > 0) {
+            LF_CUDA(cudaMemsetAsync(pi, 0xff, sizeof(int32_t) * NL * NN, s));
+            LF_CUDA(cudaMemsetAsync(pi_w, 0, sizeof(float) * NL * NN, s));
+            if (pi_val) LF_CUDA(cudaMemsetAsync(pi_val, 0, sizeof(float) * NL * NN, s));
+        }
+        if (N > 0 && diag) {
+            LF_PROF("diag", -1, s);
+            k_diag<<<persistent_grid((const void*)k_diag, 256), 256, 0, s>>>(N, A->rowptr, A->col, A->val, diag,
+                                                                           row_base);
+            LF_CUDA(cudaGetLastError());
         }
         if (rounds_dev) LF_CUDA(cudaMemsetAsync(rounds_dev, 0, sizeof(int32_t), s));
         return LF_OK;
@@ -639,18 +652,24 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
     const bool charged0 = (0 % o->m) != o->k_m;
     if (charged0) {
         LF_PROF("init_state", -1, s);
-        k_init_state<<<persistent_grid((const void*)k_init_state, 256), 256, 0, s>>>(N, w.state, o->seed, thr);
+        k_init_state<<<persistent_grid((const void*)k_init_state, 256), 256, 0, s>>>(
+            NL, w.state, o->seed, thr, part ? part->l2g : nullptr);
         LF_CUDA(cudaGetLastError());
     }
     int rounds_host = -1;
     // rounds 1..M-1 in one cooperative kernel unless the host must check maximality
-    const bool fuse = !o->until_maximal && o->M > 1;
+    const bool fuse = !o->until_maximal && o->M > 1 && !part;
     const int M_loop = fuse ? 1 : M;
     for (int k = 0; k < M_loop; k++) {
         const bool charging = (k % o->m) != o->k_m;
         const bool fresh = (k == 0);
+        if (part && (k > 0 || charged0)) {  // halo: ghost degrees and charges of round k
+            const int rc = part->pre_propose(part->ctx, k, s);
+            if (rc) return rc;
+        }
         ProposeArgs pa;
         pa.N = N;
+        pa.row_base = row_base;
         pa.rowptr = A->rowptr;
         pa.col = A->col;
         pa.val = A->val;
@@ -705,7 +724,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
                 if (fresh) {
                     // nothing proposed at all: export the empty factor
                     MutualArgs ma{};
-                    ma.N = N; ma.prop_j = w.prop_j; ma.prop_v = w.prop_v; ma.state = w.state;
+                    ma.N = N; ma.row_base = row_base; ma.gid_off = gid_off; ma.prop_j = w.prop_j; ma.prop_v = w.prop_v; ma.state = w.state;
                     ma.pi = pi; ma.pi_w = pi_w; ma.pi_val = pi_val; ma.fresh = 1;
                     k_mutual<NN><<<grid_m, 256, 0, s>>>(ma);
                     LF_CUDA(cudaGetLastError());
@@ -713,10 +732,16 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
                 break;
             }
         }
+        if (part) {  // halo: ghost proposals of round k
+            const int rc = part->pre_mutual(part->ctx, k, s);
+            if (rc) return rc;
+        }
         const bool last = !o->until_maximal && (k == M - 1);
         MutualArgs ma;
         ma.wl_zero = nullptr;
         ma.N = N;
+        ma.row_base = row_base;
+        ma.gid_off = gid_off;
         ma.wl = fresh ? nullptr : w.wl[k & 1];
         ma.wl_count = fresh ? nullptr : &w.counts[k % 3];
         ma.prop_j = w.prop_j;
@@ -744,6 +769,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         memset(&f, 0, sizeof(f));
         ProposeArgs& pa = f.pa;
         pa.N = N;
+        pa.row_base = 0;
         pa.rowptr = A->rowptr;
         pa.col = A->col;
         pa.val = A->val;
@@ -755,6 +781,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         pa.defer_list = w.long_rows;
         MutualArgs& ma = f.ma;
         ma.N = N;
+        ma.row_base = 0;
+        ma.gid_off = 0;
         ma.prop_j = w.prop_j;
         ma.prop_v = w.prop_v;
         ma.state = w.state;
@@ -793,6 +821,10 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_CUDA(cudaStreamSynchronize(s));
         }
     } else if (rounds_dev || live) {
+        if (part && part->pre_finalize) {  // global maximality flags / counters
+            const int rc = part->pre_finalize(part->ctx, s);
+            if (rc) return rc;
+        }
         LF_PROF("finalize", -1, s);
         k_finalize<<<1, 32, 0, s>>>(w.flags, o->M, o->m, o->k_m, rounds_dev, w.live_part, live);
         LF_CUDA(cudaGetLastError());
@@ -802,12 +834,12 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
 
 int factor_dispatch(const lf_csr_t* A, int n, const lf_factor_opts_t* o, int32_t* pi, float* pi_w,
                     float* pi_val, float* diag, int32_t* rounds_dev, int64_t* live, const FactorWs& w,
-                    cudaStream_t s) {
+                    cudaStream_t s, const PartCtx* part) {
     switch (n) {
-        case 1: return factor_impl<1>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
-        case 2: return factor_impl<2>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
-        case 3: return factor_impl<3>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
-        case 4: return factor_impl<4>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s);
+        case 1: return factor_impl<1>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s, part);
+        case 2: return factor_impl<2>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s, part);
+        case 3: return factor_impl<3>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s, part);
+        case 4: return factor_impl<4>(A, o, pi, pi_w, pi_val, diag, rounds_dev, live, w, s, part);
         default: return set_error(LF_EINVAL, "n must be in [1,4]");
     }
 }

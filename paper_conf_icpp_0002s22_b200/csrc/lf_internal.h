@@ -15,6 +15,8 @@ constexpr int kMaxFlagRounds = 1024;  // maximality flags kept on the device (ri
 // error state (thread-local message, lf_api.cu)
 int set_error(int code, const char* msg);
 int set_cuda_error(cudaError_t e, const char* where);
+inline int set_cuda_rc(cudaError_t e, const char* where) { return e == cudaSuccess ? LF_OK : set_cuda_error(e, where); }
+void g_err_clear();
 
 #define LF_CUDA(call)                                                     \
     do {                                                                  \
@@ -65,9 +67,22 @@ struct FactorWs {
 };
 size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w);
 
+// partitioned run of the factor (one contiguous row range of a larger graph, ghost
+// vertices filled by a halo exchange between rounds); nullptr = a whole graph
+struct PartCtx {
+    int64_t row_base;   // local id of the first own row (number of ghosts below the range)
+    int64_t gid_off;    // global id of own local vertex v is v + gid_off
+    int64_t NL;         // local vertices (ghosts below + own + ghosts above)
+    const int32_t* l2g; // [NL] global id of each local vertex
+    void* ctx;
+    int (*pre_propose)(void* ctx, int k, cudaStream_t s);  // ghost state (degree, charge)
+    int (*pre_mutual)(void* ctx, int k, cudaStream_t s);   // ghost proposals
+    int (*pre_finalize)(void* ctx, cudaStream_t s);        // global flags / counters
+};
+
 int factor_dispatch(const lf_csr_t* A, int n, const lf_factor_opts_t* o, int32_t* pi, float* pi_w,
                     float* pi_val, float* diag, int32_t* rounds_dev, int64_t* live,
-                    const FactorWs& w, cudaStream_t s);
+                    const FactorWs& w, cudaStream_t s, const PartCtx* part = nullptr);
 
 struct ForestWs {
     int2* rq1[2];          // reduced graph, cycle pass: stride pointers (ping-pong)

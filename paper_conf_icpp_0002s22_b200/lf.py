@@ -22,7 +22,9 @@ EXPORTS = (
     "lf_linear_forest_workspace_size", "lf_linear_forest", "lf_tridiag",
     "lf_pipeline_workspace_size", "lf_pipeline_host", "lf_validate_csr",
     "lf_last_error", "lf_version", "lf_profile_enable", "lf_profile_collect",
-    "lf_forest_stats",
+    "lf_forest_stats", "lf_comm_nccl_unique_id", "lf_comm_create_nccl", "lf_comm_create_loopback",
+    "lf_comm_destroy", "lf_part_create", "lf_part_destroy", "lf_part_info", "lf_part_factor",
+    "lf_part_export",
 )
 
 
@@ -65,6 +67,15 @@ def load(path: str = LIB_PATH):
     L.lf_pipeline_host.argtypes = [P, P, P, P, P, P, P, P, P, C.c_size_t, P]
     L.lf_validate_csr.argtypes = [P, P, C.c_size_t, P]
     L.lf_forest_stats.argtypes = [I64, P, C.c_size_t, P, I32]
+    L.lf_comm_nccl_unique_id.argtypes = [P]
+    L.lf_comm_create_nccl.argtypes = [P, I32, I32, P]
+    L.lf_comm_create_loopback.argtypes = [I32, P]
+    L.lf_comm_destroy.argtypes = [P]
+    L.lf_part_create.argtypes = [I32, P, I32, P, I32, P, P]
+    L.lf_part_destroy.argtypes = [P, P]
+    L.lf_part_info.argtypes = [P, P, I32]
+    L.lf_part_factor.argtypes = [P, I32, P, P, P]
+    L.lf_part_export.argtypes = [P, P, P, P, P, P, P, P]
     L.lf_profile_enable.argtypes = [I32]
     L.lf_profile_collect.argtypes = [P, I32, P, I32]
     L.lf_last_error.restype = C.c_char_p
