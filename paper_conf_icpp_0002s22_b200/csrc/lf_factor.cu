@@ -577,6 +577,7 @@ template <int NN>
 static void launch_propose_tile(int G, const ProposeArgs& pa, int64_t N, cudaStream_t s) {
     const int R = PT / G;
     const int grid = (int)((N + R - 1) / R);
+    if (grid == 0) return;
     if (pa.charging) {
         switch (G) {
             case 1: k_propose_tile<NN, 1, true><<<grid, PT, 0, s>>>(pa); break;
@@ -633,8 +634,9 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
     LF_CUDA(cudaMemsetAsync(w.counts, 0, sizeof(int32_t) * 4, s));
     if (live && !o->until_maximal && o->M > 0)
         LF_CUDA(cudaMemsetAsync(w.live_part, 0, sizeof(unsigned long long) * 128 * o->M, s));
-    if (N == 0 || (!o->until_maximal && o->M == 0)) {
-        // no rounds: empty factor
+    if ((N == 0 && !part) || (!o->until_maximal && o->M == 0)) {
+        // no rounds: empty factor (a partition with no rows still takes part in the
+        // exchanges below, so it only returns here when there are no rounds at all)
         if (NL > 0) {
             LF_CUDA(cudaMemsetAsync(pi, 0xff, sizeof(int32_t) * NL * NN, s));
             LF_CUDA(cudaMemsetAsync(pi_w, 0, sizeof(float) * NL * NN, s));
