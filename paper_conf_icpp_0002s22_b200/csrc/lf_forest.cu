@@ -29,6 +29,7 @@
 
 #include <cub/device/device_scan.cuh>
 #include <cstdint>
+#include <cstring>
 
 #include "lf_common.cuh"
 #include "lf_internal.h"
@@ -104,10 +105,12 @@ struct TileSmem {
     short2 recS[LB];      // per face: (node << 1 | start slot) of the walk that visited it
     short2 recD[LB];      // per face: distance to that node
     int nspl;             // number of splitter nodes
+    int32_t b0, tend;     // first vertex of the tile, one past its last (own range end)
 };
 
-__device__ __forceinline__ bool is_local(int32_t x, int32_t b0) {
-    return x >= b0 && x < b0 + LB;
+// x lies in this tile (the tile never extends past the own range [lo, hi))
+__device__ __forceinline__ bool is_local(int32_t x, const TileSmem& s) {
+    return x >= s.b0 && x < s.tend;
 }
 
 // Bidirectional scan inside the tile (Alg. 3, or its min variant when MINK, restricted
@@ -129,8 +132,8 @@ __device__ __noinline__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2
         const int u = tid + k * LT;
         if (skip[k]) { fin[k] = true; continue; }
         const int2 nb = s.nb[u];
-        const bool l0 = nb.x >= 0 && is_local(nb.x, b0);
-        const bool l1 = nb.y >= 0 && is_local(nb.y, b0);
+        const bool l0 = nb.x >= 0 && is_local(nb.x, s);
+        const bool l1 = nb.y >= 0 && is_local(nb.y, s);
         P[k] = make_int2(l0 ? nb.x - b0 : -(u + 1), l1 ? nb.y - b0 : -(u + 1));
         fin[k] = !l0 && !l1;
         s.P[u] = make_short2((short)P[k].x, (short)P[k].y);
@@ -229,8 +232,8 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
     for (int k = 0; k < VPT; k++) {
         const int u = tid + k * LT;
         const int2 nb = s.nb[u];
-        const bool l0 = nb.x >= 0 && is_local(nb.x, b0);
-        const bool l1 = nb.y >= 0 && is_local(nb.y, b0);
+        const bool l0 = nb.x >= 0 && is_local(nb.x, s);
+        const bool l1 = nb.y >= 0 && is_local(nb.y, s);
         const bool sp = !l0 || !l1 || hashed_splitter(b0 + u);
         short id = -1;
         if (sp) id = (short)atomicAdd(&s.nspl, 1);
@@ -250,7 +253,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         short ptr = (short)(-(i + 1));
         int dist = 0;
         uint64_t km = KEY_INF;
-        if (x >= 0 && is_local(x, b0)) {
+        if (x >= 0 && is_local(x, s)) {
             int prev = su, cur = x - b0, d = 1;
             if (MINK) {
                 const float2 ws = s.w[su];
@@ -403,8 +406,8 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
 
 // the slot of local terminal t (t not the walk's start) that leaves its segment: the
 // one that is not a local link (a remote neighbour or none)
-__device__ __forceinline__ int outward_slot(int2 nbt, int32_t b0) {
-    const bool l0 = nbt.x >= 0 && is_local(nbt.x, b0);
+__device__ __forceinline__ int outward_slot(int2 nbt, const TileSmem& s) {
+    const bool l0 = nbt.x >= 0 && is_local(nbt.x, s);
     return l0 ? 1 : 0;
 }
 
@@ -418,7 +421,15 @@ __device__ __forceinline__ void list_append(int32_t* list, int* count, int32_t g
 }
 
 struct ForestArgs {
-    int64_t N;
+    int64_t N;             // global vertex count (markers: end -(e+1), exit -(N+1+e))
+    int64_t lo, hi;        // own vertex range (a whole graph: 0, N); arrays are offset so
+                           // that vertex g is element g
+    // foreign neighbours' slots (partitioned runs): sorted ghost ids and their slots
+    const int32_t* ghost_list;
+    int64_t n_ghost, ghost_below;
+    const int2* ghost_nb;  // [local id] slots (global ids) of ghost vertices
+    ulonglong2* kraw;      // [v] final per-direction min keys of the cycle pass (boundary)
+    ulonglong2* ekb;       // [v] slot keys of boundary vertices
     const int2* __restrict__ pi2;
     const float2* __restrict__ pi2_w;
     int2* forest;
@@ -445,6 +456,19 @@ struct ForestArgs {
     int max_steps;
 };
 
+__device__ __forceinline__ bool is_foreign(int64_t x, const ForestArgs& a) { return x < a.lo || x >= a.hi; }
+
+// slots of a vertex of another rank (binary search in the sorted ghost list)
+__device__ __forceinline__ int2 ghost_slots(const ForestArgs& a, int32_t x) {
+    int64_t l = 0, h = a.n_ghost;
+    while (l < h) {
+        const int64_t m = (l + h) >> 1;
+        if (a.ghost_list[m] < x) l = m + 1; else h = m;
+    }
+    const int64_t lid = l < a.ghost_below ? l : l + (a.hi - a.lo);
+    return a.ghost_nb[lid];
+}
+
 // keys of the own vertices' slots (global; a remote min endpoint needs one gather)
 __device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int32_t b0,
                                          ulonglong2 (&ek)[VPT]) {
@@ -455,46 +479,55 @@ __device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int3
         const int2 nb = s.nb[u];
         ek[k].x = KEY_INF;
         ek[k].y = KEY_INF;
-        if (g >= a.N) { s.w[u] = make_float2(0.f, 0.f); continue; }
+        if (g >= a.hi) { s.w[u] = make_float2(0.f, 0.f); continue; }
         const float2 w = a.pi2_w[g];
         s.w[u] = w;
         if (nb.x >= 0) {
             const int32_t mn = g < nb.x ? g : nb.x;
-            const int2 nbm = is_local(mn, b0) ? s.nb[mn - b0] : a.pi2[mn];
+            const int2 nbm = is_local(mn, s) ? s.nb[mn - b0] : (is_foreign(mn, a) ? ghost_slots(a, mn) : a.pi2[mn]);
             ek[k].x = edge_key(g, nb.x, w.x, nbm);
         }
         if (nb.y >= 0) {
             const int32_t mn = g < nb.y ? g : nb.y;
-            const int2 nbm = is_local(mn, b0) ? s.nb[mn - b0] : a.pi2[mn];
+            const int2 nbm = is_local(mn, s) ? s.nb[mn - b0] : (is_foreign(mn, a) ? ghost_slots(a, mn) : a.pi2[mn]);
             ek[k].y = edge_key(g, nb.y, w.y, nbm);
         }
     }
 }
 
-__device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem& s, int32_t b0, int64_t N) {
+__device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem& s, int32_t b0, int64_t hi) {
+    if (threadIdx.x == 0) {
+        s.b0 = b0;
+        s.tend = (int32_t)((int64_t)b0 + LB < hi ? (int64_t)b0 + LB : hi);
+    }
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
         const int64_t g = (int64_t)b0 + u;
-        s.nb[u] = g < N ? src[g] : make_int2(-1, -1);
+        s.nb[u] = g < hi ? src[g] : make_int2(-1, -1);
     }
     __syncthreads();
 }
 
 // reduced-graph direction of boundary vertex g through its slot i:
-//   none -> end marker at g (distance 0); remote -> the neighbour (distance 1);
-//   local -> the segment's other terminal t: t itself if t continues in another block,
-//   else an end marker at t (distance = local length).
-__device__ __forceinline__ void reduced_dir(const TileSmem& s, int32_t b0, int32_t g, int2 nb, int i,
-                                            int2 p, int2 r, int32_t& q, int32_t& d) {
+//   none -> end marker -(g+1) (distance 0); another rank -> exit marker -(N+1+g)
+//   (distance 0; the exit list continues it); another tile -> the neighbour (distance 1);
+//   local -> the segment's other terminal t: t if t continues in another tile of this
+//   rank, else an end or exit marker at t (distance = local length).
+__device__ __forceinline__ void reduced_dir(const ForestArgs& a, const TileSmem& s, int32_t b0, int32_t g,
+                                            int2 nb, int i, int2 p, int2 r, int32_t& q, int32_t& d) {
     const int32_t x = i ? nb.y : nb.x;
     if (x < 0) { q = -(g + 1); d = 0; return; }
-    if (!is_local(x, b0)) { q = x; d = 1; return; }
+    if (is_foreign(x, a)) { q = (int32_t)(-(a.N + 1 + g)); d = 0; return; }
+    if (!is_local(x, s)) { q = x; d = 1; return; }
     const int t = -((i ? p.y : p.x) + 1);
     const int2 nbt = s.nb[t];
-    const int so = outward_slot(nbt, b0);
+    const int so = outward_slot(nbt, s);
     const int32_t xo = so ? nbt.y : nbt.x;
-    q = xo >= 0 ? (b0 + t) : -(b0 + t + 1);
+    const int32_t tg = b0 + t;
+    if (xo < 0) q = -(tg + 1);
+    else if (is_foreign(xo, a)) q = (int32_t)(-(a.N + 1 + tg));
+    else q = tg;
     d = i ? r.y : r.x;
 }
 
@@ -503,9 +536,9 @@ __device__ __forceinline__ void reduced_dir(const TileSmem& s, int32_t b0, int32
 __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
-    const int32_t b0 = blockIdx.x * LB;
+    const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     LF_PHASE_INIT;
-    load_tile(a.pi2, s, b0, a.N);
+    load_tile(a.pi2, s, b0, a.hi);
     LF_PHASE(a.ctl, 0);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
@@ -519,21 +552,22 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local1(ForestArgs a) {
         const int u = threadIdx.x + k * LT;
         const int32_t g = b0 + u;
         const int2 nb = s.nb[u];
-        const bool r0 = nb.x >= 0 && !is_local(nb.x, b0);
-        const bool r1 = nb.y >= 0 && !is_local(nb.y, b0);
-        const bool boundary = g < a.N && (r0 || r1);
-        if (g < a.N) {
+        const bool r0 = nb.x >= 0 && !is_local(nb.x, s);
+        const bool r1 = nb.y >= 0 && !is_local(nb.y, s);
+        const bool boundary = g < a.hi && (r0 || r1);
+        if (g < a.hi) {
             a.loc1[g] = make_short2((short)P[k].x, (short)P[k].y);
             if (P[k].x >= 0 && P[k].y >= 0) a.kst[g] = umin64(K[k].x, K[k].y);
         }
         if (boundary) {
             int32_t q0, q1, d0, d1;
-            reduced_dir(s, b0, g, nb, 0, P[k], R[k], q0, d0);
-            reduced_dir(s, b0, g, nb, 1, P[k], R[k], q1, d1);
+            reduced_dir(a, s, b0, g, nb, 0, P[k], R[k], q0, d0);
+            reduced_dir(a, s, b0, g, nb, 1, P[k], R[k], q1, d1);
             // key of each reduced link: the remote edge's key, or the segment's min key
             ulonglong2 rk;
-            rk.x = (nb.x < 0) ? KEY_INF : (r0 ? ek[k].x : K[k].x);
-            rk.y = (nb.y < 0) ? KEY_INF : (r1 ? ek[k].y : K[k].y);
+            rk.x = (nb.x < 0 || is_foreign(nb.x, a)) ? KEY_INF : (r0 ? ek[k].x : K[k].x);
+            rk.y = (nb.y < 0 || is_foreign(nb.y, a)) ? KEY_INF : (r1 ? ek[k].y : K[k].y);
+            if (a.ekb) a.ekb[g] = ek[k];
             const int2 q = make_int2(q0, q1);
             a.rq1[0][g] = q; a.rq1[1][g] = q;
             a.rk1[0][g] = rk; a.rk1[1][g] = rk;
@@ -629,9 +663,10 @@ __device__ __forceinline__ void red_epilogue(const ForestArgs& a, const int32_t*
             const int2 q = a.rq1[fb][v];
             const ulonglong2 k = a.rk1[fb][v];
             a.cyc_k[v] = (q.x >= 0 && q.y >= 0) ? umin64(k.x, k.y) : KEY_INF;
+            a.end2[v] = q;  // raw markers (exit list construction)
+            if (a.kraw) a.kraw[v] = k;
         } else {
-            const int2 q = a.rq2[fb][v];
-            a.end2[v] = make_int2(-(q.x + 1), -(q.y + 1));
+            a.end2[v] = a.rq2[fb][v];  // raw end markers -(e+1) (or exit markers)
             a.dist2[v] = a.rr2[fb][v];
         }
     }
@@ -732,10 +767,14 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
 #pragma unroll
     for (int k = 0; k < RNPT; k++) {
         if (v[k] < 0) continue;
+        // pointers back to vertex ids (markers pass through unchanged)
+        const int2 qg = make_int2(q[k].x >= 0 ? list[q[k].x] : q[k].x, q[k].y >= 0 ? list[q[k].y] : q[k].y);
         if (MIN) {
             a.cyc_k[v[k]] = (q[k].x >= 0 && q[k].y >= 0) ? umin64(kk[k].x, kk[k].y) : KEY_INF;
+            a.end2[v[k]] = qg;
+            if (a.kraw) a.kraw[v[k]] = kk[k];
         } else {
-            a.end2[v[k]] = make_int2(-(q[k].x + 1), -(q[k].y + 1));
+            a.end2[v[k]] = qg;
             a.dist2[v[k]] = make_int2((int)kk[k].x, (int)kk[k].y);
         }
     }
@@ -784,8 +823,8 @@ __global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
 __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
-    const int32_t b0 = blockIdx.x * LB;
-    load_tile(a.pi2, s, b0, a.N);
+    const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
+    load_tile(a.pi2, s, b0, a.hi);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
     // weakest edge of the cycle through each own vertex (INF: not on a cycle)
@@ -797,7 +836,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
         const int32_t g = b0 + u;
         const int2 nb = s.nb[u];
         f[k] = nb;
-        if (g >= a.N) continue;
+        if (g >= a.hi) continue;
         const short2 p = a.loc1[g];
         uint64_t kstar = KEY_INF;
         if (p.x >= 0 && p.y >= 0) {  // local cycle
@@ -809,7 +848,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
             for (int i = 0; i < 2; i++) {
                 const int t = -((i ? p.y : p.x) + 1);
                 const int2 nbt = s.nb[t];
-                const int so = (t == u) ? i : outward_slot(nbt, b0);
+                const int so = (t == u) ? i : outward_slot(nbt, s);
                 const int32_t xo = so ? nbt.y : nbt.x;
                 if (xo >= 0 && kstar == KEY_INF) kstar = a.cyc_k[b0 + t];
             }
@@ -844,10 +883,10 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
         const int u = threadIdx.x + k * LT;
         const int32_t g = b0 + u;
         const int2 nb = s.nb[u];
-        const bool r0 = nb.x >= 0 && !is_local(nb.x, b0);
-        const bool r1 = nb.y >= 0 && !is_local(nb.y, b0);
-        const bool boundary = g < a.N && (r0 || r1);
-        if (g < a.N) {
+        const bool r0 = nb.x >= 0 && !is_local(nb.x, s);
+        const bool r1 = nb.y >= 0 && !is_local(nb.y, s);
+        const bool boundary = g < a.hi && (r0 || r1);
+        if (g < a.hi) {
             // terminal markers (16 bits each) and local distances (16 bits each)
             const uint32_t pp = ((uint32_t)(uint16_t)(short)P[k].x) | ((uint32_t)(uint16_t)(short)P[k].y << 16);
             const uint32_t rr = ((uint32_t)(uint16_t)R[k].x) | ((uint32_t)(uint16_t)R[k].y << 16);
@@ -855,8 +894,8 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
         }
         if (boundary) {
             int32_t q0, q1, d0, d1;
-            reduced_dir(s, b0, g, nb, 0, P[k], R[k], q0, d0);
-            reduced_dir(s, b0, g, nb, 1, P[k], R[k], q1, d1);
+            reduced_dir(a, s, b0, g, nb, 0, P[k], R[k], q0, d0);
+            reduced_dir(a, s, b0, g, nb, 1, P[k], R[k], q1, d1);
             const int2 q = make_int2(q0, q1);
             const int2 d = make_int2(d0, d1);
             a.rq2[0][g] = q; a.rq2[1][g] = q;
@@ -870,13 +909,13 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
 __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
-    const int32_t b0 = blockIdx.x * LB;
-    load_tile(a.forest, s, b0, a.N);
+    const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
+    load_tile(a.forest, s, b0, a.hi);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
         const int32_t g = b0 + u;
-        if (g >= a.N) continue;
+        if (g >= a.hi) continue;
         const int2 lc = a.loc2[g];
         const int px = (short)(lc.x & 0xffff), py = (short)((uint32_t)lc.x >> 16);
         const int rx = lc.y & 0xffff, ry = (int)((uint32_t)lc.y >> 16);
@@ -887,12 +926,12 @@ __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
             const int32_t d = i ? ry : rx;
             const int2 nbt = s.nb[t];
             // the outward slot of t: slot i itself when t == u (the walk never left u)
-            const int so = (t == u) ? i : outward_slot(nbt, b0);
+            const int so = (t == u) ? i : outward_slot(nbt, s);
             const int32_t xo = so ? nbt.y : nbt.x;
-            if (xo >= 0) {  // continues in another block: reduced result of t
+            if (xo >= 0) {  // continues in another block: reduced result of t (end marker)
                 const int2 e = a.end2[b0 + t];
                 const int2 dd = a.dist2[b0 + t];
-                E[i] = so ? e.y : e.x;
+                E[i] = -((so ? e.y : e.x) + 1);
                 D[i] = d + (so ? dd.y : dd.x);
             } else {
                 E[i] = b0 + t;
@@ -992,7 +1031,10 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
     if (n_cycles) LF_CUDA(cudaMemsetAsync(n_cycles, 0, sizeof(int64_t), s));
     ForestArgs a;
+    memset(&a, 0, sizeof(a));
     a.N = N;
+    a.lo = 0;
+    a.hi = N;
     a.pi2 = (const int2*)pi2;
     a.pi2_w = (const float2*)pi2_w;
     a.forest = (int2*)forest;
