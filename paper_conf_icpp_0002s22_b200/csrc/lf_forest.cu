@@ -688,7 +688,8 @@ struct RedSmem {
 template <bool MIN>
 __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt, int* ctl, RedSmem& S) {
     const int tid = threadIdx.x;
-    int32_t* cidx = MIN ? (int32_t*)a.end2 : (int32_t*)a.dist2;  // [N] scratch, unused yet
+    // [vertex] scratch, unused yet (an int32 view of end2/dist2, indexed by vertex id)
+    int32_t* cidx = (MIN ? (int32_t*)(a.end2 + a.lo) : (int32_t*)(a.dist2 + a.lo)) - a.lo;
     int32_t v[RNPT];
 #pragma unroll
     for (int k = 0; k < RNPT; k++) {
@@ -989,6 +990,8 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     t.len = c.take<int32_t>(n);
     t.off = c.take<int32_t>(n);
     t.ctl = c.take<int>(256);
+    t.kraw = c.take<ulonglong2>(n);
+    t.ekb = c.take<ulonglong2>(n);
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
     if (w) *w = t;
@@ -1009,6 +1012,21 @@ static int coop_launch(K kernel, int block, ForestArgs& a, cudaStream_t s, size_
     return LF_OK;
 }
 
+static int forest_prepare() {
+    static bool attr_done = false;
+    if (attr_done) return LF_OK;
+    const int smem = (int)sizeof(TileSmem);
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local1, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local2, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local3, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sizeof(RedSmem)));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sizeof(RedSmem)));
+    attr_done = true;
+    return LF_OK;
+}
+
 int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
                int32_t* pos, int32_t* perm, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
                cudaStream_t s) {
@@ -1016,18 +1034,9 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         if (n_cycles) LF_CUDA(cudaMemsetAsync(n_cycles, 0, sizeof(int64_t), s));
         return LF_OK;
     }
-    static bool attr_done = false;
+    int rcp = forest_prepare();
+    if (rcp) return rcp;
     const int smem = (int)sizeof(TileSmem);
-    if (!attr_done) {
-        LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local1, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local2, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local3, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)sizeof(RedSmem)));
-        LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)sizeof(RedSmem)));
-        attr_done = true;
-    }
     LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
     if (n_cycles) LF_CUDA(cudaMemsetAsync(n_cycles, 0, sizeof(int64_t), s));
     ForestArgs a;
@@ -1114,6 +1123,348 @@ int forest_stats(const ForestWs& w, int32_t* out, int cap) {
     // [16..31]: per-phase cycle sums (units of 1024 cycles; LF_PHASE_TIMING builds only)
     const unsigned long long* ph = reinterpret_cast<const unsigned long long*>(h + 208);
     for (int i = 0; i < 16 && 16 + i < cap; i++) out[16 + i] = (int)(ph[i] >> 10);
+    return LF_OK;
+}
+
+
+// ---------------------------------------------------------------------------
+// partitioned runs: exit records, global exit-graph scan, fold-back, offsets
+// ---------------------------------------------------------------------------
+struct ExitRec {
+    int32_t g, q0, q1, d0, d1, pad;
+    uint64_t k0, k1;
+};
+
+size_t exit_record_bytes() { return sizeof(ExitRec); }
+
+__device__ __forceinline__ bool is_exit_marker(int32_t m, int64_t N) { return (int64_t)m <= -(N + 1); }
+__device__ __forceinline__ int32_t exit_vertex(int32_t m, int64_t N) { return (int32_t)(-(int64_t)m - N - 1); }
+
+// one record per own boundary vertex with a cross-rank link: per slot, the cross-rank
+// neighbour (distance 1, edge key), or the rank-local result of the reduced scan (an end
+// marker, or the next exit vertex of this rank with the distance and min key to it)
+template <bool MIN>
+__global__ void k_exit_records(ForestArgs a, const int32_t* list, const int* count, ExitRec* rec, int* rcount) {
+    const int cnt = *count;
+    const int stride = gridDim.x * blockDim.x;
+    for (int base = blockIdx.x * blockDim.x + (threadIdx.x & ~31); base < cnt; base += stride) {
+        const int idx = base + (threadIdx.x & 31);
+        bool take = false;
+        ExitRec r;
+        if (idx < cnt) {
+            const int32_t v = list[idx];
+            const int2 nb = MIN ? a.pi2[v] : a.forest[v];
+            const bool f0 = nb.x >= 0 && is_foreign(nb.x, a), f1 = nb.y >= 0 && is_foreign(nb.y, a);
+            take = f0 || f1;
+            if (take) {
+                r.g = v;
+                r.pad = 0;
+                const int2 raw = a.end2[v];
+                int32_t q[2], d[2];
+                uint64_t k[2];
+#pragma unroll
+                for (int i = 0; i < 2; i++) {
+                    const int32_t x = i ? nb.y : nb.x;
+                    const bool fx = i ? f1 : f0;
+                    d[i] = 0;
+                    k[i] = KEY_INF;
+                    if (x < 0) q[i] = -(v + 1);
+                    else if (fx) {
+                        q[i] = x;
+                        d[i] = 1;
+                        if (MIN) k[i] = i ? a.ekb[v].y : a.ekb[v].x;
+                    } else {
+                        const int32_t m = i ? raw.y : raw.x;
+                        q[i] = is_exit_marker(m, a.N) ? exit_vertex(m, a.N) : m;
+                        if (MIN) k[i] = i ? a.kraw[v].y : a.kraw[v].x;
+                        else d[i] = i ? a.dist2[v].y : a.dist2[v].x;
+                    }
+                }
+                r.q0 = q[0]; r.q1 = q[1];
+                r.d0 = d[0]; r.d1 = d[1];
+                r.k0 = k[0]; r.k1 = k[1];
+            }
+        }
+        const unsigned m = __ballot_sync(0xffffffffu, take);
+        const int lane = threadIdx.x & 31;
+        int pos = 0;
+        if (lane == 0 && m) pos = atomicAdd(rcount, __popc(m));
+        pos = __shfl_sync(0xffffffffu, pos, 0);
+        if (take) rec[pos + __popc(m & ((1u << lane) - 1u))] = r;
+    }
+}
+
+// the exit graph from the gathered records of all ranks (padding has g = -1)
+template <bool MIN>
+__global__ void k_exit_build(const ExitRec* rec, int64_t total, int2** gq, ulonglong2** gk, int2** gr,
+                             int32_t* glist, int* gcount) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const ExitRec r = rec[i];
+        if (r.g < 0) continue;
+        const int2 q = make_int2(r.q0, r.q1);
+        gq[0][r.g] = q;
+        gq[1][r.g] = q;
+        if (MIN) {
+            const ulonglong2 k = make_ulonglong2(r.k0, r.k1);
+            gk[0][r.g] = k;
+            gk[1][r.g] = k;
+        } else {
+            const int2 d = make_int2(r.d0, r.d1);
+            gr[0][r.g] = d;
+            gr[1][r.g] = d;
+        }
+        glist[atomicAdd(gcount, 1)] = r.g;
+    }
+}
+
+// exit marker at t -> the global result of t through its cross-rank slot
+template <bool MIN>
+__global__ void k_exit_fold(ForestArgs a, const int32_t* list, const int* count, const uint64_t* gcyc,
+                            const int2* gend, const int2* gdist) {
+    const int cnt = *count;
+    for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < cnt; idx += gridDim.x * blockDim.x) {
+        const int32_t b = list[idx];
+        int2 raw = a.end2[b];
+        int2 dd = MIN ? make_int2(0, 0) : a.dist2[b];
+#pragma unroll
+        for (int i = 0; i < 2; i++) {
+            const int32_t m = i ? raw.y : raw.x;
+            if (!is_exit_marker(m, a.N)) continue;
+            const int32_t t = exit_vertex(m, a.N);
+            if (MIN) {
+                if (gcyc[t] != KEY_INF) a.cyc_k[b] = gcyc[t];
+            } else {
+                const int2 nt = a.forest[t];
+                const int so = (t == b) ? i : ((nt.x >= 0 && is_foreign(nt.x, a)) ? 0 : 1);
+                const int32_t e = so ? gend[t].y : gend[t].x;
+                const int32_t dg = so ? gdist[t].y : gdist[t].x;
+                if (i) { raw.y = e; dd.y += dg; } else { raw.x = e; dd.x += dg; }
+            }
+        }
+        if (!MIN) {
+            a.end2[b] = raw;
+            a.dist2[b] = dd;
+        }
+    }
+}
+
+// rank totals -> this rank's base offset; tot[G] = base, tot[G+1] = own total
+__global__ void k_rank_base(int64_t* tot, int G, int rank) {
+    if (threadIdx.x == 0) {
+        int64_t b = 0;
+        for (int q = 0; q < rank; q++) b += tot[q];
+        tot[G] = b;
+    }
+}
+
+__global__ void k_own_total(const int32_t* len, const int32_t* off, int64_t n_own, int64_t* out) {
+    if (threadIdx.x == 0) *out = n_own > 0 ? (int64_t)off[n_own - 1] + len[n_own - 1] : 0;
+}
+
+// global offsets of the cross-rank paths whose ID vertex this rank owns
+__global__ void k_publish(const int32_t* glist, const int* gcount, const int2* gend, int64_t lo, int64_t hi,
+                          const int32_t* off_own /* indexed by global id */, const int64_t* tot, int G,
+                          int2* pub, int* pcount) {
+    const int cnt = *gcount;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
+        const int32_t g = glist[i];
+        if (g < lo || g >= hi) continue;  // each path with an own ID has an own exit vertex
+        const int2 e = gend[g];
+        const int32_t e0 = -(e.x + 1), e1 = -(e.y + 1);
+        const int32_t l = e0 < e1 ? e0 : e1;
+        if (l >= lo && l < hi) pub[atomicAdd(pcount, 1)] = make_int2(l, (int32_t)(tot[G] + off_own[l]));
+    }
+}
+
+__global__ void k_pub_apply(const int2* pub, int64_t total, int32_t* offG) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const int2 p = pub[i];
+        if (p.x >= 0) offG[p.x] = p.y;
+    }
+}
+
+__global__ void k_perm_part(int64_t lo, int64_t hi, const int32_t* path_id, const int32_t* pos, const int32_t* off,
+                            const int32_t* offG, const int64_t* tot, int G, int32_t* iperm) {
+    const int64_t base = tot[G];
+    for (int64_t v = lo + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < hi; v += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t l = path_id[v];
+        const int64_t o = (l >= lo && l < hi) ? base + off[l] : (int64_t)offG[l];
+        iperm[v] = (int32_t)(o + pos[v] - 1);
+    }
+}
+
+// the global exit-graph scan (same kernel as the reduced scan, on global-id buffers)
+template <bool MIN>
+static int exit_pass(const ForestArgs& a, const int32_t* list, const int* count, const ForestPartCtx& pc,
+                     int64_t N, cudaStream_t s) {
+    ExitRec* send = (ExitRec*)pc.rec_send;
+    ExitRec* all = (ExitRec*)pc.rec_all;
+    LF_CUDA(cudaMemsetAsync(send, 0xff, sizeof(ExitRec) * pc.exit_cap, s));
+    LF_CUDA(cudaMemsetAsync(pc.gctl, 0, sizeof(int) * 256, s));
+    {
+        LF_PROF(MIN ? "exit_records_cycles" : "exit_records_ranks", -1, s);
+        k_exit_records<MIN><<<persistent_grid((const void*)k_exit_records<MIN>, 256), 256, 0, s>>>(
+            a, list, count, send, pc.gctl + 250);
+        LF_CUDA(cudaGetLastError());
+    }
+    int rc = pc.allgather(pc.ctx, send, all, sizeof(ExitRec) * pc.exit_cap, s);
+    if (rc) return rc;
+    int2** dq = nullptr;
+    ulonglong2** dk = nullptr;
+    int2** dr = nullptr;
+    // pointer tables (small) for the build kernel
+    void* tabs = nullptr;
+    LF_CUDA(cudaMallocAsync(&tabs, sizeof(void*) * 6, s));
+    void* h[6] = {pc.gq[0], pc.gq[1], pc.gk[0], pc.gk[1], pc.gr[0], pc.gr[1]};
+    LF_CUDA(cudaMemcpyAsync(tabs, h, sizeof(h), cudaMemcpyHostToDevice, s));
+    dq = (int2**)tabs;
+    dk = (ulonglong2**)((void**)tabs + 2);
+    dr = (int2**)((void**)tabs + 4);
+    const int64_t total = (int64_t)pc.G * pc.exit_cap;
+    const int kBuildCnt = MIN ? kCtlCnt1 : kCtlCnt2;
+    k_exit_build<MIN><<<persistent_grid((const void*)k_exit_build<MIN>, 256), 256, 0, s>>>(
+        all, total, dq, dk, dr, pc.glist, pc.gctl + kBuildCnt);
+    LF_CUDA(cudaGetLastError());
+    LF_CUDA(cudaFreeAsync(tabs, s));
+    ForestArgs g;
+    memset(&g, 0, sizeof(g));
+    g.N = N;
+    g.lo = 0;
+    g.hi = N;
+    for (int i = 0; i < 2; i++) {
+        g.rq1[i] = pc.gq[i];
+        g.rk1[i] = pc.gk[i];
+        g.rq2[i] = pc.gq[i];
+        g.rr2[i] = pc.gr[i];
+    }
+    g.list1 = pc.glist;
+    g.list2 = pc.glist;
+    g.ctl = pc.gctl;
+    g.cyc_k = pc.gcyc;
+    g.end2 = pc.gend;
+    g.dist2 = pc.gdist;
+    g.max_steps = a.max_steps;
+    {
+        LF_PROF(MIN ? "exit_scan_cycles" : "exit_scan_ranks", -1, s);
+        rc = coop_launch(k_red_scan<MIN>, RT, g, s, sizeof(RedSmem));
+        if (rc) return rc;
+    }
+    {
+        LF_PROF(MIN ? "exit_fold_cycles" : "exit_fold_ranks", -1, s);
+        k_exit_fold<MIN><<<persistent_grid((const void*)k_exit_fold<MIN>, 256), 256, 0, s>>>(
+            a, list, count, pc.gcyc, pc.gend, pc.gdist);
+        LF_CUDA(cudaGetLastError());
+    }
+    return LF_OK;
+}
+
+int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
+                    int32_t* pos, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
+                    const ForestPartCtx& pc, cudaStream_t s) {
+    const int64_t lo = pc.lo, hi = pc.hi, n_own = hi - lo;
+    int rc = forest_prepare();
+    if (rc) return rc;
+    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
+    LF_CUDA(cudaMemsetAsync(pc.tot, 0, sizeof(int64_t) * (pc.G + 2), s));
+    ForestArgs a;
+    memset(&a, 0, sizeof(a));
+    a.N = N;
+    a.lo = lo;
+    a.hi = hi;
+    // own-slice buffers, offset so that vertex g is element g
+    a.pi2 = (const int2*)pi2 - lo;
+    a.pi2_w = (const float2*)pi2_w - lo;
+    a.forest = (int2*)forest - lo;
+    for (int i = 0; i < 2; i++) {
+        a.rq1[i] = w.rq1[i] - lo;
+        a.rk1[i] = w.rk1[i] - lo;
+        a.rq2[i] = w.rq2[i] - lo;
+        a.rr2[i] = w.rr2[i] - lo;
+    }
+    a.cyc_k = w.cyc_k - lo;
+    a.loc1 = w.loc1 - lo;
+    a.kst = w.kst - lo;
+    a.loc2 = w.loc2 - lo;
+    a.end2 = w.end2 - lo;
+    a.dist2 = w.dist2 - lo;
+    a.kraw = w.kraw - lo;
+    a.ekb = w.ekb - lo;
+    a.list1 = w.list1;
+    a.list2 = w.list2;
+    a.ctl = w.ctl;
+    a.path_id = path_id - lo;
+    a.pos = pos - lo;
+    a.len = w.len - lo;
+    a.n_cycles = (unsigned long long*)&pc.tot[pc.G + 1];
+    a.ghost_list = pc.ghost_list;
+    a.n_ghost = pc.n_ghost;
+    a.ghost_below = pc.ghost_below;
+    a.ghost_nb = pc.ghost_nb;
+    a.max_steps = max_steps_for(N) < kMaxSteps ? max_steps_for(N) : kMaxSteps;
+    const int tiles = (int)((n_own + LB - 1) / LB);
+    const int smem = (int)sizeof(TileSmem);
+    if (tiles > 0) {
+        LF_PROF("lf_local1", -1, s);
+        k_lf_local1<<<tiles, LT, smem, s>>>(a);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("red_scan_cycles", -1, s);
+        rc = coop_launch(k_red_scan<true>, RT, a, s, sizeof(RedSmem));
+        if (rc) return rc;
+    }
+    rc = exit_pass<true>(a, w.list1, w.ctl + kCtlCnt1, pc, N, s);
+    if (rc) return rc;
+    if (tiles > 0) {
+        LF_PROF("lf_local2", -1, s);
+        k_lf_local2<<<tiles, LT, smem, s>>>(a);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("red_scan_ranks", -1, s);
+        rc = coop_launch(k_red_scan<false>, RT, a, s, sizeof(RedSmem));
+        if (rc) return rc;
+    }
+    rc = exit_pass<false>(a, w.list2, w.ctl + kCtlCnt2, pc, N, s);
+    if (rc) return rc;
+    if (tiles > 0) {
+        LF_PROF("lf_local3", -1, s);
+        k_lf_local3<<<tiles, LT, smem, s>>>(a);
+        LF_CUDA(cudaGetLastError());
+    }
+    // path offsets: own exclusive scan, rank bases, published offsets of cross-rank paths
+    {
+        LF_PROF("path_offsets", -1, s);
+        if (n_own > 0) {
+            size_t tb = w.scan_tmp_bytes;
+            LF_CUDA(cub::DeviceScan::ExclusiveSum(w.scan_tmp, tb, w.len, w.off, (int)n_own, s));
+        }
+        k_own_total<<<1, 32, 0, s>>>(w.len, w.off, n_own, &pc.tot[pc.rank]);
+        rc = pc.allreduce_i64(pc.ctx, pc.tot, pc.G, s);  // every rank's slot is filled by its owner
+        if (rc) return rc;
+        k_rank_base<<<1, 32, 0, s>>>(pc.tot, pc.G, pc.rank);
+        LF_CUDA(cudaMemsetAsync(pc.pub_send, 0xff, sizeof(int2) * pc.exit_cap, s));
+        k_publish<<<persistent_grid((const void*)k_publish, 256), 256, 0, s>>>(
+            pc.glist, pc.gctl + kCtlCnt2, pc.gend, lo, hi, w.off - lo, pc.tot, pc.G, pc.pub_send, pc.gctl + 251);
+        LF_CUDA(cudaGetLastError());
+        rc = pc.allgather(pc.ctx, pc.pub_send, pc.pub_all, sizeof(int2) * pc.exit_cap, s);
+        if (rc) return rc;
+        k_pub_apply<<<persistent_grid((const void*)k_pub_apply, 256), 256, 0, s>>>(pc.pub_all, (int64_t)pc.G * pc.exit_cap,
+                                                                               pc.offG);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("perm", -1, s);
+        k_perm_part<<<persistent_grid((const void*)k_perm_part, 256), 256, 0, s>>>(lo, hi, path_id - lo, pos - lo,
+                                                                               w.off - lo, pc.offG, pc.tot, pc.G,
+                                                                               iperm - lo);
+        LF_CUDA(cudaGetLastError());
+    }
+    if (n_cycles) {
+        rc = pc.allreduce_i64(pc.ctx, &pc.tot[pc.G + 1], 1, s);
+        if (rc) return rc;
+        LF_CUDA(cudaMemcpyAsync(n_cycles, &pc.tot[pc.G + 1], sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+    }
     return LF_OK;
 }
 

@@ -102,8 +102,46 @@ struct ForestWs {
     int* ctl;              // [256] per-step counters, list sizes
     void* scan_tmp;        // CUB temp storage
     size_t scan_tmp_bytes;
+    ulonglong2* kraw;      // [N] per-direction min keys after the cycle pass (boundary)
+    ulonglong2* ekb;       // [N] slot keys of boundary vertices
 };
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w);
+
+// Partitioned linear forest: this rank's rows [lo, hi) of the factor;
+// paths and cycles that cross ranks are resolved through an exchanged list of "exit"
+// records (boundary vertices with a cross-rank forest link).  Buffers sized by the
+// global N are indexed by global vertex id; `exit_cap` bounds any rank's exit records.
+struct ForestPartCtx {
+    int64_t lo, hi;
+    int G, rank;
+    const int32_t* ghost_list;   // sorted global ids of ghost vertices
+    int64_t n_ghost, ghost_below;
+    const int2* ghost_nb;        // [local id] factor slots (global ids) of ghosts
+    int64_t exit_cap;
+    // global buffers
+    int2* gq[2];
+    ulonglong2* gk[2];
+    int2* gr[2];
+    uint64_t* gcyc;
+    int2* gend;
+    int2* gdist;
+    int32_t* glist;              // [G * exit_cap]
+    int* gctl;                   // [256]
+    void* rec_send;              // [exit_cap] records
+    void* rec_all;               // [G * exit_cap] records
+    int2* pub_send;              // [exit_cap] (path id, global offset)
+    int2* pub_all;               // [G * exit_cap]
+    int32_t* offG;               // [N] global offsets of cross-rank path ids
+    int64_t* tot;                // [G + 2] per-rank path-length totals, base, cycles
+    void* ctx;
+    int (*allgather)(void* ctx, const void* send, void* recv, size_t bytes_per_rank, cudaStream_t s);
+    int (*allreduce_i64)(void* ctx, int64_t* buf, int count, cudaStream_t s);
+};
+size_t exit_record_bytes();
+
+int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
+                    int32_t* pos, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
+                    const ForestPartCtx& pc, cudaStream_t s);
 
 int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
                int32_t* pos, int32_t* perm, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,

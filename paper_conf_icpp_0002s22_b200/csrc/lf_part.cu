@@ -106,6 +106,23 @@ struct Part {
     std::vector<int64_t> peer_lo, peer_hi, peer_nb;
     int64_t send_total = 0;
     bool plan_checked = false;
+    int32_t* ghost_list = nullptr;  // sorted global ids of ghosts
+    int64_t n_ghost = 0;
+    std::vector<int64_t> peer_send_total;
+    // linear forest
+    int32_t* pi2g = nullptr;     // [n_own*2] own factor slots, global ids (n = 2)
+    float* pi2w = nullptr;
+    float* pi2v = nullptr;
+    float* pdiag = nullptr;
+    int2* ghost_pi = nullptr;    // [NL] factor slots of ghosts (global ids)
+    int32_t* ghost_iperm = nullptr;
+    int32_t *forest = nullptr, *path_id = nullptr, *pos = nullptr, *iperm = nullptr;
+    int64_t* n_cycles = nullptr;
+    void* lws = nullptr;
+    size_t lws_bytes = 0;
+    ForestWs lw;
+    ForestPartCtx fpc;
+    bool lf_ready = false;
     // run
     Comm* comm = nullptr;
     FactorWs fws;
@@ -272,9 +289,11 @@ static int check_plan(Part* p) {
     Comm* c = p->comm;
     if (p->plan_checked) return LF_OK;
     if (c->kind == 1) {
+        p->peer_send_total.assign(p->G, 0);
         for (int q = 0; q < p->G; q++) {
-            if (q == p->rank) continue;
             Part* o = c->parts[q];
+            p->peer_send_total[q] = o->send_total;
+            if (q == p->rank) continue;
             if (p->send_cnt[q] != o->recv_cnt[p->rank])
                 return set_error(LF_EINPUT, "partition plan mismatch: A is not pattern-symmetric");
             p->peer_nb[q] = o->nb;
@@ -293,7 +312,9 @@ static int check_plan(Part* p) {
         LF_CUDA(cudaMemcpy(all.data(), dall, sizeof(int64_t) * all.size(), cudaMemcpyDeviceToHost));
         cudaFree(dsend);
         cudaFree(dall);
+        p->peer_send_total.assign(G, 0);
         for (int q = 0; q < G; q++) {
+            for (int r = 0; r < G; r++) p->peer_send_total[q] += all[(size_t)q * (G + 1) + r];
             p->peer_nb[q] = all[(size_t)q * (G + 1) + G];
             if (q != p->rank && all[(size_t)q * (G + 1) + p->rank] != p->recv_cnt[q])
                 return set_error(LF_EINPUT, "partition plan mismatch: A is not pattern-symmetric");
@@ -430,6 +451,265 @@ __global__ void k_export(int64_t n_own, int n, int64_t nb, const int32_t* __rest
     }
 }
 
+
+// ---------------------------------------------------------------------------
+// partitioned linear forest
+// ---------------------------------------------------------------------------
+__global__ void k_pack_pi(int64_t cnt, const int32_t* __restrict__ idx, int64_t nb, const int2* __restrict__ pi2g,
+                          int2* out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = pi2g[idx[i] - nb];
+}
+
+__global__ void k_pack_i32(int64_t cnt, const int32_t* __restrict__ idx, int64_t nb, const int32_t* __restrict__ own,
+                           int32_t* out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = own[idx[i] - nb];
+}
+
+__global__ void k_sum_parts_i64(int P, int count, int64_t** bufs) {
+    for (int i = threadIdx.x; i < count; i += blockDim.x) {
+        int64_t t = 0;
+        for (int p = 0; p < P; p++) t += bufs[p][i];
+        for (int p = 0; p < P; p++) bufs[p][i] = t;
+    }
+}
+
+static int cb_allgather(void* ctx, const void* send, void* recv, size_t bytes, cudaStream_t s) {
+    Part* p = (Part*)ctx;
+    Comm* c = p->comm;
+    if (c->kind == 0) {
+        LF_NCCL(ncclAllGather(send, recv, bytes, ncclUint8, c->nccl, s));
+        return LF_OK;
+    }
+    // loopback: every partition's send buffer is at the same place in its own context;
+    // copy all of them into this partition's receive buffer (ordering by barriers)
+    if (!c->bar.wait()) return set_error(LF_ECUDA, "loopback allgather aborted");
+    const bool is_rec = send == p->fpc.rec_send;  // exit records, or published offsets
+    if (!is_rec && send != (const void*)p->fpc.pub_send)
+        return set_error(LF_EINVAL, "loopback allgather: unknown buffer");
+    for (int q = 0; q < p->G; q++) {
+        Part* o = c->parts[q];
+        const void* src = is_rec ? o->fpc.rec_send : (const void*)o->fpc.pub_send;
+        LF_CUDA(cudaMemcpyAsync((char*)recv + (size_t)q * bytes, src, bytes, cudaMemcpyDeviceToDevice, s));
+    }
+    if (!c->bar.wait()) return set_error(LF_ECUDA, "loopback allgather aborted");
+    return LF_OK;
+}
+
+static int cb_allreduce_i64(void* ctx, int64_t* buf, int count, cudaStream_t s) {
+    Part* p = (Part*)ctx;
+    Comm* c = p->comm;
+    if (c->kind == 0) {
+        LF_NCCL(ncclAllReduce(buf, buf, count, ncclInt64, ncclSum, c->nccl, s));
+        return LF_OK;
+    }
+    if (!c->bar.wait()) return set_error(LF_ECUDA, "loopback allreduce aborted");
+    if (p->rank == 0) {
+        const int P = (int)c->parts.size();
+        const size_t off = buf - p->fpc.tot;
+        std::vector<int64_t*> b(P);
+        for (int q = 0; q < P; q++) b[q] = c->parts[q]->fpc.tot + off;
+        int64_t** db = nullptr;
+        LF_CUDA(cudaMallocAsync(&db, sizeof(void*) * P, s));
+        LF_CUDA(cudaMemcpyAsync(db, b.data(), sizeof(void*) * P, cudaMemcpyHostToDevice, s));
+        k_sum_parts_i64<<<1, 64, 0, s>>>(P, count, db);
+        LF_CUDA(cudaGetLastError());
+        LF_CUDA(cudaFreeAsync(db, s));
+        LF_CUDA(cudaStreamSynchronize(s));
+    }
+    if (!c->bar.wait()) return set_error(LF_ECUDA, "loopback allreduce aborted");
+    return LF_OK;
+}
+
+static int lf_setup(Part* p, cudaStream_t s) {
+    if (p->lf_ready) return LF_OK;
+    if (p->n != 2) return set_error(LF_EINVAL, "partitioned linear forest needs n = 2");
+    const int64_t no = p->n_own > 0 ? p->n_own : 1;
+    int rc;
+#define TRYL(x) do { rc = (x); if (rc) return rc; } while (0)
+    TRYL(dalloc(p, &p->pi2g, (size_t)no * 2, s));
+    TRYL(dalloc(p, &p->pi2w, (size_t)no * 2, s));
+    TRYL(dalloc(p, &p->pi2v, (size_t)no * 2, s));
+    TRYL(dalloc(p, &p->pdiag, (size_t)no, s));
+    TRYL(dalloc(p, &p->ghost_pi, (size_t)p->NL, s));
+    TRYL(dalloc(p, &p->ghost_iperm, (size_t)p->NL, s));
+    TRYL(dalloc(p, &p->forest, (size_t)no * 2, s));
+    TRYL(dalloc(p, &p->path_id, (size_t)no, s));
+    TRYL(dalloc(p, &p->pos, (size_t)no, s));
+    TRYL(dalloc(p, &p->iperm, (size_t)no, s));
+    TRYL(dalloc(p, &p->n_cycles, 1, s));
+    {
+        Carve c(nullptr, 0);
+        p->lws_bytes = forest_ws_carve(c, no, nullptr) + 256;
+        char* w = nullptr;
+        TRYL(dalloc(p, &w, p->lws_bytes, s));
+        p->lws = w;
+        Carve c2(p->lws, p->lws_bytes);
+        forest_ws_carve(c2, no, &p->lw);
+    }
+    ForestPartCtx& f = p->fpc;
+    memset(&f, 0, sizeof(f));
+    f.lo = p->lo;
+    f.hi = p->hi;
+    f.G = p->G;
+    f.rank = p->rank;
+    f.ghost_list = p->ghost_list;
+    f.n_ghost = p->n_ghost;
+    f.ghost_below = p->nb;
+    f.ghost_nb = p->ghost_pi;
+    int64_t cap = 1;
+    for (int q = 0; q < p->G; q++) cap = p->peer_send_total[q] > cap ? p->peer_send_total[q] : cap;
+    f.exit_cap = cap;
+    const size_t N = (size_t)p->N + 1;
+    for (int i = 0; i < 2; i++) {
+        TRYL(dalloc(p, &f.gq[i], N, s));
+        TRYL(dalloc(p, &f.gk[i], N, s));
+        TRYL(dalloc(p, &f.gr[i], N, s));
+    }
+    TRYL(dalloc(p, &f.gcyc, N, s));
+    TRYL(dalloc(p, &f.gend, N, s));
+    TRYL(dalloc(p, &f.gdist, N, s));
+    TRYL(dalloc(p, &f.glist, (size_t)p->G * cap, s));
+    TRYL(dalloc(p, &f.gctl, 256, s));
+    char* rs = nullptr;
+    TRYL(dalloc(p, &rs, exit_record_bytes() * cap, s));
+    f.rec_send = rs;
+    char* ra = nullptr;
+    TRYL(dalloc(p, &ra, exit_record_bytes() * cap * p->G, s));
+    f.rec_all = ra;
+    TRYL(dalloc(p, &f.pub_send, (size_t)cap, s));
+    TRYL(dalloc(p, &f.pub_all, (size_t)cap * p->G, s));
+    TRYL(dalloc(p, &f.offG, N, s));
+    TRYL(dalloc(p, &f.tot, (size_t)p->G + 2, s));
+    f.ctx = p;
+    f.allgather = cb_allgather;
+    f.allreduce_i64 = cb_allreduce_i64;
+#undef TRYL
+    p->lf_ready = true;
+    return LF_OK;
+}
+
+static int run_forest(Part* p, cudaStream_t s) {
+    int rc = check_plan(p);
+    if (rc) return rc;
+    rc = lf_setup(p, s);
+    if (rc) return rc;
+    // own factor with global ids, and the factor slots of ghost vertices (halo)
+    if (p->n_own > 0) {
+        k_export<<<persistent_grid((const void*)k_export, 256), 256, 0, s>>>(p->n_own, 2, p->nb, p->pi, p->pi_w,
+                                                                           p->pi_val, p->diag, p->l2g, p->pi2g,
+                                                                           p->pi2w, p->pi2v, p->pdiag);
+        LF_CUDA(cudaGetLastError());
+    }
+    if (p->send_total) {
+        k_pack_pi<<<persistent_grid((const void*)k_pack_pi, 256), 256, 0, s>>>(p->send_total, p->send_idx, p->nb,
+                                                                           (const int2*)p->pi2g, (int2*)p->sbuf);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("halo_pi", -1, s);
+        rc = exchange(p, (unsigned char*)p->ghost_pi, sizeof(int2), s);
+        if (rc) return rc;
+    }
+    return forest_part_run(p->N, p->pi2g, p->pi2w, p->forest, p->path_id, p->pos, p->iperm, p->n_cycles, p->lw,
+                           p->fpc, s);
+}
+
+// tridiagonal coefficients of the own vertices (row iperm[v]); foreign neighbours' rows
+// come from a halo exchange of iperm
+__global__ void k_part_tridiag(int64_t lo, int64_t hi, const int2* __restrict__ forest, const int32_t* __restrict__ iperm,
+                               const int2* __restrict__ pi2g, const float2* __restrict__ pi2v,
+                               const float* __restrict__ diag, const int32_t* __restrict__ ghost_list, int64_t ng,
+                               int64_t nbelow, const int32_t* __restrict__ ghost_iperm, float* a, float* b, float* c) {
+    for (int64_t v = lo + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < hi; v += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = v - lo;
+        const int32_t r = iperm[i];
+        const int2 f = forest[i];
+        const int2 pn = pi2g[i];
+        const float2 pv = pi2v[i];
+        float ar = 0.0f, cr = 0.0f;
+#pragma unroll
+        for (int k = 0; k < 2; k++) {
+            const int32_t w = k ? f.y : f.x;
+            if (w < 0) continue;
+            const float x = (pn.x == w) ? pv.x : pv.y;
+            int32_t rw;
+            if (w >= lo && w < hi) rw = iperm[w - lo];
+            else {
+                int64_t l = 0, h = ng;
+                while (l < h) {
+                    const int64_t m = (l + h) >> 1;
+                    if (ghost_list[m] < w) l = m + 1; else h = m;
+                }
+                rw = ghost_iperm[l < nbelow ? l : l + (hi - lo)];
+            }
+            if (rw == r - 1) ar = x;
+            else if (rw == r + 1) cr = x;
+        }
+        a[i] = ar;
+        b[i] = diag[i];
+        c[i] = cr;
+    }
+}
+
+static int run_tridiag(Part* p, float* a, float* b, float* c, cudaStream_t s) {
+    if (!p->lf_ready) return set_error(LF_EINVAL, "lf_part_tridiag: run lf_part_linear_forest first");
+    if (p->send_total) {
+        k_pack_i32<<<persistent_grid((const void*)k_pack_i32, 256), 256, 0, s>>>(p->send_total, p->send_idx, p->nb,
+                                                                             p->iperm, (int32_t*)p->sbuf);
+        LF_CUDA(cudaGetLastError());
+    }
+    int rc = exchange(p, (unsigned char*)p->ghost_iperm, sizeof(int32_t), s);
+    if (rc) return rc;
+    if (p->n_own > 0) {
+        LF_PROF("tridiag", -1, s);
+        k_part_tridiag<<<persistent_grid((const void*)k_part_tridiag, 256), 256, 0, s>>>(
+            p->lo, p->hi, (const int2*)p->forest, p->iperm, (const int2*)p->pi2g, (const float2*)p->pi2v, p->pdiag,
+            p->ghost_list, p->n_ghost, p->nb, p->ghost_iperm, a, b, c);
+        LF_CUDA(cudaGetLastError());
+    }
+    return LF_OK;
+}
+
+// run fn on every partition of this process (loopback: lockstep threads)
+template <class F>
+static int for_parts(void** parts, int nparts, Comm* c, F fn) {
+    if (c->kind == 0) {
+        Part* p = (Part*)parts[0];
+        p->comm = c;
+        return fn(p);
+    }
+    c->parts.assign(nparts, nullptr);
+    for (int i = 0; i < nparts; i++) {
+        Part* p = (Part*)parts[i];
+        c->parts[p->rank] = p;
+        p->comm = c;
+    }
+    c->bar.n = nparts;
+    c->bar.aborted = false;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::vector<int> rcs(nparts, 0);
+    std::vector<std::string> errs(nparts);
+    std::vector<std::thread> th;
+    for (int i = 0; i < nparts; i++) {
+        th.emplace_back([&, i] {
+            cudaSetDevice(dev);
+            const int rc = fn(c->parts[i]);
+            if (rc) {
+                errs[i] = lf_last_error();
+                c->bar.abort();
+            }
+            rcs[i] = rc;
+        });
+    }
+    for (auto& t : th) t.join();
+    for (int i = 0; i < nparts; i++)
+        if (rcs[i]) return set_error(rcs[i], errs[i].c_str());
+    return LF_OK;
+}
+
 }  // namespace lf
 
 using namespace lf;
@@ -544,7 +824,9 @@ int lf_part_create(int G, const int64_t* bounds, int rank, const lf_csr_t* A, in
     TRY(set_cuda_rc(cudaMemcpyAsync(&ng32, wpre + W, sizeof(int32_t), cudaMemcpyDeviceToHost, s), "copy"));
     TRY(set_cuda_rc(cudaStreamSynchronize(s), "sync"));
     const int64_t ng = ng32;
-    TRY(set_cuda_rc(cudaMallocAsync(&ghost, sizeof(int32_t) * (ng + 1), s), "alloc"));
+    TRY(dalloc(p, &ghost, (size_t)(ng + 1), s));
+    p->ghost_list = ghost;
+    p->n_ghost = ng;
     k_ghost_list<<<grid, 256, 0, s>>>(W + 1, bits, wpre, ghost);
     k_ghost_bounds<<<1, 128, 0, s>>>(ghost, ng, dbounds, G, gb);
     std::vector<int64_t> hgb(G + 1);
@@ -618,7 +900,6 @@ int lf_part_create(int G, const int64_t* bounds, int rank, const lf_csr_t* A, in
     cudaFreeAsync(bits, s);
     cudaFreeAsync(pc, s);
     cudaFreeAsync(wpre, s);
-    cudaFreeAsync(ghost, s);
     cudaFreeAsync(dbounds, s);
     cudaFreeAsync(gb, s);
     TRY(set_cuda_rc(cudaGetLastError(), "setup kernels"));
@@ -704,6 +985,47 @@ int lf_part_export(void* part, int32_t* pi, float* pi_w, float* pi_val, float* d
     }
     if (rounds) LF_CUDA(cudaMemcpyAsync(rounds, p->rounds, sizeof(int32_t), cudaMemcpyDeviceToDevice, s));
     if (live) LF_CUDA(cudaMemcpyAsync(live, p->live, sizeof(int64_t) * 2 * p->M, cudaMemcpyDeviceToDevice, s));
+    return LF_OK;
+}
+
+
+int lf_part_linear_forest(void** parts, int nparts, void* comm, void* stream) {
+    g_err_clear();
+    Comm* c = (Comm*)comm;
+    if (!parts || nparts < 1 || !c) return set_error(LF_EINVAL, "lf_part_linear_forest: bad arguments");
+    if (c->kind == 1 && nparts != ((Part*)parts[0])->G)
+        return set_error(LF_EINVAL, "lf_part_linear_forest: loopback needs all partitions");
+    cudaStream_t s = (cudaStream_t)stream;
+    return for_parts(parts, nparts, c, [&](Part* p) { return run_forest(p, s); });
+}
+
+int lf_part_tridiag(void** parts, int nparts, void* comm, float* const* a, float* const* b, float* const* cc,
+                    void* stream) {
+    g_err_clear();
+    Comm* c = (Comm*)comm;
+    if (!parts || nparts < 1 || !c || !a || !b || !cc) return set_error(LF_EINVAL, "lf_part_tridiag: bad arguments");
+    cudaStream_t s = (cudaStream_t)stream;
+    // outputs are given per partition in the order of `parts`
+    std::vector<Part*> order(nparts);
+    for (int i = 0; i < nparts; i++) order[i] = (Part*)parts[i];
+    return for_parts(parts, nparts, c, [&](Part* p) {
+        int i = 0;
+        while (order[i] != p) i++;
+        return run_tridiag(p, a[i], b[i], cc[i], s);
+    });
+}
+
+int lf_part_forest_export(void* part, int32_t* forest, int32_t* path_id, int32_t* pos, int32_t* iperm,
+                          int64_t* n_cycles, void* stream) {
+    Part* p = (Part*)part;
+    if (!p || !p->lf_ready) return set_error(LF_EINVAL, "lf_part_forest_export: no linear forest yet");
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t n = (size_t)p->n_own;
+    if (forest) LF_CUDA(cudaMemcpyAsync(forest, p->forest, sizeof(int32_t) * 2 * n, cudaMemcpyDeviceToDevice, s));
+    if (path_id) LF_CUDA(cudaMemcpyAsync(path_id, p->path_id, sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
+    if (pos) LF_CUDA(cudaMemcpyAsync(pos, p->pos, sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
+    if (iperm) LF_CUDA(cudaMemcpyAsync(iperm, p->iperm, sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, s));
+    if (n_cycles) LF_CUDA(cudaMemcpyAsync(n_cycles, p->n_cycles, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
     return LF_OK;
 }
 

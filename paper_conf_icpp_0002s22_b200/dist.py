@@ -168,6 +168,19 @@ class Partition:
                                              p(out["live"]) if M > 0 else None, _lf._stream()))
         return out
 
+    def forest_export(self):
+        t = self.torch
+        n = self.n_own
+        out = dict(forest=t.empty((n, 2), dtype=t.int32, device="cuda"),
+                   path_id=t.empty(n, dtype=t.int32, device="cuda"),
+                   pos=t.empty(n, dtype=t.int32, device="cuda"),
+                   iperm=t.empty(n, dtype=t.int32, device="cuda"),
+                   n_cycles=t.zeros(1, dtype=t.int64, device="cuda"))
+        p = _lf._ptr
+        _lf._check(_lf.load().lf_part_forest_export(self.h, p(out["forest"]), p(out["path_id"]), p(out["pos"]),
+                                                    p(out["iperm"]), p(out["n_cycles"]), _lf._stream()))
+        return out
+
     def close(self):
         if self.h:
             _lf.load().lf_part_destroy(self.h, _lf._stream())
@@ -180,3 +193,24 @@ def factor(parts, comm, *, M=5, m=5, k_m=0, p=0.5, seed=0):
     arr = (C.c_void_p * len(parts))(*[q.h for q in parts])
     o = _lf.opts(M, m, k_m, p, seed)
     _lf._check(L.lf_part_factor(arr, len(parts), comm.h, C.byref(o), _lf._stream()))
+
+
+def linear_forest(parts, comm):
+    """lf_part_linear_forest over the partitions of this process (after factor, n = 2)."""
+    L = _lf.load()
+    arr = (C.c_void_p * len(parts))(*[q.h for q in parts])
+    _lf._check(L.lf_part_linear_forest(arr, len(parts), comm.h, _lf._stream()))
+
+
+def tridiag(parts, comm):
+    """lf_part_tridiag -> per partition (a, b, c) over its own vertices (row = iperm)."""
+    import torch
+
+    L = _lf.load()
+    outs = [tuple(torch.empty(q.n_own, dtype=torch.float32, device="cuda") for _ in range(3)) for q in parts]
+    arr = (C.c_void_p * len(parts))(*[q.h for q in parts])
+    pa = (C.c_void_p * len(parts))(*[o[0].data_ptr() for o in outs])
+    pb = (C.c_void_p * len(parts))(*[o[1].data_ptr() for o in outs])
+    pc = (C.c_void_p * len(parts))(*[o[2].data_ptr() for o in outs])
+    _lf._check(L.lf_part_tridiag(arr, len(parts), comm.h, pa, pb, pc, _lf._stream()))
+    return outs

@@ -24,7 +24,7 @@ EXPORTS = (
     "lf_last_error", "lf_version", "lf_profile_enable", "lf_profile_collect",
     "lf_forest_stats", "lf_comm_nccl_unique_id", "lf_comm_create_nccl", "lf_comm_create_loopback",
     "lf_comm_destroy", "lf_part_create", "lf_part_destroy", "lf_part_info", "lf_part_factor",
-    "lf_part_export",
+    "lf_part_export", "lf_part_linear_forest", "lf_part_forest_export", "lf_part_tridiag",
 )
 
 
@@ -76,6 +76,9 @@ def load(path: str = LIB_PATH):
     L.lf_part_info.argtypes = [P, P, I32]
     L.lf_part_factor.argtypes = [P, I32, P, P, P]
     L.lf_part_export.argtypes = [P, P, P, P, P, P, P, P]
+    L.lf_part_linear_forest.argtypes = [P, I32, P, P]
+    L.lf_part_forest_export.argtypes = [P, P, P, P, P, P, P]
+    L.lf_part_tridiag.argtypes = [P, I32, P, P, P, P, P]
     L.lf_profile_enable.argtypes = [I32]
     L.lf_profile_collect.argtypes = [P, I32, P, I32]
     L.lf_last_error.restype = C.c_char_p

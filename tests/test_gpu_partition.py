@@ -103,3 +103,58 @@ def test_partition_with_empty_rank(torch_cuda, oracle_mod):
     pi, pw, pv, _, _ = run_parts(torch_cuda, A, bounds)
     pi_o, _, _, _, _ = oracle_mod.factor(A, 2)
     assert np.array_equal(pi, pi_o)
+
+
+LF_CASES = [
+    ("c1", lambda: lfgen.config("C1")),
+    ("c2_slab", lambda: lfgen.grid3d_7pt_aniso(24)),
+    ("c3_small", lambda: lfgen.fem27_bricks(20)),
+    ("c4_small", lambda: lfgen.chung_lu(20000)),
+    # one long cycle and one long path crossing every partition
+    ("ring_and_path", lambda: _ring_and_path(1 << 14)),
+]
+
+
+def _ring_and_path(N):
+    s = np.arange(N - 1)
+    t = s + 1
+    w = 1.0 - lfgen.edge_hash_u(s, t, N, 3)
+    keep = s != N // 2 - 1
+    s2 = np.concatenate([s[keep], [N - 1]])
+    t2 = np.concatenate([t[keep], [N // 2]])
+    w2 = np.concatenate([w[keep], [0.5]])
+    return lfgen.csr_from_edges(N, s2, t2, w2)
+
+
+@pytest.mark.parametrize("name,make", LF_CASES, ids=[c[0] for c in LF_CASES])
+@pytest.mark.parametrize("G", [2, 3, 5])
+def test_partitioned_linear_forest_matches_oracle(torch_cuda, oracle_mod, name, make, G):
+    """Boundary-end list ranking across partitions equals the oracle's walk (§8(e))."""
+    from paper_conf_icpp_0002s22_b200 import dist
+
+    torch = torch_cuda
+    A = make()
+    bounds = dist.plan_bounds(A.rowptr, G)
+    comm = dist.Comm.loopback(G)
+    parts = []
+    for r in range(G):
+        rp, col, val = dist.row_slice(A, int(bounds[r]), int(bounds[r + 1]))
+        parts.append(dist.Partition(torch.from_numpy(rp).cuda(), torch.from_numpy(col).cuda(),
+                                    torch.from_numpy(val).cuda(), bounds, r, n=2))
+    dist.factor(parts, comm)
+    dist.linear_forest(parts, comm)
+    tri = dist.tridiag(parts, comm)
+    outs = [p.forest_export() for p in parts]
+    torch.cuda.synchronize()
+    o = oracle_mod.run_pipeline(A)
+    for k in ("forest", "path_id", "pos", "iperm"):
+        got = np.concatenate([x[k].cpu().numpy() for x in outs])
+        assert np.array_equal(got, o[k]), (k, np.argwhere(got != o[k])[:5])
+    assert int(outs[0]["n_cycles"].item()) == o["n_cycles"]
+    # a/b/c by owner vertex: element v holds row iperm[v] of the single-GPU result
+    for i, name_ in enumerate("abc"):
+        got = np.concatenate([t[i].cpu().numpy() for t in tri])
+        assert np.array_equal(got.view(np.uint32), o[name_][o["iperm"]].view(np.uint32))
+    for p in parts:
+        p.close()
+    comm.close()
