@@ -512,8 +512,8 @@ __device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem
 // reduced-graph direction of boundary vertex g through its slot i:
 //   none -> end marker -(g+1) (distance 0); another rank -> exit marker -(N+1+g)
 //   (distance 0; the exit list continues it); another tile -> the neighbour (distance 1);
-//   local -> the segment's other terminal t: t if t continues in another tile of this
-//   rank, else an end or exit marker at t (distance = local length).
+//   local -> the segment's other terminal t: t if t continues (another tile or rank),
+//   else an end marker at t (distance = local length).
 __device__ __forceinline__ void reduced_dir(const ForestArgs& a, const TileSmem& s, int32_t b0, int32_t g,
                                             int2 nb, int i, int2 p, int2 r, int32_t& q, int32_t& d) {
     const int32_t x = i ? nb.y : nb.x;
@@ -525,9 +525,9 @@ __device__ __forceinline__ void reduced_dir(const ForestArgs& a, const TileSmem&
     const int so = outward_slot(nbt, s);
     const int32_t xo = so ? nbt.y : nbt.x;
     const int32_t tg = b0 + t;
-    if (xo < 0) q = -(tg + 1);
-    else if (is_foreign(xo, a)) q = (int32_t)(-(a.N + 1 + tg));
-    else q = tg;
+    // t continues (in another tile or on another rank): t is itself a boundary vertex,
+    // so point at it -- its own cross-rank slot carries the exit marker
+    q = xo < 0 ? -(tg + 1) : tg;
     d = i ? r.y : r.x;
 }
 
