@@ -17,6 +17,7 @@ from .graphs import (  # noqa: F401
     grid2d_5pt,
     aniso2d,
     grid3d_7pt_aniso,
+    grid3d_7pt_aniso_rows,
     fem27_bricks,
     chung_lu,
     grid3d_27pt,

@@ -208,6 +208,50 @@ def grid3d_7pt_aniso(n=128, seed=2, eps=(1.0, 0.1, 0.01)):
                           meta={"seed": seed, "n": n})
 
 
+def grid3d_7pt_aniso_rows(n, nz, z_lo, z_hi, seed=2, eps=(1.0, 0.1, 0.01)):
+    """Rows of the planes [z_lo, z_hi) of the n x n x nz 7-point anisotropic graph (the C2
+    recipe on a taller grid), with GLOBAL column ids: rowptr (rebased), col, val, lo, hi.
+
+    Equal to rows [lo, hi) of grid3d_7pt_aniso on the same grid (tests check this); used
+    to give every rank of a multi-GPU run its own slab without building the whole graph."""
+    N = n * n * nz
+    plane = n * n
+    lo, hi = z_lo * plane, z_hi * plane
+    v = np.arange(lo, hi, dtype=np.int64)
+    x, y, z = v % n, (v // n) % n, v // plane
+    offs = [(-plane, z > 0, 2), (-n, y > 0, 1), (-1, x > 0, 0), (0, None, None), (1, x < n - 1, 0),
+            (n, y < n - 1, 1), (plane, z < nz - 1, 2)]
+    cols, vals, masks = [], [], []
+    wsum = np.zeros(v.shape[0], dtype=np.float64)
+    for d, m, ax in offs:
+        if d == 0:
+            continue
+        j = v + d
+        u = edge_hash_u(v, j, N, seed)
+        w = (np.asarray(eps, dtype=np.float64)[ax] * (1.0 + 0.25 * u)).astype(np.float32)
+        wsum += np.where(m, np.abs(w.astype(np.float64)), 0.0)
+    diag = (wsum + 1.0).astype(np.float32)
+    for d, m, ax in offs:
+        j = v + d
+        if d == 0:
+            cols.append(j)
+            vals.append(diag)
+            masks.append(np.ones(v.shape[0], dtype=bool))
+            continue
+        u = edge_hash_u(v, j, N, seed)
+        w = (np.asarray(eps, dtype=np.float64)[ax] * (1.0 + 0.25 * u)).astype(np.float32)
+        cols.append(j)
+        vals.append(-w)
+        masks.append(m)
+    C = np.stack(cols, 1)
+    V = np.stack(vals, 1)
+    Mk = np.stack(masks, 1)
+    counts = Mk.sum(1).astype(np.int64)
+    rowptr = np.zeros(v.shape[0] + 1, dtype=np.int64)
+    np.cumsum(counts, out=rowptr[1:])
+    return rowptr, C[Mk].astype(np.int32), V[Mk].astype(np.float32), lo, hi
+
+
 def _fwd27():
     out = []
     for dz in (-1, 0, 1):

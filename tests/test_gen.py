@@ -56,3 +56,16 @@ def _e27(n):
 def test_c5_edge_count_formula():
     """C5 512^3 has 1,737,761,788 undirected edges (SURVEY.md §8(a) size table)."""
     assert _e27(512) == 1_737_761_788
+
+
+def test_slab_rows_equal_global_rows():
+    """Per-rank slab generation equals the rows of the whole graph (multi-GPU bench)."""
+    n, nz = 10, 12
+    A = lfgen.grid3d_7pt_aniso(n)  # nz == n here only for the first check below
+    rp, col, val, lo, hi = lfgen.grid3d_7pt_aniso_rows(n, n, 3, 7)
+    a, b = A.rowptr[lo], A.rowptr[hi]
+    assert np.array_equal(rp, A.rowptr[lo:hi + 1] - a)
+    assert np.array_equal(col, A.col[a:b]) and np.array_equal(val.view(np.uint32), A.val[a:b].view(np.uint32))
+    # a taller grid: rows of consecutive slabs concatenate to the full matrix
+    parts = [lfgen.grid3d_7pt_aniso_rows(n, nz, z0, z1) for z0, z1 in ((0, 5), (5, 12))]
+    assert parts[0][4] == parts[1][3] and parts[1][4] == n * n * nz
