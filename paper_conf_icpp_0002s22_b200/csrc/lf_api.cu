@@ -359,3 +359,33 @@ int lf_validate_csr(const lf_csr_t* A, void* ws, size_t ws_bytes, void* stream) 
 }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------------------
+// launch-overhead probe (diagnostics only): an empty kernel on a
+// persistent-size grid, launched cooperatively or not, optionally with one grid barrier
+// ---------------------------------------------------------------------------
+#include <cooperative_groups.h>
+namespace lf {
+__global__ void k_probe(int sync_steps) {
+    cooperative_groups::grid_group g = cooperative_groups::this_grid();
+    for (int i = 0; i < sync_steps; i++) g.sync();
+}
+__global__ void k_probe_plain(int* p) {
+    if (p && threadIdx.x == 0 && blockIdx.x == 0) atomicAdd(p, 1);
+}
+}  // namespace lf
+
+extern "C" int lf_debug_launch_probe(int mode, int block, int sync_steps, void* stream) {
+    using namespace lf;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (mode == 0) {
+        const int grid = persistent_grid((const void*)k_probe_plain, block);
+        k_probe_plain<<<grid, block, 0, s>>>(nullptr);
+        LF_CUDA(cudaGetLastError());
+        return LF_OK;
+    }
+    const int grid = persistent_grid((const void*)k_probe, block);
+    void* args[] = {&sync_steps};
+    LF_CUDA(cudaLaunchCooperativeKernel((const void*)k_probe, grid, block, args, 0, s));
+    return LF_OK;
+}

@@ -471,8 +471,11 @@ struct FusedArgs {
     int G;
 };
 
+#ifndef LF_FUSED_T
+#define LF_FUSED_T 256
+#endif
 template <int NN, int G>
-__global__ void __launch_bounds__(256) k_rounds_fused(FusedArgs f) {
+__global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {
     cg::grid_group grid = cg::this_grid();
     for (int k = 1; k < f.M; k++) {
         ProposeArgs pa = f.pa;
@@ -814,8 +817,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             case 16: kfn = (const void*)k_rounds_fused<NN, 16>; break;
             default: kfn = (const void*)k_rounds_fused<NN, 32>; break;
         }
-        const int grid = persistent_grid(kfn, 256);
-        LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, 256, args, 0, s));
+        const int grid = persistent_grid(kfn, LF_FUSED_T);
+        LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, 0, s));
     }
     if (o->until_maximal) {
         if (rounds_dev) {

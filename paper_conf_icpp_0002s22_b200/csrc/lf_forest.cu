@@ -673,8 +673,11 @@ __device__ __forceinline__ void red_epilogue(const ForestArgs& a, const int32_t*
 }
 
 constexpr int RT = 1024;                    // reduced-scan block size
-constexpr int kRedSmall = 4 * RT;           // lists up to this size run in one CTA, in smem
-constexpr int RNPT = kRedSmall / RT;
+#ifndef LF_RED_SMALL
+#define LF_RED_SMALL (4 * 1024)
+#endif
+constexpr int kRedSmall = LF_RED_SMALL;     // lists up to this size run in one CTA, in smem
+constexpr int RNPT = 4;                     // nodes per thread of the one-CTA scan
 
 // smem image of a small reduced graph (pointers are compact node indices or end markers)
 struct RedSmem {
@@ -685,9 +688,23 @@ struct RedSmem {
 // The whole reduced scan inside one CTA: load the list's nodes into shared memory with
 // compact indices (cidx maps vertex -> index), run the bidirectional scan there with
 // block barriers, write the results.  Used when the boundary list is small.
+#ifdef LF_PHASE_TIMING
+__device__ __forceinline__ unsigned long long gtime() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define RS_MARK(i) do { __syncthreads(); if (threadIdx.x == 0) atomicAdd((unsigned long long*)&a.ctl[224 + 2 * (i)], gtime() - t_start); } while (0)
+#else
+#define RS_MARK(i) do { } while (0)
+#endif
+
 template <bool MIN>
 __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt, int* ctl, RedSmem& S) {
     const int tid = threadIdx.x;
+#ifdef LF_PHASE_TIMING
+    const unsigned long long t_start = gtime();
+#endif
     // [vertex] scratch, unused yet (an int32 view of end2/dist2, indexed by vertex id)
     int32_t* cidx = (MIN ? (int32_t*)(a.end2 + a.lo) : (int32_t*)(a.dist2 + a.lo)) - a.lo;
     int32_t v[RNPT];
@@ -698,6 +715,7 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
         if (v[k] >= 0) cidx[v[k]] = idx;
     }
     __syncthreads();
+    RS_MARK(0);
     int2 q[RNPT];
     ulonglong2 kk[RNPT];
     bool fin[RNPT];
@@ -714,6 +732,7 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
         S.q[tid + k * RT] = q[k];
         S.k[tid + k * RT] = kk[k];
     }
+    RS_MARK(1);
     int step = 0;
     int notdone = 0;
 #pragma unroll
@@ -765,6 +784,7 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
             if (!any) break;
         }
     }
+    RS_MARK(2);
 #pragma unroll
     for (int k = 0; k < RNPT; k++) {
         if (v[k] < 0) continue;
@@ -779,6 +799,7 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
             a.dist2[v[k]] = make_int2((int)kk[k].x, (int)kk[k].y);
         }
     }
+    RS_MARK(3);
 }
 
 // Reduced bidirectional scan over a boundary list (one cooperative kernel).
@@ -1122,7 +1143,10 @@ int forest_stats(const ForestWs& w, int32_t* out, int cap) {
     for (int i = 0; i < cap && i < 9; i++) out[i] = v[i];
     // [16..31]: per-phase cycle sums (units of 1024 cycles; LF_PHASE_TIMING builds only)
     const unsigned long long* ph = reinterpret_cast<const unsigned long long*>(h + 208);
-    for (int i = 0; i < 16 && 16 + i < cap; i++) out[16 + i] = (int)(ph[i] >> 10);
+    for (int i = 0; i < 8 && 16 + i < cap; i++) out[16 + i] = (int)(ph[i] >> 10);
+    // [24..27]: reduced-scan small-path timestamps (ns, summed over runs; timing builds)
+    const unsigned long long* rt = reinterpret_cast<const unsigned long long*>(h + 224);
+    for (int i = 0; i < 4 && 24 + i < cap; i++) out[24 + i] = (int)(rt[i] >> 10);
     return LF_OK;
 }
 

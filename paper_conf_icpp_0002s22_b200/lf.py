@@ -301,4 +301,5 @@ def forest_stats(N, ws):
     d = dict(zip(FOREST_STATS, (int(x) for x in out[:len(FOREST_STATS)])))
     if out[16:].any():  # LF_PHASE_TIMING build: per-phase kcycles summed over tiles
         d["phase_kcycles"] = [int(x) for x in out[16:24]]
+        d["redscan_small_us_cum"] = [int(x) for x in out[24:28]]
     return d
