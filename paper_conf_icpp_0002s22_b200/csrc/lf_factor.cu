@@ -336,6 +336,179 @@ __global__ void LF_TILE_BOUNDS k_propose_tile(ProposeArgs a) {
     }
 }
 
+// ---------------------------------------------------------------------------
+// Round 0 as a pipelined stream: persistent CTAs walk their tiles while cp.async (LDGSTS)
+// copies the next tile's col/val range and the row pointers of the one after into the
+// other shared-memory stage, so HBM reads overlap the row scans.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void cp16(void* smem, const void* gmem) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(gmem));
+}
+__device__ __forceinline__ void cp8(void* smem, const void* gmem) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(d), "l"(gmem));
+}
+__device__ __forceinline__ void cp4(void* smem, const void* gmem) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(d), "l"(gmem));
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void cp_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
+constexpr int SPT = 256;      // threads
+constexpr int SETILE = 4096;  // entries per stage
+
+struct StreamSmem {
+    int32_t col[2][SETILE];
+    float val[2][SETILE];
+    int64_t rp[3][SPT + 1];
+    int64_t a0[2];            // aligned start of the staged range per stage (or -1)
+};
+
+template <int R>
+__device__ __forceinline__ void issue_rowptr(const ProposeArgs& a, int64_t t, int64_t* dst) {
+    const int64_t r0 = t * R;
+    const int64_t cnt = (r0 + R <= a.N) ? R + 1 : a.N + 1 - r0;
+    for (int i = threadIdx.x; i < cnt; i += SPT) cp8(dst + i, a.rowptr + r0 + i);
+}
+
+// stage the entry range of a tile whose row pointers are in rp; returns false if too long
+__device__ __forceinline__ void issue_entries(const ProposeArgs& a, int64_t e0, int64_t e1, int32_t* scol,
+                                              float* sval, int64_t* a0_out) {
+    const int64_t a0 = e0 & ~(int64_t)3;
+    if (e1 - a0 > SETILE) {
+        if (threadIdx.x == 0) *a0_out = -1;
+        return;
+    }
+    if (threadIdx.x == 0) *a0_out = a0;
+    const int64_t v1 = e1 & ~(int64_t)3;
+    const int nvec = (int)((v1 - a0) >> 2);
+    for (int i = threadIdx.x; i < nvec; i += SPT) {
+        cp16(scol + 4 * i, a.col + a0 + 4 * i);
+        cp16(sval + 4 * i, a.val + a0 + 4 * i);
+    }
+    for (int64_t e = v1 + threadIdx.x; e < e1; e += SPT) {
+        cp4(scol + (e - a0), a.col + e);
+        cp4(sval + (e - a0), a.val + e);
+    }
+}
+
+template <int NN, int G, bool CHARGED>
+__global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
+    constexpr int R = SPT / G;
+    extern __shared__ __align__(16) unsigned char sraw[];
+    StreamSmem& S = *reinterpret_cast<StreamSmem*>(sraw);
+    const int tid = threadIdx.x;
+    const int64_t ntiles = (a.N + R - 1) / R;
+    const int64_t t0 = blockIdx.x;
+    unsigned long long my_live = 0, my_nnz = 0;
+    int my_prop = 0;
+    if (t0 < ntiles) {
+        // prologue: row pointers of the first tile (waited), then its entries + next rowptr
+        issue_rowptr<R>(a, t0, S.rp[0]);
+        cp_commit();
+        cp_wait_all();
+        __syncthreads();
+        {
+            const int64_t rl = (t0 * R + R <= a.N) ? R : a.N - t0 * R;
+            issue_entries(a, S.rp[0][0], S.rp[0][rl], S.col[0], S.val[0], &S.a0[0]);
+        }
+        if (t0 + gridDim.x < ntiles) issue_rowptr<R>(a, t0 + gridDim.x, S.rp[1]);
+        cp_commit();
+    }
+    int i = 0;
+    for (int64_t t = t0; t < ntiles; t += gridDim.x, i++) {
+        cp_wait_all();
+        __syncthreads();
+        const int b = i & 1;
+        const int64_t* rp = S.rp[i % 3];
+        const int64_t tn = t + gridDim.x;
+        if (tn < ntiles) {  // prefetch: entries of the next tile, row pointers of the one after
+            const int64_t* rpn = S.rp[(i + 1) % 3];
+            const int64_t rl = (tn * R + R <= a.N) ? R : a.N - tn * R;
+            issue_entries(a, rpn[0], rpn[rl], S.col[b ^ 1], S.val[b ^ 1], &S.a0[b ^ 1]);
+            if (tn + gridDim.x < ntiles) issue_rowptr<R>(a, tn + gridDim.x, S.rp[(i + 2) % 3]);
+            cp_commit();
+        }
+        const int64_t a0 = S.a0[b];
+        const bool staged = a0 >= 0;
+        const int32_t* scol = S.col[b];
+        const float* sval = S.val[b];
+        const int lr = tid / G, li = tid % G;
+        const int64_t row = t * R + lr;
+        const bool valid = row < a.N;
+        const int32_t v = (int32_t)(a.row_base + row);
+        const int64_t rs = valid ? rp[lr] : 0;
+        int64_t re = valid ? rp[lr + 1] : 0;
+        const bool deferred = valid && (re - rs) > a.defer_len;
+        defer_append(a, deferred && li == 0, v);
+        if (deferred) re = rs;
+        uint32_t cv = 0;
+        if (CHARGED && valid) cv = (a.state[v] & ST_CHARGE) ? 1u : 0u;
+        uint64_t top[NN];
+#pragma unroll
+        for (int s2 = 0; s2 < NN; s2++) top[s2] = 0;
+        uint32_t theta0 = 0, dbits = 0;
+        for (int64_t e = rs + li; e < re; e += G) {
+            int32_t j;
+            uint32_t xb;
+            if (staged) { j = scol[e - a0]; xb = __float_as_uint(sval[e - a0]); }
+            else { j = __ldg(a.col + e); xb = __float_as_uint(__ldg(a.val + e)); }
+            if (j == v) { dbits = xb; continue; }                        // diagonal (L231)
+            const uint32_t ab = xb & 0x7FFFFFFFu;
+            if (ab == 0u) continue;                                      // zero (L31)
+            theta0 = 1;
+            if (CHARGED && (((a.state[j] & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
+            topn_insert_fast<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
+        }
+        if (G > 1) {
+            topn_merge_group<NN, G>(top);
+#pragma unroll
+            for (int off = G / 2; off >= 1; off >>= 1) {
+                theta0 |= __shfl_xor_sync(0xffffffffu, theta0, off);
+                dbits |= __shfl_xor_sync(0xffffffffu, dbits, off);
+            }
+        }
+        if (valid && !deferred && li == 0) {
+            int32_t pj[NN];
+            float pv[NN];
+            int np = 0;
+#pragma unroll
+            for (int s2 = 0; s2 < NN; s2++) {
+                if (top[s2] != 0) { pj[s2] = key_col(top[s2]); pv[s2] = key_val(top[s2]); np++; }
+                else { pj[s2] = (s2 == 0 && !theta0) ? PROP_RETIRED : -1; pv[s2] = 0.0f; }
+            }
+            if (NN == 2) {
+                reinterpret_cast<int2*>(a.prop_j)[v] = make_int2(pj[0], pj[NN > 1 ? 1 : 0]);
+                reinterpret_cast<float2*>(a.prop_v)[v] = make_float2(pv[0], pv[NN > 1 ? 1 : 0]);
+            } else {
+#pragma unroll
+                for (int s2 = 0; s2 < NN; s2++) {
+                    a.prop_j[(int64_t)v * NN + s2] = pj[s2];
+                    a.prop_v[(int64_t)v * NN + s2] = pv[s2];
+                }
+            }
+            if (a.diag) a.diag[v] = __uint_as_float(dbits);
+            if (theta0) { my_live++; my_nnz += (unsigned long long)(re - rs); }
+            my_prop |= np > 0;
+        }
+        __syncthreads();  // stage b and rp[i % 3] are reused two iterations later
+    }
+#pragma unroll
+    for (int off = 16; off >= 1; off >>= 1) {
+        my_live += __shfl_xor_sync(0xffffffffu, my_live, off);
+        my_nnz += __shfl_xor_sync(0xffffffffu, my_nnz, off);
+        my_prop |= __shfl_xor_sync(0xffffffffu, my_prop, off);
+    }
+    if ((tid & 31) == 0) {
+        const int slot = (int)((blockIdx.x * (SPT / 32) + (tid >> 5)) & 63);
+        if (a.live_rows && my_live) atomicAdd(a.live_rows + slot, my_live);
+        if (a.live_nnz && my_nnz) atomicAdd(a.live_nnz + slot, my_nnz);
+        if (my_prop && *(volatile int*)a.proposed == 0) atomicOr(a.proposed, 1);
+    }
+}
+
 struct MutualArgs {
     int64_t N;                       // rows in all-rows mode (round 0)
     int64_t row_base;                // vertex of row r in all-rows mode: row_base + r
@@ -576,6 +749,38 @@ static void launch_propose(int G, const ProposeArgs& pa, int grid, cudaStream_t 
     }
 }
 
+template <int NN, int G, bool CH>
+static void launch_stream_one(const ProposeArgs& pa, cudaStream_t s) {
+    static bool attr = false;
+    const int smem = (int)sizeof(StreamSmem);
+    if (!attr) {
+        cudaFuncSetAttribute((const void*)k_propose_stream<NN, G, CH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        attr = true;
+    }
+    const int grid = persistent_grid((const void*)k_propose_stream<NN, G, CH>, SPT, smem);
+    k_propose_stream<NN, G, CH><<<grid, SPT, smem, s>>>(pa);
+}
+
+template <int NN>
+static void launch_propose_stream(int G, const ProposeArgs& pa, cudaStream_t s) {
+    if (pa.N == 0) return;
+    if (pa.charging) {
+        switch (G) {
+            case 1: launch_stream_one<NN, 1, true>(pa, s); break;
+            case 2: launch_stream_one<NN, 2, true>(pa, s); break;
+            case 4: launch_stream_one<NN, 4, true>(pa, s); break;
+            default: launch_stream_one<NN, 8, true>(pa, s); break;
+        }
+    } else {
+        switch (G) {
+            case 1: launch_stream_one<NN, 1, false>(pa, s); break;
+            case 2: launch_stream_one<NN, 2, false>(pa, s); break;
+            case 4: launch_stream_one<NN, 4, false>(pa, s); break;
+            default: launch_stream_one<NN, 8, false>(pa, s); break;
+        }
+    }
+}
+
 template <int NN>
 static void launch_propose_tile(int G, const ProposeArgs& pa, int64_t N, cudaStream_t s) {
     const int R = PT / G;
@@ -701,7 +906,11 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             if (fresh) {
                 const int Gt = tile_lanes(N > 0 ? (double)A->nnz / (double)N : 1.0);
                 pa.defer_len = 32 * Gt;
+#ifdef LF_TILE_PLAIN
                 launch_propose_tile<NN>(Gt, pa, N, s);
+#else
+                launch_propose_stream<NN>(Gt, pa, s);
+#endif
             } else {
                 pa.defer_len = 32 * G;
                 launch_propose<NN>(G, pa, grid_p, s);

@@ -479,9 +479,8 @@ __device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int3
         const int2 nb = s.nb[u];
         ek[k].x = KEY_INF;
         ek[k].y = KEY_INF;
-        if (g >= a.hi) { s.w[u] = make_float2(0.f, 0.f); continue; }
-        const float2 w = a.pi2_w[g];
-        s.w[u] = w;
+        if (g >= a.hi) continue;
+        const float2 w = s.w[u];
         if (nb.x >= 0) {
             const int32_t mn = g < nb.x ? g : nb.x;
             const int2 nbm = is_local(mn, s) ? s.nb[mn - b0] : (is_foreign(mn, a) ? ghost_slots(a, mn) : a.pi2[mn]);
@@ -493,6 +492,26 @@ __device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int3
             ek[k].y = edge_key(g, nb.y, w.y, nbm);
         }
     }
+}
+
+// slots and weights of the tile in one round trip (cycle pass)
+__device__ __forceinline__ void load_tile_w(const int2* __restrict__ src, const float2* __restrict__ wsrc,
+                                            TileSmem& s, int32_t b0, int64_t hi) {
+    if (threadIdx.x == 0) {
+        s.b0 = b0;
+        s.tend = (int32_t)((int64_t)b0 + LB < hi ? (int64_t)b0 + LB : hi);
+    }
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int64_t g = (int64_t)b0 + u;
+        const bool in = g < hi;
+        const int2 nb = in ? src[g] : make_int2(-1, -1);
+        const float2 w = in ? wsrc[g] : make_float2(0.f, 0.f);
+        s.nb[u] = nb;
+        s.w[u] = w;
+    }
+    __syncthreads();
 }
 
 __device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem& s, int32_t b0, int64_t hi) {
@@ -538,7 +557,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local1(ForestArgs a) {
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     LF_PHASE_INIT;
-    load_tile(a.pi2, s, b0, a.hi);
+    load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     LF_PHASE(a.ctl, 0);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
@@ -846,7 +865,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
-    load_tile(a.pi2, s, b0, a.hi);
+    load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
     // weakest edge of the cycle through each own vertex (INF: not on a cycle)
