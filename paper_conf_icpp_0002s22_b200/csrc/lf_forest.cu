@@ -29,6 +29,7 @@
 
 #include <cub/device/device_scan.cuh>
 #include <cstdint>
+#include <climits>
 #include <cstring>
 
 #include "lf_common.cuh"
@@ -94,8 +95,14 @@ __device__ __forceinline__ uint64_t edge_key(int32_t v, int32_t w, float wabs, i
 
 // shared-memory state of one tile
 struct TileSmem {
-    int2 nb[LB];          // global neighbours (slot order), -1 = none
-    float2 w[LB];         // |w| per slot (cycle pass)
+    int2 nb[LB];          // global neighbours (slot order), -1 = none; run slots virtual
+    union {
+        float2 w[LB];     // |w| per slot (cycle pass; read by slot_keys before tile_rank)
+        struct {
+            short2 run[LB];  // (first, last) local vertex of the run of u
+            short2 vw[LB];   // edges behind each slot (a run jump spans the run)
+        } r;
+    };
     short2 P[LB];         // stride pointer per direction (vertex or splitter node), or marker
     short2 R[LB];         // edges covered per direction (rank pass)
     uint64_t K0[LB];      // min edge key, direction 0 (cycle pass)
@@ -106,7 +113,11 @@ struct TileSmem {
     short2 recD[LB];      // per face: distance to that node
     int nspl;             // number of splitter nodes
     int32_t b0, tend;     // first vertex of the tile, one past its last (own range end)
+    // cycle pass only (kernels of the rank pass allocate the struct without these)
+    uint64_t EK0[LB];     // key of the (virtual) link behind slot 0 / slot 1
+    uint64_t EK1[LB];
 };
+constexpr size_t kTileSmemNoKeys = offsetof(TileSmem, EK0);
 
 // x lies in this tile (the tile never extends past the own range [lo, hi))
 __device__ __forceinline__ bool is_local(int32_t x, const TileSmem& s) {
@@ -212,39 +223,189 @@ __device__ __forceinline__ bool hashed_splitter(int32_t g) {
     return (((uint32_t)g * 0x9E3779B1u) >> kSplitShift) == 0u;
 }
 
-// Block-local ranking by a ruling set.  Same outputs as tile_scan, but
-// O(1) work per vertex: splitters (segment terminals plus hashed vertices, density 1/16)
-// walk sequentially through shared memory to the next splitter in each direction,
-// recording (node, distance) in every vertex they pass; the bidirectional scan then runs
-// on the splitter nodes only; every vertex combines its record with its node's result.
-// Cycles without a splitter are left unvisited and fall back to tile_scan (cycle pass
-// only -- a forest has none).
+// block-wide inclusive scans over LB values, thread t owning u = VPT*t .. VPT*t+VPT-1
+__device__ __forceinline__ int block_scan_max(int x, int* sh) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x = max(x, y);
+    }
+    if (lane == 31) sh[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        int t = lane < LT / 32 ? sh[lane] : INT_MIN;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, t, o);
+            if (lane >= o) t = max(t, y);
+        }
+        if (lane < LT / 32) sh[lane] = t;
+    }
+    __syncthreads();
+    const int pre = w > 0 ? sh[w - 1] : INT_MIN;
+    __syncthreads();
+    return max(x, pre);
+}
+
+__device__ __forceinline__ int block_scan_min_rev(int x, int* sh) {
+    // suffix minimum: scan from the last thread backwards
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_down_sync(0xffffffffu, x, o);
+        if (lane + o < 32) x = min(x, y);
+    }
+    if (lane == 0) sh[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        int t = lane < LT / 32 ? sh[lane] : INT_MAX;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_down_sync(0xffffffffu, t, o);
+            if (lane + o < 32) t = min(t, y);
+        }
+        if (lane < LT / 32) sh[lane] = t;
+    }
+    __syncthreads();
+    const int suf = w + 1 < LT / 32 ? sh[w + 1] : INT_MAX;
+    __syncthreads();
+    return min(x, suf);
+}
+
+// Block-local ranking.  Same outputs as tile_scan, O(1) work per vertex:
+//  0. runs: maximal intervals of consecutive vertex ids linked in the factor (an x-line of
+//     a natural-order grid) are found with block-wide scans and contracted -- each end's
+//     slot into the run becomes a virtual link to the other end (weight = run length - 1,
+//     key = the run's weakest edge key); a run closed by a direct link between its ends is
+//     a cycle by itself.  Interior vertices drop out until step 5.
+//  1. splitters: terminals plus hashed vertices (density 1/8) among the remaining ones;
+//  2. each splitter walks sequentially through shared memory to the next splitter in both
+//     directions, recording (node, distance) in every vertex it passes;
+//  3. the bidirectional scan runs on the splitter nodes only;
+//  4. every remaining vertex combines its record with its node's result (cycles without a
+//     splitter fall back to tile_scan; cycle pass only -- a forest has none);
+//  5. interior run vertices take their run ends' results plus their offset in the run.
 template <bool MINK>
 __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
                           int2 (&R)[VPT], ulonglong2 (&K)[VPT], int* stats) {
+    __shared__ int sh[32];
     const int tid = threadIdx.x;
     LF_PHASE_INIT;
+    const int tlen = s.tend - s.b0;
     if (tid == 0) s.nspl = 0;
-    __syncthreads();
-    // 1. splitters: terminals of the local structure (a slot that is missing or remote) and
-    //    hashed vertices; node numbering by a shared counter (order does not matter)
+    // 0a. run links and (cycle pass) link keys; temporaries: sidx = lp flag, K0 = key (u-1,u)
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = tid + k * LT;
         const int2 nb = s.nb[u];
-        const bool l0 = nb.x >= 0 && is_local(nb.x, s);
-        const bool l1 = nb.y >= 0 && is_local(nb.y, s);
-        const bool sp = !l0 || !l1 || hashed_splitter(b0 + u);
+        const int32_t g = b0 + u;
+        const bool lp = u > 0 && u < tlen && (nb.x == g - 1 || nb.y == g - 1);
+        s.sidx[u] = lp ? 1 : 0;
+        if (MINK) {
+            s.EK0[u] = ek[k].x;
+            s.EK1[u] = ek[k].y;
+            s.K0[u] = lp ? (nb.x == g - 1 ? ek[k].x : ek[k].y) : KEY_INF;
+        }
+    }
+    __syncthreads();
+    // 0b. run bounds by block scans (contiguous ownership: thread t owns VPT*t..VPT*t+VPT-1)
+    {
+        __shared__ int thr[LT];
+        const int u0 = tid * VPT;
+        int st[VPT], en[VPT];
+        int run = INT_MIN;
+#pragma unroll
+        for (int j = 0; j < VPT; j++) {
+            if (!s.sidx[u0 + j]) run = u0 + j;  // u0+j starts a run
+            st[j] = run;
+        }
+        const int pre = block_scan_max(run, sh);  // inclusive over threads 0..tid
+        thr[tid] = pre;
+        __syncthreads();
+        const int prev_max = tid > 0 ? thr[tid - 1] : INT_MIN;
+        __syncthreads();
+        run = INT_MAX;
+#pragma unroll
+        for (int j = VPT - 1; j >= 0; j--) {
+            const int u = u0 + j;
+            const bool ln = u + 1 < tlen && s.sidx[u + 1];
+            if (!ln) run = u;  // u ends a run
+            en[j] = run;
+        }
+        const int suf = block_scan_min_rev(run, sh);  // inclusive over threads tid..LT-1
+        thr[tid] = suf;
+        __syncthreads();
+        const int next_min = tid + 1 < LT ? thr[tid + 1] : INT_MAX;
+#pragma unroll
+        for (int j = 0; j < VPT; j++) {
+            const int ra = st[j] == INT_MIN ? prev_max : st[j];
+            const int rb = en[j] == INT_MAX ? next_min : en[j];
+            s.r.run[u0 + j] = make_short2((short)ra, (short)rb);
+        }
+        if (MINK) {
+#pragma unroll
+            for (int j = 0; j < VPT; j++) s.K1[u0 + j] = KEY_INF;
+        }
+    }
+    __syncthreads();
+    if (MINK) {
+        // weakest link of each run, accumulated at the run's first vertex
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int u = tid + k * LT;
+            const short2 rr = s.r.run[u];
+            if (u > rr.x) atomicMin((unsigned long long*)&s.K1[rr.x], (unsigned long long)s.K0[u]);
+        }
+        __syncthreads();
+    }
+    // 0c. contract: virtual links between run ends; run cycles; interior flags (sidx = -2)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const short2 rr = s.r.run[u];
+        const int32_t g = b0 + u;
+        short2 vw = make_short2(1, 1);
+        const int len = rr.y - rr.x + 1;
+        if (len >= 2 && (u == rr.x || u == rr.y)) {
+            const int other = (u == rr.x) ? rr.y : rr.x;
+            const int32_t inside = (u == rr.x) ? g + 1 : g - 1;
+            int2 nb = s.nb[u];
+            const uint64_t rk = MINK ? s.K1[rr.x] : 0;
+            if (nb.x == inside) { nb.x = b0 + other; vw.x = (short)(len - 1); if (MINK) s.EK0[u] = rk; }
+            else { nb.y = b0 + other; vw.y = (short)(len - 1); if (MINK) s.EK1[u] = rk; }
+            s.nb[u] = nb;
+        }
+        s.r.vw[u] = vw;
+    }
+    __syncthreads();
+    // 1. splitters among run ends and single vertices; a run closed into a cycle by a
+    //    direct link between its ends is resolved here (sidx = -3)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const short2 rr = s.r.run[u];
+        const int2 nb = s.nb[u];
+        const bool interior = u > rr.x && u < rr.y;
+        const bool run_cycle = rr.y - rr.x >= 2 && nb.x == nb.y;  // both slots reach the other end
         short id = -1;
-        if (sp) id = (short)atomicAdd(&s.nspl, 1);
+        if (u >= tlen) {
+            id = (short)atomicAdd(&s.nspl, 1);  // padding: isolated terminal
+        } else if (interior || run_cycle) {
+            id = run_cycle ? -3 : -2;
+        } else {
+            const bool l0 = nb.x >= 0 && is_local(nb.x, s);
+            const bool l1 = nb.y >= 0 && is_local(nb.y, s);
+            if (!l0 || !l1 || hashed_splitter(b0 + u)) id = (short)atomicAdd(&s.nspl, 1);
+        }
         s.sidx[u] = id;
-        if (sp) s.spl[id] = (short)u;
+        if (id >= 0) s.spl[id] = (short)u;
         s.recS[u] = make_short2(-1, -1);
     }
     LF_PHASE(stats - kCtlStat, 3);
     const int C = s.nspl;
     if (tid == 0 && stats) atomicAdd(&stats[MINK ? 0 : 3], C);
-    // 2. walks: one per (node, slot), sequential through non-splitters
+    // 2. walks: one per (node, slot), sequential through non-splitters (weighted links)
     for (int wk = tid; wk < 2 * C; wk += LT) {
         const int i = wk >> 1, f = wk & 1;
         const int su = s.spl[i];
@@ -254,26 +415,20 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         int dist = 0;
         uint64_t km = KEY_INF;
         if (x >= 0 && is_local(x, s)) {
-            int prev = su, cur = x - b0, d = 1;
-            if (MINK) {
-                const float2 ws = s.w[su];
-                const int mn = su < cur ? su : cur;
-                km = edge_key(b0 + su, x, f ? ws.y : ws.x, s.nb[mn]);
-            }
+            const short2 vws = s.r.vw[su];
+            int prev = su, cur = x - b0, d = f ? vws.y : vws.x;
+            if (MINK) km = f ? s.EK1[su] : s.EK0[su];
             while (s.sidx[cur] < 0) {
                 const int2 nbc = s.nb[cur];
                 const int face = (nbc.x == b0 + prev) ? 0 : 1;
                 if (face == 0) { s.recS[cur].x = (short)((i << 1) | f); s.recD[cur].x = (short)d; }
                 else { s.recS[cur].y = (short)((i << 1) | f); s.recD[cur].y = (short)d; }
                 const int nxt = (face ? nbc.x : nbc.y) - b0;  // local (else cur were a splitter)
-                if (MINK) {
-                    const float2 wc = s.w[cur];
-                    const int mn = cur < nxt ? cur : nxt;
-                    km = umin64(km, edge_key(b0 + cur, b0 + nxt, face ? wc.x : wc.y, s.nb[mn]));
-                }
+                const short2 vwc = s.r.vw[cur];
+                d += face ? vwc.x : vwc.y;
+                if (MINK) km = umin64(km, face ? s.EK0[cur] : s.EK1[cur]);
                 prev = cur;
                 cur = nxt;
-                d++;
             }
             ptr = s.sidx[cur];
             dist = d;
@@ -338,7 +493,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         }
     }
     LF_PHASE(stats - kCtlStat, 5);
-    // 4. expand: every vertex from its node (splitter) or its walk records
+    // 4. expand run ends and single vertices from their node or walk records
     bool unvisited[VPT];
     int any_unvisited = 0;
 #pragma unroll
@@ -346,6 +501,9 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         const int u = tid + k * LT;
         unvisited[k] = false;
         const int id = s.sidx[u];
+        P[k] = make_int2(0, 0);
+        R[k] = make_int2(0, 0);
+        if (id == -2 || id == -3) continue;  // interior run vertex / run cycle: step 5
         if (id >= 0) {
             const short2 p = s.P[id];
             P[k].x = p.x;
@@ -388,16 +546,74 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         }
         if (__syncthreads_or(any_unvisited)) {
             if (tid == 0 && stats) atomicAdd(&stats[2], 1);
-            // splitter-free local cycles: the pointer-jumping scan on them alone
+            // splitter-free cycles of the contracted graph: pointer jumping on them alone,
+            // with the virtual link keys
             bool skip[VPT];
+            ulonglong2 ekv[VPT];
 #pragma unroll
-            for (int k = 0; k < VPT; k++) skip[k] = !unvisited[k];
+            for (int k = 0; k < VPT; k++) {
+                const int u = tid + k * LT;
+                skip[k] = !unvisited[k];
+                ekv[k] = make_ulonglong2(s.EK0[u], s.EK1[u]);
+            }
             int2 P2[VPT], R2[VPT];
             ulonglong2 K2[VPT];
-            tile_scan<true>(s, b0, ek, P2, R2, K2, skip);
+            tile_scan<true>(s, b0, ekv, P2, R2, K2, skip);
 #pragma unroll
             for (int k = 0; k < VPT; k++)
                 if (unvisited[k]) { P[k] = P2[k]; K[k] = K2[k]; }
+        }
+    }
+    // 5. interior run vertices and run cycles from the run ends.  Publish the ends'
+    //    results: recS = terminal markers (or (0,0) cycle), recD = distances, EK = keys.
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const short2 rr = s.r.run[u];
+        if (rr.y > rr.x && (u == rr.x || u == rr.y) && s.sidx[u] != -3) {
+            s.recS[u] = make_short2((short)P[k].x, (short)P[k].y);
+            s.recD[u] = make_short2((short)R[k].x, (short)R[k].y);
+            if (MINK) { s.EK0[u] = K[k].x; s.EK1[u] = K[k].y; }
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const int id = s.sidx[u];
+        if (id != -2 && id != -3) continue;
+        const short2 rr = s.r.run[u];
+        if (s.sidx[rr.x] == -3) {  // the run closes into a cycle through its ends' direct link
+            // weakest of the run links (virtual key) and the closing link (real key)
+            P[k] = make_int2(0, 0);
+            if (MINK) {
+                const uint64_t km = umin64(s.EK0[rr.x], s.EK1[rr.x]);
+                K[k] = make_ulonglong2(km, km);
+            }
+            continue;
+        }
+        const int32_t g = b0 + u;
+        const int2 nb = s.nb[u];
+        // interior: slot toward u-1 leads to the run start, the other to the run end
+        const short2 pa = s.recS[rr.x], pb = s.recS[rr.y];
+        const int2 nba = s.nb[rr.x], nbb = s.nb[rr.y];
+        const int oa = (nba.x == b0 + rr.y) ? 1 : 0;  // the start's outer slot
+        const int ob = (nbb.x == b0 + rr.x) ? 1 : 0;  // the end's outer slot
+        const int ta = oa ? pa.y : pa.x, tb = ob ? pb.y : pb.x;
+        const bool cyc = (pa.x >= 0 && pa.y >= 0);
+        const short2 da = s.recD[rr.x], db = s.recD[rr.y];
+        const int dA = (oa ? da.y : da.x) + (u - rr.x), dB = (ob ? db.y : db.x) + (rr.y - u);
+        const int sa = (nb.x == g - 1) ? 0 : 1;  // u's slot toward the run start
+        if (cyc) {
+            P[k] = make_int2(0, 0);
+            if (MINK) K[k] = make_ulonglong2(s.EK0[rr.x], s.EK1[rr.x]);
+        } else if (sa == 0) {
+            P[k] = make_int2(ta, tb);
+            R[k] = make_int2(dA, dB);
+        } else {
+            P[k] = make_int2(tb, ta);
+            R[k] = make_int2(dB, dA);
         }
     }
     __syncthreads();
@@ -552,7 +768,7 @@ __device__ __forceinline__ void reduced_dir(const ForestArgs& a, const TileSmem&
 
 // Pass 1, local part: local min-scan; store the local results; emit the reduced-graph
 // records of boundary vertices.
-__global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local1(ForestArgs a) {
+__global__ void __launch_bounds__(LT, 1) k_lf_local1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
@@ -1057,8 +1273,10 @@ static int forest_prepare() {
     if (attr_done) return LF_OK;
     const int smem = (int)sizeof(TileSmem);
     LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local1, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local2, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local3, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local2, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)kTileSmemNoKeys));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_local3, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)kTileSmemNoKeys));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)sizeof(RedSmem)));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1120,7 +1338,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("lf_local2", -1, s);
-        k_lf_local2<<<tiles, LT, smem, s>>>(a);
+        k_lf_local2<<<tiles, LT, kTileSmemNoKeys, s>>>(a);
         LF_CUDA(cudaGetLastError());
     }
     {
@@ -1130,7 +1348,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("lf_local3", -1, s);
-        k_lf_local3<<<tiles, LT, smem, s>>>(a);
+        k_lf_local3<<<tiles, LT, kTileSmemNoKeys, s>>>(a);
         LF_CUDA(cudaGetLastError());
     }
     {
@@ -1460,7 +1678,7 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
     if (rc) return rc;
     if (tiles > 0) {
         LF_PROF("lf_local2", -1, s);
-        k_lf_local2<<<tiles, LT, smem, s>>>(a);
+        k_lf_local2<<<tiles, LT, kTileSmemNoKeys, s>>>(a);
         LF_CUDA(cudaGetLastError());
     }
     {
@@ -1472,7 +1690,7 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
     if (rc) return rc;
     if (tiles > 0) {
         LF_PROF("lf_local3", -1, s);
-        k_lf_local3<<<tiles, LT, smem, s>>>(a);
+        k_lf_local3<<<tiles, LT, kTileSmemNoKeys, s>>>(a);
         LF_CUDA(cudaGetLastError());
     }
     // path offsets: own exclusive scan, rank bases, published offsets of cross-rank paths
