@@ -396,7 +396,9 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         } else {
             const bool l0 = nb.x >= 0 && is_local(nb.x, s);
             const bool l1 = nb.y >= 0 && is_local(nb.y, s);
-            if (!l0 || !l1 || hashed_splitter(b0 + u)) id = (short)atomicAdd(&s.nspl, 1);
+            // run ends are always splitters: every cycle through a run has one
+            const bool run_end = rr.y > rr.x;
+            if (!l0 || !l1 || run_end || hashed_splitter(b0 + u)) id = (short)atomicAdd(&s.nspl, 1);
         }
         s.sidx[u] = id;
         if (id >= 0) s.spl[id] = (short)u;
