@@ -344,21 +344,63 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
             s.r.run[u0 + j] = make_short2((short)ra, (short)rb);
         }
         if (MINK) {
+            // weakest link of each run: segmented inclusive min-scan of the link keys
+            // (segments = runs); the value at the run's last vertex is the run's minimum
+            uint64_t x[VPT];
+            bool hd[VPT];
+            uint64_t agg = KEY_INF;
+            bool anyh = false;
 #pragma unroll
-            for (int j = 0; j < VPT; j++) s.K1[u0 + j] = KEY_INF;
+            for (int j = 0; j < VPT; j++) {
+                hd[j] = !s.sidx[u0 + j];
+                const uint64_t kv = s.K0[u0 + j];
+                agg = hd[j] ? kv : umin64(agg, kv);
+                anyh |= hd[j];
+                x[j] = agg;
+            }
+            // warp scan of (head, min) pairs: (f1,x1)+(f2,x2) = (f1|f2, f2 ? x2 : min(x1,x2))
+            const int lane = tid & 31, wid = tid >> 5;
+            bool f = anyh;
+            uint64_t v = agg;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint64_t yv = __shfl_up_sync(0xffffffffu, v, o);
+                const int yf = __shfl_up_sync(0xffffffffu, (int)f, o);
+                if (lane >= o) { if (!f) v = umin64(v, yv); f = f || yf; }
+            }
+            __shared__ uint64_t wv[LT / 32];
+            __shared__ int wf[LT / 32];
+            if (lane == 31) { wv[wid] = v; wf[wid] = f; }
+            __syncthreads();
+            if (wid == 0) {
+                uint64_t tv = lane < LT / 32 ? wv[lane] : KEY_INF;
+                bool tf = lane < LT / 32 ? wf[lane] != 0 : false;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint64_t yv = __shfl_up_sync(0xffffffffu, tv, o);
+                    const int yf = __shfl_up_sync(0xffffffffu, (int)tf, o);
+                    if (lane >= o) { if (!tf) tv = umin64(tv, yv); tf = tf || yf; }
+                }
+                if (lane < LT / 32) { wv[lane] = tv; wf[lane] = tf; }
+            }
+            __syncthreads();
+            // carry into this thread: inclusive value of the previous thread
+            uint64_t cv = __shfl_up_sync(0xffffffffu, v, 1);
+            bool cf = __shfl_up_sync(0xffffffffu, (int)f, 1) != 0;
+            if (lane == 0) { cv = KEY_INF; cf = true; }
+            if (wid > 0 && !cf) cv = umin64(cv, wv[wid - 1]);
+            if (wid > 0 && lane == 0) { cv = wv[wid - 1]; cf = false; }
+            // apply the carry to the thread's prefix up to its first head
+#pragma unroll
+            for (int j = 0; j < VPT; j++) {
+                if (hd[j]) break;
+                x[j] = umin64(x[j], cv);
+            }
+#pragma unroll
+            for (int j = 0; j < VPT; j++) s.K1[u0 + j] = x[j];
         }
     }
     __syncthreads();
-    if (MINK) {
-        // weakest link of each run, accumulated at the run's first vertex
-#pragma unroll
-        for (int k = 0; k < VPT; k++) {
-            const int u = tid + k * LT;
-            const short2 rr = s.r.run[u];
-            if (u > rr.x) atomicMin((unsigned long long*)&s.K1[rr.x], (unsigned long long)s.K0[u]);
-        }
-        __syncthreads();
-    }
     // 0c. contract: virtual links between run ends; run cycles; interior flags (sidx = -2)
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
@@ -371,7 +413,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
             const int other = (u == rr.x) ? rr.y : rr.x;
             const int32_t inside = (u == rr.x) ? g + 1 : g - 1;
             int2 nb = s.nb[u];
-            const uint64_t rk = MINK ? s.K1[rr.x] : 0;
+            const uint64_t rk = MINK ? s.K1[rr.y] : 0;  // run minimum at its last vertex
             if (nb.x == inside) { nb.x = b0 + other; vw.x = (short)(len - 1); if (MINK) s.EK0[u] = rk; }
             else { nb.y = b0 + other; vw.y = (short)(len - 1); if (MINK) s.EK1[u] = rk; }
             s.nb[u] = nb;
