@@ -146,6 +146,15 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
     return 0
 
 
+def ncu_traffic(kernel):
+    """dram bytes per launch of `kernel` from the committed ncu capture (profiles/traffic.json)."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        return json.load(open(p))["bytes_per_launch"].get(kernel)
+    except (OSError, ValueError, KeyError):
+        return None
+
+
 def cpu_baseline(A, runs):
     import oracle
 
@@ -535,7 +544,8 @@ def main():
             "roofline": {
                 "kernel": dom, "bound": "hbm", "achieved": round(dom_ach, 1) if dom_ach else None,
                 "peak": peak, "peak_kind": peak_kind, "unit": "GB/s",
-                "frac": round(dom_ach / peak, 4) if dom_ach else None, "traffic": None,
+                "frac": round(dom_ach / peak, 4) if dom_ach else None,
+                "traffic": ncu_traffic(dom) if args.config == "C2" else None,
                 "alg_bytes_per_launch": int(dom_bytes),
                 "ms_per_launch": round(kavg[dom], 5) if dom else None,
             },

@@ -62,3 +62,30 @@ if __name__ == "__main__":
             print(f"\n## ncu --set full ({a})\n")
             print(full(a))
         print()
+
+
+NAME_MAP = {  # ncu kernel name prefix -> bench.py kernel record name (first launch of a step)
+    "k_lf_local1": "lf_local1", "k_lf_local2": "lf_local2", "k_lf_local3": "lf_local3",
+    "k_propose_stream": "propose[0]", "k_propose_tile": "propose[0]", "k_rounds_fused": "rounds_fused",
+    "k_mutual": "mutual[0]", "k_tridiag": "tridiag", "k_red_scan<1>": "red_scan_cycles",
+    "k_red_scan<0>": "red_scan_ranks", "k_perm": "perm",
+}
+
+
+def traffic(path):
+    """dram read+write bytes per launch from a --set full capture, keyed like bench.py."""
+    txt = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(txt)))
+    hdr = rows[0]
+    ni, ri, wi = hdr.index("Kernel Name"), hdr.index("dram__bytes_read.sum"), hdr.index("dram__bytes_write.sum")
+    units = rows[1]
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+    out = {}
+    for r in rows[2:]:
+        name = r[ni].replace("void ", "")
+        for pre, key in NAME_MAP.items():
+            if name.startswith(pre) and key not in out:
+                b = float(r[ri].replace(",", "")) * scale.get(units[ri], 1) + \
+                    float(r[wi].replace(",", "")) * scale.get(units[wi], 1)
+                out[key] = int(b)
+    return out
