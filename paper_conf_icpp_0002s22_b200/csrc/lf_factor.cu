@@ -645,7 +645,10 @@ struct FusedArgs {
 };
 
 #ifndef LF_FUSED_T
-#define LF_FUSED_T 256
+#define LF_FUSED_T 512
+#endif
+#ifndef LF_FUSED_GRID_SM
+#define LF_FUSED_GRID_SM 1   // one CTA per SM: grid barriers scale with the CTA count
 #endif
 template <int NN, int G>
 __global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {
@@ -1026,7 +1029,9 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             case 16: kfn = (const void*)k_rounds_fused<NN, 16>; break;
             default: kfn = (const void*)k_rounds_fused<NN, 32>; break;
         }
-        const int grid = persistent_grid(kfn, LF_FUSED_T);
+        int grid = sm_count() * LF_FUSED_GRID_SM;  // fewer CTAs: cheaper grid barriers
+        const int cap = persistent_grid(kfn, LF_FUSED_T);
+        if (grid > cap) grid = cap;
         LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, 0, s));
     }
     if (o->until_maximal) {

@@ -77,7 +77,7 @@ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < 
     } while (0)
 #define LF_PHASE_INIT long long ph_t = clock64()
 #else
-#define LF_PHASE(ctl, i) __syncthreads()  // a phase boundary is always a block barrier
+#define LF_PHASE(ctl, i) do { } while (0)
 #define LF_PHASE_INIT do { } while (0)
 #endif
 
@@ -248,6 +248,32 @@ __device__ __forceinline__ int block_scan_max(int x, int* sh) {
     return max(x, pre);
 }
 
+// exclusive block max-scan (over threads 0..tid-1), INT_MIN for thread 0
+__device__ __forceinline__ int block_scan_max_excl(int x, int* sh) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc = max(inc, y);
+    }
+    int exc = __shfl_up_sync(0xffffffffu, inc, 1);
+    if (lane == 0) exc = INT_MIN;
+    if (lane == 31) sh[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+        int t = lane < LT / 32 ? sh[lane] : INT_MIN;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, t, o);
+            if (lane >= o) t = max(t, y);
+        }
+        if (lane < LT / 32) sh[lane] = t;
+    }
+    __syncthreads();
+    return w > 0 ? max(exc, sh[w - 1]) : exc;
+}
+
 __device__ __forceinline__ int block_scan_min_rev(int x, int* sh) {
     // suffix minimum: scan from the last thread backwards
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -309,40 +335,34 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         }
     }
     __syncthreads();
-    // 0b. run bounds by block scans (contiguous ownership: thread t owns VPT*t..VPT*t+VPT-1)
+    // 0b. run bounds (contiguous ownership: thread t owns VPT*t..VPT*t+VPT-1): the run
+    //     start by an exclusive block max-scan; the run end by a scatter from the next
+    //     run's start (a run ends one before the next run starts)
     {
-        __shared__ int thr[LT];
         const int u0 = tid * VPT;
-        int st[VPT], en[VPT];
+        int st[VPT];
         int run = INT_MIN;
 #pragma unroll
         for (int j = 0; j < VPT; j++) {
             if (!s.sidx[u0 + j]) run = u0 + j;  // u0+j starts a run
             st[j] = run;
         }
-        const int pre = block_scan_max(run, sh);  // inclusive over threads 0..tid
-        thr[tid] = pre;
-        __syncthreads();
-        const int prev_max = tid > 0 ? thr[tid - 1] : INT_MIN;
-        __syncthreads();
-        run = INT_MAX;
-#pragma unroll
-        for (int j = VPT - 1; j >= 0; j--) {
-            const int u = u0 + j;
-            const bool ln = u + 1 < tlen && s.sidx[u + 1];
-            if (!ln) run = u;  // u ends a run
-            en[j] = run;
-        }
-        const int suf = block_scan_min_rev(run, sh);  // inclusive over threads tid..LT-1
-        thr[tid] = suf;
-        __syncthreads();
-        const int next_min = tid + 1 < LT ? thr[tid + 1] : INT_MAX;
+        const int prev_max = block_scan_max_excl(run, sh);
 #pragma unroll
         for (int j = 0; j < VPT; j++) {
-            const int ra = st[j] == INT_MIN ? prev_max : st[j];
-            const int rb = en[j] == INT_MAX ? next_min : en[j];
-            s.r.run[u0 + j] = make_short2((short)ra, (short)rb);
+            const int u = u0 + j;
+            if (st[j] == INT_MIN) st[j] = prev_max;
+            s.r.run[u].x = (short)st[j];
+            const bool is_end = u + 1 >= LB || !s.sidx[u + 1];
+            if (is_end) s.r.run[st[j]].y = (short)u;  // the run start learns its end
         }
+        __syncthreads();
+        short en[VPT];
+#pragma unroll
+        for (int j = 0; j < VPT; j++) en[j] = s.r.run[st[j]].y;
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < VPT; j++) s.r.run[u0 + j].y = en[j];
         if (MINK) {
             // weakest link of each run: segmented inclusive min-scan of the link keys
             // (segments = runs); the value at the run's last vertex is the run's minimum
@@ -446,6 +466,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         if (id >= 0) s.spl[id] = (short)u;
         s.recS[u] = make_short2(-1, -1);
     }
+    __syncthreads();
     LF_PHASE(stats - kCtlStat, 3);
     const int C = s.nspl;
     if (tid == 0 && stats) atomicAdd(&stats[MINK ? 0 : 3], C);
@@ -480,6 +501,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         if (f) { s.P[i].y = ptr; s.R[i].y = (short)dist; s.K1[i] = km; }
         else { s.P[i].x = ptr; s.R[i].x = (short)dist; s.K0[i] = km; }
     }
+    __syncthreads();
     LF_PHASE(stats - kCtlStat, 4);
     // 3. bidirectional scan over the splitter nodes (node arrays in s.P/s.R/s.K*)
     for (int step = 0; step < 16; step++) {
@@ -956,7 +978,7 @@ constexpr int RT = 1024;                    // reduced-scan block size
 #define LF_RED_SMALL (4 * 1024)
 #endif
 constexpr int kRedSmall = LF_RED_SMALL;     // lists up to this size run in one CTA, in smem
-constexpr int RNPT = 4;                     // nodes per thread of the one-CTA scan
+constexpr int RNPT = (kRedSmall + RT - 1) / RT;  // nodes per thread of the one-CTA scan
 
 // smem image of a small reduced graph (pointers are compact node indices or end markers)
 struct RedSmem {
