@@ -44,7 +44,7 @@ constexpr uint64_t KEY_INF = ~0ull;
 #define LF_LB 2048
 #endif
 #ifndef LF_LT
-#define LF_LT 512
+#define LF_LT 1024
 #endif
 #ifndef LF_LMINB
 #define LF_LMINB 2
@@ -120,8 +120,13 @@ struct TileSmem {
 constexpr size_t kTileSmemNoKeys = offsetof(TileSmem, EK0);
 
 // x lies in this tile (the tile never extends past the own range [lo, hi))
-__device__ __forceinline__ bool is_local(int32_t x, const TileSmem& s) {
-    return x >= s.b0 && x < s.tend;
+// the tile's range in registers (read once from shared memory)
+struct Tile {
+    int32_t b0, tend;
+};
+__device__ __forceinline__ Tile tile_of(const TileSmem& s) { return Tile{s.b0, s.tend}; }
+__device__ __forceinline__ bool is_local(int32_t x, const Tile& t) {
+    return (uint32_t)(x - t.b0) < (uint32_t)(t.tend - t.b0);
 }
 
 // Bidirectional scan inside the tile (Alg. 3, or its min variant when MINK, restricted
@@ -137,14 +142,15 @@ template <bool MINK>
 __device__ __noinline__ void tile_scan(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], int2 (&P)[VPT],
                           int2 (&R)[VPT], ulonglong2 (&K)[VPT], const bool (&skip)[VPT]) {
     const int tid = threadIdx.x;
+    const Tile T = tile_of(s);
     bool fin[VPT];
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = tid + k * LT;
         if (skip[k]) { fin[k] = true; continue; }
         const int2 nb = s.nb[u];
-        const bool l0 = nb.x >= 0 && is_local(nb.x, s);
-        const bool l1 = nb.y >= 0 && is_local(nb.y, s);
+        const bool l0 = nb.x >= 0 && is_local(nb.x, T);
+        const bool l1 = nb.y >= 0 && is_local(nb.y, T);
         P[k] = make_int2(l0 ? nb.x - b0 : -(u + 1), l1 ? nb.y - b0 : -(u + 1));
         fin[k] = !l0 && !l1;
         s.P[u] = make_short2((short)P[k].x, (short)P[k].y);
@@ -299,6 +305,72 @@ __device__ __forceinline__ int block_scan_min_rev(int x, int* sh) {
     return min(x, suf);
 }
 
+// Bidirectional scan over the splitter nodes 0..C-1 of a tile (node arrays in s.P and
+// s.R / s.K0,K1).  WARP: warp 0 alone, NPN nodes per lane, warp barriers; else the whole
+// block, NPN = VPT nodes per thread, block barriers.
+constexpr int kWarpScanNodes = 4;  // one warp scans up to 128 nodes
+
+template <bool MINK, int NPN, bool WARP>
+__device__ __forceinline__ void node_scan(TileSmem& s, int C, int* stats) {
+    const int tid = threadIdx.x;
+    constexpr int STRIDE = WARP ? 32 : LT;
+    for (int step = 0; step < 16; step++) {
+        int notdone = 0;
+        short2 nP[NPN], nR[NPN];
+        uint64_t nk0[NPN], nk1[NPN];
+#pragma unroll
+        for (int k = 0; k < NPN; k++) {
+            const int i = tid + k * STRIDE;
+            if (i >= C) continue;
+            const short2 p = s.P[i];
+            short2 q = p, r = s.R[i];
+            uint64_t k0 = 0, k1 = 0;
+            if (MINK) { k0 = s.K0[i]; k1 = s.K1[i]; }
+#pragma unroll
+            for (int dd = 0; dd < 2; dd++) {
+                const int w = dd ? p.y : p.x;
+                if (w < 0) continue;
+                const short2 pw = s.P[w];
+                int j = -1;
+                if (pw.x != i) j = 0;
+                else if (pw.y != i) j = 1;
+                if (j < 0) continue;  // stall (reading c13)
+                const short tgt = j ? pw.y : pw.x;
+                if (dd) q.y = tgt; else q.x = tgt;
+                if (MINK) {
+                    const uint64_t kv = j ? s.K1[w] : s.K0[w];
+                    if (dd) k1 = umin64(k1, kv); else k0 = umin64(k0, kv);
+                } else {
+                    const short2 rw = s.R[w];
+                    const short dv = j ? rw.y : rw.x;
+                    if (dd) r.y = (short)(r.y + dv); else r.x = (short)(r.x + dv);
+                }
+            }
+            nP[k] = q;
+            nR[k] = r;
+            nk0[k] = k0;
+            nk1[k] = k1;
+            const bool path_done = q.x < 0 && q.y < 0;
+            bool cyc_done = false;
+            if (MINK) cyc_done = q.x >= 0 && q.y >= 0 && (k0 == k1 || q.x == q.y);
+            notdone |= !(path_done || cyc_done);
+        }
+        if (WARP) __syncwarp(); else __syncthreads();
+#pragma unroll
+        for (int k = 0; k < NPN; k++) {
+            const int i = tid + k * STRIDE;
+            if (i >= C) continue;
+            s.P[i] = nP[k];
+            if (MINK) { s.K0[i] = nk0[k]; s.K1[i] = nk1[k]; } else s.R[i] = nR[k];
+        }
+        const bool any = WARP ? (__syncwarp(), __any_sync(0xffffffffu, notdone)) : __syncthreads_or(notdone);
+        if (!any) {
+            if (tid == 0 && stats) atomicMax(&stats[4], step + 1);
+            break;
+        }
+    }
+}
+
 // Block-local ranking.  Same outputs as tile_scan, O(1) work per vertex:
 //  0. runs: maximal intervals of consecutive vertex ids linked in the factor (an x-line of
 //     a natural-order grid) are found with block-wide scans and contracted -- each end's
@@ -318,33 +390,41 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
     __shared__ int sh[32];
     const int tid = threadIdx.x;
     LF_PHASE_INIT;
-    const int tlen = s.tend - s.b0;
+    const Tile T = tile_of(s);
+    const int tlen = T.tend - T.b0;
     if (tid == 0) s.nspl = 0;
-    // 0a. run links and (cycle pass) link keys; temporaries: sidx = lp flag, K0 = key (u-1,u)
-#pragma unroll
-    for (int k = 0; k < VPT; k++) {
-        const int u = tid + k * LT;
+    // 0a. (cycle pass) slot keys and the temporary K0 = key of the run link (u-1,u); the
+    //     barriers of the scan below order these writes before their readers
+    const auto linked_prev = [&](int u) {  // u-1 and u linked in the factor (same tile)
         const int2 nb = s.nb[u];
         const int32_t g = b0 + u;
-        const bool lp = u > 0 && u < tlen && (nb.x == g - 1 || nb.y == g - 1);
-        s.sidx[u] = lp ? 1 : 0;
-        if (MINK) {
+        return u > 0 && u < tlen && (nb.x == g - 1 || nb.y == g - 1);
+    };
+    if (MINK) {
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int u = tid + k * LT;
+            const int2 nb = s.nb[u];
+            const int32_t g = b0 + u;
+            const bool lp = u > 0 && u < tlen && (nb.x == g - 1 || nb.y == g - 1);
             s.EK0[u] = ek[k].x;
             s.EK1[u] = ek[k].y;
             s.K0[u] = lp ? (nb.x == g - 1 ? ek[k].x : ek[k].y) : KEY_INF;
         }
     }
-    __syncthreads();
     // 0b. run bounds (contiguous ownership: thread t owns VPT*t..VPT*t+VPT-1): the run
     //     start by an exclusive block max-scan; the run end by a scatter from the next
     //     run's start (a run ends one before the next run starts)
     {
         const int u0 = tid * VPT;
         int st[VPT];
+        bool lk[VPT + 1];  // lk[j]: u0+j linked to u0+j-1
+#pragma unroll
+        for (int j = 0; j <= VPT; j++) lk[j] = u0 + j < LB && linked_prev(u0 + j);
         int run = INT_MIN;
 #pragma unroll
         for (int j = 0; j < VPT; j++) {
-            if (!s.sidx[u0 + j]) run = u0 + j;  // u0+j starts a run
+            if (!lk[j]) run = u0 + j;  // u0+j starts a run
             st[j] = run;
         }
         const int prev_max = block_scan_max_excl(run, sh);
@@ -353,8 +433,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
             const int u = u0 + j;
             if (st[j] == INT_MIN) st[j] = prev_max;
             s.r.run[u].x = (short)st[j];
-            const bool is_end = u + 1 >= LB || !s.sidx[u + 1];
-            if (is_end) s.r.run[st[j]].y = (short)u;  // the run start learns its end
+            if (!lk[j + 1]) s.r.run[st[j]].y = (short)u;  // run end: the run start learns it
         }
         __syncthreads();
         short en[VPT];
@@ -372,7 +451,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
             bool anyh = false;
 #pragma unroll
             for (int j = 0; j < VPT; j++) {
-                hd[j] = !s.sidx[u0 + j];
+                hd[j] = !lk[j];
                 const uint64_t kv = s.K0[u0 + j];
                 agg = hd[j] ? kv : umin64(agg, kv);
                 anyh |= hd[j];
@@ -451,23 +530,32 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         const bool interior = u > rr.x && u < rr.y;
         const bool run_cycle = rr.y - rr.x >= 2 && nb.x == nb.y;  // both slots reach the other end
         short id = -1;
+        bool node = false;
         if (u >= tlen) {
-            id = (short)atomicAdd(&s.nspl, 1);  // padding: isolated terminal
+            node = true;  // padding: isolated terminal
         } else if (interior || run_cycle) {
             id = run_cycle ? -3 : -2;
         } else {
-            const bool l0 = nb.x >= 0 && is_local(nb.x, s);
-            const bool l1 = nb.y >= 0 && is_local(nb.y, s);
+            const bool l0 = nb.x >= 0 && is_local(nb.x, T);
+            const bool l1 = nb.y >= 0 && is_local(nb.y, T);
             // run ends are always splitters: every cycle through a run has one
             const bool run_end = rr.y > rr.x;
-            if (!l0 || !l1 || run_end || hashed_splitter(b0 + u)) id = (short)atomicAdd(&s.nspl, 1);
+            node = !l0 || !l1 || run_end || hashed_splitter(b0 + u);
+        }
+        {  // warp-aggregated node numbering
+            const unsigned m = __ballot_sync(0xffffffffu, node);
+            const int lane = tid & 31;
+            int base = 0;
+            if (lane == 0 && m) base = atomicAdd(&s.nspl, __popc(m));
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (node) id = (short)(base + __popc(m & ((1u << lane) - 1u)));
         }
         s.sidx[u] = id;
         if (id >= 0) s.spl[id] = (short)u;
         s.recS[u] = make_short2(-1, -1);
     }
     __syncthreads();
-    LF_PHASE(stats - kCtlStat, 3);
+    if (MINK) LF_PHASE(stats - kCtlStat, 3);
     const int C = s.nspl;
     if (tid == 0 && stats) atomicAdd(&stats[MINK ? 0 : 3], C);
     // 2. walks: one per (node, slot), sequential through non-splitters (weighted links)
@@ -479,7 +567,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         short ptr = (short)(-(i + 1));
         int dist = 0;
         uint64_t km = KEY_INF;
-        if (x >= 0 && is_local(x, s)) {
+        if (x >= 0 && is_local(x, T)) {
             const short2 vws = s.r.vw[su];
             int prev = su, cur = x - b0, d = f ? vws.y : vws.x;
             if (MINK) km = f ? s.EK1[su] : s.EK0[su];
@@ -502,63 +590,16 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         else { s.P[i].x = ptr; s.R[i].x = (short)dist; s.K0[i] = km; }
     }
     __syncthreads();
-    LF_PHASE(stats - kCtlStat, 4);
-    // 3. bidirectional scan over the splitter nodes (node arrays in s.P/s.R/s.K*)
-    for (int step = 0; step < 16; step++) {
-        int notdone = 0;
-        short2 nP[VPT], nR[VPT];
-        uint64_t nk0[VPT], nk1[VPT];
-#pragma unroll
-        for (int k = 0; k < VPT; k++) {
-            const int i = tid + k * LT;
-            if (i >= C) continue;
-            const short2 p = s.P[i];
-            short2 q = p, r = s.R[i];
-            uint64_t k0 = 0, k1 = 0;
-            if (MINK) { k0 = s.K0[i]; k1 = s.K1[i]; }
-#pragma unroll
-            for (int dd = 0; dd < 2; dd++) {
-                const int w = dd ? p.y : p.x;
-                if (w < 0) continue;
-                const short2 pw = s.P[w];
-                int j = -1;
-                if (pw.x != i) j = 0;
-                else if (pw.y != i) j = 1;
-                if (j < 0) continue;  // stall (reading c13)
-                const short tgt = j ? pw.y : pw.x;
-                if (dd) q.y = tgt; else q.x = tgt;
-                if (MINK) {
-                    const uint64_t kv = j ? s.K1[w] : s.K0[w];
-                    if (dd) k1 = umin64(k1, kv); else k0 = umin64(k0, kv);
-                } else {
-                    const short2 rw = s.R[w];
-                    const short dv = j ? rw.y : rw.x;
-                    if (dd) r.y = (short)(r.y + dv); else r.x = (short)(r.x + dv);
-                }
-            }
-            nP[k] = q;
-            nR[k] = r;
-            nk0[k] = k0;
-            nk1[k] = k1;
-            const bool path_done = q.x < 0 && q.y < 0;
-            bool cyc_done = false;
-            if (MINK) cyc_done = q.x >= 0 && q.y >= 0 && (k0 == k1 || q.x == q.y);
-            notdone |= !(path_done || cyc_done);
-        }
+    if (MINK) LF_PHASE(stats - kCtlStat, 4);
+    // 3. bidirectional scan over the splitter nodes (node arrays in s.P/s.R/s.K*): by one
+    //    warp with warp barriers when the nodes are few, else by the whole block
+    if (C <= 32 * kWarpScanNodes) {
+        if (tid < 32) node_scan<MINK, kWarpScanNodes, true>(s, C, stats);
         __syncthreads();
-#pragma unroll
-        for (int k = 0; k < VPT; k++) {
-            const int i = tid + k * LT;
-            if (i >= C) continue;
-            s.P[i] = nP[k];
-            if (MINK) { s.K0[i] = nk0[k]; s.K1[i] = nk1[k]; } else s.R[i] = nR[k];
-        }
-        if (!__syncthreads_or(notdone)) {
-            if (tid == 0 && stats) atomicMax(&stats[4], step + 1);
-            break;
-        }
+    } else {
+        node_scan<MINK, VPT, false>(s, C, stats);
     }
-    LF_PHASE(stats - kCtlStat, 5);
+    if (MINK) LF_PHASE(stats - kCtlStat, 5);
     // 4. expand run ends and single vertices from their node or walk records
     bool unvisited[VPT];
     int any_unvisited = 0;
@@ -602,7 +643,7 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         // a vertex on a cycle: make both pointers non-negative (cycle flag)
         if (P[k].x >= 0 || P[k].y >= 0) { P[k].x = 0; P[k].y = 0; }
     }
-    LF_PHASE(stats - kCtlStat, 6);
+    if (MINK) LF_PHASE(stats - kCtlStat, 6);
     if (MINK) {
         if (stats) {
             int nu = 0;
@@ -683,23 +724,26 @@ __device__ void tile_rank(TileSmem& s, int32_t b0, const ulonglong2 (&ek)[VPT], 
         }
     }
     __syncthreads();
-    LF_PHASE(stats - kCtlStat, 7);
+    if (MINK) LF_PHASE(stats - kCtlStat, 7);
 }
 
 // the slot of local terminal t (t not the walk's start) that leaves its segment: the
 // one that is not a local link (a remote neighbour or none)
-__device__ __forceinline__ int outward_slot(int2 nbt, const TileSmem& s) {
-    const bool l0 = nbt.x >= 0 && is_local(nbt.x, s);
+__device__ __forceinline__ int outward_slot(int2 nbt, const Tile& T) {
+    const bool l0 = nbt.x >= 0 && is_local(nbt.x, T);
     return l0 ? 1 : 0;
 }
 
-__device__ __forceinline__ void list_append(int32_t* list, int* count, int32_t g, bool take) {
+// warp-aggregated append; returns the list position of g (-1 if not taken)
+__device__ __forceinline__ int list_append(int32_t* list, int* count, int32_t g, bool take) {
     const unsigned m = __ballot_sync(0xffffffffu, take);
     const int lane = threadIdx.x & 31;
     int base = 0;
     if (lane == 0 && m) base = atomicAdd(count, __popc(m));
     base = __shfl_sync(0xffffffffu, base, 0);
-    if (take) list[base + __popc(m & ((1u << lane) - 1u))] = g;
+    const int idx = base + __popc(m & ((1u << lane) - 1u));
+    if (take) list[idx] = g;
+    return take ? idx : -1;
 }
 
 struct ForestArgs {
@@ -730,6 +774,9 @@ struct ForestArgs {
     int2* end2;            // [N] path ends per direction of a boundary vertex
     int2* dist2;           // [N] distances to them
     int32_t* list2;
+    // compact records of the list being built / scanned (list position -> record)
+    int2* cq;              // stride pointers (vertex ids or markers)
+    ulonglong2* cq_k;      // MIN: min keys; ADD: distances in the low words
     int* ctl;
     int32_t* path_id;
     int32_t* pos;
@@ -754,6 +801,7 @@ __device__ __forceinline__ int2 ghost_slots(const ForestArgs& a, int32_t x) {
 // keys of the own vertices' slots (global; a remote min endpoint needs one gather)
 __device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int32_t b0,
                                          ulonglong2 (&ek)[VPT]) {
+    const Tile T = tile_of(s);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -765,12 +813,12 @@ __device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int3
         const float2 w = s.w[u];
         if (nb.x >= 0) {
             const int32_t mn = g < nb.x ? g : nb.x;
-            const int2 nbm = is_local(mn, s) ? s.nb[mn - b0] : (is_foreign(mn, a) ? ghost_slots(a, mn) : a.pi2[mn]);
+            const int2 nbm = is_local(mn, T) ? s.nb[mn - b0] : (is_foreign(mn, a) ? ghost_slots(a, mn) : a.pi2[mn]);
             ek[k].x = edge_key(g, nb.x, w.x, nbm);
         }
         if (nb.y >= 0) {
             const int32_t mn = g < nb.y ? g : nb.y;
-            const int2 nbm = is_local(mn, s) ? s.nb[mn - b0] : (is_foreign(mn, a) ? ghost_slots(a, mn) : a.pi2[mn]);
+            const int2 nbm = is_local(mn, T) ? s.nb[mn - b0] : (is_foreign(mn, a) ? ghost_slots(a, mn) : a.pi2[mn]);
             ek[k].y = edge_key(g, nb.y, w.y, nbm);
         }
     }
@@ -817,13 +865,14 @@ __device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem
 //   else an end marker at t (distance = local length).
 __device__ __forceinline__ void reduced_dir(const ForestArgs& a, const TileSmem& s, int32_t b0, int32_t g,
                                             int2 nb, int i, int2 p, int2 r, int32_t& q, int32_t& d) {
+    const Tile T = tile_of(s);
     const int32_t x = i ? nb.y : nb.x;
     if (x < 0) { q = -(g + 1); d = 0; return; }
     if (is_foreign(x, a)) { q = (int32_t)(-(a.N + 1 + g)); d = 0; return; }
-    if (!is_local(x, s)) { q = x; d = 1; return; }
+    if (!is_local(x, T)) { q = x; d = 1; return; }
     const int t = -((i ? p.y : p.x) + 1);
     const int2 nbt = s.nb[t];
-    const int so = outward_slot(nbt, s);
+    const int so = outward_slot(nbt, T);
     const int32_t xo = so ? nbt.y : nbt.x;
     const int32_t tg = b0 + t;
     // t continues (in another tile or on another rank): t is itself a boundary vertex,
@@ -840,6 +889,7 @@ __global__ void __launch_bounds__(LT, 1) k_lf_local1(ForestArgs a) {
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     LF_PHASE_INIT;
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
+    const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     LF_PHASE(a.ctl, 0);
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
@@ -847,19 +897,19 @@ __global__ void __launch_bounds__(LT, 1) k_lf_local1(ForestArgs a) {
     int2 P[VPT], R[VPT];
     ulonglong2 K[VPT];
     tile_rank<true>(s, b0, ek, P, R, K, a.ctl + kCtlStat);
-    LF_PHASE(a.ctl, 2);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
         const int32_t g = b0 + u;
         const int2 nb = s.nb[u];
-        const bool r0 = nb.x >= 0 && !is_local(nb.x, s);
-        const bool r1 = nb.y >= 0 && !is_local(nb.y, s);
+        const bool r0 = nb.x >= 0 && !is_local(nb.x, T);
+        const bool r1 = nb.y >= 0 && !is_local(nb.y, T);
         const bool boundary = g < a.hi && (r0 || r1);
         if (g < a.hi) {
             a.loc1[g] = make_short2((short)P[k].x, (short)P[k].y);
             if (P[k].x >= 0 && P[k].y >= 0) a.kst[g] = umin64(K[k].x, K[k].y);
         }
+        const int idx = list_append(a.list1, &a.ctl[kCtlCnt1], g, boundary);
         if (boundary) {
             int32_t q0, q1, d0, d1;
             reduced_dir(a, s, b0, g, nb, 0, P[k], R[k], q0, d0);
@@ -869,12 +919,11 @@ __global__ void __launch_bounds__(LT, 1) k_lf_local1(ForestArgs a) {
             rk.x = (nb.x < 0 || is_foreign(nb.x, a)) ? KEY_INF : (r0 ? ek[k].x : K[k].x);
             rk.y = (nb.y < 0 || is_foreign(nb.y, a)) ? KEY_INF : (r1 ? ek[k].y : K[k].y);
             if (a.ekb) a.ekb[g] = ek[k];
-            const int2 q = make_int2(q0, q1);
-            a.rq1[0][g] = q; a.rq1[1][g] = q;
-            a.rk1[0][g] = rk; a.rk1[1][g] = rk;
+            a.cq[idx] = make_int2(q0, q1);
+            a.cq_k[idx] = rk;
         }
-        list_append(a.list1, &a.ctl[kCtlCnt1], g, boundary);
     }
+    LF_PHASE(a.ctl, 2);  // outputs
 }
 
 // One step of the reduced bidirectional scan for the list entries t0, t0+stride, ...
@@ -978,17 +1027,37 @@ constexpr int RT = 1024;                    // reduced-scan block size
 #define LF_RED_SMALL (4 * 1024)
 #endif
 constexpr int kRedSmall = LF_RED_SMALL;     // lists up to this size run in one CTA, in smem
-constexpr int RNPT = (kRedSmall + RT - 1) / RT;  // nodes per thread of the one-CTA scan
+constexpr int kRedHash = 2 * kRedSmall;     // open-addressing table vertex -> list position
+static_assert((kRedHash & (kRedHash - 1)) == 0, "hash table size must be a power of two");
 
-// smem image of a small reduced graph (pointers are compact node indices or end markers)
+// smem image of a small reduced graph (pointers are list positions or end markers)
 struct RedSmem {
     int2 q[kRedSmall];
     ulonglong2 k[kRedSmall];  // MIN: min keys; ADD: distances in .x/.y low words
+    int32_t v[kRedSmall];     // vertex id of each list position
+    int2 ht[kRedHash];        // (vertex, list position), vertex -1 = empty
 };
 
-// The whole reduced scan inside one CTA: load the list's nodes into shared memory with
-// compact indices (cidx maps vertex -> index), run the bidirectional scan there with
-// block barriers, write the results.  Used when the boundary list is small.
+__device__ __forceinline__ uint32_t red_hash(int32_t v) {
+    return ((uint32_t)v * 0x9E3779B1u) >> (32 - __builtin_ctz(kRedHash));
+}
+
+// list position of a listed vertex (every stride pointer of the reduced graph is one)
+__device__ __forceinline__ int red_lookup(const RedSmem& S, int32_t v) {
+    uint32_t h = red_hash(v);
+    for (int n = 0; n < kRedHash; n++) {
+        const int2 e = S.ht[h];
+        if (e.x == v) return e.y;
+        if (e.x < 0) break;
+        h = (h + 1) & (kRedHash - 1);
+    }
+    return -(v + 1);  // unreachable for a well-formed list: an end marker at v
+}
+
+// The whole reduced scan inside one CTA: the list's compact records are loaded with
+// coalesced reads, their vertex-id pointers are turned into list positions through a
+// shared-memory hash table, the bidirectional scan runs in shared memory with block
+// barriers, and the results are written per vertex.  Used when the boundary list is small.
 #ifdef LF_PHASE_TIMING
 __device__ __forceinline__ unsigned long long gtime() {
     unsigned long long t;
@@ -1000,52 +1069,62 @@ __device__ __forceinline__ unsigned long long gtime() {
 #define RS_MARK(i) do { } while (0)
 #endif
 
-template <bool MIN>
+template <int T, bool MIN>
 __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt, int* ctl, RedSmem& S) {
+    constexpr int NPT = (kRedSmall + T - 1) / T;
     const int tid = threadIdx.x;
 #ifdef LF_PHASE_TIMING
     const unsigned long long t_start = gtime();
 #endif
-    // [vertex] scratch, unused yet (an int32 view of end2/dist2, indexed by vertex id)
-    int32_t* cidx = (MIN ? (int32_t*)(a.end2 + a.lo) : (int32_t*)(a.dist2 + a.lo)) - a.lo;
-    int32_t v[RNPT];
+    for (int i = tid; i < kRedHash; i += T) S.ht[i] = make_int2(-1, -1);
+    __syncthreads();
+    int32_t v[NPT];
+    int2 q[NPT];
+    ulonglong2 kk[NPT];
 #pragma unroll
-    for (int k = 0; k < RNPT; k++) {
-        const int idx = tid + k * RT;
-        v[k] = idx < cnt ? list[idx] : -1;
-        if (v[k] >= 0) cidx[v[k]] = idx;
+    for (int k = 0; k < NPT; k++) {
+        const int idx = tid + k * T;
+        v[k] = -1;
+        if (idx >= cnt) continue;
+        v[k] = list[idx];
+        q[k] = a.cq[idx];
+        kk[k] = a.cq_k[idx];
+    }
+#pragma unroll
+    for (int k = 0; k < NPT; k++) {
+        if (v[k] < 0) continue;
+        const int idx = tid + k * T;
+        S.v[idx] = v[k];
+        uint32_t h = red_hash(v[k]);
+        while (atomicCAS(&S.ht[h].x, -1, v[k]) != -1) h = (h + 1) & (kRedHash - 1);
+        S.ht[h].y = idx;
     }
     __syncthreads();
     RS_MARK(0);
-    int2 q[RNPT];
-    ulonglong2 kk[RNPT];
-    bool fin[RNPT];
+    bool fin[NPT];
 #pragma unroll
-    for (int k = 0; k < RNPT; k++) {
+    for (int k = 0; k < NPT; k++) {
         fin[k] = true;
         if (v[k] < 0) continue;
-        int2 g = MIN ? a.rq1[0][v[k]] : a.rq2[0][v[k]];
-        q[k].x = g.x >= 0 ? cidx[g.x] : g.x;
-        q[k].y = g.y >= 0 ? cidx[g.y] : g.y;
-        if (MIN) kk[k] = a.rk1[0][v[k]];
-        else { const int2 r = a.rr2[0][v[k]]; kk[k] = make_ulonglong2((uint64_t)(uint32_t)r.x, (uint64_t)(uint32_t)r.y); }
+        if (q[k].x >= 0) q[k].x = red_lookup(S, q[k].x);
+        if (q[k].y >= 0) q[k].y = red_lookup(S, q[k].y);
         fin[k] = q[k].x < 0 && q[k].y < 0;
-        S.q[tid + k * RT] = q[k];
-        S.k[tid + k * RT] = kk[k];
+        S.q[tid + k * T] = q[k];
+        S.k[tid + k * T] = kk[k];
     }
     RS_MARK(1);
     int step = 0;
     int notdone = 0;
 #pragma unroll
-    for (int k = 0; k < RNPT; k++) notdone |= !fin[k];
+    for (int k = 0; k < NPT; k++) notdone |= !fin[k];
     if (__syncthreads_or(notdone)) {
         for (; step < a.max_steps; step++) {
-            int2 nq[RNPT];
-            ulonglong2 nk[RNPT];
+            int2 nq[NPT];
+            ulonglong2 nk[NPT];
 #pragma unroll
-            for (int k = 0; k < RNPT; k++) {
+            for (int k = 0; k < NPT; k++) {
                 if (fin[k]) continue;
-                const int me = tid + k * RT;
+                const int me = tid + k * T;
                 nq[k] = q[k];
                 nk[k] = kk[k];
 #pragma unroll
@@ -1068,9 +1147,9 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
             __syncthreads();
             notdone = 0;
 #pragma unroll
-            for (int k = 0; k < RNPT; k++) {
+            for (int k = 0; k < NPT; k++) {
                 if (fin[k]) continue;
-                const int me = tid + k * RT;
+                const int me = tid + k * T;
                 q[k] = nq[k];
                 kk[k] = nk[k];
                 S.q[me] = q[k];
@@ -1087,10 +1166,10 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
     }
     RS_MARK(2);
 #pragma unroll
-    for (int k = 0; k < RNPT; k++) {
+    for (int k = 0; k < NPT; k++) {
         if (v[k] < 0) continue;
         // pointers back to vertex ids (markers pass through unchanged)
-        const int2 qg = make_int2(q[k].x >= 0 ? list[q[k].x] : q[k].x, q[k].y >= 0 ? list[q[k].y] : q[k].y);
+        const int2 qg = make_int2(q[k].x >= 0 ? S.v[q[k].x] : q[k].x, q[k].y >= 0 ? S.v[q[k].y] : q[k].y);
         if (MIN) {
             a.cyc_k[v[k]] = (q[k].x >= 0 && q[k].y >= 0) ? umin64(kk[k].x, kk[k].y) : KEY_INF;
             a.end2[v[k]] = qg;
@@ -1107,8 +1186,8 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
 //   MIN: min-scan of edge keys; epilogue writes cyc_k (INF unless on a global cycle).
 //   ADD: position scan with weighted hops; epilogue writes end2 / dist2.
 // Small lists run in block 0 alone, in shared memory (a grid barrier costs more than the
-// work); large ones use the whole grid with grid barriers.  Both leave as soon as every
-// node is done.
+// work); large ones use the whole grid with grid barriers on vertex-indexed ping-pong
+// buffers initialised from the compact records.  Both leave as soon as every node is done.
 template <bool MIN>
 __global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
     __shared__ int sh[32];
@@ -1117,13 +1196,27 @@ __global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
     const int cnt = *(volatile int*)&a.ctl[MIN ? kCtlCnt1 : kCtlCnt2];
     int* ctl = a.ctl + (MIN ? kCtlRed1 : kCtlRed2);
     if (cnt <= kRedSmall) {
-        if (blockIdx.x == 0) red_scan_small<MIN>(a, list, cnt, ctl, *reinterpret_cast<RedSmem*>(red_smem));
+        if (blockIdx.x == 0) red_scan_small<RT, MIN>(a, list, cnt, ctl, *reinterpret_cast<RedSmem*>(red_smem));
         return;
     }
-    int step = 0;
     cg::grid_group grid = cg::this_grid();
     const int stride = gridDim.x * blockDim.x;
     const int t0 = blockIdx.x * blockDim.x + threadIdx.x;
+    for (int idx = t0; idx < cnt; idx += stride) {
+        const int32_t v = list[idx];
+        const int2 q = a.cq[idx];
+        const ulonglong2 k = a.cq_k[idx];
+        if (MIN) {
+            a.rq1[0][v] = q; a.rq1[1][v] = q;
+            a.rk1[0][v] = k; a.rk1[1][v] = k;
+        } else {
+            const int2 d = make_int2((int)k.x, (int)k.y);
+            a.rq2[0][v] = q; a.rq2[1][v] = q;
+            a.rr2[0][v] = d; a.rr2[1][v] = d;
+        }
+    }
+    grid.sync();
+    int step = 0;
     for (; step < a.max_steps; step++) {
         int notdone = red_step<MIN>(a, list, cnt, step, t0, stride);
         // block reduction of notdone, one atomic per block
@@ -1148,6 +1241,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
+    const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
     // weakest edge of the cycle through each own vertex (INF: not on a cycle)
@@ -1171,7 +1265,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
             for (int i = 0; i < 2; i++) {
                 const int t = -((i ? p.y : p.x) + 1);
                 const int2 nbt = s.nb[t];
-                const int so = (t == u) ? i : outward_slot(nbt, s);
+                const int so = (t == u) ? i : outward_slot(nbt, T);
                 const int32_t xo = so ? nbt.y : nbt.x;
                 if (xo >= 0 && kstar == KEY_INF) kstar = a.cyc_k[b0 + t];
             }
@@ -1206,8 +1300,8 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
         const int u = threadIdx.x + k * LT;
         const int32_t g = b0 + u;
         const int2 nb = s.nb[u];
-        const bool r0 = nb.x >= 0 && !is_local(nb.x, s);
-        const bool r1 = nb.y >= 0 && !is_local(nb.y, s);
+        const bool r0 = nb.x >= 0 && !is_local(nb.x, T);
+        const bool r1 = nb.y >= 0 && !is_local(nb.y, T);
         const bool boundary = g < a.hi && (r0 || r1);
         if (g < a.hi) {
             // terminal markers (16 bits each) and local distances (16 bits each)
@@ -1215,16 +1309,14 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
             const uint32_t rr = ((uint32_t)(uint16_t)R[k].x) | ((uint32_t)(uint16_t)R[k].y << 16);
             a.loc2[g] = make_int2((int)pp, (int)rr);
         }
+        const int idx = list_append(a.list2, &a.ctl[kCtlCnt2], g, boundary);
         if (boundary) {
             int32_t q0, q1, d0, d1;
             reduced_dir(a, s, b0, g, nb, 0, P[k], R[k], q0, d0);
             reduced_dir(a, s, b0, g, nb, 1, P[k], R[k], q1, d1);
-            const int2 q = make_int2(q0, q1);
-            const int2 d = make_int2(d0, d1);
-            a.rq2[0][g] = q; a.rq2[1][g] = q;
-            a.rr2[0][g] = d; a.rr2[1][g] = d;
+            a.cq[idx] = make_int2(q0, q1);
+            a.cq_k[idx] = make_ulonglong2((uint32_t)d0, (uint32_t)d1);
         }
-        list_append(a.list2, &a.ctl[kCtlCnt2], g, boundary);
     }
 }
 
@@ -1234,6 +1326,7 @@ __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     load_tile(a.forest, s, b0, a.hi);
+    const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
@@ -1249,7 +1342,7 @@ __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
             const int32_t d = i ? ry : rx;
             const int2 nbt = s.nb[t];
             // the outward slot of t: slot i itself when t == u (the walk never left u)
-            const int so = (t == u) ? i : outward_slot(nbt, s);
+            const int so = (t == u) ? i : outward_slot(nbt, T);
             const int32_t xo = so ? nbt.y : nbt.x;
             if (xo >= 0) {  // continues in another block: reduced result of t (end marker)
                 const int2 e = a.end2[b0 + t];
@@ -1314,6 +1407,8 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     t.ctl = c.take<int>(256);
     t.kraw = c.take<ulonglong2>(n);
     t.ekb = c.take<ulonglong2>(n);
+    t.cq = c.take<int2>(n);
+    t.cq_k = c.take<ulonglong2>(n);
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
     if (w) *w = t;
@@ -1385,6 +1480,8 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     a.end2 = w.end2;
     a.dist2 = w.dist2;
     a.list2 = w.list2;
+    a.cq = w.cq;
+    a.cq_k = w.cq_k;
     a.ctl = w.ctl;
     a.path_id = path_id;
     a.pos = pos;
@@ -1523,24 +1620,15 @@ __global__ void k_exit_records(ForestArgs a, const int32_t* list, const int* cou
 
 // the exit graph from the gathered records of all ranks (padding has g = -1)
 template <bool MIN>
-__global__ void k_exit_build(const ExitRec* rec, int64_t total, int2** gq, ulonglong2** gk, int2** gr,
-                             int32_t* glist, int* gcount) {
+__global__ void k_exit_build(const ExitRec* rec, int64_t total, int32_t* glist, int2* gcq, ulonglong2* gcq_k,
+                             int* gcount) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
         const ExitRec r = rec[i];
         if (r.g < 0) continue;
-        const int2 q = make_int2(r.q0, r.q1);
-        gq[0][r.g] = q;
-        gq[1][r.g] = q;
-        if (MIN) {
-            const ulonglong2 k = make_ulonglong2(r.k0, r.k1);
-            gk[0][r.g] = k;
-            gk[1][r.g] = k;
-        } else {
-            const int2 d = make_int2(r.d0, r.d1);
-            gr[0][r.g] = d;
-            gr[1][r.g] = d;
-        }
-        glist[atomicAdd(gcount, 1)] = r.g;
+        const int pos = atomicAdd(gcount, 1);
+        glist[pos] = r.g;
+        gcq[pos] = make_int2(r.q0, r.q1);
+        gcq_k[pos] = MIN ? make_ulonglong2(r.k0, r.k1) : make_ulonglong2((uint32_t)r.d0, (uint32_t)r.d1);
     }
 }
 
@@ -1636,23 +1724,11 @@ static int exit_pass(const ForestArgs& a, const int32_t* list, const int* count,
     }
     int rc = pc.allgather(pc.ctx, send, all, sizeof(ExitRec) * pc.exit_cap, s);
     if (rc) return rc;
-    int2** dq = nullptr;
-    ulonglong2** dk = nullptr;
-    int2** dr = nullptr;
-    // pointer tables (small) for the build kernel
-    void* tabs = nullptr;
-    LF_CUDA(cudaMallocAsync(&tabs, sizeof(void*) * 6, s));
-    void* h[6] = {pc.gq[0], pc.gq[1], pc.gk[0], pc.gk[1], pc.gr[0], pc.gr[1]};
-    LF_CUDA(cudaMemcpyAsync(tabs, h, sizeof(h), cudaMemcpyHostToDevice, s));
-    dq = (int2**)tabs;
-    dk = (ulonglong2**)((void**)tabs + 2);
-    dr = (int2**)((void**)tabs + 4);
     const int64_t total = (int64_t)pc.G * pc.exit_cap;
     const int kBuildCnt = MIN ? kCtlCnt1 : kCtlCnt2;
     k_exit_build<MIN><<<persistent_grid((const void*)k_exit_build<MIN>, 256), 256, 0, s>>>(
-        all, total, dq, dk, dr, pc.glist, pc.gctl + kBuildCnt);
+        all, total, pc.glist, pc.gcq, pc.gcq_k, pc.gctl + kBuildCnt);
     LF_CUDA(cudaGetLastError());
-    LF_CUDA(cudaFreeAsync(tabs, s));
     ForestArgs g;
     memset(&g, 0, sizeof(g));
     g.N = N;
@@ -1666,6 +1742,8 @@ static int exit_pass(const ForestArgs& a, const int32_t* list, const int* count,
     }
     g.list1 = pc.glist;
     g.list2 = pc.glist;
+    g.cq = pc.gcq;
+    g.cq_k = pc.gcq_k;
     g.ctl = pc.gctl;
     g.cyc_k = pc.gcyc;
     g.end2 = pc.gend;
@@ -1718,6 +1796,8 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
     a.ekb = w.ekb - lo;
     a.list1 = w.list1;
     a.list2 = w.list2;
+    a.cq = w.cq;
+    a.cq_k = w.cq_k;
     a.ctl = w.ctl;
     a.path_id = path_id - lo;
     a.pos = pos - lo;

@@ -104,6 +104,8 @@ struct ForestWs {
     size_t scan_tmp_bytes;
     ulonglong2* kraw;      // [N] per-direction min keys after the cycle pass (boundary)
     ulonglong2* ekb;       // [N] slot keys of boundary vertices
+    int2* cq;              // [list position] reduced-graph records of the boundary list being
+    ulonglong2* cq_k;      //   scanned: stride pointers (vertex ids), keys or distances
 };
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w);
 
@@ -126,6 +128,8 @@ struct ForestPartCtx {
     int2* gend;
     int2* gdist;
     int32_t* glist;              // [G * exit_cap]
+    int2* gcq;                   // [G * exit_cap] exit-graph records at glist positions
+    ulonglong2* gcq_k;
     int* gctl;                   // [256]
     void* rec_send;              // [exit_cap] records
     void* rec_all;               // [G * exit_cap] records

@@ -571,6 +571,8 @@ static int lf_setup(Part* p, cudaStream_t s) {
     TRYL(dalloc(p, &f.gend, N, s));
     TRYL(dalloc(p, &f.gdist, N, s));
     TRYL(dalloc(p, &f.glist, (size_t)p->G * cap, s));
+    TRYL(dalloc(p, &f.gcq, (size_t)p->G * cap, s));
+    TRYL(dalloc(p, &f.gcq_k, (size_t)p->G * cap, s));
     TRYL(dalloc(p, &f.gctl, 256, s));
     char* rs = nullptr;
     TRYL(dalloc(p, &rs, exit_record_bytes() * cap, s));
