@@ -233,6 +233,23 @@ int lf_linear_forest(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t*
     return forest_run(N, pi2, pi2_w, forest, path_id, pos, perm, iperm, n_cycles, w, (cudaStream_t)stream);
 }
 
+int lf_linear_forest_tridiag(int64_t N, const int32_t* pi2, const float* pi2_w, const float* pi2_val,
+                             const float* diag, int32_t* forest, int32_t* path_id, int32_t* pos,
+                             int32_t* perm, int32_t* iperm, float* a, float* b, float* c, int64_t* n_cycles,
+                             void* ws, size_t ws_bytes, void* stream) {
+    g_err[0] = 0;
+    if (N < 0 || N >= ((int64_t)1 << 31)) return set_error(LF_EINVAL, "lf_linear_forest_tridiag: bad N");
+    if (N > 0 && (!pi2 || !pi2_w || !pi2_val || !diag || !forest || !path_id || !pos || !perm || !iperm || !a ||
+                  !b || !c))
+        return set_error(LF_EINVAL, "lf_linear_forest_tridiag: NULL argument");
+    Carve cv(ws, ws_bytes);
+    ForestWs w;
+    forest_ws_carve(cv, N, &w);
+    if (N > 0 && (!ws || !cv.ok())) return set_error(LF_ENOMEM, "lf_linear_forest_tridiag: workspace too small");
+    const TriOut tri{pi2_val, diag, a, b, c};
+    return forest_run(N, pi2, pi2_w, forest, path_id, pos, perm, iperm, n_cycles, w, (cudaStream_t)stream, &tri);
+}
+
 int lf_forest_stats(int64_t N, void* ws, size_t ws_bytes, int32_t* out, int cap) {
     g_err[0] = 0;
     Carve c(ws, ws_bytes);
@@ -322,10 +339,8 @@ int lf_pipeline_host(const lf_csr_t* Ah, const lf_factor_opts_t* opts, int32_t* 
     lf_csr_t Ad{N, Ah->nnz, p.rowptr, p.col, p.val};
     int rc = lf_factor(&Ad, 2, opts, p.pi, p.pi_w, p.pi_val, p.diag, nullptr, nullptr, p.ws, p.ws_bytes, stream);
     if (rc) return rc;
-    rc = lf_linear_forest(N, p.pi, p.pi_w, p.forest, p.path_id, p.pos, p.perm, p.iperm, nullptr, p.ws,
-                          p.ws_bytes, stream);
-    if (rc) return rc;
-    rc = lf_tridiag(N, p.forest, p.iperm, p.pi, p.pi_val, p.diag, p.a, p.b, p.c, stream);
+    rc = lf_linear_forest_tridiag(N, p.pi, p.pi_w, p.pi_val, p.diag, p.forest, p.path_id, p.pos, p.perm,
+                                  p.iperm, p.a, p.b, p.c, nullptr, p.ws, p.ws_bytes, stream);
     if (rc) return rc;
     struct {
         void* h;

@@ -56,6 +56,7 @@ constexpr int kCtlRed1 = 0;       // ctl[0..63]   per-step not-done counts, redu
 constexpr int kCtlRed2 = 64;      // ctl[64..127] reduced scan 2
 constexpr int kCtlCnt1 = 128;     // boundary list sizes
 constexpr int kCtlCnt2 = 129;
+constexpr int kCtlTicket3 = 130;  // finished-CTA ticket of k_path_offsets (the last one scans tsum)
 constexpr int kMaxSteps = 62;
 constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
 // ctl[192] splitter nodes (cycle pass), [193] unvisited vertices (fallback), [194] tiles
@@ -278,6 +279,57 @@ __device__ __forceinline__ int block_scan_max_excl(int x, int* sh) {
     }
     __syncthreads();
     return w > 0 ? max(exc, sh[w - 1]) : exc;
+}
+
+// exclusive block sum-scan with a single barrier: each warp reads the other warps' sums
+// itself.  *total = the block's sum.  sh must not be reused before another barrier.
+__device__ __forceinline__ int block_scan_sum_excl1(int x, int* sh, int* total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int nw = (int)(blockDim.x >> 5);
+    int inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) sh[w] = inc;
+    __syncthreads();
+    const int ws = lane < nw ? sh[lane] : 0;
+    int before = lane < w ? ws : 0, all = ws;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        before += __shfl_xor_sync(0xffffffffu, before, o);
+        all += __shfl_xor_sync(0xffffffffu, all, o);
+    }
+    *total = all;
+    return inc - x + before;
+}
+
+// exclusive block sum-scan (over threads 0..tid-1); *total = the block's sum
+__device__ __forceinline__ int block_scan_sum_excl(int x, int* sh, int* total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) sh[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+        int t = lane < (int)(blockDim.x >> 5) ? sh[lane] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, t, o);
+            if (lane >= o) t += y;
+        }
+        sh[lane] = t;
+    }
+    __syncthreads();
+    const int res = inc - x + (w > 0 ? sh[w - 1] : 0);
+    *total = sh[31];
+    __syncthreads();
+    return res;
 }
 
 __device__ __forceinline__ int block_scan_min_rev(int x, int* sh) {
@@ -781,6 +833,7 @@ struct ForestArgs {
     int32_t* path_id;
     int32_t* pos;
     int32_t* len;
+    uint8_t* pdir;         // [N] forest slot toward the path-ID end
     unsigned long long* n_cycles;
     int max_steps;
 };
@@ -1354,22 +1407,126 @@ __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
                 D[i] = d;
             }
         }
-        int32_t l, pp;
-        if (E[0] <= E[1]) { l = E[0]; pp = D[0] + 1; } else { l = E[1]; pp = D[1] + 1; }
+        // the ID end l and the forest slot leading to it (the predecessor at p - 1)
+        const int dir = E[0] <= E[1] ? 0 : 1;
+        const int32_t l = E[dir];
         a.path_id[g] = l;
-        a.pos[g] = pp;
+        a.pos[g] = D[dir] + 1;
+        if (a.pdir) a.pdir[g] = (uint8_t)dir;
         a.len[g] = (l == g) ? (D[0] + D[1] + 1) : 0;
     }
 }
 
-// step (3): new(v) = off[l(v)] + p(v) - 1
-__global__ void k_perm(int64_t N, const int32_t* __restrict__ path_id, const int32_t* __restrict__ pos,
-                       const int32_t* __restrict__ off, int32_t* perm, int32_t* iperm) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N;
-         v += (int64_t)gridDim.x * blockDim.x) {
-        const int32_t r = __ldg(off + __ldg(path_id + v)) + __ldg(pos + v) - 1;
-        iperm[v] = r;
-        perm[r] = (int32_t)v;
+// Path offsets, single pass: CTA c scans the path lengths of chunk c (kOffChunk vertices,
+// in id order) into intra-chunk exclusive offsets and publishes the chunk total; the CTA
+// that finishes last turns the totals into an exclusive prefix (tbase).  off[l] of a path
+// ID l is then tbase[l / kOffChunk] + off[l].
+constexpr int kOffT = 1024, kOffPT = 8, kOffChunk = kOffT * kOffPT;
+
+__global__ void __launch_bounds__(kOffT) k_path_offsets(int64_t N, const int32_t* __restrict__ len,
+                                                         int32_t* __restrict__ off, int32_t* tbase,
+                                                         int* ticket) {
+    __shared__ int sh[32];
+    __shared__ int last;
+    const int64_t c0 = (int64_t)blockIdx.x * kOffChunk + (int64_t)threadIdx.x * kOffPT;
+    int x[kOffPT];
+    int sum = 0;
+    if (c0 + kOffPT <= N) {
+        const int4* p = reinterpret_cast<const int4*>(len + c0);
+#pragma unroll
+        for (int j = 0; j < kOffPT / 4; j++) {
+            const int4 q = __ldg(p + j);
+            x[4 * j] = q.x; x[4 * j + 1] = q.y; x[4 * j + 2] = q.z; x[4 * j + 3] = q.w;
+        }
+    } else {
+#pragma unroll
+        for (int j = 0; j < kOffPT; j++) x[j] = c0 + j < N ? __ldg(len + c0 + j) : 0;
+    }
+#pragma unroll
+    for (int j = 0; j < kOffPT; j++) sum += x[j];
+    int total = 0;
+    int run = block_scan_sum_excl1(sum, sh, &total);
+    if (c0 + kOffPT <= N) {
+        int4* p = reinterpret_cast<int4*>(off + c0);
+#pragma unroll
+        for (int j = 0; j < kOffPT / 4; j++) {
+            int4 q;
+            q.x = run; run += x[4 * j];
+            q.y = run; run += x[4 * j + 1];
+            q.z = run; run += x[4 * j + 2];
+            q.w = run; run += x[4 * j + 3];
+            p[j] = q;
+        }
+    } else {
+#pragma unroll
+        for (int j = 0; j < kOffPT; j++) {
+            if (c0 + j < N) off[c0 + j] = run;
+            run += x[j];
+        }
+    }
+    if (threadIdx.x == 0) {
+        tbase[blockIdx.x] = total;
+        __threadfence();
+        last = atomicAdd(ticket, 1) == (int)gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    __syncthreads();  // sh is reused below
+    int carry = 0;
+    for (int base = 0; base < (int)gridDim.x; base += kOffT) {
+        const int i = base + threadIdx.x;
+        const int v = i < (int)gridDim.x ? __ldcg(tbase + i) : 0;
+        int chunk = 0;
+        const int ex = block_scan_sum_excl(v, sh, &chunk);
+        if (i < (int)gridDim.x) tbase[i] = carry + ex;
+        carry += chunk;
+    }
+}
+
+// step (3) (+ step (4) when tri): r = new(v) = off[l(v)] + p(v) - 1 with off[l] = tile
+// prefix + intra-tile prefix; the forest neighbour in slot pdir[v] is perm[r-1], the other
+// one perm[r+1], so a[r] / c[r] are copied from the factor's signed slot values
+constexpr int kPermBatch = 4;  // vertices per thread per iteration (loads in flight)
+
+__global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __restrict__ path_id,
+                                                  const int32_t* __restrict__ pos,
+                                                  const int32_t* __restrict__ off,
+                                                  const int32_t* __restrict__ tbase,
+                                                  const uint8_t* __restrict__ pdir,
+                                                  const int2* __restrict__ forest, const int2* __restrict__ pi2,
+                                                  const float2* __restrict__ pi2_val,
+                                                  const float* __restrict__ diag, int32_t* __restrict__ perm,
+                                                  int32_t* __restrict__ iperm, float* __restrict__ ta,
+                                                  float* __restrict__ tb, float* __restrict__ tc) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < N; v0 += stride * kPermBatch) {
+        int32_t l[kPermBatch], p[kPermBatch], r[kPermBatch];
+#pragma unroll
+        for (int b = 0; b < kPermBatch; b++) {
+            const int64_t v = v0 + b * stride;
+            l[b] = v < N ? __ldg(path_id + v) : 0;
+            p[b] = v < N ? __ldg(pos + v) : 0;
+        }
+#pragma unroll
+        for (int b = 0; b < kPermBatch; b++) r[b] = __ldg(tbase + l[b] / kOffChunk) + __ldg(off + l[b]) + p[b] - 1;
+#pragma unroll
+        for (int b = 0; b < kPermBatch; b++) {
+            const int64_t v = v0 + b * stride;
+            if (v >= N) continue;
+            iperm[v] = r[b];
+            perm[r[b]] = (int32_t)v;
+            if (ta) {
+                const int2 f = __ldg(forest + v);
+                const int2 pn = __ldg(pi2 + v);
+                const float2 pv = __ldg(pi2_val + v);
+                const int d = __ldg(pdir + v);
+                const int32_t pred = d ? f.y : f.x, succ = d ? f.x : f.y;
+                ta[r[b]] = pred >= 0 ? ((pn.x == pred) ? pv.x : pv.y) : 0.0f;
+                tc[r[b]] = succ >= 0 ? ((pn.x == succ) ? pv.x : pv.y) : 0.0f;
+                tb[r[b]] = __ldg(diag + v);
+            }
+        }
     }
 }
 
@@ -1408,6 +1565,8 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     t.kraw = c.take<ulonglong2>(n);
     t.ekb = c.take<ulonglong2>(n);
     t.cq = c.take<int2>(n);
+    t.pdir = c.take<uint8_t>(n);
+    t.tsum = c.take<int32_t>(n / kOffChunk + 2);
     t.cq_k = c.take<ulonglong2>(n);
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
@@ -1448,7 +1607,7 @@ static int forest_prepare() {
 
 int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
                int32_t* pos, int32_t* perm, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
-               cudaStream_t s) {
+               cudaStream_t s, const TriOut* tri) {
     if (N == 0) {
         if (n_cycles) LF_CUDA(cudaMemsetAsync(n_cycles, 0, sizeof(int64_t), s));
         return LF_OK;
@@ -1486,6 +1645,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     a.path_id = path_id;
     a.pos = pos;
     a.len = w.len;
+    a.pdir = w.pdir;
     a.n_cycles = (unsigned long long*)n_cycles;
     a.max_steps = max_steps_for(N) < kMaxSteps ? max_steps_for(N) : kMaxSteps;
     const int tiles = (int)((N + LB - 1) / LB);
@@ -1516,12 +1676,16 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("path_offsets", -1, s);
-        size_t tb = w.scan_tmp_bytes;
-        LF_CUDA(cub::DeviceScan::ExclusiveSum(w.scan_tmp, tb, w.len, w.off, (int)N, s));
+        const int chunks = (int)((N + kOffChunk - 1) / kOffChunk);
+        k_path_offsets<<<chunks, kOffT, 0, s>>>(N, w.len, w.off, w.tsum, w.ctl + kCtlTicket3);
+        LF_CUDA(cudaGetLastError());
     }
     {
-        LF_PROF("perm", -1, s);
-        k_perm<<<persistent_grid((const void*)k_perm, 256), 256, 0, s>>>(N, path_id, pos, w.off, perm, iperm);
+        LF_PROF(tri ? "perm_tridiag" : "perm", -1, s);
+        k_perm_tri<<<persistent_grid((const void*)k_perm_tri, 256), 256, 0, s>>>(
+            N, path_id, pos, w.off, w.tsum, w.pdir, (const int2*)forest, (const int2*)pi2,
+            tri ? (const float2*)tri->pi2_val : nullptr, tri ? tri->diag : nullptr, perm, iperm,
+            tri ? tri->a : nullptr, tri ? tri->b : nullptr, tri ? tri->c : nullptr);
         LF_CUDA(cudaGetLastError());
     }
     return LF_OK;
@@ -1802,6 +1966,7 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
     a.path_id = path_id - lo;
     a.pos = pos - lo;
     a.len = w.len - lo;
+    a.pdir = w.pdir - lo;
     a.n_cycles = (unsigned long long*)&pc.tot[pc.G + 1];
     a.ghost_list = pc.ghost_list;
     a.n_ghost = pc.n_ghost;

@@ -104,6 +104,8 @@ struct ForestWs {
     size_t scan_tmp_bytes;
     ulonglong2* kraw;      // [N] per-direction min keys after the cycle pass (boundary)
     ulonglong2* ekb;       // [N] slot keys of boundary vertices
+    uint8_t* pdir;         // [N] forest slot toward the path-ID end (predecessor slot)
+    int32_t* tsum;         // [chunks + 2] path-length sums per offset chunk -> exclusive prefix
     int2* cq;              // [list position] reduced-graph records of the boundary list being
     ulonglong2* cq_k;      //   scanned: stride pointers (vertex ids), keys or distances
 };
@@ -147,9 +149,15 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
                     int32_t* pos, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
                     const ForestPartCtx& pc, cudaStream_t s);
 
+// optional fused tridiagonal copy at the end of forest_run (all NULL: none)
+struct TriOut {
+    const float* pi2_val;
+    const float* diag;
+    float *a, *b, *c;
+};
 int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
                int32_t* pos, int32_t* perm, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
-               cudaStream_t s);
+               cudaStream_t s, const TriOut* tri = nullptr);
 
 int forest_stats(const ForestWs& w, int32_t* out, int cap);
 

@@ -19,7 +19,7 @@ ERRORS = {-1: "LF_EINVAL", -2: "LF_ENOMEM", -3: "LF_ECUDA", -4: "LF_ENCCL", -5: 
 # every symbol include/lf.h declares (checked by tests/test_abi.py)
 EXPORTS = (
     "lf_factor_opts_default", "lf_factor_workspace_size", "lf_factor",
-    "lf_linear_forest_workspace_size", "lf_linear_forest", "lf_tridiag",
+    "lf_linear_forest_workspace_size", "lf_linear_forest", "lf_tridiag", "lf_linear_forest_tridiag",
     "lf_pipeline_workspace_size", "lf_pipeline_host", "lf_validate_csr",
     "lf_last_error", "lf_version", "lf_profile_enable", "lf_profile_collect",
     "lf_forest_stats", "lf_comm_nccl_unique_id", "lf_comm_create_nccl", "lf_comm_create_loopback",
@@ -62,6 +62,7 @@ def load(path: str = LIB_PATH):
     L.lf_linear_forest_workspace_size.restype = C.c_size_t
     L.lf_linear_forest.argtypes = [I64, P, P, P, P, P, P, P, P, P, C.c_size_t, P]
     L.lf_tridiag.argtypes = [I64, P, P, P, P, P, P, P, P, P]
+    L.lf_linear_forest_tridiag.argtypes = [I64, P, P, P, P, P, P, P, P, P, P, P, P, P, P, C.c_size_t, P]
     L.lf_pipeline_workspace_size.argtypes = [I64, I64]
     L.lf_pipeline_workspace_size.restype = C.c_size_t
     L.lf_pipeline_host.argtypes = [P, P, P, P, P, P, P, P, P, C.c_size_t, P]
@@ -200,6 +201,34 @@ def tridiag(forest, iperm, pi2, pi2_val, diag, *, out=None):
     return a, b, c
 
 
+def linear_forest_tridiag(pi2, pi2_w, pi2_val, diag, *, ws=None, out=None, n_cycles=True):
+    """lf_linear_forest_tridiag -> dict(forest, path_id, pos, perm, iperm, a, b, c, n_cycles)."""
+    torch = _torch()
+    L = load()
+    N = pi2.shape[0]
+    dev = pi2.device
+    if out is None:
+        out = dict(
+            forest=torch.empty((N, 2), dtype=torch.int32, device=dev),
+            path_id=torch.empty(N, dtype=torch.int32, device=dev),
+            pos=torch.empty(N, dtype=torch.int32, device=dev),
+            perm=torch.empty(N, dtype=torch.int32, device=dev),
+            iperm=torch.empty(N, dtype=torch.int32, device=dev),
+            a=torch.empty(N, dtype=torch.float32, device=dev),
+            b=torch.empty(N, dtype=torch.float32, device=dev),
+            c=torch.empty(N, dtype=torch.float32, device=dev),
+            n_cycles=torch.zeros(1, dtype=torch.int64, device=dev) if n_cycles else None,
+        )
+    nb = L.lf_linear_forest_workspace_size(N)
+    buf = (ws or _ws).get(nb)
+    _check(L.lf_linear_forest_tridiag(N, _ptr(pi2), _ptr(pi2_w), _ptr(pi2_val), _ptr(diag),
+                                      _ptr(out["forest"]), _ptr(out["path_id"]), _ptr(out["pos"]),
+                                      _ptr(out["perm"]), _ptr(out["iperm"]), _ptr(out["a"]),
+                                      _ptr(out["b"]), _ptr(out["c"]), _ptr(out["n_cycles"]), _ptr(buf),
+                                      nb, _stream()))
+    return out
+
+
 @dataclass
 class Pipeline:
     """Preallocated device buffers for the whole hot path on one graph (n=2)."""
@@ -221,7 +250,7 @@ class Pipeline:
         self.ws_l = Workspace()
         self.fac = None
         self.lf = None
-        self.tri = tuple(torch.empty(N, dtype=torch.float32, device="cuda") for _ in range(3))
+        self.tri = None
 
     def run_factor(self):
         self.fac = factor(self.rowptr, self.col, self.val, 2, M=self.M, m=self.m, k_m=self.k_m,
@@ -229,17 +258,15 @@ class Pipeline:
         return self.fac
 
     def run_forest(self):
-        self.lf = linear_forest(self.fac["pi"], self.fac["pi_w"], ws=self.ws_l, out=self.lf)
+        """Linear forest + tridiagonal copy (one fused call)."""
+        self.lf = linear_forest_tridiag(self.fac["pi"], self.fac["pi_w"], self.fac["pi_val"],
+                                        self.fac["diag"], ws=self.ws_l, out=self.lf)
+        self.tri = (self.lf["a"], self.lf["b"], self.lf["c"])
         return self.lf
-
-    def run_tridiag(self):
-        return tridiag(self.lf["forest"], self.lf["iperm"], self.fac["pi"], self.fac["pi_val"],
-                       self.fac["diag"], out=self.tri)
 
     def run(self):
         self.run_factor()
         self.run_forest()
-        self.run_tridiag()
         return self
 
 

@@ -98,6 +98,15 @@ def check_forest(torch, lfm, oracle_mod, A, fac, ref):
     ta, tb, tc = oracle_mod.tridiag(A, o["forest"], o["perm"])
     for g, e in ((a, ta), (b, tb), (c, tc)):
         assert np.array_equal(g.cpu().numpy().view(np.uint32), e.view(np.uint32))
+    # the fused call (what the pipeline / bench run) gives the same outputs
+    fu = lfm.linear_forest_tridiag(fac["pi"], fac["pi_w"], fac["pi_val"], fac["diag"])
+    torch.cuda.synchronize()
+    for k in ("forest", "path_id", "pos", "perm", "iperm"):
+        got = fu[k].cpu().numpy()
+        assert np.array_equal(got, o[k]), f"fused {k} mismatch: first at {np.argwhere(got != o[k])[:3].ravel()}"
+    assert int(fu["n_cycles"].item()) == o["n_cycles"]
+    for g, e in ((fu["a"], ta), (fu["b"], tb), (fu["c"], tc)):
+        assert np.array_equal(g.cpu().numpy().view(np.uint32), e.view(np.uint32)), "fused tridiag mismatch"
     return lf_out
 
 
