@@ -806,8 +806,12 @@ struct ForestArgs {
     const int32_t* ghost_list;
     int64_t n_ghost, ghost_below;
     const int2* ghost_nb;  // [local id] slots (global ids) of ghost vertices
-    ulonglong2* kraw;      // [v] final per-direction min keys of the cycle pass (boundary)
-    ulonglong2* ekb;       // [v] slot keys of boundary vertices
+    // results of the reduced scans are stored at list positions (compact, coalesced);
+    // bidx1 / bidx2 map a boundary vertex to its position in list1 / list2
+    int32_t* bidx1;        // [v] list1 position of a boundary vertex of the cycle pass
+    int32_t* bidx2;        // [v] list2 position of a boundary vertex of the rank pass
+    ulonglong2* kraw;      // [list1 pos] final per-direction min keys of the cycle pass
+    ulonglong2* ekb;       // [list1 pos] slot keys of boundary vertices
     const int2* __restrict__ pi2;
     const float2* __restrict__ pi2_w;
     int2* forest;
@@ -818,13 +822,13 @@ struct ForestArgs {
     // reduced graph, pass 1 (cycles)
     int2* rq1[2];
     ulonglong2* rk1[2];
-    uint64_t* cyc_k;       // [N] weakest key of the global cycle through a boundary vertex
+    uint64_t* cyc_k;       // [list1 pos] weakest key of the global cycle through it
     int32_t* list1;
     // reduced graph, pass 2 (positions)
     int2* rq2[2];
     int2* rr2[2];
-    int2* end2;            // [N] path ends per direction of a boundary vertex
-    int2* dist2;           // [N] distances to them
+    int2* end2;            // [list2 pos] path ends per direction of a boundary vertex
+    int2* dist2;           // [list2 pos] distances to them
     int32_t* list2;
     // compact records of the list being built / scanned (list position -> record)
     int2* cq;              // stride pointers (vertex ids or markers)
@@ -971,7 +975,8 @@ __global__ void __launch_bounds__(LT, 1) k_lf_local1(ForestArgs a) {
             ulonglong2 rk;
             rk.x = (nb.x < 0 || is_foreign(nb.x, a)) ? KEY_INF : (r0 ? ek[k].x : K[k].x);
             rk.y = (nb.y < 0 || is_foreign(nb.y, a)) ? KEY_INF : (r1 ? ek[k].y : K[k].y);
-            if (a.ekb) a.ekb[g] = ek[k];
+            if (a.ekb) a.ekb[idx] = ek[k];
+            a.bidx1[g] = idx;
             a.cq[idx] = make_int2(q0, q1);
             a.cq_k[idx] = rk;
         }
@@ -1065,12 +1070,12 @@ __device__ __forceinline__ void red_epilogue(const ForestArgs& a, const int32_t*
         if (MIN) {
             const int2 q = a.rq1[fb][v];
             const ulonglong2 k = a.rk1[fb][v];
-            a.cyc_k[v] = (q.x >= 0 && q.y >= 0) ? umin64(k.x, k.y) : KEY_INF;
-            a.end2[v] = q;  // raw markers (exit list construction)
-            if (a.kraw) a.kraw[v] = k;
+            a.cyc_k[idx] = (q.x >= 0 && q.y >= 0) ? umin64(k.x, k.y) : KEY_INF;
+            a.end2[idx] = q;  // raw markers (exit list construction)
+            if (a.kraw) a.kraw[idx] = k;
         } else {
-            a.end2[v] = a.rq2[fb][v];  // raw end markers -(e+1) (or exit markers)
-            a.dist2[v] = a.rr2[fb][v];
+            a.end2[idx] = a.rq2[fb][v];  // raw end markers -(e+1) (or exit markers)
+            a.dist2[idx] = a.rr2[fb][v];
         }
     }
 }
@@ -1086,7 +1091,8 @@ static_assert((kRedHash & (kRedHash - 1)) == 0, "hash table size must be a power
 // smem image of a small reduced graph (pointers are list positions or end markers)
 struct RedSmem {
     int2 q[kRedSmall];
-    ulonglong2 k[kRedSmall];  // MIN: min keys; ADD: distances in .x/.y low words
+    uint64_t k0[kRedSmall];   // MIN: min keys per direction; ADD: distances (low words)
+    uint64_t k1[kRedSmall];
     int32_t v[kRedSmall];     // vertex id of each list position
     int2 ht[kRedHash];        // (vertex, list position), vertex -1 = empty
 };
@@ -1163,7 +1169,8 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
         if (q[k].y >= 0) q[k].y = red_lookup(S, q[k].y);
         fin[k] = q[k].x < 0 && q[k].y < 0;
         S.q[tid + k * T] = q[k];
-        S.k[tid + k * T] = kk[k];
+        S.k0[tid + k * T] = kk[k].x;
+        S.k1[tid + k * T] = kk[k].y;
     }
     RS_MARK(1);
     int step = 0;
@@ -1191,8 +1198,7 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
                     if (j < 0) continue;  // stall (reading c13)
                     const int tgt = j ? qw.y : qw.x;
                     if (i) nq[k].y = tgt; else nq[k].x = tgt;
-                    const ulonglong2 kw = S.k[w];
-                    const uint64_t kv = j ? kw.y : kw.x;
+                    const uint64_t kv = j ? S.k1[w] : S.k0[w];
                     if (MIN) { if (i) nk[k].y = umin64(nk[k].y, kv); else nk[k].x = umin64(nk[k].x, kv); }
                     else { if (i) nk[k].y += kv; else nk[k].x += kv; }
                 }
@@ -1206,7 +1212,8 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
                 q[k] = nq[k];
                 kk[k] = nk[k];
                 S.q[me] = q[k];
-                S.k[me] = kk[k];
+                S.k0[me] = kk[k].x;
+                S.k1[me] = kk[k].y;
                 fin[k] = q[k].x < 0 && q[k].y < 0;
                 bool cyc_done = false;
                 if (MIN) cyc_done = q[k].x >= 0 && q[k].y >= 0 && (kk[k].x == kk[k].y || q[k].x == q[k].y);
@@ -1223,13 +1230,14 @@ __device__ void red_scan_small(const ForestArgs& a, const int32_t* list, int cnt
         if (v[k] < 0) continue;
         // pointers back to vertex ids (markers pass through unchanged)
         const int2 qg = make_int2(q[k].x >= 0 ? S.v[q[k].x] : q[k].x, q[k].y >= 0 ? S.v[q[k].y] : q[k].y);
+        const int idx = tid + k * T;
         if (MIN) {
-            a.cyc_k[v[k]] = (q[k].x >= 0 && q[k].y >= 0) ? umin64(kk[k].x, kk[k].y) : KEY_INF;
-            a.end2[v[k]] = qg;
-            if (a.kraw) a.kraw[v[k]] = kk[k];
+            a.cyc_k[idx] = (q[k].x >= 0 && q[k].y >= 0) ? umin64(kk[k].x, kk[k].y) : KEY_INF;
+            a.end2[idx] = qg;
+            if (a.kraw) a.kraw[idx] = kk[k];
         } else {
-            a.end2[v[k]] = qg;
-            a.dist2[v[k]] = make_int2((int)kk[k].x, (int)kk[k].y);
+            a.end2[idx] = qg;
+            a.dist2[idx] = make_int2((int)kk[k].x, (int)kk[k].y);
         }
     }
     RS_MARK(3);
@@ -1320,7 +1328,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
                 const int2 nbt = s.nb[t];
                 const int so = (t == u) ? i : outward_slot(nbt, T);
                 const int32_t xo = so ? nbt.y : nbt.x;
-                if (xo >= 0 && kstar == KEY_INF) kstar = a.cyc_k[b0 + t];
+                if (xo >= 0 && kstar == KEY_INF) kstar = a.cyc_k[a.bidx1[b0 + t]];
             }
         }
         if (kstar != KEY_INF) {
@@ -1364,6 +1372,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
         }
         const int idx = list_append(a.list2, &a.ctl[kCtlCnt2], g, boundary);
         if (boundary) {
+            a.bidx2[g] = idx;
             int32_t q0, q1, d0, d1;
             reduced_dir(a, s, b0, g, nb, 0, P[k], R[k], q0, d0);
             reduced_dir(a, s, b0, g, nb, 1, P[k], R[k], q1, d1);
@@ -1398,8 +1407,9 @@ __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
             const int so = (t == u) ? i : outward_slot(nbt, T);
             const int32_t xo = so ? nbt.y : nbt.x;
             if (xo >= 0) {  // continues in another block: reduced result of t (end marker)
-                const int2 e = a.end2[b0 + t];
-                const int2 dd = a.dist2[b0 + t];
+                const int bi = a.bidx2[b0 + t];
+                const int2 e = a.end2[bi];
+                const int2 dd = a.dist2[bi];
                 E[i] = -((so ? e.y : e.x) + 1);
                 D[i] = d + (so ? dd.y : dd.x);
             } else {
@@ -1565,6 +1575,8 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     t.kraw = c.take<ulonglong2>(n);
     t.ekb = c.take<ulonglong2>(n);
     t.cq = c.take<int2>(n);
+    t.bidx1 = c.take<int32_t>(n);
+    t.bidx2 = c.take<int32_t>(n);
     t.pdir = c.take<uint8_t>(n);
     t.tsum = c.take<int32_t>(n / kOffChunk + 2);
     t.cq_k = c.take<ulonglong2>(n);
@@ -1632,6 +1644,8 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         a.rr2[i] = w.rr2[i];
     }
     a.cyc_k = w.cyc_k;
+    a.bidx1 = w.bidx1;
+    a.bidx2 = w.bidx2;
     a.loc1 = w.loc1;
     a.kst = w.kst;
     a.loc2 = w.loc2;
@@ -1747,7 +1761,7 @@ __global__ void k_exit_records(ForestArgs a, const int32_t* list, const int* cou
             if (take) {
                 r.g = v;
                 r.pad = 0;
-                const int2 raw = a.end2[v];
+                const int2 raw = a.end2[idx];
                 int32_t q[2], d[2];
                 uint64_t k[2];
 #pragma unroll
@@ -1760,12 +1774,12 @@ __global__ void k_exit_records(ForestArgs a, const int32_t* list, const int* cou
                     else if (fx) {
                         q[i] = x;
                         d[i] = 1;
-                        if (MIN) k[i] = i ? a.ekb[v].y : a.ekb[v].x;
+                        if (MIN) k[i] = i ? a.ekb[idx].y : a.ekb[idx].x;
                     } else {
                         const int32_t m = i ? raw.y : raw.x;
                         q[i] = is_exit_marker(m, a.N) ? exit_vertex(m, a.N) : m;
-                        if (MIN) k[i] = i ? a.kraw[v].y : a.kraw[v].x;
-                        else d[i] = i ? a.dist2[v].y : a.dist2[v].x;
+                        if (MIN) k[i] = i ? a.kraw[idx].y : a.kraw[idx].x;
+                        else d[i] = i ? a.dist2[idx].y : a.dist2[idx].x;
                     }
                 }
                 r.q0 = q[0]; r.q1 = q[1];
@@ -1785,12 +1799,13 @@ __global__ void k_exit_records(ForestArgs a, const int32_t* list, const int* cou
 // the exit graph from the gathered records of all ranks (padding has g = -1)
 template <bool MIN>
 __global__ void k_exit_build(const ExitRec* rec, int64_t total, int32_t* glist, int2* gcq, ulonglong2* gcq_k,
-                             int* gcount) {
+                             int32_t* gbidx, int* gcount) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
         const ExitRec r = rec[i];
         if (r.g < 0) continue;
         const int pos = atomicAdd(gcount, 1);
         glist[pos] = r.g;
+        gbidx[r.g] = pos;
         gcq[pos] = make_int2(r.q0, r.q1);
         gcq_k[pos] = MIN ? make_ulonglong2(r.k0, r.k1) : make_ulonglong2((uint32_t)r.d0, (uint32_t)r.d1);
     }
@@ -1799,30 +1814,31 @@ __global__ void k_exit_build(const ExitRec* rec, int64_t total, int32_t* glist, 
 // exit marker at t -> the global result of t through its cross-rank slot
 template <bool MIN>
 __global__ void k_exit_fold(ForestArgs a, const int32_t* list, const int* count, const uint64_t* gcyc,
-                            const int2* gend, const int2* gdist) {
+                            const int2* gend, const int2* gdist, const int32_t* gbidx) {
     const int cnt = *count;
     for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < cnt; idx += gridDim.x * blockDim.x) {
         const int32_t b = list[idx];
-        int2 raw = a.end2[b];
-        int2 dd = MIN ? make_int2(0, 0) : a.dist2[b];
+        int2 raw = a.end2[idx];
+        int2 dd = MIN ? make_int2(0, 0) : a.dist2[idx];
 #pragma unroll
         for (int i = 0; i < 2; i++) {
             const int32_t m = i ? raw.y : raw.x;
             if (!is_exit_marker(m, a.N)) continue;
             const int32_t t = exit_vertex(m, a.N);
+            const int gi = gbidx[t];
             if (MIN) {
-                if (gcyc[t] != KEY_INF) a.cyc_k[b] = gcyc[t];
+                if (gcyc[gi] != KEY_INF) a.cyc_k[idx] = gcyc[gi];
             } else {
                 const int2 nt = a.forest[t];
                 const int so = (t == b) ? i : ((nt.x >= 0 && is_foreign(nt.x, a)) ? 0 : 1);
-                const int32_t e = so ? gend[t].y : gend[t].x;
-                const int32_t dg = so ? gdist[t].y : gdist[t].x;
+                const int32_t e = so ? gend[gi].y : gend[gi].x;
+                const int32_t dg = so ? gdist[gi].y : gdist[gi].x;
                 if (i) { raw.y = e; dd.y += dg; } else { raw.x = e; dd.x += dg; }
             }
         }
         if (!MIN) {
-            a.end2[b] = raw;
-            a.dist2[b] = dd;
+            a.end2[idx] = raw;
+            a.dist2[idx] = dd;
         }
     }
 }
@@ -1848,7 +1864,7 @@ __global__ void k_publish(const int32_t* glist, const int* gcount, const int2* g
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
         const int32_t g = glist[i];
         if (g < lo || g >= hi) continue;  // each path with an own ID has an own exit vertex
-        const int2 e = gend[g];
+        const int2 e = gend[i];
         const int32_t e0 = -(e.x + 1), e1 = -(e.y + 1);
         const int32_t l = e0 < e1 ? e0 : e1;
         if (l >= lo && l < hi) pub[atomicAdd(pcount, 1)] = make_int2(l, (int32_t)(tot[G] + off_own[l]));
@@ -1891,7 +1907,7 @@ static int exit_pass(const ForestArgs& a, const int32_t* list, const int* count,
     const int64_t total = (int64_t)pc.G * pc.exit_cap;
     const int kBuildCnt = MIN ? kCtlCnt1 : kCtlCnt2;
     k_exit_build<MIN><<<persistent_grid((const void*)k_exit_build<MIN>, 256), 256, 0, s>>>(
-        all, total, pc.glist, pc.gcq, pc.gcq_k, pc.gctl + kBuildCnt);
+        all, total, pc.glist, pc.gcq, pc.gcq_k, pc.gbidx, pc.gctl + kBuildCnt);
     LF_CUDA(cudaGetLastError());
     ForestArgs g;
     memset(&g, 0, sizeof(g));
@@ -1921,7 +1937,7 @@ static int exit_pass(const ForestArgs& a, const int32_t* list, const int* count,
     {
         LF_PROF(MIN ? "exit_fold_cycles" : "exit_fold_ranks", -1, s);
         k_exit_fold<MIN><<<persistent_grid((const void*)k_exit_fold<MIN>, 256), 256, 0, s>>>(
-            a, list, count, pc.gcyc, pc.gend, pc.gdist);
+            a, list, count, pc.gcyc, pc.gend, pc.gdist, pc.gbidx);
         LF_CUDA(cudaGetLastError());
     }
     return LF_OK;
@@ -1950,14 +1966,16 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
         a.rq2[i] = w.rq2[i] - lo;
         a.rr2[i] = w.rr2[i] - lo;
     }
-    a.cyc_k = w.cyc_k - lo;
+    a.cyc_k = w.cyc_k;
+    a.bidx1 = w.bidx1 - lo;
+    a.bidx2 = w.bidx2 - lo;
     a.loc1 = w.loc1 - lo;
     a.kst = w.kst - lo;
     a.loc2 = w.loc2 - lo;
-    a.end2 = w.end2 - lo;
-    a.dist2 = w.dist2 - lo;
-    a.kraw = w.kraw - lo;
-    a.ekb = w.ekb - lo;
+    a.end2 = w.end2;
+    a.dist2 = w.dist2;
+    a.kraw = w.kraw;
+    a.ekb = w.ekb;
     a.list1 = w.list1;
     a.list2 = w.list2;
     a.cq = w.cq;

@@ -92,9 +92,11 @@ struct ForestWs {
     short2* loc1;          // [N] local results of the cycle pass
     uint64_t* kst;         // [N] weakest key of a local cycle
     int2* loc2;            // [N] local results of the rank pass
-    uint64_t* cyc_k;       // [N] weakest edge key of the global cycle through a boundary vertex
-    int2* end2;            // [N] path ends per direction of a boundary vertex
-    int2* dist2;           // [N] distances to them
+    uint64_t* cyc_k;       // [list1 pos] weakest edge key of the global cycle through a boundary vertex
+    int2* end2;            // [list pos] path ends per direction of a boundary vertex
+    int2* dist2;           // [list2 pos] distances to them
+    int32_t* bidx1;        // [N] list1 position of a boundary vertex
+    int32_t* bidx2;        // [N] list2 position of a boundary vertex
     int32_t* list1;        // boundary vertices, cycle pass
     int32_t* list2;        // boundary vertices, rank pass
     int32_t* len;          // [N] path length at the path-ID vertex, else 0
@@ -102,8 +104,8 @@ struct ForestWs {
     int* ctl;              // [256] per-step counters, list sizes
     void* scan_tmp;        // CUB temp storage
     size_t scan_tmp_bytes;
-    ulonglong2* kraw;      // [N] per-direction min keys after the cycle pass (boundary)
-    ulonglong2* ekb;       // [N] slot keys of boundary vertices
+    ulonglong2* kraw;      // [list1 pos] per-direction min keys after the cycle pass
+    ulonglong2* ekb;       // [list1 pos] slot keys of boundary vertices
     uint8_t* pdir;         // [N] forest slot toward the path-ID end (predecessor slot)
     int32_t* tsum;         // [chunks + 2] path-length sums per offset chunk -> exclusive prefix
     int2* cq;              // [list position] reduced-graph records of the boundary list being
@@ -126,9 +128,10 @@ struct ForestPartCtx {
     int2* gq[2];
     ulonglong2* gk[2];
     int2* gr[2];
-    uint64_t* gcyc;
+    uint64_t* gcyc;              // [glist pos] exit-graph results (compact)
     int2* gend;
     int2* gdist;
+    int32_t* gbidx;              // [N] glist position of an exit vertex
     int32_t* glist;              // [G * exit_cap]
     int2* gcq;                   // [G * exit_cap] exit-graph records at glist positions
     ulonglong2* gcq_k;

@@ -567,9 +567,11 @@ static int lf_setup(Part* p, cudaStream_t s) {
         TRYL(dalloc(p, &f.gk[i], N, s));
         TRYL(dalloc(p, &f.gr[i], N, s));
     }
-    TRYL(dalloc(p, &f.gcyc, N, s));
-    TRYL(dalloc(p, &f.gend, N, s));
-    TRYL(dalloc(p, &f.gdist, N, s));
+    const size_t NG = N > (size_t)p->G * cap ? N : (size_t)p->G * cap;  // glist positions
+    TRYL(dalloc(p, &f.gcyc, NG, s));
+    TRYL(dalloc(p, &f.gend, NG, s));
+    TRYL(dalloc(p, &f.gdist, NG, s));
+    TRYL(dalloc(p, &f.gbidx, N, s));
     TRYL(dalloc(p, &f.glist, (size_t)p->G * cap, s));
     TRYL(dalloc(p, &f.gcq, (size_t)p->G * cap, s));
     TRYL(dalloc(p, &f.gcq_k, (size_t)p->G * cap, s));
