@@ -4,6 +4,7 @@
 
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <unordered_map>
@@ -86,6 +87,11 @@ int sm_count() {
     return n;
 }
 
+bool pdl_enabled() {
+    static const bool on = getenv("LF_NO_PDL") == nullptr;
+    return on;
+}
+
 int persistent_grid(const void* kernel, int block, size_t smem) {
     static std::mutex mu;
     static std::unordered_map<const void*, int> cache;
@@ -109,11 +115,13 @@ size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w) {
     t.prop_v = c.take<float>(nn * n);
     t.wl[0] = c.take<int32_t>(nn);
     t.wl[1] = c.take<int32_t>(nn);
+    // control block, contiguous so that one memset clears it: counts | flags | long_count |
+    // live_part (the factor zeroes up to live_part + 128 M)
     t.counts = c.take<int32_t>(4);
     t.flags = c.take<int>(kMaxFlagRounds);
-    t.long_rows = c.take<int32_t>(nn);
     t.long_count = c.take<int32_t>(kMaxFlagRounds);
     t.live_part = c.take<unsigned long long>((size_t)kMaxFlagRounds * 128);
+    t.long_rows = c.take<int32_t>(nn);
     if (w) *w = t;
     return c.off;
 }

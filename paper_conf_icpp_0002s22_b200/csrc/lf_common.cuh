@@ -110,4 +110,9 @@ constexpr uint8_t ST_CHARGE = 0x8;
 // prop_j slot value for a row whose charge-free candidate set is empty (retired)
 constexpr int32_t PROP_RETIRED = -2;
 
+// PDL (see launch_pdl): wait until the stream predecessor grid has completed and its
+// writes are visible (a no-op for an ordinary launch); let the successor grid launch early
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 }  // namespace lf

@@ -171,6 +171,8 @@ __device__ __forceinline__ void propose_phase(const ProposeArgs& a) {
 
 template <int NN, int G>
 __global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
+    pdl_wait();
+    pdl_trigger();
     propose_phase<NN, G>(a);
 }
 
@@ -193,6 +195,17 @@ __device__ __forceinline__ void topn_insert_fast(uint64_t (&t)[NN], uint64_t x) 
         else { t[i] = x; return; }
     }
     t[0] = x;
+}
+
+// branch-free insertion network: t stays sorted descending; x = 0 leaves it unchanged
+template <int NN>
+__device__ __forceinline__ void topn_insert_net(uint64_t (&t)[NN], uint64_t x) {
+#pragma unroll
+    for (int i = 0; i < NN; i++) {
+        const uint64_t h = t[i] > x ? t[i] : x;
+        x = t[i] > x ? x : t[i];
+        t[i] = h;
+    }
 }
 
 #if defined(LF_TILE_MINB) && LF_TILE_MINB > 0
@@ -356,8 +369,14 @@ __device__ __forceinline__ void cp4(void* smem, const void* gmem) {
 __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 __device__ __forceinline__ void cp_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
-constexpr int SPT = 256;      // threads
-constexpr int SETILE = 4096;  // entries per stage
+#ifndef LF_SETILE
+#define LF_SETILE 4096
+#endif
+#ifndef LF_SPT
+#define LF_SPT 256
+#endif
+constexpr int SPT = LF_SPT;         // threads
+constexpr int SETILE = LF_SETILE;   // entries per stage
 
 struct StreamSmem {
     int32_t col[2][SETILE];
@@ -399,6 +418,7 @@ __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
     constexpr int R = SPT / G;
     extern __shared__ __align__(16) unsigned char sraw[];
     StreamSmem& S = *reinterpret_cast<StreamSmem*>(sraw);
+    pdl_trigger();  // the long-row pass may launch and wait meanwhile
     const int tid = threadIdx.x;
     const int64_t ntiles = (a.N + R - 1) / R;
     const int64_t t0 = blockIdx.x;
@@ -450,17 +470,34 @@ __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
 #pragma unroll
         for (int s2 = 0; s2 < NN; s2++) top[s2] = 0;
         uint32_t theta0 = 0, dbits = 0;
-        for (int64_t e = rs + li; e < re; e += G) {
-            int32_t j;
-            uint32_t xb;
-            if (staged) { j = scol[e - a0]; xb = __float_as_uint(sval[e - a0]); }
-            else { j = __ldg(a.col + e); xb = __float_as_uint(__ldg(a.val + e)); }
-            if (j == v) { dbits = xb; continue; }                        // diagonal (L231)
-            const uint32_t ab = xb & 0x7FFFFFFFu;
-            if (ab == 0u) continue;                                      // zero (L31)
-            theta0 = 1;
-            if (CHARGED && (((a.state[j] & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
-            topn_insert_fast<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
+        if (staged) {
+            // branch-free scan of the staged row: 32-bit smem offsets, a rejected entry
+            // becomes key 0, which the insertion network never keeps
+            const int lo = (int)(rs - a0) + li, hi = (int)(re - a0);
+#pragma unroll 4
+            for (int e = lo; e < hi; e += G) {
+                const int32_t j = scol[e];
+                const uint32_t xb = __float_as_uint(sval[e]);
+                const uint32_t ab = xb & 0x7FFFFFFFu;
+                const bool isd = j == v;                                 // diagonal (L231)
+                dbits = isd ? xb : dbits;
+                bool ok = !isd && ab != 0u;                              // zero (L31)
+                theta0 |= ok ? 1u : 0u;
+                if (CHARGED) ok = ok && (((a.state[j] & ST_CHARGE) ? 1u : 0u) != cv);  // L17
+                const uint64_t key = ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31));
+                topn_insert_net<NN>(top, ok ? key : 0ull);
+            }
+        } else {
+            for (int64_t e = rs + li; e < re; e += G) {
+                const int32_t j = __ldg(a.col + e);
+                const uint32_t xb = __float_as_uint(__ldg(a.val + e));
+                if (j == v) { dbits = xb; continue; }                    // diagonal (L231)
+                const uint32_t ab = xb & 0x7FFFFFFFu;
+                if (ab == 0u) continue;                                  // zero (L31)
+                theta0 = 1;
+                if (CHARGED && (((a.state[j] & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
+                topn_insert_fast<NN>(top, ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)));
+            }
         }
         if (G > 1) {
             topn_merge_group<NN, G>(top);
@@ -625,6 +662,7 @@ __device__ __forceinline__ void mutual_phase(const MutualArgs& a) {
 
 template <int NN>
 __global__ void __launch_bounds__(256) k_mutual(MutualArgs a) {
+    pdl_wait();
     mutual_phase<NN>(a);
 }
 
@@ -650,8 +688,12 @@ struct FusedArgs {
 #ifndef LF_FUSED_GRID_SM
 #define LF_FUSED_GRID_SM 1   // one CTA per SM: grid barriers scale with the CTA count
 #endif
+#ifndef LF_FUSED_GRID
+#define LF_FUSED_GRID 0      // > 0: absolute CTA count of the fused rounds kernel
+#endif
 template <int NN, int G>
 __global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {
+    pdl_trigger();  // k_finalize (one CTA) may launch and wait meanwhile
     cg::grid_group grid = cg::this_grid();
     for (int k = 1; k < f.M; k++) {
         ProposeArgs pa = f.pa;
@@ -717,6 +759,7 @@ __global__ void k_diag(int64_t N, const int64_t* __restrict__ rowptr, const int3
 // also sums the live-row counter slots into live[k], live[M+k]
 __global__ void k_finalize(const int* flags, int M, int m, int k_m, int32_t* rounds,
                            const unsigned long long* part, int64_t* live) {
+    pdl_wait();
     if (threadIdx.x == 0 && rounds) {
         int r = M;
         for (int k = 0; k < M; k++)
@@ -840,11 +883,11 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
     const int grid_p = persistent_grid((const void*)k_propose<NN, 32>, 256);
     const int grid_m = persistent_grid((const void*)k_mutual<NN>, 256);
 
-    LF_CUDA(cudaMemsetAsync(w.flags, 0, sizeof(int) * kMaxFlagRounds, s));
-    LF_CUDA(cudaMemsetAsync(w.long_count, 0, sizeof(int32_t) * kMaxFlagRounds, s));
-    LF_CUDA(cudaMemsetAsync(w.counts, 0, sizeof(int32_t) * 4, s));
-    if (live && !o->until_maximal && o->M > 0)
-        LF_CUDA(cudaMemsetAsync(w.live_part, 0, sizeof(unsigned long long) * 128 * o->M, s));
+    {  // one memset for the contiguous control block (counts, flags, long_count, live_part)
+        const bool lv = live && !o->until_maximal && o->M > 0;
+        const char* end = lv ? (const char*)(w.live_part + (size_t)128 * o->M) : (const char*)w.live_part;
+        LF_CUDA(cudaMemsetAsync(w.counts, 0, (size_t)(end - (const char*)w.counts), s));
+    }
     if ((N == 0 && !part) || (!o->until_maximal && o->M == 0)) {
         // no rounds: empty factor (a partition with no rows still takes part in the
         // exchanges below, so it only returns here when there are no rounds at all)
@@ -927,8 +970,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             pl.wl = w.long_rows;
             pl.wl_count = pa.defer_count;
             pl.defer_len = INT64_MAX;
-            k_propose<NN, 32><<<grid_p, 256, 0, s>>>(pl);
-            LF_CUDA(cudaGetLastError());
+            LF_CUDA(launch_pdl(k_propose<NN, 32>, grid_p, 256, 0, s, pl));
         }
 
         if (o->until_maximal && (k % o->m) == o->k_m) {
@@ -977,8 +1019,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         ma.thr = thr;
         {
             LF_PROF("mutual", k, s);
-            k_mutual<NN><<<grid_m, 256, 0, s>>>(ma);
-            LF_CUDA(cudaGetLastError());
+            LF_CUDA(launch_pdl(k_mutual<NN>, grid_m, 256, 0, s, ma));
         }
     }
     if (fuse) {
@@ -1029,7 +1070,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             case 16: kfn = (const void*)k_rounds_fused<NN, 16>; break;
             default: kfn = (const void*)k_rounds_fused<NN, 32>; break;
         }
-        int grid = sm_count() * LF_FUSED_GRID_SM;  // fewer CTAs: cheaper grid barriers
+        int grid = LF_FUSED_GRID > 0 ? LF_FUSED_GRID : sm_count() * LF_FUSED_GRID_SM;  // fewer CTAs: cheaper barriers
         const int cap = persistent_grid(kfn, LF_FUSED_T);
         if (grid > cap) grid = cap;
         LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, 0, s));
@@ -1045,8 +1086,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             if (rc) return rc;
         }
         LF_PROF("finalize", -1, s);
-        k_finalize<<<1, 32, 0, s>>>(w.flags, o->M, o->m, o->k_m, rounds_dev, w.live_part, live);
-        LF_CUDA(cudaGetLastError());
+        LF_CUDA(launch_pdl(k_finalize, 1, 32, 0, s, (const int*)w.flags, o->M, o->m, o->k_m, rounds_dev,
+                           (const unsigned long long*)w.live_part, live));
     }
     return LF_OK;
 }

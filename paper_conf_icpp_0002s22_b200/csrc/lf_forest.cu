@@ -945,6 +945,7 @@ __global__ void __launch_bounds__(LT, 1) k_lf_local1(ForestArgs a) {
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     LF_PHASE_INIT;
+    if (a.n_cycles && blockIdx.x == 0 && threadIdx.x == 0) *a.n_cycles = 0;  // summed by local2
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     LF_PHASE(a.ctl, 0);
@@ -1253,6 +1254,7 @@ template <bool MIN>
 __global__ void __launch_bounds__(RT) k_red_scan(ForestArgs a) {
     __shared__ int sh[32];
     extern __shared__ __align__(16) unsigned char red_smem[];
+    pdl_trigger();  // the next tile kernel may launch and wait meanwhile
     const int32_t* list = MIN ? a.list1 : a.list2;
     const int cnt = *(volatile int*)&a.ctl[MIN ? kCtlCnt1 : kCtlCnt2];
     int* ctl = a.ctl + (MIN ? kCtlRed1 : kCtlRed2);
@@ -1305,6 +1307,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_local2(ForestArgs a) {
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
+    pdl_wait();  // the factor slots above predate the chain; the cycle results below do not
     // weakest edge of the cycle through each own vertex (INF: not on a cycle)
     int2 f[VPT];
     unsigned long long ncyc = 0;
@@ -1387,6 +1390,7 @@ __global__ void __launch_bounds__(LT) k_lf_local3(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmem& s = *reinterpret_cast<TileSmem*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
+    pdl_wait();
     load_tile(a.forest, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
 #pragma unroll
@@ -1438,6 +1442,8 @@ __global__ void __launch_bounds__(kOffT) k_path_offsets(int64_t N, const int32_t
                                                          int* ticket) {
     __shared__ int sh[32];
     __shared__ int last;
+    pdl_wait();
+    pdl_trigger();  // one wave: the permutation kernel may launch and wait meanwhile
     const int64_t c0 = (int64_t)blockIdx.x * kOffChunk + (int64_t)threadIdx.x * kOffPT;
     int x[kOffPT];
     int sum = 0;
@@ -1509,6 +1515,7 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
                                                   const float* __restrict__ diag, int32_t* __restrict__ perm,
                                                   int32_t* __restrict__ iperm, float* __restrict__ ta,
                                                   float* __restrict__ tb, float* __restrict__ tc) {
+    pdl_wait();
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < N; v0 += stride * kPermBatch) {
         int32_t l[kPermBatch], p[kPermBatch], r[kPermBatch];
@@ -1627,8 +1634,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     int rcp = forest_prepare();
     if (rcp) return rcp;
     const int smem = (int)sizeof(TileSmem);
-    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
-    if (n_cycles) LF_CUDA(cudaMemsetAsync(n_cycles, 0, sizeof(int64_t), s));
+    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));  // n_cycles: zeroed by k_lf_local1
     ForestArgs a;
     memset(&a, 0, sizeof(a));
     a.N = N;
@@ -1675,8 +1681,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("lf_local2", -1, s);
-        k_lf_local2<<<tiles, LT, kTileSmemNoKeys, s>>>(a);
-        LF_CUDA(cudaGetLastError());
+        LF_CUDA(launch_pdl(k_lf_local2, tiles, LT, kTileSmemNoKeys, s, a));
     }
     {
         LF_PROF("red_scan_ranks", -1, s);
@@ -1685,22 +1690,22 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("lf_local3", -1, s);
-        k_lf_local3<<<tiles, LT, kTileSmemNoKeys, s>>>(a);
-        LF_CUDA(cudaGetLastError());
+        LF_CUDA(launch_pdl(k_lf_local3, tiles, LT, kTileSmemNoKeys, s, a));
     }
     {
         LF_PROF("path_offsets", -1, s);
         const int chunks = (int)((N + kOffChunk - 1) / kOffChunk);
-        k_path_offsets<<<chunks, kOffT, 0, s>>>(N, w.len, w.off, w.tsum, w.ctl + kCtlTicket3);
-        LF_CUDA(cudaGetLastError());
+        LF_CUDA(launch_pdl(k_path_offsets, chunks, kOffT, 0, s, N, (const int32_t*)w.len, w.off, w.tsum,
+                           w.ctl + kCtlTicket3));
     }
     {
         LF_PROF(tri ? "perm_tridiag" : "perm", -1, s);
-        k_perm_tri<<<persistent_grid((const void*)k_perm_tri, 256), 256, 0, s>>>(
-            N, path_id, pos, w.off, w.tsum, w.pdir, (const int2*)forest, (const int2*)pi2,
-            tri ? (const float2*)tri->pi2_val : nullptr, tri ? tri->diag : nullptr, perm, iperm,
-            tri ? tri->a : nullptr, tri ? tri->b : nullptr, tri ? tri->c : nullptr);
-        LF_CUDA(cudaGetLastError());
+        LF_CUDA(launch_pdl(k_perm_tri, persistent_grid((const void*)k_perm_tri, 256), 256, 0, s, N,
+                           (const int32_t*)path_id, (const int32_t*)pos, (const int32_t*)w.off,
+                           (const int32_t*)w.tsum, (const uint8_t*)w.pdir, (const int2*)forest,
+                           (const int2*)pi2, tri ? (const float2*)tri->pi2_val : nullptr,
+                           tri ? tri->diag : nullptr, perm, iperm, tri ? tri->a : nullptr,
+                           tri ? tri->b : nullptr, tri ? tri->c : nullptr));
     }
     return LF_OK;
 }

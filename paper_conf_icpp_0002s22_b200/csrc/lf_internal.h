@@ -34,6 +34,27 @@ struct ProfScope {
 };
 #define LF_PROF(name, k, s) ::lf::ProfScope lf_prof_scope_(name, k, s)
 
+// Programmatic dependent launch (PDL): a kernel launched this way may be scheduled while
+// its stream predecessor (a kernel) is still finishing; it calls pdl_wait() before it
+// touches anything the predecessor writes.  Disabled by the environment variable
+// LF_NO_PDL (then an ordinary launch).
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, static_cast<Args&&>(args)...);
+}
+
 // grid of a persistent kernel: resident blocks per SM x SM count (cached per kernel)
 int persistent_grid(const void* kernel, int block, size_t smem = 0);
 int sm_count();
