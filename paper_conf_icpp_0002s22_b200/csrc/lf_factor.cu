@@ -666,6 +666,151 @@ __global__ void __launch_bounds__(256) k_mutual(MutualArgs a) {
     mutual_phase<NN>(a);
 }
 
+// NN consecutive slots of one row in one load (NN = 2, 4: 8- / 16-byte vector)
+template <int NN, class T>
+__device__ __forceinline__ void load_slots(const T* __restrict__ p, T (&o)[NN]) {
+    if constexpr (NN == 2 && sizeof(T) == 4) {
+        const uint2 x = *reinterpret_cast<const uint2*>(p);
+        o[0] = *reinterpret_cast<const T*>(&x.x); o[1] = *reinterpret_cast<const T*>(&x.y);
+    } else if constexpr (NN == 4 && sizeof(T) == 4) {
+        const uint4 x = *reinterpret_cast<const uint4*>(p);
+        o[0] = *reinterpret_cast<const T*>(&x.x); o[1] = *reinterpret_cast<const T*>(&x.y);
+        o[2] = *reinterpret_cast<const T*>(&x.z); o[3] = *reinterpret_cast<const T*>(&x.w);
+    } else {
+#pragma unroll
+        for (int s = 0; s < NN; s++) o[s] = p[s];
+    }
+}
+template <int NN, class T>
+__device__ __forceinline__ void store_slots(T* __restrict__ p, const T (&o)[NN]) {
+    if constexpr (NN == 2 && sizeof(T) == 4) {
+        uint2 x;
+        x.x = *reinterpret_cast<const uint32_t*>(&o[0]); x.y = *reinterpret_cast<const uint32_t*>(&o[1]);
+        *reinterpret_cast<uint2*>(p) = x;
+    } else if constexpr (NN == 4 && sizeof(T) == 4) {
+        uint4 x;
+        x.x = *reinterpret_cast<const uint32_t*>(&o[0]); x.y = *reinterpret_cast<const uint32_t*>(&o[1]);
+        x.z = *reinterpret_cast<const uint32_t*>(&o[2]); x.w = *reinterpret_cast<const uint32_t*>(&o[3]);
+        *reinterpret_cast<uint4*>(p) = x;
+    } else {
+#pragma unroll
+        for (int s = 0; s < NN; s++) p[s] = o[s];
+    }
+}
+
+// Round 0's confirmation (Alg. 2 L26-L28 at k = 0) over all rows: the same outputs as
+// mutual_phase with fresh = 1, with MB rows per thread whose loads are all issued before
+// any result is used (the proposal gathers are the latency chain of this pass).  In a
+// fresh round pi is empty and the proposals are already in key order, so the confirmed
+// ones are copied in place order without a merge.
+constexpr int kMutual0Rows = 4;
+
+template <int NN, int MB>
+__global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
+    pdl_wait();
+    if (a.wl_zero && blockIdx.x == 0 && threadIdx.x == 0) *a.wl_zero = 0;
+    const int lane = threadIdx.x & 31;
+    const int64_t chunk = (int64_t)blockDim.x * MB;
+    for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < a.N; c0 += (int64_t)gridDim.x * chunk) {
+        int32_t pj[MB][NN], pw[MB][NN][NN];
+        float pv[MB][NN];
+#pragma unroll
+        for (int b = 0; b < MB; b++) {
+            const int64_t r = c0 + threadIdx.x + (int64_t)b * blockDim.x;
+            if (r < a.N) {
+                const int64_t v = a.row_base + r;
+                load_slots<NN>(a.prop_j + v * NN, pj[b]);
+                load_slots<NN>(a.prop_v + v * NN, pv[b]);
+            } else {
+#pragma unroll
+                for (int s = 0; s < NN; s++) pj[b][s] = -1;
+            }
+        }
+#pragma unroll
+        for (int b = 0; b < MB; b++)
+#pragma unroll
+            for (int s = 0; s < NN; s++) {
+                if (pj[b][s] >= 0) {
+                    load_slots<NN>(a.prop_j + (int64_t)pj[b][s] * NN, pw[b][s]);
+                } else {
+#pragma unroll
+                    for (int t = 0; t < NN; t++) pw[b][s][t] = -1;
+                }
+            }
+#pragma unroll
+        for (int b = 0; b < MB; b++) {
+            const int64_t r = c0 + threadIdx.x + (int64_t)b * blockDim.x;
+            const int32_t v = (int32_t)(a.row_base + r);
+            int32_t oj[NN];
+            float ow[NN], ov[NN];
+            int deg = 0;
+#pragma unroll
+            for (int s = 0; s < NN; s++) { oj[s] = -1; ow[s] = 0.0f; ov[s] = 0.0f; }
+#pragma unroll
+            for (int s = 0; s < NN; s++) {
+                bool mutual = false;
+#pragma unroll
+                for (int t = 0; t < NN; t++) mutual |= (pw[b][s][t] == v);
+                if (pj[b][s] >= 0 && mutual) {
+                    // deg <= s: write the confirmed slot at position deg (predicated moves)
+#pragma unroll
+                    for (int q = 0; q < NN; q++)
+                        if (q == deg) { oj[q] = pj[b][s]; ov[q] = pv[b][s]; ow[q] = fabsf(pv[b][s]); }
+                    deg++;
+                }
+            }
+            bool keep = false;
+            if (r < a.N) {
+                store_slots<NN>(a.pi + (int64_t)v * NN, oj);
+                store_slots<NN>(a.pi_w + (int64_t)v * NN, ow);
+                if (a.pi_val) store_slots<NN>(a.pi_val + (int64_t)v * NN, ov);
+                uint32_t ch = 0;
+                if (a.wl_next) {
+                    keep = pj[b][0] != PROP_RETIRED && deg < NN;
+                    if (keep && a.next_charging) ch = charge_bit((uint32_t)(v + a.gid_off), a.next_k, a.seed, a.thr);
+                }
+                a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0));
+            }
+            if (a.wl_next) {
+                const unsigned m = __ballot_sync(0xffffffffu, keep);
+                int32_t basepos = 0;
+                if (lane == 0 && m) basepos = atomicAdd(a.wl_next_count, __popc(m));
+                basepos = __shfl_sync(0xffffffffu, basepos, 0);
+                if (keep) a.wl_next[basepos + __popc(m & ((1u << lane) - 1u))] = v;
+            }
+        }
+    }
+}
+
+// Alg. 2 L23-L24 / L30: rounds = k+1 for the first uncharged round without proposals;
+// also sums the live-row counter slots into live[k], live[M+k]
+__device__ __forceinline__ void finalize_body(const int* flags, int M, int m, int k_m, int32_t* rounds,
+                                              const unsigned long long* part, int64_t* live) {
+    if (threadIdx.x == 0 && rounds) {
+        int r = M;
+        for (int k = 0; k < M; k++)
+            if ((k % m) == k_m && flags[k] == 0) {
+                r = k + 1;
+                break;
+            }
+        *rounds = r;
+    }
+    if (live) {
+        for (int i = threadIdx.x; i < 2 * M; i += blockDim.x) {
+            const int k = i % M, which = i / M;
+            unsigned long long t = 0;
+            for (int j = 0; j < 64; j++) t += part[(size_t)k * 128 + which * 64 + j];
+            live[i] = (int64_t)t;
+        }
+    }
+}
+
+__global__ void k_finalize(const int* flags, int M, int m, int k_m, int32_t* rounds,
+                           const unsigned long long* part, int64_t* live) {
+    pdl_wait();
+    finalize_body(flags, M, m, k_m, rounds, part, live);
+}
+
 // Rounds 1..M-1 in one cooperative persistent kernel: after round 0 only the live rows
 // (2-40% of them) remain, and separate launches would be latency-bound.  Per round:
 // propose over the worklist | long rows warp-per-row | mutual, separated by grid barriers.
@@ -680,6 +825,8 @@ struct FusedArgs {
     unsigned long long* live_part;
     int M, m, k_m;
     int G;
+    int32_t* rounds;     // finalize outputs (k_finalize's work, done by CTA 0 in the last round)
+    int64_t* live;
 };
 
 #ifndef LF_FUSED_T
@@ -719,6 +866,10 @@ __global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {
         }
         MutualArgs ma = f.ma;
         const bool last = k == f.M - 1;
+        // every round's flags and live-row partial sums are final once the last round's
+        // proposals are (the barriers above): finalize here instead of a dependent launch
+        if (last && blockIdx.x == 0 && (f.rounds || f.live))
+            finalize_body(f.flags, f.M, f.m, f.k_m, f.rounds, f.live_part, f.live);
         ma.wl = f.wl[k & 1];
         ma.wl_count = &f.counts[k % 3];
         ma.wl_next = last ? nullptr : f.wl[(k + 1) & 1];
@@ -752,30 +903,6 @@ __global__ void k_diag(int64_t N, const int64_t* __restrict__ rowptr, const int3
         for (int64_t e = rowptr[r]; e < rowptr[r + 1]; e++)
             if (col[e] == v) d = val[e];
         diag[v] = d;
-    }
-}
-
-// Alg. 2 L23-L24 / L30: rounds = k+1 for the first uncharged round without proposals;
-// also sums the live-row counter slots into live[k], live[M+k]
-__global__ void k_finalize(const int* flags, int M, int m, int k_m, int32_t* rounds,
-                           const unsigned long long* part, int64_t* live) {
-    pdl_wait();
-    if (threadIdx.x == 0 && rounds) {
-        int r = M;
-        for (int k = 0; k < M; k++)
-            if ((k % m) == k_m && flags[k] == 0) {
-                r = k + 1;
-                break;
-            }
-        *rounds = r;
-    }
-    if (live) {
-        for (int i = threadIdx.x; i < 2 * M; i += blockDim.x) {
-            const int k = i % M, which = i / M;
-            unsigned long long t = 0;
-            for (int j = 0; j < 64; j++) t += part[(size_t)k * 128 + which * 64 + j];
-            live[i] = (int64_t)t;
-        }
     }
 }
 
@@ -1019,7 +1146,17 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         ma.thr = thr;
         {
             LF_PROF("mutual", k, s);
-            LF_CUDA(launch_pdl(k_mutual<NN>, grid_m, 256, 0, s, ma));
+            // all-rows round 0: batched kernel with vector slot loads (needs aligned slots)
+            const uintptr_t amask = (NN == 2 ? 7 : (NN == 4 ? 15 : 3));
+            const bool aligned = ((uintptr_t)pi & amask) == 0 && ((uintptr_t)pi_w & amask) == 0 &&
+                                 (!pi_val || ((uintptr_t)pi_val & amask) == 0);
+            if (fresh && aligned && N > 0) {
+                const int64_t per = 256 * (int64_t)kMutual0Rows;
+                const int64_t g = (N + per - 1) / per;
+                LF_CUDA(launch_pdl(k_mutual0<NN, kMutual0Rows>, (int)(g < (1 << 20) ? g : (1 << 20)), 256, 0, s, ma));
+            } else {
+                LF_CUDA(launch_pdl(k_mutual<NN>, grid_m, 256, 0, s, ma));
+            }
         }
     }
     if (fuse) {
@@ -1060,6 +1197,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         f.m = o->m;
         f.k_m = o->k_m;
         f.G = G;
+        f.rounds = rounds_dev;
+        f.live = live;
         LF_PROF("rounds_fused", -1, s);
         void* args[] = {&f};
         const void* kfn;
@@ -1080,7 +1219,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_CUDA(cudaMemcpyAsync(rounds_dev, &rounds_host, sizeof(int32_t), cudaMemcpyHostToDevice, s));
             LF_CUDA(cudaStreamSynchronize(s));
         }
-    } else if (rounds_dev || live) {
+    } else if (!fuse && (rounds_dev || live)) {
         if (part && part->pre_finalize) {  // global maximality flags / counters
             const int rc = part->pre_finalize(part->ctx, s);
             if (rc) return rc;
