@@ -56,7 +56,8 @@ constexpr int kCtlRed1 = 0;       // ctl[0..63]   per-step not-done counts, redu
 constexpr int kCtlRed2 = 64;      // ctl[64..127] reduced scan 2
 constexpr int kCtlCnt1 = 128;     // boundary list sizes
 constexpr int kCtlCnt2 = 129;
-constexpr int kCtlTicket3 = 130;  // finished-CTA ticket of k_path_offsets (the last one scans tsum)
+constexpr int kCtlTicket3 = 130;  // finished-CTA ticket of k_path_offsets / k_lf_full2 (the last one scans tsum)
+constexpr int kCtlNcyc = 131;     // broken cycles (single-pass forest)
 constexpr int kMaxSteps = 62;
 constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
 // ctl[192] splitter nodes (cycle pass), [193] unvisited vertices (fallback), [194] tiles
@@ -125,7 +126,8 @@ constexpr size_t kTileSmemNoKeys = offsetof(TileSmem, EK0);
 struct Tile {
     int32_t b0, tend;
 };
-__device__ __forceinline__ Tile tile_of(const TileSmem& s) { return Tile{s.b0, s.tend}; }
+template <class S>
+__device__ __forceinline__ Tile tile_of(const S& s) { return Tile{s.b0, s.tend}; }
 __device__ __forceinline__ bool is_local(int32_t x, const Tile& t) {
     return (uint32_t)(x - t.b0) < (uint32_t)(t.tend - t.b0);
 }
@@ -840,6 +842,13 @@ struct ForestArgs {
     uint8_t* pdir;         // [N] forest slot toward the path-ID end
     unsigned long long* n_cycles;
     int max_steps;
+    // single-pass forest (FULL windows): reduced records and results at list positions
+    int2* cq_r;            // [list pos] initial window lengths per direction
+    int2* cq_dk;           // [list pos] initial DK per direction
+    int2* dk2;             // [list pos] final DK per direction
+    int2* rdk[2];          // grid-path ping-pong DK
+    int32_t* off;          // [N] exclusive tile prefix of path lengths (at path-ID vertices)
+    int32_t* tsum;         // [tiles] tile totals -> exclusive prefix (last expand CTA)
 };
 
 __device__ __forceinline__ bool is_foreign(int64_t x, const ForestArgs& a) { return x < a.lo || x >= a.hi; }
@@ -856,7 +865,8 @@ __device__ __forceinline__ int2 ghost_slots(const ForestArgs& a, int32_t x) {
 }
 
 // keys of the own vertices' slots (global; a remote min endpoint needs one gather)
-__device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int32_t b0,
+template <class S>
+__device__ __forceinline__ void slot_keys(const ForestArgs& a, S& s, int32_t b0,
                                          ulonglong2 (&ek)[VPT]) {
     const Tile T = tile_of(s);
 #pragma unroll
@@ -882,8 +892,9 @@ __device__ __forceinline__ void slot_keys(const ForestArgs& a, TileSmem& s, int3
 }
 
 // slots and weights of the tile in one round trip (cycle pass)
+template <class S>
 __device__ __forceinline__ void load_tile_w(const int2* __restrict__ src, const float2* __restrict__ wsrc,
-                                            TileSmem& s, int32_t b0, int64_t hi) {
+                                            S& s, int32_t b0, int64_t hi) {
     if (threadIdx.x == 0) {
         s.b0 = b0;
         s.tend = (int32_t)((int64_t)b0 + LB < hi ? (int64_t)b0 + LB : hi);
@@ -901,7 +912,8 @@ __device__ __forceinline__ void load_tile_w(const int2* __restrict__ src, const 
     __syncthreads();
 }
 
-__device__ __forceinline__ void load_tile(const int2* __restrict__ src, TileSmem& s, int32_t b0, int64_t hi) {
+template <class S>
+__device__ __forceinline__ void load_tile(const int2* __restrict__ src, S& s, int32_t b0, int64_t hi) {
     if (threadIdx.x == 0) {
         s.b0 = b0;
         s.tend = (int32_t)((int64_t)b0 + LB < hi ? (int64_t)b0 + LB : hi);
@@ -1508,7 +1520,7 @@ constexpr int kPermBatch = 4;  // vertices per thread per iteration (loads in fl
 __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __restrict__ path_id,
                                                   const int32_t* __restrict__ pos,
                                                   const int32_t* __restrict__ off,
-                                                  const int32_t* __restrict__ tbase,
+                                                  const int32_t* __restrict__ tbase, int chunk,
                                                   const uint8_t* __restrict__ pdir,
                                                   const int2* __restrict__ forest, const int2* __restrict__ pi2,
                                                   const float2* __restrict__ pi2_val,
@@ -1526,7 +1538,7 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
             p[b] = v < N ? __ldg(pos + v) : 0;
         }
 #pragma unroll
-        for (int b = 0; b < kPermBatch; b++) r[b] = __ldg(tbase + l[b] / kOffChunk) + __ldg(off + l[b]) + p[b] - 1;
+        for (int b = 0; b < kPermBatch; b++) r[b] = __ldg(tbase + l[b] / chunk) + __ldg(off + l[b]) + p[b] - 1;
 #pragma unroll
         for (int b = 0; b < kPermBatch; b++) {
             const int64_t v = v0 + b * stride;
@@ -1545,6 +1557,928 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
             }
         }
     }
+}
+
+// ===========================================================================
+// Single-pass linear forest.  Every scan level carries the FULL window
+// of a vertex in one direction instead of one quantity per pass:
+//   pointer | R = edges covered | K = minimum edge key | DK = 2 * (distance to the near
+//   endpoint of that minimum edge) + [the near endpoint is the edge's min-id endpoint].
+// Appending window B (starting where A ends) to A:  R = R_A + R_B;  if K_B < K_A then
+// K = K_B, DK = 2 R_A + DK_B.  The strict '<' keeps the first occurrence, so on a cycle
+// DK is the true distance to the weakest edge (reading c9) in that direction, and with
+// K (whose rank field names the min-id endpoint x, reading c11) it gives every cycle
+// vertex its position on the broken cycle directly: pos = distance to x + 1 (reading c12).
+// So cycles are broken AND all vertices ranked by one tile pass (k_lf_full1), one reduced
+// scan (k_red_full) and one expand pass (k_lf_full2), instead of two of each.
+// ===========================================================================
+
+// the min-id endpoint of the edge behind a key (rank = 2 min + c, see edge_key)
+__device__ __forceinline__ int32_t key_min_end(uint64_t k) {
+    return (int32_t)((0xFFFFFFFFu - (uint32_t)k) >> 1);
+}
+
+struct TileSmemF {
+    int2 nb[LB];          // slots (global ids); run slots virtual after contraction
+    union {
+        float2 w[LB];     // |w| per slot (read by slot_keys)
+        struct {
+            short2 run[LB];
+            short2 vw[LB];
+        } r;
+    };
+    uint64_t EK0[LB];     // key of the (virtual) link behind slot 0 / slot 1
+    uint64_t EK1[LB];
+    short sidx[LB];
+    short spl[LB];
+    short2 recS[LB];
+    short2 recD[LB];
+    // splitter-node arrays
+    short2 P[LB];
+    short2 R[LB];
+    short2 DK[LB];
+    uint64_t K0[LB];      // (also per-vertex temporaries of the run scan, before the walks)
+    uint64_t K1[LB];
+    uint64_t WK0[LB];     // minimum of each node's walk per slot (kept through the node scan)
+    uint64_t WK1[LB];
+    short2 WD[LB];        // DK of that minimum, from the node
+    int nspl;
+    int32_t b0, tend;
+};
+static_assert(sizeof(TileSmemF) <= 227 * 1024, "tile smem");
+
+// DK of the (possibly virtual) link behind slot `slot` of local vertex u, from u
+__device__ __forceinline__ int slot_dk(const TileSmemF& s, int u, int32_t g, int slot) {
+    const int2 nb = s.nb[u];
+    const int32_t z = slot ? nb.y : nb.x;
+    const short2 vw = s.r.vw[u];
+    if ((slot ? vw.y : vw.x) == 1) return g < z ? 1 : 0;  // a real link: near endpoint u
+    const int32_t m = key_min_end(slot ? s.EK1[u] : s.EK0[u]);  // run minimum: link (m, m+1)
+    return z > g ? 2 * (m - g) + 1 : 2 * (g - (m + 1));
+}
+
+// the virtual (run) slot of run end u whose other end is o
+__device__ __forceinline__ int run_slot(const TileSmemF& s, int u, int32_t og) {
+    const short2 vw = s.r.vw[u];
+    if (vw.x > 1) return 0;
+    if (vw.y > 1) return 1;
+    return s.nb[u].x == og ? 0 : 1;
+}
+
+// Result of the tile pass for one own vertex
+struct VRes {
+    bool cyc;         // on a cycle that lies inside the tile
+    int2 T;           // path type: local terminals per slot
+    int2 R;           //   distances to them
+    uint64_t Ks;      // cycle: its weakest edge key
+    int2 C;           //   DK per slot (toward the weakest edge)
+    ulonglong2 Kn;    // splitter node: window keys per slot (reduced records)
+    int2 Dn;          //   window DK per slot
+};
+
+// bidirectional scan over the splitter nodes with full windows; WARP: warp 0 alone
+template <int NPN, bool WARP>
+__device__ __forceinline__ void node_scan_full(TileSmemF& s, int C, int* stats) {
+    const int tid = threadIdx.x;
+    constexpr int STRIDE = WARP ? 32 : LT;
+    for (int step = 0; step < 16; step++) {
+        int notdone = 0;
+        short2 nP[NPN], nR[NPN], nD[NPN];
+        uint64_t nk0[NPN], nk1[NPN];
+#pragma unroll
+        for (int k = 0; k < NPN; k++) {
+            const int i = tid + k * STRIDE;
+            if (i >= C) continue;
+            const short2 p = s.P[i];
+            short2 q = p, r = s.R[i], dk = s.DK[i];
+            uint64_t k0 = s.K0[i], k1 = s.K1[i];
+#pragma unroll
+            for (int dd = 0; dd < 2; dd++) {
+                const int w = dd ? p.y : p.x;
+                if (w < 0) continue;
+                const short2 pw = s.P[w];
+                const int Rd = dd ? r.y : r.x;
+                uint64_t kc = dd ? k1 : k0;
+                int dc = dd ? dk.y : dk.x;
+                int j = -1;
+                if (pw.x != i) j = 0;
+                else if (pw.y != i) j = 1;
+                const short2 rw = s.R[w], dw = s.DK[w];
+                const uint64_t kw0 = s.K0[w], kw1 = s.K1[w];
+                if (j >= 0) {
+                    const uint64_t kw = j ? kw1 : kw0;
+                    if (kw < kc) { kc = kw; dc = 2 * Rd + (j ? dw.y : dw.x); }
+                    const short tgt = j ? pw.y : pw.x;
+                    const short nr = (short)(Rd + (j ? rw.y : rw.x));
+                    if (dd) { q.y = tgt; r.y = nr; } else { q.x = tgt; r.x = nr; }
+                } else {
+                    // stall (reading c13): both windows of w return here; the one that
+                    // continues covers the rest of the cycle, the other only repeats this
+                    // window's edges and can never win the strict compare
+                    if (kw0 < kc) { kc = kw0; dc = 2 * Rd + dw.x; }
+                    if (kw1 < kc) { kc = kw1; dc = 2 * Rd + dw.y; }
+                }
+                if (dd) { k1 = kc; dk.y = (short)dc; } else { k0 = kc; dk.x = (short)dc; }
+            }
+            nP[k] = q; nR[k] = r; nD[k] = dk; nk0[k] = k0; nk1[k] = k1;
+            const bool path_done = q.x < 0 && q.y < 0;
+            const bool cyc_done = q.x >= 0 && q.y >= 0 && k0 == k1;
+            notdone |= !(path_done || cyc_done);
+        }
+        if (WARP) __syncwarp(); else __syncthreads();
+#pragma unroll
+        for (int k = 0; k < NPN; k++) {
+            const int i = tid + k * STRIDE;
+            if (i >= C) continue;
+            s.P[i] = nP[k]; s.R[i] = nR[k]; s.DK[i] = nD[k]; s.K0[i] = nk0[k]; s.K1[i] = nk1[k];
+        }
+        const bool any = WARP ? (__syncwarp(), __any_sync(0xffffffffu, notdone)) : __syncthreads_or(notdone);
+        if (!any) {
+            if (tid == 0 && stats) atomicMax(&stats[4], step + 1);
+            break;
+        }
+    }
+}
+
+// Block-local ranking with full windows (same phases as tile_rank).
+// ek: real slot keys of the own vertices.  On return o[k] holds the vertex's result.
+__device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[VPT], VRes (&o)[VPT],
+                               int* stats) {
+    __shared__ int sh[32];
+    const int tid = threadIdx.x;
+    const Tile T = tile_of(s);
+    const int tlen = T.tend - T.b0;
+    if (tid == 0) s.nspl = 0;
+    const auto linked_prev = [&](int u) {
+        const int2 nb = s.nb[u];
+        const int32_t g = b0 + u;
+        return u > 0 && u < tlen && (nb.x == g - 1 || nb.y == g - 1);
+    };
+    // 0a. slot keys; K0 = key of the run link (u-1, u)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const int2 nb = s.nb[u];
+        const int32_t g = b0 + u;
+        const bool lp = u > 0 && u < tlen && (nb.x == g - 1 || nb.y == g - 1);
+        s.EK0[u] = ek[k].x;
+        s.EK1[u] = ek[k].y;
+        s.K0[u] = lp ? (nb.x == g - 1 ? ek[k].x : ek[k].y) : KEY_INF;
+    }
+    // 0b. run bounds (block max-scan) and each run's weakest link (segmented min-scan)
+    {
+        const int u0 = tid * VPT;
+        int st[VPT];
+        bool lk[VPT + 1];
+#pragma unroll
+        for (int j = 0; j <= VPT; j++) lk[j] = u0 + j < LB && linked_prev(u0 + j);
+        int run = INT_MIN;
+#pragma unroll
+        for (int j = 0; j < VPT; j++) {
+            if (!lk[j]) run = u0 + j;
+            st[j] = run;
+        }
+        const int prev_max = block_scan_max_excl(run, sh);
+#pragma unroll
+        for (int j = 0; j < VPT; j++) {
+            const int u = u0 + j;
+            if (st[j] == INT_MIN) st[j] = prev_max;
+            s.r.run[u].x = (short)st[j];
+            if (!lk[j + 1]) s.r.run[st[j]].y = (short)u;
+        }
+        __syncthreads();
+        short en[VPT];
+#pragma unroll
+        for (int j = 0; j < VPT; j++) en[j] = s.r.run[st[j]].y;
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < VPT; j++) s.r.run[u0 + j].y = en[j];
+        uint64_t x[VPT];
+        bool hd[VPT];
+        uint64_t agg = KEY_INF;
+        bool anyh = false;
+#pragma unroll
+        for (int j = 0; j < VPT; j++) {
+            hd[j] = !lk[j];
+            const uint64_t kv = s.K0[u0 + j];
+            agg = hd[j] ? kv : umin64(agg, kv);
+            anyh |= hd[j];
+            x[j] = agg;
+        }
+        const int lane = tid & 31, wid = tid >> 5;
+        bool f = anyh;
+        uint64_t v = agg;
+#pragma unroll
+        for (int o2 = 1; o2 < 32; o2 <<= 1) {
+            const uint64_t yv = __shfl_up_sync(0xffffffffu, v, o2);
+            const int yf = __shfl_up_sync(0xffffffffu, (int)f, o2);
+            if (lane >= o2) { if (!f) v = umin64(v, yv); f = f || yf; }
+        }
+        __shared__ uint64_t wv[LT / 32];
+        __shared__ int wf[LT / 32];
+        if (lane == 31) { wv[wid] = v; wf[wid] = f; }
+        __syncthreads();
+        if (wid == 0) {
+            uint64_t tv = lane < LT / 32 ? wv[lane] : KEY_INF;
+            bool tf = lane < LT / 32 ? wf[lane] != 0 : false;
+#pragma unroll
+            for (int o2 = 1; o2 < 32; o2 <<= 1) {
+                const uint64_t yv = __shfl_up_sync(0xffffffffu, tv, o2);
+                const int yf = __shfl_up_sync(0xffffffffu, (int)tf, o2);
+                if (lane >= o2) { if (!tf) tv = umin64(tv, yv); tf = tf || yf; }
+            }
+            if (lane < LT / 32) { wv[lane] = tv; wf[lane] = tf; }
+        }
+        __syncthreads();
+        uint64_t cv = __shfl_up_sync(0xffffffffu, v, 1);
+        bool cf = __shfl_up_sync(0xffffffffu, (int)f, 1) != 0;
+        if (lane == 0) { cv = KEY_INF; cf = true; }
+        if (wid > 0 && !cf) cv = umin64(cv, wv[wid - 1]);
+        if (wid > 0 && lane == 0) { cv = wv[wid - 1]; cf = false; }
+#pragma unroll
+        for (int j = 0; j < VPT; j++) {
+            if (hd[j]) break;
+            x[j] = umin64(x[j], cv);
+        }
+#pragma unroll
+        for (int j = 0; j < VPT; j++) s.K1[u0 + j] = x[j];
+    }
+    __syncthreads();
+    // 0c. contract runs: virtual links between run ends (length, weakest key)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const short2 rr = s.r.run[u];
+        const int32_t g = b0 + u;
+        short2 vw = make_short2(1, 1);
+        const int len = rr.y - rr.x + 1;
+        if (len >= 2 && (u == rr.x || u == rr.y)) {
+            const int other = (u == rr.x) ? rr.y : rr.x;
+            const int32_t inside = (u == rr.x) ? g + 1 : g - 1;
+            int2 nb = s.nb[u];
+            const uint64_t rk = s.K1[rr.y];
+            if (nb.x == inside) { nb.x = b0 + other; vw.x = (short)(len - 1); s.EK0[u] = rk; }
+            else { nb.y = b0 + other; vw.y = (short)(len - 1); s.EK1[u] = rk; }
+            s.nb[u] = nb;
+        }
+        s.r.vw[u] = vw;
+    }
+    __syncthreads();
+    // 1. splitters (run ends, terminals, hashed vertices); run cycles -3, interiors -2
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const short2 rr = s.r.run[u];
+        const int2 nb = s.nb[u];
+        const bool interior = u > rr.x && u < rr.y;
+        const bool run_cycle = rr.y - rr.x >= 2 && nb.x == nb.y;
+        short id = -1;
+        bool node = false;
+        if (u >= tlen) {
+            node = true;
+        } else if (interior || run_cycle) {
+            id = run_cycle ? -3 : -2;
+        } else {
+            const bool l0 = nb.x >= 0 && is_local(nb.x, T);
+            const bool l1 = nb.y >= 0 && is_local(nb.y, T);
+            node = !l0 || !l1 || rr.y > rr.x || hashed_splitter(b0 + u);
+        }
+        {
+            const unsigned m = __ballot_sync(0xffffffffu, node);
+            const int lane = tid & 31;
+            int base = 0;
+            if (lane == 0 && m) base = atomicAdd(&s.nspl, __popc(m));
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (node) id = (short)(base + __popc(m & ((1u << lane) - 1u)));
+        }
+        s.sidx[u] = id;
+        if (id >= 0) s.spl[id] = (short)u;
+        s.recS[u] = make_short2(-1, -1);
+    }
+    __syncthreads();
+    const int C = s.nspl;
+    if (tid == 0 && stats) atomicAdd(&stats[0], C);
+    // 2. walks from every (node, slot) to the next node: length, weakest link and its DK
+    for (int wk = tid; wk < 2 * C; wk += LT) {
+        const int i = wk >> 1, f = wk & 1;
+        const int su = s.spl[i];
+        const int2 nbs = s.nb[su];
+        const int32_t x = f ? nbs.y : nbs.x;
+        short ptr = (short)(-(i + 1));
+        int dist = 0, dk = 0;
+        uint64_t km = KEY_INF;
+        if (x >= 0 && is_local(x, T)) {
+            const short2 vws = s.r.vw[su];
+            int prev = su, cur = x - b0, d = f ? vws.y : vws.x;
+            km = f ? s.EK1[su] : s.EK0[su];
+            dk = slot_dk(s, su, b0 + su, f);
+            while (s.sidx[cur] < 0) {
+                const int2 nbc = s.nb[cur];
+                const int face = (nbc.x == b0 + prev) ? 0 : 1;
+                if (face == 0) { s.recS[cur].x = (short)((i << 1) | f); s.recD[cur].x = (short)d; }
+                else { s.recS[cur].y = (short)((i << 1) | f); s.recD[cur].y = (short)d; }
+                const int nxt = (face ? nbc.x : nbc.y) - b0;
+                const uint64_t kk = face ? s.EK0[cur] : s.EK1[cur];
+                if (kk < km) {  // a walk passes real links only (run ends are nodes)
+                    km = kk;
+                    dk = 2 * d + ((b0 + cur) < (face ? nbc.x : nbc.y) ? 1 : 0);
+                }
+                d += 1;
+                prev = cur;
+                cur = nxt;
+            }
+            ptr = s.sidx[cur];
+            dist = d;
+        }
+        if (f) { s.P[i].y = ptr; s.R[i].y = (short)dist; s.DK[i].y = (short)dk; s.K1[i] = km; s.WK1[i] = km; s.WD[i].y = (short)dk; }
+        else { s.P[i].x = ptr; s.R[i].x = (short)dist; s.DK[i].x = (short)dk; s.K0[i] = km; s.WK0[i] = km; s.WD[i].x = (short)dk; }
+    }
+    __syncthreads();
+    // 3. node scan
+    if (C <= 32 * kWarpScanNodes) {
+        if (tid < 32) node_scan_full<kWarpScanNodes, true>(s, C, stats);
+        __syncthreads();
+    } else {
+        node_scan_full<VPT, false>(s, C, stats);
+    }
+    // 4. nodes and walk-visited vertices
+    bool unvisited[VPT];
+    int any_unvisited = 0;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        unvisited[k] = false;
+        VRes& r = o[k];
+        r.cyc = false;
+        r.T = make_int2(u, u);
+        r.R = make_int2(0, 0);
+        r.Ks = KEY_INF;
+        r.C = make_int2(0, 0);
+        r.Kn = make_ulonglong2(KEY_INF, KEY_INF);
+        r.Dn = make_int2(0, 0);
+        const int id = s.sidx[u];
+        if (id == -2 || id == -3) continue;
+        if (id >= 0) {
+            const short2 p = s.P[id];
+            const short2 dk = s.DK[id];
+            r.Kn = make_ulonglong2(s.K0[id], s.K1[id]);
+            r.Dn = make_int2(dk.x, dk.y);
+            if (p.x >= 0 && p.y >= 0) {
+                r.cyc = true;
+                r.Ks = s.K0[id];
+                r.C = make_int2(dk.x, dk.y);
+            } else {
+                const short2 rr = s.R[id];
+                r.T = make_int2(s.spl[-(p.x + 1)], s.spl[-(p.y + 1)]);
+                r.R = make_int2(rr.x, rr.y);
+            }
+            continue;
+        }
+        const short2 rs = s.recS[u];
+        if (rs.x < 0 && rs.y < 0) { unvisited[k] = true; any_unvisited = 1; continue; }
+        const short2 rd = s.recD[u];
+#pragma unroll
+        for (int f = 0; f < 2; f++) {
+            const int rec = f ? rs.y : rs.x;
+            const int i = rec >> 1, f0 = rec & 1, away = f0 ^ 1;
+            const short2 p = s.P[i];
+            const int pa = away ? p.y : p.x;
+            const int d = f ? rd.y : rd.x;
+            if (pa >= 0) {  // cycle: the weakest key is the node's (both windows agree)
+                const uint64_t kc = s.K0[i];
+                const uint64_t wk = f0 ? s.WK1[i] : s.WK0[i];
+                const short2 wdp = s.WD[i];
+                const int wd = f0 ? wdp.y : wdp.x;
+                int cf;
+                if (wk == kc && (wd >> 1) + 1 <= d) cf = 2 * (d - (wd >> 1) - 1) + ((wd & 1) ^ 1);
+                else { const short2 dk = s.DK[i]; cf = 2 * d + (away ? dk.y : dk.x); }
+                r.cyc = true;
+                r.Ks = kc;
+                if (f) r.C.y = cf; else r.C.x = cf;
+            } else {
+                const short2 rr = s.R[i];
+                const int t = s.spl[-(pa + 1)];
+                const int dd = d + (away ? rr.y : rr.x);
+                if (f) { r.T.y = t; r.R.y = dd; } else { r.T.x = t; r.R.x = dd; }
+            }
+        }
+    }
+    // 4b. cycles of the contracted tile graph without a splitter (real links only): each
+    //     of their vertices walks its cycle once
+    if (__syncthreads_or(any_unvisited)) {
+        if (tid == 0 && stats) atomicAdd(&stats[2], 1);
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            if (!unvisited[k]) continue;
+            const int u = tid + k * LT;
+            if (stats) atomicAdd(&stats[1], 1);
+            int prev = u, cur = s.nb[u].x - b0, d = 1;
+            uint64_t km = s.EK0[u];
+            int kd = (b0 + u) < s.nb[u].x ? 1 : 0;
+            while (cur != u) {
+                const int2 nbc = s.nb[cur];
+                const int face = (nbc.x == b0 + prev) ? 0 : 1;
+                const uint64_t kk = face ? s.EK0[cur] : s.EK1[cur];
+                const int32_t z = face ? nbc.x : nbc.y;
+                if (kk < km) { km = kk; kd = 2 * d + ((b0 + cur) < z ? 1 : 0); }
+                prev = cur;
+                cur = z - b0;
+                d++;
+            }
+            o[k].cyc = true;
+            o[k].Ks = km;
+            o[k].C = make_int2(kd, 2 * (d - (kd >> 1) - 1) + ((kd & 1) ^ 1));
+        }
+    }
+    // 5. interior run vertices and run cycles, from the run ends' node windows
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = tid + k * LT;
+        const int id = s.sidx[u];
+        if (id != -2 && id != -3) continue;
+        VRes& r = o[k];
+        const short2 rr = s.r.run[u];
+        const int a = rr.x, b = rr.y;
+        const int32_t g = b0 + u;
+        const int2 nb = s.nb[u];
+        const int va = run_slot(s, a, b0 + b);
+        const uint64_t RK = va ? s.EK1[a] : s.EK0[a];       // the run's weakest link
+        const int ml = key_min_end(RK) - b0;                 // it is (ml, ml+1)
+        // slots of u toward u-1 ("down") and u+1 ("up"); for the ends of a run cycle the
+        // closing link continues the direction
+        int sdown;
+        if (u == a) sdown = va ^ 1;
+        else if (u == b) sdown = run_slot(s, b, b0 + a);
+        else sdown = (nb.x == g - 1) ? 0 : 1;
+        int down, up;  // DK toward u-1 / u+1 (cycles)
+        if (s.sidx[a] == -3) {  // the run closes into a cycle through the link (b, a)
+            const uint64_t CK = va ? s.EK0[a] : s.EK1[a];
+            const uint64_t ks = umin64(RK, CK);
+            if (ks == CK) {
+                up = 2 * (b - u);            // near endpoint b (not the min id)
+                down = 2 * (u - a) + 1;      // near endpoint a = x
+            } else {
+                up = (u <= ml) ? 2 * (ml - u) + 1 : 2 * ((b - u) + 1 + (ml - a)) + 1;
+                down = (u >= ml + 1) ? 2 * (u - ml - 1) : 2 * ((u - a) + 1 + (b - ml - 1));
+            }
+            r.cyc = true;
+            r.Ks = ks;
+        } else {
+            const int ia = s.sidx[a], ib = s.sidx[b];
+            const int oa = va ^ 1, ob = run_slot(s, b, b0 + a) ^ 1;   // outer slots of the ends
+            const short2 pa = s.P[ia], pb = s.P[ib];
+            const int qa = oa ? pa.y : pa.x, qb = ob ? pb.y : pb.x;
+            if (qa >= 0) {  // on a cycle
+                const uint64_t ks = s.K0[ia];
+                const short2 da = s.DK[ia], db = s.DK[ib];
+                down = (ks == RK && ml + 1 <= u) ? 2 * (u - ml - 1) : 2 * (u - a) + (oa ? da.y : da.x);
+                up = (ks == RK && ml >= u) ? 2 * (ml - u) + 1 : 2 * (b - u) + (ob ? db.y : db.x);
+                r.cyc = true;
+                r.Ks = ks;
+            } else {
+                const short2 ra = s.R[ia], rb = s.R[ib];
+                const int ta = s.spl[-(qa + 1)], tb = s.spl[-(qb + 1)];
+                const int dA = (u - a) + (oa ? ra.y : ra.x), dB = (b - u) + (ob ? rb.y : rb.x);
+                r.cyc = false;
+                if (sdown == 0) { r.T = make_int2(ta, tb); r.R = make_int2(dA, dB); }
+                else { r.T = make_int2(tb, ta); r.R = make_int2(dB, dA); }
+                continue;
+            }
+        }
+        r.C = sdown == 0 ? make_int2(down, up) : make_int2(up, down);
+    }
+}
+
+// A vertex on a cycle (weakest key ks, DK per slot c): path id, position, forest slots,
+// predecessor slot, path length at the path-ID vertex.  Reading c11/c12/c15/c9.
+struct CycOut {
+    int32_t l, pos, len;
+    int2 f;
+    uint8_t pdir;
+    int ncyc;
+};
+__device__ __forceinline__ CycOut cycle_finish(int32_t g, int2 nb, ulonglong2 ek, uint64_t ks, int2 c) {
+    CycOut o;
+    o.l = key_min_end(ks);
+    const int dir = (c.x & 1) ? 0 : 1;           // the slot whose near endpoint is x
+    o.pos = ((dir ? c.y : c.x) >> 1) + 1;
+    o.len = (g == o.l) ? (c.x >> 1) + (c.y >> 1) + 1 : 0;
+    const int rs = (ek.x == ks) ? 0 : ((ek.y == ks) ? 1 : -1);
+    o.f = nb;
+    o.ncyc = 0;
+    if (rs == 0) { o.f = make_int2(nb.y, -1); o.ncyc = g < nb.x; }
+    else if (rs == 1) { o.f = make_int2(nb.x, -1); o.ncyc = g < nb.y; }
+    o.pdir = (uint8_t)((rs == 0) ? (dir ^ 1) : dir);
+    return o;
+}
+
+constexpr int32_t kLocDone = INT_MIN;
+
+// the expand pass needs only the tile's slots and weights
+struct TileSmemE {
+    int2 nb[LB];
+    float2 w[LB];
+    int32_t b0, tend;
+};  // loc marker: the tile pass wrote the final results
+
+// Tile pass: full-window scan; local cycles finished here; per-vertex local results and
+// the reduced records of boundary vertices.
+__global__ void __launch_bounds__(LT, 1) k_lf_full1(ForestArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    TileSmemF& s = *reinterpret_cast<TileSmemF*>(smem_raw);
+    const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
+    load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
+    const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
+    ulonglong2 ek[VPT];
+    slot_keys(a, s, b0, ek);
+    int2 orig[VPT];
+#pragma unroll
+    for (int k = 0; k < VPT; k++) orig[k] = s.nb[threadIdx.x + k * LT];
+    VRes o[VPT];
+    tile_rank_full(s, b0, ek, o, a.ctl + kCtlStat);
+    int ncyc = 0;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        const int2 nb = orig[k];
+        const bool r0 = nb.x >= 0 && !is_local(nb.x, T);
+        const bool r1 = nb.y >= 0 && !is_local(nb.y, T);
+        const bool boundary = g < a.hi && (r0 || r1);
+        if (g < a.hi) {
+            if (o[k].cyc) {
+                const CycOut c = cycle_finish(g, nb, ek[k], o[k].Ks, o[k].C);
+                a.path_id[g] = c.l;
+                a.pos[g] = c.pos;
+                a.len[g] = c.len;
+                a.forest[g] = c.f;
+                a.pdir[g] = c.pdir;
+                ncyc += c.ncyc;
+                a.loc2[g] = make_int2(kLocDone, 0);
+            } else {
+                const uint32_t tt = (uint32_t)(uint16_t)o[k].T.x | ((uint32_t)(uint16_t)o[k].T.y << 16);
+                const uint32_t rr = (uint32_t)(uint16_t)o[k].R.x | ((uint32_t)(uint16_t)o[k].R.y << 16);
+                a.loc2[g] = make_int2((int)tt, (int)rr);
+            }
+        }
+        const int idx = list_append(a.list1, &a.ctl[kCtlCnt1], g, boundary);
+        if (boundary) {
+            int2 q, rl, dk;
+            ulonglong2 kk;
+#pragma unroll
+            for (int i = 0; i < 2; i++) {
+                const int32_t x = i ? nb.y : nb.x;
+                int32_t qi, ri, di;
+                uint64_t ki;
+                if (x < 0) { qi = -(g + 1); ri = 0; ki = KEY_INF; di = 0; }
+                else if (!is_local(x, T)) { qi = x; ri = 1; ki = i ? ek[k].y : ek[k].x; di = g < x ? 1 : 0; }
+                else {
+                    const int t = i ? o[k].T.y : o[k].T.x;
+                    const int2 nbt = s.nb[t];
+                    const int32_t xo = outward_slot(nbt, T) ? nbt.y : nbt.x;
+                    const int32_t tg = b0 + t;
+                    qi = xo < 0 ? -(tg + 1) : tg;
+                    ri = i ? o[k].R.y : o[k].R.x;
+                    ki = i ? o[k].Kn.y : o[k].Kn.x;
+                    di = i ? o[k].Dn.y : o[k].Dn.x;
+                }
+                if (i) { q.y = qi; rl.y = ri; kk.y = ki; dk.y = di; }
+                else { q.x = qi; rl.x = ri; kk.x = ki; dk.x = di; }
+            }
+            a.bidx1[g] = idx;
+            a.cq[idx] = q;
+            a.cq_r[idx] = rl;
+            a.cq_k[idx] = kk;
+            a.cq_dk[idx] = dk;
+        }
+    }
+#pragma unroll
+    for (int o2 = 16; o2; o2 >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o2);
+    if ((threadIdx.x & 31) == 0 && ncyc) atomicAdd(&a.ctl[kCtlNcyc], ncyc);
+}
+
+// ---------------------------------------------------------------------------
+// Reduced scan with full windows over the boundary list (pointers are list positions)
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void win_append(int32_t& R, uint64_t& K, int32_t& D, int32_t Rw, uint64_t Kw, int32_t Dw) {
+    if (Kw < K) { K = Kw; D = 2 * R + Dw; }
+    R += Rw;
+}
+
+constexpr int kRedSmallF = 3 * 1024;   // lists up to this size: one CTA, shared memory
+
+struct RedSmemF {
+    int2 q[kRedSmallF];
+    int2 r[kRedSmallF];
+    int2 d[kRedSmallF];
+    uint64_t k0[kRedSmallF];
+    uint64_t k1[kRedSmallF];
+};
+
+// list position of the vertex a record points at (markers pass through)
+__device__ __forceinline__ int2 to_pos(const ForestArgs& a, int2 q) {
+    return make_int2(q.x >= 0 ? __ldg(a.bidx1 + q.x) : q.x, q.y >= 0 ? __ldg(a.bidx1 + q.y) : q.y);
+}
+
+template <int T>
+__device__ void red_full_small(const ForestArgs& a, int cnt, int* ctl, RedSmemF& S) {
+    constexpr int NPT = (kRedSmallF + T - 1) / T;
+    const int tid = threadIdx.x;
+    bool fin[NPT];
+    int notdone = 0;
+#pragma unroll
+    for (int k = 0; k < NPT; k++) {
+        const int idx = tid + k * T;
+        fin[k] = true;
+        if (idx >= cnt) continue;
+        const int2 q = to_pos(a, a.cq[idx]);
+        const ulonglong2 kk = a.cq_k[idx];
+        S.q[idx] = q;
+        S.r[idx] = a.cq_r[idx];
+        S.d[idx] = a.cq_dk[idx];
+        S.k0[idx] = kk.x;
+        S.k1[idx] = kk.y;
+        fin[k] = q.x < 0 && q.y < 0;
+        notdone |= !fin[k];
+    }
+    if (__syncthreads_or(notdone)) {
+        for (int step = 0; step < a.max_steps; step++) {
+            int2 nq[NPT], nr[NPT], nd[NPT];
+            uint64_t nk0[NPT], nk1[NPT];
+            notdone = 0;
+#pragma unroll
+            for (int k = 0; k < NPT; k++) {
+                if (fin[k]) continue;
+                const int me = tid + k * T;
+                const int2 q = S.q[me];
+                nq[k] = q; nr[k] = S.r[me]; nd[k] = S.d[me]; nk0[k] = S.k0[me]; nk1[k] = S.k1[me];
+#pragma unroll
+                for (int i = 0; i < 2; i++) {
+                    const int w = i ? q.y : q.x;
+                    if (w < 0) continue;
+                    const int2 qw = S.q[w];
+                    int32_t R = i ? nr[k].y : nr[k].x, D = i ? nd[k].y : nd[k].x;
+                    uint64_t K = i ? nk1[k] : nk0[k];
+                    const int2 rw = S.r[w], dw = S.d[w];
+                    const uint64_t kw0 = S.k0[w], kw1 = S.k1[w];
+                    int j = -1;
+                    if (qw.x != me) j = 0;
+                    else if (qw.y != me) j = 1;
+                    int32_t tgt = w;
+                    if (j >= 0) {
+                        tgt = j ? qw.y : qw.x;
+                        win_append(R, K, D, j ? rw.y : rw.x, j ? kw1 : kw0, j ? dw.y : dw.x);
+                    } else {  // stall (reading c13): see node_scan_full
+                        if (kw0 < K) { K = kw0; D = 2 * R + dw.x; }
+                        if (kw1 < K) { K = kw1; D = 2 * R + dw.y; }
+                    }
+                    if (i) { nq[k].y = tgt; nr[k].y = R; nd[k].y = D; nk1[k] = K; }
+                    else { nq[k].x = tgt; nr[k].x = R; nd[k].x = D; nk0[k] = K; }
+                }
+                const bool path_done = nq[k].x < 0 && nq[k].y < 0;
+                const bool cyc_done = nq[k].x >= 0 && nq[k].y >= 0 && nk0[k] == nk1[k];
+                notdone |= !(path_done || cyc_done);
+            }
+            __syncthreads();
+#pragma unroll
+            for (int k = 0; k < NPT; k++) {
+                if (fin[k]) continue;
+                const int me = tid + k * T;
+                S.q[me] = nq[k]; S.r[me] = nr[k]; S.d[me] = nd[k]; S.k0[me] = nk0[k]; S.k1[me] = nk1[k];
+                fin[k] = nq[k].x < 0 && nq[k].y < 0;
+            }
+            const int any = __syncthreads_or(notdone);
+            if (tid == 0) ctl[step] = 1;
+            if (!any) break;
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < NPT; k++) {
+        const int idx = tid + k * T;
+        if (idx >= cnt) continue;
+        a.end2[idx] = S.q[idx];   // markers (paths); cycles keep list positions >= 0
+        a.dist2[idx] = S.r[idx];
+        a.kraw[idx] = make_ulonglong2(S.k0[idx], S.k1[idx]);
+        a.dk2[idx] = S.d[idx];
+    }
+}
+
+// one synchronous step over list positions t0, t0+stride, ... (grid path)
+__device__ __forceinline__ int red_full_step(const ForestArgs& a, int cnt, int step, int t0, int stride) {
+    const int2* __restrict__ qs = a.rq1[step & 1];
+    int2* __restrict__ qd = a.rq1[(step & 1) ^ 1];
+    const ulonglong2* __restrict__ ks = a.rk1[step & 1];
+    ulonglong2* __restrict__ kd = a.rk1[(step & 1) ^ 1];
+    const int2* __restrict__ rs = a.rr2[step & 1];
+    int2* __restrict__ rd = a.rr2[(step & 1) ^ 1];
+    const int2* __restrict__ ds = a.rdk[step & 1];
+    int2* __restrict__ dd = a.rdk[(step & 1) ^ 1];
+    int notdone = 0;
+    for (int me = t0; me < cnt; me += stride) {
+        const int2 q = qs[me];
+        int2 r = rs[me], d = ds[me];
+        ulonglong2 k = ks[me];
+        if (q.x < 0 && q.y < 0) {  // final: keep both buffers equal
+            qd[me] = q; kd[me] = k; rd[me] = r; dd[me] = d;
+            continue;
+        }
+        int2 nq = q;
+#pragma unroll
+        for (int i = 0; i < 2; i++) {
+            const int w = i ? q.y : q.x;
+            if (w < 0) continue;
+            const int2 qw = qs[w], rw = rs[w], dw = ds[w];
+            const ulonglong2 kw = ks[w];
+            int32_t R = i ? r.y : r.x, D = i ? d.y : d.x;
+            uint64_t K = i ? k.y : k.x;
+            int j = -1;
+            if (qw.x != me) j = 0;
+            else if (qw.y != me) j = 1;
+            int32_t tgt = w;
+            if (j >= 0) {
+                tgt = j ? qw.y : qw.x;
+                win_append(R, K, D, j ? rw.y : rw.x, j ? kw.y : kw.x, j ? dw.y : dw.x);
+            } else {
+                if (kw.x < K) { K = kw.x; D = 2 * R + dw.x; }
+                if (kw.y < K) { K = kw.y; D = 2 * R + dw.y; }
+            }
+            if (i) { nq.y = tgt; r.y = R; d.y = D; k.y = K; } else { nq.x = tgt; r.x = R; d.x = D; k.x = K; }
+        }
+        qd[me] = nq; kd[me] = k; rd[me] = r; dd[me] = d;
+        const bool path_done = nq.x < 0 && nq.y < 0;
+        const bool cyc_done = nq.x >= 0 && nq.y >= 0 && k.x == k.y;
+        notdone += (path_done || cyc_done) ? 0 : 1;
+    }
+    return notdone;
+}
+
+__global__ void __launch_bounds__(RT) k_red_full(ForestArgs a) {
+    __shared__ int sh[32];
+    extern __shared__ __align__(16) unsigned char red_smem[];
+    pdl_trigger();
+    const int cnt = *(volatile int*)&a.ctl[kCtlCnt1];
+    int* ctl = a.ctl + kCtlRed1;
+    if (cnt <= kRedSmallF) {
+        if (blockIdx.x == 0) red_full_small<RT>(a, cnt, ctl, *reinterpret_cast<RedSmemF*>(red_smem));
+        return;
+    }
+    cg::grid_group grid = cg::this_grid();
+    const int stride = gridDim.x * blockDim.x;
+    const int t0 = blockIdx.x * blockDim.x + threadIdx.x;
+    for (int me = t0; me < cnt; me += stride) {
+        const int2 q = to_pos(a, a.cq[me]);
+        a.rq1[0][me] = q;
+        a.rk1[0][me] = a.cq_k[me];
+        a.rr2[0][me] = a.cq_r[me];
+        a.rdk[0][me] = a.cq_dk[me];
+    }
+    grid.sync();
+    int step = 0;
+    for (; step < a.max_steps; step++) {
+        int notdone = red_full_step(a, cnt, step, t0, stride);
+#pragma unroll
+        for (int o = 16; o; o >>= 1) notdone += __shfl_xor_sync(0xffffffffu, notdone, o);
+        if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = notdone;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int tot = 0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); w++) tot += sh[w];
+            if (tot) atomicAdd(&ctl[step], tot);
+        }
+        grid.sync();
+        if (*(volatile int*)&ctl[step] == 0) { step++; break; }
+    }
+    const int fb = step & 1;
+    for (int me = t0; me < cnt; me += stride) {
+        a.end2[me] = a.rq1[fb][me];
+        a.dist2[me] = a.rr2[fb][me];
+        a.kraw[me] = a.rk1[fb][me];
+        a.dk2[me] = a.rdk[fb][me];
+    }
+}
+
+// Expand pass: every vertex not finished by the tile pass combines its local result with
+// the reduced results of its terminals; then the tile's path lengths are scanned into
+// offsets (the last CTA turns the tile totals into an exclusive prefix).
+__global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    TileSmemE& s = *reinterpret_cast<TileSmemE*>(smem_raw);
+    __shared__ int sh[32];
+    __shared__ int last;
+    const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
+    load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
+    const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
+    ulonglong2 ek[VPT];
+    slot_keys(a, s, b0, ek);
+    pdl_wait();  // the factor slots above predate the chain; the tile/reduced results do not
+    int lens[VPT];
+    int ncyc = 0;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        lens[k] = 0;
+        if (g >= a.hi) continue;
+        const int2 lc = a.loc2[g];
+        if (lc.x == kLocDone) { lens[k] = a.len[g]; continue; }
+        const int2 nb = s.nb[u];
+        const int Tl[2] = {(int)(lc.x & 0xffff), (int)((uint32_t)lc.x >> 16)};
+        const int Rl[2] = {(int)(lc.y & 0xffff), (int)((uint32_t)lc.y >> 16)};
+        int32_t E[2], D[2];
+        int bi[2], so[2];
+        bool cyc = false;
+#pragma unroll
+        for (int i = 0; i < 2; i++) {
+            const int t = Tl[i];
+            const int2 nbt = s.nb[t];
+            so[i] = (t == u) ? i : outward_slot(nbt, T);
+            const int32_t xo = so[i] ? nbt.y : nbt.x;
+            bi[i] = -1;
+            if (xo < 0) { E[i] = b0 + t; D[i] = Rl[i]; continue; }
+            bi[i] = a.bidx1[b0 + t];
+            const int2 e = a.end2[bi[i]];
+            const int32_t fq = so[i] ? e.y : e.x;
+            if (fq >= 0) { cyc = true; continue; }
+            const int2 dd = a.dist2[bi[i]];
+            E[i] = -(fq + 1);
+            D[i] = Rl[i] + (so[i] ? dd.y : dd.x);
+        }
+        if (!cyc) {
+            const int dir = E[0] <= E[1] ? 0 : 1;
+            const int32_t l = E[dir];
+            a.path_id[g] = l;
+            a.pos[g] = D[dir] + 1;
+            a.pdir[g] = (uint8_t)dir;
+            a.forest[g] = nb;
+            lens[k] = (l == g) ? D[0] + D[1] + 1 : 0;
+            a.len[g] = lens[k];
+            continue;
+        }
+        // on a cycle through other tiles: both terminals continue
+        const ulonglong2 kf0 = a.kraw[bi[0]];
+        const uint64_t ks = so[0] ? kf0.y : kf0.x;
+        const int2 dA = a.dk2[bi[0]], dB = a.dk2[bi[1]];
+        const int dko0 = so[0] ? dA.y : dA.x, dko1 = so[1] ? dB.y : dB.x;
+        // is the weakest edge inside this vertex's segment?  t0's inward window spans it
+        const ulonglong2 ki = a.cq_k[bi[0]];
+        const int2 di = a.cq_dk[bi[0]];
+        const uint64_t kseg = so[0] ? ki.x : ki.y;
+        const int dseg = so[0] ? di.x : di.y;
+        int2 c;
+        if (kseg == ks) {
+            const int delta = dseg >> 1, bt = dseg & 1;
+            if (Rl[0] >= delta + 1) c = make_int2(2 * (Rl[0] - delta - 1) + (bt ^ 1), 2 * Rl[1] + dko1);
+            else c = make_int2(2 * Rl[0] + dko0, 2 * (delta - Rl[0]) + bt);
+        } else {
+            c = make_int2(2 * Rl[0] + dko0, 2 * Rl[1] + dko1);
+        }
+        const CycOut co = cycle_finish(g, nb, ek[k], ks, c);
+        a.path_id[g] = co.l;
+        a.pos[g] = co.pos;
+        a.pdir[g] = co.pdir;
+        a.forest[g] = co.f;
+        lens[k] = co.len;
+        a.len[g] = co.len;
+        ncyc += co.ncyc;
+    }
+    // tile-local exclusive prefix of the path lengths (thread t owns u = t, t+LT: scan in
+    // that order is not id order, so scan pairs (t, t+LT) as two halves)
+    {
+        int tot0 = 0, tot1 = 0;
+        const int e0 = block_scan_sum_excl(lens[0], sh, &tot0);
+        const int e1 = VPT > 1 ? block_scan_sum_excl(lens[VPT - 1], sh, &tot1) : 0;
+        const int32_t g0 = b0 + (int)threadIdx.x;
+        if (g0 < a.hi && lens[0]) a.off[g0] = e0;
+        if (VPT > 1) {
+            const int32_t g1 = b0 + (int)threadIdx.x + LT;
+            if (g1 < a.hi && lens[VPT - 1]) a.off[g1] = tot0 + e1;
+        }
+        static_assert(VPT <= 2, "tile offsets assume at most two vertices per thread");
+        if (threadIdx.x == 0) a.tsum[blockIdx.x] = tot0 + tot1;
+    }
+#pragma unroll
+    for (int o2 = 16; o2; o2 >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o2);
+    if ((threadIdx.x & 31) == 0 && ncyc) atomicAdd(&a.ctl[kCtlNcyc], ncyc);
+    // the last CTA: exclusive prefix of the tile totals; the cycle count
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        last = atomicAdd(&a.ctl[kCtlTicket3], 1) == (int)gridDim.x - 1;
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    int carry = 0;
+    for (int base = 0; base < (int)gridDim.x; base += LT) {
+        const int i = base + threadIdx.x;
+        const int v = i < (int)gridDim.x ? __ldcg(a.tsum + i) : 0;
+        int chunk = 0;
+        const int ex = block_scan_sum_excl(v, sh, &chunk);
+        if (i < (int)gridDim.x) a.tsum[i] = carry + ex;
+        carry += chunk;
+    }
+    if (threadIdx.x == 0 && a.n_cycles) *a.n_cycles = (unsigned long long)__ldcg(&a.ctl[kCtlNcyc]);
 }
 
 static size_t scan_temp_bytes(int64_t N) {
@@ -1585,8 +2519,13 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     t.bidx1 = c.take<int32_t>(n);
     t.bidx2 = c.take<int32_t>(n);
     t.pdir = c.take<uint8_t>(n);
-    t.tsum = c.take<int32_t>(n / kOffChunk + 2);
+    t.tsum = c.take<int32_t>(n / 256 + 2);  // per offset chunk (8192) or tile (>= 256)
     t.cq_k = c.take<ulonglong2>(n);
+    t.cq_r = c.take<int2>(n);
+    t.cq_dk = c.take<int2>(n);
+    t.dk2 = c.take<int2>(n);
+    t.rdk[0] = c.take<int2>(n);
+    t.rdk[1] = c.take<int2>(n);
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
     if (w) *w = t;
@@ -1620,6 +2559,12 @@ static int forest_prepare() {
                                  (int)sizeof(RedSmem)));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)sizeof(RedSmem)));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_full1, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sizeof(TileSmemF)));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_red_full, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sizeof(RedSmemF)));
+    LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_full2, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sizeof(TileSmemE)));
     attr_done = true;
     return LF_OK;
 }
@@ -1633,8 +2578,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     int rcp = forest_prepare();
     if (rcp) return rcp;
-    const int smem = (int)sizeof(TileSmem);
-    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));  // n_cycles: zeroed by k_lf_local1
+    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
     ForestArgs a;
     memset(&a, 0, sizeof(a));
     a.N = N;
@@ -1646,63 +2590,49 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     for (int i = 0; i < 2; i++) {
         a.rq1[i] = w.rq1[i];
         a.rk1[i] = w.rk1[i];
-        a.rq2[i] = w.rq2[i];
         a.rr2[i] = w.rr2[i];
+        a.rdk[i] = w.rdk[i];
     }
-    a.cyc_k = w.cyc_k;
     a.bidx1 = w.bidx1;
-    a.bidx2 = w.bidx2;
-    a.loc1 = w.loc1;
-    a.kst = w.kst;
     a.loc2 = w.loc2;
     a.list1 = w.list1;
     a.end2 = w.end2;
     a.dist2 = w.dist2;
-    a.list2 = w.list2;
+    a.kraw = w.kraw;
+    a.dk2 = w.dk2;
     a.cq = w.cq;
     a.cq_k = w.cq_k;
+    a.cq_r = w.cq_r;
+    a.cq_dk = w.cq_dk;
     a.ctl = w.ctl;
     a.path_id = path_id;
     a.pos = pos;
     a.len = w.len;
+    a.off = w.off;
+    a.tsum = w.tsum;
     a.pdir = w.pdir;
     a.n_cycles = (unsigned long long*)n_cycles;
     a.max_steps = max_steps_for(N) < kMaxSteps ? max_steps_for(N) : kMaxSteps;
     const int tiles = (int)((N + LB - 1) / LB);
     {
-        LF_PROF("lf_local1", -1, s);
-        k_lf_local1<<<tiles, LT, smem, s>>>(a);
+        LF_PROF("lf_tile", -1, s);
+        k_lf_full1<<<tiles, LT, sizeof(TileSmemF), s>>>(a);
         LF_CUDA(cudaGetLastError());
     }
     {
-        LF_PROF("red_scan_cycles", -1, s);
-        int rc = coop_launch(k_red_scan<true>, RT, a, s, sizeof(RedSmem));
+        LF_PROF("red_scan", -1, s);
+        int rc = coop_launch(k_red_full, RT, a, s, sizeof(RedSmemF));
         if (rc) return rc;
     }
     {
-        LF_PROF("lf_local2", -1, s);
-        LF_CUDA(launch_pdl(k_lf_local2, tiles, LT, kTileSmemNoKeys, s, a));
-    }
-    {
-        LF_PROF("red_scan_ranks", -1, s);
-        int rc = coop_launch(k_red_scan<false>, RT, a, s, sizeof(RedSmem));
-        if (rc) return rc;
-    }
-    {
-        LF_PROF("lf_local3", -1, s);
-        LF_CUDA(launch_pdl(k_lf_local3, tiles, LT, kTileSmemNoKeys, s, a));
-    }
-    {
-        LF_PROF("path_offsets", -1, s);
-        const int chunks = (int)((N + kOffChunk - 1) / kOffChunk);
-        LF_CUDA(launch_pdl(k_path_offsets, chunks, kOffT, 0, s, N, (const int32_t*)w.len, w.off, w.tsum,
-                           w.ctl + kCtlTicket3));
+        LF_PROF("lf_expand", -1, s);
+        LF_CUDA(launch_pdl(k_lf_full2, tiles, LT, sizeof(TileSmemE), s, a));
     }
     {
         LF_PROF(tri ? "perm_tridiag" : "perm", -1, s);
         LF_CUDA(launch_pdl(k_perm_tri, persistent_grid((const void*)k_perm_tri, 256), 256, 0, s, N,
                            (const int32_t*)path_id, (const int32_t*)pos, (const int32_t*)w.off,
-                           (const int32_t*)w.tsum, (const uint8_t*)w.pdir, (const int2*)forest,
+                           (const int32_t*)w.tsum, (int)LB, (const uint8_t*)w.pdir, (const int2*)forest,
                            (const int2*)pi2, tri ? (const float2*)tri->pi2_val : nullptr,
                            tri ? tri->diag : nullptr, perm, iperm, tri ? tri->a : nullptr,
                            tri ? tri->b : nullptr, tri ? tri->c : nullptr));

@@ -131,6 +131,10 @@ struct ForestWs {
     int32_t* tsum;         // [chunks + 2] path-length sums per offset chunk -> exclusive prefix
     int2* cq;              // [list position] reduced-graph records of the boundary list being
     ulonglong2* cq_k;      //   scanned: stride pointers (vertex ids), keys or distances
+    int2* cq_r;            // [list position] single-pass forest: initial window lengths,
+    int2* cq_dk;           //   initial DK (2 * distance to the minimum's near endpoint + bit),
+    int2* dk2;             //   final DK per direction
+    int2* rdk[2];          //   grid-path ping-pong DK
 };
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w);
 
