@@ -58,6 +58,7 @@ constexpr int kCtlCnt1 = 128;     // boundary list sizes
 constexpr int kCtlCnt2 = 129;
 constexpr int kCtlTicket3 = 130;  // finished-CTA ticket of k_path_offsets / k_lf_full2 (the last one scans tsum)
 constexpr int kCtlNcyc = 131;     // broken cycles (single-pass forest)
+constexpr int kCtlGridBar = 133;  // arrival counter of k_red_full's grid barrier
 constexpr int kMaxSteps = 62;
 constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
 // ctl[192] splitter nodes (cycle pass), [193] unvisited vertices (fallback), [194] tiles
@@ -1516,6 +1517,7 @@ __global__ void __launch_bounds__(kOffT) k_path_offsets(int64_t N, const int32_t
 // prefix + intra-tile prefix; the forest neighbour in slot pdir[v] is perm[r-1], the other
 // one perm[r+1], so a[r] / c[r] are copied from the factor's signed slot values
 constexpr int kPermBatch = 4;  // vertices per thread per iteration (loads in flight)
+constexpr int kNoSlot = 2;     // pdir: no predecessor / successor slot (k_lf_full1/2)
 
 __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __restrict__ path_id,
                                                   const int32_t* __restrict__ pos,
@@ -1546,13 +1548,11 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
             iperm[v] = r[b];
             perm[r[b]] = (int32_t)v;
             if (ta) {
-                const int2 f = __ldg(forest + v);
-                const int2 pn = __ldg(pi2 + v);
                 const float2 pv = __ldg(pi2_val + v);
                 const int d = __ldg(pdir + v);
-                const int32_t pred = d ? f.y : f.x, succ = d ? f.x : f.y;
-                ta[r[b]] = pred >= 0 ? ((pn.x == pred) ? pv.x : pv.y) : 0.0f;
-                tc[r[b]] = succ >= 0 ? ((pn.x == succ) ? pv.x : pv.y) : 0.0f;
+                const int ps = d & 3, ss = (d >> 2) & 3;
+                ta[r[b]] = ps == kNoSlot ? 0.0f : (ps ? pv.y : pv.x);
+                tc[r[b]] = ss == kNoSlot ? 0.0f : (ss ? pv.y : pv.x);
                 tb[r[b]] = __ldg(diag + v);
             }
         }
@@ -1708,6 +1708,8 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
     const int tid = threadIdx.x;
     const Tile T = tile_of(s);
     const int tlen = T.tend - T.b0;
+    int* ctlp = stats - kCtlStat;
+    LF_PHASE_INIT;
     if (tid == 0) s.nspl = 0;
     const auto linked_prev = [&](int u) {
         const int2 nb = s.nb[u];
@@ -1824,6 +1826,7 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
         s.r.vw[u] = vw;
     }
     __syncthreads();
+    LF_PHASE(ctlp, 0);
     // 1. splitters (run ends, terminals, hashed vertices); run cycles -3, interiors -2
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
@@ -1856,6 +1859,7 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
         s.recS[u] = make_short2(-1, -1);
     }
     __syncthreads();
+    LF_PHASE(ctlp, 1);
     const int C = s.nspl;
     if (tid == 0 && stats) atomicAdd(&stats[0], C);
     // 2. walks from every (node, slot) to the next node: length, weakest link and its DK
@@ -1894,6 +1898,7 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
         else { s.P[i].x = ptr; s.R[i].x = (short)dist; s.DK[i].x = (short)dk; s.K0[i] = km; s.WK0[i] = km; s.WD[i].x = (short)dk; }
     }
     __syncthreads();
+    LF_PHASE(ctlp, 2);
     // 3. node scan
     if (C <= 32 * kWarpScanNodes) {
         if (tid < 32) node_scan_full<kWarpScanNodes, true>(s, C, stats);
@@ -1901,6 +1906,7 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
     } else {
         node_scan_full<VPT, false>(s, C, stats);
     }
+    LF_PHASE(ctlp, 3);
     // 4. nodes and walk-visited vertices
     bool unvisited[VPT];
     int any_unvisited = 0;
@@ -1992,6 +1998,7 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
     }
     // 5. interior run vertices and run cycles, from the run ends' node windows
     __syncthreads();
+    LF_PHASE(ctlp, 4);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = tid + k * LT;
@@ -2048,10 +2055,21 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
         }
         r.C = sdown == 0 ? make_int2(down, up) : make_int2(up, down);
     }
+    LF_PHASE(ctlp, 5);
 }
 
 // A vertex on a cycle (weakest key ks, DK per slot c): path id, position, forest slots,
 // predecessor slot, path length at the path-ID vertex.  Reading c11/c12/c15/c9.
+// predecessor / successor slots of a vertex in pi2-slot terms for the tridiagonal copy:
+// bits 0-1 the slot toward the path-ID end (position p - 1), bits 2-3 the other one
+// (p + 1); kNoSlot where that neighbour is missing or its edge was removed (slot rs)
+__device__ __forceinline__ uint8_t nbr_slots(int2 nb, int dir, int rs) {
+    const int32_t xp = dir ? nb.y : nb.x, xs = dir ? nb.x : nb.y;
+    const int ps = (dir != rs && xp >= 0) ? dir : kNoSlot;
+    const int ss = ((dir ^ 1) != rs && xs >= 0) ? (dir ^ 1) : kNoSlot;
+    return (uint8_t)(ps | (ss << 2));
+}
+
 struct CycOut {
     int32_t l, pos, len;
     int2 f;
@@ -2069,8 +2087,141 @@ __device__ __forceinline__ CycOut cycle_finish(int32_t g, int2 nb, ulonglong2 ek
     o.ncyc = 0;
     if (rs == 0) { o.f = make_int2(nb.y, -1); o.ncyc = g < nb.x; }
     else if (rs == 1) { o.f = make_int2(nb.x, -1); o.ncyc = g < nb.y; }
-    o.pdir = (uint8_t)((rs == 0) ? (dir ^ 1) : dir);
+    o.pdir = nbr_slots(nb, dir, rs);
     return o;
+}
+
+// ---------------------------------------------------------------------------
+// Reduced scan with full windows over the boundary list (pointers are list positions)
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void win_append(int32_t& R, uint64_t& K, int32_t& D, int32_t Rw, uint64_t Kw, int32_t Dw) {
+    if (Kw < K) { K = Kw; D = 2 * R + Dw; }
+    R += Rw;
+}
+
+constexpr int kRedSmallF = 4 * 1024;   // lists up to this size: one CTA, shared memory
+
+// per direction d (0/1): the pointer, length, DK and minimum key of every node's window
+struct RedSmemF {
+    int2 q[kRedSmallF];
+    int r[2][kRedSmallF];
+    int d[2][kRedSmallF];
+    uint64_t k[2][kRedSmallF];
+};
+
+// list position of the vertex a record points at (markers pass through)
+__device__ __forceinline__ int2 to_pos(const ForestArgs& a, int2 q) {
+    return make_int2(q.x >= 0 ? __ldcg(a.bidx1 + q.x) : q.x, q.y >= 0 ? __ldcg(a.bidx1 + q.y) : q.y);
+}
+
+// The whole reduced scan in one CTA's shared memory (lists up to kRedSmallF nodes).  Each
+// step reads, per direction, the target's pointers and then only the continuing window's
+// length / DK / key (one direction's arrays: fewer random shared-memory words).
+template <int T>
+__device__ void red_full_small(const ForestArgs& a, int cnt, int* ctl, RedSmemF& S) {
+    constexpr int NPT = (kRedSmallF + T - 1) / T;
+    const int tid = threadIdx.x;
+#ifdef LF_PHASE_TIMING
+    const unsigned long long t_start = gtime();
+#endif
+    bool fin[NPT];
+    int notdone = 0;
+    {
+        int2 q[NPT], r[NPT], d[NPT];
+        ulonglong2 kk[NPT];
+#pragma unroll
+        for (int k = 0; k < NPT; k++) {
+            const int idx = tid + k * T;
+            if (idx >= cnt) continue;
+            q[k] = __ldcg(a.cq + idx);
+            r[k] = __ldcg(a.cq_r + idx);
+            d[k] = __ldcg(a.cq_dk + idx);
+            kk[k] = __ldcg(a.cq_k + idx);
+        }
+#pragma unroll
+        for (int k = 0; k < NPT; k++) {
+            const int idx = tid + k * T;
+            if (idx >= cnt) continue;
+            q[k] = to_pos(a, q[k]);
+        }
+#pragma unroll
+        for (int k = 0; k < NPT; k++) {
+            const int idx = tid + k * T;
+            fin[k] = true;
+            if (idx >= cnt) continue;
+            S.q[idx] = q[k];
+            S.r[0][idx] = r[k].x; S.r[1][idx] = r[k].y;
+            S.d[0][idx] = d[k].x; S.d[1][idx] = d[k].y;
+            S.k[0][idx] = kk[k].x; S.k[1][idx] = kk[k].y;
+            fin[k] = q[k].x < 0 && q[k].y < 0;
+            notdone |= !fin[k];
+        }
+    }
+    const int any0 = __syncthreads_or(notdone);
+    RS_MARK(0);
+    if (any0) {
+        for (int step = 0; step < a.max_steps; step++) {
+            int2 nq[NPT];
+            int nr[NPT][2], nd[NPT][2];
+            uint64_t nk[NPT][2];
+            notdone = 0;
+#pragma unroll
+            for (int k = 0; k < NPT; k++) {
+                if (fin[k]) continue;
+                const int me = tid + k * T;
+                const int2 q = S.q[me];
+                nq[k] = q;
+#pragma unroll
+                for (int i = 0; i < 2; i++) {
+                    const int w = i ? q.y : q.x;
+                    int32_t R = S.r[i][me], D = S.d[i][me];
+                    uint64_t K = S.k[i][me];
+                    if (w >= 0) {
+                        const int2 qw = S.q[w];
+                        int j = -1;
+                        if (qw.x != me) j = 0;
+                        else if (qw.y != me) j = 1;
+                        if (j >= 0) {
+                            win_append(R, K, D, S.r[j][w], S.k[j][w], S.d[j][w]);
+                            if (i) nq[k].y = j ? qw.y : qw.x; else nq[k].x = j ? qw.y : qw.x;
+                        } else {  // stall (reading c13): see node_scan_full
+                            const uint64_t kw0 = S.k[0][w], kw1 = S.k[1][w];
+                            if (kw0 < K) { K = kw0; D = 2 * R + S.d[0][w]; }
+                            if (kw1 < K) { K = kw1; D = 2 * R + S.d[1][w]; }
+                        }
+                    }
+                    nr[k][i] = R; nd[k][i] = D; nk[k][i] = K;
+                }
+                const bool path_done = nq[k].x < 0 && nq[k].y < 0;
+                const bool cyc_done = nq[k].x >= 0 && nq[k].y >= 0 && nk[k][0] == nk[k][1];
+                notdone |= !(path_done || cyc_done);
+            }
+            __syncthreads();
+#pragma unroll
+            for (int k = 0; k < NPT; k++) {
+                if (fin[k]) continue;
+                const int me = tid + k * T;
+                S.q[me] = nq[k];
+#pragma unroll
+                for (int i = 0; i < 2; i++) { S.r[i][me] = nr[k][i]; S.d[i][me] = nd[k][i]; S.k[i][me] = nk[k][i]; }
+                fin[k] = nq[k].x < 0 && nq[k].y < 0;
+            }
+            const int any = __syncthreads_or(notdone);
+            if (tid == 0) ctl[step] = 1;
+            if (!any) break;
+        }
+    }
+    RS_MARK(1);
+#pragma unroll
+    for (int k = 0; k < NPT; k++) {
+        const int idx = tid + k * T;
+        if (idx >= cnt) continue;
+        a.end2[idx] = S.q[idx];   // markers (paths); cycles keep list positions >= 0
+        a.dist2[idx] = make_int2(S.r[0][idx], S.r[1][idx]);
+        a.kraw[idx] = make_ulonglong2(S.k[0][idx], S.k[1][idx]);
+        a.dk2[idx] = make_int2(S.d[0][idx], S.d[1][idx]);
+    }
+    RS_MARK(2);
 }
 
 constexpr int32_t kLocDone = INT_MIN;
@@ -2088,15 +2239,20 @@ __global__ void __launch_bounds__(LT, 1) k_lf_full1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemF& s = *reinterpret_cast<TileSmemF*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
+    LF_PHASE_INIT;
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
+    LF_PHASE(a.ctl, 6);
     int2 orig[VPT];
 #pragma unroll
     for (int k = 0; k < VPT; k++) orig[k] = s.nb[threadIdx.x + k * LT];
     VRes o[VPT];
     tile_rank_full(s, b0, ek, o, a.ctl + kCtlStat);
+#ifdef LF_PHASE_TIMING
+    ph_t = clock64();
+#endif
     int ncyc = 0;
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
@@ -2156,113 +2312,9 @@ __global__ void __launch_bounds__(LT, 1) k_lf_full1(ForestArgs a) {
 #pragma unroll
     for (int o2 = 16; o2; o2 >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o2);
     if ((threadIdx.x & 31) == 0 && ncyc) atomicAdd(&a.ctl[kCtlNcyc], ncyc);
+    LF_PHASE(a.ctl, 7);
 }
-
-// ---------------------------------------------------------------------------
-// Reduced scan with full windows over the boundary list (pointers are list positions)
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ void win_append(int32_t& R, uint64_t& K, int32_t& D, int32_t Rw, uint64_t Kw, int32_t Dw) {
-    if (Kw < K) { K = Kw; D = 2 * R + Dw; }
-    R += Rw;
-}
-
-constexpr int kRedSmallF = 3 * 1024;   // lists up to this size: one CTA, shared memory
-
-struct RedSmemF {
-    int2 q[kRedSmallF];
-    int2 r[kRedSmallF];
-    int2 d[kRedSmallF];
-    uint64_t k0[kRedSmallF];
-    uint64_t k1[kRedSmallF];
-};
-
-// list position of the vertex a record points at (markers pass through)
-__device__ __forceinline__ int2 to_pos(const ForestArgs& a, int2 q) {
-    return make_int2(q.x >= 0 ? __ldg(a.bidx1 + q.x) : q.x, q.y >= 0 ? __ldg(a.bidx1 + q.y) : q.y);
-}
-
-template <int T>
-__device__ void red_full_small(const ForestArgs& a, int cnt, int* ctl, RedSmemF& S) {
-    constexpr int NPT = (kRedSmallF + T - 1) / T;
-    const int tid = threadIdx.x;
-    bool fin[NPT];
-    int notdone = 0;
-#pragma unroll
-    for (int k = 0; k < NPT; k++) {
-        const int idx = tid + k * T;
-        fin[k] = true;
-        if (idx >= cnt) continue;
-        const int2 q = to_pos(a, a.cq[idx]);
-        const ulonglong2 kk = a.cq_k[idx];
-        S.q[idx] = q;
-        S.r[idx] = a.cq_r[idx];
-        S.d[idx] = a.cq_dk[idx];
-        S.k0[idx] = kk.x;
-        S.k1[idx] = kk.y;
-        fin[k] = q.x < 0 && q.y < 0;
-        notdone |= !fin[k];
-    }
-    if (__syncthreads_or(notdone)) {
-        for (int step = 0; step < a.max_steps; step++) {
-            int2 nq[NPT], nr[NPT], nd[NPT];
-            uint64_t nk0[NPT], nk1[NPT];
-            notdone = 0;
-#pragma unroll
-            for (int k = 0; k < NPT; k++) {
-                if (fin[k]) continue;
-                const int me = tid + k * T;
-                const int2 q = S.q[me];
-                nq[k] = q; nr[k] = S.r[me]; nd[k] = S.d[me]; nk0[k] = S.k0[me]; nk1[k] = S.k1[me];
-#pragma unroll
-                for (int i = 0; i < 2; i++) {
-                    const int w = i ? q.y : q.x;
-                    if (w < 0) continue;
-                    const int2 qw = S.q[w];
-                    int32_t R = i ? nr[k].y : nr[k].x, D = i ? nd[k].y : nd[k].x;
-                    uint64_t K = i ? nk1[k] : nk0[k];
-                    const int2 rw = S.r[w], dw = S.d[w];
-                    const uint64_t kw0 = S.k0[w], kw1 = S.k1[w];
-                    int j = -1;
-                    if (qw.x != me) j = 0;
-                    else if (qw.y != me) j = 1;
-                    int32_t tgt = w;
-                    if (j >= 0) {
-                        tgt = j ? qw.y : qw.x;
-                        win_append(R, K, D, j ? rw.y : rw.x, j ? kw1 : kw0, j ? dw.y : dw.x);
-                    } else {  // stall (reading c13): see node_scan_full
-                        if (kw0 < K) { K = kw0; D = 2 * R + dw.x; }
-                        if (kw1 < K) { K = kw1; D = 2 * R + dw.y; }
-                    }
-                    if (i) { nq[k].y = tgt; nr[k].y = R; nd[k].y = D; nk1[k] = K; }
-                    else { nq[k].x = tgt; nr[k].x = R; nd[k].x = D; nk0[k] = K; }
-                }
-                const bool path_done = nq[k].x < 0 && nq[k].y < 0;
-                const bool cyc_done = nq[k].x >= 0 && nq[k].y >= 0 && nk0[k] == nk1[k];
-                notdone |= !(path_done || cyc_done);
-            }
-            __syncthreads();
-#pragma unroll
-            for (int k = 0; k < NPT; k++) {
-                if (fin[k]) continue;
-                const int me = tid + k * T;
-                S.q[me] = nq[k]; S.r[me] = nr[k]; S.d[me] = nd[k]; S.k0[me] = nk0[k]; S.k1[me] = nk1[k];
-                fin[k] = nq[k].x < 0 && nq[k].y < 0;
-            }
-            const int any = __syncthreads_or(notdone);
-            if (tid == 0) ctl[step] = 1;
-            if (!any) break;
-        }
-    }
-#pragma unroll
-    for (int k = 0; k < NPT; k++) {
-        const int idx = tid + k * T;
-        if (idx >= cnt) continue;
-        a.end2[idx] = S.q[idx];   // markers (paths); cycles keep list positions >= 0
-        a.dist2[idx] = S.r[idx];
-        a.kraw[idx] = make_ulonglong2(S.k0[idx], S.k1[idx]);
-        a.dk2[idx] = S.d[idx];
-    }
-}
+constexpr size_t kFull1Smem = sizeof(TileSmemF);
 
 // one synchronous step over list positions t0, t0+stride, ... (grid path)
 __device__ __forceinline__ int red_full_step(const ForestArgs& a, int cnt, int step, int t0, int stride) {
@@ -2276,9 +2328,9 @@ __device__ __forceinline__ int red_full_step(const ForestArgs& a, int cnt, int s
     int2* __restrict__ dd = a.rdk[(step & 1) ^ 1];
     int notdone = 0;
     for (int me = t0; me < cnt; me += stride) {
-        const int2 q = qs[me];
-        int2 r = rs[me], d = ds[me];
-        ulonglong2 k = ks[me];
+        const int2 q = __ldcg(qs + me);
+        int2 r = __ldcg(rs + me), d = __ldcg(ds + me);
+        ulonglong2 k = __ldcg(ks + me);
         if (q.x < 0 && q.y < 0) {  // final: keep both buffers equal
             qd[me] = q; kd[me] = k; rd[me] = r; dd[me] = d;
             continue;
@@ -2288,8 +2340,8 @@ __device__ __forceinline__ int red_full_step(const ForestArgs& a, int cnt, int s
         for (int i = 0; i < 2; i++) {
             const int w = i ? q.y : q.x;
             if (w < 0) continue;
-            const int2 qw = qs[w], rw = rs[w], dw = ds[w];
-            const ulonglong2 kw = ks[w];
+            const int2 qw = __ldcg(qs + w), rw = __ldcg(rs + w), dw = __ldcg(ds + w);
+            const ulonglong2 kw = __ldcg(ks + w);
             int32_t R = i ? r.y : r.x, D = i ? d.y : d.x;
             uint64_t K = i ? k.y : k.x;
             int j = -1;
@@ -2313,17 +2365,39 @@ __device__ __forceinline__ int red_full_step(const ForestArgs& a, int cnt, int s
     return notdone;
 }
 
+// Grid barrier of k_red_full (monotone arrival counter; `gen` counts the barriers passed).
+// k_red_full runs one CTA per SM with a CTA's worth of shared memory each and is launched
+// after its stream predecessor has completed, while its own successor can only launch
+// once every CTA has triggered (after the last barrier): all its CTAs are co-resident.
+__device__ __forceinline__ void red_grid_sync(int* ctr, int& gen) {
+    __syncthreads();
+    gen++;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(ctr, 1);
+        const int target = gen * (int)gridDim.x;
+        while (true) {
+            int v;
+            asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+            if (v >= target) break;
+            __nanosleep(32);
+        }
+    }
+    __syncthreads();
+}
+
 __global__ void __launch_bounds__(RT) k_red_full(ForestArgs a) {
     __shared__ int sh[32];
     extern __shared__ __align__(16) unsigned char red_smem[];
-    pdl_trigger();
     const int cnt = *(volatile int*)&a.ctl[kCtlCnt1];
     int* ctl = a.ctl + kCtlRed1;
     if (cnt <= kRedSmallF) {
+        pdl_trigger();  // the expand kernel's tile-only prologue overlaps this scan
         if (blockIdx.x == 0) red_full_small<RT>(a, cnt, ctl, *reinterpret_cast<RedSmemF*>(red_smem));
         return;
     }
-    cg::grid_group grid = cg::this_grid();
+    int* bar = a.ctl + kCtlGridBar;
+    int gen = 0;
     const int stride = gridDim.x * blockDim.x;
     const int t0 = blockIdx.x * blockDim.x + threadIdx.x;
     for (int me = t0; me < cnt; me += stride) {
@@ -2333,7 +2407,7 @@ __global__ void __launch_bounds__(RT) k_red_full(ForestArgs a) {
         a.rr2[0][me] = a.cq_r[me];
         a.rdk[0][me] = a.cq_dk[me];
     }
-    grid.sync();
+    red_grid_sync(bar, gen);
     int step = 0;
     for (; step < a.max_steps; step++) {
         int notdone = red_full_step(a, cnt, step, t0, stride);
@@ -2346,92 +2420,147 @@ __global__ void __launch_bounds__(RT) k_red_full(ForestArgs a) {
             for (int w = 0; w < (int)(blockDim.x >> 5); w++) tot += sh[w];
             if (tot) atomicAdd(&ctl[step], tot);
         }
-        grid.sync();
-        if (*(volatile int*)&ctl[step] == 0) { step++; break; }
+        red_grid_sync(bar, gen);
+        if (__ldcg(&ctl[step]) == 0) { step++; break; }
     }
+    pdl_trigger();
     const int fb = step & 1;
     for (int me = t0; me < cnt; me += stride) {
-        a.end2[me] = a.rq1[fb][me];
-        a.dist2[me] = a.rr2[fb][me];
-        a.kraw[me] = a.rk1[fb][me];
-        a.dk2[me] = a.rdk[fb][me];
+        a.end2[me] = __ldcg(&a.rq1[fb][me]);
+        a.dist2[me] = __ldcg(&a.rr2[fb][me]);
+        a.kraw[me] = __ldcg(&a.rk1[fb][me]);
+        a.dk2[me] = __ldcg(&a.rdk[fb][me]);
     }
 }
 
 // Expand pass: every vertex not finished by the tile pass combines its local result with
 // the reduced results of its terminals; then the tile's path lengths are scanned into
-// offsets (the last CTA turns the tile totals into an exclusive prefix).
+// tile-local offsets and a tile total.  Everything that depends only on the tile pass
+// (tile slots, slot keys, local results, terminal list positions, segment records -- all
+// complete before the reduced scan even started) is done BEFORE pdl_wait, overlapping the
+// reduced scan; vertices whose two terminals are path ends finish there too.
+
+struct ExpState {       // a vertex waiting for reduced results
+    int bi0, bi1;       // list positions of its terminals (-1: a path end)
+    int so;             // bit i: outward slot of terminal i
+    int R0, R1;
+    uint64_t kseg;      // t0's inward segment window: weakest key, DK
+    int dseg;
+};
+
 __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemE& s = *reinterpret_cast<TileSmemE*>(smem_raw);
     __shared__ int sh[32];
-    __shared__ int last;
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
-    pdl_wait();  // the factor slots above predate the chain; the tile/reduced results do not
     int lens[VPT];
+    bool wait[VPT];
+    ExpState st[VPT];
     int ncyc = 0;
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int u = threadIdx.x + k * LT;
         const int32_t g = b0 + u;
         lens[k] = 0;
+        wait[k] = false;
         if (g >= a.hi) continue;
         const int2 lc = a.loc2[g];
         if (lc.x == kLocDone) { lens[k] = a.len[g]; continue; }
-        const int2 nb = s.nb[u];
         const int Tl[2] = {(int)(lc.x & 0xffff), (int)((uint32_t)lc.x >> 16)};
-        const int Rl[2] = {(int)(lc.y & 0xffff), (int)((uint32_t)lc.y >> 16)};
-        int32_t E[2], D[2];
-        int bi[2], so[2];
-        bool cyc = false;
+        st[k].R0 = (int)(lc.y & 0xffff);
+        st[k].R1 = (int)((uint32_t)lc.y >> 16);
+        st[k].so = 0;
+        int bi[2];
 #pragma unroll
         for (int i = 0; i < 2; i++) {
             const int t = Tl[i];
             const int2 nbt = s.nb[t];
-            so[i] = (t == u) ? i : outward_slot(nbt, T);
-            const int32_t xo = so[i] ? nbt.y : nbt.x;
-            bi[i] = -1;
-            if (xo < 0) { E[i] = b0 + t; D[i] = Rl[i]; continue; }
-            bi[i] = a.bidx1[b0 + t];
+            const int so = (t == u) ? i : outward_slot(nbt, T);
+            st[k].so |= so << i;
+            bi[i] = (so ? nbt.y : nbt.x) < 0 ? -1 : a.bidx1[b0 + t];
+        }
+        st[k].bi0 = bi[0];
+        st[k].bi1 = bi[1];
+        if (bi[0] < 0 && bi[1] < 0) {  // a path inside the tile: both terminals are its ends
+            const int2 nb = s.nb[u];
+            const int32_t E0 = b0 + Tl[0], E1 = b0 + Tl[1];
+            const int dir = E0 <= E1 ? 0 : 1;
+            const int32_t l = dir ? E1 : E0;
+            a.path_id[g] = l;
+            a.pos[g] = (dir ? st[k].R1 : st[k].R0) + 1;
+            a.pdir[g] = nbr_slots(nb, dir, -1);
+            a.forest[g] = nb;
+            lens[k] = (l == g) ? st[k].R0 + st[k].R1 + 1 : 0;
+            continue;
+        }
+        wait[k] = true;
+        st[k].kseg = KEY_INF;
+        st[k].dseg = 0;
+        if (bi[0] >= 0) {  // t0's inward window spans this vertex's segment
+            const ulonglong2 ki = a.cq_k[bi[0]];
+            const int2 di = a.cq_dk[bi[0]];
+            st[k].kseg = (st[k].so & 1) ? ki.x : ki.y;
+            st[k].dseg = (st[k].so & 1) ? di.x : di.y;
+        }
+    }
+    pdl_wait();  // the reduced scan's results
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        if (!wait[k]) continue;
+        const int u = threadIdx.x + k * LT;
+        const int32_t g = b0 + u;
+        const int2 nb = s.nb[u];
+        const int Rl[2] = {st[k].R0, st[k].R1};
+        const int bi[2] = {st[k].bi0, st[k].bi1};
+        int32_t E[2], D[2];
+        int dko[2] = {0, 0};
+        uint64_t ks = KEY_INF;
+        bool cyc = false;
+#pragma unroll
+        for (int i = 0; i < 2; i++) {
+            const int so = (st[k].so >> i) & 1;
+            if (bi[i] < 0) {  // a path end (the vertex reached it inside the tile)
+                const int t = i ? (int)((uint32_t)a.loc2[g].x >> 16) : (int)(a.loc2[g].x & 0xffff);
+                E[i] = b0 + t;
+                D[i] = Rl[i];
+                continue;
+            }
             const int2 e = a.end2[bi[i]];
-            const int32_t fq = so[i] ? e.y : e.x;
-            if (fq >= 0) { cyc = true; continue; }
+            const int32_t fq = so ? e.y : e.x;
+            if (fq >= 0) {
+                cyc = true;
+                const int2 dk = a.dk2[bi[i]];
+                dko[i] = so ? dk.y : dk.x;
+                if (i == 0) { const ulonglong2 kf = a.kraw[bi[0]]; ks = so ? kf.y : kf.x; }
+                continue;
+            }
             const int2 dd = a.dist2[bi[i]];
             E[i] = -(fq + 1);
-            D[i] = Rl[i] + (so[i] ? dd.y : dd.x);
+            D[i] = Rl[i] + (so ? dd.y : dd.x);
         }
         if (!cyc) {
             const int dir = E[0] <= E[1] ? 0 : 1;
             const int32_t l = E[dir];
             a.path_id[g] = l;
             a.pos[g] = D[dir] + 1;
-            a.pdir[g] = (uint8_t)dir;
+            a.pdir[g] = nbr_slots(nb, dir, -1);
             a.forest[g] = nb;
             lens[k] = (l == g) ? D[0] + D[1] + 1 : 0;
-            a.len[g] = lens[k];
             continue;
         }
-        // on a cycle through other tiles: both terminals continue
-        const ulonglong2 kf0 = a.kraw[bi[0]];
-        const uint64_t ks = so[0] ? kf0.y : kf0.x;
-        const int2 dA = a.dk2[bi[0]], dB = a.dk2[bi[1]];
-        const int dko0 = so[0] ? dA.y : dA.x, dko1 = so[1] ? dB.y : dB.x;
-        // is the weakest edge inside this vertex's segment?  t0's inward window spans it
-        const ulonglong2 ki = a.cq_k[bi[0]];
-        const int2 di = a.cq_dk[bi[0]];
-        const uint64_t kseg = so[0] ? ki.x : ki.y;
-        const int dseg = so[0] ? di.x : di.y;
+        // on a cycle through other tiles (both terminals continue): is its weakest edge
+        // inside this vertex's segment?  (reading c9)
         int2 c;
-        if (kseg == ks) {
-            const int delta = dseg >> 1, bt = dseg & 1;
-            if (Rl[0] >= delta + 1) c = make_int2(2 * (Rl[0] - delta - 1) + (bt ^ 1), 2 * Rl[1] + dko1);
-            else c = make_int2(2 * Rl[0] + dko0, 2 * (delta - Rl[0]) + bt);
+        if (st[k].kseg == ks) {
+            const int delta = st[k].dseg >> 1, bt = st[k].dseg & 1;
+            if (Rl[0] >= delta + 1) c = make_int2(2 * (Rl[0] - delta - 1) + (bt ^ 1), 2 * Rl[1] + dko[1]);
+            else c = make_int2(2 * Rl[0] + dko[0], 2 * (delta - Rl[0]) + bt);
         } else {
-            c = make_int2(2 * Rl[0] + dko0, 2 * Rl[1] + dko1);
+            c = make_int2(2 * Rl[0] + dko[0], 2 * Rl[1] + dko[1]);
         }
         const CycOut co = cycle_finish(g, nb, ek[k], ks, c);
         a.path_id[g] = co.l;
@@ -2439,46 +2568,56 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
         a.pdir[g] = co.pdir;
         a.forest[g] = co.f;
         lens[k] = co.len;
-        a.len[g] = co.len;
         ncyc += co.ncyc;
     }
-    // tile-local exclusive prefix of the path lengths (thread t owns u = t, t+LT: scan in
-    // that order is not id order, so scan pairs (t, t+LT) as two halves)
+    // tile-local exclusive prefix of the path lengths in id order (thread t owns
+    // u = t + k LT: one block scan per k, carried)
     {
-        int tot0 = 0, tot1 = 0;
-        const int e0 = block_scan_sum_excl(lens[0], sh, &tot0);
-        const int e1 = VPT > 1 ? block_scan_sum_excl(lens[VPT - 1], sh, &tot1) : 0;
-        const int32_t g0 = b0 + (int)threadIdx.x;
-        if (g0 < a.hi && lens[0]) a.off[g0] = e0;
-        if (VPT > 1) {
-            const int32_t g1 = b0 + (int)threadIdx.x + LT;
-            if (g1 < a.hi && lens[VPT - 1]) a.off[g1] = tot0 + e1;
+        int carry = 0;
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            int tot = 0;
+            const int e = block_scan_sum_excl(lens[k], sh, &tot);
+            const int32_t gk = b0 + (int)threadIdx.x + k * LT;
+            if (gk < a.hi && lens[k]) a.off[gk] = carry + e;
+            carry += tot;
         }
-        static_assert(VPT <= 2, "tile offsets assume at most two vertices per thread");
-        if (threadIdx.x == 0) a.tsum[blockIdx.x] = tot0 + tot1;
+        if (threadIdx.x == 0) a.tsum[blockIdx.x] = carry;
     }
 #pragma unroll
     for (int o2 = 16; o2; o2 >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o2);
     if ((threadIdx.x & 31) == 0 && ncyc) atomicAdd(&a.ctl[kCtlNcyc], ncyc);
-    // the last CTA: exclusive prefix of the tile totals; the cycle count
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        last = atomicAdd(&a.ctl[kCtlTicket3], 1) == (int)gridDim.x - 1;
-    }
-    __syncthreads();
-    if (!last) return;
-    __threadfence();
+}
+
+// Exclusive prefix of the tile totals (one CTA; the permutation kernel then finds the
+// new index r = tsum[tile of l] + off[l] + p - 1, reading c14), and the cycle count.
+constexpr int kPrefT = 1024, kPrefPT = 8;
+
+__global__ void __launch_bounds__(kPrefT) k_tile_prefix(int32_t* tsum, int tiles, const int* ctl,
+                                                        unsigned long long* n_cycles) {
+    __shared__ int sh[32];
+    pdl_wait();
+    pdl_trigger();
+    if (n_cycles && threadIdx.x == 0) *n_cycles = (unsigned long long)__ldcg(ctl + kCtlNcyc);
     int carry = 0;
-    for (int base = 0; base < (int)gridDim.x; base += LT) {
-        const int i = base + threadIdx.x;
-        const int v = i < (int)gridDim.x ? __ldcg(a.tsum + i) : 0;
-        int chunk = 0;
-        const int ex = block_scan_sum_excl(v, sh, &chunk);
-        if (i < (int)gridDim.x) a.tsum[i] = carry + ex;
-        carry += chunk;
+    for (int base = 0; base < tiles; base += kPrefT * kPrefPT) {
+        int x[kPrefPT], sum = 0;
+#pragma unroll
+        for (int j = 0; j < kPrefPT; j++) {
+            const int i = base + threadIdx.x * kPrefPT + j;
+            x[j] = i < tiles ? __ldcg(tsum + i) : 0;
+            sum += x[j];
+        }
+        int total = 0;
+        int run = carry + block_scan_sum_excl(sum, sh, &total);
+#pragma unroll
+        for (int j = 0; j < kPrefPT; j++) {
+            const int i = base + threadIdx.x * kPrefPT + j;
+            if (i < tiles) tsum[i] = run;
+            run += x[j];
+        }
+        carry += total;
     }
-    if (threadIdx.x == 0 && a.n_cycles) *a.n_cycles = (unsigned long long)__ldcg(&a.ctl[kCtlNcyc]);
 }
 
 static size_t scan_temp_bytes(int64_t N) {
@@ -2560,7 +2699,7 @@ static int forest_prepare() {
     LF_CUDA(cudaFuncSetAttribute((const void*)k_red_scan<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)sizeof(RedSmem)));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_full1, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)sizeof(TileSmemF)));
+                                 (int)kFull1Smem));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_red_full, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)sizeof(RedSmemF)));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_full2, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -2616,13 +2755,15 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     const int tiles = (int)((N + LB - 1) / LB);
     {
         LF_PROF("lf_tile", -1, s);
-        k_lf_full1<<<tiles, LT, sizeof(TileSmemF), s>>>(a);
+        k_lf_full1<<<tiles, LT, kFull1Smem, s>>>(a);
         LF_CUDA(cudaGetLastError());
     }
     {
         LF_PROF("red_scan", -1, s);
-        int rc = coop_launch(k_red_full, RT, a, s, sizeof(RedSmemF));
-        if (rc) return rc;
+#ifndef LF_NO_GRID_RED  // diagnostics only: measures the launch cost (wrong for lists > kRedSmallF)
+        // one CTA per SM (its shared memory admits no second one): see red_grid_sync
+        LF_CUDA(launch_pdl(k_red_full, sm_count(), RT, sizeof(RedSmemF), s, a));
+#endif
     }
     {
         LF_PROF("lf_expand", -1, s);
@@ -2630,6 +2771,8 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF(tri ? "perm_tridiag" : "perm", -1, s);
+        LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, tiles, (const int*)w.ctl,
+                           (unsigned long long*)n_cycles));
         LF_CUDA(launch_pdl(k_perm_tri, persistent_grid((const void*)k_perm_tri, 256), 256, 0, s, N,
                            (const int32_t*)path_id, (const int32_t*)pos, (const int32_t*)w.off,
                            (const int32_t*)w.tsum, (int)LB, (const uint8_t*)w.pdir, (const int2*)forest,
