@@ -1636,18 +1636,31 @@ struct VRes {
     int2 Dn;          //   window DK per slot
 };
 
-// bidirectional scan over the splitter nodes with full windows; WARP: warp 0 alone
-template <int NPN, bool WARP>
-__device__ __forceinline__ void node_scan_full(TileSmemF& s, int C, int* stats) {
+// named barrier 1 over the first nt threads (nt a multiple of 32), with an OR reduction
+__device__ __forceinline__ void group_sync(int nt) {
+    if (nt == LT) __syncthreads();
+    else asm volatile("bar.sync 1, %0;" ::"r"(nt) : "memory");
+}
+__device__ __forceinline__ int group_or(int nt, int pred) {
+    if (nt == LT) return __syncthreads_or(pred);
+    int r;
+    asm volatile("{\n\t.reg .pred p, q;\n\tsetp.ne.s32 p, %1, 0;\n\tbar.red.or.pred q, 1, %2, p;\n\tselp.s32 %0, 1, 0, q;\n\t}"
+                 : "=r"(r) : "r"(pred), "r"(nt) : "memory");
+    return r;
+}
+
+// bidirectional scan over the splitter nodes with full windows, by the first nt threads
+// (NPN nodes each); the caller synchronises the block afterwards
+template <int NPN>
+__device__ __forceinline__ void node_scan_full(TileSmemF& s, int C, int nt, int* stats) {
     const int tid = threadIdx.x;
-    constexpr int STRIDE = WARP ? 32 : LT;
     for (int step = 0; step < 16; step++) {
         int notdone = 0;
         short2 nP[NPN], nR[NPN], nD[NPN];
         uint64_t nk0[NPN], nk1[NPN];
 #pragma unroll
         for (int k = 0; k < NPN; k++) {
-            const int i = tid + k * STRIDE;
+            const int i = tid + k * nt;
             if (i >= C) continue;
             const short2 p = s.P[i];
             short2 q = p, r = s.R[i], dk = s.DK[i];
@@ -1685,15 +1698,14 @@ __device__ __forceinline__ void node_scan_full(TileSmemF& s, int C, int* stats) 
             const bool cyc_done = q.x >= 0 && q.y >= 0 && k0 == k1;
             notdone |= !(path_done || cyc_done);
         }
-        if (WARP) __syncwarp(); else __syncthreads();
+        group_sync(nt);
 #pragma unroll
         for (int k = 0; k < NPN; k++) {
-            const int i = tid + k * STRIDE;
+            const int i = tid + k * nt;
             if (i >= C) continue;
             s.P[i] = nP[k]; s.R[i] = nR[k]; s.DK[i] = nD[k]; s.K0[i] = nk0[k]; s.K1[i] = nk1[k];
         }
-        const bool any = WARP ? (__syncwarp(), __any_sync(0xffffffffu, notdone)) : __syncthreads_or(notdone);
-        if (!any) {
+        if (!group_or(nt, notdone)) {
             if (tid == 0 && stats) atomicMax(&stats[4], step + 1);
             break;
         }
@@ -1899,12 +1911,16 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
     }
     __syncthreads();
     LF_PHASE(ctlp, 2);
-    // 3. node scan
-    if (C <= 32 * kWarpScanNodes) {
-        if (tid < 32) node_scan_full<kWarpScanNodes, true>(s, C, stats);
+    // 3. node scan: one node per thread of the smallest group that holds them all
+    if (C <= 128 && LT > 128) {
+        if (tid < 128) node_scan_full<1>(s, C, 128, stats);
+        __syncthreads();
+    } else if (C <= 512 && LT > 512) {
+        if (tid < 512) node_scan_full<1>(s, C, 512, stats);
         __syncthreads();
     } else {
-        node_scan_full<VPT, false>(s, C, stats);
+        node_scan_full<VPT>(s, C, LT, stats);
+        __syncthreads();
     }
     LF_PHASE(ctlp, 3);
     // 4. nodes and walk-visited vertices
