@@ -133,6 +133,14 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
                    for kk in range(1, len(live_rows)))
     # linear forest: B_LF = 40N attributed to the kernel that moves it;
     # block-local intermediates (loc1/loc2, boundary records) are implementation traffic
+    # single-pass forest: the tile pass reads the factor; the tile pass (local
+    # vertices) and the expand pass (the rest) together write forest, path_id, pos once each
+    if base == "lf_tile":
+        return 16 * N  # read pi2 + pi2_w
+    if base == "lf_expand":
+        return 16 * N  # write forest, path_id, pos
+    if base == "red_scan":
+        return 0  # boundary records only: implementation traffic
     if base == "lf_local1":
         return 16 * N  # read pi2 + pi2_w
     if base == "lf_local2":
@@ -452,7 +460,8 @@ def main():
         ev1.synchronize()
         prof_step_ms.append(ev0.elapsed_time(ev1))
         recs = lf.profile_collect()
-        launches_per_step = len(recs)
+        # one record per stage; the perm stage launches k_tile_prefix + k_perm_tri
+        launches_per_step = sum(2 if nm in ("perm", "perm_tridiag") else 1 for nm, _ in recs)
         for nm, ms in recs:
             kern.setdefault(nm, []).append(ms)
     torch.cuda.synchronize()
