@@ -49,6 +49,9 @@ constexpr uint64_t KEY_INF = ~0ull;
 #ifndef LF_LMINB
 #define LF_LMINB 2
 #endif
+#ifndef LF_F1MINB
+#define LF_F1MINB 1   // resident tile-pass CTAs per SM (k_lf_full1)
+#endif
 constexpr int LB = LF_LB;         // vertices per block-local tile
 constexpr int LT = LF_LT;         // threads per tile CTA
 constexpr int VPT = LB / LT;      // vertices per thread
@@ -2251,7 +2254,7 @@ struct TileSmemE {
 
 // Tile pass: full-window scan; local cycles finished here; per-vertex local results and
 // the reduced records of boundary vertices.
-__global__ void __launch_bounds__(LT, 1) k_lf_full1(ForestArgs a) {
+__global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemF& s = *reinterpret_cast<TileSmemF*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
