@@ -20,6 +20,8 @@
 #include "lf_common.cuh"
 #include "lf_internal.h"
 
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 namespace cg = cooperative_groups;
@@ -795,12 +797,15 @@ __device__ __forceinline__ void finalize_body(const int* flags, int M, int m, in
             }
         *rounds = r;
     }
-    if (live) {
-        for (int i = threadIdx.x; i < 2 * M; i += blockDim.x) {
+    if (live) {  // one warp per counter: lanes sum two of its 64 slots
+        const int lane = threadIdx.x & 31;
+        for (int i = threadIdx.x >> 5; i < 2 * M; i += blockDim.x >> 5) {
             const int k = i % M, which = i / M;
-            unsigned long long t = 0;
-            for (int j = 0; j < 64; j++) t += part[(size_t)k * 128 + which * 64 + j];
-            live[i] = (int64_t)t;
+            const unsigned long long* q = part + (size_t)k * 128 + which * 64;
+            unsigned long long t = q[lane] + q[lane + 32];
+#pragma unroll
+            for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+            if (lane == 0) live[i] = (int64_t)t;
         }
     }
 }
@@ -827,6 +832,8 @@ struct FusedArgs {
     int G;
     int32_t* rounds;     // finalize outputs (k_finalize's work, done by CTA 0 in the last round)
     int64_t* live;
+    int cached;          // try the shared-memory cached mode (rounds_cached) first
+    int32_t* bail;       // grid-wide "does not fit" flag of the cached mode (zeroed per run)
 };
 
 #ifndef LF_FUSED_T
@@ -838,10 +845,301 @@ struct FusedArgs {
 #ifndef LF_FUSED_GRID
 #define LF_FUSED_GRID 0      // > 0: absolute CTA count of the fused rounds kernel
 #endif
+// ---------------------------------------------------------------------------
+// Cached mode of rounds 1..M-1: every CTA owns a fixed slice of the round-1 worklist L1
+// (the rows mutual(0) kept) and keeps those rows -- state, confirmed keys and their CSR
+// entries as keys -- in shared memory for all rounds.  Rows outside L1 never propose
+// again and are never proposed to, so the slices cover every row the
+// rounds touch.  Per round only two gathers remain: the state bytes of the entries'
+// targets (before propose, L15/L17) and the partners' proposals (before mutual, L27),
+// each one L2 level with every load of a CTA in flight together, instead of the
+// worklist -> rowptr -> col -> state chains of the uncached phases.  The semantics are
+// those of propose_phase/mutual_phase entry for entry (same eligibility tests in the same
+// order, same keys), so the factor is bit-identical.  A slice that does not fit (too many
+// rows, entries or a row longer than kCacheMaxRow) makes the whole grid bail out (a
+// grid-wide flag) before anything global is written; the uncached loop then runs.
+// ---------------------------------------------------------------------------
+constexpr int kCacheMaxRow = 256;
+template <int NN>
+struct CacheCap {
+    static constexpr int R = 1024;    // rows per CTA
+    static constexpr int E = 6144;    // CSR entries per CTA
+};
+template <int NN>
+struct CacheSmem {
+    uint64_t pik[CacheCap<NN>::R * NN];   // confirmed keys per row, descending (0 = empty)
+    uint64_t prk[CacheCap<NN>::R * NN];   // this round's proposals (keys; 0 = none)
+    uint64_t ek[CacheCap<NN>::E];         // entry keys make_key(a_vj, j); 0 = not an edge
+    int64_t rs[CacheCap<NN>::R];          // CSR start of each row
+    int32_t gid[CacheCap<NN>::R];
+    int32_t rlen[CacheCap<NN>::R];        // CSR row length (live-nnz counter)
+    int32_t est[CacheCap<NN>::R];         // first pool entry of each row
+    int16_t erow[CacheCap<NN>::E];        // row of each pool entry
+    uint8_t esj[CacheCap<NN>::E];         // state byte of the entry's target (this round)
+    uint8_t st[CacheCap<NN>::R];          // state byte (degree | charge)
+    uint8_t act[CacheCap<NN>::R];         // bit 0: in this round's worklist, bit 1: retired
+    int pool, ovf;
+    unsigned long long red[3][LF_FUSED_T / 32];
+};
+template <int NN>
+constexpr size_t cache_smem_bytes() { return sizeof(CacheSmem<NN>); }
+
+template <int NN>
+__device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
+    using Cap = CacheCap<NN>;
+    constexpr int T = LF_FUSED_T;
+    constexpr int RPT = Cap::R / T;   // rows per thread
+    constexpr int EPT = Cap::E / T;   // pool entries per thread
+    extern __shared__ __align__(16) unsigned char fz_smem[];
+    CacheSmem<NN>& S = *reinterpret_cast<CacheSmem<NN>*>(fz_smem);
+    const int tid = threadIdx.x;
+    const ProposeArgs& pa = f.pa;
+    const int L = *(volatile const int32_t*)&f.counts[1];   // round-1 worklist (mutual(0))
+    const int C = gridDim.x;
+    const int RPC = (L + C - 1) / C;
+    const int base = blockIdx.x * RPC;
+    const int nmine = max(0, min(L - base, RPC));
+    const int32_t* wl1 = f.wl[1];
+    if (tid == 0) { S.pool = 0; S.ovf = RPC > Cap::R || f.M > kMaxFlagRounds; }
+    __syncthreads();
+    // A. own rows: id, state, confirmed keys, row extent
+#pragma unroll
+    for (int q = 0; q < RPT; q++) {
+        const int s = tid + q * T;
+        if (s >= nmine || s >= Cap::R) continue;
+        const int32_t v = __ldcg(wl1 + base + s);
+        const uint8_t stt = __ldcg(f.ma.state + v);
+        int32_t pj[NN];
+        float pw[NN], pv[NN];
+#pragma unroll
+        for (int t = 0; t < NN; t++) {
+            const int64_t o = (int64_t)v * NN + t;
+            pj[t] = f.ma.pi[o];
+            pw[t] = f.ma.pi_w[o];
+            pv[t] = f.ma.pi_val ? f.ma.pi_val[o] : 0.0f;
+        }
+        const int64_t r0 = __ldg(pa.rowptr + v), r1 = __ldg(pa.rowptr + v + 1);
+        S.gid[s] = v;
+        S.st[s] = stt;
+        S.act[s] = 1;
+        const int deg = stt & ST_DEG;
+#pragma unroll
+        for (int t = 0; t < NN; t++)
+            S.pik[s * NN + t] = t < deg ? make_key_abs(pw[t], __float_as_uint(pv[t]) >> 31, pj[t]) : 0ull;
+        const int len = (int)(r1 - r0);
+        S.rs[s] = r0;
+        S.rlen[s] = len;
+        const int off = atomicAdd(&S.pool, len);
+        S.est[s] = off;
+        if (len > kCacheMaxRow || off + len > Cap::E) S.ovf = 1;
+    }
+    __syncthreads();
+    if (tid == 0 && S.ovf) atomicOr(f.bail, 1);
+    grid.sync();
+    if (*(volatile int32_t*)f.bail) return false;   // uniform: nothing global written yet
+#pragma unroll
+    for (int q = 0; q < RPT; q++) {
+        const int s = tid + q * T;
+        if (s >= nmine) continue;
+        const int e0 = S.est[s], len = S.rlen[s];
+        for (int e = 0; e < len; e++) S.erow[e0 + e] = (int16_t)s;
+    }
+    __syncthreads();
+    const int P = S.pool;
+    // B. the rows' entries as keys (diagonal and zeros -- not edges, L31/L231 -- as key 0)
+    {
+        int32_t j[EPT];
+        float x[EPT];
+#pragma unroll
+        for (int q = 0; q < EPT; q++) {
+            const int p = tid + q * T;
+            if (p >= P) continue;
+            const int sr = S.erow[p];
+            const int64_t e = S.rs[sr] + (p - S.est[sr]);
+            j[q] = __ldg(pa.col + e);
+            x[q] = __ldg(pa.val + e);
+        }
+#pragma unroll
+        for (int q = 0; q < EPT; q++) {
+            const int p = tid + q * T;
+            if (p >= P) continue;
+            const bool edge = j[q] != S.gid[S.erow[p]] && (__float_as_uint(x[q]) & 0x7FFFFFFFu) != 0u;
+            S.ek[p] = edge ? make_key(x[q], j[q]) : 0ull;
+        }
+    }
+    __syncthreads();
+    for (int k = 1; k < f.M; k++) {
+        const bool charging = (k % f.m) != f.k_m;
+        const bool last = k == f.M - 1;
+        // the targets' state bytes (round k), every load of the CTA in flight together
+        {
+            uint8_t sj[EPT];
+#pragma unroll
+            for (int q = 0; q < EPT; q++) {
+                const int p = tid + q * T;
+                sj[q] = (uint8_t)NN;
+                if (p >= P) continue;
+                const uint64_t key = S.ek[p];
+                if (key && (S.act[S.erow[p]] & 1)) sj[q] = __ldcg(f.ma.state + key_col(key));
+            }
+#pragma unroll
+            for (int q = 0; q < EPT; q++) {
+                const int p = tid + q * T;
+                if (p < P) S.esj[p] = sj[q];
+            }
+        }
+        __syncthreads();
+        // propose (Alg. 2 L13-L22), the tests of propose_phase in its order
+        unsigned long long my_live = 0, my_nnz = 0, my_prop = 0;
+#pragma unroll
+        for (int q = 0; q < RPT; q++) {
+            const int s = tid + q * T;
+            if (s >= nmine || !(S.act[s] & 1)) continue;
+            const uint8_t stt = S.st[s];
+            const int deg = stt & ST_DEG;
+            const uint32_t cv = (stt & ST_CHARGE) ? 1u : 0u;
+            int32_t pc[NN];
+#pragma unroll
+            for (int t = 0; t < NN; t++) pc[t] = t < deg ? key_col(S.pik[s * NN + t]) : -1;
+            uint64_t top[NN];
+#pragma unroll
+            for (int t = 0; t < NN; t++) top[t] = 0;
+            bool theta0 = false;
+            const int e0 = S.est[s], e1 = e0 + S.rlen[s];
+            for (int e = e0; e < e1; e++) {
+                const uint64_t key = S.ek[e];
+                if (!key) continue;                              // diagonal / zero
+                const uint32_t sj = S.esj[e];
+                if ((int)(sj & ST_DEG) == NN) continue;          // saturated (L15)
+                const int32_t j = key_col(key);
+                bool in_pi = false;
+#pragma unroll
+                for (int t = 0; t < NN; t++) in_pi |= (pc[t] == j);
+                if (in_pi) continue;                             // L19
+                theta0 = true;
+                if (charging && (((sj & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
+                topn_insert<NN>(top, key);
+            }
+            const int need = NN - deg;
+            const int32_t v = S.gid[s];
+            int np = 0;
+#pragma unroll
+            for (int t = 0; t < NN; t++) {
+                const uint64_t tk = (t < need) ? top[t] : 0ull;
+                S.prk[s * NN + t] = tk;
+                pa.prop_j[(int64_t)v * NN + t] = tk ? key_col(tk) : -1;
+                np += tk != 0;
+            }
+            S.act[s] = theta0 ? 1 : 3;
+            if (theta0) { my_live += 1; my_nnz += (unsigned long long)S.rlen[s]; }
+            my_prop |= (np > 0);
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            my_live += __shfl_xor_sync(0xffffffffu, my_live, o);
+            my_nnz += __shfl_xor_sync(0xffffffffu, my_nnz, o);
+            my_prop |= __shfl_xor_sync(0xffffffffu, my_prop, o);
+        }
+        if ((tid & 31) == 0) { S.red[0][tid >> 5] = my_live; S.red[1][tid >> 5] = my_nnz; S.red[2][tid >> 5] = my_prop; }
+        __syncthreads();
+        if (tid < 32) {
+            unsigned long long a0 = tid < T / 32 ? S.red[0][tid] : 0, a1 = tid < T / 32 ? S.red[1][tid] : 0,
+                               a2 = tid < T / 32 ? S.red[2][tid] : 0;
+#pragma unroll
+            for (int o = 16; o; o >>= 1) {
+                a0 += __shfl_xor_sync(0xffffffffu, a0, o);
+                a1 += __shfl_xor_sync(0xffffffffu, a1, o);
+                a2 |= __shfl_xor_sync(0xffffffffu, a2, o);
+            }
+            if (tid == 0) {
+                const int slot = blockIdx.x & 63;
+                if (f.live_part && a0) atomicAdd(f.live_part + (size_t)k * 128 + slot, a0);
+                if (f.live_part && a1) atomicAdd(f.live_part + (size_t)k * 128 + 64 + slot, a1);
+                if (a2) atomicOr(&f.flags[k], 1);
+            }
+        }
+        grid.sync();  // every proposal of round k is visible
+        // mutual (Alg. 2 L26-L28): keep w iff v is in prop(w); w proposed this round
+#pragma unroll
+        for (int q = 0; q < RPT; q++) {
+            const int s = tid + q * T;
+            if (s >= nmine || !(S.act[s] & 1)) continue;
+            const int32_t v = S.gid[s];
+            int32_t pw[NN][NN];
+#pragma unroll
+            for (int u = 0; u < NN; u++) {
+                const uint64_t tk = S.prk[s * NN + u];
+#pragma unroll
+                for (int x = 0; x < NN; x++) pw[u][x] = -1;
+                if (!tk) continue;
+                const int32_t* q2 = pa.prop_j + (int64_t)key_col(tk) * NN;
+#pragma unroll
+                for (int x = 0; x < NN; x++) pw[u][x] = __ldcg(q2 + x);
+            }
+            uint64_t t[NN];
+#pragma unroll
+            for (int u = 0; u < NN; u++) t[u] = S.pik[s * NN + u];
+            int nconf = 0;
+#pragma unroll
+            for (int u = 0; u < NN; u++) {
+                bool mutual = false;
+#pragma unroll
+                for (int x = 0; x < NN; x++) mutual |= (pw[u][x] == v);
+                if (mutual) { topn_insert<NN>(t, S.prk[s * NN + u]); nconf++; }
+            }
+            int deg = S.st[s] & ST_DEG;
+            if (nconf) {
+#pragma unroll
+                for (int u = 0; u < NN; u++) S.pik[s * NN + u] = t[u];
+                deg += nconf;
+            }
+            if (!last) {
+                const bool keep = !(S.act[s] & 2) && deg < NN;
+                uint32_t ch = 0;
+                if (keep && ((k + 1) % f.m) != f.k_m) ch = charge_bit((uint32_t)v, (uint32_t)(k + 1), f.ma.seed, f.ma.thr);
+                const uint8_t ns = (uint8_t)(deg | (ch ? ST_CHARGE : 0));
+                S.st[s] = ns;
+                f.ma.state[v] = ns;
+                S.act[s] = keep ? 1 : 0;
+            } else if (nconf) {
+                S.st[s] = (uint8_t)deg;
+            }
+        }
+        if (!last) grid.sync();  // round k+1's states visible; round k's proposals consumed
+    }
+    // write back the rows' factor slots and state
+#pragma unroll
+    for (int q = 0; q < RPT; q++) {
+        const int s = tid + q * T;
+        if (s >= nmine) continue;
+        const int32_t v = S.gid[s];
+#pragma unroll
+        for (int u = 0; u < NN; u++) {
+            const uint64_t key = S.pik[s * NN + u];
+            const int64_t o = (int64_t)v * NN + u;
+            f.ma.pi[o] = key ? key_col(key) : -1;
+            f.ma.pi_w[o] = key ? key_abs(key) : 0.0f;
+            if (f.ma.pi_val) f.ma.pi_val[o] = key ? key_val(key) : 0.0f;
+        }
+        f.ma.state[v] = S.st[s];
+    }
+    // every CTA's counters of the last round were added before the last barrier
+    if (blockIdx.x == 0 && (f.rounds || f.live))
+        finalize_body(f.flags, f.M, f.m, f.k_m, f.rounds, f.live_part, f.live);
+    return true;
+}
+
+static bool cached_rounds_enabled() {
+    static int on = -1;
+    if (on < 0) on = getenv("LF_NO_CACHED_ROUNDS") ? 0 : 1;
+    return on == 1;
+}
+
 template <int NN, int G>
 __global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {
     pdl_trigger();  // k_finalize (one CTA) may launch and wait meanwhile
     cg::grid_group grid = cg::this_grid();
+    if (f.cached && rounds_cached<NN>(f, grid)) return;
     for (int k = 1; k < f.M; k++) {
         ProposeArgs pa = f.pa;
         pa.wl = f.wl[k & 1];
@@ -1199,6 +1497,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         f.G = G;
         f.rounds = rounds_dev;
         f.live = live;
+        f.cached = cached_rounds_enabled() ? 1 : 0;
+        f.bail = &w.counts[3];
         LF_PROF("rounds_fused", -1, s);
         void* args[] = {&f};
         const void* kfn;
@@ -1209,10 +1509,19 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             case 16: kfn = (const void*)k_rounds_fused<NN, 16>; break;
             default: kfn = (const void*)k_rounds_fused<NN, 32>; break;
         }
+        const size_t smem = f.cached ? cache_smem_bytes<NN>() : 0;
+        if (f.cached) {
+            static bool attr[5] = {false, false, false, false, false};
+            const int gi = G == 2 ? 0 : G == 4 ? 1 : G == 8 ? 2 : G == 16 ? 3 : 4;
+            if (!attr[gi]) {
+                LF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                attr[gi] = true;
+            }
+        }
         int grid = LF_FUSED_GRID > 0 ? LF_FUSED_GRID : sm_count() * LF_FUSED_GRID_SM;  // fewer CTAs: cheaper barriers
-        const int cap = persistent_grid(kfn, LF_FUSED_T);
+        const int cap = persistent_grid(kfn, LF_FUSED_T, smem);
         if (grid > cap) grid = cap;
-        LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, 0, s));
+        LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, smem, s));
     }
     if (o->until_maximal) {
         if (rounds_dev) {
