@@ -894,6 +894,14 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
     CacheSmem<NN>& S = *reinterpret_cast<CacheSmem<NN>*>(fz_smem);
     const int tid = threadIdx.x;
     const ProposeArgs& pa = f.pa;
+#ifdef LF_CACHE_TIMING
+    unsigned long long tm[24];
+    int ntm = 0;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tm[ntm++]));
+#define CC_MARK() do { __syncthreads(); asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tm[ntm < 23 ? ntm++ : 23])); } while (0)
+#else
+#define CC_MARK() do { } while (0)
+#endif
     const int L = *(volatile const int32_t*)&f.counts[1];   // round-1 worklist (mutual(0))
     const int C = gridDim.x;
     const int RPC = (L + C - 1) / C;
@@ -934,8 +942,10 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
         if (len > kCacheMaxRow || off + len > Cap::E) S.ovf = 1;
     }
     __syncthreads();
+    CC_MARK();
     if (tid == 0 && S.ovf) atomicOr(f.bail, 1);
     grid.sync();
+    CC_MARK();
     if (*(volatile int32_t*)f.bail) return false;   // uniform: nothing global written yet
 #pragma unroll
     for (int q = 0; q < RPT; q++) {
@@ -967,7 +977,8 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
             S.ek[p] = edge ? make_key(x[q], j[q]) : 0ull;
         }
     }
-    __syncthreads();
+    __syncthreads();  // the entry keys
+    CC_MARK();
     for (int k = 1; k < f.M; k++) {
         const bool charging = (k % f.m) != f.k_m;
         const bool last = k == f.M - 1;
@@ -988,7 +999,8 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
                 if (p < P) S.esj[p] = sj[q];
             }
         }
-        __syncthreads();
+        __syncthreads();  // the targets' states
+        CC_MARK();
         // propose (Alg. 2 L13-L22), the tests of propose_phase in its order
         unsigned long long my_live = 0, my_nnz = 0, my_prop = 0;
 #pragma unroll
@@ -1058,7 +1070,9 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
                 if (a2) atomicOr(&f.flags[k], 1);
             }
         }
+        CC_MARK();
         grid.sync();  // every proposal of round k is visible
+        CC_MARK();
         // mutual (Alg. 2 L26-L28): keep w iff v is in prop(w); w proposed this round
 #pragma unroll
         for (int q = 0; q < RPT; q++) {
@@ -1105,7 +1119,9 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
                 S.st[s] = (uint8_t)deg;
             }
         }
+        CC_MARK();
         if (!last) grid.sync();  // round k+1's states visible; round k's proposals consumed
+        CC_MARK();
     }
     // write back the rows' factor slots and state
 #pragma unroll
@@ -1126,14 +1142,18 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
     // every CTA's counters of the last round were added before the last barrier
     if (blockIdx.x == 0 && (f.rounds || f.live))
         finalize_body(f.flags, f.M, f.m, f.k_m, f.rounds, f.live_part, f.live);
+#ifdef LF_CACHE_TIMING
+    CC_MARK();
+    if (tid == 0 && (blockIdx.x == 0 || blockIdx.x == 100)) {
+        printf("cached blk %d L=%d nmine=%d P=%d:", blockIdx.x, L, nmine, P);
+        for (int i = 1; i < ntm; i++) printf(" %llu", tm[i] - tm[i - 1]);
+        printf("\n");
+    }
+#endif
     return true;
 }
 
-static bool cached_rounds_enabled() {
-    static int on = -1;
-    if (on < 0) on = getenv("LF_NO_CACHED_ROUNDS") ? 0 : 1;
-    return on == 1;
-}
+static bool cached_rounds_enabled() { return getenv("LF_NO_CACHED_ROUNDS") == nullptr; }
 
 template <int NN, int G>
 __global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {

@@ -211,6 +211,29 @@ def test_c2_full_size(torch_cuda, lfm, oracle_mod, n):
         check_forest(torch_cuda, lfm, oracle_mod, A, fac, ref)
 
 
+@pytest.mark.parametrize("cfg", ["C2", "C3"])
+def test_repeated_runs_cached_and_uncached_rounds(torch_cuda, lfm, oracle_mod, monkeypatch, cfg):
+    """Rounds 1..M-1 in both modes (shared-memory cached / global worklists),
+    five back-to-back runs each on one workspace without a host sync in between: every run
+    equals the oracle-checked first one (catches races that a single run can miss)."""
+    torch = torch_cuda
+    A = _cached(cfg)
+    ref, _ = check_factor(torch, lfm, oracle_mod, A, 2)
+    rp, col, val = dev(torch, A)
+    ws = lfm.Workspace()
+    for mode in ("cached", "uncached"):
+        if mode == "uncached":
+            monkeypatch.setenv("LF_NO_CACHED_ROUNDS", "1")
+        else:
+            monkeypatch.delenv("LF_NO_CACHED_ROUNDS", raising=False)
+        outs = [lfm.factor(rp, col, val, 2, live=True, ws=ws) for _ in range(5)]
+        torch.cuda.synchronize()
+        for i, out in enumerate(outs):
+            for k in ("pi", "pi_w", "pi_val", "live", "rounds"):
+                assert torch.equal(out[k], ref[k]), f"{mode} run {i}: {k} differs"
+    monkeypatch.delenv("LF_NO_CACHED_ROUNDS", raising=False)
+
+
 @pytest.mark.parametrize("cfg", ["C1", "C3", "C4"])
 def test_config_full_size(torch_cuda, lfm, oracle_mod, cfg):
     A = _cached(cfg)
