@@ -2118,129 +2118,122 @@ __device__ __forceinline__ void win_append(int32_t& R, uint64_t& K, int32_t& D, 
     R += Rw;
 }
 
-constexpr int kRedSmallF = 4 * 1024;   // lists up to this size: one CTA, shared memory
-
-// per direction d (0/1): the pointer, length, DK and minimum key of every node's window
-struct RedSmemF {
-    int2 q[kRedSmallF];
-    int r[2][kRedSmallF];
-    int d[2][kRedSmallF];
-    uint64_t k[2][kRedSmallF];
-};
-
 // list position of the vertex a record points at (markers pass through)
 __device__ __forceinline__ int2 to_pos(const ForestArgs& a, int2 q) {
     return make_int2(q.x >= 0 ? __ldcg(a.bidx1 + q.x) : q.x, q.y >= 0 ? __ldcg(a.bidx1 + q.y) : q.y);
 }
 
-// The whole reduced scan in one CTA's shared memory (lists up to kRedSmallF nodes).  Each
-// step reads, per direction, the target's pointers and then only the continuing window's
-// length / DK / key (one direction's arrays: fewer random shared-memory words).
-template <int T>
-__device__ void red_full_small(const ForestArgs& a, int cnt, int* ctl, RedSmemF& S) {
-    constexpr int NPT = (kRedSmallF + T - 1) / T;
+// The reduced scan of lists up to kRedCl * kRedClNodes nodes on ONE thread-block cluster:
+// node i lives in shared memory of CTA i / NPC (slot i % NPC) and every step reads the
+// target's window through DSMEM.  One CTA's shared memory would hold C2's 3.4 k nodes,
+// but then every step's random (bank-conflicted) window reads are served by a single SM;
+// sixteen SMs serve them sixteen times faster.  Windows are ping-ponged between two
+// buffers (a step reads buffer b everywhere and writes buffer b^1 of its own nodes), so
+// one cluster barrier per step suffices; finished path nodes are copied forward.
+constexpr int kRedCl = 16;           // CTAs of the cluster (non-portable size)
+constexpr int kRedClNodes = 2048;    // nodes per CTA
+struct RedSmemC {
+    int2 q[2][kRedClNodes];
+    int r[2][2][kRedClNodes];        // [buffer][direction][slot]
+    int d[2][2][kRedClNodes];
+    uint64_t k[2][2][kRedClNodes];
+    int nd[2];                       // this CTA's "some node not done" per step parity
+};
+
+__device__ void red_full_cluster(const ForestArgs& a, int cnt, int* ctl, RedSmemC& S) {
+    constexpr int NPT = kRedClNodes / RT;
+    cg::cluster_group cl = cg::this_cluster();
+    const int rank = (int)cl.block_rank();
     const int tid = threadIdx.x;
-#ifdef LF_PHASE_TIMING
-    const unsigned long long t_start = gtime();
-#endif
-    bool fin[NPT];
-    int notdone = 0;
+    const int NPC = (cnt + kRedCl - 1) / kRedCl;
+    const int base = rank * NPC;
+    const int nmine = max(0, min(cnt - base, NPC));
+    __shared__ RedSmemC* rem[kRedCl];
+    if (tid < kRedCl) rem[tid] = cl.map_shared_rank(&S, tid);
     {
         int2 q[NPT], r[NPT], d[NPT];
         ulonglong2 kk[NPT];
 #pragma unroll
         for (int k = 0; k < NPT; k++) {
-            const int idx = tid + k * T;
-            if (idx >= cnt) continue;
-            q[k] = __ldcg(a.cq + idx);
-            r[k] = __ldcg(a.cq_r + idx);
-            d[k] = __ldcg(a.cq_dk + idx);
-            kk[k] = __ldcg(a.cq_k + idx);
+            const int t = tid + k * RT;
+            if (t >= nmine) continue;
+            q[k] = __ldcg(a.cq + base + t);
+            r[k] = __ldcg(a.cq_r + base + t);
+            d[k] = __ldcg(a.cq_dk + base + t);
+            kk[k] = __ldcg(a.cq_k + base + t);
         }
 #pragma unroll
         for (int k = 0; k < NPT; k++) {
-            const int idx = tid + k * T;
-            if (idx >= cnt) continue;
+            const int t = tid + k * RT;
+            if (t >= nmine) continue;
             q[k] = to_pos(a, q[k]);
-        }
-#pragma unroll
-        for (int k = 0; k < NPT; k++) {
-            const int idx = tid + k * T;
-            fin[k] = true;
-            if (idx >= cnt) continue;
-            S.q[idx] = q[k];
-            S.r[0][idx] = r[k].x; S.r[1][idx] = r[k].y;
-            S.d[0][idx] = d[k].x; S.d[1][idx] = d[k].y;
-            S.k[0][idx] = kk[k].x; S.k[1][idx] = kk[k].y;
-            fin[k] = q[k].x < 0 && q[k].y < 0;
-            notdone |= !fin[k];
+            S.q[0][t] = q[k];
+            S.r[0][0][t] = r[k].x; S.r[0][1][t] = r[k].y;
+            S.d[0][0][t] = d[k].x; S.d[0][1][t] = d[k].y;
+            S.k[0][0][t] = kk[k].x; S.k[0][1][t] = kk[k].y;
         }
     }
-    const int any0 = __syncthreads_or(notdone);
-    RS_MARK(0);
-    if (any0) {
-        for (int step = 0; step < a.max_steps; step++) {
-            int2 nq[NPT];
-            int nr[NPT][2], nd[NPT][2];
-            uint64_t nk[NPT][2];
-            notdone = 0;
+    cl.sync();
+    int b = 0;
+    for (int step = 0; step < a.max_steps; step++) {
+        int notdone = 0;
 #pragma unroll
-            for (int k = 0; k < NPT; k++) {
-                if (fin[k]) continue;
-                const int me = tid + k * T;
-                const int2 q = S.q[me];
-                nq[k] = q;
+        for (int k = 0; k < NPT; k++) {
+            const int t = tid + k * RT;
+            if (t >= nmine) continue;
+            const int me = base + t;
+            const int2 q = S.q[b][t];
+            int2 nq = q;
+            int32_t R[2] = {S.r[b][0][t], S.r[b][1][t]}, D[2] = {S.d[b][0][t], S.d[b][1][t]};
+            uint64_t K[2] = {S.k[b][0][t], S.k[b][1][t]};
+            if (!(q.x < 0 && q.y < 0)) {  // finished paths are only copied forward
 #pragma unroll
                 for (int i = 0; i < 2; i++) {
                     const int w = i ? q.y : q.x;
-                    int32_t R = S.r[i][me], D = S.d[i][me];
-                    uint64_t K = S.k[i][me];
-                    if (w >= 0) {
-                        const int2 qw = S.q[w];
-                        int j = -1;
-                        if (qw.x != me) j = 0;
-                        else if (qw.y != me) j = 1;
-                        if (j >= 0) {
-                            win_append(R, K, D, S.r[j][w], S.k[j][w], S.d[j][w]);
-                            if (i) nq[k].y = j ? qw.y : qw.x; else nq[k].x = j ? qw.y : qw.x;
-                        } else {  // stall (reading c13): see node_scan_full
-                            const uint64_t kw0 = S.k[0][w], kw1 = S.k[1][w];
-                            if (kw0 < K) { K = kw0; D = 2 * R + S.d[0][w]; }
-                            if (kw1 < K) { K = kw1; D = 2 * R + S.d[1][w]; }
-                        }
+                    if (w < 0) continue;
+                    const int rw = w / NPC, sw = w - rw * NPC;
+                    const RedSmemC* P = rem[rw];
+                    const int2 qw = P->q[b][sw];
+                    int j = -1;
+                    if (qw.x != me) j = 0;
+                    else if (qw.y != me) j = 1;
+                    if (j >= 0) {
+                        win_append(R[i], K[i], D[i], P->r[b][j][sw], P->k[b][j][sw], P->d[b][j][sw]);
+                        if (i) nq.y = j ? qw.y : qw.x; else nq.x = j ? qw.y : qw.x;
+                    } else {  // stall (reading c13): see node_scan_full
+                        const uint64_t kw0 = P->k[b][0][sw], kw1 = P->k[b][1][sw];
+                        if (kw0 < K[i]) { K[i] = kw0; D[i] = 2 * R[i] + P->d[b][0][sw]; }
+                        if (kw1 < K[i]) { K[i] = kw1; D[i] = 2 * R[i] + P->d[b][1][sw]; }
                     }
-                    nr[k][i] = R; nd[k][i] = D; nk[k][i] = K;
                 }
-                const bool path_done = nq[k].x < 0 && nq[k].y < 0;
-                const bool cyc_done = nq[k].x >= 0 && nq[k].y >= 0 && nk[k][0] == nk[k][1];
+                const bool path_done = nq.x < 0 && nq.y < 0;
+                const bool cyc_done = nq.x >= 0 && nq.y >= 0 && K[0] == K[1];
                 notdone |= !(path_done || cyc_done);
             }
-            __syncthreads();
+            S.q[b ^ 1][t] = nq;
 #pragma unroll
-            for (int k = 0; k < NPT; k++) {
-                if (fin[k]) continue;
-                const int me = tid + k * T;
-                S.q[me] = nq[k];
-#pragma unroll
-                for (int i = 0; i < 2; i++) { S.r[i][me] = nr[k][i]; S.d[i][me] = nd[k][i]; S.k[i][me] = nk[k][i]; }
-                fin[k] = nq[k].x < 0 && nq[k].y < 0;
-            }
-            const int any = __syncthreads_or(notdone);
-            if (tid == 0) ctl[step] = 1;
-            if (!any) break;
+            for (int i = 0; i < 2; i++) { S.r[b ^ 1][i][t] = R[i]; S.d[b ^ 1][i][t] = D[i]; S.k[b ^ 1][i][t] = K[i]; }
         }
+        const int any_local = __syncthreads_or(notdone);
+        if (tid == 0) S.nd[step & 1] = any_local;
+        cl.sync();  // buffer b^1 and the flags complete everywhere; nobody reads b any more
+        b ^= 1;
+        int f = tid < kRedCl ? rem[tid]->nd[step & 1] : 0;
+        const int any = __syncthreads_or(f);
+        if (rank == 0 && tid == 0) ctl[step] = 1;
+        if (!any) break;
     }
-    RS_MARK(1);
 #pragma unroll
     for (int k = 0; k < NPT; k++) {
-        const int idx = tid + k * T;
-        if (idx >= cnt) continue;
-        a.end2[idx] = S.q[idx];   // markers (paths); cycles keep list positions >= 0
-        a.dist2[idx] = make_int2(S.r[0][idx], S.r[1][idx]);
-        a.kraw[idx] = make_ulonglong2(S.k[0][idx], S.k[1][idx]);
-        a.dk2[idx] = make_int2(S.d[0][idx], S.d[1][idx]);
+        const int t = tid + k * RT;
+        if (t >= nmine) continue;
+        const int idx = base + t;
+        a.end2[idx] = S.q[b][t];   // markers (paths); cycles keep list positions >= 0
+        a.dist2[idx] = make_int2(S.r[b][0][t], S.r[b][1][t]);
+        a.kraw[idx] = make_ulonglong2(S.k[b][0][t], S.k[b][1][t]);
+        a.dk2[idx] = make_int2(S.d[b][0][t], S.d[b][1][t]);
     }
-    RS_MARK(2);
+    cl.sync();  // the last step's flag reads are done before any CTA leaves
 }
 
 constexpr int32_t kLocDone = INT_MIN;
@@ -2408,11 +2401,12 @@ __device__ __forceinline__ void red_grid_sync(int* ctr, int& gen) {
 __global__ void __launch_bounds__(RT) k_red_full(ForestArgs a) {
     __shared__ int sh[32];
     extern __shared__ __align__(16) unsigned char red_smem[];
+    pdl_wait();  // the tile pass's records
     const int cnt = *(volatile int*)&a.ctl[kCtlCnt1];
     int* ctl = a.ctl + kCtlRed1;
-    if (cnt <= kRedSmallF) {
+    if (cnt <= kRedCl * kRedClNodes) {
         pdl_trigger();  // the expand kernel's tile-only prologue overlaps this scan
-        if (blockIdx.x == 0) red_full_small<RT>(a, cnt, ctl, *reinterpret_cast<RedSmemF*>(red_smem));
+        if (blockIdx.x < kRedCl) red_full_cluster(a, cnt, ctl, *reinterpret_cast<RedSmemC*>(red_smem));
         return;
     }
     int* bar = a.ctl + kCtlGridBar;
@@ -2720,11 +2714,44 @@ static int forest_prepare() {
     LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_full1, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)kFull1Smem));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_red_full, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)sizeof(RedSmemF)));
+                                 (int)sizeof(RedSmemC)));
     LF_CUDA(cudaFuncSetAttribute((const void*)k_lf_full2, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)sizeof(TileSmemE)));
     attr_done = true;
     return LF_OK;
+}
+
+// k_red_full: clusters of kRedCl CTAs (the small path runs on the first cluster), as
+// many clusters as can be resident at once (the grid path's barrier needs them all)
+static cudaError_t launch_red_full(const ForestArgs& a, cudaStream_t s) {
+    static int nclusters = 0;
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3(RT);
+    cfg.dynamicSmemBytes = sizeof(RedSmemC);
+    cfg.stream = s;
+    cudaLaunchAttribute at[2];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = kRedCl;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    if (nclusters == 0) {
+        cudaError_t e = cudaFuncSetAttribute((const void*)k_red_full, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        if (e != cudaSuccess) return e;
+        cfg.gridDim = dim3(kRedCl);
+        cfg.numAttrs = 1;
+        int n = 0;
+        e = cudaOccupancyMaxActiveClusters(&n, (const void*)k_red_full, &cfg);
+        if (e != cudaSuccess) return e;
+        if (n < 1) return cudaErrorLaunchOutOfResources;
+        nclusters = n < sm_count() / kRedCl ? n : sm_count() / kRedCl;
+        if (nclusters < 1) nclusters = 1;
+    }
+    cfg.gridDim = dim3(kRedCl * nclusters);
+    cfg.numAttrs = pdl_enabled() ? 2 : 1;
+    return cudaLaunchKernelEx(&cfg, k_red_full, a);
 }
 
 int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
@@ -2779,9 +2806,9 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("red_scan", -1, s);
-#ifndef LF_NO_GRID_RED  // diagnostics only: measures the launch cost (wrong for lists > kRedSmallF)
+#ifndef LF_NO_GRID_RED  // diagnostics only: measures the launch cost (wrong results)
         // one CTA per SM (its shared memory admits no second one): see red_grid_sync
-        LF_CUDA(launch_pdl(k_red_full, sm_count(), RT, sizeof(RedSmemF), s, a));
+        LF_CUDA(launch_red_full(a, s));
 #endif
     }
     {
