@@ -372,7 +372,7 @@ __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_grou
 __device__ __forceinline__ void cp_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
 #ifndef LF_SETILE
-#define LF_SETILE 4096
+#define LF_SETILE 2048   // 38 KB of stages: 5 CTAs per SM (4096: 3), more bytes in flight
 #endif
 #ifndef LF_SPT
 #define LF_SPT 256
@@ -1295,10 +1295,11 @@ static void launch_propose_tile(int G, const ProposeArgs& pa, int64_t N, cudaStr
 }
 
 // lanes per row of the staged round-0 kernel (thread per row for sparse rows)
+// lanes per row of the round-0 stream: an average tile (256 / G rows) fits a SETILE stage
 static int tile_lanes(double avg) {
-    if (avg <= 12) return 1;
-    if (avg <= 24) return 2;
-    if (avg <= 48) return 4;
+    if (avg <= 7) return 1;
+    if (avg <= 14) return 2;
+    if (avg <= 28) return 4;
     return 8;
 }
 

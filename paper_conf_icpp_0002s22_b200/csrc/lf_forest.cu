@@ -2254,12 +2254,19 @@ __global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
     LF_PHASE_INIT;
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
+    int2 orig[VPT];
+    int idx_[VPT];  // boundary-list slots, claimed now: the atomic's round trip overlaps the ranking
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        orig[k] = s.nb[threadIdx.x + k * LT];
+        const int32_t g = b0 + (int)threadIdx.x + k * LT;
+        const bool r0 = orig[k].x >= 0 && !is_local(orig[k].x, T);
+        const bool r1 = orig[k].y >= 0 && !is_local(orig[k].y, T);
+        idx_[k] = list_append(a.list1, &a.ctl[kCtlCnt1], g, g < a.hi && (r0 || r1));
+    }
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
     LF_PHASE(a.ctl, 6);
-    int2 orig[VPT];
-#pragma unroll
-    for (int k = 0; k < VPT; k++) orig[k] = s.nb[threadIdx.x + k * LT];
     VRes o[VPT];
     tile_rank_full(s, b0, ek, o, a.ctl + kCtlStat);
 #ifdef LF_PHASE_TIMING
@@ -2290,8 +2297,8 @@ __global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
                 a.loc2[g] = make_int2((int)tt, (int)rr);
             }
         }
-        const int idx = list_append(a.list1, &a.ctl[kCtlCnt1], g, boundary);
         if (boundary) {
+            const int idx = idx_[k];
             int2 q, rl, dk;
             ulonglong2 kk;
 #pragma unroll
