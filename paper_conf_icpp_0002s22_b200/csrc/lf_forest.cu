@@ -40,17 +40,20 @@ namespace cg = cooperative_groups;
 namespace lf {
 
 constexpr uint64_t KEY_INF = ~0ull;
+// 1024-vertex tiles, 512 threads: two tile-pass CTAs per SM (92 KB of shared memory each)
+// overlap one tile's barriers and loads with the other's work (measured on C2: 1024/512/2
+// beats 2048/1024/1 by 6 us per step even though the boundary list grows by half)
 #ifndef LF_LB
-#define LF_LB 2048
+#define LF_LB 1024
 #endif
 #ifndef LF_LT
-#define LF_LT 1024
+#define LF_LT 512
 #endif
 #ifndef LF_LMINB
-#define LF_LMINB 2
+#define LF_LMINB 4    // expand / local2 CTAs per SM
 #endif
 #ifndef LF_F1MINB
-#define LF_F1MINB 1   // resident tile-pass CTAs per SM (k_lf_full1)
+#define LF_F1MINB 2   // resident tile-pass CTAs per SM (k_lf_full1)
 #endif
 constexpr int LB = LF_LB;         // vertices per block-local tile
 constexpr int LT = LF_LT;         // threads per tile CTA
