@@ -739,6 +739,7 @@ __global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
                     for (int t = 0; t < NN; t++) pw[b][s][t] = -1;
                 }
             }
+        bool keepb[MB];
 #pragma unroll
         for (int b = 0; b < MB; b++) {
             const int64_t r = c0 + threadIdx.x + (int64_t)b * blockDim.x;
@@ -773,12 +774,21 @@ __global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
                 }
                 a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0));
             }
-            if (a.wl_next) {
-                const unsigned m = __ballot_sync(0xffffffffu, keep);
-                int32_t basepos = 0;
-                if (lane == 0 && m) basepos = atomicAdd(a.wl_next_count, __popc(m));
-                basepos = __shfl_sync(0xffffffffu, basepos, 0);
-                if (keep) a.wl_next[basepos + __popc(m & ((1u << lane) - 1u))] = v;
+            keepb[b] = keep;
+        }
+        if (a.wl_next) {  // one worklist atomic per warp for all MB row batches
+            unsigned m[MB];
+            int tot = 0;
+#pragma unroll
+            for (int b = 0; b < MB; b++) { m[b] = __ballot_sync(0xffffffffu, keepb[b]); tot += __popc(m[b]); }
+            int32_t basepos = 0;
+            if (lane == 0 && tot) basepos = atomicAdd(a.wl_next_count, tot);
+            basepos = __shfl_sync(0xffffffffu, basepos, 0);
+#pragma unroll
+            for (int b = 0; b < MB; b++) {
+                const int64_t r = c0 + threadIdx.x + (int64_t)b * blockDim.x;
+                if (keepb[b]) a.wl_next[basepos + __popc(m[b] & ((1u << lane) - 1u))] = (int32_t)(a.row_base + r);
+                basepos += __popc(m[b]);
             }
         }
     }

@@ -50,7 +50,7 @@ constexpr uint64_t KEY_INF = ~0ull;
 #define LF_LT 512
 #endif
 #ifndef LF_LMINB
-#define LF_LMINB 4    // expand / local2 CTAs per SM
+#define LF_LMINB 3    // expand / local2 CTAs per SM (4: register spills)
 #endif
 #ifndef LF_F1MINB
 #define LF_F1MINB 2   // resident tile-pass CTAs per SM (k_lf_full1)
