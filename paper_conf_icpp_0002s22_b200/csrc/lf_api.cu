@@ -398,6 +398,13 @@ __global__ void k_probe_plain(int* p) {
 }
 }  // namespace lf
 
+// Diagnostics only (not part of include/lf.h): per-kernel timeline of LF_TIMELINE builds.
+// out[0..15] factor kernels, out[16..31] forest kernels; reset != 0 clears.  -1 otherwise.
+extern "C" int lf_debug_timeline(unsigned long long* out, int reset) {
+    if (reset) return lf::timeline_factor(nullptr, 1) | lf::timeline_forest(nullptr, 1);
+    return lf::timeline_factor(out, 0) | lf::timeline_forest(out + 16, 0);
+}
+
 extern "C" int lf_debug_launch_probe(int mode, int block, int sync_steps, void* stream) {
     using namespace lf;
     cudaStream_t s = (cudaStream_t)stream;

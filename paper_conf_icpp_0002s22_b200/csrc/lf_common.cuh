@@ -115,4 +115,26 @@ constexpr int32_t PROP_RETIRED = -2;
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
+// Diagnostic timeline (builds with -DLF_TIMELINE only): earliest CTA start / latest CTA
+// exit of each kernel of the step, on the global timer; read by lf_debug_timeline.
+#ifdef LF_TIMELINE
+__device__ __forceinline__ unsigned long long tl_now() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+struct TlScope {
+    unsigned long long* slot;
+    __device__ explicit TlScope(unsigned long long* s) : slot(s) {
+        if (threadIdx.x == 0) atomicMin(slot, tl_now());
+    }
+    __device__ ~TlScope() {
+        if (threadIdx.x == 0) atomicMax(slot + 1, tl_now());
+    }
+};
+#define LF_TL(arr, id) ::lf::TlScope lf_tl_scope_(&(arr)[2 * (id)])
+#else
+#define LF_TL(arr, id) do { } while (0)
+#endif
+
 }  // namespace lf

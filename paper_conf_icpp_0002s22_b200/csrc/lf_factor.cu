@@ -28,6 +28,10 @@ namespace cg = cooperative_groups;
 
 namespace lf {
 
+#ifdef LF_TIMELINE
+__device__ unsigned long long g_tl_factor[16];
+#endif
+
 struct ProposeArgs {
     int64_t N;                           // CSR rows (this partition's own rows)
     int64_t row_base;                    // vertex id of CSR row r is row_base + r
@@ -173,6 +177,7 @@ __device__ __forceinline__ void propose_phase(const ProposeArgs& a) {
 
 template <int NN, int G>
 __global__ void __launch_bounds__(256) k_propose(ProposeArgs a) {
+    LF_TL(g_tl_factor, 1);
     pdl_wait();
     pdl_trigger();
     propose_phase<NN, G>(a);
@@ -417,6 +422,7 @@ __device__ __forceinline__ void issue_entries(const ProposeArgs& a, int64_t e0, 
 
 template <int NN, int G, bool CHARGED>
 __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
+    LF_TL(g_tl_factor, 0);
     constexpr int R = SPT / G;
     extern __shared__ __align__(16) unsigned char sraw[];
     StreamSmem& S = *reinterpret_cast<StreamSmem*>(sraw);
@@ -709,6 +715,7 @@ constexpr int kMutual0Rows = 4;
 
 template <int NN, int MB>
 __global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
+    LF_TL(g_tl_factor, 2);
     pdl_wait();
     if (a.wl_zero && blockIdx.x == 0 && threadIdx.x == 0) *a.wl_zero = 0;
     const int lane = threadIdx.x & 31;
@@ -1167,6 +1174,7 @@ static bool cached_rounds_enabled() { return getenv("LF_NO_CACHED_ROUNDS") == nu
 
 template <int NN, int G>
 __global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {
+    LF_TL(g_tl_factor, 3);
     pdl_trigger();  // k_finalize (one CTA) may launch and wait meanwhile
     cg::grid_group grid = cg::this_grid();
     if (f.cached && rounds_cached<NN>(f, grid)) return;
@@ -1583,4 +1591,16 @@ int factor_dispatch(const lf_csr_t* A, int n, const lf_factor_opts_t* o, int32_t
     }
 }
 
+#ifdef LF_TIMELINE
+int timeline_factor(unsigned long long* out, int reset) {
+    if (reset) {
+        unsigned long long h[16];
+        for (int i = 0; i < 16; i += 2) { h[i] = ~0ull; h[i + 1] = 0; }
+        return cudaMemcpyToSymbol(g_tl_factor, h, sizeof(h)) == cudaSuccess ? 0 : -1;
+    }
+    return cudaMemcpyFromSymbol(out, g_tl_factor, sizeof(g_tl_factor)) == cudaSuccess ? 0 : -1;
+}
+#else
+int timeline_factor(unsigned long long*, int) { return -1; }
+#endif
 }  // namespace lf

@@ -39,6 +39,10 @@ namespace cg = cooperative_groups;
 
 namespace lf {
 
+#ifdef LF_TIMELINE
+__device__ unsigned long long g_tl_forest[16];
+#endif
+
 constexpr uint64_t KEY_INF = ~0ull;
 // 1024-vertex tiles, 512 threads: two tile-pass CTAs per SM (92 KB of shared memory each)
 // overlap one tile's barriers and loads with the other's work (measured on C2: 1024/512/2
@@ -1535,6 +1539,7 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
                                                   const float* __restrict__ diag, int32_t* __restrict__ perm,
                                                   int32_t* __restrict__ iperm, float* __restrict__ ta,
                                                   float* __restrict__ tb, float* __restrict__ tc) {
+    LF_TL(g_tl_forest, 4);
     pdl_wait();
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < N; v0 += stride * kPermBatch) {
@@ -1653,6 +1658,69 @@ __device__ __forceinline__ int group_or(int nt, int pred) {
     asm volatile("{\n\t.reg .pred p, q;\n\tsetp.ne.s32 p, %1, 0;\n\tbar.red.or.pred q, 1, %2, p;\n\tselp.s32 %0, 1, 0, q;\n\t}"
                  : "=r"(r) : "r"(pred), "r"(nt) : "memory");
     return r;
+}
+
+// the same scan for C <= 32 nodes by one warp, node i in lane i: the targets' windows
+// come by shuffles, so a step needs no shared memory and no barrier (C2's contracted
+// tiles have ~16 nodes)
+__device__ __forceinline__ void node_scan_warp(TileSmemF& s, int C, int* stats) {
+    const int i = threadIdx.x & 31;
+    const bool on = i < C;
+    int2 p = make_int2(-1, -1), r = make_int2(0, 0), dk = make_int2(0, 0);
+    uint64_t k0 = KEY_INF, k1 = KEY_INF;
+    if (on) {
+        const short2 ps = s.P[i], rs = s.R[i], ds = s.DK[i];
+        p = make_int2(ps.x, ps.y);
+        r = make_int2(rs.x, rs.y);
+        dk = make_int2(ds.x, ds.y);
+        k0 = s.K0[i];
+        k1 = s.K1[i];
+    }
+    for (int step = 0; step < 16; step++) {
+        int2 q = p, nr = r, nd = dk;
+        uint64_t n0 = k0, n1 = k1;
+#pragma unroll
+        for (int dd = 0; dd < 2; dd++) {
+            const int w = dd ? p.y : p.x;
+            const int src = (on && w >= 0) ? w : i;
+            const int pwx = __shfl_sync(0xffffffffu, p.x, src), pwy = __shfl_sync(0xffffffffu, p.y, src);
+            const int rwx = __shfl_sync(0xffffffffu, r.x, src), rwy = __shfl_sync(0xffffffffu, r.y, src);
+            const int dwx = __shfl_sync(0xffffffffu, dk.x, src), dwy = __shfl_sync(0xffffffffu, dk.y, src);
+            const uint64_t kw0 = __shfl_sync(0xffffffffu, k0, src), kw1 = __shfl_sync(0xffffffffu, k1, src);
+            if (!on || w < 0) continue;
+            const int Rd = dd ? r.y : r.x;
+            uint64_t kc = dd ? k1 : k0;
+            int dc = dd ? dk.y : dk.x;
+            int j = -1;
+            if (pwx != i) j = 0;
+            else if (pwy != i) j = 1;
+            if (j >= 0) {
+                const uint64_t kw = j ? kw1 : kw0;
+                if (kw < kc) { kc = kw; dc = 2 * Rd + (j ? dwy : dwx); }
+                const int tgt = j ? pwy : pwx;
+                const int rr = Rd + (j ? rwy : rwx);
+                if (dd) { q.y = tgt; nr.y = rr; } else { q.x = tgt; nr.x = rr; }
+            } else {  // stall (reading c13), as in node_scan_full
+                if (kw0 < kc) { kc = kw0; dc = 2 * Rd + dwx; }
+                if (kw1 < kc) { kc = kw1; dc = 2 * Rd + dwy; }
+            }
+            if (dd) { n1 = kc; nd.y = dc; } else { n0 = kc; nd.x = dc; }
+        }
+        p = q; r = nr; dk = nd; k0 = n0; k1 = n1;
+        const bool path_done = q.x < 0 && q.y < 0;
+        const bool cyc_done = q.x >= 0 && q.y >= 0 && n0 == n1;
+        if (!__any_sync(0xffffffffu, on && !(path_done || cyc_done))) {
+            if (i == 0 && stats) atomicMax(&stats[4], step + 1);
+            break;
+        }
+    }
+    if (on) {
+        s.P[i] = make_short2((short)p.x, (short)p.y);
+        s.R[i] = make_short2((short)r.x, (short)r.y);
+        s.DK[i] = make_short2((short)dk.x, (short)dk.y);
+        s.K0[i] = k0;
+        s.K1[i] = k1;
+    }
 }
 
 // bidirectional scan over the splitter nodes with full windows, by the first nt threads
@@ -1917,8 +1985,11 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
     }
     __syncthreads();
     LF_PHASE(ctlp, 2);
-    // 3. node scan: one node per thread of the smallest group that holds them all
-    if (C <= 128 && LT > 128) {
+    // 3. node scan: one warp (shuffles) or one node per thread of the smallest group
+    if (C <= 32) {
+        if (tid < 32) node_scan_warp(s, C, stats);
+        __syncthreads();
+    } else if (C <= 128 && LT > 128) {
         if (tid < 128) node_scan_full<1>(s, C, 128, stats);
         __syncthreads();
     } else if (C <= 512 && LT > 512) {
@@ -2251,6 +2322,8 @@ struct TileSmemE {
 // Tile pass: full-window scan; local cycles finished here; per-vertex local results and
 // the reduced records of boundary vertices.
 __global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
+    LF_TL(g_tl_forest, 0);
+    pdl_wait();  // k_ctl_zero, and through it the factor
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemF& s = *reinterpret_cast<TileSmemF*>(smem_raw);
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
@@ -2409,6 +2482,7 @@ __device__ __forceinline__ void red_grid_sync(int* ctr, int& gen) {
 }
 
 __global__ void __launch_bounds__(RT) k_red_full(ForestArgs a) {
+    LF_TL(g_tl_forest, 1);
     __shared__ int sh[32];
     extern __shared__ __align__(16) unsigned char red_smem[];
     pdl_wait();  // the tile pass's records
@@ -2472,6 +2546,7 @@ struct ExpState {       // a vertex waiting for reduced results
 };
 
 __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
+    LF_TL(g_tl_forest, 2);
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemE& s = *reinterpret_cast<TileSmemE*>(smem_raw);
     __shared__ int sh[32];
@@ -2618,6 +2693,7 @@ constexpr int kPrefT = 1024, kPrefPT = 8;
 
 __global__ void __launch_bounds__(kPrefT) k_tile_prefix(int32_t* tsum, int tiles, const int* ctl,
                                                         unsigned long long* n_cycles) {
+    LF_TL(g_tl_forest, 3);
     __shared__ int sh[32];
     pdl_wait();
     pdl_trigger();
@@ -2708,6 +2784,13 @@ static int coop_launch(K kernel, int block, ForestArgs& a, cudaStream_t s, size_
     return LF_OK;
 }
 
+// zero the 256-int control block; complete only once the stream predecessor has
+__global__ void k_ctl_zero(int* ctl) {
+    ctl[threadIdx.x] = 0;
+    pdl_trigger();
+    pdl_wait();
+}
+
 static int forest_prepare() {
     static bool attr_done = false;
     if (attr_done) return LF_OK;
@@ -2773,7 +2856,10 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     int rcp = forest_prepare();
     if (rcp) return rcp;
-    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
+    // zero the control block in a PDL kernel: it runs while the factor's last kernel is
+    // still finishing, and k_lf_full1's CTAs become resident meanwhile (a memset node
+    // would serialise: ~5 us between the factor and the tile pass)
+    LF_CUDA(launch_pdl(k_ctl_zero, 1, 256, 0, s, w.ctl));
     ForestArgs a;
     memset(&a, 0, sizeof(a));
     a.N = N;
@@ -2811,7 +2897,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     const int tiles = (int)((N + LB - 1) / LB);
     {
         LF_PROF("lf_tile", -1, s);
-        k_lf_full1<<<tiles, LT, kFull1Smem, s>>>(a);
+        LF_CUDA(launch_pdl(k_lf_full1, tiles, LT, kFull1Smem, s, a));
         LF_CUDA(cudaGetLastError());
     }
     {
@@ -3192,4 +3278,16 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
     return LF_OK;
 }
 
+#ifdef LF_TIMELINE
+int timeline_forest(unsigned long long* out, int reset) {
+    if (reset) {
+        unsigned long long h[16];
+        for (int i = 0; i < 16; i += 2) { h[i] = ~0ull; h[i + 1] = 0; }
+        return cudaMemcpyToSymbol(g_tl_forest, h, sizeof(h)) == cudaSuccess ? 0 : -1;
+    }
+    return cudaMemcpyFromSymbol(out, g_tl_forest, sizeof(g_tl_forest)) == cudaSuccess ? 0 : -1;
+}
+#else
+int timeline_forest(unsigned long long*, int) { return -1; }
+#endif
 }  // namespace lf
