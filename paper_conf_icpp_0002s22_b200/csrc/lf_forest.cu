@@ -1813,83 +1813,81 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
         s.EK1[u] = ek[k].y;
         s.K0[u] = lp ? (nb.x == g - 1 ? ek[k].x : ek[k].y) : KEY_INF;
     }
-    // 0b. run bounds (block max-scan) and each run's weakest link (segmented min-scan)
+    // 0b. run bounds and each run's weakest link, with one block barrier: heads (no link
+    //     to u-1) by warp ballots, the running minimum of K0 by a warp segmented scan,
+    //     and the runs that cross warps from per-warp aggregates (last / first head, tail
+    //     minimum) that every warp reduces for itself.  Position 0 is always a head.
+    __syncthreads();  // K0 of 0a (other threads' vertices)
     {
-        const int u0 = tid * VPT;
-        int st[VPT];
-        bool lk[VPT + 1];
-#pragma unroll
-        for (int j = 0; j <= VPT; j++) lk[j] = u0 + j < LB && linked_prev(u0 + j);
-        int run = INT_MIN;
-#pragma unroll
-        for (int j = 0; j < VPT; j++) {
-            if (!lk[j]) run = u0 + j;
-            st[j] = run;
-        }
-        const int prev_max = block_scan_max_excl(run, sh);
-#pragma unroll
-        for (int j = 0; j < VPT; j++) {
-            const int u = u0 + j;
-            if (st[j] == INT_MIN) st[j] = prev_max;
-            s.r.run[u].x = (short)st[j];
-            if (!lk[j + 1]) s.r.run[st[j]].y = (short)u;
-        }
-        __syncthreads();
-        short en[VPT];
-#pragma unroll
-        for (int j = 0; j < VPT; j++) en[j] = s.r.run[st[j]].y;
-        __syncthreads();
-#pragma unroll
-        for (int j = 0; j < VPT; j++) s.r.run[u0 + j].y = en[j];
-        uint64_t x[VPT];
-        bool hd[VPT];
-        uint64_t agg = KEY_INF;
-        bool anyh = false;
-#pragma unroll
-        for (int j = 0; j < VPT; j++) {
-            hd[j] = !lk[j];
-            const uint64_t kv = s.K0[u0 + j];
-            agg = hd[j] ? kv : umin64(agg, kv);
-            anyh |= hd[j];
-            x[j] = agg;
-        }
+        constexpr int NW = LT / 32;
+        __shared__ int w_last[NW], w_first[NW], w_has[NW];
+        __shared__ uint64_t w_min[NW];
         const int lane = tid & 31, wid = tid >> 5;
-        bool f = anyh;
-        uint64_t v = agg;
+        const int u0 = tid * VPT;
+        bool lk[VPT];
+        uint64_t kv[VPT];
+        int firstHead = INT_MAX, lastHead = -1;
+        uint64_t tmin = KEY_INF;
+#pragma unroll
+        for (int j = 0; j < VPT; j++) {
+            lk[j] = linked_prev(u0 + j);
+            kv[j] = s.K0[u0 + j];
+            if (!lk[j]) { if (firstHead == INT_MAX) firstHead = u0 + j; lastHead = u0 + j; }
+            tmin = lk[j] ? umin64(tmin, kv[j]) : kv[j];
+        }
+        // warp segmented inclusive scan of the thread tails (reset at a thread with a head)
+        uint64_t v = tmin;
+        bool f = lastHead >= 0;
 #pragma unroll
         for (int o2 = 1; o2 < 32; o2 <<= 1) {
             const uint64_t yv = __shfl_up_sync(0xffffffffu, v, o2);
             const int yf = __shfl_up_sync(0xffffffffu, (int)f, o2);
             if (lane >= o2) { if (!f) v = umin64(v, yv); f = f || yf; }
         }
-        __shared__ uint64_t wv[LT / 32];
-        __shared__ int wf[LT / 32];
-        if (lane == 31) { wv[wid] = v; wf[wid] = f; }
-        __syncthreads();
-        if (wid == 0) {
-            uint64_t tv = lane < LT / 32 ? wv[lane] : KEY_INF;
-            bool tf = lane < LT / 32 ? wf[lane] != 0 : false;
-#pragma unroll
-            for (int o2 = 1; o2 < 32; o2 <<= 1) {
-                const uint64_t yv = __shfl_up_sync(0xffffffffu, tv, o2);
-                const int yf = __shfl_up_sync(0xffffffffu, (int)tf, o2);
-                if (lane >= o2) { if (!tf) tv = umin64(tv, yv); tf = tf || yf; }
-            }
-            if (lane < LT / 32) { wv[lane] = tv; wf[lane] = tf; }
-        }
-        __syncthreads();
         uint64_t cv = __shfl_up_sync(0xffffffffu, v, 1);
         bool cf = __shfl_up_sync(0xffffffffu, (int)f, 1) != 0;
-        if (lane == 0) { cv = KEY_INF; cf = true; }
-        if (wid > 0 && !cf) cv = umin64(cv, wv[wid - 1]);
-        if (wid > 0 && lane == 0) { cv = wv[wid - 1]; cf = false; }
+        if (lane == 0) { cv = KEY_INF; cf = false; }
+        const unsigned hm = __ballot_sync(0xffffffffu, lastHead >= 0);
+        const int wl = __reduce_max_sync(0xffffffffu, lastHead);
+        const unsigned wf = __reduce_min_sync(0xffffffffu, (unsigned)firstHead);
+        if (lane == 31) { w_min[wid] = v; w_has[wid] = f; }
+        if (lane == 0) { w_last[wid] = wl; w_first[wid] = (int)wf; }
+        __syncthreads();
+        // from the other warps: the last head before, the first head after, and the
+        // minimum over the run that enters this warp from before
+        const int pl = lane < wid ? w_last[lane] : -1;
+        const int prevLast = __reduce_max_sync(0xffffffffu, pl);
+        const unsigned nfv = (lane > wid && lane < NW) ? (unsigned)w_first[lane] : (unsigned)INT_MAX;
+        const int nextFirst = (int)__reduce_min_sync(0xffffffffu, nfv);
+        const int hw = __reduce_max_sync(0xffffffffu, (lane < wid && w_has[lane]) ? lane : 0);
+        uint64_t cm = (lane >= hw && lane < wid) ? w_min[lane] : KEY_INF;
+#pragma unroll
+        for (int o2 = 16; o2; o2 >>= 1) cm = umin64(cm, __shfl_xor_sync(0xffffffffu, cm, o2));
+        // this thread's incoming run start, running minimum and next head
+        const unsigned before = hm & ((1u << lane) - 1u);
+        const int srcb = before ? 31 - __clz(before) : lane;
+        const int lastB = __shfl_sync(0xffffffffu, lastHead, srcb);
+        int start = before ? lastB : prevLast;
+        const unsigned after = lane == 31 ? 0u : (hm & ~((2u << lane) - 1u));
+        const int srca = after ? __ffs(after) - 1 : lane;
+        const int firstA = __shfl_sync(0xffffffffu, firstHead, srca);
+        int nh = after ? firstA : nextFirst;
+        uint64_t r = cf ? cv : umin64(cv, cm);
+        short2 rr[VPT];
+        uint64_t km[VPT];
 #pragma unroll
         for (int j = 0; j < VPT; j++) {
-            if (hd[j]) break;
-            x[j] = umin64(x[j], cv);
+            if (!lk[j]) { start = u0 + j; r = kv[j]; } else r = umin64(r, kv[j]);
+            rr[j].x = (short)start;
+            km[j] = r;
         }
 #pragma unroll
-        for (int j = 0; j < VPT; j++) s.K1[u0 + j] = x[j];
+        for (int j = VPT - 1; j >= 0; j--) {
+            rr[j].y = (short)(nh == INT_MAX ? LB - 1 : nh - 1);
+            if (!lk[j]) nh = u0 + j;
+        }
+#pragma unroll
+        for (int j = 0; j < VPT; j++) { s.r.run[u0 + j] = rr[j]; s.K1[u0 + j] = km[j]; }
     }
     __syncthreads();
     // 0c. contract runs: virtual links between run ends (length, weakest key)
