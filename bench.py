@@ -462,8 +462,9 @@ def main():
         ev1.synchronize()
         prof_step_ms.append(ev0.elapsed_time(ev1))
         recs = lf.profile_collect()
-        # one record per stage; the perm stage launches k_tile_prefix + k_perm_tri
-        launches_per_step = sum(2 if nm in ("perm", "perm_tridiag") else 1 for nm, _ in recs)
+        # one record per stage; the perm stage launches k_tile_prefix + k_perm_tri, and every
+        # lf_linear_forest call starts with the (unrecorded) control-block kernel k_ctl_zero
+        launches_per_step = sum(2 if nm in ("perm", "perm_tridiag") else 1 for nm, _ in recs) + 1
         for nm, ms in recs:
             kern.setdefault(nm, []).append(ms)
     torch.cuda.synchronize()

@@ -27,7 +27,7 @@ for w in $WHAT; do
         --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 2 --warmup 1 --no-graph --no-cpu-baseline \
         > gpurun_out/ncu_launch_$TAG.log 2>&1
       timeout 900 ncu --set full --clock-control none --import-source on \
-        -k regex:"k_propose_tile|k_mutual0|k_rounds_fused|k_lf_full1|k_red_full|k_lf_full2|k_perm_tri" -c 7 \
+        -k regex:"k_propose_stream|k_mutual0|k_rounds_fused|k_lf_full1|k_red_full|k_lf_full2|k_perm_tri" -c 7 \
         -o gpurun_out/prof_$TAG -f python bench.py --steps 1 --warmup 1 --no-graph --no-cpu-baseline \
         > gpurun_out/ncu_full_$TAG.log 2>&1 ;;
     phase)
