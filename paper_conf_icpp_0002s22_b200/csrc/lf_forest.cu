@@ -2549,6 +2549,12 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
     TileSmemE& s = *reinterpret_cast<TileSmemE*>(smem_raw);
     __shared__ int sh[32];
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
+    int2 lcs[VPT];  // the tile pass's local results, in flight with the tile's slots
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int64_t g = (int64_t)b0 + threadIdx.x + k * LT;
+        lcs[k] = g < a.hi ? __ldg(a.loc2 + g) : make_int2(0, 0);
+    }
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     ulonglong2 ek[VPT];
@@ -2564,7 +2570,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
         lens[k] = 0;
         wait[k] = false;
         if (g >= a.hi) continue;
-        const int2 lc = a.loc2[g];
+        const int2 lc = lcs[k];
         if (lc.x == kLocDone) { lens[k] = a.len[g]; continue; }
         const int Tl[2] = {(int)(lc.x & 0xffff), (int)((uint32_t)lc.x >> 16)};
         st[k].R0 = (int)(lc.y & 0xffff);
@@ -2620,7 +2626,7 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
         for (int i = 0; i < 2; i++) {
             const int so = (st[k].so >> i) & 1;
             if (bi[i] < 0) {  // a path end (the vertex reached it inside the tile)
-                const int t = i ? (int)((uint32_t)a.loc2[g].x >> 16) : (int)(a.loc2[g].x & 0xffff);
+                const int t = i ? (int)((uint32_t)lcs[k].x >> 16) : (int)(lcs[k].x & 0xffff);
                 E[i] = b0 + t;
                 D[i] = Rl[i];
                 continue;
