@@ -215,6 +215,19 @@ __device__ __forceinline__ void topn_insert_net(uint64_t (&t)[NN], uint64_t x) {
     }
 }
 
+// the same network guarded by a predicate (no key masking, one 64-bit compare per slot):
+// the round-0 stream is ALU-bound, and this is most of its per-entry work
+template <int NN>
+__device__ __forceinline__ void topn_insert_pred(uint64_t (&t)[NN], uint64_t x, bool ok) {
+#pragma unroll
+    for (int i = 0; i < NN; i++) {
+        const bool c = ok && x > t[i];
+        const uint64_t h = c ? x : t[i];
+        x = c ? t[i] : x;
+        t[i] = h;
+    }
+}
+
 #if defined(LF_TILE_MINB) && LF_TILE_MINB > 0
 #define LF_TILE_BOUNDS __launch_bounds__(PT, LF_TILE_MINB)
 #else
@@ -490,11 +503,16 @@ __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
                 const bool isd = j == v;                                 // diagonal (L231)
                 dbits = isd ? xb : dbits;
                 bool ok = !isd && ab != 0u;                              // zero (L31)
-                theta0 |= ok ? 1u : 0u;
-                if (CHARGED) ok = ok && (((a.state[j] & ST_CHARGE) ? 1u : 0u) != cv);  // L17
+                if (CHARGED) {
+                    theta0 |= ok ? 1u : 0u;
+                    ok = ok && (((a.state[j] & ST_CHARGE) ? 1u : 0u) != cv);  // L17
+                }
                 const uint64_t key = ((uint64_t)ab << 32) | (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31));
-                topn_insert_net<NN>(top, ok ? key : 0ull);
+                topn_insert_pred<NN>(top, key, ok);
             }
+            // uncharged: every eligible entry entered the top list, so theta0 (some
+            // eligible entry, L19) is "the list is not empty"; lanes merge it below
+            if (!CHARGED) theta0 |= top[0] != 0 ? 1u : 0u;
         } else {
             for (int64_t e = rs + li; e < re; e += G) {
                 const int32_t j = __ldg(a.col + e);
