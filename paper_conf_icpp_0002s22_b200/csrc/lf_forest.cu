@@ -876,13 +876,14 @@ __device__ __forceinline__ int2 ghost_slots(const ForestArgs& a, int32_t x) {
 }
 
 // keys of the own vertices' slots (global; a remote min endpoint needs one gather)
-template <class S>
+template <class S, int TT = LT>
 __device__ __forceinline__ void slot_keys(const ForestArgs& a, S& s, int32_t b0,
-                                         ulonglong2 (&ek)[VPT]) {
+                                         ulonglong2 (&ek)[LB / TT]) {
+    constexpr int VV = LB / TT;
     const Tile T = tile_of(s);
 #pragma unroll
-    for (int k = 0; k < VPT; k++) {
-        const int u = threadIdx.x + k * LT;
+    for (int k = 0; k < VV; k++) {
+        const int u = threadIdx.x + k * TT;
         const int32_t g = b0 + u;
         const int2 nb = s.nb[u];
         ek[k].x = KEY_INF;
@@ -903,16 +904,17 @@ __device__ __forceinline__ void slot_keys(const ForestArgs& a, S& s, int32_t b0,
 }
 
 // slots and weights of the tile in one round trip (cycle pass)
-template <class S>
+template <class S, int TT = LT>
 __device__ __forceinline__ void load_tile_w(const int2* __restrict__ src, const float2* __restrict__ wsrc,
                                             S& s, int32_t b0, int64_t hi) {
+    constexpr int VV = LB / TT;
     if (threadIdx.x == 0) {
         s.b0 = b0;
         s.tend = (int32_t)((int64_t)b0 + LB < hi ? (int64_t)b0 + LB : hi);
     }
 #pragma unroll
-    for (int k = 0; k < VPT; k++) {
-        const int u = threadIdx.x + k * LT;
+    for (int k = 0; k < VV; k++) {
+        const int u = threadIdx.x + k * TT;
         const int64_t g = (int64_t)b0 + u;
         const bool in = g < hi;
         const int2 nb = in ? src[g] : make_int2(-1, -1);
@@ -2543,29 +2545,40 @@ struct ExpState {       // a vertex waiting for reduced results
     int dseg;
 };
 
-__global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
+// threads and resident CTAs of the expand pass (measured on C2: 512 x 3 beats 256 x 4,
+// 256 x 3 and 128 x 8 -- fewer threads per tile serialise each thread's vertices)
+#ifndef LF_ET
+#define LF_ET 512
+#endif
+#ifndef LF_EMINB
+#define LF_EMINB 3
+#endif
+constexpr int ET = LF_ET;
+constexpr int EV = LB / ET;
+
+__global__ void __launch_bounds__(ET, LF_EMINB) k_lf_full2(ForestArgs a) {
     LF_TL(g_tl_forest, 2);
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemE& s = *reinterpret_cast<TileSmemE*>(smem_raw);
     __shared__ int sh[32];
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
-    int2 lcs[VPT];  // the tile pass's local results, in flight with the tile's slots
+    int2 lcs[EV];  // the tile pass's local results, in flight with the tile's slots
 #pragma unroll
-    for (int k = 0; k < VPT; k++) {
-        const int64_t g = (int64_t)b0 + threadIdx.x + k * LT;
+    for (int k = 0; k < EV; k++) {
+        const int64_t g = (int64_t)b0 + threadIdx.x + k * ET;
         lcs[k] = g < a.hi ? __ldg(a.loc2 + g) : make_int2(0, 0);
     }
-    load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
+    load_tile_w<TileSmemE, ET>(a.pi2, a.pi2_w, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
-    ulonglong2 ek[VPT];
-    slot_keys(a, s, b0, ek);
-    int lens[VPT];
-    bool wait[VPT];
-    ExpState st[VPT];
+    ulonglong2 ek[EV];
+    slot_keys<TileSmemE, ET>(a, s, b0, ek);
+    int lens[EV];
+    bool wait[EV];
+    ExpState st[EV];
     int ncyc = 0;
 #pragma unroll
-    for (int k = 0; k < VPT; k++) {
-        const int u = threadIdx.x + k * LT;
+    for (int k = 0; k < EV; k++) {
+        const int u = threadIdx.x + k * ET;
         const int32_t g = b0 + u;
         lens[k] = 0;
         wait[k] = false;
@@ -2611,9 +2624,9 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
     }
     pdl_wait();  // the reduced scan's results
 #pragma unroll
-    for (int k = 0; k < VPT; k++) {
+    for (int k = 0; k < EV; k++) {
         if (!wait[k]) continue;
-        const int u = threadIdx.x + k * LT;
+        const int u = threadIdx.x + k * ET;
         const int32_t g = b0 + u;
         const int2 nb = s.nb[u];
         const int Rl[2] = {st[k].R0, st[k].R1};
@@ -2673,14 +2686,14 @@ __global__ void __launch_bounds__(LT, LF_LMINB) k_lf_full2(ForestArgs a) {
         ncyc += co.ncyc;
     }
     // tile-local exclusive prefix of the path lengths in id order (thread t owns
-    // u = t + k LT: one block scan per k, carried)
+    // u = t + k ET: one block scan per k, carried)
     {
         int carry = 0;
 #pragma unroll
-        for (int k = 0; k < VPT; k++) {
+        for (int k = 0; k < EV; k++) {
             int tot = 0;
             const int e = block_scan_sum_excl(lens[k], sh, &tot);
-            const int32_t gk = b0 + (int)threadIdx.x + k * LT;
+            const int32_t gk = b0 + (int)threadIdx.x + k * ET;
             if (gk < a.hi && lens[k]) a.off[gk] = carry + e;
             carry += tot;
         }
@@ -2913,7 +2926,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     }
     {
         LF_PROF("lf_expand", -1, s);
-        LF_CUDA(launch_pdl(k_lf_full2, tiles, LT, sizeof(TileSmemE), s, a));
+        LF_CUDA(launch_pdl(k_lf_full2, tiles, ET, sizeof(TileSmemE), s, a));
     }
     {
         LF_PROF(tri ? "perm_tridiag" : "perm", -1, s);
