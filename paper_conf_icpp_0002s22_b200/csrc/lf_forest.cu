@@ -1528,7 +1528,10 @@ __global__ void __launch_bounds__(kOffT) k_path_offsets(int64_t N, const int32_t
 // step (3) (+ step (4) when tri): r = new(v) = off[l(v)] + p(v) - 1 with off[l] = tile
 // prefix + intra-tile prefix; the forest neighbour in slot pdir[v] is perm[r-1], the other
 // one perm[r+1], so a[r] / c[r] are copied from the factor's signed slot values
-constexpr int kPermBatch = 4;  // vertices per thread per iteration (loads in flight)
+#ifndef LF_PERMB
+#define LF_PERMB 2
+#endif
+constexpr int kPermBatch = LF_PERMB;  // vertices per thread per iteration (loads in flight)
 constexpr int kNoSlot = 2;     // pdir: no predecessor / successor slot (k_lf_full1/2)
 
 __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __restrict__ path_id,
@@ -1546,11 +1549,21 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < N; v0 += stride * kPermBatch) {
         int32_t l[kPermBatch], p[kPermBatch], r[kPermBatch];
+        float2 pv[kPermBatch];
+        float dg[kPermBatch];
+        int d[kPermBatch];
+        // every per-vertex load first (the coefficients do not depend on the new index)
 #pragma unroll
         for (int b = 0; b < kPermBatch; b++) {
             const int64_t v = v0 + b * stride;
-            l[b] = v < N ? __ldg(path_id + v) : 0;
-            p[b] = v < N ? __ldg(pos + v) : 0;
+            const bool in = v < N;
+            l[b] = in ? __ldg(path_id + v) : 0;
+            p[b] = in ? __ldg(pos + v) : 0;
+            if (ta) {
+                pv[b] = in ? __ldg(pi2_val + v) : make_float2(0.f, 0.f);
+                d[b] = in ? __ldg(pdir + v) : 0;
+                dg[b] = in ? __ldg(diag + v) : 0.f;
+            }
         }
 #pragma unroll
         for (int b = 0; b < kPermBatch; b++) r[b] = __ldg(tbase + l[b] / chunk) + __ldg(off + l[b]) + p[b] - 1;
@@ -1561,12 +1574,10 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
             iperm[v] = r[b];
             perm[r[b]] = (int32_t)v;
             if (ta) {
-                const float2 pv = __ldg(pi2_val + v);
-                const int d = __ldg(pdir + v);
-                const int ps = d & 3, ss = (d >> 2) & 3;
-                ta[r[b]] = ps == kNoSlot ? 0.0f : (ps ? pv.y : pv.x);
-                tc[r[b]] = ss == kNoSlot ? 0.0f : (ss ? pv.y : pv.x);
-                tb[r[b]] = __ldg(diag + v);
+                const int ps = d[b] & 3, ss = (d[b] >> 2) & 3;
+                ta[r[b]] = ps == kNoSlot ? 0.0f : (ps ? pv[b].y : pv[b].x);
+                tc[r[b]] = ss == kNoSlot ? 0.0f : (ss ? pv[b].y : pv[b].x);
+                tb[r[b]] = dg[b];
             }
         }
     }
