@@ -729,7 +729,10 @@ __device__ __forceinline__ void store_slots(T* __restrict__ p, const T (&o)[NN])
 // any result is used (the proposal gathers are the latency chain of this pass).  In a
 // fresh round pi is empty and the proposals are already in key order, so the confirmed
 // ones are copied in place order without a merge.
-constexpr int kMutual0Rows = 4;
+#ifndef LF_M0ROWS
+#define LF_M0ROWS 4
+#endif
+constexpr int kMutual0Rows = LF_M0ROWS;  // rows per thread of k_mutual0 (loads in flight)
 
 template <int NN, int MB>
 __global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
