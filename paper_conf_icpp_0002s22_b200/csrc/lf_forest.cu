@@ -799,6 +799,26 @@ __device__ __forceinline__ int outward_slot(int2 nbt, const Tile& T) {
     return l0 ? 1 : 0;
 }
 
+// warp-aggregated slot claim in two halves, so that nothing waits for the atomic's return
+// until the slot is used: claim_issue (ballot + one atomic per warp, result in lane 0) and
+// claim_pos (broadcast + rank; -1 if not taken)
+struct Claim {
+    unsigned m;
+    int base;  // lane 0: the warp's first slot
+};
+__device__ __forceinline__ Claim claim_issue(int* count, bool take) {
+    Claim c;
+    c.m = __ballot_sync(0xffffffffu, take);
+    c.base = 0;
+    if ((threadIdx.x & 31) == 0 && c.m) c.base = atomicAdd(count, __popc(c.m));
+    return c;
+}
+__device__ __forceinline__ int claim_pos(const Claim& c) {
+    const int lane = threadIdx.x & 31;
+    const int base = __shfl_sync(0xffffffffu, c.base, 0);
+    return ((c.m >> lane) & 1u) ? base + __popc(c.m & ((1u << lane) - 1u)) : -1;
+}
+
 // warp-aggregated append; returns the list position of g (-1 if not taken)
 __device__ __forceinline__ int list_append(int32_t* list, int* count, int32_t g, bool take) {
     const unsigned m = __ballot_sync(0xffffffffu, take);
@@ -2342,14 +2362,14 @@ __global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
     load_tile_w(a.pi2, a.pi2_w, s, b0, a.hi);
     const Tile T{b0, (int32_t)((int64_t)b0 + LB < a.hi ? (int64_t)b0 + LB : a.hi)};
     int2 orig[VPT];
-    int idx_[VPT];  // boundary-list slots, claimed now: the atomic's round trip overlaps the ranking
+    Claim cl_[VPT];  // boundary-list slots, claimed now: the atomic's round trip overlaps the ranking
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         orig[k] = s.nb[threadIdx.x + k * LT];
         const int32_t g = b0 + (int)threadIdx.x + k * LT;
         const bool r0 = orig[k].x >= 0 && !is_local(orig[k].x, T);
         const bool r1 = orig[k].y >= 0 && !is_local(orig[k].y, T);
-        idx_[k] = list_append(a.list1, &a.ctl[kCtlCnt1], g, g < a.hi && (r0 || r1));
+        cl_[k] = claim_issue(&a.ctl[kCtlCnt1], g < a.hi && (r0 || r1));  // positions in phase 7
     }
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
@@ -2368,6 +2388,7 @@ __global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
         const bool r0 = nb.x >= 0 && !is_local(nb.x, T);
         const bool r1 = nb.y >= 0 && !is_local(nb.y, T);
         const bool boundary = g < a.hi && (r0 || r1);
+        const int idx = claim_pos(cl_[k]);  // warp-uniform (shuffle)
         if (g < a.hi) {
             if (o[k].cyc) {
                 const CycOut c = cycle_finish(g, nb, ek[k], o[k].Ks, o[k].C);
@@ -2385,7 +2406,7 @@ __global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
             }
         }
         if (boundary) {
-            const int idx = idx_[k];
+            a.list1[idx] = g;
             int2 q, rl, dk;
             ulonglong2 kk;
 #pragma unroll
