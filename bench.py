@@ -158,13 +158,27 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz, cluster_ran=False):
     return 0
 
 
-def ncu_traffic(kernel):
-    """dram bytes per launch of `kernel` from the committed ncu capture (profiles/traffic.json)."""
+def ncu_traffic(kernel, key="bytes_per_launch"):
+    """dram bytes (or warp instructions) per launch of `kernel` from the committed ncu
+    capture (profiles/traffic.json)."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     try:
-        return json.load(open(p))["bytes_per_launch"].get(kernel)
+        return json.load(open(p))[key].get(kernel)
     except (OSError, ValueError, KeyError):
         return None
+
+
+def issue_view(kernel, ms, sm_count, mhz):
+    """The dominant kernel against the SM issue rate (4 warp instructions per SM per cycle):
+    its ncu warp-instruction count per launch over its live launch time."""
+    inst = ncu_traffic(kernel, "warp_inst_per_launch")
+    if not inst or not ms or not mhz:
+        return None
+    ach = inst / (ms * 1e-3) / 1e9
+    peak = 4 * sm_count * mhz * 1e6 / 1e9
+    return {"bound": "issue", "achieved": round(ach, 1), "peak": round(peak, 1),
+            "unit": "G warp-inst/s", "frac": round(ach / peak, 4), "warp_inst_per_launch": inst,
+            "source": "ncu smsp__inst_executed.sum (profiles/traffic.json) / live launch time"}
 
 
 def cpu_baseline(A, runs):
@@ -559,6 +573,8 @@ def main():
                 "peak": peak, "peak_kind": peak_kind, "unit": "GB/s",
                 "frac": round(dom_ach / peak, 4) if dom_ach else None,
                 "traffic": ncu_traffic(dom) if args.config == "C2" else None,
+                "issue_view": issue_view(dom, kavg.get(dom), torch.cuda.get_device_properties(0).multi_processor_count,
+                                         clk.get("sm_mhz")) if args.config == "C2" and dom else None,
                 "alg_bytes_per_launch": int(dom_bytes),
                 "ms_per_launch": round(kavg[dom], 5) if dom else None,
             },
