@@ -1942,7 +1942,8 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
         }
         s.r.vw[u] = vw;
     }
-    __syncthreads();
+    // no barrier: phase 1 reads only its own vertices' contracted slots and runs (this
+    // thread wrote the slots; the runs are from before the last barrier)
     LF_PHASE(ctlp, 0);
     // 1. splitters (run ends, terminals, hashed vertices); run cycles -3, interiors -2
 #pragma unroll
@@ -2120,8 +2121,8 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
             o[k].C = make_int2(kd, 2 * (d - (kd >> 1) - 1) + ((kd & 1) ^ 1));
         }
     }
-    // 5. interior run vertices and run cycles, from the run ends' node windows
-    __syncthreads();
+    // 5. interior run vertices and run cycles, from the run ends' node windows (phase 4
+    //    wrote registers only: no barrier needed since the one inside it)
     LF_PHASE(ctlp, 4);
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
