@@ -401,9 +401,31 @@ constexpr int SETILE = LF_SETILE;   // entries per stage
 struct StreamSmem {
     int32_t col[2][SETILE];
     float val[2][SETILE];
-    int64_t rp[3][SPT + 1];
+    int64_t rp[3][SPT + 2];   // +2: rows of 16-byte multiples (bulk copies)
     int64_t a0[2];            // aligned start of the staged range per stage (or -1)
+    unsigned long long bar[2];  // mbarriers of the bulk copies, one per prefetch batch parity
 };
+
+// one-thread bulk copies (TMA engine, no per-thread address arithmetic: the round-0 stream is
+// ALU-bound and per-thread cp.async staging was a quarter of its instructions)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init1(unsigned long long* b) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(unsigned long long* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(unsigned long long* b, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "LF_MBW_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra LF_MBW_%=;\n}" ::"r"(smem_u32(b)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, unsigned long long* b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(b)) : "memory");
+}
 
 template <int R>
 __device__ __forceinline__ void issue_rowptr(const ProposeArgs& a, int64_t t, int64_t* dst) {
@@ -445,33 +467,64 @@ __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
     const int64_t t0 = blockIdx.x;
     unsigned long long my_live = 0, my_nnz = 0;
     int my_prop = 0;
+    // a prefetch batch: the entries of tile te (row pointers rpe, already staged) into stage
+    // sb and the row pointers of tile tr (if any) into rps, on mbarrier bar; ranges the bulk
+    // engine cannot take (the arrays' ends) fall back to per-thread cp.async
+    const int64_t nnz = __ldg(a.rowptr + a.N);
+    auto issue_batch = [&](int64_t te, const int64_t* rpe, int sb, int64_t tr, int64_t* rps,
+                           unsigned long long* bar) {
+        const int64_t rle = (te * R + R <= a.N) ? R : a.N - te * R;
+        const int64_t e0 = rpe[0], e1 = rpe[rle];
+        const int64_t ea = e0 & ~(int64_t)3, eb = (e1 + 3) & ~(int64_t)3;
+        const bool fits = e1 - ea <= SETILE;
+        const bool bulkE = fits && eb <= nnz && eb - ea <= SETILE;
+        const bool hasR = tr < ntiles;
+        const int64_t r0 = tr * R;
+        const int64_t rc = hasR ? ((r0 + R + 1 <= a.N + 1) ? R + 1 : a.N + 1 - r0) : 0;
+        const int64_t rc2 = (rc + 1) & ~(int64_t)1;
+        const bool bulkR = hasR && r0 + rc2 <= a.N + 1;
+        if (tid == 0) {
+            S.a0[sb] = fits ? ea : -1;
+            const uint32_t bytes = (bulkE ? (uint32_t)(eb - ea) * 8u : 0u) + (bulkR ? (uint32_t)rc2 * 8u : 0u);
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive_tx(bar, bytes);
+            if (bulkE) {
+                bulk_g2s(S.col[sb], a.col + ea, (uint32_t)(eb - ea) * 4u, bar);
+                bulk_g2s(S.val[sb], a.val + ea, (uint32_t)(eb - ea) * 4u, bar);
+            }
+            if (bulkR) bulk_g2s(rps, a.rowptr + r0, (uint32_t)rc2 * 8u, bar);
+        }
+        if (fits && !bulkE) {
+            int64_t dummy;
+            issue_entries(a, e0, e1, S.col[sb], S.val[sb], &dummy);
+        }
+        if (hasR && !bulkR) issue_rowptr<R>(a, tr, rps);
+        cp_commit();
+    };
     if (t0 < ntiles) {
-        // prologue: row pointers of the first tile (waited), then its entries + next rowptr
+        if (tid == 0) {
+            mbar_init1(&S.bar[0]);
+            mbar_init1(&S.bar[1]);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        // prologue: row pointers of the first tile (waited), then batch 0: its entries and
+        // the next tile's row pointers
         issue_rowptr<R>(a, t0, S.rp[0]);
         cp_commit();
         cp_wait_all();
         __syncthreads();
-        {
-            const int64_t rl = (t0 * R + R <= a.N) ? R : a.N - t0 * R;
-            issue_entries(a, S.rp[0][0], S.rp[0][rl], S.col[0], S.val[0], &S.a0[0]);
-        }
-        if (t0 + gridDim.x < ntiles) issue_rowptr<R>(a, t0 + gridDim.x, S.rp[1]);
-        cp_commit();
+        issue_batch(t0, S.rp[0], 0, t0 + gridDim.x, S.rp[1], &S.bar[0]);
     }
     int i = 0;
     for (int64_t t = t0; t < ntiles; t += gridDim.x, i++) {
         cp_wait_all();
+        mbar_wait_parity(&S.bar[i & 1], (uint32_t)((i >> 1) & 1));
         __syncthreads();
         const int b = i & 1;
         const int64_t* rp = S.rp[i % 3];
         const int64_t tn = t + gridDim.x;
-        if (tn < ntiles) {  // prefetch: entries of the next tile, row pointers of the one after
-            const int64_t* rpn = S.rp[(i + 1) % 3];
-            const int64_t rl = (tn * R + R <= a.N) ? R : a.N - tn * R;
-            issue_entries(a, rpn[0], rpn[rl], S.col[b ^ 1], S.val[b ^ 1], &S.a0[b ^ 1]);
-            if (tn + gridDim.x < ntiles) issue_rowptr<R>(a, tn + gridDim.x, S.rp[(i + 2) % 3]);
-            cp_commit();
-        }
+        if (tn < ntiles)  // prefetch: entries of the next tile, row pointers of the one after
+            issue_batch(tn, S.rp[(i + 1) % 3], b ^ 1, tn + gridDim.x, S.rp[(i + 2) % 3], &S.bar[(i + 1) & 1]);
         const int64_t a0 = S.a0[b];
         const bool staged = a0 >= 0;
         const int32_t* scol = S.col[b];
