@@ -443,6 +443,13 @@ __device__ __forceinline__ void issue_entries(const ProposeArgs& a, int64_t e0, 
         return;
     }
     if (threadIdx.x == 0) *a0_out = a0;
+    if ((((uintptr_t)a.col | (uintptr_t)a.val) & 15) != 0) {  // offset views: 4-byte copies
+        for (int64_t e = e0 + threadIdx.x; e < e1; e += SPT) {
+            cp4(scol + (e - a0), a.col + e);
+            cp4(sval + (e - a0), a.val + e);
+        }
+        return;
+    }
     const int64_t v1 = e1 & ~(int64_t)3;
     const int nvec = (int)((v1 - a0) >> 2);
     for (int i = threadIdx.x; i < nvec; i += SPT) {
@@ -471,18 +478,20 @@ __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
     // sb and the row pointers of tile tr (if any) into rps, on mbarrier bar; ranges the bulk
     // engine cannot take (the arrays' ends) fall back to per-thread cp.async
     const int64_t nnz = __ldg(a.rowptr + a.N);
+    // bulk copies need 16-byte aligned sources (the caller's arrays may be offset views)
+    const bool aligned_cv = (((uintptr_t)a.col | (uintptr_t)a.val) & 15) == 0;
     auto issue_batch = [&](int64_t te, const int64_t* rpe, int sb, int64_t tr, int64_t* rps,
                            unsigned long long* bar) {
         const int64_t rle = (te * R + R <= a.N) ? R : a.N - te * R;
         const int64_t e0 = rpe[0], e1 = rpe[rle];
         const int64_t ea = e0 & ~(int64_t)3, eb = (e1 + 3) & ~(int64_t)3;
         const bool fits = e1 - ea <= SETILE;
-        const bool bulkE = fits && eb <= nnz && eb - ea <= SETILE;
+        const bool bulkE = fits && aligned_cv && eb <= nnz && eb - ea <= SETILE;
         const bool hasR = tr < ntiles;
         const int64_t r0 = tr * R;
         const int64_t rc = hasR ? ((r0 + R + 1 <= a.N + 1) ? R + 1 : a.N + 1 - r0) : 0;
         const int64_t rc2 = (rc + 1) & ~(int64_t)1;
-        const bool bulkR = hasR && r0 + rc2 <= a.N + 1;
+        const bool bulkR = hasR && r0 + rc2 <= a.N + 1 && ((uintptr_t)(a.rowptr + r0) & 15) == 0;
         if (tid == 0) {
             S.a0[sb] = fits ? ea : -1;
             const uint32_t bytes = (bulkE ? (uint32_t)(eb - ea) * 8u : 0u) + (bulkR ? (uint32_t)rc2 * 8u : 0u);

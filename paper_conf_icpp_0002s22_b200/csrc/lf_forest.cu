@@ -345,6 +345,41 @@ __device__ __forceinline__ int block_scan_sum_excl(int x, int* sh, int* total) {
     return res;
 }
 
+// V independent exclusive block scans at once (sh: 32 * V ints)
+template <int V>
+__device__ __forceinline__ void block_scan_sum_excl_v(const int (&x)[V], int* sh, int (&ex)[V], int (&total)[V]) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int nw = (int)(blockDim.x >> 5);
+    int inc[V];
+#pragma unroll
+    for (int v = 0; v < V; v++) inc[v] = x[v];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+        for (int v = 0; v < V; v++) {
+            const int y = __shfl_up_sync(0xffffffffu, inc[v], o);
+            if (lane >= o) inc[v] += y;
+        }
+    }
+    if (lane == 31) {
+#pragma unroll
+        for (int v = 0; v < V; v++) sh[v * 32 + w] = inc[v];
+    }
+    __syncthreads();
+#pragma unroll
+    for (int v = 0; v < V; v++) {
+        const int ws = lane < nw ? sh[v * 32 + lane] : 0;
+        int before = lane < w ? ws : 0, all = ws;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+            before += __shfl_xor_sync(0xffffffffu, before, o);
+            all += __shfl_xor_sync(0xffffffffu, all, o);
+        }
+        ex[v] = inc[v] - x[v] + before;
+        total[v] = all;
+    }
+}
+
 __device__ __forceinline__ int block_scan_min_rev(int x, int* sh) {
     // suffix minimum: scan from the last thread backwards
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -2593,7 +2628,7 @@ __global__ void __launch_bounds__(ET, LF_EMINB) k_lf_full2(ForestArgs a) {
     LF_TL(g_tl_forest, 2);
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemE& s = *reinterpret_cast<TileSmemE*>(smem_raw);
-    __shared__ int sh[32];
+    __shared__ int sh[32 * EV];  // the final vector scan (read once: no reuse barrier)
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     int2 lcs[EV];  // the tile pass's local results, in flight with the tile's slots
 #pragma unroll
@@ -2719,16 +2754,16 @@ __global__ void __launch_bounds__(ET, LF_EMINB) k_lf_full2(ForestArgs a) {
         ncyc += co.ncyc;
     }
     // tile-local exclusive prefix of the path lengths in id order (thread t owns
-    // u = t + k ET: one block scan per k, carried)
+    // u = t + k ET): the EV scans run together in one block scan (one set of barriers)
     {
+        int e[EV], tot[EV];
+        block_scan_sum_excl_v<EV>(lens, sh, e, tot);
         int carry = 0;
 #pragma unroll
         for (int k = 0; k < EV; k++) {
-            int tot = 0;
-            const int e = block_scan_sum_excl(lens[k], sh, &tot);
             const int32_t gk = b0 + (int)threadIdx.x + k * ET;
-            if (gk < a.hi && lens[k]) a.off[gk] = carry + e;
-            carry += tot;
+            if (gk < a.hi && lens[k]) a.off[gk] = carry + e[k];
+            carry += tot[k];
         }
         if (threadIdx.x == 0) a.tsum[blockIdx.x] = carry;
     }

@@ -211,6 +211,22 @@ def test_c2_full_size(torch_cuda, lfm, oracle_mod, n):
         check_forest(torch_cuda, lfm, oracle_mod, A, fac, ref)
 
 
+def test_factor_unaligned_inputs(torch_cuda, lfm, oracle_mod):
+    """CSR arrays that are offset views (col/val 4-byte, rowptr 8-byte aligned, not 16):
+    the round-0 stream must fall back from bulk copies to per-thread staging."""
+    torch = torch_cuda
+    A = _cached("C1")
+    pad = lambda x: torch.cat([torch.zeros(1, dtype=x.dtype), x]).cuda()[1:]
+    rp, col, val = pad(torch.from_numpy(A.rowptr)), pad(torch.from_numpy(A.col)), pad(torch.from_numpy(A.val))
+    assert col.data_ptr() % 16 != 0 and rp.data_ptr() % 16 != 0
+    out = lfm.factor(rp, col, val, 2, live=True)
+    torch.cuda.synchronize()
+    pi_o, pw_o, rounds_o, lr, ln = oracle_mod.factor(A, 2, counters=True)
+    assert np.array_equal(out["pi"].cpu().numpy(), pi_o)
+    assert np.array_equal(out["pi_w"].cpu().numpy().view(np.uint32), pw_o.view(np.uint32))
+    assert np.array_equal(out["live"].cpu().numpy()[:5], lr)
+
+
 @pytest.mark.parametrize("cfg", ["C2", "C3"])
 def test_repeated_runs_cached_and_uncached_rounds(torch_cuda, lfm, oracle_mod, monkeypatch, cfg):
     """Rounds 1..M-1 in both modes (shared-memory cached / global worklists),
