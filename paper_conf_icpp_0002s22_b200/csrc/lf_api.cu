@@ -234,6 +234,8 @@ int lf_linear_forest(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t*
     if (N < 0 || N >= ((int64_t)1 << 31)) return set_error(LF_EINVAL, "lf_linear_forest: bad N");
     if (N > 0 && (!pi2 || !pi2_w || !forest || !path_id || !pos || !perm || !iperm))
         return set_error(LF_EINVAL, "lf_linear_forest: NULL argument");
+    if (((uintptr_t)pi2 | (uintptr_t)pi2_w | (uintptr_t)forest) & 7)
+        return set_error(LF_EINVAL, "lf_linear_forest: pi2, pi2_w and forest must be 8-byte aligned");
     Carve c(ws, ws_bytes);
     ForestWs w;
     forest_ws_carve(c, N, &w);
@@ -250,6 +252,8 @@ int lf_linear_forest_tridiag(int64_t N, const int32_t* pi2, const float* pi2_w, 
     if (N > 0 && (!pi2 || !pi2_w || !pi2_val || !diag || !forest || !path_id || !pos || !perm || !iperm || !a ||
                   !b || !c))
         return set_error(LF_EINVAL, "lf_linear_forest_tridiag: NULL argument");
+    if (((uintptr_t)pi2 | (uintptr_t)pi2_w | (uintptr_t)pi2_val | (uintptr_t)forest) & 7)
+        return set_error(LF_EINVAL, "lf_linear_forest_tridiag: pi2, pi2_w, pi2_val and forest must be 8-byte aligned");
     Carve cv(ws, ws_bytes);
     ForestWs w;
     forest_ws_carve(cv, N, &w);
@@ -273,6 +277,8 @@ int lf_tridiag(int64_t N, const int32_t* forest, const int32_t* iperm, const int
     if (N < 0 || N >= ((int64_t)1 << 31)) return set_error(LF_EINVAL, "lf_tridiag: bad N");
     if (N > 0 && (!forest || !iperm || !pi2 || !pi2_val || !diag || !a || !b || !c))
         return set_error(LF_EINVAL, "lf_tridiag: NULL argument");
+    if (((uintptr_t)forest | (uintptr_t)pi2 | (uintptr_t)pi2_val) & 7)
+        return set_error(LF_EINVAL, "lf_tridiag: forest, pi2 and pi2_val must be 8-byte aligned");
     return tridiag_run(N, forest, iperm, pi2, pi2_val, diag, a, b, c, (cudaStream_t)stream);
 }
 

@@ -65,6 +65,12 @@ def test_invalid_arguments_rejected_before_launch(lib):
     assert lib.lf_factor(C.byref(A), 2, C.byref(o), 1, 1, None, None, None, None, None, 0, None) == -1
     assert lib.lf_linear_forest(-1, None, None, None, None, None, None, None, None, None, 0, None) == -1
     assert lib.lf_tridiag(5, None, None, None, None, None, None, None, None, None) == -1
+    # pair arrays read as 8-byte (int2 / float2) vectors must be 8-byte aligned
+    bad, ok = C.c_void_p(0x1004), C.c_void_p(0x1000)
+    assert lib.lf_linear_forest(4, bad, ok, ok, ok, ok, ok, ok, None, None, 0, None) == -1
+    assert b"aligned" in lib.lf_last_error()
+    assert lib.lf_tridiag(4, ok, ok, bad, ok, ok, ok, ok, ok, None) == -1
+    assert b"aligned" in lib.lf_last_error()
 
 
 def test_product_package_does_not_import_oracle():
