@@ -2271,7 +2271,10 @@ __device__ __forceinline__ int2 to_pos(const ForestArgs& a, int2 q) {
 // sixteen SMs serve them sixteen times faster.  Windows are ping-ponged between two
 // buffers (a step reads buffer b everywhere and writes buffer b^1 of its own nodes), so
 // one cluster barrier per step suffices; finished path nodes are copied forward.
-constexpr int kRedCl = 16;           // CTAs of the cluster (non-portable size)
+#ifndef LF_REDCL
+#define LF_REDCL 8
+#endif
+constexpr int kRedCl = LF_REDCL;     // CTAs of the cluster (portable size; 16 measured the same on C2)
 constexpr int kRedClNodes = 2048;    // nodes per CTA
 struct RedSmemC {
     int2 q[2][kRedClNodes];
