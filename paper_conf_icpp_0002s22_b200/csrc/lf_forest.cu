@@ -2266,9 +2266,10 @@ __device__ __forceinline__ int2 to_pos(const ForestArgs& a, int2 q) {
 
 // The reduced scan of lists up to kRedCl * kRedClNodes nodes on ONE thread-block cluster:
 // node i lives in shared memory of CTA i / NPC (slot i % NPC) and every step reads the
-// target's window through DSMEM.  One CTA's shared memory would hold C2's 3.4 k nodes,
+// target's window through DSMEM.  One CTA's shared memory would hold C2's 5 k nodes,
 // but then every step's random (bank-conflicted) window reads are served by a single SM;
-// sixteen SMs serve them sixteen times faster.  Windows are ping-ponged between two
+// a cluster spreads them over kRedCl SMs (8 and 16 measure the same on C2; 4 is slower).
+// Windows are ping-ponged between two
 // buffers (a step reads buffer b everywhere and writes buffer b^1 of its own nodes), so
 // one cluster barrier per step suffices; finished path nodes are copied forward.
 #ifndef LF_REDCL
