@@ -190,3 +190,43 @@ def run_pipeline(A, n=2, M=5, m=5, k_m=0, p=0.5, seed=0):
         out.update(lf)
         out["a"], out["b"], out["c"] = tridiag(A, lf["forest"], lf["perm"])
     return out
+
+
+def tri_solve(a, b, c, x):
+    """Apply the tridiagonal preconditioner: y = T^{-1} x, fp64.
+
+    T is the tridiagonal matrix lf_tridiag writes (§3.3 step (4), L219, L297),
+    in the permuted order: row r is a[r]*y[r-1] + b[r]*y[r] + c[r]*y[r+1] (a[0] and
+    c[N-1] ignored).  The paper inverts it with the solver of its ref. [21] (L37, L447,
+    "scaled partial pivoting"); the plain definition of that result is T^{-1} x, computed
+    here by LAPACK's banded LU with partial pivoting (scipy.linalg.solve_banded, gbsv) on
+    the whole N x N system in fp64 -- a library primitive as one step, no segmentation.
+    Pinned in tests/test_oracle_trisolve.py by a closed form (1-D Laplacian), a
+    manufactured solution, dense brute force and the block-decoupling invariant.
+    """
+    from scipy.linalg import solve_banded
+
+    a = np.asarray(a, dtype=np.float64)
+    b = np.asarray(b, dtype=np.float64)
+    c = np.asarray(c, dtype=np.float64)
+    x = np.asarray(x, dtype=np.float64)
+    N = b.shape[0]
+    if N == 0:
+        return np.zeros(0)
+    ab = np.zeros((3, N))
+    ab[0, 1:] = c[:-1]   # superdiagonal: T[r, r+1] = c[r]
+    ab[1, :] = b
+    ab[2, :-1] = a[1:]   # subdiagonal:   T[r, r-1] = a[r]
+    return solve_banded((1, 1), ab, x, check_finite=True)
+
+
+def tri_matvec(a, b, c, y):
+    """T y in fp64, the definition of row r above written out (for residual checks)."""
+    a = np.asarray(a, dtype=np.float64)
+    b = np.asarray(b, dtype=np.float64)
+    c = np.asarray(c, dtype=np.float64)
+    y = np.asarray(y, dtype=np.float64)
+    out = b * y
+    out[1:] += a[1:] * y[:-1]
+    out[:-1] += c[:-1] * y[1:]
+    return out
