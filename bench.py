@@ -537,6 +537,37 @@ def main():
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         e2e_t = float(t.item())
 
+    # SURVEY.md §8(f) f2 (next row, not part of the step): apply the preconditioner,
+    # y = T^{-1} x on the step's (a, b, c); L2 flushed before each launch; 20 B/row
+    # algorithmic (read a, b, c, x; write y), DESIGN.md §4.6
+    ta, tb, tc = P.tri
+    xr = torch.randn(N, device="cuda", dtype=torch.float32, generator=torch.Generator("cuda").manual_seed(1))
+    ts_ws, ts_y = lf.Workspace(), torch.empty(N, device="cuda", dtype=torch.float32)
+    for _ in range(3):
+        lf.tri_solve(ta, tb, tc, xr, ws=ts_ws, out=ts_y)
+    ts_ms, ts_k = [], {}
+    for prof in (False, True):
+        for _ in range(max(3, args.steps)):
+            flush.zero_()
+            lf.profile_enable(prof)
+            ev0.record(stream)
+            lf.tri_solve(ta, tb, tc, xr, ws=ts_ws, out=ts_y)
+            ev1.record(stream)
+            ev1.synchronize()
+            if not prof:
+                ts_ms.append(ev0.elapsed_time(ev1))
+                continue
+            for nm, ms in lf.profile_collect():
+                ts_k.setdefault(nm, []).append(ms)
+    lf.profile_enable(False)
+    ts_t = sum(ts_ms) / len(ts_ms)
+    ts_bytes = 20 * N
+    tri_solve_rec = {"ms": round(ts_t, 5), "Mrows_per_s": round(N / (ts_t * 1e-3) / 1e6, 1),
+                     "kernels_ms": {k: round(sum(v) / len(v), 5) for k, v in ts_k.items()},
+                     "roofline": {"bound": "hbm", "alg_bytes": ts_bytes,
+                                  "achieved": round(ts_bytes / (ts_t * 1e-3) / 1e9, 1), "peak": peak,
+                                  "unit": "GB/s", "frac": round(ts_bytes / (ts_t * 1e-3) / 1e9 / peak, 4)}}
+
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(A, args.cpu_runs)
@@ -588,6 +619,7 @@ def main():
                     "d2h_bytes_per_step": int(24 * N)},
             "gpu_launches": launches_per_step,
             "clocks": clk,
+            "next_rows": {"f2_tri_solve": tri_solve_rec},
         }
         if cpu is not None:
             out["cpu_baseline"] = cpu

@@ -329,6 +329,20 @@ static size_t pipe_carve(Carve& c, int64_t N, int64_t nnz, PipeWs* p) {
     return c.off;
 }
 
+size_t lf_tri_solve_workspace_size(int64_t N) { return N > 0 ? trisolve_ws_bytes(N) : 0; }
+
+int lf_tri_solve(int64_t N, const float* a, const float* b, const float* c, const float* x, float* y,
+                 void* ws, size_t ws_bytes, void* stream) {
+    g_err[0] = 0;
+    if (N < 0 || N >= ((int64_t)1 << 31)) return set_error(LF_EINVAL, "lf_tri_solve: bad N");
+    if (N == 0) return LF_OK;
+    if (!a || !b || !c || !x || !y) return set_error(LF_EINVAL, "lf_tri_solve: NULL argument");
+    if (!ws || ws_bytes < trisolve_ws_bytes(N) || ((uintptr_t)ws & 255))
+        return set_error(LF_ENOMEM, "lf_tri_solve: workspace too small or not 256-byte aligned");
+    if (y == x) return set_error(LF_EINVAL, "lf_tri_solve: y must not alias x");
+    return trisolve_run(N, a, b, c, x, y, ws, (cudaStream_t)stream);
+}
+
 size_t lf_pipeline_workspace_size(int64_t N, int64_t nnz) {
     Carve c(nullptr, 0);
     return pipe_carve(c, N, nnz, nullptr) + 256;

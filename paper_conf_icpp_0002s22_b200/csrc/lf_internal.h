@@ -193,6 +193,10 @@ int tridiag_run(int64_t N, const int32_t* forest, const int32_t* iperm, const in
                 const float* pi2_val, const float* diag, float* a, float* b, float* c,
                 cudaStream_t s);
 
+size_t trisolve_ws_bytes(int64_t N);
+int trisolve_run(int64_t N, const float* a, const float* b, const float* c, const float* x,
+                 float* y, void* ws, cudaStream_t s);
+
 // diagnostic timeline (LF_TIMELINE builds): [2 i] first start, [2 i + 1] last exit (ns)
 int timeline_factor(unsigned long long* out, int reset);
 int timeline_forest(unsigned long long* out, int reset);

@@ -1,0 +1,432 @@
+// lf_trisolve.cu -- apply the tridiagonal preconditioner: y = T^{-1} x for the (a, b, c)
+// that lf_tridiag writes (§1 "Tridiagonal systems can be
+// inverted at the bandwidth limit of the GPU [21]", §6).
+//
+// T is block diagonal: row r is uncoupled from row r-1 exactly when a[r] = c[r-1] = 0,
+// which is the case at every path boundary of the linear forest (L219).  Each such
+// segment is an independent tridiagonal system.  Two kernels:
+//   1. k_seg_starts: one thread per row flags segment starts and compacts them into a
+//      list (warp-aggregated atomic; list order is irrelevant to the result).
+//   2. k_seg_solve: one thread per segment runs Gaussian elimination with scaled partial
+//      pivoting (the pivoting strategy of [21]; reading f2-1) streaming down
+//      the segment with the pending row in registers, writes each row of U with its
+//      right-hand side as one float4, then back-substitutes upwards.  fp32 throughout
+//      (the paper's GPU path is fp32).
+// Paths are short compared with N (hundreds of rows on the paper's matrices), so thread
+// per segment exposes O(N / mean path length) independent chains; the U rows written in
+// the forward sweep are re-read in the backward sweep mostly from L1/L2.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "lf_common.cuh"
+#include "lf_internal.h"
+
+namespace lf {
+
+struct TriCtl {
+    unsigned int seq;    // 1: use the sequential pivoting path
+    unsigned int count;  // number of segments (sequential path)
+};
+
+__device__ __forceinline__ bool seg_start(int64_t r, const float* __restrict__ a,
+                                          const float* __restrict__ c) {
+    return r == 0 || (__ldg(a + r) == 0.0f && __ldg(c + r - 1) == 0.0f);
+}
+
+__global__ void __launch_bounds__(256) k_seg_starts(int64_t N, const float* __restrict__ a,
+                                                    const float* __restrict__ c,
+                                                    int32_t* __restrict__ starts,
+                                                    TriCtl* __restrict__ ctl) {
+    if (!ctl->seq) return;
+    unsigned int* count = &ctl->count;
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < N;
+         base += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = base + threadIdx.x;
+        const bool s = r < N && seg_start(r, a, c);
+        const unsigned m = __ballot_sync(0xffffffffu, s);
+        if (m == 0) continue;
+        unsigned slot0 = 0;
+        const int leader = __ffs(m) - 1;
+        if (lane == leader) slot0 = atomicAdd(count, (unsigned)__popc(m));
+        slot0 = __shfl_sync(0xffffffffu, slot0, leader);
+        if (s) starts[slot0 + __popc(m & ((1u << lane) - 1u))] = (int32_t)r;
+    }
+}
+
+__device__ __forceinline__ float row_scale(float l, float d, float u) {
+    return fmaxf(fabsf(l), fmaxf(fabsf(d), fabsf(u)));
+}
+
+__global__ void __launch_bounds__(128) k_seg_solve(int64_t N, const float* __restrict__ a,
+                                                   const float* __restrict__ b,
+                                                   const float* __restrict__ c,
+                                                   const float* __restrict__ x,
+                                                   const int32_t* __restrict__ starts,
+                                                   const TriCtl* __restrict__ ctl,
+                                                   float4* __restrict__ U, float* __restrict__ y) {
+    if (!ctl->seq) return;
+    const unsigned nseg = ctl->count;
+    for (unsigned t = blockIdx.x * blockDim.x + threadIdx.x; t < nseg;
+         t += gridDim.x * blockDim.x) {
+        const int64_t s = starts[t];
+        // pending row i: p*y[i] + q*y[i+1] = rr, scale sc of the original row it came from
+        float p = __ldg(b + s), q = __ldg(c + s), rr = __ldg(x + s);
+        float sc = row_scale(s > 0 ? __ldg(a + s) : 0.0f, p, q);
+        float cprev = q;  // original c[i] (for the segment-end test)
+        int64_t i = s;
+        for (;;) {
+            const int64_t nx = i + 1;
+            if (nx >= N) break;
+            const float l = __ldg(a + nx);
+            if (l == 0.0f && cprev == 0.0f) break;  // nx starts the next segment
+            const float d = __ldg(b + nx), u = __ldg(c + nx), xn = __ldg(x + nx);
+            const float sn = row_scale(l, d, u);
+            if (fabsf(p) * sn >= fabsf(l) * sc) {  // |p|/sc >= |l|/sn: keep row i as pivot
+                U[i] = make_float4(p, q, 0.0f, rr);
+                const float f = l / p;
+                p = fmaf(-f, q, d);
+                q = u;
+                rr = fmaf(-f, rr, xn);
+                sc = sn;
+            } else {  // interchange: row nx is the pivot row of column i
+                U[i] = make_float4(l, d, u, xn);
+                const float f = p / l;
+                p = fmaf(-f, d, q);
+                q = -f * u;
+                rr = fmaf(-f, xn, rr);
+            }
+            cprev = u;
+            i = nx;
+        }
+        // back substitution, rows i (= segment end) .. s
+        float y1 = rr / p, y2 = 0.0f;
+        y[i] = y1;
+        for (int64_t k = i - 1; k >= s; --k) {
+            const float4 w = U[k];
+            const float yk = (w.w - w.y * y1 - w.z * y2) / w.x;
+            y[k] = yk;
+            y2 = y1;
+            y1 = yk;
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------
+// Partition path (diagonally dominant T): fixed chunks of PK rows, one
+// thread per chunk, PB chunks per block staged through shared memory with coalesced loads.
+//   pass 1: each chunk solves T_j z = rhs for rhs = x_j, -a[s] e_1, -c[e] e_K (Thomas,
+//           no pivoting: stable under diagonal dominance) and keeps the first and last
+//           entries of the three solutions: y_j = P + G y[s-1] + H y[e+1].
+//   chain:  one thread per chain of coupled chunks sweeps the 2-unknowns-per-chunk reduced
+//           system (F_j = y[s], L_j = y[e]) forward and back.
+//   pass 2: each chunk re-solves with x[s] -= a[s] L_{j-1}, x[e] -= c[e] F_{j+1}.
+// Pass 1 also checks |b| >= |a| + |c|, b != 0 on every row and a nonzero Thomas pivot; any
+// failure sets ctl->seq and the partition results are overwritten by the pivoting path.
+// ---------------------------------------------------------------------------------------
+constexpr int PK = 32;   // rows per chunk
+constexpr int PB = 64;   // chunks (threads) per block
+constexpr int PS = PK + 1;  // padded smem row stride (conflict-free column walks)
+constexpr unsigned TS_SPLIT = 1, TS_DEC = 2, TS_DECNEXT = 4;
+
+struct ChunkSmem {
+    float a[PB * PS], b[PB * PS], c[PB * PS], x[PB * PS];
+};
+
+// staging of rows [r0, r0 + PB*PK) into the padded [thread][PS] layout: one 4-byte
+// cp.async per element (coalesced across the block, all in flight at once, no registers);
+// a[0] and c[N-1] are ignored (0) and rows past N become identity rows
+__device__ __forceinline__ void cp_async4(float* dst, const float* src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(d), "l"(src) : "memory");
+}
+
+__device__ __forceinline__ void stage_chunks(int64_t N, int64_t r0, const float* __restrict__ a,
+                                             const float* __restrict__ b,
+                                             const float* __restrict__ c,
+                                             const float* __restrict__ x, ChunkSmem& S) {
+    if (r0 + PB * PK <= N) {
+#pragma unroll 8
+        for (int k = threadIdx.x; k < PB * PK; k += PB) {
+            const int o = (k / PK) * PS + (k % PK);
+            cp_async4(S.a + o, a + r0 + k);
+            cp_async4(S.b + o, b + r0 + k);
+            cp_async4(S.c + o, c + r0 + k);
+            cp_async4(S.x + o, x + r0 + k);
+        }
+    } else {
+        for (int k = threadIdx.x; k < PB * PK; k += PB) {
+            const int64_t r = r0 + k;
+            const int o = (k / PK) * PS + (k % PK);
+            if (r < N) {
+                cp_async4(S.a + o, a + r);
+                cp_async4(S.b + o, b + r);
+                cp_async4(S.c + o, c + r);
+                cp_async4(S.x + o, x + r);
+            } else {
+                S.a[o] = 0.0f;
+                S.b[o] = 1.0f;
+                S.c[o] = 0.0f;
+                S.x[o] = 0.0f;
+            }
+        }
+    }
+    asm volatile("cp.async.wait_all;" ::: "memory");
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (r0 == 0) S.a[0] = 0.0f;
+        if (r0 <= N - 1 && N - 1 < r0 + PB * PK) {
+            const int k = (int)(N - 1 - r0);
+            S.c[(k / PK) * PS + (k % PK)] = 0.0f;
+        }
+    }
+}
+
+__global__ void __launch_bounds__(PB) k_part_pass1(int64_t N, const float* __restrict__ a,
+                                                   const float* __restrict__ b,
+                                                   const float* __restrict__ c,
+                                                   const float* __restrict__ x,
+                                                   float4* __restrict__ pg, float4* __restrict__ hh,
+                                                   TriCtl* __restrict__ ctl) {
+    __shared__ ChunkSmem S;
+    const int64_t r0 = (int64_t)blockIdx.x * PB * PK;
+    stage_chunks(N, r0, a, b, c, x, S);
+    __syncthreads();
+    const int64_t j = (int64_t)blockIdx.x * PB + threadIdx.x;
+    if (r0 + (int64_t)threadIdx.x * PK >= N) return;
+    float* A = S.a + threadIdx.x * PS;
+    float* B = S.b + threadIdx.x * PS;
+    float* Cc = S.c + threadIdx.x * PS;
+    float* X = S.x + threadIdx.x * PS;
+    // chain flags (from the original rows, before they are overwritten):
+    //   SPLIT: a[r] = c[r-1] = 0 for some r in (s, e] -- the chunk's head no longer sees
+    //          y[e+1] and its tail no longer sees y[s-1] (G_last = H_first = 0 exactly);
+    //   DEC / DECNEXT: no coupling to the previous / next chunk (or none exists)
+    const int64_t s0 = r0 + (int64_t)threadIdx.x * PK, e0 = s0 + PK - 1;
+    unsigned fl = 0;
+    for (int i = 1; i < PK; ++i)
+        if (A[i] == 0.0f && Cc[i - 1] == 0.0f) fl |= TS_SPLIT;
+    if (s0 == 0 || (A[0] == 0.0f && __ldg(c + s0 - 1) == 0.0f)) fl |= TS_DEC;
+    if (e0 + 1 >= N || (Cc[PK - 1] == 0.0f && __ldg(a + e0 + 1) == 0.0f)) fl |= TS_DECNEXT;
+    bool ok = true;
+    // forward: Cc <- c', X <- d'(x), B <- d'(G); the H rhs is -c[e] e_K: only its last d'
+    float cp = 0.0f, dx = 0.0f, dg = 0.0f;
+    for (int i = 0; i < PK; ++i) {
+        const float ai = A[i], bi = B[i], ci = Cc[i];
+        ok &= (fabsf(bi) >= fabsf(ai) + fabsf(ci)) && bi != 0.0f;
+        const float l = (i == 0) ? 0.0f : ai;  // row 0's a is the coupling to y[s-1]
+        const float m = fmaf(-l, cp, bi);
+        ok &= m != 0.0f;
+        const float gi = (i == 0) ? -ai : 0.0f;
+        dx = fmaf(-l, dx, X[i]) / m;  // correctly rounded: a diagonal T gives x / b exactly
+        dg = fmaf(-l, dg, gi) / m;
+        cp = (i == PK - 1) ? 0.0f : ci / m;  // last row's c is the coupling to y[e+1]
+        Cc[i] = cp;
+        X[i] = dx;
+        B[i] = dg;
+        if (i == PK - 1) A[i] = -ci / m;  // d'(H) at the last row
+    }
+    // back substitution of the three solutions, keeping first and last entries
+    const float pL = X[PK - 1], gL = B[PK - 1], hL = A[PK - 1];
+    float zx = pL, zg = gL, zh = hL;
+    for (int i = PK - 2; i >= 0; --i) {
+        const float cpi = Cc[i];
+        zx = fmaf(-cpi, zx, X[i]);
+        zg = fmaf(-cpi, zg, B[i]);
+        zh = -cpi * zh;
+    }
+    pg[j] = make_float4(zx, zg, pL, gL);  // P_first, G_first, P_last, G_last
+    hh[j] = make_float4(zh, hL, __uint_as_float(fl), 0.0f);  // H_first, H_last, flags
+    ok &= isfinite(zx) && isfinite(zg) && isfinite(zh) && isfinite(pL);
+    if (!ok) atomicOr(&ctl->seq, 1u);
+}
+
+// one thread per chain of coupled chunks: forward sweep over
+//   F_j = pF + gF L_{j-1} + hF F_{j+1},  L_j = pL + gL L_{j-1} + hL F_{j+1}
+// with L_{j-1} = u + v F_j, then back substitution F_j = alpha + beta F_{j+1}.
+// A chain ends at chunk j when F_j no longer depends on F_{j+1} (SPLIT(j): hF = 0, or
+// DECNEXT(j)); the next chain starts at j + 1 with L_j = pL_j + hL_j F_{j+1} (SPLIT, gL
+// = 0) or with nothing (DEC).  Chains are therefore as short as the distance between
+// path boundaries, not between chunk-aligned ones.
+__device__ __forceinline__ unsigned ts_flags(const float4& h) { return __float_as_uint(h.z); }
+
+__global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __restrict__ pg,
+                                                    const float4* __restrict__ hh,
+                                                    float4* __restrict__ sweep,
+                                                    float2* __restrict__ FL,
+                                                    TriCtl* __restrict__ ctl) {
+    if (ctl->seq) return;
+    for (int64_t j0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j0 < NC;
+         j0 += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned f0 = ts_flags(hh[j0]);
+        const bool prev_split = j0 > 0 && (ts_flags(hh[j0 - 1]) & TS_SPLIT);
+        if (!(f0 & TS_DEC) && !prev_split) continue;
+        const bool from_split = !(f0 & TS_DEC);  // L_{j0-1} = pL + hL F_{j0}
+        float u = 0.0f, v = 0.0f;
+        if (from_split) {
+            u = pg[j0 - 1].z;
+            v = hh[j0 - 1].y;
+        }
+        int64_t j = j0;
+        bool ok = true, end_dec = false;
+        // the walk is a dependent chain; the next CB chunks' parameters are loaded as one
+        // batch (independent loads) ahead of their use
+        constexpr int CB = 8;
+        float4 qb[CB], hb[CB];
+        for (bool done = false; !done;) {
+#pragma unroll
+            for (int t = 0; t < CB; ++t) {
+                if (j + t < NC) {
+                    qb[t] = pg[j + t];
+                    hb[t] = hh[j + t];
+                }
+            }
+#pragma unroll
+            for (int t = 0; t < CB; ++t) {
+                const float4 q = qb[t];
+                const float4 h = hb[t];
+                const unsigned f = ts_flags(h);
+                const float den = fmaf(-q.y, v, 1.0f);
+                ok &= den != 0.0f;
+                const float al = fmaf(q.y, u, q.x) / den, be = h.x / den;
+                sweep[j] = make_float4(al, be, u, v);  // u, v: L_{j-1} = u + v F_j
+                const float un = fmaf(q.w, fmaf(v, al, u), q.z);
+                const float vn = fmaf(q.w * v, be, h.y);
+                u = un;
+                v = vn;
+                if (f & (TS_SPLIT | TS_DECNEXT)) {
+                    end_dec = (f & TS_DECNEXT) != 0;
+                    done = true;
+                    break;
+                }
+                ++j;
+            }
+        }
+        // chain end j: F_j = alpha_j (beta_j = 0)
+        float Fn = 0.0f;
+#pragma unroll 4
+        for (int64_t k = j; k >= j0; --k) {
+            const float4 w = sweep[k];
+            const float F = fmaf(w.y, Fn, w.x);
+            FL[k].x = F;
+            if (k > j0 || from_split) FL[k - 1].y = fmaf(w.w, F, w.z);  // L_{k-1} = u + v F_k
+            Fn = F;
+        }
+        // L_j = u + v F_{j+1}: here if nothing follows (v = 0), else by the next chain
+        if (end_dec) FL[j].y = u;
+        ok &= isfinite(Fn) && isfinite(u);
+        if (!ok) atomicOr(&ctl->seq, 1u);
+    }
+}
+
+__global__ void __launch_bounds__(PB) k_part_pass2(int64_t N, int64_t NC,
+                                                   const float* __restrict__ a,
+                                                   const float* __restrict__ b,
+                                                   const float* __restrict__ c,
+                                                   const float* __restrict__ x,
+                                                   const float2* __restrict__ FL,
+                                                   float* __restrict__ y,
+                                                   const TriCtl* __restrict__ ctl) {
+    if (ctl->seq) return;
+    __shared__ ChunkSmem S;
+    const int64_t r0 = (int64_t)blockIdx.x * PB * PK;
+    stage_chunks(N, r0, a, b, c, x, S);
+    __syncthreads();
+    const int64_t j = (int64_t)blockIdx.x * PB + threadIdx.x;
+    if (r0 + (int64_t)threadIdx.x * PK < N) {
+        float* A = S.a + threadIdx.x * PS;
+        float* B = S.b + threadIdx.x * PS;
+        float* Cc = S.c + threadIdx.x * PS;
+        float* X = S.x + threadIdx.x * PS;
+        const float yl = j > 0 ? FL[j - 1].y : 0.0f;
+        const float yr = j + 1 < NC ? FL[j + 1].x : 0.0f;
+        float cp = 0.0f, dx = 0.0f;
+        for (int i = 0; i < PK; ++i) {
+            const float ai = A[i], ci = Cc[i];
+            float xi = X[i];
+            if (i == 0) xi = fmaf(-ai, yl, xi);
+            if (i == PK - 1) xi = fmaf(-ci, yr, xi);
+            const float l = (i == 0) ? 0.0f : ai;
+            const float m = fmaf(-l, cp, B[i]);
+            dx = fmaf(-l, dx, xi) / m;
+            cp = (i == PK - 1) ? 0.0f : ci / m;
+            Cc[i] = cp;
+            X[i] = dx;
+        }
+        float z = dx;
+        for (int i = PK - 2; i >= 0; --i) {
+            z = fmaf(-Cc[i], z, X[i]);
+            X[i] = z;
+        }
+    }
+    __syncthreads();
+    for (int k = threadIdx.x; k < PB * PK; k += PB) {
+        const int64_t r = r0 + k;
+        if (r < N) y[r] = S.x[(k / PK) * PS + (k % PK)];
+    }
+}
+
+static inline size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+static inline int64_t n_chunks(int64_t N) { return (N + PK - 1) / PK; }
+
+size_t trisolve_ws_bytes(int64_t N) {
+    const int64_t NC = n_chunks(N);
+    return 256 + align256((size_t)N * 4) + align256((size_t)N * 16) + align256((size_t)NC * 16) * 3 +
+           align256((size_t)NC * 8);
+}
+
+int trisolve_run(int64_t N, const float* a, const float* b, const float* c, const float* x,
+                 float* y, void* ws, cudaStream_t s) {
+    if (N == 0) return LF_OK;
+    const int64_t NC = n_chunks(N);
+    char* w = (char*)ws;
+    TriCtl* ctl = (TriCtl*)w;
+    w += 256;
+    int32_t* starts = (int32_t*)w;
+    w += align256((size_t)N * 4);
+    float4* U = (float4*)w;
+    w += align256((size_t)N * 16);
+    float4* pg = (float4*)w;
+    w += align256((size_t)NC * 16);
+    float4* sweep = (float4*)w;
+    w += align256((size_t)NC * 16);
+    float4* hh = (float4*)w;
+    w += align256((size_t)NC * 16);
+    float2* FL = (float2*)w;
+    LF_CUDA(cudaMemsetAsync(ctl, 0, sizeof(TriCtl), s));
+    const int pgrid = (int)((NC + PB - 1) / PB);
+    {
+        LF_PROF("trisolve_part1", -1, s);
+        k_part_pass1<<<pgrid, PB, 0, s>>>(N, a, b, c, x, pg, hh, ctl);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("trisolve_chain", -1, s);
+        const int64_t blocks = (NC + 127) / 128;
+        k_part_chain<<<(int)(blocks < 148 * 16 ? blocks : 148 * 16), 128, 0, s>>>(NC, pg, hh, sweep, FL, ctl);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("trisolve_part2", -1, s);
+        k_part_pass2<<<pgrid, PB, 0, s>>>(N, NC, a, b, c, x, FL, y, ctl);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("trisolve_starts", -1, s);
+        k_seg_starts<<<persistent_grid((const void*)k_seg_starts, 256), 256, 0, s>>>(N, a, c, starts, ctl);
+        LF_CUDA(cudaGetLastError());
+    }
+    {
+        LF_PROF("trisolve", -1, s);
+        // a thread per segment (grid-stride; the count is only known on the device)
+        const int64_t blocks = (N + 127) / 128;
+        const int grid = (int)(blocks < 148 * 8 ? blocks : 148 * 8);
+        k_seg_solve<<<grid, 128, 0, s>>>(N, a, b, c, x, starts, ctl, U, y);
+        LF_CUDA(cudaGetLastError());
+    }
+    return LF_OK;
+}
+
+}  // namespace lf

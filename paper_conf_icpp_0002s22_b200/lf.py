@@ -25,6 +25,7 @@ EXPORTS = (
     "lf_forest_stats", "lf_comm_nccl_unique_id", "lf_comm_create_nccl", "lf_comm_create_loopback",
     "lf_comm_destroy", "lf_part_create", "lf_part_destroy", "lf_part_info", "lf_part_factor",
     "lf_part_export", "lf_part_linear_forest", "lf_part_forest_export", "lf_part_tridiag",
+    "lf_tri_solve_workspace_size", "lf_tri_solve",
 )
 
 
@@ -80,6 +81,10 @@ def load(path: str = LIB_PATH):
     L.lf_part_linear_forest.argtypes = [P, I32, P, P]
     L.lf_part_forest_export.argtypes = [P, P, P, P, P, P, P]
     L.lf_part_tridiag.argtypes = [P, I32, P, P, P, P, P]
+    L.lf_tri_solve_workspace_size.argtypes = [I64]
+    L.lf_tri_solve_workspace_size.restype = C.c_size_t
+    L.lf_tri_solve.argtypes = [I64, P, P, P, P, P, P, C.c_size_t, P]
+    L.lf_tri_solve.restype = C.c_int
     L.lf_profile_enable.argtypes = [I32]
     L.lf_profile_collect.argtypes = [P, I32, P, I32]
     L.lf_last_error.restype = C.c_char_p
@@ -268,6 +273,18 @@ class Pipeline:
         self.run_factor()
         self.run_forest()
         return self
+
+
+def tri_solve(a, b, c, x, *, ws=None, out=None):
+    """y = T^{-1} x for the tridiagonal (a, b, c) of lf_tridiag (include/lf.h lf_tri_solve)."""
+    torch = _torch()
+    L = load()
+    N = b.numel()
+    y = out if out is not None else torch.empty(N, dtype=torch.float32, device=b.device)
+    nb = L.lf_tri_solve_workspace_size(N)
+    w = (ws or Workspace()).get(nb) if N > 0 else None
+    _check(L.lf_tri_solve(N, _ptr(a), _ptr(b), _ptr(c), _ptr(x), _ptr(y), _ptr(w), nb, _stream()))
+    return y
 
 
 def pipeline_host(rowptr_h, col_h, val_h, *, M=5, m=5, k_m=0, p=0.5, seed=0, ws=None, outs=None):
