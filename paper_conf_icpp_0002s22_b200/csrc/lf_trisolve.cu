@@ -219,13 +219,14 @@ __global__ void __launch_bounds__(PB) k_part_pass1(int64_t N, const float* __res
         const float m = fmaf(-l, cp, bi);
         ok &= m != 0.0f;
         const float gi = (i == 0) ? -ai : 0.0f;
-        dx = fmaf(-l, dx, X[i]) / m;  // correctly rounded: a diagonal T gives x / b exactly
-        dg = fmaf(-l, dg, gi) / m;
-        cp = (i == PK - 1) ? 0.0f : ci / m;  // last row's c is the coupling to y[e+1]
+        const float rm = __frcp_rn(m);  // one reciprocal per row (<= 1.5 ulp per quotient)
+        dx = fmaf(-l, dx, X[i]) * rm;
+        dg = fmaf(-l, dg, gi) * rm;
+        cp = (i == PK - 1) ? 0.0f : ci * rm;  // last row's c is the coupling to y[e+1]
         Cc[i] = cp;
         X[i] = dx;
         B[i] = dg;
-        if (i == PK - 1) A[i] = -ci / m;  // d'(H) at the last row
+        if (i == PK - 1) A[i] = -ci * rm;  // d'(H) at the last row
     }
     // back substitution of the three solutions, keeping first and last entries
     const float pL = X[PK - 1], gL = B[PK - 1], hL = A[PK - 1];
@@ -289,7 +290,8 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
                 const unsigned f = ts_flags(h);
                 const float den = fmaf(-q.y, v, 1.0f);
                 ok &= den != 0.0f;
-                const float al = fmaf(q.y, u, q.x) / den, be = h.x / den;
+                const float rd = __frcp_rn(den);
+                const float al = fmaf(q.y, u, q.x) * rd, be = h.x * rd;
                 sweep[j] = make_float4(al, be, u, v);  // u, v: L_{j-1} = u + v F_j
                 const float un = fmaf(q.w, fmaf(v, al, u), q.z);
                 const float vn = fmaf(q.w * v, be, h.y);
@@ -348,9 +350,9 @@ __global__ void __launch_bounds__(PB) k_part_pass2(int64_t N, int64_t NC,
             if (i == 0) xi = fmaf(-ai, yl, xi);
             if (i == PK - 1) xi = fmaf(-ci, yr, xi);
             const float l = (i == 0) ? 0.0f : ai;
-            const float m = fmaf(-l, cp, B[i]);
-            dx = fmaf(-l, dx, xi) / m;
-            cp = (i == PK - 1) ? 0.0f : ci / m;
+            const float rm = __frcp_rn(fmaf(-l, cp, B[i]));
+            dx = fmaf(-l, dx, xi) * rm;
+            cp = (i == PK - 1) ? 0.0f : ci * rm;
             Cc[i] = cp;
             X[i] = dx;
         }
