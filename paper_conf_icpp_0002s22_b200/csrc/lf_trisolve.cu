@@ -125,8 +125,14 @@ __global__ void __launch_bounds__(128) k_seg_solve(int64_t N, const float* __res
 // Pass 1 also checks |b| >= |a| + |c|, b != 0 on every row and a nonzero Thomas pivot; any
 // failure sets ctl->seq and the partition results are overwritten by the pivoting path.
 // ---------------------------------------------------------------------------------------
-constexpr int PK = 32;   // rows per chunk
-constexpr int PB = 64;   // chunks (threads) per block
+#ifndef LF_TS_PK
+#define LF_TS_PK 32
+#endif
+#ifndef LF_TS_CB
+#define LF_TS_CB 8
+#endif
+constexpr int PK = LF_TS_PK;  // rows per chunk
+constexpr int PB = 64;        // chunks (threads) per block
 constexpr int PS = PK + 1;  // padded smem row stride (conflict-free column walks)
 constexpr unsigned TS_SPLIT = 1, TS_DEC = 2, TS_DECNEXT = 4;
 
@@ -273,7 +279,7 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
         bool ok = true, end_dec = false;
         // the walk is a dependent chain; the next CB chunks' parameters are loaded as one
         // batch (independent loads) ahead of their use
-        constexpr int CB = 8;
+        constexpr int CB = LF_TS_CB;
         float4 qb[CB], hb[CB];
         for (bool done = false; !done;) {
 #pragma unroll

@@ -23,3 +23,17 @@ y = torch.empty(N, device="cuda")
 for _ in range(3):
     lf.tri_solve(*t, ws=ws, out=y)
 torch.cuda.synchronize()
+
+if len(sys.argv) > 1 and sys.argv[1] == "--time":
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for _ in range(30):
+        flush.zero_()
+        e0.record()
+        lf.tri_solve(*t, ws=ws, out=y)
+        e1.record()
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    ts.sort()
+    print(f"{os.environ.get('LF_LIB_PATH', 'default')}: median {ts[len(ts) // 2] * 1e3:.1f} us, min {ts[0] * 1e3:.1f} us")
