@@ -136,6 +136,14 @@ constexpr int PB = 64;        // chunks (threads) per block
 constexpr int PS = PK + 1;  // padded smem row stride (conflict-free column walks)
 constexpr unsigned TS_SPLIT = 1, TS_DEC = 2, TS_DECNEXT = 4;
 
+// reciprocal without the IEEE slow path: MUFU approximation + one Newton step (about
+// 1 ulp; no branch, two dependent FMAs instead of __frcp_rn's checked sequence)
+__device__ __forceinline__ float rcp_nr(float m) {
+    float r;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(m));
+    return fmaf(r, fmaf(-m, r, 1.0f), r);
+}
+
 struct ChunkSmem {
     float a[PB * PS], b[PB * PS], c[PB * PS], x[PB * PS];
 };
@@ -225,7 +233,7 @@ __global__ void __launch_bounds__(PB) k_part_pass1(int64_t N, const float* __res
         const float m = fmaf(-l, cp, bi);
         ok &= m != 0.0f;
         const float gi = (i == 0) ? -ai : 0.0f;
-        const float rm = __frcp_rn(m);  // one reciprocal per row (<= 1.5 ulp per quotient)
+        const float rm = rcp_nr(m);  // one reciprocal per row
         dx = fmaf(-l, dx, X[i]) * rm;
         dg = fmaf(-l, dg, gi) * rm;
         cp = (i == PK - 1) ? 0.0f : ci * rm;  // last row's c is the coupling to y[e+1]
@@ -280,13 +288,21 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
         // the walk is a dependent chain; the next CB chunks' parameters are loaded as one
         // batch (independent loads) ahead of their use
         constexpr int CB = LF_TS_CB;
-        float4 qb[CB], hb[CB];
+        // (double-buffered: batch k + 1 is in flight while batch k is swept)
+        float4 qb[CB], hb[CB], qn[CB], hn[CB];
+#pragma unroll
+        for (int t = 0; t < CB; ++t) {
+            if (j + t < NC) {
+                qb[t] = pg[j + t];
+                hb[t] = hh[j + t];
+            }
+        }
         for (bool done = false; !done;) {
 #pragma unroll
             for (int t = 0; t < CB; ++t) {
-                if (j + t < NC) {
-                    qb[t] = pg[j + t];
-                    hb[t] = hh[j + t];
+                if (j + CB + t < NC) {
+                    qn[t] = pg[j + CB + t];
+                    hn[t] = hh[j + CB + t];
                 }
             }
 #pragma unroll
@@ -296,7 +312,7 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
                 const unsigned f = ts_flags(h);
                 const float den = fmaf(-q.y, v, 1.0f);
                 ok &= den != 0.0f;
-                const float rd = __frcp_rn(den);
+                const float rd = rcp_nr(den);
                 const float al = fmaf(q.y, u, q.x) * rd, be = h.x * rd;
                 sweep[j] = make_float4(al, be, u, v);  // u, v: L_{j-1} = u + v F_j
                 const float un = fmaf(q.w, fmaf(v, al, u), q.z);
@@ -309,6 +325,11 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
                     break;
                 }
                 ++j;
+            }
+#pragma unroll
+            for (int t = 0; t < CB; ++t) {
+                qb[t] = qn[t];
+                hb[t] = hn[t];
             }
         }
         // chain end j: F_j = alpha_j (beta_j = 0)
@@ -356,7 +377,7 @@ __global__ void __launch_bounds__(PB) k_part_pass2(int64_t N, int64_t NC,
             if (i == 0) xi = fmaf(-ai, yl, xi);
             if (i == PK - 1) xi = fmaf(-ci, yr, xi);
             const float l = (i == 0) ? 0.0f : ai;
-            const float rm = __frcp_rn(fmaf(-l, cp, B[i]));
+            const float rm = rcp_nr(fmaf(-l, cp, B[i]));
             dx = fmaf(-l, dx, xi) * rm;
             cp = (i == PK - 1) ? 0.0f : ci * rm;
             Cc[i] = cp;
