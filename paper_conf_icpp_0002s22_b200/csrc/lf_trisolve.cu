@@ -288,21 +288,13 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
         // the walk is a dependent chain; the next CB chunks' parameters are loaded as one
         // batch (independent loads) ahead of their use
         constexpr int CB = LF_TS_CB;
-        // (double-buffered: batch k + 1 is in flight while batch k is swept)
-        float4 qb[CB], hb[CB], qn[CB], hn[CB];
-#pragma unroll
-        for (int t = 0; t < CB; ++t) {
-            if (j + t < NC) {
-                qb[t] = pg[j + t];
-                hb[t] = hh[j + t];
-            }
-        }
+        float4 qb[CB], hb[CB];
         for (bool done = false; !done;) {
 #pragma unroll
             for (int t = 0; t < CB; ++t) {
-                if (j + CB + t < NC) {
-                    qn[t] = pg[j + CB + t];
-                    hn[t] = hh[j + CB + t];
+                if (j + t < NC) {
+                    qb[t] = pg[j + t];
+                    hb[t] = hh[j + t];
                 }
             }
 #pragma unroll
@@ -325,11 +317,6 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
                     break;
                 }
                 ++j;
-            }
-#pragma unroll
-            for (int t = 0; t < CB; ++t) {
-                qb[t] = qn[t];
-                hb[t] = hn[t];
             }
         }
         // chain end j: F_j = alpha_j (beta_j = 0)
