@@ -224,33 +224,42 @@ __global__ void __launch_bounds__(PB) k_part_pass1(int64_t N, const float* __res
     if (s0 == 0 || (A[0] == 0.0f && __ldg(c + s0 - 1) == 0.0f)) fl |= TS_DEC;
     if (e0 + 1 >= N || (Cc[PK - 1] == 0.0f && __ldg(a + e0 + 1) == 0.0f)) fl |= TS_DECNEXT;
     bool ok = true;
-    // forward: Cc <- c', X <- d'(x), B <- d'(G); the H rhs is -c[e] e_K: only its last d'
-    float cp = 0.0f, dx = 0.0f, dg = 0.0f;
+    // Two eliminations of the same chunk, interleaved (independent chains, no stores):
+    //  - top-down Thomas gives the LAST entries of the three solutions (rhs x, the G rhs
+    //    -a[s] e_1, the H rhs -c[e] e_K);
+    //  - bottom-up Thomas (the mirror: a and c swap roles) gives the FIRST entries.
+    // Row 0's a and row PK-1's c are the couplings and stay out of both eliminations.
+    float cp = 0.0f, dx = 0.0f, dg = 0.0f, mL = 1.0f;   // top-down
+    float cq = 0.0f, ex = 0.0f, eh = 0.0f, m0 = 1.0f;   // bottom-up
+#pragma unroll 8
     for (int i = 0; i < PK; ++i) {
-        const float ai = A[i], bi = B[i], ci = Cc[i];
-        ok &= (fabsf(bi) >= fabsf(ai) + fabsf(ci)) && bi != 0.0f;
-        const float l = (i == 0) ? 0.0f : ai;  // row 0's a is the coupling to y[s-1]
-        const float m = fmaf(-l, cp, bi);
-        ok &= m != 0.0f;
-        const float gi = (i == 0) ? -ai : 0.0f;
-        const float rm = rcp_nr(m);  // one reciprocal per row
-        dx = fmaf(-l, dx, X[i]) * rm;
-        dg = fmaf(-l, dg, gi) * rm;
-        cp = (i == PK - 1) ? 0.0f : ci * rm;  // last row's c is the coupling to y[e+1]
-        Cc[i] = cp;
-        X[i] = dx;
-        B[i] = dg;
-        if (i == PK - 1) A[i] = -ci * rm;  // d'(H) at the last row
+        {  // top-down, row i
+            const float ai = A[i], bi = B[i], ci = Cc[i];
+            ok &= (fabsf(bi) >= fabsf(ai) + fabsf(ci)) && bi != 0.0f;
+            const float l = (i == 0) ? 0.0f : ai;
+            const float m = fmaf(-l, cp, bi);
+            ok &= m != 0.0f;
+            const float rm = rcp_nr(m);
+            dx = fmaf(-l, dx, X[i]) * rm;
+            dg = fmaf(-l, dg, (i == 0) ? -ai : 0.0f) * rm;
+            cp = ci * rm;
+            mL = rm;
+        }
+        {  // bottom-up, row k
+            const int k = PK - 1 - i;
+            const float ak = A[k], bk = B[k], ck = Cc[k];
+            const float u = (k == PK - 1) ? 0.0f : ck;
+            const float m = fmaf(-u, cq, bk);
+            ok &= m != 0.0f;
+            const float rm = rcp_nr(m);
+            ex = fmaf(-u, ex, X[k]) * rm;
+            eh = fmaf(-u, eh, (k == PK - 1) ? -ck : 0.0f) * rm;
+            cq = ak * rm;
+            m0 = rm;
+        }
     }
-    // back substitution of the three solutions, keeping first and last entries
-    const float pL = X[PK - 1], gL = B[PK - 1], hL = A[PK - 1];
-    float zx = pL, zg = gL, zh = hL;
-    for (int i = PK - 2; i >= 0; --i) {
-        const float cpi = Cc[i];
-        zx = fmaf(-cpi, zx, X[i]);
-        zg = fmaf(-cpi, zg, B[i]);
-        zh = -cpi * zh;
-    }
+    const float pL = dx, gL = dg, hL = -Cc[PK - 1] * mL;  // H's last entry: -c[e] / m_last
+    const float zx = ex, zh = eh, zg = -A[0] * m0;          // G's first entry: -a[s] / m'_first
     pg[j] = make_float4(zx, zg, pL, gL);  // P_first, G_first, P_last, G_last
     hh[j] = make_float4(zh, hL, __uint_as_float(fl), 0.0f);  // H_first, H_last, flags
     ok &= isfinite(zx) && isfinite(zg) && isfinite(zh) && isfinite(pL);
