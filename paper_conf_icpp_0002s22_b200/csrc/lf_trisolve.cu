@@ -366,23 +366,44 @@ __global__ void __launch_bounds__(PB) k_part_pass2(int64_t N, int64_t NC,
         float* X = S.x + threadIdx.x * PS;
         const float yl = j > 0 ? FL[j - 1].y : 0.0f;
         const float yr = j + 1 < NC ? FL[j + 1].x : 0.0f;
-        float cp = 0.0f, dx = 0.0f;
-        for (int i = 0; i < PK; ++i) {
-            const float ai = A[i], ci = Cc[i];
-            float xi = X[i];
-            if (i == 0) xi = fmaf(-ai, yl, xi);
-            if (i == PK - 1) xi = fmaf(-ci, yr, xi);
-            const float l = (i == 0) ? 0.0f : ai;
-            const float rm = rcp_nr(fmaf(-l, cp, B[i]));
-            dx = fmaf(-l, dx, xi) * rm;
-            cp = (i == PK - 1) ? 0.0f : ci * rm;
-            Cc[i] = cp;
-            X[i] = dx;
+        // twisted factorisation: top-down over rows [0, H), bottom-up over [H, PK), both
+        // chains interleaved; the two meet in a 2x2 system for y[H-1], y[H], then both
+        // halves back-substitute outwards (serial length PK/2 + PK/2 instead of 2 PK)
+        constexpr int H = PK / 2;
+        const float x0 = fmaf(-A[0], yl, X[0]);
+        const float xe = fmaf(-Cc[PK - 1], yr, X[PK - 1]);
+        float cp = 0.0f, dx = 0.0f, cq = 0.0f, ex = 0.0f;
+#pragma unroll 8
+        for (int i = 0; i < H; ++i) {
+            {
+                const float l = (i == 0) ? 0.0f : A[i];
+                const float rm = rcp_nr(fmaf(-l, cp, B[i]));
+                dx = fmaf(-l, dx, (i == 0) ? x0 : X[i]) * rm;
+                cp = Cc[i] * rm;
+                Cc[i] = cp;
+                X[i] = dx;
+            }
+            {
+                const int k = PK - 1 - i;
+                const float u = (k == PK - 1) ? 0.0f : Cc[k];
+                const float rm = rcp_nr(fmaf(-u, cq, B[k]));
+                ex = fmaf(-u, ex, (k == PK - 1) ? xe : X[k]) * rm;
+                cq = A[k] * rm;
+                A[k] = cq;
+                X[k] = ex;
+            }
         }
-        float z = dx;
-        for (int i = PK - 2; i >= 0; --i) {
-            z = fmaf(-Cc[i], z, X[i]);
-            X[i] = z;
+        // y[H-1] + cp y[H] = dx,  y[H] + cq y[H-1] = ex
+        float zt = (dx - cp * ex) * rcp_nr(fmaf(-cp, cq, 1.0f));
+        float zb = fmaf(-cq, zt, ex);
+        X[H - 1] = zt;
+        X[H] = zb;
+#pragma unroll 8
+        for (int i = 1; i < H; ++i) {
+            zt = fmaf(-Cc[H - 1 - i], zt, X[H - 1 - i]);
+            X[H - 1 - i] = zt;
+            zb = fmaf(-A[H + i], zb, X[H + i]);
+            X[H + i] = zb;
         }
     }
     __syncthreads();
