@@ -148,8 +148,9 @@ struct ChunkSmem {
     float a[PB * PS], b[PB * PS], c[PB * PS], x[PB * PS];
 };
 
-// staging of rows [r0, r0 + PB*PK) into the padded [thread][PS] layout: one 4-byte
-// cp.async per element (coalesced across the block, all in flight at once, no registers);
+// staging of rows [r0, r0 + PB*PK) into the padded [thread][PS] layout: 16-byte loads
+// through registers when the block is full and the arrays are 16-byte aligned, else one
+// 4-byte cp.async per element (coalesced across the block, all in flight at once);
 // a[0] and c[N-1] are ignored (0) and rows past N become identity rows
 __device__ __forceinline__ void cp_async4(float* dst, const float* src) {
     const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
@@ -160,7 +161,36 @@ __device__ __forceinline__ void stage_chunks(int64_t N, int64_t r0, const float*
                                              const float* __restrict__ b,
                                              const float* __restrict__ c,
                                              const float* __restrict__ x, ChunkSmem& S) {
-    if (r0 + PB * PK <= N) {
+    const bool al16 = ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b) |
+                        reinterpret_cast<uintptr_t>(c) | reinterpret_cast<uintptr_t>(x)) & 15) == 0;
+    if (r0 + PB * PK <= N && al16) {
+        // full block, 16-byte aligned arrays: 16-byte loads, all 4 x 8 in flight per thread,
+        // then scalar stores into the padded layout (a float4 never straddles a chunk and
+        // the 32 lanes of a warp hit 32 distinct banks)
+        constexpr int NV = PB * PK / 4 / PB;
+        float4 va[NV], vb[NV], vc[NV], vx[NV];
+        const float4* a4 = reinterpret_cast<const float4*>(a + r0);
+        const float4* b4 = reinterpret_cast<const float4*>(b + r0);
+        const float4* c4 = reinterpret_cast<const float4*>(c + r0);
+        const float4* x4 = reinterpret_cast<const float4*>(x + r0);
+#pragma unroll
+        for (int n = 0; n < NV; ++n) {
+            const int q = threadIdx.x + n * PB;
+            va[n] = __ldg(a4 + q);
+            vb[n] = __ldg(b4 + q);
+            vc[n] = __ldg(c4 + q);
+            vx[n] = __ldg(x4 + q);
+        }
+#pragma unroll
+        for (int n = 0; n < NV; ++n) {
+            const int k = 4 * (threadIdx.x + n * PB);
+            const int o = (k / PK) * PS + (k % PK);
+            S.a[o] = va[n].x, S.a[o + 1] = va[n].y, S.a[o + 2] = va[n].z, S.a[o + 3] = va[n].w;
+            S.b[o] = vb[n].x, S.b[o + 1] = vb[n].y, S.b[o + 2] = vb[n].z, S.b[o + 3] = vb[n].w;
+            S.c[o] = vc[n].x, S.c[o + 1] = vc[n].y, S.c[o + 2] = vc[n].z, S.c[o + 3] = vc[n].w;
+            S.x[o] = vx[n].x, S.x[o + 1] = vx[n].y, S.x[o + 2] = vx[n].z, S.x[o + 3] = vx[n].w;
+        }
+    } else if (r0 + PB * PK <= N) {
 #pragma unroll 8
         for (int k = threadIdx.x; k < PB * PK; k += PB) {
             const int o = (k / PK) * PS + (k % PK);

@@ -181,3 +181,27 @@ def test_dominant_ragged_couplings(torch_cuda, lfm, oracle_mod, N):
     x = rng.standard_normal(N).astype(np.float32)
     y = gpu_solve(torch_cuda, lfm, a, b, c, x)
     check(oracle_mod, a, b, c, x, y)
+
+
+def test_unaligned_inputs(torch_cuda, lfm, oracle_mod):
+    """a, b, c, x as 4-byte-offset views (the staging falls back from 16-byte loads to
+    4-byte copies): same bar as aligned inputs."""
+    torch = torch_cuda
+    N = 50_001
+    rng = np.random.default_rng(21)
+    a = -rng.uniform(0.1, 1, N).astype(np.float32)
+    c = -rng.uniform(0.1, 1, N).astype(np.float32)
+    b = (np.abs(a) + np.abs(c) + rng.uniform(0.01, 0.5, N)).astype(np.float32)
+    cut = np.flatnonzero(rng.random(N) < 0.01)
+    cut = cut[cut > 0]
+    a[cut] = 0.0
+    c[cut - 1] = 0.0
+    x = rng.standard_normal(N).astype(np.float32)
+    views = []
+    for v in (a, b, c, x):
+        buf = torch.empty(N + 1, device="cuda")
+        buf[1:] = torch.from_numpy(v).cuda()
+        views.append(buf[1:])
+    y = lfm.tri_solve(*views)
+    torch.cuda.synchronize()
+    check(oracle_mod, a, b, c, x, y.cpu().numpy())
