@@ -4,17 +4,17 @@
 //
 // T is block diagonal: row r is uncoupled from row r-1 exactly when a[r] = c[r-1] = 0,
 // which is the case at every path boundary of the linear forest (L219).  Each such
-// segment is an independent tridiagonal system.  Two kernels:
-//   1. k_seg_starts: one thread per row flags segment starts and compacts them into a
-//      list (warp-aggregated atomic; list order is irrelevant to the result).
-//   2. k_seg_solve: one thread per segment runs Gaussian elimination with scaled partial
-//      pivoting (the pivoting strategy of [21]; reading f2-1) streaming down
-//      the segment with the pending row in registers, writes each row of U with its
-//      right-hand side as one float4, then back-substitutes upwards.  fp32 throughout
-//      (the paper's GPU path is fp32).
-// Paths are short compared with N (hundreds of rows on the paper's matrices), so thread
-// per segment exposes O(N / mean path length) independent chains; the U rows written in
-// the forward sweep are re-read in the backward sweep mostly from L1/L2.
+// segment is an independent tridiagonal system.  Two paths, both always launched; a
+// device flag (TriCtl::seq, set by the partition path's checks) makes one of them exit:
+//   - partition path (diagonally dominant T; k_part_pass1 / k_part_chain / k_part_pass2,
+//     below): fixed 32-row chunks, a reduced system of two unknowns per chunk swept per
+//     chain of coupled chunks, then one more pass per chunk;
+//   - sequential path (any other T): k_seg_solve, one thread per segment (found by a
+//     grid-stride scan of the rows), Gaussian elimination with scaled partial pivoting
+//     (the pivoting strategy of [21]; reading f2-1) streaming down the segment
+//     with the pending row in registers, U rows with their right-hand side stored as one
+//     float4, then back substitution upwards.
+// fp32 throughout (the paper's GPU path is fp32).
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -26,33 +26,11 @@ namespace lf {
 
 struct TriCtl {
     unsigned int seq;    // 1: use the sequential pivoting path
-    unsigned int count;  // number of segments (sequential path)
 };
 
 __device__ __forceinline__ bool seg_start(int64_t r, const float* __restrict__ a,
                                           const float* __restrict__ c) {
     return r == 0 || (__ldg(a + r) == 0.0f && __ldg(c + r - 1) == 0.0f);
-}
-
-__global__ void __launch_bounds__(256) k_seg_starts(int64_t N, const float* __restrict__ a,
-                                                    const float* __restrict__ c,
-                                                    int32_t* __restrict__ starts,
-                                                    TriCtl* __restrict__ ctl) {
-    if (!ctl->seq) return;
-    unsigned int* count = &ctl->count;
-    const int lane = threadIdx.x & 31;
-    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < N;
-         base += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t r = base + threadIdx.x;
-        const bool s = r < N && seg_start(r, a, c);
-        const unsigned m = __ballot_sync(0xffffffffu, s);
-        if (m == 0) continue;
-        unsigned slot0 = 0;
-        const int leader = __ffs(m) - 1;
-        if (lane == leader) slot0 = atomicAdd(count, (unsigned)__popc(m));
-        slot0 = __shfl_sync(0xffffffffu, slot0, leader);
-        if (s) starts[slot0 + __popc(m & ((1u << lane) - 1u))] = (int32_t)r;
-    }
 }
 
 __device__ __forceinline__ float row_scale(float l, float d, float u) {
@@ -63,14 +41,13 @@ __global__ void __launch_bounds__(128) k_seg_solve(int64_t N, const float* __res
                                                    const float* __restrict__ b,
                                                    const float* __restrict__ c,
                                                    const float* __restrict__ x,
-                                                   const int32_t* __restrict__ starts,
                                                    const TriCtl* __restrict__ ctl,
                                                    float4* __restrict__ U, float* __restrict__ y) {
     if (!ctl->seq) return;
-    const unsigned nseg = ctl->count;
-    for (unsigned t = blockIdx.x * blockDim.x + threadIdx.x; t < nseg;
-         t += gridDim.x * blockDim.x) {
-        const int64_t s = starts[t];
+    // grid-stride over rows; the thread that owns a segment's first row solves it
+    for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < N;
+         s += (int64_t)gridDim.x * blockDim.x) {
+        if (!seg_start(s, a, c)) continue;
         // pending row i: p*y[i] + q*y[i+1] = rr, scale sc of the original row it came from
         float p = __ldg(b + s), q = __ldg(c + s), rr = __ldg(x + s);
         float sc = row_scale(s > 0 ? __ldg(a + s) : 0.0f, p, q);
@@ -449,7 +426,7 @@ static inline int64_t n_chunks(int64_t N) { return (N + PK - 1) / PK; }
 
 size_t trisolve_ws_bytes(int64_t N) {
     const int64_t NC = n_chunks(N);
-    return 256 + align256((size_t)N * 4) + align256((size_t)N * 16) + align256((size_t)NC * 16) * 3 +
+    return 256 + align256((size_t)N * 16) + align256((size_t)NC * 16) * 3 +
            align256((size_t)NC * 8);
 }
 
@@ -460,8 +437,6 @@ int trisolve_run(int64_t N, const float* a, const float* b, const float* c, cons
     char* w = (char*)ws;
     TriCtl* ctl = (TriCtl*)w;
     w += 256;
-    int32_t* starts = (int32_t*)w;
-    w += align256((size_t)N * 4);
     float4* U = (float4*)w;
     w += align256((size_t)N * 16);
     float4* pg = (float4*)w;
@@ -490,16 +465,11 @@ int trisolve_run(int64_t N, const float* a, const float* b, const float* c, cons
         LF_CUDA(cudaGetLastError());
     }
     {
-        LF_PROF("trisolve_starts", -1, s);
-        k_seg_starts<<<persistent_grid((const void*)k_seg_starts, 256), 256, 0, s>>>(N, a, c, starts, ctl);
-        LF_CUDA(cudaGetLastError());
-    }
-    {
         LF_PROF("trisolve", -1, s);
-        // a thread per segment (grid-stride; the count is only known on the device)
+        // a thread per segment, found by a grid-stride scan of the rows
         const int64_t blocks = (N + 127) / 128;
         const int grid = (int)(blocks < 148 * 8 ? blocks : 148 * 8);
-        k_seg_solve<<<grid, 128, 0, s>>>(N, a, b, c, x, starts, ctl, U, y);
+        k_seg_solve<<<grid, 128, 0, s>>>(N, a, b, c, x, ctl, U, y);
         LF_CUDA(cudaGetLastError());
     }
     return LF_OK;
