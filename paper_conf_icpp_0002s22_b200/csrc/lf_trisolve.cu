@@ -43,6 +43,7 @@ __global__ void __launch_bounds__(128) k_seg_solve(int64_t N, const float* __res
                                                    const float* __restrict__ x,
                                                    const TriCtl* __restrict__ ctl,
                                                    float4* __restrict__ U, float* __restrict__ y) {
+    pdl_wait();
     if (!ctl->seq) return;
     // grid-stride over rows; the thread that owns a segment's first row solves it
     for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < N;
@@ -287,6 +288,8 @@ __global__ void __launch_bounds__(128) k_part_chain(int64_t NC, const float4* __
                                                     float4* __restrict__ sweep,
                                                     float2* __restrict__ FL,
                                                     TriCtl* __restrict__ ctl) {
+    pdl_wait();
+    pdl_trigger();  // pass 2 may launch now and stage its (read-only) inputs meanwhile
     if (ctl->seq) return;
     for (int64_t j0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j0 < NC;
          j0 += (int64_t)gridDim.x * blockDim.x) {
@@ -360,11 +363,12 @@ __global__ void __launch_bounds__(PB) k_part_pass2(int64_t N, int64_t NC,
                                                    const float2* __restrict__ FL,
                                                    float* __restrict__ y,
                                                    const TriCtl* __restrict__ ctl) {
-    if (ctl->seq) return;
     __shared__ ChunkSmem S;
     const int64_t r0 = (int64_t)blockIdx.x * PB * PK;
-    stage_chunks(N, r0, a, b, c, x, S);
+    stage_chunks(N, r0, a, b, c, x, S);  // inputs only: overlaps the chain kernel (PDL)
     __syncthreads();
+    pdl_wait();
+    if (ctl->seq) return;
     const int64_t j = (int64_t)blockIdx.x * PB + threadIdx.x;
     if (r0 + (int64_t)threadIdx.x * PK < N) {
         float* A = S.a + threadIdx.x * PS;
@@ -456,12 +460,14 @@ int trisolve_run(int64_t N, const float* a, const float* b, const float* c, cons
     {
         LF_PROF("trisolve_chain", -1, s);
         const int64_t blocks = (NC + 127) / 128;
-        k_part_chain<<<(int)(blocks < 148 * 16 ? blocks : 148 * 16), 128, 0, s>>>(NC, pg, hh, sweep, FL, ctl);
+        LF_CUDA(launch_pdl(k_part_chain, (int)(blocks < 148 * 16 ? blocks : 148 * 16), 128, 0, s, NC,
+                           (const float4*)pg, (const float4*)hh, sweep, FL, ctl));
         LF_CUDA(cudaGetLastError());
     }
     {
         LF_PROF("trisolve_part2", -1, s);
-        k_part_pass2<<<pgrid, PB, 0, s>>>(N, NC, a, b, c, x, FL, y, ctl);
+        LF_CUDA(launch_pdl(k_part_pass2, pgrid, PB, 0, s, N, NC, a, b, c, x, (const float2*)FL, y,
+                           (const TriCtl*)ctl));
         LF_CUDA(cudaGetLastError());
     }
     {
@@ -469,7 +475,7 @@ int trisolve_run(int64_t N, const float* a, const float* b, const float* c, cons
         // a thread per segment, found by a grid-stride scan of the rows
         const int64_t blocks = (N + 127) / 128;
         const int grid = (int)(blocks < 148 * 8 ? blocks : 148 * 8);
-        k_seg_solve<<<grid, 128, 0, s>>>(N, a, b, c, x, ctl, U, y);
+        LF_CUDA(launch_pdl(k_seg_solve, grid, 128, 0, s, N, a, b, c, x, (const TriCtl*)ctl, U, y));
         LF_CUDA(cudaGetLastError());
     }
     return LF_OK;
