@@ -73,6 +73,25 @@ def test_invalid_arguments_rejected_before_launch(lib):
     assert b"aligned" in lib.lf_last_error()
 
 
+def test_tri_solve_arguments_rejected_before_launch(lib):
+    """lf_tri_solve's checks (include/lf.h): bad N, NULL, workspace size/alignment, y == x;
+    N = 0 is a no-op.  None of these reaches the device."""
+    from paper_conf_icpp_0002s22_b200 import lf
+
+    L = lf.load()
+    p = C.c_void_p(0x1000)
+    nb = L.lf_tri_solve_workspace_size(1000)
+    assert nb > 16 * 1000 and L.lf_tri_solve_workspace_size(0) == 0
+    assert L.lf_tri_solve(-1, p, p, p, p, C.c_void_p(0x2000), p, nb, None) == -1
+    assert L.lf_tri_solve(0, None, None, None, None, None, None, 0, None) == 0
+    assert L.lf_tri_solve(1000, None, p, p, p, C.c_void_p(0x2000), p, nb, None) == -1
+    assert b"NULL" in L.lf_last_error()
+    assert L.lf_tri_solve(1000, p, p, p, p, C.c_void_p(0x2000), p, nb - 1, None) == -2
+    assert L.lf_tri_solve(1000, p, p, p, p, C.c_void_p(0x2000), C.c_void_p(0x1010), nb, None) == -2
+    assert L.lf_tri_solve(1000, p, p, p, C.c_void_p(0x3000), C.c_void_p(0x3000), p, nb, None) == -1
+    assert b"alias" in L.lf_last_error()
+
+
 def test_product_package_does_not_import_oracle():
     pkg = os.path.join(ROOT, "paper_conf_icpp_0002s22_b200")
     for dp, _, fs in os.walk(pkg):
