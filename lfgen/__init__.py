@@ -22,6 +22,9 @@ from .graphs import (  # noqa: F401
     chung_lu,
     grid3d_27pt,
     grid3d_27pt_slab_edges,
+    grid3d_27pt_rows,
+    grid3d_27pt_big,
+    grid27_nnz,
     random_graph,
     config,
     CONFIG_NAMES,

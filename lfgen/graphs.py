@@ -34,6 +34,8 @@ class CSR:
     @property
     def n_edges(self) -> int:
         """Undirected off-diagonal edges with nonzero weight (E in SURVEY.md §8)."""
+        if "E_exact" in self.meta:  # closed form of a streamed generator (no O(nnz) temporaries)
+            return int(self.meta["E_exact"])
         rows = np.repeat(np.arange(self.N, dtype=np.int64), np.diff(self.rowptr))
         off = (rows != self.col) & (self.val != 0)
         return int(off.sum()) // 2
@@ -276,6 +278,79 @@ def grid3d_27pt_slab_edges(n, z_lo, z_hi, seed=5):
     s, t, _ = _grid3d_edges(n, n, n, _fwd27(), z_lo, z_hi)
     w = (1.0 - edge_hash_u(s, t, N, seed)).astype(np.float32)
     return s, t, w
+
+
+# the 27 stencil offsets (dx, dy, dz) in ascending column order of a natural-order row
+_OFF27 = [(dx, dy, dz) for dz in (-1, 0, 1) for dy in (-1, 0, 1) for dx in (-1, 0, 1)]
+
+
+def grid27_nnz(n, z_lo=0, z_hi=None, nz=None):
+    """Stored entries (diagonal included) of the planes [z_lo, z_hi) of the n x n x nz
+    27-point graph: every row stores cx*cy*cz entries, c = 3 minus the missing sides."""
+    nz = n if nz is None else nz
+    z_hi = nz if z_hi is None else z_hi
+    s = 3 * n - 2 if n > 1 else 1
+    cz = sum(3 - (z == 0) - (z == nz - 1) if nz > 1 else 1 for z in range(z_lo, z_hi))
+    return s * s * cz
+
+
+def grid3d_27pt_rows(n, z_lo, z_hi, seed=5, nz=None):
+    """Rows of the planes [z_lo, z_hi) of the n x n x nz 27-point graph (the C5 recipe:
+    natural order, w = 1 - u), with GLOBAL column ids: rowptr (rebased), col, val, lo, hi.
+
+    Row by row, the same matrix as grid3d_27pt (tests/test_gen.py checks it at small n):
+    columns ascend because the offsets are visited in (dz, dy, dx) order, and the diagonal
+    is the exact fp64 sum of the row's |w| plus 1 (every w is a multiple of 2^-24, so the
+    sum is exact in any order) rounded to fp32.  Needs only O(rows) memory, so the 512^3
+    graph (3.6e9 entries) can be built slab by slab (grid3d_27pt_big)."""
+    nz = n if nz is None else nz
+    N = n * n * nz
+    plane = n * n
+    lo, hi = z_lo * plane, z_hi * plane
+    v = np.arange(lo, hi, dtype=np.int64)
+    x, y, z = v % n, (v // n) % n, v // plane
+    C = np.empty((v.shape[0], 27), dtype=np.int64)
+    W = np.zeros((v.shape[0], 27), dtype=np.float32)
+    Mk = np.empty((v.shape[0], 27), dtype=bool)
+    for i, (dx, dy, dz) in enumerate(_OFF27):
+        m = ((x + dx >= 0) & (x + dx < n) & (y + dy >= 0) & (y + dy < n)
+             & (z + dz >= 0) & (z + dz < nz))
+        j = v + dx + n * (dy + n * dz)
+        C[:, i] = j
+        Mk[:, i] = m
+        if (dx, dy, dz) != (0, 0, 0):
+            jj = np.where(m, j, v + 1)  # any valid id; masked out below
+            W[:, i] = np.where(m, (1.0 - edge_hash_u(v, jj, N, seed)), 0.0).astype(np.float32)
+    diag = (np.abs(W.astype(np.float64)).sum(1) + 1.0).astype(np.float32)
+    V = -W
+    V[:, 13] = diag  # offset (0, 0, 0)
+    counts = Mk.sum(1).astype(np.int64)
+    rowptr = np.zeros(v.shape[0] + 1, dtype=np.int64)
+    np.cumsum(counts, out=rowptr[1:])
+    return rowptr, C[Mk].astype(np.int32), V[Mk].astype(np.float32), lo, hi
+
+
+def grid3d_27pt_big(n=512, seed=5, planes_per_chunk=2):
+    """The whole n^3 27-point graph (C5) built slab by slab into preallocated arrays
+    (30 GB at n = 512, no temporaries of that size).  Same matrix as grid3d_27pt."""
+    N = n ** 3
+    Z = grid27_nnz(n)
+    rowptr = np.empty(N + 1, dtype=np.int64)
+    col = np.empty(Z, dtype=np.int32)
+    val = np.empty(Z, dtype=np.float32)
+    rowptr[0] = 0
+    e = 0
+    for z0 in range(0, n, planes_per_chunk):
+        z1 = min(n, z0 + planes_per_chunk)
+        rp, c, w, lo, hi = grid3d_27pt_rows(n, z0, z1, seed)
+        rowptr[lo + 1:hi + 1] = rp[1:] + e
+        col[e:e + c.shape[0]] = c
+        val[e:e + c.shape[0]] = w
+        e += c.shape[0]
+    assert e == Z
+    E = (Z - N) // 2
+    return CSR(N=N, rowptr=rowptr, col=col, val=val, name=f"grid3d_27pt_{n}",
+               meta={"seed": seed, "n": n, "E": E, "E_exact": E})
 
 
 def fem27_bricks(n=100, seed=3, dropout=0.02, brick=5, jitter=0.3):

@@ -339,7 +339,16 @@ int lf_tri_solve(int64_t N, const float* a, const float* b, const float* c, cons
     if (!a || !b || !c || !x || !y) return set_error(LF_EINVAL, "lf_tri_solve: NULL argument");
     if (!ws || ws_bytes < trisolve_ws_bytes(N) || ((uintptr_t)ws & 255))
         return set_error(LF_ENOMEM, "lf_tri_solve: workspace too small or not 256-byte aligned");
-    if (y == x) return set_error(LF_EINVAL, "lf_tri_solve: y must not alias x");
+    // y is written while a, b, c, x are still being read (other blocks, other segments):
+    // any overlap of [y, y+N) with one of them is rejected, not just y == x
+    {
+        const uintptr_t y0 = (uintptr_t)y, y1 = y0 + (uintptr_t)N * sizeof(float);
+        const float* ins[4] = {a, b, c, x};
+        for (const float* q : ins) {
+            const uintptr_t q0 = (uintptr_t)q, q1 = q0 + (uintptr_t)N * sizeof(float);
+            if (q0 < y1 && y0 < q1) return set_error(LF_EINVAL, "lf_tri_solve: y overlaps a, b, c or x");
+        }
+    }
     return trisolve_run(N, a, b, c, x, y, ws, (cudaStream_t)stream);
 }
 

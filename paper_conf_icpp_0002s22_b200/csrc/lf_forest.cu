@@ -2533,9 +2533,8 @@ __device__ __forceinline__ int red_full_step(const ForestArgs& a, int cnt, int s
 }
 
 // Grid barrier of k_red_full (monotone arrival counter; `gen` counts the barriers passed).
-// k_red_full runs one CTA per SM with a CTA's worth of shared memory each and is launched
-// after its stream predecessor has completed, while its own successor can only launch
-// once every CTA has triggered (after the last barrier): all its CTAs are co-resident.
+// k_red_full is a cooperative cluster launch (launch_red_full): the runtime guarantees
+// that all its CTAs are co-resident, or fails the launch.
 __device__ __forceinline__ void red_grid_sync(int* ctr, int& gen) {
     __syncthreads();
     gen++;
@@ -2873,11 +2872,13 @@ static int coop_launch(K kernel, int block, ForestArgs& a, cudaStream_t s, size_
     return LF_OK;
 }
 
-// zero the 256-int control block; complete only once the stream predecessor has
+// zero the 256-int control block once the stream predecessor has completed (its CTAs
+// may still be running when this one is scheduled: nothing is written before pdl_wait,
+// since the caller may hand the same workspace to consecutive calls)
 __global__ void k_ctl_zero(int* ctl) {
-    ctl[threadIdx.x] = 0;
     pdl_trigger();
     pdl_wait();
+    ctl[threadIdx.x] = 0;
 }
 
 static int forest_prepare() {
@@ -2911,13 +2912,11 @@ static cudaError_t launch_red_full(const ForestArgs& a, cudaStream_t s) {
     cfg.blockDim = dim3(RT);
     cfg.dynamicSmemBytes = sizeof(RedSmemC);
     cfg.stream = s;
-    cudaLaunchAttribute at[2];
+    cudaLaunchAttribute at[3];
     at[0].id = cudaLaunchAttributeClusterDimension;
     at[0].val.clusterDim.x = kRedCl;
     at[0].val.clusterDim.y = 1;
     at[0].val.clusterDim.z = 1;
-    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    at[1].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     if (nclusters == 0) {
         cudaError_t e = cudaFuncSetAttribute((const void*)k_red_full, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
@@ -2932,7 +2931,13 @@ static cudaError_t launch_red_full(const ForestArgs& a, cudaStream_t s) {
         if (nclusters < 1) nclusters = 1;
     }
     cfg.gridDim = dim3(kRedCl * nclusters);
-    cfg.numAttrs = pdl_enabled() ? 2 : 1;
+    // the grid path's barrier needs every CTA resident: a cooperative launch makes the
+    // runtime guarantee it (or fail the launch) instead of a scheduling argument
+    at[1].id = cudaLaunchAttributeCooperative;
+    at[1].val.cooperative = 1;
+    at[2].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[2].val.programmaticStreamSerializationAllowed = 1;
+    cfg.numAttrs = pdl_enabled() ? 3 : 2;
     return cudaLaunchKernelEx(&cfg, k_red_full, a);
 }
 
@@ -2992,7 +2997,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     {
         LF_PROF("red_scan", -1, s);
 #ifndef LF_NO_GRID_RED  // diagnostics only: measures the launch cost (wrong results)
-        // one CTA per SM (its shared memory admits no second one): see red_grid_sync
+        // cooperative cluster launch (the grid path's barrier): see launch_red_full
         LF_CUDA(launch_red_full(a, s));
 #endif
     }

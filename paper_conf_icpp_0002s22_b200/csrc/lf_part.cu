@@ -284,7 +284,7 @@ __global__ void k_reduce_parts(int P, int M, int** flags, unsigned long long** l
 // ---------------------------------------------------------------------------
 // exchange
 // ---------------------------------------------------------------------------
-static int check_plan(Part* p) {
+static int check_plan(Part* p, cudaStream_t s) {
     // the counts p sends to q must be what q expects from p (symmetric pattern)
     Comm* c = p->comm;
     if (p->plan_checked) return LF_OK;
@@ -306,10 +306,12 @@ static int check_plan(Part* p) {
         std::vector<int64_t> mine(G + 1);
         for (int q = 0; q < G; q++) mine[q] = p->send_cnt[q];
         mine[G] = p->nb;
-        LF_CUDA(cudaMemcpy(dsend, mine.data(), sizeof(int64_t) * (G + 1), cudaMemcpyHostToDevice));
-        LF_NCCL(ncclAllGather(dsend, dall, G + 1, ncclInt64, c->nccl, 0));
+        // on the caller's stream (not the legacy default stream), then one host sync
+        LF_CUDA(cudaMemcpyAsync(dsend, mine.data(), sizeof(int64_t) * (G + 1), cudaMemcpyHostToDevice, s));
+        LF_NCCL(ncclAllGather(dsend, dall, G + 1, ncclInt64, c->nccl, s));
         std::vector<int64_t> all((size_t)(G + 1) * G);
-        LF_CUDA(cudaMemcpy(all.data(), dall, sizeof(int64_t) * all.size(), cudaMemcpyDeviceToHost));
+        LF_CUDA(cudaMemcpyAsync(all.data(), dall, sizeof(int64_t) * all.size(), cudaMemcpyDeviceToHost, s));
+        LF_CUDA(cudaStreamSynchronize(s));
         cudaFree(dsend);
         cudaFree(dall);
         p->peer_send_total.assign(G, 0);
@@ -419,7 +421,7 @@ static int hook_pre_finalize(void* ctx, cudaStream_t s) {
 }
 
 static int run_factor(Part* p, const lf_factor_opts_t* o, cudaStream_t s) {
-    int rc = check_plan(p);
+    int rc = check_plan(p, s);
     if (rc) return rc;
     lf_csr_t A{p->n_own, p->nnz, p->rowptr, p->col_local, p->val};
     PartCtx pc;
@@ -595,7 +597,7 @@ static int lf_setup(Part* p, cudaStream_t s) {
 }
 
 static int run_forest(Part* p, cudaStream_t s) {
-    int rc = check_plan(p);
+    int rc = check_plan(p, s);
     if (rc) return rc;
     rc = lf_setup(p, s);
     if (rc) return rc;

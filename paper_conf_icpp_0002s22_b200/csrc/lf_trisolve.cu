@@ -459,8 +459,8 @@ int trisolve_run(int64_t N, const float* a, const float* b, const float* c, cons
     }
     {
         LF_PROF("trisolve_chain", -1, s);
-        const int64_t blocks = (NC + 127) / 128;
-        LF_CUDA(launch_pdl(k_part_chain, (int)(blocks < 148 * 16 ? blocks : 148 * 16), 128, 0, s, NC,
+        const int64_t blocks = (NC + 127) / 128, cap = (int64_t)sm_count() * 16;
+        LF_CUDA(launch_pdl(k_part_chain, (int)(blocks < cap ? blocks : cap), 128, 0, s, NC,
                            (const float4*)pg, (const float4*)hh, sweep, FL, ctl));
         LF_CUDA(cudaGetLastError());
     }
@@ -473,8 +473,8 @@ int trisolve_run(int64_t N, const float* a, const float* b, const float* c, cons
     {
         LF_PROF("trisolve", -1, s);
         // a thread per segment, found by a grid-stride scan of the rows
-        const int64_t blocks = (N + 127) / 128;
-        const int grid = (int)(blocks < 148 * 8 ? blocks : 148 * 8);
+        const int64_t blocks = (N + 127) / 128, cap = (int64_t)sm_count() * 8;
+        const int grid = (int)(blocks < cap ? blocks : cap);
         LF_CUDA(launch_pdl(k_seg_solve, grid, 128, 0, s, N, a, b, c, x, (const TriCtl*)ctl, U, y));
         LF_CUDA(cudaGetLastError());
     }

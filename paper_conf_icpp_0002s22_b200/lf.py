@@ -281,6 +281,10 @@ def tri_solve(a, b, c, x, *, ws=None, out=None):
     L = load()
     N = b.numel()
     y = out if out is not None else torch.empty(N, dtype=torch.float32, device=b.device)
+    for nm, t in (("a", a), ("b", b), ("c", c), ("x", x), ("out", y)):
+        # raw pointers cross the ABI: a wrong dtype, stride or length would read out of bounds
+        if not (t.is_cuda and t.dtype == torch.float32 and t.is_contiguous() and t.numel() == N):
+            raise LFError(f"tri_solve: {nm} must be a contiguous float32 CUDA tensor of {N} elements")
     nb = L.lf_tri_solve_workspace_size(N)
     w = (ws or Workspace()).get(nb) if N > 0 else None
     _check(L.lf_tri_solve(N, _ptr(a), _ptr(b), _ptr(c), _ptr(x), _ptr(y), _ptr(w), nb, _stream()))

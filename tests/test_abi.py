@@ -74,7 +74,7 @@ def test_invalid_arguments_rejected_before_launch(lib):
 
 
 def test_tri_solve_arguments_rejected_before_launch(lib):
-    """lf_tri_solve's checks (include/lf.h): bad N, NULL, workspace size/alignment, y == x;
+    """lf_tri_solve's checks (include/lf.h): bad N, NULL, workspace size/alignment, y overlapping an input;
     N = 0 is a no-op.  None of these reaches the device."""
     from paper_conf_icpp_0002s22_b200 import lf
 
@@ -89,7 +89,12 @@ def test_tri_solve_arguments_rejected_before_launch(lib):
     assert L.lf_tri_solve(1000, p, p, p, p, C.c_void_p(0x2000), p, nb - 1, None) == -2
     assert L.lf_tri_solve(1000, p, p, p, p, C.c_void_p(0x2000), C.c_void_p(0x1010), nb, None) == -2
     assert L.lf_tri_solve(1000, p, p, p, C.c_void_p(0x3000), C.c_void_p(0x3000), p, nb, None) == -1
-    assert b"alias" in L.lf_last_error()
+    assert b"overlaps" in L.lf_last_error()
+    # partial overlaps (offset views) of y with x, a, b or c are rejected as well
+    A, B, Cc, X = (C.c_void_p(0x10000 * k) for k in (1, 2, 3, 4))
+    for y in (0x40000 + 4 * 999, 0x40000 - 4 * 999, 0x10000 + 8, 0x20000 - 4 * 999 + 4, 0x30000 + 3996):
+        assert L.lf_tri_solve(1000, A, B, Cc, X, C.c_void_p(y), p, nb, None) == -1, hex(y)
+        assert b"overlaps" in L.lf_last_error()
 
 
 def test_product_package_does_not_import_oracle():
