@@ -103,9 +103,12 @@ __device__ __forceinline__ uint32_t charge_bit(uint32_t v, uint32_t k, uint32_t 
 }
 
 // vertex state byte: bits 0..2 = number of confirmed edges (0..4),
-// bit 3 = charge of v in the current round.
+// bit 3 = charge of v in the current round, bit 4 = live (below).
 constexpr uint8_t ST_DEG = 0x7;
 constexpr uint8_t ST_CHARGE = 0x8;
+// bit 4: v is live at the current round's start (deg < n and not retired) -- the rows mode
+// of the rounds streams the rows carrying it (lf_factor.cu k_rounds_rows)
+constexpr uint8_t ST_LIVE = 0x10;
 
 // prop_j slot value for a row whose charge-free candidate set is empty (retired)
 constexpr int32_t PROP_RETIRED = -2;

@@ -732,7 +732,7 @@ __device__ __forceinline__ void mutual_phase(const MutualArgs& a) {
                 uint32_t ch = 0;
                 keep = !retired && deg < NN;
                 if (keep && a.next_charging) ch = charge_bit((uint32_t)(v + a.gid_off), a.next_k, a.seed, a.thr);
-                a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0));
+                a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0) | (keep ? ST_LIVE : 0));
             } else if (a.fresh || nconf > 0) {
                 a.state[v] = (uint8_t)deg;
             }
@@ -862,7 +862,7 @@ __global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
                     keep = pj[b][0] != PROP_RETIRED && deg < NN;
                     if (keep && a.next_charging) ch = charge_bit((uint32_t)(v + a.gid_off), a.next_k, a.seed, a.thr);
                 }
-                a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0));
+                a.state[v] = (uint8_t)(deg | (ch ? ST_CHARGE : 0) | (keep ? ST_LIVE : 0));
             }
             keepb[b] = keep;
         }
@@ -1255,49 +1255,355 @@ __device__ bool rounds_cached(const FusedArgs& f, cg::grid_group& grid) {
 
 static bool cached_rounds_enabled() { return getenv("LF_NO_CACHED_ROUNDS") == nullptr; }
 
-template <int NN, int G>
+// Rounds 1..M-1, step 1: the cached mode (small live sets).  When the round-1 worklist does
+// not fit (or the mode is disabled) the kernel only raises the bail flag, and the rows-mode
+// kernel k_rounds_rows that follows it on the stream runs the rounds instead.
+template <int NN>
 __global__ void __launch_bounds__(LF_FUSED_T) k_rounds_fused(FusedArgs f) {
     LF_TL(g_tl_factor, 3);
-    pdl_trigger();  // k_finalize (one CTA) may launch and wait meanwhile
+    pdl_trigger();  // k_rounds_rows may launch and wait meanwhile
     cg::grid_group grid = cg::this_grid();
     if (f.cached && rounds_cached<NN>(f, grid)) return;
-    for (int k = 1; k < f.M; k++) {
-        ProposeArgs pa = f.pa;
-        pa.wl = f.wl[k & 1];
-        pa.wl_count = &f.counts[k % 3];
-        pa.charging = (k % f.m) != f.k_m;
-        pa.proposed = &f.flags[k];
-        pa.defer_count = &f.long_count[k];
-        pa.defer_len = 32 * G;
-        if (f.live_part) {
-            pa.live_rows = f.live_part + (size_t)k * 128;
-            pa.live_nnz = f.live_part + (size_t)k * 128 + 64;
+    if (!f.cached && blockIdx.x == 0 && threadIdx.x == 0) *f.bail = 1;
+}
+
+// ---------------------------------------------------------------------------
+// Rows mode of rounds 1..M-1 (live sets too large for the cached mode: C2 with n = 1, 3,
+// C3, C4, C5).  The rows still live at a round's start carry ST_LIVE in their state byte
+// (set by the previous mutual phase for exactly the rows the worklist would hold), and
+// every phase streams the rows in natural order, skipping the others after one coalesced
+// state load: neighbouring rows' entries are adjacent in HBM and their targets' state
+// bytes are L2-local, instead of the worklist's scattered order and its extra dependent
+// load.  One cooperative kernel at full occupancy (the cached mode needs one CTA per SM);
+// per round: propose | long rows (a CTA per row) | mutual, separated by grid barriers.
+// Semantics per row are those of propose_phase / mutual_phase (same tests, same order,
+// same keys), so the factor is bit-identical.
+// ---------------------------------------------------------------------------
+struct RowsArgs {
+    int64_t N;
+    const int64_t* __restrict__ rowptr;
+    const int32_t* __restrict__ col;
+    const float* __restrict__ val;
+    uint8_t* __restrict__ state;
+    int32_t* __restrict__ pi;
+    float* __restrict__ pi_w;
+    float* __restrict__ pi_val;
+    int32_t* __restrict__ prop_j;
+    float* __restrict__ prop_v;
+    int* flags;
+    unsigned long long* live_part;   // NULL: no counters
+    int32_t* long_rows;
+    int32_t* long_count;             // [kMaxFlagRounds]
+    int64_t defer_len;
+    int M, m, k_m;
+    uint32_t seed;
+    unsigned long long thr;
+    const int32_t* bail;             // the cached mode's flag: 0 = it already ran the rounds
+    int32_t* rounds;
+    int64_t* live;
+};
+constexpr int kRowsT = 4;  // entries per lane per pass (loads in flight per lane)
+
+// top-NN proposal of one row by the G lanes of a group (lane index li), entries [rs, re):
+// the eligibility tests of propose_phase in its order; returns the merged list in top
+template <int NN, int G>
+__device__ __forceinline__ void row_topn(const RowsArgs& a, int32_t v, int64_t rs, int64_t re, int li,
+                                         const int32_t (&p)[NN], uint32_t cv, bool charging,
+                                         uint64_t (&top)[NN], uint32_t& theta0) {
+#pragma unroll
+    for (int s = 0; s < NN; s++) top[s] = 0;
+    theta0 = 0;
+    for (int64_t b = rs; b < re; b += G * kRowsT) {
+        int32_t j[kRowsT];
+        uint32_t xb[kRowsT];
+#pragma unroll
+        for (int t = 0; t < kRowsT; t++) {
+            const int64_t e = b + li + t * G;
+            const bool in = e < re;
+            j[t] = in ? __ldg(a.col + e) : v;
+            xb[t] = in ? __float_as_uint(__ldg(a.val + e)) : 0u;
         }
-        propose_phase<NN, G>(pa);
+        uint32_t sj[kRowsT];
+#pragma unroll
+        for (int t = 0; t < kRowsT; t++) {
+            const bool edge = j[t] != v && (xb[t] & 0x7FFFFFFFu) != 0u;  // A' = |A| - diag, zeros (L31, L231)
+            sj[t] = edge ? (a.state ? (uint32_t)__ldcg(a.state + j[t]) : 0u) : (uint32_t)NN;
+        }
+#pragma unroll
+        for (int t = 0; t < kRowsT; t++) {
+            if ((int)(sj[t] & ST_DEG) == NN) continue;  // not an edge, or j saturated (L15)
+            bool in_pi = false;
+#pragma unroll
+            for (int s = 0; s < NN; s++) in_pi |= (p[s] == j[t]);
+            if (in_pi) continue;  // L19: W \ pi(v)
+            theta0 = 1;
+            if (charging && (((sj[t] & ST_CHARGE) ? 1u : 0u) == cv)) continue;  // L17
+            topn_insert<NN>(top, ((uint64_t)(xb[t] & 0x7FFFFFFFu) << 32) |
+                                     (((0x7FFFFFFFu - (uint32_t)j[t]) << 1) | (xb[t] >> 31)));
+        }
+    }
+    topn_merge_group<NN, G>(top);
+#pragma unroll
+    for (int off = G / 2; off >= 1; off >>= 1) theta0 |= __shfl_xor_sync(0xffffffffu, theta0, off);
+}
+
+template <int NN>
+__device__ __forceinline__ void write_prop(const RowsArgs& a, int32_t v, int deg, const uint64_t (&top)[NN],
+                                           uint32_t theta0, int& np) {
+    const int need = NN - deg;
+    np = 0;
+#pragma unroll
+    for (int s = 0; s < NN; s++) {
+        const uint64_t tk = s < need ? top[s] : 0ull;
+        a.prop_j[(int64_t)v * NN + s] = tk ? key_col(tk) : ((s == 0 && !theta0) ? PROP_RETIRED : -1);
+        a.prop_v[(int64_t)v * NN + s] = tk ? key_val(tk) : 0.0f;
+        np += tk != 0;
+    }
+}
+
+// propose (Alg. 2 L13-L22) of round k over the live rows, warps over 32-row chunks
+template <int NN, int G>
+__device__ void rows_propose(const RowsArgs& a, int k, bool charging) {
+    constexpr int RPW = 32 / G;
+    const int lane = threadIdx.x & 31, li = lane & (G - 1), grp = lane / G;
+    const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    unsigned long long my_live = 0, my_nnz = 0;
+    int my_prop = 0;
+    for (int64_t c0 = wg * 32; c0 < a.N; c0 += nw * 32) {
+        const int64_t v = c0 + lane;
+        const uint32_t st = v < a.N ? (uint32_t)__ldcg(a.state + v) : 0u;
+        const bool live = (st & ST_LIVE) != 0;
+        int64_t rs = 0, re = 0;
+        if (live) { rs = __ldg(a.rowptr + v); re = __ldg(a.rowptr + v + 1); }
+        const bool lng = live && (re - rs) > a.defer_len;
+        {   // long rows: a CTA per row after the barrier
+            const unsigned m = __ballot_sync(0xffffffffu, lng);
+            if (m) {
+                int base = 0;
+                if (lane == 0) base = atomicAdd(&a.long_count[k], __popc(m));
+                base = __shfl_sync(0xffffffffu, base, 0);
+                if (lng) a.long_rows[base + __popc(m & ((1u << lane) - 1u))] = (int32_t)v;
+            }
+        }
+        unsigned mask = __ballot_sync(0xffffffffu, live && !lng);
+        while (mask) {
+            // group grp takes the grp-th live row left in mask; the lowest RPW are consumed
+            const int cnt = __popc(mask);
+            unsigned m2 = mask;
+            for (int i = 0; i < grp && m2; i++) m2 &= m2 - 1u;
+            const int src = grp < cnt ? __ffs(m2) - 1 : -1;
+            if (cnt > RPW) {
+#pragma unroll
+                for (int i = 0; i < RPW; i++) mask &= mask - 1u;
+            } else {
+                mask = 0;
+            }
+            const int sl = src < 0 ? lane : src;
+            const int32_t vv = (int32_t)(c0 + sl);
+            const uint32_t sv = __shfl_sync(0xffffffffu, st, sl);
+            const int64_t r0 = __shfl_sync(0xffffffffu, rs, sl);
+            const int64_t r1s = __shfl_sync(0xffffffffu, re, sl);  // every lane shuffles
+            const int64_t r1 = src < 0 ? r0 : r1s;
+            const int deg = sv & ST_DEG;
+            const uint32_t cv = (sv & ST_CHARGE) ? 1u : 0u;
+            int32_t p[NN];
+#pragma unroll
+            for (int s = 0; s < NN; s++) p[s] = -1;
+            if (src >= 0 && deg > 0) {
+#pragma unroll
+                for (int s = 0; s < NN; s++) p[s] = __ldcg(a.pi + (int64_t)vv * NN + s);
+            }
+            uint64_t top[NN];
+            uint32_t theta0;
+            row_topn<NN, G>(a, vv, r0, r1, li, p, cv, charging, top, theta0);
+            if (src >= 0 && li == 0) {
+                int np;
+                write_prop<NN>(a, vv, deg, top, theta0, np);
+                if (theta0) { my_live++; my_nnz += (unsigned long long)(r1 - r0); }
+                my_prop |= np > 0;
+            }
+        }
+    }
+#pragma unroll
+    for (int off = 16; off >= 1; off >>= 1) {
+        my_live += __shfl_xor_sync(0xffffffffu, my_live, off);
+        my_nnz += __shfl_xor_sync(0xffffffffu, my_nnz, off);
+        my_prop |= __shfl_xor_sync(0xffffffffu, my_prop, off);
+    }
+    if (lane == 0) {
+        const int slot = (int)(wg & 63);
+        if (a.live_part && my_live) atomicAdd(a.live_part + (size_t)k * 128 + slot, my_live);
+        if (a.live_part && my_nnz) atomicAdd(a.live_part + (size_t)k * 128 + 64 + slot, my_nnz);
+        if (my_prop && *(volatile int*)&a.flags[k] == 0) atomicOr(&a.flags[k], 1);
+    }
+}
+
+// one long row per CTA (hub rows of power-law graphs): the CTA's threads stride the row,
+// warps merge their lists with shuffles, warp 0 merges the warps' lists
+template <int NN>
+__device__ void block_row_topn(const RowsArgs& a, int32_t v, int64_t rs, int64_t re, const int32_t (&p)[NN],
+                               uint32_t cv, bool charging, uint64_t (&top)[NN], uint32_t& theta0) {
+    __shared__ uint64_t wk[32][NN];
+    __shared__ uint32_t wth[32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+    uint64_t t[NN];
+    uint32_t th = 0;
+#pragma unroll
+    for (int s = 0; s < NN; s++) t[s] = 0;
+    for (int64_t b = rs + w * 32 * kRowsT; b < re; b += (int64_t)blockDim.x * kRowsT) {
+        uint64_t tt[NN];
+        uint32_t th2;
+        row_topn<NN, 32>(a, v, b, (b + 32 * kRowsT < re ? b + 32 * kRowsT : re), lane, p, cv, charging, tt, th2);
+        th |= th2;
+#pragma unroll
+        for (int s = 0; s < NN; s++) topn_insert<NN>(t, tt[s]);
+    }
+    if (lane == 0) {
+#pragma unroll
+        for (int s = 0; s < NN; s++) wk[w][s] = t[s];
+        wth[w] = th;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int s = 0; s < NN; s++) top[s] = 0;
+    theta0 = 0;
+    for (int q = 0; q < nwarp; q++) {
+#pragma unroll
+        for (int s = 0; s < NN; s++) topn_insert<NN>(top, wk[q][s]);
+        theta0 |= wth[q];
+    }
+    __syncthreads();  // wk reused by the next row
+}
+
+template <int NN>
+__device__ void rows_long(const RowsArgs& a, int k, bool charging) {
+    const int cnt = *(volatile int32_t*)&a.long_count[k];
+    unsigned long long my_live = 0, my_nnz = 0;
+    int my_prop = 0;
+    for (int i = blockIdx.x; i < cnt; i += gridDim.x) {
+        const int32_t v = __ldcg(a.long_rows + i);
+        const uint32_t sv = __ldcg(a.state + v);
+        const int64_t rs = __ldg(a.rowptr + v), re = __ldg(a.rowptr + v + 1);
+        const int deg = sv & ST_DEG;
+        int32_t p[NN];
+#pragma unroll
+        for (int s = 0; s < NN; s++) p[s] = deg > 0 ? __ldcg(a.pi + (int64_t)v * NN + s) : -1;
+        uint64_t top[NN];
+        uint32_t theta0;
+        block_row_topn<NN>(a, v, rs, re, p, (sv & ST_CHARGE) ? 1u : 0u, charging, top, theta0);
+        if (threadIdx.x == 0) {
+            int np;
+            write_prop<NN>(a, v, deg, top, theta0, np);
+            if (theta0) { my_live++; my_nnz += (unsigned long long)(re - rs); }
+            my_prop |= np > 0;
+        }
+    }
+    if (threadIdx.x == 0) {
+        const int slot = blockIdx.x & 63;
+        if (a.live_part && my_live) atomicAdd(a.live_part + (size_t)k * 128 + slot, my_live);
+        if (a.live_part && my_nnz) atomicAdd(a.live_part + (size_t)k * 128 + 64 + slot, my_nnz);
+        if (my_prop && *(volatile int*)&a.flags[k] == 0) atomicOr(&a.flags[k], 1);
+    }
+}
+
+// mutual (Alg. 2 L26-L28) of round k over the live rows, MB rows per thread in flight
+template <int NN, int MB>
+__device__ void rows_mutual(const RowsArgs& a, int k, bool last) {
+    const int64_t chunk = (int64_t)blockDim.x * MB;
+    const bool next_charging = ((k + 1) % a.m) != a.k_m;
+    for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < a.N; c0 += (int64_t)gridDim.x * chunk) {
+        uint32_t st[MB];
+        int32_t pj[MB][NN], pw[MB][NN][NN];
+#pragma unroll
+        for (int b = 0; b < MB; b++) {
+            const int64_t v = c0 + threadIdx.x + (int64_t)b * blockDim.x;
+            st[b] = v < a.N ? (uint32_t)__ldcg(a.state + v) : 0u;
+#pragma unroll
+            for (int s = 0; s < NN; s++) pj[b][s] = (st[b] & ST_LIVE) ? __ldcg(a.prop_j + v * NN + s) : -1;
+        }
+#pragma unroll
+        for (int b = 0; b < MB; b++)
+#pragma unroll
+            for (int s = 0; s < NN; s++)
+#pragma unroll
+                for (int t = 0; t < NN; t++)
+                    pw[b][s][t] = pj[b][s] >= 0 ? __ldcg(a.prop_j + (int64_t)pj[b][s] * NN + t) : -1;
+#pragma unroll
+        for (int b = 0; b < MB; b++) {
+            if (!(st[b] & ST_LIVE)) continue;
+            const int64_t v = c0 + threadIdx.x + (int64_t)b * blockDim.x;
+            uint64_t conf[NN];
+            int nconf = 0;
+#pragma unroll
+            for (int s = 0; s < NN; s++) {
+                conf[s] = 0;
+                bool mutual = false;
+#pragma unroll
+                for (int t = 0; t < NN; t++) mutual |= (pw[b][s][t] == (int32_t)v);
+                if (pj[b][s] >= 0 && mutual) {
+                    conf[s] = make_key(__ldcg(a.prop_v + v * NN + s), pj[b][s]);
+                    nconf++;
+                }
+            }
+            int deg = st[b] & ST_DEG;
+            if (nconf > 0) {
+                uint64_t t[NN];
+#pragma unroll
+                for (int s = 0; s < NN; s++) {
+                    t[s] = 0;
+                    if (s < deg) {
+                        const int64_t o = v * NN + s;
+                        const uint32_t sg = a.pi_val ? (__float_as_uint(a.pi_val[o]) >> 31) : 0u;
+                        t[s] = make_key_abs(a.pi_w[o], sg, a.pi[o]);
+                    }
+                }
+#pragma unroll
+                for (int s = 0; s < NN; s++)
+                    if (conf[s]) topn_insert<NN>(t, conf[s]);
+#pragma unroll
+                for (int s = 0; s < NN; s++) {
+                    const int64_t o = v * NN + s;
+                    a.pi[o] = t[s] ? key_col(t[s]) : -1;
+                    a.pi_w[o] = t[s] ? key_abs(t[s]) : 0.0f;
+                    if (a.pi_val) a.pi_val[o] = t[s] ? key_val(t[s]) : 0.0f;
+                }
+                deg += nconf;
+            }
+            uint32_t ns = (uint32_t)deg;
+            if (!last) {
+                const bool keep = pj[b][0] != PROP_RETIRED && deg < NN;
+                if (keep) {
+                    ns |= ST_LIVE;
+                    if (next_charging && charge_bit((uint32_t)v, (uint32_t)(k + 1), a.seed, a.thr)) ns |= ST_CHARGE;
+                }
+            }
+            a.state[v] = (uint8_t)ns;
+        }
+    }
+}
+
+#ifndef LF_ROWS_T
+#define LF_ROWS_T 256
+#endif
+template <int NN, int G>
+__global__ void __launch_bounds__(LF_ROWS_T) k_rounds_rows(RowsArgs a) {
+    LF_TL(g_tl_factor, 4);
+    pdl_wait();
+    if (*(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
+    cg::grid_group grid = cg::this_grid();
+    for (int k = 1; k < a.M; k++) {
+        const bool charging = (k % a.m) != a.k_m;
+        const bool last = k == a.M - 1;
+        rows_propose<NN, G>(a, k, charging);
         grid.sync();
-        if (*(volatile int32_t*)pa.defer_count > 0) {
-            ProposeArgs pl = pa;
-            pl.wl = f.long_rows;
-            pl.wl_count = pa.defer_count;
-            pl.defer_len = INT64_MAX;
-            propose_phase<NN, 32>(pl);
+        if (*(volatile int32_t*)&a.long_count[k] > 0) {
+            rows_long<NN>(a, k, charging);
             grid.sync();
         }
-        MutualArgs ma = f.ma;
-        const bool last = k == f.M - 1;
-        // every round's flags and live-row partial sums are final once the last round's
-        // proposals are (the barriers above): finalize here instead of a dependent launch
-        if (last && blockIdx.x == 0 && (f.rounds || f.live))
-            finalize_body(f.flags, f.M, f.m, f.k_m, f.rounds, f.live_part, f.live);
-        ma.wl = f.wl[k & 1];
-        ma.wl_count = &f.counts[k % 3];
-        ma.wl_next = last ? nullptr : f.wl[(k + 1) & 1];
-        ma.wl_next_count = last ? nullptr : &f.counts[(k + 1) % 3];
-        ma.wl_zero = last ? nullptr : &f.counts[(k + 2) % 3];
-        ma.fresh = 0;
-        ma.next_charging = ((k + 1) % f.m) != f.k_m;
-        ma.next_k = (uint32_t)(k + 1);
-        mutual_phase<NN>(ma);
+        if (last && blockIdx.x == 0 && (a.rounds || a.live))
+            finalize_body(a.flags, a.M, a.m, a.k_m, a.rounds, a.live_part, a.live);
+        rows_mutual<NN, 2>(a, k, last);
         if (!last) grid.sync();
     }
 }
@@ -1402,6 +1708,15 @@ static int tile_lanes(double avg) {
     if (avg <= 14) return 2;
     if (avg <= 28) return 4;
     return 8;
+}
+
+// lanes per row of the rows-mode rounds: kRowsT entries per lane cover an average row
+static int rows_lanes(double avg) {
+    if (avg <= 4) return 1;
+    if (avg <= 8) return 2;
+    if (avg <= 16) return 4;
+    if (avg <= 32) return 8;
+    return 16;
 }
 
 static int lanes_per_row(double avg) {
@@ -1616,34 +1931,77 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         f.M = o->M;
         f.m = o->m;
         f.k_m = o->k_m;
-        f.G = G;
         f.rounds = rounds_dev;
         f.live = live;
         f.cached = cached_rounds_enabled() ? 1 : 0;
         f.bail = &w.counts[3];
-        LF_PROF("rounds_fused", -1, s);
-        void* args[] = {&f};
-        const void* kfn;
-        switch (G) {
-            case 2: kfn = (const void*)k_rounds_fused<NN, 2>; break;
-            case 4: kfn = (const void*)k_rounds_fused<NN, 4>; break;
-            case 8: kfn = (const void*)k_rounds_fused<NN, 8>; break;
-            case 16: kfn = (const void*)k_rounds_fused<NN, 16>; break;
-            default: kfn = (const void*)k_rounds_fused<NN, 32>; break;
-        }
-        const size_t smem = f.cached ? cache_smem_bytes<NN>() : 0;
-        if (f.cached) {
-            static bool attr[5] = {false, false, false, false, false};
-            const int gi = G == 2 ? 0 : G == 4 ? 1 : G == 8 ? 2 : G == 16 ? 3 : 4;
-            if (!attr[gi]) {
-                LF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-                attr[gi] = true;
+        {
+            LF_PROF("rounds_fused", -1, s);
+            void* args[] = {&f};
+            const void* kfn = (const void*)k_rounds_fused<NN>;
+            const size_t smem = f.cached ? cache_smem_bytes<NN>() : 0;
+            if (f.cached) {
+                static bool attr = false;
+                if (!attr) {
+                    LF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                    attr = true;
+                }
             }
+            int grid = LF_FUSED_GRID > 0 ? LF_FUSED_GRID : sm_count() * LF_FUSED_GRID_SM;  // fewer CTAs: cheaper barriers
+            const int cap = persistent_grid(kfn, LF_FUSED_T, smem);
+            if (grid > cap) grid = cap;
+            LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, smem, s));
         }
-        int grid = LF_FUSED_GRID > 0 ? LF_FUSED_GRID : sm_count() * LF_FUSED_GRID_SM;  // fewer CTAs: cheaper barriers
-        const int cap = persistent_grid(kfn, LF_FUSED_T, smem);
-        if (grid > cap) grid = cap;
-        LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, smem, s));
+        {
+            LF_PROF("rounds_rows", -1, s);
+            RowsArgs r;
+            memset(&r, 0, sizeof(r));
+            r.N = N;
+            r.rowptr = A->rowptr;
+            r.col = A->col;
+            r.val = A->val;
+            r.state = w.state;
+            r.pi = pi;
+            r.pi_w = pi_w;
+            r.pi_val = pi_val;
+            r.prop_j = w.prop_j;
+            r.prop_v = w.prop_v;
+            r.flags = w.flags;
+            r.live_part = f.live_part;
+            r.long_rows = w.long_rows;
+            r.long_count = w.long_count;
+            r.M = o->M;
+            r.m = o->m;
+            r.k_m = o->k_m;
+            r.seed = o->seed;
+            r.thr = thr;
+            r.bail = f.bail;
+            r.rounds = rounds_dev;
+            r.live = live;
+            const int Gr = rows_lanes(N > 0 ? (double)A->nnz / (double)N : 1.0);
+            r.defer_len = (int64_t)8 * Gr * kRowsT;
+            const void* kfn;
+            switch (Gr) {
+                case 1: kfn = (const void*)k_rounds_rows<NN, 1>; break;
+                case 2: kfn = (const void*)k_rounds_rows<NN, 2>; break;
+                case 4: kfn = (const void*)k_rounds_rows<NN, 4>; break;
+                case 8: kfn = (const void*)k_rounds_rows<NN, 8>; break;
+                default: kfn = (const void*)k_rounds_rows<NN, 16>; break;
+            }
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(persistent_grid(kfn, LF_ROWS_T));
+            cfg.blockDim = dim3(LF_ROWS_T);
+            cfg.stream = s;
+            cudaLaunchAttribute at[2];
+            at[0].id = cudaLaunchAttributeCooperative;
+            at[0].val.cooperative = 1;
+            at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[1].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = pdl_enabled() ? 2 : 1;
+            void* args[] = {&r};
+            LF_CUDA(cudaLaunchKernelExC(&cfg, kfn, args));
+        }
     }
     if (o->until_maximal) {
         if (rounds_dev) {
