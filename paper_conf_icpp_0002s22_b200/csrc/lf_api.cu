@@ -51,8 +51,8 @@ static void record_event(cudaEvent_t e, cudaStream_t s) {
     else cudaEventRecord(e, s);
 }
 
-void prof_begin(const char* name, int k, cudaStream_t s) {
-    if (!g_prof) return;
+int prof_begin(const char* name, int k, cudaStream_t s) {
+    if (!g_prof) return -1;
     std::lock_guard<std::mutex> lk(g_prof_mu);
     const size_t i = g_recs.size();
     if (i >= g_pool.size()) {
@@ -68,12 +68,14 @@ void prof_begin(const char* name, int k, cudaStream_t s) {
     r.b = g_pool[i].second;
     g_recs.push_back(r);
     record_event(r.a, s);
+    return (int)i;
 }
 
-void prof_end(cudaStream_t s) {
-    if (!g_prof) return;
+// closes record `idx` (scopes nest: an outer stage around per-kernel records)
+void prof_end(cudaStream_t s, int idx) {
+    if (!g_prof || idx < 0) return;
     std::lock_guard<std::mutex> lk(g_prof_mu);
-    if (!g_recs.empty()) record_event(g_recs.back().b, s);
+    if ((size_t)idx < g_recs.size()) record_event(g_recs[idx].b, s);
 }
 
 int sm_count() {
@@ -189,6 +191,7 @@ int lf_profile_collect(char* names, int name_stride, float* ms, int cap) {
         if (names && name_stride > 0) snprintf(names + (size_t)n * name_stride, name_stride, "%s", r.name);
         n++;
     }
+    (void)cudaGetLastError();  // an unrecorded event must not leak into a later launch check
     return n;
 }
 

@@ -15,6 +15,7 @@
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
+#include <climits>
 #include <cstdint>
 
 #include "lf_common.cuh"
@@ -1301,6 +1302,10 @@ struct RowsArgs {
     const int32_t* bail;             // the cached mode's flag: 0 = it already ran the rounds
     int32_t* rounds;
     int64_t* live;
+    int only_k, only_phase;          // > 0: run only phase only_phase (0 propose, 1 long rows,
+                                     // 2 mutual) of round only_k (per-phase profiling launches)
+    int32_t* wl[2];                  // worklists: round k's live rows in wl[k & 1] (mutual(k-1)
+    int32_t* counts;                 //   appends them, roughly in id order), sizes counts[k % 3]
 };
 constexpr int kRowsT = 4;  // entries per lane per pass (loads in flight per lane)
 
@@ -1361,70 +1366,191 @@ __device__ __forceinline__ void write_prop(const RowsArgs& a, int32_t v, int deg
     }
 }
 
-// propose (Alg. 2 L13-L22) of round k over the live rows, warps over 32-row chunks
+// propose (Alg. 2 L13-L22) of round k over its worklist (the rows still live, appended by
+// the previous mutual phase roughly in id order), one row per lane.  A warp takes 32
+// worklist entries, loads their state, row extent and confirmed slots (one round trip; the
+// next 32 entries' ids are already in flight) and queues the rows in shared memory; every
+// batch of queued rows whose aligned ranges fit the warp's slice is staged with 16-byte
+// cp.async (all rows in flight), then every entry's target state word is fetched with a
+// 4-byte cp.async (all in flight), then each lane reduces its row from shared memory with
+// the tests of propose_phase and a branch-free top-n network.
+#ifndef LF_ROWS_T
+#define LF_ROWS_T 256
+#endif
+constexpr int kRowsBud = 640;   // staged entries per warp (3 CTAs of 8 warps per SM)
+constexpr int kRowsWarps = LF_ROWS_T / 32;
+struct RowsWarpSmem {
+    int32_t col[kRowsBud];
+    uint32_t val[kRowsBud];
+    uint32_t sjw[kRowsBud];  // the 4-byte state word holding byte col & 3
+    int64_t qrs[64];      // queue of live rows: CSR start
+    int32_t qv[64];       //   vertex
+    int32_t qlen[64];     //   entries
+    int32_t qp[64][4];    //   confirmed slots
+    uint8_t qst[64];      //   state byte
+};
+struct RowsSmem {
+    RowsWarpSmem w[kRowsWarps];
+};
+
+// one batch: the longest prefix of the queue whose aligned ranges fit; returns its size
+template <int NN>
+__device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmem& S, int qcnt, bool charging,
+                                          bool bulk_ok, int64_t nnz, unsigned long long& my_live,
+                                          unsigned long long& my_nnz, int& my_prop) {
+    const int lane = threadIdx.x & 31;
+    const bool has = lane < qcnt;
+    int64_t rs = 0;
+    int len = 0;
+    if (has) { rs = S.qrs[lane]; len = S.qlen[lane]; }
+    const int64_t as = rs & ~(int64_t)3, ae = (rs + len + 3) & ~(int64_t)3;
+    const int plen = has ? (int)(ae - as) : 0;
+    int incl = plen;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += y;
+    }
+    const bool take = has && incl <= kRowsBud;
+    const int nb = __popc(__ballot_sync(0xffffffffu, take));
+    const int boff = incl - plen;
+    const int q0 = boff + (int)(rs - as), q1 = q0 + len;
+    if (take) {  // stage the row (16-byte copies of its aligned range, else per entry)
+        if (bulk_ok && ae <= nnz) {
+            for (int c = 0; c < plen; c += 4) {
+                cp16(&S.col[boff + c], a.col + as + c);
+                cp16(&S.val[boff + c], a.val + as + c);
+            }
+        } else {
+            for (int e = 0; e < len; e++) {
+                cp4(&S.col[q0 + e], a.col + rs + e);
+                cp4(&S.val[q0 + e], a.val + rs + e);
+            }
+        }
+    }
+    cp_commit();
+    cp_wait_all();
+    __syncwarp();
+    if (take) {  // the targets' state words (L15/L17), every entry's copy in flight
+        for (int q = q0; q < q1; q++) cp4(&S.sjw[q], a.state + (S.col[q] & ~3));
+    }
+    cp_commit();
+    cp_wait_all();
+    __syncwarp();
+    if (take) {
+        const int32_t v = S.qv[lane];
+        const uint32_t sv = S.qst[lane];
+        int32_t p[NN];
+#pragma unroll
+        for (int s2 = 0; s2 < NN; s2++) p[s2] = S.qp[lane][s2];
+        const uint32_t cv = (sv & ST_CHARGE) ? 1u : 0u;
+        uint64_t top[NN];
+#pragma unroll
+        for (int s2 = 0; s2 < NN; s2++) top[s2] = 0;
+        uint32_t theta0 = 0;
+        for (int q = q0; q < q1; q++) {
+            const int32_t j = S.col[q];
+            const uint32_t xb = S.val[q];
+            const uint32_t sj = (S.sjw[q] >> (8 * (j & 3))) & 0xffu;
+            bool in_pi = false;
+#pragma unroll
+            for (int s2 = 0; s2 < NN; s2++) in_pi |= (p[s2] == j);
+            // A' = |A| - diag and zeros (L31, L231); j saturated (L15); W \ pi(v) (L19)
+            const bool elig = j != v && (xb & 0x7FFFFFFFu) != 0u && (int)(sj & ST_DEG) != NN && !in_pi;
+            theta0 |= elig ? 1u : 0u;
+            const bool ok = elig && !(charging && (((sj & ST_CHARGE) ? 1u : 0u) == cv));  // L17
+            topn_insert_pred<NN>(top, ((uint64_t)(xb & 0x7FFFFFFFu) << 32) |
+                                          (((0x7FFFFFFFu - (uint32_t)j) << 1) | (xb >> 31)), ok);
+        }
+        int np;
+        write_prop<NN>(a, v, sv & ST_DEG, top, theta0, np);
+        if (theta0) { my_live++; my_nnz += (unsigned long long)len; }
+        my_prop |= np > 0;
+    }
+    __syncwarp();
+    // drop the batch from the queue (slots nb..qcnt-1 move down)
+    int64_t mrs[2];
+    int32_t mv[2], ml[2], mp[2][NN];
+    uint8_t mst[2];
+#pragma unroll
+    for (int h = 0; h < 2; h++) {
+        const int src = nb + lane + 32 * h;
+        if (src < qcnt) {
+            mrs[h] = S.qrs[src]; mv[h] = S.qv[src]; ml[h] = S.qlen[src]; mst[h] = S.qst[src];
+#pragma unroll
+            for (int s2 = 0; s2 < NN; s2++) mp[h][s2] = S.qp[src][s2];
+        }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int h = 0; h < 2; h++) {
+        const int src = nb + lane + 32 * h;
+        if (src < qcnt) {
+            const int d = lane + 32 * h;
+            S.qrs[d] = mrs[h]; S.qv[d] = mv[h]; S.qlen[d] = ml[h]; S.qst[d] = mst[h];
+#pragma unroll
+            for (int s2 = 0; s2 < NN; s2++) S.qp[d][s2] = mp[h][s2];
+        }
+    }
+    __syncwarp();
+    return nb;
+}
+
 template <int NN, int G>
-__device__ void rows_propose(const RowsArgs& a, int k, bool charging) {
-    constexpr int RPW = 32 / G;
-    const int lane = threadIdx.x & 31, li = lane & (G - 1), grp = lane / G;
+__device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool charging, RowsWarpSmem& S) {
+    const int lane = threadIdx.x & 31;
     const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t nnz = __ldg(a.rowptr + a.N);
+    const bool bulk_ok = ((((uintptr_t)a.col) | ((uintptr_t)a.val)) & 15) == 0;
+    const int32_t* __restrict__ wl = a.wl[k & 1];
+    const int64_t cnt = __ldcg(a.counts + k % 3);
     unsigned long long my_live = 0, my_nnz = 0;
     int my_prop = 0;
-    for (int64_t c0 = wg * 32; c0 < a.N; c0 += nw * 32) {
-        const int64_t v = c0 + lane;
-        const uint32_t st = v < a.N ? (uint32_t)__ldcg(a.state + v) : 0u;
-        const bool live = (st & ST_LIVE) != 0;
+    int qcnt = 0;
+    int64_t i0 = wg * 32;
+    int32_t vn = (i0 + lane < cnt) ? __ldcg(wl + i0 + lane) : -1;
+    for (; i0 < cnt; i0 += nw * 32) {
+        const int32_t v = vn;
+        const int64_t i1 = i0 + nw * 32;
+        vn = (i1 + lane < cnt) ? __ldcg(wl + i1 + lane) : -1;  // the next entries, in flight
+        const bool valid = v >= 0;
+        uint32_t st = 0;
         int64_t rs = 0, re = 0;
-        if (live) { rs = __ldg(a.rowptr + v); re = __ldg(a.rowptr + v + 1); }
-        const bool lng = live && (re - rs) > a.defer_len;
+        int32_t p[NN];
+        if (valid) {  // live: deg < n, so pi's unused slots hold -1
+            st = __ldcg(a.state + v);
+            rs = __ldg(a.rowptr + v);
+            re = __ldg(a.rowptr + v + 1);
+#pragma unroll
+            for (int s2 = 0; s2 < NN; s2++) p[s2] = __ldcg(a.pi + (int64_t)v * NN + s2);
+        }
+        const bool lng = valid && (re - rs) > a.defer_len;
         {   // long rows: a CTA per row after the barrier
             const unsigned m = __ballot_sync(0xffffffffu, lng);
             if (m) {
                 int base = 0;
                 if (lane == 0) base = atomicAdd(&a.long_count[k], __popc(m));
                 base = __shfl_sync(0xffffffffu, base, 0);
-                if (lng) a.long_rows[base + __popc(m & ((1u << lane) - 1u))] = (int32_t)v;
+                if (lng) a.long_rows[base + __popc(m & ((1u << lane) - 1u))] = v;
             }
         }
-        unsigned mask = __ballot_sync(0xffffffffu, live && !lng);
-        while (mask) {
-            // group grp takes the grp-th live row left in mask; the lowest RPW are consumed
-            const int cnt = __popc(mask);
-            unsigned m2 = mask;
-            for (int i = 0; i < grp && m2; i++) m2 &= m2 - 1u;
-            const int src = grp < cnt ? __ffs(m2) - 1 : -1;
-            if (cnt > RPW) {
+        const bool enq = valid && !lng;
+        const unsigned m = __ballot_sync(0xffffffffu, enq);
+        if (enq) {
+            const int pos = qcnt + __popc(m & ((1u << lane) - 1u));
+            S.qrs[pos] = rs;
+            S.qv[pos] = v;
+            S.qlen[pos] = (int)(re - rs);
+            S.qst[pos] = (uint8_t)st;
 #pragma unroll
-                for (int i = 0; i < RPW; i++) mask &= mask - 1u;
-            } else {
-                mask = 0;
-            }
-            const int sl = src < 0 ? lane : src;
-            const int32_t vv = (int32_t)(c0 + sl);
-            const uint32_t sv = __shfl_sync(0xffffffffu, st, sl);
-            const int64_t r0 = __shfl_sync(0xffffffffu, rs, sl);
-            const int64_t r1s = __shfl_sync(0xffffffffu, re, sl);  // every lane shuffles
-            const int64_t r1 = src < 0 ? r0 : r1s;
-            const int deg = sv & ST_DEG;
-            const uint32_t cv = (sv & ST_CHARGE) ? 1u : 0u;
-            int32_t p[NN];
-#pragma unroll
-            for (int s = 0; s < NN; s++) p[s] = -1;
-            if (src >= 0 && deg > 0) {
-#pragma unroll
-                for (int s = 0; s < NN; s++) p[s] = __ldcg(a.pi + (int64_t)vv * NN + s);
-            }
-            uint64_t top[NN];
-            uint32_t theta0;
-            row_topn<NN, G>(a, vv, r0, r1, li, p, cv, charging, top, theta0);
-            if (src >= 0 && li == 0) {
-                int np;
-                write_prop<NN>(a, vv, deg, top, theta0, np);
-                if (theta0) { my_live++; my_nnz += (unsigned long long)(r1 - r0); }
-                my_prop |= np > 0;
-            }
+            for (int s2 = 0; s2 < NN; s2++) S.qp[pos][s2] = p[s2];
         }
+        qcnt += __popc(m);
+        __syncwarp();
+        while (qcnt >= 32) qcnt -= rows_batch<NN>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
     }
+    while (qcnt > 0) qcnt -= rows_batch<NN>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
 #pragma unroll
     for (int off = 16; off >= 1; off >>= 1) {
         my_live += __shfl_xor_sync(0xffffffffu, my_live, off);
@@ -1442,7 +1568,7 @@ __device__ void rows_propose(const RowsArgs& a, int k, bool charging) {
 // one long row per CTA (hub rows of power-law graphs): the CTA's threads stride the row,
 // warps merge their lists with shuffles, warp 0 merges the warps' lists
 template <int NN>
-__device__ void block_row_topn(const RowsArgs& a, int32_t v, int64_t rs, int64_t re, const int32_t (&p)[NN],
+__device__ __forceinline__ void block_row_topn(const RowsArgs& a, int32_t v, int64_t rs, int64_t re, const int32_t (&p)[NN],
                                uint32_t cv, bool charging, uint64_t (&top)[NN], uint32_t& theta0) {
     __shared__ uint64_t wk[32][NN];
     __shared__ uint32_t wth[32];
@@ -1477,7 +1603,7 @@ __device__ void block_row_topn(const RowsArgs& a, int32_t v, int64_t rs, int64_t
 }
 
 template <int NN>
-__device__ void rows_long(const RowsArgs& a, int k, bool charging) {
+__device__ __forceinline__ void rows_long(const RowsArgs& a, int k, bool charging) {
     const int cnt = *(volatile int32_t*)&a.long_count[k];
     unsigned long long my_live = 0, my_nnz = 0;
     int my_prop = 0;
@@ -1507,20 +1633,32 @@ __device__ void rows_long(const RowsArgs& a, int k, bool charging) {
     }
 }
 
-// mutual (Alg. 2 L26-L28) of round k over the live rows, MB rows per thread in flight
+// mutual (Alg. 2 L26-L28) of round k over its worklist, MB rows per thread in flight; the
+// rows that stay live are appended to round k+1's worklist (one atomic per warp)
 template <int NN, int MB>
-__device__ void rows_mutual(const RowsArgs& a, int k, bool last) {
+__device__ __forceinline__ void rows_mutual(const RowsArgs& a, int k, bool last) {
     const int64_t chunk = (int64_t)blockDim.x * MB;
     const bool next_charging = ((k + 1) % a.m) != a.k_m;
-    for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < a.N; c0 += (int64_t)gridDim.x * chunk) {
+    const int32_t* __restrict__ wl = a.wl[k & 1];
+    int32_t* wn = a.wl[(k + 1) & 1];
+    int32_t* cn = a.counts + (k + 1) % 3;
+    const int64_t cnt = __ldcg(a.counts + k % 3);
+    if (!last && blockIdx.x == 0 && threadIdx.x == 0) a.counts[(k + 2) % 3] = 0;  // round k+2's appends
+    const int lane = threadIdx.x & 31;
+    for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < cnt; c0 += (int64_t)gridDim.x * chunk) {
+        int32_t vv[MB];
         uint32_t st[MB];
         int32_t pj[MB][NN], pw[MB][NN][NN];
 #pragma unroll
         for (int b = 0; b < MB; b++) {
-            const int64_t v = c0 + threadIdx.x + (int64_t)b * blockDim.x;
-            st[b] = v < a.N ? (uint32_t)__ldcg(a.state + v) : 0u;
+            const int64_t i = c0 + threadIdx.x + (int64_t)b * blockDim.x;
+            vv[b] = i < cnt ? __ldcg(wl + i) : -1;
+        }
 #pragma unroll
-            for (int s = 0; s < NN; s++) pj[b][s] = (st[b] & ST_LIVE) ? __ldcg(a.prop_j + v * NN + s) : -1;
+        for (int b = 0; b < MB; b++) {
+            st[b] = vv[b] >= 0 ? (uint32_t)__ldcg(a.state + vv[b]) : 0u;
+#pragma unroll
+            for (int s = 0; s < NN; s++) pj[b][s] = vv[b] >= 0 ? __ldcg(a.prop_j + (int64_t)vv[b] * NN + s) : -1;
         }
 #pragma unroll
         for (int b = 0; b < MB; b++)
@@ -1529,10 +1667,13 @@ __device__ void rows_mutual(const RowsArgs& a, int k, bool last) {
 #pragma unroll
                 for (int t = 0; t < NN; t++)
                     pw[b][s][t] = pj[b][s] >= 0 ? __ldcg(a.prop_j + (int64_t)pj[b][s] * NN + t) : -1;
+        bool keepb[MB];
 #pragma unroll
         for (int b = 0; b < MB; b++) {
-            if (!(st[b] & ST_LIVE)) continue;
-            const int64_t v = c0 + threadIdx.x + (int64_t)b * blockDim.x;
+            keepb[b] = false;
+            const int32_t v32 = vv[b];
+            if (v32 < 0) continue;
+            const int64_t v = v32;
             uint64_t conf[NN];
             int nconf = 0;
 #pragma unroll
@@ -1540,7 +1681,7 @@ __device__ void rows_mutual(const RowsArgs& a, int k, bool last) {
                 conf[s] = 0;
                 bool mutual = false;
 #pragma unroll
-                for (int t = 0; t < NN; t++) mutual |= (pw[b][s][t] == (int32_t)v);
+                for (int t = 0; t < NN; t++) mutual |= (pw[b][s][t] == v32);
                 if (pj[b][s] >= 0 && mutual) {
                     conf[s] = make_key(__ldcg(a.prop_v + v * NN + s), pj[b][s]);
                     nconf++;
@@ -1572,30 +1713,56 @@ __device__ void rows_mutual(const RowsArgs& a, int k, bool last) {
             }
             uint32_t ns = (uint32_t)deg;
             if (!last) {
-                const bool keep = pj[b][0] != PROP_RETIRED && deg < NN;
-                if (keep) {
+                keepb[b] = pj[b][0] != PROP_RETIRED && deg < NN;
+                if (keepb[b]) {
                     ns |= ST_LIVE;
                     if (next_charging && charge_bit((uint32_t)v, (uint32_t)(k + 1), a.seed, a.thr)) ns |= ST_CHARGE;
                 }
             }
-            a.state[v] = (uint8_t)ns;
+            if (ns != st[b]) a.state[v] = (uint8_t)ns;
+        }
+        if (!last) {  // one worklist atomic per warp for all MB row batches
+            unsigned m[MB];
+            int tot = 0;
+#pragma unroll
+            for (int b = 0; b < MB; b++) { m[b] = __ballot_sync(0xffffffffu, keepb[b]); tot += __popc(m[b]); }
+            int32_t basepos = 0;
+            if (lane == 0 && tot) basepos = atomicAdd(cn, tot);
+            basepos = __shfl_sync(0xffffffffu, basepos, 0);
+#pragma unroll
+            for (int b = 0; b < MB; b++) {
+                if (keepb[b]) wn[basepos + __popc(m[b] & ((1u << lane) - 1u))] = vv[b];
+                basepos += __popc(m[b]);
+            }
         }
     }
 }
 
-#ifndef LF_ROWS_T
-#define LF_ROWS_T 256
-#endif
 template <int NN, int G>
-__global__ void __launch_bounds__(LF_ROWS_T) k_rounds_rows(RowsArgs a) {
+__global__ void __launch_bounds__(LF_ROWS_T, 3) k_rounds_rows(RowsArgs a) {
     LF_TL(g_tl_factor, 4);
+    extern __shared__ __align__(16) unsigned char rows_smem[];
+    RowsWarpSmem& S = reinterpret_cast<RowsSmem*>(rows_smem)->w[threadIdx.x >> 5];
     pdl_wait();
     if (*(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
+    if (a.only_k > 0) {
+        const int k = a.only_k;
+        const bool charging = (k % a.m) != a.k_m;
+        const bool last = k == a.M - 1;
+        if (a.only_phase == 0) rows_propose<NN, G>(a, k, charging, S);
+        if (a.only_phase == 1 && *(volatile int32_t*)&a.long_count[k] > 0) rows_long<NN>(a, k, charging);
+        if (a.only_phase == 2) {
+            if (last && blockIdx.x == 0 && (a.rounds || a.live))
+                finalize_body(a.flags, a.M, a.m, a.k_m, a.rounds, a.live_part, a.live);
+            rows_mutual<NN, 2>(a, k, last);
+        }
+        return;
+    }
     cg::grid_group grid = cg::this_grid();
     for (int k = 1; k < a.M; k++) {
         const bool charging = (k % a.m) != a.k_m;
         const bool last = k == a.M - 1;
-        rows_propose<NN, G>(a, k, charging);
+        rows_propose<NN, G>(a, k, charging, S);
         grid.sync();
         if (*(volatile int32_t*)&a.long_count[k] > 0) {
             rows_long<NN>(a, k, charging);
@@ -1978,8 +2145,11 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             r.bail = f.bail;
             r.rounds = rounds_dev;
             r.live = live;
+            r.wl[0] = w.wl[0];
+            r.wl[1] = w.wl[1];
+            r.counts = w.counts;
             const int Gr = rows_lanes(N > 0 ? (double)A->nnz / (double)N : 1.0);
-            r.defer_len = (int64_t)8 * Gr * kRowsT;
+            r.defer_len = 128;  // longer rows: a CTA per row (and 32 padded rows of <= 24 fit kRowsBud)
             const void* kfn;
             switch (Gr) {
                 case 1: kfn = (const void*)k_rounds_rows<NN, 1>; break;
@@ -1988,9 +2158,19 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
                 case 8: kfn = (const void*)k_rounds_rows<NN, 8>; break;
                 default: kfn = (const void*)k_rounds_rows<NN, 16>; break;
             }
+            const int rsm = (int)sizeof(RowsSmem);
+            {
+                static bool attr[5] = {false, false, false, false, false};
+                const int gi = Gr == 1 ? 0 : Gr == 2 ? 1 : Gr == 4 ? 2 : Gr == 8 ? 3 : 4;
+                if (!attr[gi]) {
+                    LF_CUDA(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, rsm));
+                    attr[gi] = true;
+                }
+            }
             cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3(persistent_grid(kfn, LF_ROWS_T));
+            cfg.gridDim = dim3(persistent_grid(kfn, LF_ROWS_T, rsm));
             cfg.blockDim = dim3(LF_ROWS_T);
+            cfg.dynamicSmemBytes = rsm;
             cfg.stream = s;
             cudaLaunchAttribute at[2];
             at[0].id = cudaLaunchAttributeCooperative;
@@ -2000,7 +2180,18 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             cfg.attrs = at;
             cfg.numAttrs = pdl_enabled() ? 2 : 1;
             void* args[] = {&r};
-            LF_CUDA(cudaLaunchKernelExC(&cfg, kfn, args));
+            if (getenv("LF_ROWS_SPLIT")) {  // diagnostics: one launch per phase, each timed
+                static const char* pn[3] = {"rows_propose", "rows_long", "rows_mutual"};
+                for (int k = 1; k < o->M; k++)
+                    for (int ph = 0; ph < 3; ph++) {
+                        r.only_k = k;
+                        r.only_phase = ph;
+                        LF_PROF(pn[ph], k, s);
+                        LF_CUDA(cudaLaunchKernelExC(&cfg, kfn, args));
+                    }
+            } else {
+                LF_CUDA(cudaLaunchKernelExC(&cfg, kfn, args));
+            }
         }
     }
     if (o->until_maximal) {

@@ -30,6 +30,7 @@
 #include <cub/device/device_scan.cuh>
 #include <cstdint>
 #include <climits>
+#include <cstdlib>
 #include <cstring>
 
 #include "lf_common.cuh"
@@ -40,7 +41,7 @@ namespace cg = cooperative_groups;
 namespace lf {
 
 #ifdef LF_TIMELINE
-__device__ unsigned long long g_tl_forest[16];
+__device__ unsigned long long g_tl_forest[32];
 #endif
 
 constexpr uint64_t KEY_INF = ~0ull;
@@ -915,6 +916,20 @@ struct ForestArgs {
     int2* rdk[2];          // grid-path ping-pong DK
     int32_t* off;          // [N] exclusive tile prefix of path lengths (at path-ID vertices)
     int32_t* tsum;         // [tiles] tile totals -> exclusive prefix (last expand CTA)
+    // global ruling set (k_grs_*): packed records, visit bitmap, splitter-free cycles, and
+    // the permutation / tridiagonal outputs its last walk writes directly
+    int4* grs_rec;
+    int4* grs_erec;        // [N] (signed slot values, diag, 0): the emit walk's per-vertex reads
+    int4* grs_orec;        // [N] at the new index r: (path_id, pos, forest) -> k_grs_out
+    uint32_t* grs_bits;
+    int4* grs_cyc;
+    uint64_t* grs_cyck;
+    int32_t* perm;
+    int32_t* iperm;
+    float *ta, *tb, *tc;
+    const float2* pi2_val;
+    const float* diag;
+    int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
 };
 
 __device__ __forceinline__ bool is_foreign(int64_t x, const ForestArgs& a) { return x < a.lo || x >= a.hi; }
@@ -2852,6 +2867,12 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     t.dk2 = c.take<int2>(n);
     t.rdk[0] = c.take<int2>(n);
     t.rdk[1] = c.take<int2>(n);
+    t.grs_rec = c.take<int4>(n);
+    t.grs_erec = c.take<int4>(n);
+    t.grs_orec = c.take<int4>(n);
+    t.grs_bits = c.take<uint32_t>(n / 32 + 1);
+    t.grs_cyc = c.take<int4>(n / 3 + 1);
+    t.grs_cyck = c.take<uint64_t>(n / 3 + 1);
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
     if (w) *w = t;
@@ -2941,6 +2962,454 @@ static cudaError_t launch_red_full(const ForestArgs& a, cudaStream_t s) {
     return cudaLaunchKernelEx(&cfg, k_red_full, a);
 }
 
+// ===========================================================================
+// Global ruling set (GRS) -- the single-pass window scan without the tile level, for
+// graphs whose paths leave every tile (C5's 27-point snakes: 96% of the vertices are tile
+// boundary vertices, so the reduced graph is nearly the whole graph and pointer jumping
+// over it costs ~20 full passes).  DESIGN.md §4.3a.  Random accesses dominate, so every
+// kernel is organised to touch as few 32-byte sectors per vertex as possible:
+//   1. k_grs_pack: one coalesced pass packs each vertex's factor slots, |w|, signed values
+//      and diagonal into one 32-byte record (one sector per visit later); splitters = path
+//      ends (fewer than two factor neighbours) and a hashed 1/64 of the others, listed in
+//      list1/bidx1 and pre-set in a visit bitmap (L2-resident: N/8 bytes); len := 0.
+//   2. k_grs_walk: from every splitter in each direction, a sequential walk through the
+//      non-splitters to the next splitter folds the full window (R, K, DK) of the segment:
+//      the reduced records (cq, cq_r, cq_k, cq_dk) of the splitter list; walked vertices are
+//      marked in the bitmap.
+//   3. k_red_full on the splitter list (the reduced scan of the tile path, unchanged).
+//   4. k_grs_len: every splitter knows its path's ends and length, or its cycle's weakest
+//      edge (K, DK both ways, L = p_f + p_b + 1): the path length at the path-ID vertex.
+//      k_grs_cycfind: vertices left unmarked lie on cycles without a splitter; the
+//      lowest-priority vertex of each walks it and records it.
+//   5. k_grs_lenscan + k_tile_prefix: the exclusive prefix of the path lengths in id order.
+//   6. k_grs_emit: every segment is walked once more (by its smaller-id splitter; the
+//      splitter-free cycles by their recorded vertex).  A vertex at distance d from the
+//      splitter derives path id, position, forest slots from d and the splitter's final
+//      windows (paths: both ends; cycles: the weakest edge ahead / behind); its new index
+//      r = prefix(l) + p - 1 is consecutive along the walk, so perm, a, b, c are written
+//      sequentially, and only iperm, path_id, pos, forest are scattered.
+// Every output equals the tile path's (and the oracle's) bit for bit: the windows fold the
+// same edge keys in the same walk order, and the readings c9/c11/c12/c14/c15 are applied by
+// the same cycle_finish / path rules as k_lf_full2 / k_perm_tri.
+// ===========================================================================
+#ifndef LF_GRS_SHIFT
+#define LF_GRS_SHIFT 24  // hashed splitter density 2^-(32 - 24) = 1/256 (C5: 1/16..1/256 measured, sparse wins)
+#endif
+constexpr int kGrsShift = LF_GRS_SHIFT;
+constexpr int kCtlCyc = 134;      // splitter-free cycles recorded by k_grs_cycfind
+
+__device__ __forceinline__ bool grs_splitter(const ForestArgs& a, int32_t v, int2 nb) {
+    return nb.x < 0 || nb.y < 0 || (((uint32_t)v * 0x9E3779B1u) >> a.grs_shift) == 0u;
+}
+// what a walk reads per vertex: slots and |w| (one 16-byte packed record, or the two arrays)
+__device__ __forceinline__ void grs_load(const ForestArgs& a, int32_t v, int2& nb, float2& w) {
+    if (a.grs_rec) {
+        const int4 r = __ldg(a.grs_rec + v);
+        nb = make_int2(r.x, r.y);
+        w = make_float2(__int_as_float(r.z), __int_as_float(r.w));
+    } else {
+        nb = __ldg(a.pi2 + v);
+        w = __ldg(a.pi2_w + v);
+    }
+}
+
+__global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
+    LF_TL(g_tl_forest, 5);
+    pdl_wait();
+    pdl_trigger();
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t b = (int64_t)blockIdx.x * blockDim.x; b < a.N; b += stride) {  // warp-uniform
+        const int64_t v = b + threadIdx.x;
+        const bool in = v < a.N;
+        int2 nb = make_int2(0, 0);
+        float2 w = make_float2(0.f, 0.f);
+        if (in) {
+            nb = __ldg(a.pi2 + v);
+            if (a.grs_rec) w = __ldg(a.pi2_w + v);
+        }
+        const bool spl = in && grs_splitter(a, (int32_t)v, nb);
+        const int p = list_append(a.list1, &a.ctl[kCtlCnt1], (int32_t)v, spl);
+        const unsigned m = __ballot_sync(0xffffffffu, spl);
+        if (in) {
+            a.bidx1[v] = p;
+            a.len[v] = 0;
+            if (a.grs_rec) a.grs_rec[v] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
+            if (a.ta) {
+                const float2 pv = __ldg(a.pi2_val + v);
+                a.grs_erec[v] = make_int4(__float_as_int(pv.x), __float_as_int(pv.y), __float_as_int(__ldg(a.diag + v)), 0);
+            }
+            if ((threadIdx.x & 31) == 0) a.grs_bits[v >> 5] = m;  // b is a multiple of 32
+        }
+    }
+}
+
+// one (splitter, direction) per thread: the segment's full window and the next splitter
+__global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
+    LF_TL(g_tl_forest, 6);
+    pdl_wait();
+    pdl_trigger();
+    const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
+    const int stride = gridDim.x * blockDim.x;
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt; t += stride) {
+        const int i = t >> 1, f = t & 1;
+        const int32_t sv = __ldcg(a.list1 + i);
+        int2 nbs;
+        float2 ws;
+        grs_load(a, sv, nbs, ws);
+        const int32_t x = f ? nbs.y : nbs.x;
+        int32_t tgt, R = 0, DK = 0;
+        uint64_t K = KEY_INF;
+        if (x < 0) {
+            tgt = -(sv + 1);  // a path end: marker
+        } else {
+            int32_t prev = sv, cur = x;
+            int2 nbc;
+            float2 wc;
+            grs_load(a, cur, nbc, wc);
+            K = edge_key(sv, cur, f ? ws.y : ws.x, sv < cur ? nbs : nbc);
+            DK = sv < cur ? 1 : 0;
+            R = 1;
+            while (!grs_splitter(a, cur, nbc)) {
+                const int fs = nbc.x == prev ? 1 : 0;  // the slot away from prev
+                const int32_t nxt = fs ? nbc.y : nbc.x;
+                // each interior vertex is walked from both ends: the walker with prev < nxt marks it
+                if (prev < nxt) atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
+                const float wn = fs ? wc.y : wc.x;
+                int2 nbn;
+                float2 wnx;
+                grs_load(a, nxt, nbn, wnx);
+                const uint64_t k = edge_key(cur, nxt, wn, cur < nxt ? nbc : nbn);
+                if (k < K) { K = k; DK = 2 * R + (cur < nxt ? 1 : 0); }
+                R++;
+                prev = cur;
+                cur = nxt;
+                nbc = nbn;
+                wc = wnx;
+            }
+            tgt = cur;
+        }
+        int32_t* q = reinterpret_cast<int32_t*>(a.cq + i);
+        int32_t* r = reinterpret_cast<int32_t*>(a.cq_r + i);
+        int32_t* d = reinterpret_cast<int32_t*>(a.cq_dk + i);
+        uint64_t* k = reinterpret_cast<uint64_t*>(a.cq_k + i);
+        q[f] = tgt;
+        r[f] = R;
+        d[f] = DK;
+        k[f] = K;
+    }
+}
+
+// a splitter's final windows oriented along its direction f (forward) and 1 - f (backward)
+struct GrsWin {
+    bool cyc;
+    int32_t Ef, Eb;   // path: end vertices ahead / behind
+    int32_t Rf, Rb;   // path: distances from s to them
+    uint64_t ks;      // cycle: weakest key
+    int32_t pf, pb;   // cycle: distance from s to the weakest edge's near endpoint, ahead / behind
+    int32_t bf, bb;   //        and whether that endpoint is the edge's min-id end
+};
+
+__device__ __forceinline__ GrsWin grs_window(const ForestArgs& a, int i, int f) {
+    const int2 e2 = __ldcg(a.end2 + i), d2 = __ldcg(a.dist2 + i), dk = __ldcg(a.dk2 + i);
+    GrsWin W;
+    W.cyc = !(e2.x < 0 && e2.y < 0);
+    const int32_t ef = f ? e2.y : e2.x, eb = f ? e2.x : e2.y;
+    W.Ef = -(ef + 1);
+    W.Eb = -(eb + 1);
+    W.Rf = f ? d2.y : d2.x;
+    W.Rb = f ? d2.x : d2.y;
+    W.ks = __ldcg(&a.kraw[i].x);
+    const int32_t dkf = f ? dk.y : dk.x, dkb = f ? dk.x : dk.y;
+    W.pf = dkf >> 1;
+    W.bf = dkf & 1;
+    W.pb = dkb >> 1;
+    W.bb = dkb & 1;
+    return W;
+}
+
+// path id of the walk of a splitter (constant along it) and its length
+__device__ __forceinline__ int32_t grs_path_id(const GrsWin& W, int32_t& L) {
+    if (W.cyc) {
+        L = W.pf + W.pb + 1;
+        return key_min_end(W.ks);
+    }
+    L = W.Rf + W.Rb + 1;
+    return W.Eb < W.Ef ? W.Eb : W.Ef;
+}
+
+// results of a vertex at forward distance d from the splitter (d = 0: the splitter)
+struct GrsOut {
+    int32_t l, p;
+    int2 f;
+    int dir, rs;      // slot toward the path-id end; removed slot (-1: none)
+    int ncyc;
+};
+
+__device__ __forceinline__ GrsOut grs_vertex(int32_t x, int2 nb, int fslot, int32_t d, const GrsWin& W) {
+    const int bslot = fslot ^ 1;
+    GrsOut o;
+    o.ncyc = 0;
+    o.rs = -1;
+    o.f = nb;
+    if (!W.cyc) {
+        const int32_t Df = W.Rf - d, Db = W.Rb + d;
+        // the smaller end is the path id (reading c11); equal ends: a single vertex (slot 0)
+        if (W.Eb < W.Ef || (W.Eb == W.Ef && bslot == 0)) { o.dir = bslot; o.l = W.Eb; o.p = Db + 1; }
+        else { o.dir = fslot; o.l = W.Ef; o.p = Df + 1; }
+        return o;
+    }
+    const int32_t L = W.pf + W.pb + 1;
+    int32_t dkf, dkb;
+    if (d <= W.pf) { dkf = 2 * (W.pf - d) + W.bf; dkb = 2 * (d + W.pb) + W.bb; }
+    else { dkf = 2 * (L - d + W.pf) + W.bf; dkb = 2 * (d - W.pf - 1) + W.bb; }
+    // the weakest edge is the forward one (x its near endpoint) or the backward one
+    // (x its far endpoint; for d = 0 the edge closing the cycle behind s)
+    const bool remf = d == W.pf, remb = d == W.pf + 1 || (d == 0 && W.pb == 0);
+    int2 c;
+    ulonglong2 ek;
+    if (fslot == 0) { c = make_int2(dkf, dkb); ek = make_ulonglong2(remf ? W.ks : 0ull, remb ? W.ks : 0ull); }
+    else { c = make_int2(dkb, dkf); ek = make_ulonglong2(remb ? W.ks : 0ull, remf ? W.ks : 0ull); }
+    const CycOut co = cycle_finish(x, nb, ek, W.ks, c);
+    o.l = co.l;
+    o.p = co.pos;
+    o.f = co.f;
+    o.dir = (c.x & 1) ? 0 : 1;
+    o.rs = (ek.x == W.ks) ? 0 : ((ek.y == W.ks) ? 1 : -1);
+    o.ncyc = co.ncyc;
+    return o;
+}
+
+// path lengths at path-ID vertices, from the splitters' final windows
+__global__ void __launch_bounds__(256) k_grs_len(ForestArgs a) {
+    LF_TL(g_tl_forest, 7);
+    pdl_wait();
+    pdl_trigger();
+    const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
+        const GrsWin W = grs_window(a, i, 0);
+        int32_t L;
+        const int32_t l = grs_path_id(W, L);
+        // paths: the path-id end writes; cycles: every splitter on it (the same value)
+        if (W.cyc || l == __ldcg(a.list1 + i)) a.len[l] = L;
+    }
+}
+
+// walk priority on splitter-free cycles: a hash, so that the walks that stop at the first
+// lower-priority vertex are short whatever the id order along the cycle
+__device__ __forceinline__ uint64_t grs_prio(int32_t v) {
+    return ((uint64_t)((uint32_t)v * 0x85EBCA6Bu ^ 0xC2B2AE35u) << 32) | (uint32_t)v;
+}
+
+// vertices no walk visited lie on cycles without a splitter: the lowest-priority vertex of
+// each walks it (slot 0 ahead), records the weakest edge (first occurrence, reading c9)
+// and writes the path length at the path-ID vertex
+__global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
+    LF_TL(g_tl_forest, 8);
+    pdl_wait();
+    pdl_trigger();
+    const int64_t words = (a.N + 31) >> 5;
+    for (int64_t wi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; wi < words;
+         wi += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t m = ~__ldcg(a.grs_bits + wi);
+        if ((wi + 1) * 32 > a.N) m &= (1u << (a.N - wi * 32)) - 1u;
+        while (m) {
+            const int bit = __ffs(m) - 1;
+            m &= m - 1u;
+            const int32_t v = (int32_t)(wi * 32 + bit);
+            int2 nbv;
+            float2 wv;
+            grs_load(a, v, nbv, wv);
+            const uint64_t pv = grs_prio(v);
+            bool lowest = true;
+            {
+                int32_t prev = v, cur = nbv.x;
+                while (cur != v) {
+                    if (grs_prio(cur) < pv) { lowest = false; break; }
+                    int2 nb;
+                    float2 w;
+                    grs_load(a, cur, nb, w);
+                    const int32_t nxt = nb.x == prev ? nb.y : nb.x;
+                    prev = cur;
+                    cur = nxt;
+                }
+            }
+            if (!lowest) continue;
+            uint64_t K = KEY_INF;
+            int32_t DK = 0, R = 0;
+            int32_t prev = v, cur = v;
+            int2 nbc = nbv;
+            float2 wc = wv;
+            int fs = 0;
+            do {
+                const int32_t nxt = fs ? nbc.y : nbc.x;
+                const float wn = fs ? wc.y : wc.x;
+                int2 nbn;
+                float2 wnx;
+                grs_load(a, nxt, nbn, wnx);
+                const uint64_t k = edge_key(cur, nxt, wn, cur < nxt ? nbc : nbn);
+                if (k < K) { K = k; DK = 2 * R + (cur < nxt ? 1 : 0); }
+                R++;
+                prev = cur;
+                cur = nxt;
+                nbc = nbn;
+                wc = wnx;
+                fs = nbc.x == prev ? 1 : 0;
+            } while (cur != v);
+            const int c = atomicAdd(&a.ctl[kCtlCyc], 1);
+            a.grs_cyc[c] = make_int4(v, DK, R, 0);
+            a.grs_cyck[c] = K;
+            a.len[key_min_end(K)] = R;
+        }
+    }
+}
+
+// tile-local exclusive prefix of the path lengths (the tail of k_lf_full2)
+__global__ void __launch_bounds__(ET) k_grs_lenscan(ForestArgs a) {
+    LF_TL(g_tl_forest, 9);
+    __shared__ int sh[32 * EV];
+    pdl_wait();
+    pdl_trigger();
+    const int64_t b0 = a.lo + (int64_t)blockIdx.x * LB;
+    int lens[EV], e[EV], tot[EV];
+#pragma unroll
+    for (int k = 0; k < EV; k++) {
+        const int64_t g = b0 + threadIdx.x + k * ET;
+        lens[k] = g < a.hi ? __ldcg(a.len + g) : 0;
+    }
+    block_scan_sum_excl_v<EV>(lens, sh, e, tot);
+    int carry = 0;
+#pragma unroll
+    for (int k = 0; k < EV; k++) {
+        const int64_t gk = b0 + threadIdx.x + k * ET;
+        if (gk < a.hi && lens[k]) a.off[gk] = carry + e[k];
+        carry += tot[k];
+    }
+    if (threadIdx.x == 0) a.tsum[blockIdx.x] = carry;
+}
+
+// one vertex of a walk: the scattered vertex-indexed outputs and the sequential ones at r
+__device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 nb, int fslot, int32_t d,
+                                         const GrsWin& W, int32_t base, int& ncyc) {
+    const GrsOut o = grs_vertex(x, nb, fslot, d, W);
+    const int32_t r = base + o.p - 1;
+    // one scattered store (iperm); the rest goes to index r, consecutive along the walk;
+    // k_grs_out moves path_id / pos / forest to vertex order with one gather per vertex
+    a.iperm[x] = r;
+    a.perm[r] = x;
+    a.grs_orec[r] = make_int4(o.l, o.p, o.f.x, o.f.y);
+    ncyc += o.ncyc;
+    if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
+        const int4 q = __ldg(a.grs_erec + x);
+        const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
+        const int ss = ((o.dir ^ 1) != o.rs && (o.dir ? nb.x : nb.y) >= 0) ? (o.dir ^ 1) : -1;
+        a.ta[r] = ps < 0 ? 0.0f : __int_as_float(ps ? q.y : q.x);
+        a.tc[r] = ss < 0 ? 0.0f : __int_as_float(ss ? q.y : q.x);
+        a.tb[r] = __int_as_float(q.z);
+    }
+}
+
+__global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
+    LF_TL(g_tl_forest, 10);
+    pdl_wait();
+    const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
+    const int ncl = __ldcg(&a.ctl[kCtlCyc]);
+    const int stride = gridDim.x * blockDim.x;
+    int ncyc = 0;
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt + ncl; t += stride) {
+        GrsWin W;
+        int32_t sv, x, fs0;
+        int2 nbs;
+        if (t < 2 * cnt) {
+            const int i = t >> 1, f = t & 1;
+            sv = __ldcg(a.list1 + i);
+            float2 ws;
+            grs_load(a, sv, nbs, ws);
+            W = grs_window(a, i, f);
+            x = f ? nbs.y : nbs.x;
+            const int32_t tgt = reinterpret_cast<const int32_t*>(a.cq + i)[f];
+            fs0 = f;
+            int32_t L;
+            const int32_t l = grs_path_id(W, L);
+            const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
+            if (f == 0) grs_write(a, sv, nbs, 0, 0, W, base, ncyc);  // the splitter itself
+            if (x < 0 || tgt < 0) continue;
+            if (tgt == sv ? f == 1 : tgt < sv) continue;  // the segment belongs to the other end
+            int32_t prev = sv, cur = x, d = 1;
+            int2 nbc;
+            float2 wc;
+            grs_load(a, cur, nbc, wc);
+            while (!grs_splitter(a, cur, nbc)) {
+                const int fs = nbc.x == prev ? 1 : 0;
+                grs_write(a, cur, nbc, fs, d, W, base, ncyc);
+                prev = cur;
+                cur = fs ? nbc.y : nbc.x;
+                grs_load(a, cur, nbc, wc);
+                d++;
+            }
+        } else {  // a cycle without splitters, from its recorded vertex (slot 0 ahead)
+            const int c = t - 2 * cnt;
+            const int4 cr = __ldcg(a.grs_cyc + c);
+            sv = cr.x;
+            W.cyc = true;
+            W.ks = __ldcg(a.grs_cyck + c);
+            W.pf = cr.y >> 1;
+            W.bf = cr.y & 1;
+            W.pb = cr.z - W.pf - 1;
+            W.bb = W.bf ^ 1;  // the far endpoint of the weakest edge
+            const int32_t l = key_min_end(W.ks);
+            const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
+            float2 ws;
+            grs_load(a, sv, nbs, ws);
+            grs_write(a, sv, nbs, 0, 0, W, base, ncyc);
+            int32_t prev = sv, cur = nbs.x, d = 1;
+            while (cur != sv) {
+                int2 nbc;
+                float2 wc;
+                grs_load(a, cur, nbc, wc);
+                const int fs = nbc.x == prev ? 1 : 0;
+                grs_write(a, cur, nbc, fs, d, W, base, ncyc);
+                prev = cur;
+                cur = fs ? nbc.y : nbc.x;
+                d++;
+            }
+        }
+        (void)fs0;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o);
+    if ((threadIdx.x & 31) == 0 && ncyc && a.n_cycles) atomicAdd(a.n_cycles, (unsigned long long)ncyc);
+}
+
+// vertex-order outputs from the records k_grs_emit left at each vertex's new index
+__global__ void __launch_bounds__(256) k_grs_out(ForestArgs a) {
+    LF_TL(g_tl_forest, 11);
+    pdl_wait();
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += 2 * stride) {
+        const int64_t v2 = v + stride;
+        const int32_t r0 = __ldcg(a.iperm + v), r1 = v2 < a.N ? __ldcg(a.iperm + v2) : 0;
+        const int4 o0 = __ldcg(a.grs_orec + r0);
+        const int4 o1 = v2 < a.N ? __ldcg(a.grs_orec + r1) : make_int4(0, 0, 0, 0);
+        a.path_id[v] = o0.x;
+        a.pos[v] = o0.y;
+        a.forest[v] = make_int2(o0.z, o0.w);
+        if (v2 < a.N) {
+            a.path_id[v2] = o1.x;
+            a.pos[v2] = o1.y;
+            a.forest[v2] = make_int2(o1.z, o1.w);
+        }
+    }
+}
+
+// which linear-forest algorithm: the tile path for graphs whose paths stay in 1024-id
+// tiles (C1-C3), the global ruling set for large graphs (LF_FOREST=tile|grs overrides)
+static bool use_grs(int64_t N) {
+    const char* e = getenv("LF_FOREST");
+    if (e && !strcmp(e, "grs")) return true;
+    if (e && !strcmp(e, "tile")) return false;
+    return N >= ((int64_t)1 << 22);
+}
+
 int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* forest, int32_t* path_id,
                int32_t* pos, int32_t* perm, int32_t* iperm, int64_t* n_cycles, const ForestWs& w,
                cudaStream_t s, const TriOut* tri) {
@@ -2989,21 +3458,69 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     a.n_cycles = (unsigned long long*)n_cycles;
     a.max_steps = max_steps_for(N) < kMaxSteps ? max_steps_for(N) : kMaxSteps;
     const int tiles = (int)((N + LB - 1) / LB);
-    {
-        LF_PROF("lf_tile", -1, s);
-        LF_CUDA(launch_pdl(k_lf_full1, tiles, LT, kFull1Smem, s, a));
-        LF_CUDA(cudaGetLastError());
-    }
-    {
-        LF_PROF("red_scan", -1, s);
+    if (use_grs(N)) {
+        a.list1 = w.list1;
+        a.grs_rec = (getenv("LF_GRS_PACK") && !strcmp(getenv("LF_GRS_PACK"), "0")) ? nullptr : w.grs_rec;
+        a.grs_shift = getenv("LF_GRS_SHIFT") ? atoi(getenv("LF_GRS_SHIFT")) : kGrsShift;
+        if (a.grs_shift < 20 || a.grs_shift > 31) a.grs_shift = kGrsShift;
+        a.grs_bits = w.grs_bits;
+        a.grs_erec = w.grs_erec;
+        a.grs_orec = w.grs_orec;
+        a.grs_cyc = w.grs_cyc;
+        a.grs_cyck = w.grs_cyck;
+        a.perm = perm;
+        a.iperm = iperm;
+        a.pi2_val = tri ? (const float2*)tri->pi2_val : nullptr;
+        a.diag = tri ? tri->diag : nullptr;
+        a.ta = tri ? tri->a : nullptr;
+        a.tb = tri ? tri->b : nullptr;
+        a.tc = tri ? tri->c : nullptr;
+        {
+            LF_PROF("grs_pack", -1, s);
+            LF_CUDA(launch_pdl(k_grs_pack, persistent_grid((const void*)k_grs_pack, 256), 256, 0, s, a));
+        }
+        {
+            LF_PROF("grs_walk", -1, s);
+            LF_CUDA(launch_pdl(k_grs_walk, persistent_grid((const void*)k_grs_walk, 256), 256, 0, s, a));
+        }
+        {
+            LF_PROF("red_scan", -1, s);
+            LF_CUDA(launch_red_full(a, s));
+        }
+        {
+            LF_PROF("grs_len", -1, s);
+            LF_CUDA(launch_pdl(k_grs_len, persistent_grid((const void*)k_grs_len, 256), 256, 0, s, a));
+            LF_CUDA(launch_pdl(k_grs_cycfind, persistent_grid((const void*)k_grs_cycfind, 256), 256, 0, s, a));
+            LF_CUDA(launch_pdl(k_grs_lenscan, tiles, ET, 0, s, a));
+            LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, tiles, (const int*)w.ctl,
+                               (unsigned long long*)n_cycles));
+        }
+        {
+            LF_PROF(tri ? "grs_emit_tri" : "grs_emit", -1, s);
+            LF_CUDA(launch_pdl(k_grs_emit, persistent_grid((const void*)k_grs_emit, 256), 256, 0, s, a));
+        }
+        {
+            LF_PROF("grs_out", -1, s);
+            LF_CUDA(launch_pdl(k_grs_out, persistent_grid((const void*)k_grs_out, 256), 256, 0, s, a));
+        }
+        return LF_OK;
+    } else {
+        {
+            LF_PROF("lf_tile", -1, s);
+            LF_CUDA(launch_pdl(k_lf_full1, tiles, LT, kFull1Smem, s, a));
+            LF_CUDA(cudaGetLastError());
+        }
+        {
+            LF_PROF("red_scan", -1, s);
 #ifndef LF_NO_GRID_RED  // diagnostics only: measures the launch cost (wrong results)
-        // cooperative cluster launch (the grid path's barrier): see launch_red_full
-        LF_CUDA(launch_red_full(a, s));
+            // cooperative cluster launch (the grid path's barrier): see launch_red_full
+            LF_CUDA(launch_red_full(a, s));
 #endif
-    }
-    {
-        LF_PROF("lf_expand", -1, s);
-        LF_CUDA(launch_pdl(k_lf_full2, tiles, ET, sizeof(TileSmemE), s, a));
+        }
+        {
+            LF_PROF("lf_expand", -1, s);
+            LF_CUDA(launch_pdl(k_lf_full2, tiles, ET, sizeof(TileSmemE), s, a));
+        }
     }
     {
         LF_PROF(tri ? "perm_tridiag" : "perm", -1, s);
@@ -3375,8 +3892,8 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
 #ifdef LF_TIMELINE
 int timeline_forest(unsigned long long* out, int reset) {
     if (reset) {
-        unsigned long long h[16];
-        for (int i = 0; i < 16; i += 2) { h[i] = ~0ull; h[i + 1] = 0; }
+        unsigned long long h[32];
+        for (int i = 0; i < 32; i += 2) { h[i] = ~0ull; h[i + 1] = 0; }
         return cudaMemcpyToSymbol(g_tl_forest, h, sizeof(h)) == cudaSuccess ? 0 : -1;
     }
     return cudaMemcpyFromSymbol(out, g_tl_forest, sizeof(g_tl_forest)) == cudaSuccess ? 0 : -1;

@@ -25,12 +25,13 @@ void g_err_clear();
     } while (0)
 
 // optional per-kernel event timing (lf_profile_enable / lf_profile_collect)
-void prof_begin(const char* name, int k, cudaStream_t s);
-void prof_end(cudaStream_t s);
+int prof_begin(const char* name, int k, cudaStream_t s);
+void prof_end(cudaStream_t s, int idx);
 struct ProfScope {
     cudaStream_t s;
-    ProfScope(const char* name, int k, cudaStream_t st) : s(st) { prof_begin(name, k, s); }
-    ~ProfScope() { prof_end(s); }
+    int idx;
+    ProfScope(const char* name, int k, cudaStream_t st) : s(st), idx(prof_begin(name, k, st)) {}
+    ~ProfScope() { prof_end(s, idx); }
 };
 #define LF_PROF(name, k, s) ::lf::ProfScope lf_prof_scope_(name, k, s)
 
@@ -135,6 +136,14 @@ struct ForestWs {
     int2* cq_dk;           //   initial DK (2 * distance to the minimum's near endpoint + bit),
     int2* dk2;             //   final DK per direction
     int2* rdk[2];          //   grid-path ping-pong DK
+    // global ruling set (lf_forest.cu k_grs_*): packed per-vertex records, visit bitmap,
+    // records of splitter-free cycles
+    int4* grs_rec;         // [N] (slots, |w|) packed
+    int4* grs_erec;        // [N] (signed values, diag)
+    int4* grs_orec;        // [N] outputs at the new index
+    uint32_t* grs_bits;    // [N/32 + 1] splitter or visited by a walk
+    int4* grs_cyc;         // [N/3 + 1] (lowest vertex, DK, L, 0) of a cycle without splitters
+    uint64_t* grs_cyck;    // [N/3 + 1] its weakest key
 };
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w);
 

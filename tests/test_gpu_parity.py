@@ -131,11 +131,45 @@ def test_factor_small(torch_cuda, lfm, oracle_mod, name, make, n):
     check_factor(torch_cuda, lfm, oracle_mod, A, n)
 
 
-@pytest.mark.parametrize("name,make", SMALL, ids=[s[0] for s in SMALL])
-def test_pipeline_small(torch_cuda, lfm, oracle_mod, name, make):
+def with_zeros(A, seed=7, frac=0.15):
+    """A copy of A with ~frac of its edges stored as explicit +0.0 and ~frac as -0.0 (both
+    triangles): zero entries are not edges (PAPER.md:L31 w(e) != 0; A' = |A| - diag, L231)."""
+    import copy
+
+    B = copy.deepcopy(A)
+    rows = np.repeat(np.arange(B.N, dtype=np.int64), np.diff(B.rowptr))
+    col = B.col.astype(np.int64)
+    off = rows != col
+    u = lfgen.edge_hash_u(rows, col, B.N, seed)  # symmetric in (row, col)
+    B.val[off & (u < frac)] = np.float32(0.0)
+    B.val[off & (u >= frac) & (u < 2 * frac)] = np.float32(-0.0)
+    B.name = A.name + "_zeros"
+    return B
+
+
+SMALL_ZEROS = [
+    ("c1_zeros", lambda: with_zeros(lfgen.config("C1"))),
+    ("c5_small_zeros", lambda: with_zeros(lfgen.grid3d_27pt(12), frac=0.3)),
+    ("random_zeros_shuffled", lambda: with_zeros(lfgen.random_graph(2000, 7000, seed=2, shuffle_cols_seed=4))),
+]
+FOREST_MODES = ["tile", "grs"]  # DESIGN.md §4.3 tile path / §4.3a global ruling set
+
+
+@pytest.mark.parametrize("forest", FOREST_MODES)
+@pytest.mark.parametrize("name,make", SMALL + SMALL_ZEROS, ids=[s[0] for s in SMALL + SMALL_ZEROS])
+def test_pipeline_small(torch_cuda, lfm, oracle_mod, monkeypatch, name, make, forest):
+    monkeypatch.setenv("LF_FOREST", forest)
     A = make()
     fac, ref = check_factor(torch_cuda, lfm, oracle_mod, A, 2)
     check_forest(torch_cuda, lfm, oracle_mod, A, fac, ref)
+
+
+@pytest.mark.parametrize("name,make", SMALL_ZEROS, ids=[s[0] for s in SMALL_ZEROS])
+@pytest.mark.parametrize("n", [1, 3, 4])
+def test_factor_explicit_zeros(torch_cuda, lfm, oracle_mod, name, make, n):
+    A = make()
+    assert (A.val == 0).sum() > 0 and np.signbit(A.val[A.val == 0]).any()
+    check_factor(torch_cuda, lfm, oracle_mod, A, n)
 
 
 @pytest.mark.parametrize("m,k_m,M,seed", [(5, 1, 5, 0), (1, 0, 7, 0), (3, 2, 9, 17), (2, 1, 6, 123)])
@@ -155,8 +189,10 @@ def test_factor_until_maximal(torch_cuda, lfm, oracle_mod):
                  until_maximal=True)
 
 
-def test_edge_cases(torch_cuda, lfm, oracle_mod):
+@pytest.mark.parametrize("forest", FOREST_MODES)
+def test_edge_cases(torch_cuda, lfm, oracle_mod, monkeypatch, forest):
     """Empty graph, single vertex, edgeless graph, M=0, a single path, a single cycle."""
+    monkeypatch.setenv("LF_FOREST", forest)
     torch = torch_cuda
     cases = [
         lfgen.csr_from_edges(1, np.zeros(0, int), np.zeros(0, int), np.zeros(0)),
@@ -175,8 +211,10 @@ def test_edge_cases(torch_cuda, lfm, oracle_mod):
     check_factor(torch, lfm, oracle_mod, A, 2, M=0)
 
 
-def test_long_paths_and_cycles(torch_cuda, lfm, oracle_mod):
+@pytest.mark.parametrize("forest", FOREST_MODES)
+def test_long_paths_and_cycles(torch_cuda, lfm, oracle_mod, monkeypatch, forest):
     """A 2-factor that is one huge cycle and one long path: ranking across 2^17 steps."""
+    monkeypatch.setenv("LF_FOREST", forest)
     N = 1 << 17
     s = np.arange(N - 1)
     t = s + 1
@@ -191,7 +229,9 @@ def test_long_paths_and_cycles(torch_cuda, lfm, oracle_mod):
     check_forest(torch_cuda, lfm, oracle_mod, A, fac, ref)
 
 
-def test_random_graph_sweep(torch_cuda, lfm, oracle_mod):
+@pytest.mark.parametrize("forest", FOREST_MODES)
+def test_random_graph_sweep(torch_cuda, lfm, oracle_mod, monkeypatch, forest):
+    monkeypatch.setenv("LF_FOREST", forest)
     for seed in range(6):
         A = lfgen.random_graph(2000 + 300 * seed, 5000 + 2000 * seed, seed=seed, ties=seed % 2 == 0,
                                shuffle_cols_seed=seed if seed % 3 == 0 else None)
@@ -250,8 +290,10 @@ def test_repeated_runs_cached_and_uncached_rounds(torch_cuda, lfm, oracle_mod, m
     monkeypatch.delenv("LF_NO_CACHED_ROUNDS", raising=False)
 
 
-@pytest.mark.parametrize("cfg", ["C1", "C3", "C4"])
-def test_config_full_size(torch_cuda, lfm, oracle_mod, cfg):
+@pytest.mark.parametrize("forest", FOREST_MODES)
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C4"])
+def test_config_full_size(torch_cuda, lfm, oracle_mod, monkeypatch, cfg, forest):
+    monkeypatch.setenv("LF_FOREST", forest)
     A = _cached(cfg)
     fac, ref = check_factor(torch_cuda, lfm, oracle_mod, A, 2)
     check_forest(torch_cuda, lfm, oracle_mod, A, fac, ref)
@@ -286,3 +328,58 @@ def _cached(name):
     if name not in _CACHE:
         _CACHE[name] = lfgen.config(name)
     return _CACHE[name]
+
+
+def canonical_factor(N, s, t, w):
+    """A [0,2]-factor (max degree 2) from undirected edges, in lf_factor's canonical slot
+    form: slots sorted by (|w| desc, id asc), -1 padding last (reading c8)."""
+    pi = -np.ones((N, 2), np.int32)
+    pw = np.zeros((N, 2), np.float32)
+    nbrs = [[] for _ in range(N)]
+    for a, b, x in zip(s.tolist(), t.tolist(), np.asarray(w, np.float32).tolist()):
+        nbrs[a].append((-x, b))
+        nbrs[b].append((-x, a))
+    for v, L in enumerate(nbrs):
+        assert len(L) <= 2
+        for i, (nx, u) in enumerate(sorted(L)):
+            pi[v, i] = u
+            pw[v, i] = -nx
+    return pi, pw
+
+
+@pytest.mark.parametrize("forest", FOREST_MODES)
+@pytest.mark.parametrize("ties", [False, True])
+def test_forest_cycles_and_paths_of_all_lengths(torch_cuda, lfm, oracle_mod, monkeypatch, forest, ties):
+    """Cycles of every length 3..300 and paths of length 1..300 under a random relabelling,
+    given directly as a [0,2]-factor: in GRS mode most short cycles hold no splitter (they
+    are walked by their lowest-priority vertex) and long ones several; tie-heavy weights
+    exercise reading c9."""
+    torch = torch_cuda
+    monkeypatch.setenv("LF_FOREST", forest)
+    rng = np.random.default_rng(11 + ties)
+    segs, N = [], 0
+    for L in list(range(3, 301)) + [1000, 4099]:
+        segs.append(("c", N, L))
+        N += L
+    for L in list(range(1, 301)) + [2000]:
+        segs.append(("p", N, L))
+        N += L
+    N += 37  # isolated vertices
+    lab = rng.permutation(N)
+    s, t = [], []
+    for kind, b, L in segs:
+        ids = np.arange(b, b + L)
+        if kind == "c":
+            s += ids.tolist(); t += np.roll(ids, -1).tolist()
+        else:
+            s += ids[:-1].tolist(); t += ids[1:].tolist()
+    s, t = lab[np.array(s)], lab[np.array(t)]
+    w = (np.floor(rng.random(s.shape[0]) * 3) + 1) / 4 if ties else 1.0 - lfgen.edge_hash_u(s, t, N, 5)
+    pi, pw = canonical_factor(N, s, t, w)
+    o = oracle_mod.linear_forest(pi, pw)
+    out = lfm.linear_forest(torch.from_numpy(pi).cuda(), torch.from_numpy(pw).cuda())
+    torch.cuda.synchronize()
+    for k in ("forest", "path_id", "pos", "perm", "iperm"):
+        got = out[k].cpu().numpy()
+        assert np.array_equal(got, o[k]), f"{k} mismatch: first at {np.argwhere(got != o[k])[:3].ravel()}"
+    assert int(out["n_cycles"].item()) == o["n_cycles"] == 300
