@@ -112,7 +112,7 @@ int persistent_grid(const void* kernel, int block, size_t smem) {
 size_t factor_ws_carve(Carve& c, int64_t N, int n, FactorWs* w) {
     FactorWs t;
     const size_t nn = (size_t)(N > 0 ? N : 1);
-    t.state = c.take<uint8_t>(nn);
+    t.state = c.take<uint8_t>(nn + 4);  // + 4: word-sized state fetches past the last vertex
     t.prop_j = c.take<int32_t>(nn * n);
     t.prop_v = c.take<float>(nn * n);
     t.wl[0] = c.take<int32_t>(nn);
@@ -139,19 +139,86 @@ static bool csr_ok(const lf_csr_t* A) {
 // ---------------------------------------------------------------------------
 // validation kernel
 // ---------------------------------------------------------------------------
+// pass 1: row pointers, column range, finite values; per row: strictly ascending columns
+// (sorted[v] = 1), else a duplicate search within the row (O(deg^2), unsorted rows only)
 __global__ void k_validate(int64_t N, int64_t nnz, const int64_t* rowptr, const int32_t* col,
-                           const float* val, int* bad) {
+                           const float* val, int* bad, uint8_t* sorted) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v <= N; v += stride) {
         const int64_t r = rowptr[v];
         if (v == 0 && r != 0) atomicOr(bad, 1);
         if (v == N && r != nnz) atomicOr(bad, 1);
-        if (v < N && rowptr[v + 1] < r) atomicOr(bad, 1);
+        if (v < N && (rowptr[v + 1] < r || r < 0 || r > nnz)) atomicOr(bad, 1);
     }
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += stride) {
         const int32_t j = col[e];
         if (j < 0 || (int64_t)j >= N) atomicOr(bad, 2);
         if (!isfinite(val[e])) atomicOr(bad, 4);
+    }
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N; v += stride) {
+        const int64_t r0 = min(max(rowptr[v], (int64_t)0), nnz), r1 = min(max(rowptr[v + 1], r0), nnz);
+        bool asc = true;
+        for (int64_t e = r0 + 1; e < r1 && asc; e++) asc = col[e] > col[e - 1];
+        sorted[v] = asc ? 1 : 0;
+        if (asc) continue;
+        bool dup = false;
+        for (int64_t e = r0; e < r1 && !dup; e++)
+            for (int64_t f = e + 1; f < r1; f++)
+                if (col[e] == col[f]) { dup = true; break; }
+        if (dup) atomicOr(bad, 8);
+    }
+}
+
+// pass 2 (a warp per row): every edge (i, j) -- j != i, a_ij != 0, PAPER.md:L31, L231 --
+// needs the entry (j, i) with the same |a| (an undirected weighted graph, L315)
+__global__ void k_validate_sym(int64_t N, int64_t nnz, const int64_t* rowptr, const int32_t* col,
+                               const float* val, int* bad, const uint8_t* sorted) {
+    const int lane = threadIdx.x & 31;
+    const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = w0; i < N; i += nw) {
+        const int64_t r0 = min(max(rowptr[i], (int64_t)0), nnz), r1 = min(max(rowptr[i + 1], r0), nnz);
+        for (int64_t e = r0 + lane; e < r1; e += 32) {
+            const int32_t j = col[e];
+            const uint32_t x = __float_as_uint(val[e]) & 0x7FFFFFFFu;
+            if (j < 0 || (int64_t)j >= N || (int64_t)j == i || x == 0u) continue;
+            const int64_t s0 = min(max(rowptr[j], (int64_t)0), nnz), s1 = min(max(rowptr[j + 1], s0), nnz);
+            int64_t hit = -1;
+            if (sorted[j]) {
+                int64_t lo = s0, hi = s1;
+                while (lo < hi) {
+                    const int64_t m = (lo + hi) >> 1;
+                    if ((int64_t)col[m] < i) lo = m + 1; else hi = m;
+                }
+                if (lo < s1 && (int64_t)col[lo] == i) hit = lo;
+            } else {
+                for (int64_t f = s0; f < s1; f++)
+                    if ((int64_t)col[f] == i) { hit = f; break; }
+            }
+            if (hit < 0) atomicOr(bad, 16);
+            else if ((__float_as_uint(val[hit]) & 0x7FFFFFFFu) != x) atomicOr(bad, 32);
+        }
+    }
+}
+
+// a [0,n]-factor in lf_factor's canonical form: ids in range, no self loop, valid slots
+// first and -1 padding last, no repeated neighbour, symmetric (w in pi(v) <=> v in pi(w))
+__global__ void k_validate_factor(int64_t N, int n, const int32_t* pi, int* bad) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N; v += stride) {
+        bool pad = false;
+        for (int s = 0; s < n; s++) {
+            const int32_t w = pi[v * n + s];
+            if (w < -1 || (int64_t)w >= N || (int64_t)w == v) { atomicOr(bad, 64); break; }
+            if (w < 0) { pad = true; continue; }
+            if (pad) { atomicOr(bad, 64); break; }  // a neighbour after padding
+            bool back = false;
+            for (int t = 0; t < n; t++) {
+                if (t != s && pi[v * n + t] == w) atomicOr(bad, 64);
+                back |= pi[(int64_t)w * n + t] == (int32_t)v;
+            }
+            if (!back) atomicOr(bad, 128);
+        }
     }
 }
 
@@ -399,10 +466,16 @@ int lf_validate_csr(const lf_csr_t* A, void* ws, size_t ws_bytes, void* stream) 
     if (!csr_ok(A)) return set_error(LF_EINVAL, "lf_validate_csr: invalid CSR descriptor");
     if (!ws || ws_bytes < sizeof(int)) return set_error(LF_ENOMEM, "lf_validate_csr: workspace too small");
     cudaStream_t s = (cudaStream_t)stream;
+    if (!ws || ws_bytes < lf_validate_workspace_size(A->n) || ((uintptr_t)ws & 255))
+        return set_error(LF_ENOMEM, "lf_validate_csr: workspace smaller than lf_validate_workspace_size(N)");
     int* bad = (int*)ws;
+    uint8_t* sorted = (uint8_t*)ws + 256;
     LF_CUDA(cudaMemsetAsync(bad, 0, sizeof(int), s));
     k_validate<<<persistent_grid((const void*)k_validate, 256), 256, 0, s>>>(A->n, A->nnz, A->rowptr, A->col,
-                                                                         A->val, bad);
+                                                                         A->val, bad, sorted);
+    LF_CUDA(cudaGetLastError());
+    k_validate_sym<<<persistent_grid((const void*)k_validate_sym, 256), 256, 0, s>>>(A->n, A->nnz, A->rowptr,
+                                                                                 A->col, A->val, bad, sorted);
     LF_CUDA(cudaGetLastError());
     int h = 0;
     LF_CUDA(cudaMemcpyAsync(&h, bad, sizeof(int), cudaMemcpyDeviceToHost, s));
@@ -410,44 +483,40 @@ int lf_validate_csr(const lf_csr_t* A, void* ws, size_t ws_bytes, void* stream) 
     if (h & 1) return set_error(LF_EINPUT, "lf_validate_csr: rowptr not monotone or wrong ends");
     if (h & 2) return set_error(LF_EINPUT, "lf_validate_csr: column index out of range");
     if (h & 4) return set_error(LF_EINPUT, "lf_validate_csr: NaN or Inf value");
+    if (h & 8) return set_error(LF_EINPUT, "lf_validate_csr: duplicate (i,j) entry");
+    if (h & 16) return set_error(LF_EINPUT, "lf_validate_csr: pattern not symmetric (edge (i,j) without (j,i))");
+    if (h & 32) return set_error(LF_EINPUT, "lf_validate_csr: |a_ij| != |a_ji| (values not symmetric)");
+    return LF_OK;
+}
+
+size_t lf_validate_workspace_size(int64_t N) { return 256 + (size_t)(N > 0 ? N : 0) + 256; }
+
+int lf_validate_factor(int64_t N, int n, const int32_t* pi, void* ws, size_t ws_bytes, void* stream) {
+    g_err[0] = 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (N < 0 || N >= ((int64_t)1 << 31)) return set_error(LF_EINVAL, "lf_validate_factor: bad N");
+    if (n < 1 || n > 4) return set_error(LF_EINVAL, "lf_validate_factor: n must be in [1,4]");
+    if (N == 0) return LF_OK;
+    if (!pi) return set_error(LF_EINVAL, "lf_validate_factor: NULL pi");
+    if (!ws || ws_bytes < 256 || ((uintptr_t)ws & 255))
+        return set_error(LF_ENOMEM, "lf_validate_factor: workspace smaller than 256 bytes");
+    int* bad = (int*)ws;
+    LF_CUDA(cudaMemsetAsync(bad, 0, sizeof(int), s));
+    k_validate_factor<<<persistent_grid((const void*)k_validate_factor, 256), 256, 0, s>>>(N, n, pi, bad);
+    LF_CUDA(cudaGetLastError());
+    int h = 0;
+    LF_CUDA(cudaMemcpyAsync(&h, bad, sizeof(int), cudaMemcpyDeviceToHost, s));
+    LF_CUDA(cudaStreamSynchronize(s));
+    if (h & 64) return set_error(LF_EINPUT, "lf_validate_factor: bad slot (id range, self loop, order or repeat)");
+    if (h & 128) return set_error(LF_EINPUT, "lf_validate_factor: not symmetric (w in pi(v) but v not in pi(w))");
     return LF_OK;
 }
 
 }  // extern "C"
 
-// ---------------------------------------------------------------------------
-// launch-overhead probe (diagnostics only): an empty kernel on a
-// persistent-size grid, launched cooperatively or not, optionally with one grid barrier
-// ---------------------------------------------------------------------------
-#include <cooperative_groups.h>
-namespace lf {
-__global__ void k_probe(int sync_steps) {
-    cooperative_groups::grid_group g = cooperative_groups::this_grid();
-    for (int i = 0; i < sync_steps; i++) g.sync();
-}
-__global__ void k_probe_plain(int* p) {
-    if (p && threadIdx.x == 0 && blockIdx.x == 0) atomicAdd(p, 1);
-}
-}  // namespace lf
-
 // Diagnostics only (not part of include/lf.h): per-kernel timeline of LF_TIMELINE builds.
-// out[0..15] factor kernels, out[16..31] forest kernels; reset != 0 clears.  -1 otherwise.
+// out[0..15] factor kernels, out[16..47] forest kernels; reset != 0 clears.  -1 otherwise.
 extern "C" int lf_debug_timeline(unsigned long long* out, int reset) {
     if (reset) return lf::timeline_factor(nullptr, 1) | lf::timeline_forest(nullptr, 1);
     return lf::timeline_factor(out, 0) | lf::timeline_forest(out + 16, 0);
-}
-
-extern "C" int lf_debug_launch_probe(int mode, int block, int sync_steps, void* stream) {
-    using namespace lf;
-    cudaStream_t s = (cudaStream_t)stream;
-    if (mode == 0) {
-        const int grid = persistent_grid((const void*)k_probe_plain, block);
-        k_probe_plain<<<grid, block, 0, s>>>(nullptr);
-        LF_CUDA(cudaGetLastError());
-        return LF_OK;
-    }
-    const int grid = persistent_grid((const void*)k_probe, block);
-    void* args[] = {&sync_steps};
-    LF_CUDA(cudaLaunchCooperativeKernel((const void*)k_probe, grid, block, args, 0, s));
-    return LF_OK;
 }

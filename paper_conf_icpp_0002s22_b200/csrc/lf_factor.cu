@@ -651,6 +651,8 @@ struct MutualArgs {
     int32_t* __restrict__ wl_next_count;
     int32_t* __restrict__ wl_zero;   // count slot to reset for round k+2 (NULL: none)
     int fresh;                       // round 0 from scratch: state/pi not initialised yet
+    int pad_state;                   // k_mutual0 also zeroes state[N..N+3] (whole-graph runs:
+                                     // the rows mode fetches state bytes as aligned words)
     int next_charging;
     uint32_t next_k;
     uint32_t seed;
@@ -802,6 +804,7 @@ __global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
     LF_TL(g_tl_factor, 2);
     pdl_wait();
     if (a.wl_zero && blockIdx.x == 0 && threadIdx.x == 0) *a.wl_zero = 0;
+    if (a.pad_state && blockIdx.x == 0 && threadIdx.x < 4) a.state[a.N + threadIdx.x] = 0;
     const int lane = threadIdx.x & 31;
     const int64_t chunk = (int64_t)blockDim.x * MB;
     for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < a.N; c0 += (int64_t)gridDim.x * chunk) {
@@ -2042,6 +2045,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         ma.wl_next_count = last ? nullptr : &w.counts[(k + 1) % 3];
         ma.wl_zero = last ? nullptr : &w.counts[(k + 2) % 3];
         ma.fresh = fresh ? 1 : 0;
+        ma.pad_state = (fresh && !part) ? 1 : 0;
         ma.next_charging = ((k + 1) % o->m) != o->k_m;
         ma.next_k = (uint32_t)(k + 1);
         ma.seed = o->seed;

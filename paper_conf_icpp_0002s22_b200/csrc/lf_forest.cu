@@ -70,6 +70,8 @@ constexpr int kCtlCnt2 = 129;
 constexpr int kCtlTicket3 = 130;  // finished-CTA ticket of k_path_offsets / k_lf_full2 (the last one scans tsum)
 constexpr int kCtlNcyc = 131;     // broken cycles (single-pass forest)
 constexpr int kCtlGridBar = 133;  // arrival counter of k_red_full's grid barrier
+constexpr int kCtlBad = 135;      // the tile path met a malformed factor: later kernels leave
+constexpr int kCtlBadGrs = 136;   // a ruling-set walk met one (bounded; records stay well formed)
 constexpr int kMaxSteps = 62;
 constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
 // ctl[192] splitter nodes (cycle pass), [193] unvisited vertices (fallback), [194] tiles
@@ -1613,9 +1615,11 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
                                                   const float2* __restrict__ pi2_val,
                                                   const float* __restrict__ diag, int32_t* __restrict__ perm,
                                                   int32_t* __restrict__ iperm, float* __restrict__ ta,
-                                                  float* __restrict__ tb, float* __restrict__ tc) {
+                                                  float* __restrict__ tb, float* __restrict__ tc,
+                                                  const int* __restrict__ ctl) {
     LF_TL(g_tl_forest, 4);
     pdl_wait();
+    if (ctl && __ldcg(ctl + kCtlBad)) return;  // a malformed factor: see k_lf_full1
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < N; v0 += stride * kPermBatch) {
         int32_t l[kPermBatch], p[kPermBatch], r[kPermBatch];
@@ -1636,7 +1640,8 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
             }
         }
 #pragma unroll
-        for (int b = 0; b < kPermBatch; b++) r[b] = __ldg(tbase + l[b] / chunk) + __ldg(off + l[b]) + p[b] - 1;
+        for (int b = 0; b < kPermBatch; b++)
+            r[b] = v0 + b * stride < N ? __ldg(tbase + l[b] / chunk) + __ldg(off + l[b]) + p[b] - 1 : 0;
 #pragma unroll
         for (int b = 0; b < kPermBatch; b++) {
             const int64_t v = v0 + b * stride;
@@ -2044,12 +2049,16 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
             int prev = su, cur = x - b0, d = f ? vws.y : vws.x;
             km = f ? s.EK1[su] : s.EK0[su];
             dk = slot_dk(s, su, b0 + su, f);
-            while (s.sidx[cur] < 0) {
+            for (int guard = 0; s.sidx[cur] < 0; guard++) {
                 const int2 nbc = s.nb[cur];
                 const int face = (nbc.x == b0 + prev) ? 0 : 1;
                 if (face == 0) { s.recS[cur].x = (short)((i << 1) | f); s.recD[cur].x = (short)d; }
                 else { s.recS[cur].y = (short)((i << 1) | f); s.recD[cur].y = (short)d; }
                 const int nxt = (face ? nbc.x : nbc.y) - b0;
+                if ((unsigned)nxt >= (unsigned)LB || guard >= LB) {  // a malformed factor (not symmetric)
+                    if (stats) atomicOr(stats + (kCtlBad - kCtlStat), 1);
+                    break;
+                }
                 const uint64_t kk = face ? s.EK0[cur] : s.EK1[cur];
                 if (kk < km) {  // a walk passes real links only (run ends are nodes)
                     km = kk;
@@ -2156,7 +2165,11 @@ __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[
             int prev = u, cur = s.nb[u].x - b0, d = 1;
             uint64_t km = s.EK0[u];
             int kd = (b0 + u) < s.nb[u].x ? 1 : 0;
-            while (cur != u) {
+            for (int guard = 0; cur != u; guard++) {
+                if ((unsigned)cur >= (unsigned)LB || guard >= LB) {  // a malformed factor
+                    if (stats) atomicOr(stats + (kCtlBad - kCtlStat), 1);
+                    break;
+                }
                 const int2 nbc = s.nb[cur];
                 const int face = (nbc.x == b0 + prev) ? 0 : 1;
                 const uint64_t kk = face ? s.EK0[cur] : s.EK1[cur];
@@ -2428,6 +2441,31 @@ __global__ void __launch_bounds__(LT, LF_F1MINB) k_lf_full1(ForestArgs a) {
     }
     ulonglong2 ek[VPT];
     slot_keys(a, s, b0, ek);
+    {   // the input must be a symmetric [0,2]-factor in canonical form (include/lf.h): a tile
+        // that is not stops here and flags it, and the later kernels leave (no walk can fault)
+        bool bad = false;
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int u = threadIdx.x + k * LT;
+            const int32_t g = b0 + u;
+            if (g >= a.hi) continue;
+            const int2 nb = s.nb[u];
+            bad |= nb.x < -1 || nb.y < -1 || (int64_t)nb.x >= a.N || (int64_t)nb.y >= a.N || nb.x == g ||
+                   nb.y == g || (nb.x < 0 && nb.y >= 0) || (nb.x >= 0 && nb.x == nb.y);
+            if (bad) continue;
+#pragma unroll
+            for (int i = 0; i < 2; i++) {
+                const int32_t x = i ? nb.y : nb.x;
+                if (x < 0) continue;
+                const int2 px = is_local(x, T) ? s.nb[x - b0] : (is_foreign(x, a) ? ghost_slots(a, x) : a.pi2[x]);
+                bad |= px.x != g && px.y != g;
+            }
+        }
+        if (__syncthreads_or(bad)) {
+            if (threadIdx.x == 0) atomicOr(&a.ctl[kCtlBad], 1);
+            return;
+        }
+    }
     LF_PHASE(a.ctl, 6);
     VRes o[VPT];
     tile_rank_full(s, b0, ek, o, a.ctl + kCtlStat);
@@ -2572,6 +2610,7 @@ __global__ void __launch_bounds__(RT) k_red_full(ForestArgs a) {
     __shared__ int sh[32];
     extern __shared__ __align__(16) unsigned char red_smem[];
     pdl_wait();  // the tile pass's records
+    if (*(volatile int*)&a.ctl[kCtlBad]) return;  // a malformed factor (k_lf_full1): uniform
     const int cnt = *(volatile int*)&a.ctl[kCtlCnt1];
     int* ctl = a.ctl + kCtlRed1;
     if (cnt <= kRedCl * kRedClNodes) {
@@ -2647,6 +2686,8 @@ __global__ void __launch_bounds__(ET, LF_EMINB) k_lf_full2(ForestArgs a) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     TileSmemE& s = *reinterpret_cast<TileSmemE*>(smem_raw);
     __shared__ int sh[32 * EV];  // the final vector scan (read once: no reuse barrier)
+    // the tile pass completed before the reduced scan triggered this launch: its flag is final
+    if (*(volatile int*)&a.ctl[kCtlBad]) return;
     const int32_t b0 = (int32_t)(a.lo + (int64_t)blockIdx.x * LB);
     int2 lcs[EV];  // the tile pass's local results, in flight with the tile's slots
 #pragma unroll
@@ -2795,12 +2836,13 @@ __global__ void __launch_bounds__(ET, LF_EMINB) k_lf_full2(ForestArgs a) {
 constexpr int kPrefT = 1024, kPrefPT = 8;
 
 __global__ void __launch_bounds__(kPrefT) k_tile_prefix(int32_t* tsum, int tiles, const int* ctl,
-                                                        unsigned long long* n_cycles) {
+                                                        unsigned long long* n_cycles, int grs_mode) {
     LF_TL(g_tl_forest, 3);
     __shared__ int sh[32];
     pdl_wait();
     pdl_trigger();
     if (n_cycles && threadIdx.x == 0) *n_cycles = (unsigned long long)__ldcg(ctl + kCtlNcyc);
+    if (__ldcg(ctl + kCtlBad) && !grs_mode) return;  // a malformed factor: see k_lf_full1
     int carry = 0;
     for (int base = 0; base < tiles; base += kPrefT * kPrefPT) {
         int x[kPrefPT], sum = 0;
@@ -3069,9 +3111,11 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
             K = edge_key(sv, cur, f ? ws.y : ws.x, sv < cur ? nbs : nbc);
             DK = sv < cur ? 1 : 0;
             R = 1;
+            bool bad = false;
             while (!grs_splitter(a, cur, nbc)) {
                 const int fs = nbc.x == prev ? 1 : 0;  // the slot away from prev
                 const int32_t nxt = fs ? nbc.y : nbc.x;
+                if (R > a.N || (uint32_t)nxt >= (uint32_t)a.N) { bad = true; break; }  // a malformed factor
                 // each interior vertex is walked from both ends: the walker with prev < nxt marks it
                 if (prev < nxt) atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
                 const float wn = fs ? wc.y : wc.x;
@@ -3087,6 +3131,11 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
                 wc = wnx;
             }
             tgt = cur;
+            if (bad) {  // end the segment here as if at a path end: no reduced record points at
+                        // a non-splitter, so every later kernel stays in bounds
+                atomicOr(&a.ctl[kCtlBadGrs], 1);
+                tgt = -(sv + 1);
+            }
         }
         int32_t* q = reinterpret_cast<int32_t*>(a.cq + i);
         int32_t* r = reinterpret_cast<int32_t*>(a.cq_r + i);
@@ -3190,6 +3239,7 @@ __global__ void __launch_bounds__(256) k_grs_len(ForestArgs a) {
         int32_t L;
         const int32_t l = grs_path_id(W, L);
         // paths: the path-id end writes; cycles: every splitter on it (the same value)
+        if (l < 0 || (int64_t)l >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }  // malformed
         if (W.cyc || l == __ldcg(a.list1 + i)) a.len[l] = L;
     }
 }
@@ -3223,7 +3273,8 @@ __global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
             bool lowest = true;
             {
                 int32_t prev = v, cur = nbv.x;
-                while (cur != v) {
+                for (int64_t guard = 0; cur != v; guard++) {
+                    if ((uint32_t)cur >= (uint32_t)a.N || guard > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); lowest = false; break; }
                     if (grs_prio(cur) < pv) { lowest = false; break; }
                     int2 nb;
                     float2 w;
@@ -3243,6 +3294,7 @@ __global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
             do {
                 const int32_t nxt = fs ? nbc.y : nbc.x;
                 const float wn = fs ? wc.y : wc.x;
+                if (nxt < 0 || R > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
                 int2 nbn;
                 float2 wnx;
                 grs_load(a, nxt, nbn, wnx);
@@ -3255,10 +3307,14 @@ __global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
                 wc = wnx;
                 fs = nbc.x == prev ? 1 : 0;
             } while (cur != v);
+            if (cur != v) continue;  // the walk was stopped (a malformed factor)
             const int c = atomicAdd(&a.ctl[kCtlCyc], 1);
+            if ((int64_t)c > a.N / 3) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }  // overlapping "cycles"
             a.grs_cyc[c] = make_int4(v, DK, R, 0);
             a.grs_cyck[c] = K;
-            a.len[key_min_end(K)] = R;
+            const int32_t lk = key_min_end(K);
+            if (K == KEY_INF || lk < 0 || (int64_t)lk >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }
+            a.len[lk] = R;
         }
     }
 }
@@ -3292,6 +3348,10 @@ __device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 n
                                          const GrsWin& W, int32_t base, int& ncyc) {
     const GrsOut o = grs_vertex(x, nb, fslot, d, W);
     const int32_t r = base + o.p - 1;
+    if (r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {  // a malformed factor
+        atomicOr(&a.ctl[kCtlBadGrs], 1);
+        return;
+    }
     // one scattered store (iperm); the rest goes to index r, consecutive along the walk;
     // k_grs_out moves path_id / pos / forest to vertex order with one gather per vertex
     a.iperm[x] = r;
@@ -3312,7 +3372,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
     LF_TL(g_tl_forest, 10);
     pdl_wait();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
-    const int ncl = __ldcg(&a.ctl[kCtlCyc]);
+    const int ncl = (int)min((int64_t)__ldcg(&a.ctl[kCtlCyc]), a.N / 3 + 1);
     const int stride = gridDim.x * blockDim.x;
     int ncyc = 0;
     for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt + ncl; t += stride) {
@@ -3330,6 +3390,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             fs0 = f;
             int32_t L;
             const int32_t l = grs_path_id(W, L);
+            if (l < 0 || (int64_t)l >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }  // malformed
             const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
             if (f == 0) grs_write(a, sv, nbs, 0, 0, W, base, ncyc);  // the splitter itself
             if (x < 0 || tgt < 0) continue;
@@ -3339,10 +3400,12 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             float2 wc;
             grs_load(a, cur, nbc, wc);
             while (!grs_splitter(a, cur, nbc)) {
+                if (d > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }  // a malformed factor
                 const int fs = nbc.x == prev ? 1 : 0;
                 grs_write(a, cur, nbc, fs, d, W, base, ncyc);
                 prev = cur;
                 cur = fs ? nbc.y : nbc.x;
+                if ((uint32_t)cur >= (uint32_t)a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
                 grs_load(a, cur, nbc, wc);
                 d++;
             }
@@ -3357,12 +3420,14 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             W.pb = cr.z - W.pf - 1;
             W.bb = W.bf ^ 1;  // the far endpoint of the weakest edge
             const int32_t l = key_min_end(W.ks);
+            if (l < 0 || (int64_t)l >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }
             const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
             float2 ws;
             grs_load(a, sv, nbs, ws);
             grs_write(a, sv, nbs, 0, 0, W, base, ncyc);
             int32_t prev = sv, cur = nbs.x, d = 1;
             while (cur != sv) {
+                if (cur < 0 || d > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
                 int2 nbc;
                 float2 wc;
                 grs_load(a, cur, nbc, wc);
@@ -3387,9 +3452,13 @@ __global__ void __launch_bounds__(256) k_grs_out(ForestArgs a) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += 2 * stride) {
         const int64_t v2 = v + stride;
-        const int32_t r0 = __ldcg(a.iperm + v), r1 = v2 < a.N ? __ldcg(a.iperm + v2) : 0;
-        const int4 o0 = __ldcg(a.grs_orec + r0);
-        const int4 o1 = v2 < a.N ? __ldcg(a.grs_orec + r1) : make_int4(0, 0, 0, 0);
+        int32_t r0 = __ldcg(a.iperm + v), r1 = v2 < a.N ? __ldcg(a.iperm + v2) : 0;
+        // every vertex of a valid factor was written by a walk; a malformed one may leave
+        // some unvisited (iperm stale): they get -1s instead of an out-of-range gather
+        const bool ok0 = (uint32_t)r0 < (uint32_t)a.N, ok1 = (uint32_t)r1 < (uint32_t)a.N;
+        if (!ok0 || (v2 < a.N && !ok1)) atomicOr(&a.ctl[kCtlBadGrs], 1);
+        const int4 o0 = ok0 ? __ldcg(a.grs_orec + r0) : make_int4(-1, -1, -1, -1);
+        const int4 o1 = (v2 < a.N && ok1) ? __ldcg(a.grs_orec + r1) : make_int4(-1, -1, -1, -1);
         a.path_id[v] = o0.x;
         a.pos[v] = o0.y;
         a.forest[v] = make_int2(o0.z, o0.w);
@@ -3493,7 +3562,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
             LF_CUDA(launch_pdl(k_grs_cycfind, persistent_grid((const void*)k_grs_cycfind, 256), 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_lenscan, tiles, ET, 0, s, a));
             LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, tiles, (const int*)w.ctl,
-                               (unsigned long long*)n_cycles));
+                               (unsigned long long*)n_cycles, 1));
         }
         {
             LF_PROF(tri ? "grs_emit_tri" : "grs_emit", -1, s);
@@ -3525,13 +3594,13 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     {
         LF_PROF(tri ? "perm_tridiag" : "perm", -1, s);
         LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, tiles, (const int*)w.ctl,
-                           (unsigned long long*)n_cycles));
+                           (unsigned long long*)n_cycles, 0));
         LF_CUDA(launch_pdl(k_perm_tri, persistent_grid((const void*)k_perm_tri, 256), 256, 0, s, N,
                            (const int32_t*)path_id, (const int32_t*)pos, (const int32_t*)w.off,
                            (const int32_t*)w.tsum, (int)LB, (const uint8_t*)w.pdir, (const int2*)forest,
                            (const int2*)pi2, tri ? (const float2*)tri->pi2_val : nullptr,
                            tri ? tri->diag : nullptr, perm, iperm, tri ? tri->a : nullptr,
-                           tri ? tri->b : nullptr, tri ? tri->c : nullptr));
+                           tri ? tri->b : nullptr, tri ? tri->c : nullptr, (const int*)w.ctl));
     }
     return LF_OK;
 }
@@ -3547,9 +3616,9 @@ int forest_stats(const ForestWs& w, int32_t* out, int cap) {
         if (h[kCtlRed1 + i]) steps1 = i + 2;
         if (h[kCtlRed2 + i]) steps2 = i + 2;
     }
-    int v[9] = {h[kCtlCnt1], h[kCtlCnt2], steps1, steps2, h[kCtlStat], h[kCtlStat + 1], h[kCtlStat + 2],
-                h[kCtlStat + 3], h[kCtlStat + 4]};
-    for (int i = 0; i < cap && i < 9; i++) out[i] = v[i];
+    int v[10] = {h[kCtlCnt1], h[kCtlCnt2], steps1, steps2, h[kCtlStat], h[kCtlStat + 1], h[kCtlStat + 2],
+                 h[kCtlStat + 3], h[kCtlStat + 4], h[kCtlBad] | h[kCtlBadGrs]};
+    for (int i = 0; i < cap && i < 10; i++) out[i] = v[i];
     // [16..31]: per-phase cycle sums (units of 1024 cycles; LF_PHASE_TIMING builds only)
     const unsigned long long* ph = reinterpret_cast<const unsigned long long*>(h + 208);
     for (int i = 0; i < 8 && 16 + i < cap; i++) out[16 + i] = (int)(ph[i] >> 10);

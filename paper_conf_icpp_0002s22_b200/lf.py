@@ -20,7 +20,8 @@ ERRORS = {-1: "LF_EINVAL", -2: "LF_ENOMEM", -3: "LF_ECUDA", -4: "LF_ENCCL", -5: 
 EXPORTS = (
     "lf_factor_opts_default", "lf_factor_workspace_size", "lf_factor",
     "lf_linear_forest_workspace_size", "lf_linear_forest", "lf_tridiag", "lf_linear_forest_tridiag",
-    "lf_pipeline_workspace_size", "lf_pipeline_host", "lf_validate_csr",
+    "lf_pipeline_workspace_size", "lf_pipeline_host", "lf_validate_csr", "lf_validate_workspace_size",
+    "lf_validate_factor",
     "lf_last_error", "lf_version", "lf_profile_enable", "lf_profile_collect",
     "lf_forest_stats", "lf_comm_nccl_unique_id", "lf_comm_create_nccl", "lf_comm_create_loopback",
     "lf_comm_destroy", "lf_part_create", "lf_part_destroy", "lf_part_info", "lf_part_factor",
@@ -68,6 +69,10 @@ def load(path: str = LIB_PATH):
     L.lf_pipeline_workspace_size.restype = C.c_size_t
     L.lf_pipeline_host.argtypes = [P, P, P, P, P, P, P, P, P, C.c_size_t, P]
     L.lf_validate_csr.argtypes = [P, P, C.c_size_t, P]
+    L.lf_validate_workspace_size.argtypes = [I64]
+    L.lf_validate_workspace_size.restype = C.c_size_t
+    L.lf_validate_factor.argtypes = [I64, I32, P, P, C.c_size_t, P]
+    L.lf_validate_factor.restype = C.c_int
     L.lf_forest_stats.argtypes = [I64, P, C.c_size_t, P, I32]
     L.lf_comm_nccl_unique_id.argtypes = [P]
     L.lf_comm_create_nccl.argtypes = [P, I32, I32, P]
@@ -309,11 +314,22 @@ def pipeline_host(rowptr_h, col_h, val_h, *, M=5, m=5, k_m=0, p=0.5, seed=0, ws=
     return outs
 
 
-def validate(rowptr, col, val):
+def validate(rowptr, col, val, ws=None):
+    """lf_validate_csr: raises LFError (LF_EINPUT) on a CSR that violates lf_factor's
+    preconditions (include/lf.h)."""
     L = load()
     A = _csr_desc(rowptr, col, val)
-    buf = _ws.get(256)
-    _check(L.lf_validate_csr(C.byref(A), _ptr(buf), 256, _stream()))
+    nb = L.lf_validate_workspace_size(rowptr.numel() - 1)
+    buf = (ws or _ws).get(nb)
+    _check(L.lf_validate_csr(C.byref(A), _ptr(buf), nb, _stream()))
+
+
+def validate_factor(pi, ws=None):
+    """lf_validate_factor on a device pi[N, n] (canonical [0,n]-factor form)."""
+    L = load()
+    N, n = pi.shape
+    buf = (ws or _ws).get(256)
+    _check(L.lf_validate_factor(N, n, _ptr(pi), _ptr(buf), 256, _stream()))
 
 
 def profile_enable(on: bool = True):
@@ -336,7 +352,7 @@ def profile_collect(cap: int = 4096):
 
 FOREST_STATS = ("boundary_cycle_pass", "boundary_rank_pass", "reduced_steps_cycle",
                 "reduced_steps_rank", "splitters_cycle_pass", "unvisited", "fallback_tiles",
-                "splitters_rank_pass", "max_node_scan_steps")
+                "splitters_rank_pass", "max_node_scan_steps", "malformed_input")
 
 
 def forest_stats(N, ws):

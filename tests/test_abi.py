@@ -105,3 +105,20 @@ def test_product_package_does_not_import_oracle():
                 txt = open(os.path.join(dp, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, f
                 assert "lf_oracle" not in txt, f
+
+
+def test_validate_arguments_rejected_before_launch(lib):
+    """lf_validate_csr needs lf_validate_workspace_size(n) bytes; lf_validate_factor checks
+    N, n and NULL before any launch (include/lf.h)."""
+    from paper_conf_icpp_0002s22_b200 import lf
+
+    L = lf.load()
+    assert L.lf_validate_workspace_size(1000) >= 1000 + 256
+    A = lf.CSRDesc(1000, 5000, 0x1000, 0x2000, 0x3000)
+    assert L.lf_validate_csr(C.byref(A), C.c_void_p(0x10000), 256, None) == -2
+    assert b"workspace" in L.lf_last_error()
+    assert L.lf_validate_factor(-1, 2, C.c_void_p(0x1000), C.c_void_p(0x10000), 256, None) == -1
+    assert L.lf_validate_factor(10, 5, C.c_void_p(0x1000), C.c_void_p(0x10000), 256, None) == -1
+    assert L.lf_validate_factor(10, 2, None, C.c_void_p(0x10000), 256, None) == -1
+    assert L.lf_validate_factor(0, 2, None, None, 0, None) == 0
+    assert L.lf_validate_factor(10, 2, C.c_void_p(0x1000), C.c_void_p(0x10000), 128, None) == -2
