@@ -153,10 +153,16 @@ def survey_bytes(N, n, live_rows, live_nnz, with_lf=True):
             "B_alg": int(bf + blf + btri)}
 
 
-def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
-    """Algorithmic HBM bytes of one launch: what the method must move."""
+def kernel_bytes(name, N, Z, n, live_rows, live_nnz, rows_ran=False):
+    """Algorithmic HBM bytes of one launch: what the method must move.
+    Rounds 1..M-1 run in ONE of two kernels (rows_ran: the rows mode did, the cached mode
+    only raised its bail flag); their bytes go to that one."""
     base = name.split("[")[0]
     k = int(name.split("[")[1].rstrip("]")) if "[" in name else -1
+    if base == "rows_propose":  # rounds 1..M-1 as per-round kernels (large graphs)
+        base = "propose"
+    if base == "rows_mutual":
+        base = "mutual"
     if base == "propose":
         if k == 0:  # whole CSR + rowptr; write prop (j, value) and the diagonal
             return 8 * Z + 8 * (N + 1) + 8 * n * N + 4 * N
@@ -169,7 +175,9 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
         Na = live_rows[k]
         nxt = live_rows[k + 1] if k + 1 < len(live_rows) else 0
         return 4 * Na + 8 * n * Na + 8 * n * Na + Na + 4 * nxt
-    if base == "rounds_fused":  # rounds 1..M-1: live rows' propose + mutual traffic
+    if base in ("rounds_fused", "rounds_rows"):  # rounds 1..M-1: live rows' propose + mutual traffic
+        if (base == "rounds_rows") != rows_ran:
+            return 0
         return sum(kernel_bytes(f"propose[{kk}]", N, Z, n, live_rows, live_nnz)
                    + kernel_bytes(f"mutual[{kk}]", N, Z, n, live_rows, live_nnz)
                    for kk in range(1, len(live_rows)))
@@ -191,6 +199,18 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz):
         return 8 * N
     if base == "perm_tridiag":  # write perm, iperm; read forest, pi2, pi2_val, diag; write a, b, c
         return 8 * N + 8 * N + 8 * N + 8 * N + 4 * N + 12 * N
+    # global ruling set: the pack reads the factor, the emit walk writes perm
+    # and iperm and the tridiagonal part (reads signed values and diag, writes a, b, c), the
+    # vertex-order pass writes forest, path_id, pos; walks and the reduced scan are
+    # implementation traffic
+    if base == "grs_pack":
+        return 16 * N
+    if base == "grs_emit_tri":
+        return 8 * N + 12 * N + 12 * N
+    if base == "grs_emit":
+        return 8 * N
+    if base == "grs_out":
+        return 16 * N
     if base == "tridiag":
         return 8 * N + 4 * N + 8 * N + 8 * N + 4 * N + 12 * N
     return 0
@@ -332,7 +352,8 @@ def roofline(rec, cfg, sm_mhz, sm_count):
         return None
     dom = max(kavg, key=kavg.get)
     N, Z, n = rec["N"], rec["nnz"], rec["n"]
-    b = kernel_bytes(dom, N, Z, n, rec["live_rows"], rec["live_nnz"])
+    rows_ran = kavg.get("rounds_rows", 0.0) > 2 * kavg.get("rounds_fused", 0.0)
+    b = kernel_bytes(dom, N, Z, n, rec["live_rows"], rec["live_nnz"], rows_ran)
     peak, kind = load_peaks()
     ach = b / (kavg[dom] * 1e-3) / 1e9
     prof = ncu_profile(cfg)

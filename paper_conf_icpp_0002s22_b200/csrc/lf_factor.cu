@@ -1380,25 +1380,35 @@ __device__ __forceinline__ void write_prop(const RowsArgs& a, int32_t v, int deg
 #ifndef LF_ROWS_T
 #define LF_ROWS_T 256
 #endif
-constexpr int kRowsBud = 640;   // staged entries per warp (3 CTAs of 8 warps per SM)
+#ifndef LF_ROWS_BUD
+#define LF_ROWS_BUD 640
+#endif
+constexpr int kRowsBud = LF_ROWS_BUD;  // staged entries per warp (640: 3 CTAs of 8 warps per SM)
 constexpr int kRowsWarps = LF_ROWS_T / 32;
-struct RowsWarpSmem {
-    int32_t col[kRowsBud];
-    uint32_t val[kRowsBud];
-    uint32_t sjw[kRowsBud];  // the 4-byte state word holding byte col & 3
+template <int BUD>
+struct RowsWarpSmemT {
+    int32_t col[BUD];
+    uint32_t val[BUD];
+    uint32_t sjw[BUD];  // the 4-byte state word holding byte col & 3
     int64_t qrs[64];      // queue of live rows: CSR start
     int32_t qv[64];       //   vertex
     int32_t qlen[64];     //   entries
     int32_t qp[64][4];    //   confirmed slots
     uint8_t qst[64];      //   state byte
 };
+using RowsWarpSmem = RowsWarpSmemT<kRowsBud>;
 struct RowsSmem {
     RowsWarpSmem w[kRowsWarps];
 };
+// the per-round propose kernel of large graphs: 4 warps per CTA, whole 32-row batches
+constexpr int kRowsBudK = 1024, kRowsTK = 128;
+struct RowsSmemK {
+    RowsWarpSmemT<kRowsBudK> w[kRowsTK / 32];
+};
 
 // one batch: the longest prefix of the queue whose aligned ranges fit; returns its size
-template <int NN>
-__device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmem& S, int qcnt, bool charging,
+template <int NN, int BUD>
+__device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmemT<BUD>& S, int qcnt, bool charging,
                                           bool bulk_ok, int64_t nnz, unsigned long long& my_live,
                                           unsigned long long& my_nnz, int& my_prop) {
     const int lane = threadIdx.x & 31;
@@ -1414,7 +1424,7 @@ __device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmem& S, in
         const int y = __shfl_up_sync(0xffffffffu, incl, o);
         if (lane >= o) incl += y;
     }
-    const bool take = has && incl <= kRowsBud;
+    const bool take = has && incl <= BUD;
     const int nb = __popc(__ballot_sync(0xffffffffu, take));
     const int boff = incl - plen;
     const int q0 = boff + (int)(rs - as), q1 = q0 + len;
@@ -1499,8 +1509,8 @@ __device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmem& S, in
     return nb;
 }
 
-template <int NN, int G>
-__device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool charging, RowsWarpSmem& S) {
+template <int NN, int G, int BUD>
+__device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool charging, RowsWarpSmemT<BUD>& S) {
     const int lane = threadIdx.x & 31;
     const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -1551,9 +1561,9 @@ __device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool char
         }
         qcnt += __popc(m);
         __syncwarp();
-        while (qcnt >= 32) qcnt -= rows_batch<NN>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
+        while (qcnt >= 32) qcnt -= rows_batch<NN, BUD>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
     }
-    while (qcnt > 0) qcnt -= rows_batch<NN>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
+    while (qcnt > 0) qcnt -= rows_batch<NN, BUD>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
 #pragma unroll
     for (int off = 16; off >= 1; off >>= 1) {
         my_live += __shfl_xor_sync(0xffffffffu, my_live, off);
@@ -1752,7 +1762,7 @@ __global__ void __launch_bounds__(LF_ROWS_T, 3) k_rounds_rows(RowsArgs a) {
         const int k = a.only_k;
         const bool charging = (k % a.m) != a.k_m;
         const bool last = k == a.M - 1;
-        if (a.only_phase == 0) rows_propose<NN, G>(a, k, charging, S);
+        if (a.only_phase == 0) rows_propose<NN, G, kRowsBud>(a, k, charging, S);
         if (a.only_phase == 1 && *(volatile int32_t*)&a.long_count[k] > 0) rows_long<NN>(a, k, charging);
         if (a.only_phase == 2) {
             if (last && blockIdx.x == 0 && (a.rounds || a.live))
@@ -1765,7 +1775,7 @@ __global__ void __launch_bounds__(LF_ROWS_T, 3) k_rounds_rows(RowsArgs a) {
     for (int k = 1; k < a.M; k++) {
         const bool charging = (k % a.m) != a.k_m;
         const bool last = k == a.M - 1;
-        rows_propose<NN, G>(a, k, charging, S);
+        rows_propose<NN, G, kRowsBud>(a, k, charging, S);
         grid.sync();
         if (*(volatile int32_t*)&a.long_count[k] > 0) {
             rows_long<NN>(a, k, charging);
@@ -1776,6 +1786,40 @@ __global__ void __launch_bounds__(LF_ROWS_T, 3) k_rounds_rows(RowsArgs a) {
         rows_mutual<NN, 2>(a, k, last);
         if (!last) grid.sync();
     }
+}
+
+// Rows mode of large graphs as three kernels per round (propose | long rows | mutual): the
+// propose kernel runs 4-warp CTAs with whole 32-row batches in shared memory, the mutual
+// kernel needs no shared memory and runs at full occupancy with 4 rows per thread in
+// flight -- one cooperative kernel would hold both at the propose kernel's occupancy.
+template <int NN>
+__global__ void __launch_bounds__(kRowsTK) k_rows_propose_k(RowsArgs a) {
+    LF_TL(g_tl_factor, 5);
+    extern __shared__ __align__(16) unsigned char rows_smem_k[];
+    auto& S = reinterpret_cast<RowsSmemK*>(rows_smem_k)->w[threadIdx.x >> 5];
+    pdl_wait();
+    pdl_trigger();
+    if (*(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
+    rows_propose<NN, 1, kRowsBudK>(a, a.only_k, (a.only_k % a.m) != a.k_m, S);
+}
+template <int NN>
+__global__ void __launch_bounds__(256) k_rows_long_k(RowsArgs a) {
+    pdl_wait();
+    pdl_trigger();
+    if (*(volatile const int32_t*)a.bail == 0) return;
+    if (*(volatile int32_t*)&a.long_count[a.only_k] > 0) rows_long<NN>(a, a.only_k, (a.only_k % a.m) != a.k_m);
+}
+template <int NN>
+__global__ void __launch_bounds__(256) k_rows_mutual_k(RowsArgs a) {
+    LF_TL(g_tl_factor, 6);
+    pdl_wait();
+    pdl_trigger();
+    if (*(volatile const int32_t*)a.bail == 0) return;
+    const int k = a.only_k;
+    const bool last = k == a.M - 1;
+    if (last && blockIdx.x == 0 && (a.rounds || a.live))
+        finalize_body(a.flags, a.M, a.m, a.k_m, a.rounds, a.live_part, a.live);
+    rows_mutual<NN, 4>(a, k, last);
 }
 
 // state of round 0 when round 0 is charged (k_m != 0): degree 0 + charge(v, 0)
@@ -2124,7 +2168,6 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_CUDA(cudaLaunchCooperativeKernel(kfn, grid, LF_FUSED_T, args, smem, s));
         }
         {
-            LF_PROF("rounds_rows", -1, s);
             RowsArgs r;
             memset(&r, 0, sizeof(r));
             r.N = N;
@@ -2184,16 +2227,46 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             cfg.attrs = at;
             cfg.numAttrs = pdl_enabled() ? 2 : 1;
             void* args[] = {&r};
-            if (getenv("LF_ROWS_SPLIT")) {  // diagnostics: one launch per phase, each timed
-                static const char* pn[3] = {"rows_propose", "rows_long", "rows_mutual"};
-                for (int k = 1; k < o->M; k++)
-                    for (int ph = 0; ph < 3; ph++) {
-                        r.only_k = k;
-                        r.only_phase = ph;
-                        LF_PROF(pn[ph], k, s);
-                        LF_CUDA(cudaLaunchKernelExC(&cfg, kfn, args));
+            // large graphs: three kernels per round (k_rows_*_k); others: one cooperative kernel
+            const char* sp = getenv("LF_ROWS_SPLIT");
+            const bool split = sp ? strcmp(sp, "0") != 0 : N >= ((int64_t)1 << 22);
+            if (split) {
+                const void* kp = (const void*)k_rows_propose_k<NN>;
+                const int psm = (int)sizeof(RowsSmemK);
+                static bool pattr = false;
+                if (!pattr) {
+                    LF_CUDA(cudaFuncSetAttribute(kp, cudaFuncAttributeMaxDynamicSharedMemorySize, psm));
+                    pattr = true;
+                }
+                cudaLaunchConfig_t c2 = cfg;
+                c2.attrs = at + 1;  // PDL only
+                c2.numAttrs = pdl_enabled() ? 1 : 0;
+                const void* kl = (const void*)k_rows_long_k<NN>;
+                const void* km = (const void*)k_rows_mutual_k<NN>;
+                for (int k = 1; k < o->M; k++) {
+                    r.only_k = k;
+                    {
+                        LF_PROF("rows_propose", k, s);
+                        c2.gridDim = dim3(persistent_grid(kp, kRowsTK, psm));
+                        c2.blockDim = dim3(kRowsTK);
+                        c2.dynamicSmemBytes = psm;
+                        LF_CUDA(cudaLaunchKernelExC(&c2, kp, args));
                     }
+                    {
+                        LF_PROF("rows_long", k, s);
+                        c2.gridDim = dim3(persistent_grid(kl, 256));
+                        c2.blockDim = dim3(256);
+                        c2.dynamicSmemBytes = 0;
+                        LF_CUDA(cudaLaunchKernelExC(&c2, kl, args));
+                    }
+                    {
+                        LF_PROF("rows_mutual", k, s);
+                        c2.gridDim = dim3(persistent_grid(km, 256));
+                        LF_CUDA(cudaLaunchKernelExC(&c2, km, args));
+                    }
+                }
             } else {
+                LF_PROF("rounds_rows", -1, s);
                 LF_CUDA(cudaLaunchKernelExC(&cfg, kfn, args));
             }
         }

@@ -932,6 +932,7 @@ struct ForestArgs {
     const float2* pi2_val;
     const float* diag;
     int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
+    int grs_rec32;         // 1: one 32-byte record per vertex (walk half | emit half)
 };
 
 __device__ __forceinline__ bool is_foreign(int64_t x, const ForestArgs& a) { return x < a.lo || x >= a.hi; }
@@ -2876,7 +2877,7 @@ static size_t scan_temp_bytes(int64_t N) {
     return b > bound ? b : bound;
 }
 
-size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
+size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     ForestWs t;
     const size_t n = (size_t)(N > 0 ? N : 1);
     for (int i = 0; i < 2; i++) {
@@ -2909,12 +2910,13 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w) {
     t.dk2 = c.take<int2>(n);
     t.rdk[0] = c.take<int2>(n);
     t.rdk[1] = c.take<int2>(n);
-    t.grs_rec = c.take<int4>(n);
-    t.grs_erec = c.take<int4>(n);
-    t.grs_orec = c.take<int4>(n);
-    t.grs_bits = c.take<uint32_t>(n / 32 + 1);
-    t.grs_cyc = c.take<int4>(n / 3 + 1);
-    t.grs_cyck = c.take<uint64_t>(n / 3 + 1);
+    const size_t ng = with_grs ? n : 1;  // the partitioned path runs the tile scans only
+    t.grs_rec = c.take<int4>(2 * ng);  // 32-byte records when grs_rec32
+    t.grs_erec = c.take<int4>(ng);
+    t.grs_orec = c.take<int4>(ng);
+    t.grs_bits = c.take<uint32_t>(ng / 32 + 1);
+    t.grs_cyc = c.take<int4>(ng / 3 + 1);
+    t.grs_cyck = c.take<uint64_t>(ng / 3 + 1);
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
     if (w) *w = t;
@@ -3046,7 +3048,7 @@ __device__ __forceinline__ bool grs_splitter(const ForestArgs& a, int32_t v, int
 // what a walk reads per vertex: slots and |w| (one 16-byte packed record, or the two arrays)
 __device__ __forceinline__ void grs_load(const ForestArgs& a, int32_t v, int2& nb, float2& w) {
     if (a.grs_rec) {
-        const int4 r = __ldg(a.grs_rec + v);
+        const int4 r = __ldg(a.grs_rec + ((int64_t)v << a.grs_rec32));
         nb = make_int2(r.x, r.y);
         w = make_float2(__int_as_float(r.z), __int_as_float(r.w));
     } else {
@@ -3055,33 +3057,65 @@ __device__ __forceinline__ void grs_load(const ForestArgs& a, int32_t v, int2& n
     }
 }
 
+// 8 vertices per thread per iteration: one list atomic per 2048 vertices (the splitter
+// counter is a single address; a warp-level atomic per 32 vertices serialised ~4 M times on C5)
+constexpr int kPackV = 8;
 __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
     LF_TL(g_tl_forest, 5);
+    __shared__ int wsum[8];
+    __shared__ int bbase;
     pdl_wait();
     pdl_trigger();
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t b = (int64_t)blockIdx.x * blockDim.x; b < a.N; b += stride) {  // warp-uniform
-        const int64_t v = b + threadIdx.x;
-        const bool in = v < a.N;
-        int2 nb = make_int2(0, 0);
-        float2 w = make_float2(0.f, 0.f);
-        if (in) {
-            nb = __ldg(a.pi2 + v);
-            if (a.grs_rec) w = __ldg(a.pi2_w + v);
-        }
-        const bool spl = in && grs_splitter(a, (int32_t)v, nb);
-        const int p = list_append(a.list1, &a.ctl[kCtlCnt1], (int32_t)v, spl);
-        const unsigned m = __ballot_sync(0xffffffffu, spl);
-        if (in) {
-            a.bidx1[v] = p;
-            a.len[v] = 0;
-            if (a.grs_rec) a.grs_rec[v] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
-            if (a.ta) {
-                const float2 pv = __ldg(a.pi2_val + v);
-                a.grs_erec[v] = make_int4(__float_as_int(pv.x), __float_as_int(pv.y), __float_as_int(__ldg(a.diag + v)), 0);
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t chunk = (int64_t)blockDim.x * kPackV;
+    for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < a.N; c0 += (int64_t)gridDim.x * chunk) {
+        unsigned m[kPackV];
+        int mine = 0;
+#pragma unroll
+        for (int k = 0; k < kPackV; k++) {
+            const int64_t v = c0 + threadIdx.x + (int64_t)k * blockDim.x;  // warp-uniform in/out
+            const bool in = v < a.N;
+            int2 nb = make_int2(0, 0);
+            float2 w = make_float2(0.f, 0.f);
+            if (in) {
+                nb = __ldg(a.pi2 + v);
+                if (a.grs_rec) w = __ldg(a.pi2_w + v);
             }
-            if ((threadIdx.x & 31) == 0) a.grs_bits[v >> 5] = m;  // b is a multiple of 32
+            const bool spl = in && grs_splitter(a, (int32_t)v, nb);
+            m[k] = __ballot_sync(0xffffffffu, spl);
+            mine += __popc(m[k]);
+            if (in) {
+                a.len[v] = 0;
+                if (a.grs_rec) a.grs_rec[v << a.grs_rec32] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
+                if (a.ta) {
+                    const float2 pv = __ldg(a.pi2_val + v);
+                    const int4 e = make_int4(__float_as_int(pv.x), __float_as_int(pv.y), __float_as_int(__ldg(a.diag + v)), 0);
+                    if (a.grs_rec32) a.grs_rec[2 * v + 1] = e;
+                    else a.grs_erec[v] = e;
+                }
+                if (lane == 0) a.grs_bits[v >> 5] = m[k];  // v - lane is a multiple of 32
+            }
         }
+        if (lane == 0) wsum[wid] = mine;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int t = 0;
+            for (int q = 0; q < (int)(blockDim.x >> 5); q++) { const int x = wsum[q]; wsum[q] = t; t += x; }
+            bbase = t ? atomicAdd(&a.ctl[kCtlCnt1], t) : 0;
+        }
+        __syncthreads();
+        int pos = bbase + wsum[wid];
+#pragma unroll
+        for (int k = 0; k < kPackV; k++) {
+            const int64_t v = c0 + threadIdx.x + (int64_t)k * blockDim.x;
+            if ((m[k] >> lane) & 1u) {
+                const int p = pos + __popc(m[k] & ((1u << lane) - 1u));
+                a.list1[p] = (int32_t)v;
+                a.bidx1[v] = p;
+            }
+            pos += __popc(m[k]);
+        }
+        __syncthreads();  // wsum / bbase reused
     }
 }
 
@@ -3344,8 +3378,14 @@ __global__ void __launch_bounds__(ET) k_grs_lenscan(ForestArgs a) {
 }
 
 // one vertex of a walk: the scattered vertex-indexed outputs and the sequential ones at r
+// the emit half of x's record (signed slot values, diag), loaded a step ahead by the walk
+__device__ __forceinline__ int4 grs_eload(const ForestArgs& a, int32_t x) {
+    if (!a.ta) return make_int4(0, 0, 0, 0);
+    return a.grs_rec32 ? __ldg(a.grs_rec + 2 * (int64_t)x + 1) : __ldg(a.grs_erec + x);
+}
+
 __device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 nb, int fslot, int32_t d,
-                                         const GrsWin& W, int32_t base, int& ncyc) {
+                                         const GrsWin& W, int32_t base, int& ncyc, int4 q) {
     const GrsOut o = grs_vertex(x, nb, fslot, d, W);
     const int32_t r = base + o.p - 1;
     if (r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {  // a malformed factor
@@ -3359,7 +3399,6 @@ __device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 n
     a.grs_orec[r] = make_int4(o.l, o.p, o.f.x, o.f.y);
     ncyc += o.ncyc;
     if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
-        const int4 q = __ldg(a.grs_erec + x);
         const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
         const int ss = ((o.dir ^ 1) != o.rs && (o.dir ? nb.x : nb.y) >= 0) ? (o.dir ^ 1) : -1;
         a.ta[r] = ps < 0 ? 0.0f : __int_as_float(ps ? q.y : q.x);
@@ -3392,21 +3431,27 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             const int32_t l = grs_path_id(W, L);
             if (l < 0 || (int64_t)l >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }  // malformed
             const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
-            if (f == 0) grs_write(a, sv, nbs, 0, 0, W, base, ncyc);  // the splitter itself
+            if (f == 0) grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv));  // the splitter itself
             if (x < 0 || tgt < 0) continue;
             if (tgt == sv ? f == 1 : tgt < sv) continue;  // the segment belongs to the other end
             int32_t prev = sv, cur = x, d = 1;
             int2 nbc;
             float2 wc;
             grs_load(a, cur, nbc, wc);
+            int4 qc = grs_eload(a, cur);
             while (!grs_splitter(a, cur, nbc)) {
-                if (d > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }  // a malformed factor
                 const int fs = nbc.x == prev ? 1 : 0;
-                grs_write(a, cur, nbc, fs, d, W, base, ncyc);
+                const int32_t nxt = fs ? nbc.y : nbc.x;
+                if (d > a.N || (uint32_t)nxt >= (uint32_t)a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }  // malformed
+                int2 nbn;
+                float2 wn;
+                grs_load(a, nxt, nbn, wn);  // the next vertex's records are in flight while this one is written
+                const int4 qn = grs_eload(a, nxt);
+                grs_write(a, cur, nbc, fs, d, W, base, ncyc, qc);
                 prev = cur;
-                cur = fs ? nbc.y : nbc.x;
-                if ((uint32_t)cur >= (uint32_t)a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
-                grs_load(a, cur, nbc, wc);
+                cur = nxt;
+                nbc = nbn;
+                qc = qn;
                 d++;
             }
         } else {  // a cycle without splitters, from its recorded vertex (slot 0 ahead)
@@ -3424,15 +3469,15 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
             float2 ws;
             grs_load(a, sv, nbs, ws);
-            grs_write(a, sv, nbs, 0, 0, W, base, ncyc);
+            grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv));
             int32_t prev = sv, cur = nbs.x, d = 1;
             while (cur != sv) {
-                if (cur < 0 || d > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
+                if ((uint32_t)cur >= (uint32_t)a.N || d > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
                 int2 nbc;
                 float2 wc;
                 grs_load(a, cur, nbc, wc);
                 const int fs = nbc.x == prev ? 1 : 0;
-                grs_write(a, cur, nbc, fs, d, W, base, ncyc);
+                grs_write(a, cur, nbc, fs, d, W, base, ncyc, grs_eload(a, cur));
                 prev = cur;
                 cur = fs ? nbc.y : nbc.x;
                 d++;
@@ -3532,6 +3577,9 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         a.grs_rec = (getenv("LF_GRS_PACK") && !strcmp(getenv("LF_GRS_PACK"), "0")) ? nullptr : w.grs_rec;
         a.grs_shift = getenv("LF_GRS_SHIFT") ? atoi(getenv("LF_GRS_SHIFT")) : kGrsShift;
         if (a.grs_shift < 20 || a.grs_shift > 31) a.grs_shift = kGrsShift;
+        // one 32-byte record (walk half | emit half): the emit walk's reads are one sector
+        // per vertex (C5: 29.5 -> 25.7 ms emit, 9.1 -> 9.9 ms walk); LF_GRS_REC32=0: two arrays
+        a.grs_rec32 = (a.grs_rec && !(getenv("LF_GRS_REC32") && !strcmp(getenv("LF_GRS_REC32"), "0"))) ? 1 : 0;
         a.grs_bits = w.grs_bits;
         a.grs_erec = w.grs_erec;
         a.grs_orec = w.grs_orec;

@@ -145,7 +145,7 @@ struct ForestWs {
     int4* grs_cyc;         // [N/3 + 1] (lowest vertex, DK, L, 0) of a cycle without splitters
     uint64_t* grs_cyck;    // [N/3 + 1] its weakest key
 };
-size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w);
+size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs = true);
 
 // Partitioned linear forest: this rank's rows [lo, hi) of the factor;
 // paths and cycles that cross ranks are resolved through an exchanged list of "exit"

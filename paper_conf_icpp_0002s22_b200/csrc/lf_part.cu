@@ -543,12 +543,12 @@ static int lf_setup(Part* p, cudaStream_t s) {
     TRYL(dalloc(p, &p->n_cycles, 1, s));
     {
         Carve c(nullptr, 0);
-        p->lws_bytes = forest_ws_carve(c, no, nullptr) + 256;
+        p->lws_bytes = forest_ws_carve(c, no, nullptr, false) + 256;
         char* w = nullptr;
         TRYL(dalloc(p, &w, p->lws_bytes, s));
         p->lws = w;
         Carve c2(p->lws, p->lws_bytes);
-        forest_ws_carve(c2, no, &p->lw);
+        forest_ws_carve(c2, no, &p->lw, false);
     }
     ForestPartCtx& f = p->fpc;
     memset(&f, 0, sizeof(f));
