@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--cpu-runs", type=int, default=3)
     ap.add_argument("--force-multi", action="store_true",
                     help="use the row-partitioned multi-GPU path even at one rank (testing)")
+    ap.add_argument("--grid", type=int, default=C5_N,
+                    help="N > 1 / --force-multi: the C5 recipe on grid^3 (512 = C5; smaller for tests)")
     return ap.parse_args()
 
 
@@ -448,7 +450,7 @@ def run_multi(args, ws, rank, local):
     _build.build()
     lf.load()
     lfgen.gpu.build()
-    n = C5_N
+    n = args.grid
     bounds = dist.slab_bounds(n, n * n, ws)
     z0, z1 = int(bounds[rank]) // (n * n), int(bounds[rank + 1]) // (n * n)
     rpd, cold, vald = lfgen.gpu.grid27_rows(n, z0, z1, seed=5)
@@ -556,8 +558,9 @@ def run_multi(args, ws, rank, local):
             "dtype": "f32",
             "data": "synthetic",
             "config": {
-                "workload": CONFIG_DESC["C5"] + f", z-slabs of {n // ws} planes per rank",
-                "name": "C5", "N": N, "E": E, "nnz": Z, "n": 2, "M": 5, "m": 5, "k_m": 0,
+                "workload": (CONFIG_DESC["C5"] if n == C5_N else f"C5 recipe (27-pt, seed 5) on {n}^3")
+                + f", z-slabs of {n // ws} planes per rank",
+                "name": "C5" if n == C5_N else f"C5-{n}", "N": N, "E": E, "nnz": Z, "n": 2, "M": 5, "m": 5, "k_m": 0,
                 "parallelism": f"row-partitioned z-slabs x{ws}, NCCL halo exchange + boundary-end list",
                 "halo_entries_per_exchange_rank0": info["halo_sent"],
                 "l2": "flushed between steps (512 MB write)", "graph": False,

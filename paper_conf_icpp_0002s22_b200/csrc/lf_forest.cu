@@ -3,27 +3,23 @@
 //
 // The paper runs its bidirectional scan (stride-doubling pointer jumping over the
 // unoriented doubly-linked list, end markers -(e+1), ping-pong buffers) as ceil(log2 N)
-// global launches over all N vertices, twice (cycles, then positions).  On B200 the same
-// scan runs hierarchically:
+// global launches over all N vertices, twice (cycles, then positions).  Here every scan
+// level carries the FULL window of a vertex per direction (pointer, edges covered, minimum
+// edge key, DK = distance to that edge's near endpoint), so ONE pass breaks the cycles and
+// ranks the paths, in one of two organisations:
 //
-//   1. block-local scan (k_lf_local1): a CTA loads 2048 consecutive vertices into shared
-//      memory and runs the bidirectional scan on the links that stay inside the block
-//      (a link to another block is an "exit" and ends the local walk like a path end).
-//      Every vertex learns the local terminal it reaches in each direction, the local
-//      distance and the minimum edge key on the way; cycles that lie inside the block are
-//      complete.  Only "boundary" vertices (with a link leaving the block) go on.
-//   2. reduced scan (k_red_scan, one cooperative kernel): the same bidirectional scan on
-//      the reduced graph whose nodes are boundary vertices and whose links are either a
-//      cross-block edge or a whole local segment (weighted by its length and minimum
-//      key).  It leaves as soon as every node is done.
-//   3. expand (k_lf_local2 / k_lf_local3): the stored local result of each vertex (its
-//      two local terminals and distances, 4-8 bytes) is combined with the reduced results
-//      of those terminals.
+//   tile path (graphs whose paths stay in 1024-id tiles: C1-C3) -- k_lf_full1 ranks each
+//     tile in shared memory (run contraction + ruling set) and emits one record per
+//     boundary vertex; k_red_full scans that reduced list (one cluster through DSMEM, or
+//     the whole grid, cooperative launch); k_lf_full2 expands; k_tile_prefix + k_perm_tri
+//     write the permutation and the tridiagonal copy;
+//   global ruling set (paths that leave every tile: C4, C5) -- k_grs_pack,
+//     k_grs_walk (splitter-to-splitter walks), k_red_full on the splitter list, k_grs_len /
+//     k_grs_cycfind / k_grs_lenscan (path offsets), k_grs_emit (one more walk per segment
+//     writing perm and a/b/c sequentially at the new index) and k_grs_out.
 //
-// Step (1) (cycles) and step (2) (positions) each take one local + one reduced pass; the
-// forest is written between them by the fused kernel k_lf_local2, which also runs the
-// step-(2) local scan on the freshly broken forest while it is still in shared memory.
-// Step (3) is a CUB exclusive scan of path lengths plus a scatter.
+// The row-partitioned multi-GPU path (forest_part_run) still uses the older two-pass
+// kernels k_lf_local1/2/3 + k_red_scan: its exit-record exchange is built on them.
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
