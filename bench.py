@@ -428,7 +428,7 @@ def run_reference(args):
         "e2e": {"value": round(val, 3), "unit": "Medges/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(out), flush=True)
+    emit_line(out)
 
 
 # ---------------------------------------------------------------------------
@@ -574,7 +574,7 @@ def run_multi(args, ws, rank, local):
         }
         if e2e:
             out["e2e"] = e2e
-        print(json.dumps(out), flush=True)
+        emit_line(out)
     part.close()
     comm.close()
     tdist.destroy_process_group()
@@ -614,7 +614,29 @@ def e2e_single(torch, lf, g, steps):
             "host_buffers": "pinned" if pinned else "pageable"}
 
 
+_STDOUT_FD = None
+
+
+def emit_line(obj):
+    """The one JSON line on the real stdout (native libraries' banners -- e.g. NCCL's version
+    line -- were sent to stderr by quiet_native_stdout)."""
+    line = (json.dumps(obj) + "\n").encode()
+    if _STDOUT_FD is not None:
+        os.write(_STDOUT_FD, line)
+    else:
+        sys.stdout.write(line.decode())
+        sys.stdout.flush()
+
+
+def quiet_native_stdout():
+    global _STDOUT_FD
+    sys.stdout.flush()
+    _STDOUT_FD = os.dup(1)
+    os.dup2(2, 1)
+
+
 def main():
+    quiet_native_stdout()
     args = parse()
     if args.impl == "reference":
         run_reference(args)
@@ -709,7 +731,7 @@ def main():
         out["e2e"] = e2e
     if cpu:
         out["cpu_baseline"] = cpu
-    print(json.dumps(out), flush=True)
+    emit_line(out)
 
 
 if __name__ == "__main__":

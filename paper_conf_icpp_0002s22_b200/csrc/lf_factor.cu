@@ -1309,6 +1309,8 @@ struct RowsArgs {
                                      // 2 mutual) of round only_k (per-phase profiling launches)
     int32_t* wl[2];                  // worklists: round k's live rows in wl[k & 1] (mutual(k-1)
     int32_t* counts;                 //   appends them, roughly in id order), sizes counts[k % 3]
+    int64_t row_base;                // partitioned runs: CSR row of vertex v is v - row_base,
+    int64_t gid_off;                 //   its global id (charges) v + gid_off; NULL bail = always run
 };
 constexpr int kRowsT = 4;  // entries per lane per pass (loads in flight per lane)
 
@@ -1533,8 +1535,8 @@ __device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool char
         int32_t p[NN];
         if (valid) {  // live: deg < n, so pi's unused slots hold -1
             st = __ldcg(a.state + v);
-            rs = __ldg(a.rowptr + v);
-            re = __ldg(a.rowptr + v + 1);
+            rs = __ldg(a.rowptr + (v - a.row_base));
+            re = __ldg(a.rowptr + (v - a.row_base) + 1);
 #pragma unroll
             for (int s2 = 0; s2 < NN; s2++) p[s2] = __ldcg(a.pi + (int64_t)v * NN + s2);
         }
@@ -1623,7 +1625,7 @@ __device__ __forceinline__ void rows_long(const RowsArgs& a, int k, bool chargin
     for (int i = blockIdx.x; i < cnt; i += gridDim.x) {
         const int32_t v = __ldcg(a.long_rows + i);
         const uint32_t sv = __ldcg(a.state + v);
-        const int64_t rs = __ldg(a.rowptr + v), re = __ldg(a.rowptr + v + 1);
+        const int64_t rs = __ldg(a.rowptr + (v - a.row_base)), re = __ldg(a.rowptr + (v - a.row_base) + 1);
         const int deg = sv & ST_DEG;
         int32_t p[NN];
 #pragma unroll
@@ -1729,7 +1731,7 @@ __device__ __forceinline__ void rows_mutual(const RowsArgs& a, int k, bool last)
                 keepb[b] = pj[b][0] != PROP_RETIRED && deg < NN;
                 if (keepb[b]) {
                     ns |= ST_LIVE;
-                    if (next_charging && charge_bit((uint32_t)v, (uint32_t)(k + 1), a.seed, a.thr)) ns |= ST_CHARGE;
+                    if (next_charging && charge_bit((uint32_t)(v + a.gid_off), (uint32_t)(k + 1), a.seed, a.thr)) ns |= ST_CHARGE;
                 }
             }
             if (ns != st[b]) a.state[v] = (uint8_t)ns;
@@ -1757,7 +1759,7 @@ __global__ void __launch_bounds__(LF_ROWS_T, 3) k_rounds_rows(RowsArgs a) {
     extern __shared__ __align__(16) unsigned char rows_smem[];
     RowsWarpSmem& S = reinterpret_cast<RowsSmem*>(rows_smem)->w[threadIdx.x >> 5];
     pdl_wait();
-    if (*(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
+    if (a.bail && *(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
     if (a.only_k > 0) {
         const int k = a.only_k;
         const bool charging = (k % a.m) != a.k_m;
@@ -1788,6 +1790,60 @@ __global__ void __launch_bounds__(LF_ROWS_T, 3) k_rounds_rows(RowsArgs a) {
     }
 }
 
+// Deferred long rows of a per-round propose (hub rows of power-law graphs; C4's reach 44 k
+// entries): a CTA per row instead of a warp, with propose_phase's semantics for one row
+// (round 0 also captures the diagonal; state / pi may be NULL in a fresh round 0).
+template <int NN>
+__global__ void __launch_bounds__(256) k_propose_long_blk(ProposeArgs pa) {
+    LF_TL(g_tl_factor, 7);
+    pdl_wait();
+    pdl_trigger();
+    const int cnt = *(volatile const int32_t*)pa.wl_count;
+    RowsArgs ra;
+    memset(&ra, 0, sizeof(ra));
+    ra.col = pa.col;
+    ra.val = pa.val;
+    ra.state = const_cast<uint8_t*>(pa.state);
+    unsigned long long my_live = 0, my_nnz = 0;
+    int my_prop = 0;
+    for (int i = blockIdx.x; i < cnt; i += gridDim.x) {
+        const int32_t v = __ldcg(pa.wl + i);
+        const int64_t row = (int64_t)v - pa.row_base;
+        const int64_t rs = __ldg(pa.rowptr + row), re = __ldg(pa.rowptr + row + 1);
+        const uint32_t sv = pa.state ? (uint32_t)__ldcg(pa.state + v) : 0u;
+        const int deg = sv & ST_DEG;
+        int32_t p[NN];
+#pragma unroll
+        for (int s2 = 0; s2 < NN; s2++) p[s2] = (pa.pi && deg > 0) ? __ldcg(pa.pi + (int64_t)v * NN + s2) : -1;
+        if (pa.diag) {  // the diagonal entry (L231: not an edge), at most one per row
+            for (int64_t e = rs + threadIdx.x; e < re; e += blockDim.x)
+                if (__ldg(pa.col + e) == v) pa.diag[v] = __ldg(pa.val + e);
+        }
+        uint64_t top[NN];
+        uint32_t theta0;
+        block_row_topn<NN>(ra, v, rs, re, p, (sv & ST_CHARGE) ? 1u : 0u, pa.charging != 0, top, theta0);
+        if (threadIdx.x == 0) {
+            const int need = NN - deg;
+            int np = 0;
+#pragma unroll
+            for (int s2 = 0; s2 < NN; s2++) {
+                const uint64_t tk = s2 < need ? top[s2] : 0ull;
+                pa.prop_j[(int64_t)v * NN + s2] = tk ? key_col(tk) : ((s2 == 0 && !theta0) ? PROP_RETIRED : -1);
+                pa.prop_v[(int64_t)v * NN + s2] = tk ? key_val(tk) : 0.0f;
+                np += tk != 0;
+            }
+            if (theta0) { my_live++; my_nnz += (unsigned long long)(re - rs); }
+            my_prop |= np > 0;
+        }
+    }
+    if (threadIdx.x == 0) {
+        const int slot = blockIdx.x & 63;
+        if (pa.live_rows && my_live) atomicAdd(pa.live_rows + slot, my_live);
+        if (pa.live_nnz && my_nnz) atomicAdd(pa.live_nnz + slot, my_nnz);
+        if (my_prop && *(volatile int*)pa.proposed == 0) atomicOr(pa.proposed, 1);
+    }
+}
+
 // Rows mode of large graphs as three kernels per round (propose | long rows | mutual): the
 // propose kernel runs 4-warp CTAs with whole 32-row batches in shared memory, the mutual
 // kernel needs no shared memory and runs at full occupancy with 4 rows per thread in
@@ -1799,14 +1855,14 @@ __global__ void __launch_bounds__(kRowsTK) k_rows_propose_k(RowsArgs a) {
     auto& S = reinterpret_cast<RowsSmemK*>(rows_smem_k)->w[threadIdx.x >> 5];
     pdl_wait();
     pdl_trigger();
-    if (*(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
+    if (a.bail && *(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
     rows_propose<NN, 1, kRowsBudK>(a, a.only_k, (a.only_k % a.m) != a.k_m, S);
 }
 template <int NN>
 __global__ void __launch_bounds__(256) k_rows_long_k(RowsArgs a) {
     pdl_wait();
     pdl_trigger();
-    if (*(volatile const int32_t*)a.bail == 0) return;
+    if (a.bail && *(volatile const int32_t*)a.bail == 0) return;
     if (*(volatile int32_t*)&a.long_count[a.only_k] > 0) rows_long<NN>(a, a.only_k, (a.only_k % a.m) != a.k_m);
 }
 template <int NN>
@@ -1814,7 +1870,7 @@ __global__ void __launch_bounds__(256) k_rows_mutual_k(RowsArgs a) {
     LF_TL(g_tl_factor, 6);
     pdl_wait();
     pdl_trigger();
-    if (*(volatile const int32_t*)a.bail == 0) return;
+    if (a.bail && *(volatile const int32_t*)a.bail == 0) return;
     const int k = a.only_k;
     const bool last = k == a.M - 1;
     if (last && blockIdx.x == 0 && (a.rounds || a.live))
@@ -1989,6 +2045,49 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         LF_CUDA(cudaGetLastError());
     }
     int rounds_host = -1;
+    // partitioned runs (rounds cannot be fused: two halo exchanges per round) use the rows-mode
+    // kernels per round for large row ranges (LF_PART_ROWS=0/1 overrides)
+    RowsArgs pr;
+    memset(&pr, 0, sizeof(pr));
+    const char* prs = getenv("LF_PART_ROWS");
+    const bool rows_part = part && !o->until_maximal && o->M <= kMaxFlagRounds &&
+                           (prs ? strcmp(prs, "0") != 0 : N >= ((int64_t)1 << 20));
+    if (rows_part) {
+        pr.N = N;
+        pr.rowptr = A->rowptr;
+        pr.col = A->col;
+        pr.val = A->val;
+        pr.state = w.state;
+        pr.pi = pi;
+        pr.pi_w = pi_w;
+        pr.pi_val = pi_val;
+        pr.prop_j = w.prop_j;
+        pr.prop_v = w.prop_v;
+        pr.flags = w.flags;
+        pr.live_part = live ? w.live_part : nullptr;
+        pr.long_rows = w.long_rows;
+        pr.long_count = w.long_count;
+        pr.defer_len = 128;
+        pr.M = o->M;
+        pr.m = o->m;
+        pr.k_m = o->k_m;
+        pr.seed = o->seed;
+        pr.thr = thr;
+        pr.bail = nullptr;    // always run
+        pr.rounds = nullptr;  // the host's pre_finalize hook reduces the flags first: k_finalize
+        pr.live = nullptr;
+        pr.wl[0] = w.wl[0];
+        pr.wl[1] = w.wl[1];
+        pr.counts = w.counts;
+        pr.row_base = row_base;
+        pr.gid_off = gid_off;
+        static bool pattr = false;
+        if (!pattr) {
+            LF_CUDA(cudaFuncSetAttribute((const void*)k_rows_propose_k<NN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)sizeof(RowsSmemK)));
+            pattr = true;
+        }
+    }
     // rounds 1..M-1 in one cooperative kernel unless the host must check maximality
     const bool fuse = !o->until_maximal && o->M > 1 && !part;
     const int M_loop = fuse ? 1 : M;
@@ -2033,6 +2132,11 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
 #else
                 launch_propose_stream<NN>(Gt, pa, s);
 #endif
+            } else if (rows_part) {
+                pr.only_k = k;
+                LF_CUDA(launch_pdl(k_rows_propose_k<NN>,
+                                   persistent_grid((const void*)k_rows_propose_k<NN>, kRowsTK, sizeof(RowsSmemK)),
+                                   kRowsTK, sizeof(RowsSmemK), s, pr));
             } else {
                 pa.defer_len = 32 * G;
                 launch_propose<NN>(G, pa, grid_p, s);
@@ -2040,13 +2144,14 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_CUDA(cudaGetLastError());
         }
         {
-            // long rows of this round: one warp per row
+            // long rows of this round: one CTA per row
             LF_PROF("propose_long", k, s);
             ProposeArgs pl = pa;
             pl.wl = w.long_rows;
             pl.wl_count = pa.defer_count;
             pl.defer_len = INT64_MAX;
-            LF_CUDA(launch_pdl(k_propose<NN, 32>, grid_p, 256, 0, s, pl));
+            LF_CUDA(launch_pdl(k_propose_long_blk<NN>, persistent_grid((const void*)k_propose_long_blk<NN>, 256),
+                               256, 0, s, pl));
         }
 
         if (o->until_maximal && (k % o->m) == o->k_m) {
@@ -2104,6 +2209,10 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
                 const int64_t per = 256 * (int64_t)kMutual0Rows;
                 const int64_t g = (N + per - 1) / per;
                 LF_CUDA(launch_pdl(k_mutual0<NN, kMutual0Rows>, (int)(g < (1 << 20) ? g : (1 << 20)), 256, 0, s, ma));
+            } else if (rows_part && !fresh) {
+                pr.only_k = k;
+                LF_CUDA(launch_pdl(k_rows_mutual_k<NN>, persistent_grid((const void*)k_rows_mutual_k<NN>, 256), 256, 0,
+                                   s, pr));
             } else {
                 LF_CUDA(launch_pdl(k_mutual<NN>, grid_m, 256, 0, s, ma));
             }

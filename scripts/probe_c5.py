@@ -12,12 +12,17 @@ import torch  # noqa: E402
 import lfgen.gpu  # noqa: E402
 from paper_conf_icpp_0002s22_b200 import _build, lf  # noqa: E402
 
-n = int(sys.argv[1]) if len(sys.argv) > 1 else 512
+n = sys.argv[1] if len(sys.argv) > 1 else "512"   # an n (C5 recipe on n^3) or a config name
 variants = sys.argv[2:] or [""]
 _build.build()
 lf.load()
 lfgen.gpu.build()
-rp, col, val = lfgen.gpu.grid27_rows(n, 0, n, seed=5)
+if n.isdigit():
+    n = int(n)
+    rp, col, val = lfgen.gpu.grid27_rows(n, 0, n, seed=5)
+else:
+    A = lfgen.config(n)
+    rp, col, val = (torch.from_numpy(x).cuda() for x in (A.rowptr, A.col, A.val))
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 P = lf.Pipeline(rp, col, val)
 ref = None

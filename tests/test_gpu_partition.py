@@ -54,10 +54,15 @@ CASES = [
 ]
 
 
+@pytest.mark.parametrize("rows", ["0", "1"])
 @pytest.mark.parametrize("name,make,bspec", CASES, ids=[c[0] for c in CASES])
 @pytest.mark.parametrize("G", [2, 3, 4])
-def test_partitioned_factor_matches_oracle(torch_cuda, oracle_mod, name, make, bspec, G):
+def test_partitioned_factor_matches_oracle(torch_cuda, oracle_mod, monkeypatch, name, make, bspec, G, rows):
+    """rows = 1: rounds 1..M-1 through the rows-mode kernels (k_rows_*_k),
+    the default for partitions of >= 2^20 rows; rows = 0: the per-round worklist kernels."""
     from paper_conf_icpp_0002s22_b200 import dist
+
+    monkeypatch.setenv("LF_PART_ROWS", rows)
 
     A = make()
     if bspec == "slab":
@@ -84,9 +89,12 @@ def test_partitioned_factor_matches_oracle(torch_cuda, oracle_mod, name, make, b
         assert inf["ghosts_below"] + inf["ghosts_above"] == int(recv.sum())
 
 
+@pytest.mark.parametrize("rows", ["0", "1"])
 @pytest.mark.parametrize("m,k_m,seed", [(5, 1, 0), (1, 0, 3), (3, 2, 17)])
-def test_partitioned_charge_schedules(torch_cuda, oracle_mod, m, k_m, seed):
+def test_partitioned_charge_schedules(torch_cuda, oracle_mod, monkeypatch, m, k_m, seed, rows):
     from paper_conf_icpp_0002s22_b200 import dist
+
+    monkeypatch.setenv("LF_PART_ROWS", rows)
 
     A = lfgen.fem27_bricks(10)
     bounds = dist.plan_bounds(A.rowptr, 3)
@@ -126,11 +134,14 @@ def _ring_and_path(N):
     return lfgen.csr_from_edges(N, s2, t2, w2)
 
 
+@pytest.mark.parametrize("rows", ["0", "1"])
 @pytest.mark.parametrize("name,make", LF_CASES, ids=[c[0] for c in LF_CASES])
 @pytest.mark.parametrize("G", [2, 3, 5])
-def test_partitioned_linear_forest_matches_oracle(torch_cuda, oracle_mod, name, make, G):
+def test_partitioned_linear_forest_matches_oracle(torch_cuda, oracle_mod, monkeypatch, name, make, G, rows):
     """Boundary-end list ranking across partitions equals the oracle's walk (§8(e))."""
     from paper_conf_icpp_0002s22_b200 import dist
+
+    monkeypatch.setenv("LF_PART_ROWS", rows)
 
     torch = torch_cuda
     A = make()
