@@ -917,8 +917,6 @@ struct ForestArgs {
     // global ruling set (k_grs_*): packed records, visit bitmap, splitter-free cycles, and
     // the permutation / tridiagonal outputs its last walk writes directly
     int4* grs_rec;
-    int4* grs_erec;        // [N] (signed slot values, diag, 0): the emit walk's per-vertex reads
-    int4* grs_orec;        // [N] at the new index r: (path_id, pos, forest) -> k_grs_out
     uint32_t* grs_bits;
     int4* grs_cyc;
     uint64_t* grs_cyck;
@@ -928,7 +926,6 @@ struct ForestArgs {
     const float2* pi2_val;
     const float* diag;
     int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
-    int grs_rec32;         // 1: one 32-byte record per vertex (walk half | emit half)
 };
 
 __device__ __forceinline__ bool is_foreign(int64_t x, const ForestArgs& a) { return x < a.lo || x >= a.hi; }
@@ -2907,9 +2904,7 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.rdk[0] = c.take<int2>(n);
     t.rdk[1] = c.take<int2>(n);
     const size_t ng = with_grs ? n : 1;  // the partitioned path runs the tile scans only
-    t.grs_rec = c.take<int4>(2 * ng);  // 32-byte records when grs_rec32
-    t.grs_erec = c.take<int4>(ng);
-    t.grs_orec = c.take<int4>(ng);
+    t.grs_rec = c.take<int4>(2 * ng);  // one 32-byte record per vertex
     t.grs_bits = c.take<uint32_t>(ng / 32 + 1);
     t.grs_cyc = c.take<int4>(ng / 3 + 1);
     t.grs_cyck = c.take<uint64_t>(ng / 3 + 1);
@@ -3041,16 +3036,17 @@ constexpr int kCtlCyc = 134;      // splitter-free cycles recorded by k_grs_cycf
 __device__ __forceinline__ bool grs_splitter(const ForestArgs& a, int32_t v, int2 nb) {
     return nb.x < 0 || nb.y < 0 || (((uint32_t)v * 0x9E3779B1u) >> a.grs_shift) == 0u;
 }
-// what a walk reads per vertex: slots and |w| (one 16-byte packed record, or the two arrays)
+// The 32-byte record of vertex v (one sector; a random visit costs one DRAM access):
+//   [2v]     slots (nb.x, nb.y) | |w| per slot            -- read by every walk
+//   [2v + 1] signed slot values | diag | 0                -- read by the emit walk
+// The emit walk then overwrites, in the sector it has just read, [2v].zw with the forest
+// slots and [2v + 1] with (path_id, pos, iperm): k_grs_out copies them to the output
+// arrays in one coalesced pass instead of scattered stores.  Other walks
+// only read [2v].xy of a splitter concurrently, which stays.
 __device__ __forceinline__ void grs_load(const ForestArgs& a, int32_t v, int2& nb, float2& w) {
-    if (a.grs_rec) {
-        const int4 r = __ldg(a.grs_rec + ((int64_t)v << a.grs_rec32));
-        nb = make_int2(r.x, r.y);
-        w = make_float2(__int_as_float(r.z), __int_as_float(r.w));
-    } else {
-        nb = __ldg(a.pi2 + v);
-        w = __ldg(a.pi2_w + v);
-    }
+    const int4 r = __ldcg(a.grs_rec + 2 * (int64_t)v);
+    nb = make_int2(r.x, r.y);
+    w = make_float2(__int_as_float(r.z), __int_as_float(r.w));
 }
 
 // 8 vertices per thread per iteration: one list atomic per 2048 vertices (the splitter
@@ -3075,20 +3071,18 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
             float2 w = make_float2(0.f, 0.f);
             if (in) {
                 nb = __ldg(a.pi2 + v);
-                if (a.grs_rec) w = __ldg(a.pi2_w + v);
+                w = __ldg(a.pi2_w + v);
             }
             const bool spl = in && grs_splitter(a, (int32_t)v, nb);
             m[k] = __ballot_sync(0xffffffffu, spl);
             mine += __popc(m[k]);
             if (in) {
                 a.len[v] = 0;
-                if (a.grs_rec) a.grs_rec[v << a.grs_rec32] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
-                if (a.ta) {
-                    const float2 pv = __ldg(a.pi2_val + v);
-                    const int4 e = make_int4(__float_as_int(pv.x), __float_as_int(pv.y), __float_as_int(__ldg(a.diag + v)), 0);
-                    if (a.grs_rec32) a.grs_rec[2 * v + 1] = e;
-                    else a.grs_erec[v] = e;
-                }
+                a.grs_rec[2 * v] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
+                // emit half; .w = -1 until the emit walk writes the vertex (k_grs_out checks it)
+                const float2 pv = a.ta ? __ldg(a.pi2_val + v) : make_float2(0.f, 0.f);
+                const float dg = a.ta ? __ldg(a.diag + v) : 0.f;
+                a.grs_rec[2 * v + 1] = make_int4(__float_as_int(pv.x), __float_as_int(pv.y), __float_as_int(dg), -1);
                 if (lane == 0) a.grs_bits[v >> 5] = m[k];  // v - lane is a multiple of 32
             }
         }
@@ -3377,7 +3371,7 @@ __global__ void __launch_bounds__(ET) k_grs_lenscan(ForestArgs a) {
 // the emit half of x's record (signed slot values, diag), loaded a step ahead by the walk
 __device__ __forceinline__ int4 grs_eload(const ForestArgs& a, int32_t x) {
     if (!a.ta) return make_int4(0, 0, 0, 0);
-    return a.grs_rec32 ? __ldg(a.grs_rec + 2 * (int64_t)x + 1) : __ldg(a.grs_erec + x);
+    return __ldcg(a.grs_rec + 2 * (int64_t)x + 1);
 }
 
 __device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 nb, int fslot, int32_t d,
@@ -3388,11 +3382,11 @@ __device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 n
         atomicOr(&a.ctl[kCtlBadGrs], 1);
         return;
     }
-    // one scattered store (iperm); the rest goes to index r, consecutive along the walk;
-    // k_grs_out moves path_id / pos / forest to vertex order with one gather per vertex
-    a.iperm[x] = r;
+    // perm, a, b, c go to index r, consecutive along the walk; the vertex-indexed outputs go
+    // into x's own record sector (just read): k_grs_out copies them out coalesced
     a.perm[r] = x;
-    a.grs_orec[r] = make_int4(o.l, o.p, o.f.x, o.f.y);
+    a.grs_rec[2 * (int64_t)x] = make_int4(nb.x, nb.y, o.f.x, o.f.y);
+    a.grs_rec[2 * (int64_t)x + 1] = make_int4(o.l, o.p, r, 0);
     ncyc += o.ncyc;
     if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
         const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
@@ -3486,28 +3480,22 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
     if ((threadIdx.x & 31) == 0 && ncyc && a.n_cycles) atomicAdd(a.n_cycles, (unsigned long long)ncyc);
 }
 
-// vertex-order outputs from the records k_grs_emit left at each vertex's new index
+// vertex-order outputs from the records k_grs_emit left in each vertex's record: one
+// coalesced pass (32 bytes read, 20 written per vertex)
 __global__ void __launch_bounds__(256) k_grs_out(ForestArgs a) {
     LF_TL(g_tl_forest, 11);
     pdl_wait();
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += 2 * stride) {
-        const int64_t v2 = v + stride;
-        int32_t r0 = __ldcg(a.iperm + v), r1 = v2 < a.N ? __ldcg(a.iperm + v2) : 0;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += stride) {
+        const int4 f = __ldcs(a.grs_rec + 2 * v), o = __ldcs(a.grs_rec + 2 * v + 1);
         // every vertex of a valid factor was written by a walk; a malformed one may leave
-        // some unvisited (iperm stale): they get -1s instead of an out-of-range gather
-        const bool ok0 = (uint32_t)r0 < (uint32_t)a.N, ok1 = (uint32_t)r1 < (uint32_t)a.N;
-        if (!ok0 || (v2 < a.N && !ok1)) atomicOr(&a.ctl[kCtlBadGrs], 1);
-        const int4 o0 = ok0 ? __ldcg(a.grs_orec + r0) : make_int4(-1, -1, -1, -1);
-        const int4 o1 = (v2 < a.N && ok1) ? __ldcg(a.grs_orec + r1) : make_int4(-1, -1, -1, -1);
-        a.path_id[v] = o0.x;
-        a.pos[v] = o0.y;
-        a.forest[v] = make_int2(o0.z, o0.w);
-        if (v2 < a.N) {
-            a.path_id[v2] = o1.x;
-            a.pos[v2] = o1.y;
-            a.forest[v2] = make_int2(o1.z, o1.w);
-        }
+        // some unvisited (the record still holds the packed input): flag them, -1 outputs
+        const bool ok = (uint32_t)o.z < (uint32_t)a.N && o.w == 0 && (uint32_t)o.x < (uint32_t)a.N && o.y >= 1;
+        if (!ok) atomicOr(&a.ctl[kCtlBadGrs], 1);
+        a.path_id[v] = ok ? o.x : -1;
+        a.pos[v] = ok ? o.y : -1;
+        a.iperm[v] = ok ? o.z : -1;
+        a.forest[v] = ok ? make_int2(f.z, f.w) : make_int2(-1, -1);
     }
 }
 
@@ -3570,15 +3558,10 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     const int tiles = (int)((N + LB - 1) / LB);
     if (use_grs(N)) {
         a.list1 = w.list1;
-        a.grs_rec = (getenv("LF_GRS_PACK") && !strcmp(getenv("LF_GRS_PACK"), "0")) ? nullptr : w.grs_rec;
+        a.grs_rec = w.grs_rec;
         a.grs_shift = getenv("LF_GRS_SHIFT") ? atoi(getenv("LF_GRS_SHIFT")) : kGrsShift;
         if (a.grs_shift < 20 || a.grs_shift > 31) a.grs_shift = kGrsShift;
-        // one 32-byte record (walk half | emit half): the emit walk's reads are one sector
-        // per vertex (C5: 29.5 -> 25.7 ms emit, 9.1 -> 9.9 ms walk); LF_GRS_REC32=0: two arrays
-        a.grs_rec32 = (a.grs_rec && !(getenv("LF_GRS_REC32") && !strcmp(getenv("LF_GRS_REC32"), "0"))) ? 1 : 0;
         a.grs_bits = w.grs_bits;
-        a.grs_erec = w.grs_erec;
-        a.grs_orec = w.grs_orec;
         a.grs_cyc = w.grs_cyc;
         a.grs_cyck = w.grs_cyck;
         a.perm = perm;
