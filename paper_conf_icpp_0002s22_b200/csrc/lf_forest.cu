@@ -3374,31 +3374,75 @@ __device__ __forceinline__ int4 grs_eload(const ForestArgs& a, int32_t x) {
     return __ldcg(a.grs_rec + 2 * (int64_t)x + 1);
 }
 
+// The outputs at the new index (perm, a, b, c) are consecutive along a walk, but one
+// thread fills a 32-byte sector only every 8 steps, and a partially written sector that
+// leaves L2 costs a read-modify-write in DRAM.  Each thread therefore collects the current
+// sector of the four arrays in shared memory and stores it when the walk moves on: whole
+// sectors as 16-byte vector stores, partial ones (walk ends) element by element.
+struct EmitBuf {
+    uint32_t w[4][8];
+};
+struct EmitSec {
+    int32_t sec;   // sector (r >> 3) being collected, -1 none
+    uint32_t mask; // its filled elements
+};
+__device__ __forceinline__ void emit_flush(const ForestArgs& a, EmitBuf& B, EmitSec& E, bool vec) {
+    if (E.sec < 0 || !E.mask) return;
+    const int64_t r0 = (int64_t)E.sec * 8;
+    uint32_t* dst[4] = {reinterpret_cast<uint32_t*>(a.perm), reinterpret_cast<uint32_t*>(a.ta),
+                        reinterpret_cast<uint32_t*>(a.tb), reinterpret_cast<uint32_t*>(a.tc)};
+    const int na = a.ta ? 4 : 1;
+    if (E.mask == 0xffu && vec) {
+        for (int q = 0; q < na; q++) {
+            uint4* d4 = reinterpret_cast<uint4*>(dst[q] + r0);
+            d4[0] = make_uint4(B.w[q][0], B.w[q][1], B.w[q][2], B.w[q][3]);
+            d4[1] = make_uint4(B.w[q][4], B.w[q][5], B.w[q][6], B.w[q][7]);
+        }
+    } else {
+        for (int i = 0; i < 8; i++) {
+            if (!((E.mask >> i) & 1u)) continue;
+            for (int q = 0; q < na; q++) dst[q][r0 + i] = B.w[q][i];
+        }
+    }
+    E.mask = 0;
+}
+
 __device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 nb, int fslot, int32_t d,
-                                         const GrsWin& W, int32_t base, int& ncyc, int4 q) {
+                                         const GrsWin& W, int32_t base, int& ncyc, int4 q, EmitBuf& B,
+                                         EmitSec& E, bool vec) {
     const GrsOut o = grs_vertex(x, nb, fslot, d, W);
     const int32_t r = base + o.p - 1;
     if (r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {  // a malformed factor
         atomicOr(&a.ctl[kCtlBadGrs], 1);
         return;
     }
-    // perm, a, b, c go to index r, consecutive along the walk; the vertex-indexed outputs go
-    // into x's own record sector (just read): k_grs_out copies them out coalesced
-    a.perm[r] = x;
+    // the vertex-indexed outputs go into x's own record sector (just read): k_grs_out copies
+    // them out coalesced; perm, a, b, c go to index r through the sector buffer
     a.grs_rec[2 * (int64_t)x] = make_int4(nb.x, nb.y, o.f.x, o.f.y);
     a.grs_rec[2 * (int64_t)x + 1] = make_int4(o.l, o.p, r, 0);
     ncyc += o.ncyc;
+    if ((r >> 3) != E.sec) {
+        emit_flush(a, B, E, vec);
+        E.sec = r >> 3;
+    }
+    const int i = r & 7;
+    E.mask |= 1u << i;
+    B.w[0][i] = (uint32_t)x;
     if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
         const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
         const int ss = ((o.dir ^ 1) != o.rs && (o.dir ? nb.x : nb.y) >= 0) ? (o.dir ^ 1) : -1;
-        a.ta[r] = ps < 0 ? 0.0f : __int_as_float(ps ? q.y : q.x);
-        a.tc[r] = ss < 0 ? 0.0f : __int_as_float(ss ? q.y : q.x);
-        a.tb[r] = __int_as_float(q.z);
+        B.w[1][i] = ps < 0 ? 0u : (uint32_t)(ps ? q.y : q.x);
+        B.w[3][i] = ss < 0 ? 0u : (uint32_t)(ss ? q.y : q.x);
+        B.w[2][i] = (uint32_t)q.z;
     }
 }
 
 __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
     LF_TL(g_tl_forest, 10);
+    __shared__ EmitBuf bufs[256];
+    EmitBuf& B = bufs[threadIdx.x];
+    EmitSec E{-1, 0u};
+    const bool vec = ((((uintptr_t)a.perm) | ((uintptr_t)a.ta) | ((uintptr_t)a.tb) | ((uintptr_t)a.tc)) & 15) == 0;
     pdl_wait();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     const int ncl = (int)min((int64_t)__ldcg(&a.ctl[kCtlCyc]), a.N / 3 + 1);
@@ -3421,7 +3465,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             const int32_t l = grs_path_id(W, L);
             if (l < 0 || (int64_t)l >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }  // malformed
             const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
-            if (f == 0) grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv));  // the splitter itself
+            if (f == 0) grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv), B, E, vec);  // the splitter itself
             if (x < 0 || tgt < 0) continue;
             if (tgt == sv ? f == 1 : tgt < sv) continue;  // the segment belongs to the other end
             int32_t prev = sv, cur = x, d = 1;
@@ -3437,7 +3481,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
                 float2 wn;
                 grs_load(a, nxt, nbn, wn);  // the next vertex's records are in flight while this one is written
                 const int4 qn = grs_eload(a, nxt);
-                grs_write(a, cur, nbc, fs, d, W, base, ncyc, qc);
+                grs_write(a, cur, nbc, fs, d, W, base, ncyc, qc, B, E, vec);
                 prev = cur;
                 cur = nxt;
                 nbc = nbn;
@@ -3459,7 +3503,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
             float2 ws;
             grs_load(a, sv, nbs, ws);
-            grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv));
+            grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv), B, E, vec);
             int32_t prev = sv, cur = nbs.x, d = 1;
             while (cur != sv) {
                 if ((uint32_t)cur >= (uint32_t)a.N || d > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
@@ -3467,7 +3511,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
                 float2 wc;
                 grs_load(a, cur, nbc, wc);
                 const int fs = nbc.x == prev ? 1 : 0;
-                grs_write(a, cur, nbc, fs, d, W, base, ncyc, grs_eload(a, cur));
+                grs_write(a, cur, nbc, fs, d, W, base, ncyc, grs_eload(a, cur), B, E, vec);
                 prev = cur;
                 cur = fs ? nbc.y : nbc.x;
                 d++;
@@ -3475,6 +3519,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
         }
         (void)fs0;
     }
+    emit_flush(a, B, E, vec);
 #pragma unroll
     for (int o = 16; o; o >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o);
     if ((threadIdx.x & 31) == 0 && ncyc && a.n_cycles) atomicAdd(a.n_cycles, (unsigned long long)ncyc);
