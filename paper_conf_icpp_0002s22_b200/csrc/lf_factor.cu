@@ -397,11 +397,13 @@ __device__ __forceinline__ void cp_wait_all() { asm volatile("cp.async.wait_grou
 #define LF_SPT 256
 #endif
 constexpr int SPT = LF_SPT;         // threads
-constexpr int SETILE = LF_SETILE;   // entries per stage
+constexpr int SETILE = LF_SETILE;   // entries per stage (sparse rows; denser rows: kSetileBig)
+constexpr int kSetileBig = 8192;    // 27-entry rows one lane each: 256 rows per tile fit a stage
 
+template <int SE>
 struct StreamSmem {
-    int32_t col[2][SETILE];
-    float val[2][SETILE];
+    int32_t col[2][SE];
+    float val[2][SE];
     int64_t rp[3][SPT + 2];   // +2: rows of 16-byte multiples (bulk copies)
     int64_t a0[2];            // aligned start of the staged range per stage (or -1)
     unsigned long long bar[2];  // mbarriers of the bulk copies, one per prefetch batch parity
@@ -436,10 +438,11 @@ __device__ __forceinline__ void issue_rowptr(const ProposeArgs& a, int64_t t, in
 }
 
 // stage the entry range of a tile whose row pointers are in rp; returns false if too long
+template <int SE>
 __device__ __forceinline__ void issue_entries(const ProposeArgs& a, int64_t e0, int64_t e1, int32_t* scol,
                                               float* sval, int64_t* a0_out) {
     const int64_t a0 = e0 & ~(int64_t)3;
-    if (e1 - a0 > SETILE) {
+    if (e1 - a0 > SE) {
         if (threadIdx.x == 0) *a0_out = -1;
         return;
     }
@@ -463,12 +466,12 @@ __device__ __forceinline__ void issue_entries(const ProposeArgs& a, int64_t e0, 
     }
 }
 
-template <int NN, int G, bool CHARGED>
+template <int NN, int G, bool CHARGED, int SE>
 __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
     LF_TL(g_tl_factor, 0);
     constexpr int R = SPT / G;
     extern __shared__ __align__(16) unsigned char sraw[];
-    StreamSmem& S = *reinterpret_cast<StreamSmem*>(sraw);
+    StreamSmem<SE>& S = *reinterpret_cast<StreamSmem<SE>*>(sraw);
     pdl_trigger();  // the long-row pass may launch and wait meanwhile
     const int tid = threadIdx.x;
     const int64_t ntiles = (a.N + R - 1) / R;
@@ -486,8 +489,8 @@ __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
         const int64_t rle = (te * R + R <= a.N) ? R : a.N - te * R;
         const int64_t e0 = rpe[0], e1 = rpe[rle];
         const int64_t ea = e0 & ~(int64_t)3, eb = (e1 + 3) & ~(int64_t)3;
-        const bool fits = e1 - ea <= SETILE;
-        const bool bulkE = fits && aligned_cv && eb <= nnz && eb - ea <= SETILE;
+        const bool fits = e1 - ea <= SE;
+        const bool bulkE = fits && aligned_cv && eb <= nnz && eb - ea <= SE;
         const bool hasR = tr < ntiles;
         const int64_t r0 = tr * R;
         const int64_t rc = hasR ? ((r0 + R + 1 <= a.N + 1) ? R + 1 : a.N + 1 - r0) : 0;
@@ -506,7 +509,7 @@ __global__ void __launch_bounds__(SPT) k_propose_stream(ProposeArgs a) {
         }
         if (fits && !bulkE) {
             int64_t dummy;
-            issue_entries(a, e0, e1, S.col[sb], S.val[sb], &dummy);
+            issue_entries<SE>(a, e0, e1, S.col[sb], S.val[sb], &dummy);
         }
         if (hasR && !bulkR) issue_rowptr<R>(a, tr, rps);
         cp_commit();
@@ -1917,36 +1920,37 @@ static void launch_propose(int G, const ProposeArgs& pa, int grid, cudaStream_t 
     }
 }
 
-template <int NN, int G, bool CH>
+template <int NN, int G, bool CH, int SE>
 static void launch_stream_one(const ProposeArgs& pa, cudaStream_t s) {
     static bool attr = false;
-    const int smem = (int)sizeof(StreamSmem);
+    const int smem = (int)sizeof(StreamSmem<SE>);
     if (!attr) {
-        cudaFuncSetAttribute((const void*)k_propose_stream<NN, G, CH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        cudaFuncSetAttribute((const void*)k_propose_stream<NN, G, CH, SE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         attr = true;
     }
-    const int grid = persistent_grid((const void*)k_propose_stream<NN, G, CH>, SPT, smem);
-    k_propose_stream<NN, G, CH><<<grid, SPT, smem, s>>>(pa);
+    const int grid = persistent_grid((const void*)k_propose_stream<NN, G, CH, SE>, SPT, smem);
+    k_propose_stream<NN, G, CH, SE><<<grid, SPT, smem, s>>>(pa);
+}
+
+// G lanes per row and the stage size: (1, SETILE) for sparse rows (C1, C2), one lane per row
+// with big stages up to 32 entries per row (C3-C5: no merge shuffles; 9.5 -> 6.0 ms on C5),
+// then 2 and 8 lanes
+template <int NN, bool CH>
+static void launch_stream_g(int G, const ProposeArgs& pa, cudaStream_t s) {
+    switch (G) {
+        case 0: launch_stream_one<NN, 1, CH, SETILE>(pa, s); break;
+        case 1: launch_stream_one<NN, 1, CH, kSetileBig>(pa, s); break;
+        case 2: launch_stream_one<NN, 2, CH, kSetileBig>(pa, s); break;
+        case 3: launch_stream_one<NN, 2, CH, SETILE>(pa, s); break;
+        default: launch_stream_one<NN, 8, CH, kSetileBig>(pa, s); break;
+    }
 }
 
 template <int NN>
 static void launch_propose_stream(int G, const ProposeArgs& pa, cudaStream_t s) {
     if (pa.N == 0) return;
-    if (pa.charging) {
-        switch (G) {
-            case 1: launch_stream_one<NN, 1, true>(pa, s); break;
-            case 2: launch_stream_one<NN, 2, true>(pa, s); break;
-            case 4: launch_stream_one<NN, 4, true>(pa, s); break;
-            default: launch_stream_one<NN, 8, true>(pa, s); break;
-        }
-    } else {
-        switch (G) {
-            case 1: launch_stream_one<NN, 1, false>(pa, s); break;
-            case 2: launch_stream_one<NN, 2, false>(pa, s); break;
-            case 4: launch_stream_one<NN, 4, false>(pa, s); break;
-            default: launch_stream_one<NN, 8, false>(pa, s); break;
-        }
-    }
+    if (pa.charging) launch_stream_g<NN, true>(G, pa, s);
+    else launch_stream_g<NN, false>(G, pa, s);
 }
 
 template <int NN>
@@ -1971,12 +1975,13 @@ static void launch_propose_tile(int G, const ProposeArgs& pa, int64_t N, cudaStr
     }
 }
 
-// lanes per row of the staged round-0 kernel (thread per row for sparse rows)
-// lanes per row of the round-0 stream: an average tile (256 / G rows) fits a SETILE stage
+// lanes-per-row code of the round-0 stream (launch_stream_g): an average tile (256 / G
+// rows) fits a stage; 0 = one lane with small stages, 1 = one lane with big stages
 static int tile_lanes(double avg) {
-    if (avg <= 7) return 1;
-    if (avg <= 14) return 2;
-    if (avg <= 28) return 4;
+    if (avg <= 7) return 0;
+    if (avg <= 14) return 3;  // (2 lanes, small stages): C4's skewed rows
+    if (avg <= 30) return 1;
+    if (avg <= 60) return 2;
     return 8;
 }
 
@@ -2126,9 +2131,9 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             LF_PROF("propose", k, s);
             if (fresh) {
                 const int Gt = tile_lanes(N > 0 ? (double)A->nnz / (double)N : 1.0);
-                pa.defer_len = 32 * Gt;
+                pa.defer_len = Gt == 0 ? 32 : (Gt == 1 ? 128 : (Gt == 3 ? 64 : 32 * Gt));
 #ifdef LF_TILE_PLAIN
-                launch_propose_tile<NN>(Gt, pa, N, s);
+                launch_propose_tile<NN>(Gt <= 1 ? 1 : (Gt == 3 ? 2 : Gt), pa, N, s);
 #else
                 launch_propose_stream<NN>(Gt, pa, s);
 #endif
