@@ -3437,7 +3437,10 @@ __device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 n
     }
 }
 
-__global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
+#ifndef LF_EMIT_MINB
+#define LF_EMIT_MINB 1
+#endif
+__global__ void __launch_bounds__(256, LF_EMIT_MINB) k_grs_emit(ForestArgs a) {
     LF_TL(g_tl_forest, 10);
     __shared__ EmitBuf bufs[256];
     EmitBuf& B = bufs[threadIdx.x];

@@ -23,6 +23,15 @@ if n.isdigit():
 else:
     A = lfgen.config(n)
     rp, col, val = (torch.from_numpy(x).cuda() for x in (A.rowptr, A.col, A.val))
+if os.environ.get("LF_L2FETCH"):  # cudaLimitMaxL2FetchGranularity (0x05) experiment
+    import ctypes
+    import glob
+    rt = ctypes.CDLL(sorted(glob.glob(os.path.join(os.path.dirname(torch.__file__), "..", "nvidia", "cuda_runtime", "lib", "libcudart.so*")))[0])
+    torch.cuda.synchronize()
+    print("setlimit", rt.cudaDeviceSetLimit(0x05, ctypes.c_size_t(int(os.environ["LF_L2FETCH"]))), file=sys.stderr)
+    v = ctypes.c_size_t(0)
+    rt.cudaDeviceGetLimit(ctypes.byref(v), 0x05)
+    print("l2 fetch granularity", v.value, file=sys.stderr)
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 P = lf.Pipeline(rp, col, val)
 ref = None
