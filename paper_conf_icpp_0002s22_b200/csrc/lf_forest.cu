@@ -926,6 +926,10 @@ struct ForestArgs {
     const float2* pi2_val;
     const float* diag;
     int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
+    uint32_t* grs_spl;     // [N/32 + 1] splitter bitmap (read-only after k_grs_pack)
+    int4* grs_meet;        // [2N] per (vertex, slot): the partial window of the walk that stopped
+    uint64_t* grs_meetk;   //   there looking along that slot: (item, R, DK, 0) and K
+    int2* grs_mstop;       // [2 cnt] (last, next) of a walk that met its partner, (-1, -1) final
 };
 
 __device__ __forceinline__ bool is_foreign(int64_t x, const ForestArgs& a) { return x < a.lo || x >= a.hi; }
@@ -2905,6 +2909,10 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.rdk[1] = c.take<int2>(n);
     const size_t ng = with_grs ? n : 1;  // the partitioned path runs the tile scans only
     t.grs_rec = c.take<int4>(2 * ng);  // one 32-byte record per vertex
+    t.grs_spl = c.take<uint32_t>(ng / 32 + 1);
+    t.grs_meet = c.take<int4>(2 * ng);
+    t.grs_meetk = c.take<uint64_t>(2 * ng);
+    t.grs_mstop = c.take<int2>(2 * ng);
     t.grs_bits = c.take<uint32_t>(ng / 32 + 1);
     t.grs_cyc = c.take<int4>(ng / 3 + 1);
     t.grs_cyck = c.take<uint64_t>(ng / 3 + 1);
@@ -3083,7 +3091,10 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
                 const float2 pv = a.ta ? __ldg(a.pi2_val + v) : make_float2(0.f, 0.f);
                 const float dg = a.ta ? __ldg(a.diag + v) : 0.f;
                 a.grs_rec[2 * v + 1] = make_int4(__float_as_int(pv.x), __float_as_int(pv.y), __float_as_int(dg), -1);
-                if (lane == 0) a.grs_bits[v >> 5] = m[k];  // v - lane is a multiple of 32
+                if (lane == 0) {  // v - lane is a multiple of 32
+                    a.grs_bits[v >> 5] = m[k];
+                    a.grs_spl[v >> 5] = m[k];
+                }
             }
         }
         if (lane == 0) wsum[wid] = mine;
@@ -3109,7 +3120,20 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
     }
 }
 
-// one (splitter, direction) per thread: the segment's full window and the next splitter
+// One (splitter, direction) per walk: the segment's full window and the next splitter.
+// The two walks of a segment start at its two ends and meet in the middle: each claims
+// every vertex it steps on in the visit bitmap (atomicOr) and stops at the first one its
+// partner claimed, so every interior vertex is read by ONE walk (a random 32-byte visit
+// costs ~128 bytes of DRAM traffic: this halves the kernel's).  A walk that stops at a
+// splitter is final; every walk also leaves its partial window (without the stop edge) at
+// (last vertex, slot toward the stop), where k_grs_meet finds it: a walk that met its
+// partner becomes  own window ⊕ stop edge ⊕ reverse(partner's window).
+__device__ __forceinline__ void walk_leave(const ForestArgs& a, int t, int32_t last, int slot, int32_t R,
+                                           uint64_t K, int32_t DK) {
+    a.grs_meet[2 * (int64_t)last + slot] = make_int4(t, R, DK, 0);
+    a.grs_meetk[2 * (int64_t)last + slot] = K;
+}
+
 __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
     LF_TL(g_tl_forest, 6);
     pdl_wait();
@@ -3125,42 +3149,50 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
         const int32_t x = f ? nbs.y : nbs.x;
         int32_t tgt, R = 0, DK = 0;
         uint64_t K = KEY_INF;
+        int2 stop = make_int2(-1, -1);
         if (x < 0) {
             tgt = -(sv + 1);  // a path end: marker
         } else {
             int32_t prev = sv, cur = x;
-            int2 nbc;
-            float2 wc;
-            grs_load(a, cur, nbc, wc);
-            K = edge_key(sv, cur, f ? ws.y : ws.x, sv < cur ? nbs : nbc);
-            DK = sv < cur ? 1 : 0;
-            R = 1;
-            bool bad = false;
-            while (!grs_splitter(a, cur, nbc)) {
+            int2 nbp = nbs;                  // slots of prev
+            int sp = f;                      // prev's slot toward cur
+            float wpc = f ? ws.y : ws.x;     // |w| of edge prev-cur
+            while (true) {
+                const bool spl = (__ldcg(a.grs_spl + (cur >> 5)) >> (cur & 31)) & 1u;
+                bool mine = false;
+                if (!spl) {
+                    const uint32_t old = atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
+                    mine = !((old >> (cur & 31)) & 1u);
+                }
+                if (!spl && !mine) {  // the partner's: met
+                    walk_leave(a, t, prev, sp, R, K, DK);
+                    stop = make_int2(prev, cur);
+                    tgt = cur;
+                    break;
+                }
+                int2 nbc;
+                float2 wc;
+                grs_load(a, cur, nbc, wc);
+                if (spl) walk_leave(a, t, prev, sp, R, K, DK);  // for the walk from that splitter
+                const uint64_t k = edge_key(prev, cur, wpc, prev < cur ? nbp : nbc);
+                if (k < K) { K = k; DK = 2 * R + (prev < cur ? 1 : 0); }
+                R++;
+                if (spl) { tgt = cur; break; }
                 const int fs = nbc.x == prev ? 1 : 0;  // the slot away from prev
                 const int32_t nxt = fs ? nbc.y : nbc.x;
-                if (R > a.N || (uint32_t)nxt >= (uint32_t)a.N) { bad = true; break; }  // a malformed factor
-                // each interior vertex is walked from both ends: the walker with prev < nxt marks it
-                if (prev < nxt) atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
-                const float wn = fs ? wc.y : wc.x;
-                int2 nbn;
-                float2 wnx;
-                grs_load(a, nxt, nbn, wnx);
-                const uint64_t k = edge_key(cur, nxt, wn, cur < nxt ? nbc : nbn);
-                if (k < K) { K = k; DK = 2 * R + (cur < nxt ? 1 : 0); }
-                R++;
+                if (R > a.N || (uint32_t)nxt >= (uint32_t)a.N) {  // a malformed factor: end the segment
+                    atomicOr(&a.ctl[kCtlBadGrs], 1);                // as if at a path end
+                    tgt = -(sv + 1);
+                    break;
+                }
+                wpc = fs ? wc.y : wc.x;
+                nbp = nbc;
+                sp = fs;
                 prev = cur;
                 cur = nxt;
-                nbc = nbn;
-                wc = wnx;
-            }
-            tgt = cur;
-            if (bad) {  // end the segment here as if at a path end: no reduced record points at
-                        // a non-splitter, so every later kernel stays in bounds
-                atomicOr(&a.ctl[kCtlBadGrs], 1);
-                tgt = -(sv + 1);
             }
         }
+        a.grs_mstop[t] = stop;
         int32_t* q = reinterpret_cast<int32_t*>(a.cq + i);
         int32_t* r = reinterpret_cast<int32_t*>(a.cq_r + i);
         int32_t* d = reinterpret_cast<int32_t*>(a.cq_dk + i);
@@ -3169,6 +3201,46 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
         r[f] = R;
         d[f] = DK;
         k[f] = K;
+    }
+}
+
+// Walks that met their partner: own window ⊕ stop edge ⊕ reverse(partner's window); the
+// segment's far splitter is the partner's start.
+__global__ void __launch_bounds__(256) k_grs_meet(ForestArgs a) {
+    LF_TL(g_tl_forest, 12);
+    pdl_wait();
+    pdl_trigger();
+    const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt; t += gridDim.x * blockDim.x) {
+        const int2 st = __ldcg(a.grs_mstop + t);
+        if (st.x < 0) continue;
+        const int i = t >> 1, f = t & 1;
+        const int32_t last = st.x, nxt = st.y;
+        int2 nbl, nbn;
+        float2 wl, wn;
+        grs_load(a, last, nbl, wl);
+        grs_load(a, nxt, nbn, wn);
+        const int sl = nbl.x == nxt ? 0 : 1;   // last's slot toward nxt
+        const int sn = nbn.x == last ? 0 : 1;  // nxt's slot toward last: the partner's key
+        const int4 pm = __ldcg(a.grs_meet + 2 * (int64_t)nxt + sn);
+        const uint64_t pk = __ldcg(a.grs_meetk + 2 * (int64_t)nxt + sn);
+        int32_t* q = reinterpret_cast<int32_t*>(a.cq + i);
+        int32_t* r = reinterpret_cast<int32_t*>(a.cq_r + i);
+        int32_t* d = reinterpret_cast<int32_t*>(a.cq_dk + i);
+        uint64_t* kk = reinterpret_cast<uint64_t*>(a.cq_k + i);
+        int32_t R = r[f], DK = d[f];
+        uint64_t K = kk[f];
+        if (pm.x < 0 || pm.x >= 2 * cnt) {  // no partner record: a malformed factor
+            atomicOr(&a.ctl[kCtlBadGrs], 1);
+            q[f] = -(__ldcg(a.list1 + i) + 1);
+            continue;
+        }
+        win_append(R, K, DK, 1, edge_key(last, nxt, sl ? wl.y : wl.x, last < nxt ? nbl : nbn), last < nxt ? 1 : 0);
+        win_append(R, K, DK, pm.y, pk, pk == KEY_INF ? 0 : 2 * pm.y - 1 - pm.z);
+        q[f] = __ldcg(a.list1 + (pm.x >> 1));
+        r[f] = R;
+        d[f] = DK;
+        kk[f] = K;
     }
 }
 
@@ -3612,6 +3684,10 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         a.grs_bits = w.grs_bits;
         a.grs_cyc = w.grs_cyc;
         a.grs_cyck = w.grs_cyck;
+        a.grs_spl = w.grs_spl;
+        a.grs_meet = w.grs_meet;
+        a.grs_meetk = w.grs_meetk;
+        a.grs_mstop = w.grs_mstop;
         a.perm = perm;
         a.iperm = iperm;
         a.pi2_val = tri ? (const float2*)tri->pi2_val : nullptr;
@@ -3626,6 +3702,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         {
             LF_PROF("grs_walk", -1, s);
             LF_CUDA(launch_pdl(k_grs_walk, persistent_grid((const void*)k_grs_walk, 256), 256, 0, s, a));
+            LF_CUDA(launch_pdl(k_grs_meet, persistent_grid((const void*)k_grs_meet, 256), 256, 0, s, a));
         }
         {
             LF_PROF("red_scan", -1, s);
