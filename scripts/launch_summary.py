@@ -18,7 +18,10 @@ launches = {}
 for r in rows:
     k = int(r["ID"])
     d = launches.setdefault(k, {"name": r["Kernel Name"]})
-    d[r["Metric Name"]] = float(r["Metric Value"].replace(",", ""))
+    try:
+        d[r["Metric Name"]] = float(r["Metric Value"].replace(",", ""))
+    except ValueError:
+        d[r["Metric Name"]] = 0.0
 
 
 def short(n):
@@ -34,7 +37,7 @@ step = seq[starts[-1]:]
 PROF = {"k_propose_stream": "propose[0]", "k_propose_long_blk": "propose_long", "k_mutual0": "mutual[0]",
         "k_rounds_fused": "rounds_fused", "k_rows_propose_k": "rows_propose", "k_rows_long_k": "rows_long",
         "k_rows_mutual_k": "rows_mutual", "k_grs_pack": "grs_pack", "k_grs_walk": "grs_walk",
-        "k_red_full": "red_scan", "k_grs_len": "grs_len", "k_grs_cycfind": "grs_len", "k_grs_lenscan": "grs_len",
+        "k_red_full": "red_scan", "k_grs_meet": "grs_walk", "k_grs_len": "grs_len", "k_grs_cycfind": "grs_len", "k_grs_lenscan": "grs_len",
         "k_tile_prefix": "grs_len", "k_grs_emit": "grs_emit_tri", "k_grs_out": "grs_out", "k_ctl_zero": "ctl_zero",
         "k_lf_full1": "lf_tile", "k_lf_full2": "lf_expand", "k_perm_tri": "perm_tridiag"}
 tot = sum(x["gpu__time_duration.sum"] for x in step)
@@ -48,8 +51,9 @@ for x in step:
         p = f"{p}[{ridx[p] if p != 'propose_long' else 0}]" if p != "propose_long" else "propose_long[0]"
     a = agg.setdefault(p, {"ns": 0.0, "dram": 0.0, "inst": 0.0, "launches": 0})
     a["ns"] += x["gpu__time_duration.sum"]
-    a["dram"] += x.get("dram__bytes_read.sum", 0) + x.get("dram__bytes_write.sum", 0)
-    a["inst"] += x.get("smsp__inst_executed.sum", 0)
+    nz = lambda v: 0.0 if v != v else v  # noqa: E731  (NaN: metric not collected)
+    a["dram"] += nz(x.get("dram__bytes_read.sum", 0)) + nz(x.get("dram__bytes_write.sum", 0))
+    a["inst"] += nz(x.get("smsp__inst_executed.sum", 0))
     a["launches"] += 1
 out = [f"# {tag}: ncu launch list of one bench step ({cfg}), cold-cache serialised launches",
        "", f"source: `{os.path.basename(path)}` ({len(step)} launches in the last step, "
