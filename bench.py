@@ -201,18 +201,19 @@ def kernel_bytes(name, N, Z, n, live_rows, live_nnz, rows_ran=False):
         return 8 * N
     if base == "perm_tridiag":  # write perm, iperm; read forest, pi2, pi2_val, diag; write a, b, c
         return 8 * N + 8 * N + 8 * N + 8 * N + 4 * N + 12 * N
-    # global ruling set: the pack reads the factor, the emit walk writes perm
-    # and iperm and the tridiagonal part (reads signed values and diag, writes a, b, c), the
-    # vertex-order pass writes forest, path_id, pos; walks and the reduced scan are
+    # global ruling set: the pack reads the factor, the emit pass writes every
+    # output (and reads signed values and diag for a, b, c); walks and the reduced scan are
     # implementation traffic
     if base == "grs_pack":
         return 16 * N
-    if base == "grs_emit_tri":
+    if base == "grs_emit_tri":  # write forest, path_id, pos, iperm; read signed values + diag
         return 8 * N + 12 * N + 12 * N
     if base == "grs_emit":
-        return 8 * N
-    if base == "grs_out":
+        return 8 * N + 12 * N
+    if base == "grs_split_tri":  # write perm, a, b, c
         return 16 * N
+    if base == "grs_split":
+        return 4 * N
     if base == "tridiag":
         return 8 * N + 4 * N + 8 * N + 8 * N + 4 * N + 12 * N
     return 0

@@ -927,9 +927,12 @@ struct ForestArgs {
     const float* diag;
     int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
     uint32_t* grs_spl;     // [N/32 + 1] splitter bitmap (read-only after k_grs_pack)
+    int grs_dbg;           // diagnostics (LF_GRS_DBG): 1 skip the r-side stores, 2 skip the window gathers
     int4* grs_meet;        // [2N] per (vertex, slot): the partial window of the walk that stopped
     uint64_t* grs_meetk;   //   there looking along that slot: (item, R, DK, 0) and K
     int2* grs_mstop;       // [2 cnt] (last, next) of a walk that met its partner, (-1, -1) final
+    int4* grs_rout;        // [N] (perm, a, b, c) at the new index (the meet records' storage, free by then)
+    int4* grs_desc;        // [2 (cnt + cycles)] walk descriptors (k_grs_desc); cnt + cycles <= N
 };
 
 __device__ __forceinline__ bool is_foreign(int64_t x, const ForestArgs& a) { return x < a.lo || x >= a.hi; }
@@ -2908,7 +2911,7 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.rdk[0] = c.take<int2>(n);
     t.rdk[1] = c.take<int2>(n);
     const size_t ng = with_grs ? n : 1;  // the partitioned path runs the tile scans only
-    t.grs_rec = c.take<int4>(2 * ng);  // one 32-byte record per vertex
+    t.grs_rec = c.take<int4>(ng);  // one 16-byte record per vertex
     t.grs_spl = c.take<uint32_t>(ng / 32 + 1);
     t.grs_meet = c.take<int4>(2 * ng);
     t.grs_meetk = c.take<uint64_t>(2 * ng);
@@ -2916,6 +2919,7 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.grs_bits = c.take<uint32_t>(ng / 32 + 1);
     t.grs_cyc = c.take<int4>(ng / 3 + 1);
     t.grs_cyck = c.take<uint64_t>(ng / 3 + 1);
+    t.grs_desc = c.take<int4>(2 * ng);  // splitters + splitter-free cycles <= N (a cycle has >= 3 vertices)
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
     if (w) *w = t;
@@ -3044,17 +3048,19 @@ constexpr int kCtlCyc = 134;      // splitter-free cycles recorded by k_grs_cycf
 __device__ __forceinline__ bool grs_splitter(const ForestArgs& a, int32_t v, int2 nb) {
     return nb.x < 0 || nb.y < 0 || (((uint32_t)v * 0x9E3779B1u) >> a.grs_shift) == 0u;
 }
-// The 32-byte record of vertex v (one sector; a random visit costs one DRAM access):
-//   [2v]     slots (nb.x, nb.y) | |w| per slot            -- read by every walk
-//   [2v + 1] signed slot values | diag | 0                -- read by the emit walk
-// The emit walk then overwrites, in the sector it has just read, [2v].zw with the forest
-// slots and [2v + 1] with (path_id, pos, iperm): k_grs_out copies them to the output
-// arrays in one coalesced pass instead of scattered stores.  Other walks
-// only read [2v].xy of a splitter concurrently, which stays.
+// The 16-byte record of vertex v: (slot 0, slot 1, |w| slot 0, |w| slot 1) -- one random
+// visit per walk step.  The walk that claims a non-splitter v (the visit bitmap) overwrites
+// the |w| half it has just read with (walk t, 2d + fslot): v lies at distance d from the
+// walk's splitter, fslot its slot pointing away from it.  k_grs_emit then derives every
+// output of v in ONE coalesced pass over the vertices; the splitter-free
+// cycles of k_grs_cycfind claim theirs as walks t = 2 cnt + c.  Splitters keep their record.
 __device__ __forceinline__ void grs_load(const ForestArgs& a, int32_t v, int2& nb, float2& w) {
-    const int4 r = __ldcg(a.grs_rec + 2 * (int64_t)v);
+    const int4 r = __ldcg(a.grs_rec + (int64_t)v);
     nb = make_int2(r.x, r.y);
     w = make_float2(__int_as_float(r.z), __int_as_float(r.w));
+}
+__device__ __forceinline__ void grs_claim(const ForestArgs& a, int32_t v, int t, int32_t d, int fs) {
+    reinterpret_cast<int2*>(a.grs_rec + (int64_t)v)[1] = make_int2(t, (int32_t)(((uint32_t)d << 1) | (uint32_t)fs));
 }
 
 // 8 vertices per thread per iteration: one list atomic per 2048 vertices (the splitter
@@ -3086,11 +3092,7 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
             mine += __popc(m[k]);
             if (in) {
                 a.len[v] = 0;
-                a.grs_rec[2 * v] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
-                // emit half; .w = -1 until the emit walk writes the vertex (k_grs_out checks it)
-                const float2 pv = a.ta ? __ldg(a.pi2_val + v) : make_float2(0.f, 0.f);
-                const float dg = a.ta ? __ldg(a.diag + v) : 0.f;
-                a.grs_rec[2 * v + 1] = make_int4(__float_as_int(pv.x), __float_as_int(pv.y), __float_as_int(dg), -1);
+                a.grs_rec[v] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
                 if (lane == 0) {  // v - lane is a multiple of 32
                     a.grs_bits[v >> 5] = m[k];
                     a.grs_spl[v >> 5] = m[k];
@@ -3179,6 +3181,7 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
                 R++;
                 if (spl) { tgt = cur; break; }
                 const int fs = nbc.x == prev ? 1 : 0;  // the slot away from prev
+                grs_claim(a, cur, t, R, fs);           // cur's |w| half was read above
                 const int32_t nxt = fs ? nbc.y : nbc.x;
                 if (R > a.N || (uint32_t)nxt >= (uint32_t)a.N) {  // a malformed factor: end the segment
                     atomicOr(&a.ctl[kCtlBadGrs], 1);                // as if at a path end
@@ -3216,10 +3219,9 @@ __global__ void __launch_bounds__(256) k_grs_meet(ForestArgs a) {
         if (st.x < 0) continue;
         const int i = t >> 1, f = t & 1;
         const int32_t last = st.x, nxt = st.y;
-        int2 nbl, nbn;
-        float2 wl, wn;
-        grs_load(a, last, nbl, wl);
-        grs_load(a, nxt, nbn, wn);
+        // both records were claimed (their |w| half overwritten): the factor arrays themselves
+        const int2 nbl = __ldg(a.pi2 + last), nbn = __ldg(a.pi2 + nxt);
+        const float2 wl = __ldg(a.pi2_w + last), wn = __ldg(a.pi2_w + nxt);
         const int sl = nbl.x == nxt ? 0 : 1;   // last's slot toward nxt
         const int sn = nbn.x == last ? 0 : 1;  // nxt's slot toward last: the partner's key
         const int4 pm = __ldcg(a.grs_meet + 2 * (int64_t)nxt + sn);
@@ -3411,6 +3413,24 @@ __global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
             const int32_t lk = key_min_end(K);
             if (K == KEY_INF || lk < 0 || (int64_t)lk >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }
             a.len[lk] = R;
+            // claim the cycle's records as walk 2 cnt + c from v (slot 0 ahead) for k_grs_emit
+            const int tc = 2 * __ldcg(&a.ctl[kCtlCnt1]) + c;
+            prev = v;
+            cur = v;
+            nbc = nbv;
+            fs = 0;
+            int32_t d = 0;
+            do {
+                grs_claim(a, cur, tc, d, fs);
+                atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
+                const int32_t nxt = fs ? nbc.y : nbc.x;
+                const int4 rn = __ldcg(a.grs_rec + (int64_t)nxt);
+                prev = cur;
+                cur = nxt;
+                nbc = make_int2(rn.x, rn.y);
+                fs = nbc.x == prev ? 1 : 0;
+                d++;
+            } while (cur != v);
         }
     }
 }
@@ -3439,183 +3459,168 @@ __global__ void __launch_bounds__(ET) k_grs_lenscan(ForestArgs a) {
     if (threadIdx.x == 0) a.tsum[blockIdx.x] = carry;
 }
 
-// one vertex of a walk: the scattered vertex-indexed outputs and the sequential ones at r
-// the emit half of x's record (signed slot values, diag), loaded a step ahead by the walk
-__device__ __forceinline__ int4 grs_eload(const ForestArgs& a, int32_t x) {
-    if (!a.ta) return make_int4(0, 0, 0, 0);
-    return __ldcg(a.grs_rec + 2 * (int64_t)x + 1);
-}
-
-// The outputs at the new index (perm, a, b, c) are consecutive along a walk, but one
-// thread fills a 32-byte sector only every 8 steps, and a partially written sector that
-// leaves L2 costs a read-modify-write in DRAM.  Each thread therefore collects the current
-// sector of the four arrays in shared memory and stores it when the walk moves on: whole
-// sectors as 16-byte vector stores, partial ones (walk ends) element by element.
-struct EmitBuf {
-    uint32_t w[4][8];
-};
-struct EmitSec {
-    int32_t sec;   // sector (r >> 3) being collected, -1 none
-    uint32_t mask; // its filled elements
-};
-__device__ __forceinline__ void emit_flush(const ForestArgs& a, EmitBuf& B, EmitSec& E, bool vec) {
-    if (E.sec < 0 || !E.mask) return;
-    const int64_t r0 = (int64_t)E.sec * 8;
-    uint32_t* dst[4] = {reinterpret_cast<uint32_t*>(a.perm), reinterpret_cast<uint32_t*>(a.ta),
-                        reinterpret_cast<uint32_t*>(a.tb), reinterpret_cast<uint32_t*>(a.tc)};
-    const int na = a.ta ? 4 : 1;
-    if (E.mask == 0xffu && vec) {
-        for (int q = 0; q < na; q++) {
-            uint4* d4 = reinterpret_cast<uint4*>(dst[q] + r0);
-            d4[0] = make_uint4(B.w[q][0], B.w[q][1], B.w[q][2], B.w[q][3]);
-            d4[1] = make_uint4(B.w[q][4], B.w[q][5], B.w[q][6], B.w[q][7]);
-        }
-    } else {
-        for (int i = 0; i < 8; i++) {
-            if (!((E.mask >> i) & 1u)) continue;
-            for (int q = 0; q < na; q++) dst[q][r0 + i] = B.w[q][i];
-        }
-    }
-    E.mask = 0;
-}
-
-__device__ __forceinline__ void grs_write(const ForestArgs& a, int32_t x, int2 nb, int fslot, int32_t d,
-                                         const GrsWin& W, int32_t base, int& ncyc, int4 q, EmitBuf& B,
-                                         EmitSec& E, bool vec) {
-    const GrsOut o = grs_vertex(x, nb, fslot, d, W);
-    const int32_t r = base + o.p - 1;
-    if (r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {  // a malformed factor
-        atomicOr(&a.ctl[kCtlBadGrs], 1);
-        return;
-    }
-    // the vertex-indexed outputs go into x's own record sector (just read): k_grs_out copies
-    // them out coalesced; perm, a, b, c go to index r through the sector buffer
-    a.grs_rec[2 * (int64_t)x] = make_int4(nb.x, nb.y, o.f.x, o.f.y);
-    a.grs_rec[2 * (int64_t)x + 1] = make_int4(o.l, o.p, r, 0);
-    ncyc += o.ncyc;
-    if ((r >> 3) != E.sec) {
-        emit_flush(a, B, E, vec);
-        E.sec = r >> 3;
-    }
-    const int i = r & 7;
-    E.mask |= 1u << i;
-    B.w[0][i] = (uint32_t)x;
-    if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
-        const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
-        const int ss = ((o.dir ^ 1) != o.rs && (o.dir ? nb.x : nb.y) >= 0) ? (o.dir ^ 1) : -1;
-        B.w[1][i] = ps < 0 ? 0u : (uint32_t)(ps ? q.y : q.x);
-        B.w[3][i] = ss < 0 ? 0u : (uint32_t)(ss ? q.y : q.x);
-        B.w[2][i] = (uint32_t)q.z;
-    }
-}
-
-#ifndef LF_EMIT_MINB
-#define LF_EMIT_MINB 1
-#endif
-__global__ void __launch_bounds__(256, LF_EMIT_MINB) k_grs_emit(ForestArgs a) {
-    LF_TL(g_tl_forest, 10);
-    __shared__ EmitBuf bufs[256];
-    EmitBuf& B = bufs[threadIdx.x];
-    EmitSec E{-1, 0u};
-    const bool vec = ((((uintptr_t)a.perm) | ((uintptr_t)a.ta) | ((uintptr_t)a.tb) | ((uintptr_t)a.tc)) & 15) == 0;
+// Walk descriptors: one 32-byte record per splitter j < cnt (its walks t = 2j + f) and per
+// splitter-free cycle (j = cnt + c, walk t = 2 cnt + c), so that the emit reads ONE sector
+// per vertex instead of the window arrays and the path offset.
+//   path:  {kind 0, base, l, p_s | sgn, 0, 0, 0}: the splitter sits at position p_s; a vertex
+//          at distance d along direction f has p = p_s + sgn_f d, sgn_f = f ? -sgn : sgn
+//   cycle: {kind 1 | bf << 1 | bb << 2, base, pf, pb | ks}: the window of direction 0
+//   kind & 8: a malformed factor (path id out of range)
+// base = prefix(l), the exclusive prefix of the path lengths at the path id l.
+constexpr int kDescBad = 8;
+__global__ void __launch_bounds__(256) k_grs_desc(ForestArgs a) {
+    LF_TL(g_tl_forest, 13);
     pdl_wait();
+    pdl_trigger();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
-    const int ncl = (int)min((int64_t)__ldcg(&a.ctl[kCtlCyc]), a.N / 3 + 1);
-    const int stride = gridDim.x * blockDim.x;
-    int ncyc = 0;
-    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt + ncl; t += stride) {
+    // descriptors fit [N]: splitters and splitter-free cycles (>= 3 vertices each) are
+    // disjoint on a valid factor; a malformed one is cut off (its vertices flag it in the emit)
+    const int ncl = (int)min(min((int64_t)__ldcg(&a.ctl[kCtlCyc]), a.N / 3 + 1), a.N - cnt);
+    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < cnt + ncl; j += gridDim.x * blockDim.x) {
         GrsWin W;
-        int32_t sv, x, fs0;
-        int2 nbs;
-        if (t < 2 * cnt) {
-            const int i = t >> 1, f = t & 1;
-            sv = __ldcg(a.list1 + i);
-            float2 ws;
-            grs_load(a, sv, nbs, ws);
-            W = grs_window(a, i, f);
-            x = f ? nbs.y : nbs.x;
-            const int32_t tgt = reinterpret_cast<const int32_t*>(a.cq + i)[f];
-            fs0 = f;
-            int32_t L;
-            const int32_t l = grs_path_id(W, L);
-            if (l < 0 || (int64_t)l >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }  // malformed
-            const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
-            if (f == 0) grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv), B, E, vec);  // the splitter itself
-            if (x < 0 || tgt < 0) continue;
-            if (tgt == sv ? f == 1 : tgt < sv) continue;  // the segment belongs to the other end
-            int32_t prev = sv, cur = x, d = 1;
-            int2 nbc;
-            float2 wc;
-            grs_load(a, cur, nbc, wc);
-            int4 qc = grs_eload(a, cur);
-            while (!grs_splitter(a, cur, nbc)) {
-                const int fs = nbc.x == prev ? 1 : 0;
-                const int32_t nxt = fs ? nbc.y : nbc.x;
-                if (d > a.N || (uint32_t)nxt >= (uint32_t)a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }  // malformed
-                int2 nbn;
-                float2 wn;
-                grs_load(a, nxt, nbn, wn);  // the next vertex's records are in flight while this one is written
-                const int4 qn = grs_eload(a, nxt);
-                grs_write(a, cur, nbc, fs, d, W, base, ncyc, qc, B, E, vec);
-                prev = cur;
-                cur = nxt;
-                nbc = nbn;
-                qc = qn;
-                d++;
-            }
-        } else {  // a cycle without splitters, from its recorded vertex (slot 0 ahead)
-            const int c = t - 2 * cnt;
+        if (j < cnt) {
+            W = grs_window(a, j, 0);
+        } else {
+            const int c = j - cnt;
             const int4 cr = __ldcg(a.grs_cyc + c);
-            sv = cr.x;
             W.cyc = true;
             W.ks = __ldcg(a.grs_cyck + c);
             W.pf = cr.y >> 1;
             W.bf = cr.y & 1;
             W.pb = cr.z - W.pf - 1;
             W.bb = W.bf ^ 1;  // the far endpoint of the weakest edge
-            const int32_t l = key_min_end(W.ks);
-            if (l < 0 || (int64_t)l >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }
+        }
+        int32_t L;
+        const int32_t l = grs_path_id(W, L);
+        int4 h0, h1 = make_int4(0, 0, 0, 0);
+        if (l < 0 || (int64_t)l >= a.N) {
+            h0 = make_int4(kDescBad, 0, 0, 0);
+        } else {
             const int32_t base = __ldcg(a.tsum + l / LB) + __ldcg(a.off + l);
-            float2 ws;
-            grs_load(a, sv, nbs, ws);
-            grs_write(a, sv, nbs, 0, 0, W, base, ncyc, grs_eload(a, sv), B, E, vec);
-            int32_t prev = sv, cur = nbs.x, d = 1;
-            while (cur != sv) {
-                if ((uint32_t)cur >= (uint32_t)a.N || d > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
-                int2 nbc;
-                float2 wc;
-                grs_load(a, cur, nbc, wc);
-                const int fs = nbc.x == prev ? 1 : 0;
-                grs_write(a, cur, nbc, fs, d, W, base, ncyc, grs_eload(a, cur), B, E, vec);
-                prev = cur;
-                cur = fs ? nbc.y : nbc.x;
-                d++;
+            if (W.cyc) {
+                h0 = make_int4(1 | (W.bf << 1) | (W.bb << 2), base, W.pf, W.pb);
+                h1 = make_int4((int32_t)(uint32_t)W.ks, (int32_t)(uint32_t)(W.ks >> 32), 0, 0);
+            } else {  // grs_vertex's path rule at d = 0, fslot 0: the back end is the path id iff Eb < Ef
+                const bool back = W.Eb < W.Ef;
+                h0 = make_int4(0, base, l, back ? W.Rb + 1 : W.Rf + 1);
+                h1 = make_int4(back ? 1 : -1, 0, 0, 0);
             }
         }
-        (void)fs0;
+        a.grs_desc[2 * (int64_t)j] = h0;
+        a.grs_desc[2 * (int64_t)j + 1] = h1;
     }
-    emit_flush(a, B, E, vec);
+}
+
+// Every vertex's outputs in one coalesced pass over the vertices: its claim (walk t, d,
+// fslot) selects the descriptor of walk t, from which d gives path id, position, forest
+// slots and r = prefix(l) + p - 1 (grs_vertex's rules; cycles through grs_vertex itself).
+// path_id, pos, iperm, forest are written in vertex order; (perm, a, b, c) go to r as one
+// 16-byte record: the 32-byte sector of r-space is complete once the path neighbour
+// (r xor 1) has been swept -- one or two planes later on C5 -- while four separate 4-byte
+// stores per vertex left most sectors partial in L2 and paid a DRAM read-modify-write each
+// (14.3 vs 6.6 ms).  k_grs_split copies the records out to the four arrays.
+__global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
+    LF_TL(g_tl_forest, 10);
+    pdl_wait();
+    const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
+    const int ncl = (int)min(min((int64_t)__ldcg(&a.ctl[kCtlCyc]), a.N / 3 + 1), a.N - cnt);  // as k_grs_desc
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    uint64_t pol = 0;
+    if (a.grs_dbg & 4) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    int ncyc = 0;
+    bool bad = false;
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += stride) {
+        const int4 rc = __ldcs(a.grs_rec + v);
+        const int2 nb = make_int2(rc.x, rc.y);
+        const uint32_t bit = 1u << (v & 31);
+        int32_t d = 0;
+        int fs = 0, f = 0, j = -1;
+        if (__ldcg(a.grs_spl + (v >> 5)) & bit) {  // a splitter: d = 0 on its slot-0 window
+            j = __ldcg(a.bidx1 + v);
+        } else if (__ldcg(a.grs_bits + (v >> 5)) & bit) {  // claimed by walk t
+            const int t = rc.z;
+            d = (int32_t)((uint32_t)rc.w >> 1);
+            fs = rc.w & 1;
+            if (t >= 0 && t < 2 * cnt) { j = t >> 1; f = t & 1; }
+            else if (t >= 2 * cnt && t - 2 * cnt < ncl) j = cnt + (t - 2 * cnt);
+        }  // else no walk claimed it: a malformed factor
+        int4 h0 = make_int4(kDescBad, 0, 0, 0), h1;
+        if (j >= 0) {
+            h0 = __ldcg(a.grs_desc + 2 * (int64_t)j);
+            h1 = __ldcg(a.grs_desc + 2 * (int64_t)j + 1);
+        }
+        GrsOut o;
+        if (!(h0.x & kDescBad)) {
+            if (!(h0.x & 1)) {  // a path
+                const int32_t sg = f ? -h1.x : h1.x;
+                o.l = h0.z;
+                o.p = h0.w + sg * d;
+                o.dir = sg > 0 ? fs ^ 1 : fs;
+                o.f = nb;
+                o.rs = -1;
+                o.ncyc = 0;
+            } else {
+                GrsWin W;
+                W.cyc = true;
+                W.ks = (uint64_t)(uint32_t)h1.x | ((uint64_t)(uint32_t)h1.y << 32);
+                const int bf = (h0.x >> 1) & 1, bb = (h0.x >> 2) & 1;
+                W.pf = f ? h0.w : h0.z;
+                W.pb = f ? h0.z : h0.w;
+                W.bf = f ? bb : bf;
+                W.bb = f ? bf : bb;
+                o = grs_vertex((int32_t)v, nb, fs, d, W);
+            }
+        }
+        const int32_t r = (a.grs_dbg & 2) ? (int32_t)v : h0.y + o.p - 1;
+        if ((h0.x & kDescBad) || r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {
+            bad = true;
+            __stcs(a.path_id + v, -1);
+            __stcs(a.pos + v, -1);
+            __stcs(a.iperm + v, -1);
+            __stcs(a.forest + v, make_int2(-1, -1));
+            continue;
+        }
+        __stcs(a.path_id + v, o.l);
+        __stcs(a.pos + v, o.p);
+        __stcs(a.iperm + v, r);
+        __stcs(a.forest + v, o.f);
+        ncyc += o.ncyc;
+        if (a.grs_dbg & 1) continue;
+        int4 q4 = make_int4((int32_t)v, 0, 0, 0);
+        if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
+            const float2 q = __ldcs(a.pi2_val + v);
+            const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
+            const int ss = ((o.dir ^ 1) != o.rs && (o.dir ? nb.x : nb.y) >= 0) ? (o.dir ^ 1) : -1;
+            q4.y = ps < 0 ? 0 : __float_as_int(ps ? q.y : q.x);
+            q4.z = __float_as_int(__ldcs(a.diag + v));
+            q4.w = ss < 0 ? 0 : __float_as_int(ss ? q.y : q.x);
+        }
+        if (a.grs_dbg & 4) {
+            asm volatile("st.global.L2::cache_hint.v4.s32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(a.grs_rout + r),
+                         "r"(q4.x), "r"(q4.y), "r"(q4.z), "r"(q4.w), "l"(pol) : "memory");
+        } else {
+            a.grs_rout[r] = q4;
+        }
+    }
+    if (bad) atomicOr(&a.ctl[kCtlBadGrs], 1);
 #pragma unroll
     for (int o = 16; o; o >>= 1) ncyc += __shfl_xor_sync(0xffffffffu, ncyc, o);
     if ((threadIdx.x & 31) == 0 && ncyc && a.n_cycles) atomicAdd(a.n_cycles, (unsigned long long)ncyc);
 }
 
-// vertex-order outputs from the records k_grs_emit left in each vertex's record: one
-// coalesced pass (32 bytes read, 20 written per vertex)
-__global__ void __launch_bounds__(256) k_grs_out(ForestArgs a) {
+// perm, a, b, c from the emit's interleaved records at r: one coalesced pass
+__global__ void __launch_bounds__(256) k_grs_split(ForestArgs a) {
     LF_TL(g_tl_forest, 11);
     pdl_wait();
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += stride) {
-        const int4 f = __ldcs(a.grs_rec + 2 * v), o = __ldcs(a.grs_rec + 2 * v + 1);
-        // every vertex of a valid factor was written by a walk; a malformed one may leave
-        // some unvisited (the record still holds the packed input): flag them, -1 outputs
-        const bool ok = (uint32_t)o.z < (uint32_t)a.N && o.w == 0 && (uint32_t)o.x < (uint32_t)a.N && o.y >= 1;
-        if (!ok) atomicOr(&a.ctl[kCtlBadGrs], 1);
-        a.path_id[v] = ok ? o.x : -1;
-        a.pos[v] = ok ? o.y : -1;
-        a.iperm[v] = ok ? o.z : -1;
-        a.forest[v] = ok ? make_int2(f.z, f.w) : make_int2(-1, -1);
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < a.N; r += stride) {
+        const int4 q = __ldcs(a.grs_rout + r);
+        __stcs(a.perm + r, q.x);
+        if (a.ta) {
+            __stcs(reinterpret_cast<int32_t*>(a.ta) + r, q.y);
+            __stcs(reinterpret_cast<int32_t*>(a.tb) + r, q.z);
+            __stcs(reinterpret_cast<int32_t*>(a.tc) + r, q.w);
+        }
     }
 }
 
@@ -3681,6 +3686,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         a.grs_rec = w.grs_rec;
         a.grs_shift = getenv("LF_GRS_SHIFT") ? atoi(getenv("LF_GRS_SHIFT")) : kGrsShift;
         if (a.grs_shift < 20 || a.grs_shift > 31) a.grs_shift = kGrsShift;
+        a.grs_dbg = getenv("LF_GRS_DBG") ? atoi(getenv("LF_GRS_DBG")) : 0;
         a.grs_bits = w.grs_bits;
         a.grs_cyc = w.grs_cyc;
         a.grs_cyck = w.grs_cyck;
@@ -3701,7 +3707,9 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         }
         {
             LF_PROF("grs_walk", -1, s);
-            LF_CUDA(launch_pdl(k_grs_walk, persistent_grid((const void*)k_grs_walk, 256), 256, 0, s, a));
+            int wg = persistent_grid((const void*)k_grs_walk, 256);
+            if (getenv("LF_WALK_BPSM")) wg = sm_count() * atoi(getenv("LF_WALK_BPSM"));
+            LF_CUDA(launch_pdl(k_grs_walk, wg, 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_meet, persistent_grid((const void*)k_grs_meet, 256), 256, 0, s, a));
         }
         {
@@ -3716,13 +3724,19 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
             LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, tiles, (const int*)w.ctl,
                                (unsigned long long*)n_cycles, 1));
         }
+        a.grs_rout = w.grs_meet;  // [2N] int4, unused after k_grs_meet
+        a.grs_desc = w.grs_desc;
+        {
+            LF_PROF("grs_desc", -1, s);
+            LF_CUDA(launch_pdl(k_grs_desc, persistent_grid((const void*)k_grs_desc, 256), 256, 0, s, a));
+        }
         {
             LF_PROF(tri ? "grs_emit_tri" : "grs_emit", -1, s);
             LF_CUDA(launch_pdl(k_grs_emit, persistent_grid((const void*)k_grs_emit, 256), 256, 0, s, a));
         }
         {
-            LF_PROF("grs_out", -1, s);
-            LF_CUDA(launch_pdl(k_grs_out, persistent_grid((const void*)k_grs_out, 256), 256, 0, s, a));
+            LF_PROF(tri ? "grs_split_tri" : "grs_split", -1, s);
+            LF_CUDA(launch_pdl(k_grs_split, persistent_grid((const void*)k_grs_split, 256), 256, 0, s, a));
         }
         return LF_OK;
     } else {

@@ -138,7 +138,7 @@ struct ForestWs {
     int2* rdk[2];          //   grid-path ping-pong DK
     // global ruling set (lf_forest.cu k_grs_*): packed per-vertex records, visit bitmap,
     // records of splitter-free cycles
-    int4* grs_rec;         // [2N] 32-byte per-vertex records (lf_forest.cu grs_load)
+    int4* grs_rec;         // [N] 16-byte per-vertex records (lf_forest.cu grs_load)
     uint32_t* grs_spl;     // splitter bitmap
     int4* grs_meet;        // [2N] meet records per (vertex, slot)
     uint64_t* grs_meetk;
@@ -146,6 +146,7 @@ struct ForestWs {
     uint32_t* grs_bits;    // [N/32 + 1] splitter or visited by a walk
     int4* grs_cyc;         // [N/3 + 1] (lowest vertex, DK, L, 0) of a cycle without splitters
     uint64_t* grs_cyck;    // [N/3 + 1] its weakest key
+    int4* grs_desc;        // [2N] walk descriptors (32 bytes per splitter / splitter-free cycle)
 };
 size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs = true);
 
