@@ -926,7 +926,6 @@ struct ForestArgs {
     const float2* pi2_val;
     const float* diag;
     int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
-    uint32_t* grs_spl;     // [N/32 + 1] splitter bitmap (read-only after k_grs_pack)
     int grs_dbg;           // diagnostics (LF_GRS_DBG): 1 skip the r-side stores, 2 skip the window gathers
     int4* grs_meet;        // [2N] per (vertex, slot): the partial window of the walk that stopped
     uint64_t* grs_meetk;   //   there looking along that slot: (item, R, DK, 0) and K
@@ -2912,7 +2911,6 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.rdk[1] = c.take<int2>(n);
     const size_t ng = with_grs ? n : 1;  // the partitioned path runs the tile scans only
     t.grs_rec = c.take<int4>(ng);  // one 16-byte record per vertex
-    t.grs_spl = c.take<uint32_t>(ng / 32 + 1);
     t.grs_meet = c.take<int4>(2 * ng);
     t.grs_meetk = c.take<uint64_t>(2 * ng);
     t.grs_mstop = c.take<int2>(2 * ng);
@@ -3045,8 +3043,11 @@ static cudaError_t launch_red_full(const ForestArgs& a, cudaStream_t s) {
 constexpr int kGrsShift = LF_GRS_SHIFT;
 constexpr int kCtlCyc = 134;      // splitter-free cycles recorded by k_grs_cycfind
 
+__device__ __forceinline__ bool grs_hashed(const ForestArgs& a, int32_t v) {
+    return (((uint32_t)v * 0x9E3779B1u) >> a.grs_shift) == 0u;
+}
 __device__ __forceinline__ bool grs_splitter(const ForestArgs& a, int32_t v, int2 nb) {
-    return nb.x < 0 || nb.y < 0 || (((uint32_t)v * 0x9E3779B1u) >> a.grs_shift) == 0u;
+    return nb.x < 0 || nb.y < 0 || grs_hashed(a, v);
 }
 // The 16-byte record of vertex v: (slot 0, slot 1, |w| slot 0, |w| slot 1) -- one random
 // visit per walk step.  The walk that claims a non-splitter v (the visit bitmap) overwrites
@@ -3093,10 +3094,7 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
             if (in) {
                 a.len[v] = 0;
                 a.grs_rec[v] = make_int4(nb.x, nb.y, __float_as_int(w.x), __float_as_int(w.y));
-                if (lane == 0) {  // v - lane is a multiple of 32
-                    a.grs_bits[v >> 5] = m[k];
-                    a.grs_spl[v >> 5] = m[k];
-                }
+                if (lane == 0) a.grs_bits[v >> 5] = m[k];  // v - lane is a multiple of 32
             }
         }
         if (lane == 0) wsum[wid] = mine;
@@ -3160,28 +3158,29 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
             int sp = f;                      // prev's slot toward cur
             float wpc = f ? ws.y : ws.x;     // |w| of edge prev-cur
             while (true) {
-                const bool spl = (__ldcg(a.grs_spl + (cur >> 5)) >> (cur & 31)) & 1u;
-                bool mine = false;
-                if (!spl) {
-                    const uint32_t old = atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
-                    mine = !((old >> (cur & 31)) & 1u);
-                }
-                if (!spl && !mine) {  // the partner's: met
+                // the claim (visit bitmap) and the record load are independent: both are in
+                // flight at once, and whether cur is a splitter follows from its id (hashed)
+                // and its record (a path end) -- one memory round trip per step
+                const bool hs = grs_hashed(a, cur);
+                uint32_t old = ~0u;
+                if (!hs) old = atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
+                int2 nbc;
+                float2 wc;
+                grs_load(a, cur, nbc, wc);
+                const bool spl = hs || nbc.x < 0 || nbc.y < 0;  // a path end's bit was set by the pack
+                if (!spl && ((old >> (cur & 31)) & 1u)) {  // the partner's: met (its record is not used)
                     walk_leave(a, t, prev, sp, R, K, DK);
                     stop = make_int2(prev, cur);
                     tgt = cur;
                     break;
                 }
-                int2 nbc;
-                float2 wc;
-                grs_load(a, cur, nbc, wc);
                 if (spl) walk_leave(a, t, prev, sp, R, K, DK);  // for the walk from that splitter
                 const uint64_t k = edge_key(prev, cur, wpc, prev < cur ? nbp : nbc);
                 if (k < K) { K = k; DK = 2 * R + (prev < cur ? 1 : 0); }
                 R++;
                 if (spl) { tgt = cur; break; }
                 const int fs = nbc.x == prev ? 1 : 0;  // the slot away from prev
-                grs_claim(a, cur, t, R, fs);           // cur's |w| half was read above
+                if (!(a.grs_dbg & 8)) grs_claim(a, cur, t, R, fs);  // cur's |w| half was read above
                 const int32_t nxt = fs ? nbc.y : nbc.x;
                 if (R > a.N || (uint32_t)nxt >= (uint32_t)a.N) {  // a malformed factor: end the segment
                     atomicOr(&a.ctl[kCtlBadGrs], 1);                // as if at a path end
@@ -3535,7 +3534,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
         const uint32_t bit = 1u << (v & 31);
         int32_t d = 0;
         int fs = 0, f = 0, j = -1;
-        if (__ldcg(a.grs_spl + (v >> 5)) & bit) {  // a splitter: d = 0 on its slot-0 window
+        if (grs_splitter(a, (int32_t)v, nb)) {  // a splitter: d = 0 on its slot-0 window
             j = __ldcg(a.bidx1 + v);
         } else if (__ldcg(a.grs_bits + (v >> 5)) & bit) {  // claimed by walk t
             const int t = rc.z;
@@ -3690,7 +3689,6 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         a.grs_bits = w.grs_bits;
         a.grs_cyc = w.grs_cyc;
         a.grs_cyck = w.grs_cyck;
-        a.grs_spl = w.grs_spl;
         a.grs_meet = w.grs_meet;
         a.grs_meetk = w.grs_meetk;
         a.grs_mstop = w.grs_mstop;

@@ -139,7 +139,6 @@ struct ForestWs {
     // global ruling set (lf_forest.cu k_grs_*): packed per-vertex records, visit bitmap,
     // records of splitter-free cycles
     int4* grs_rec;         // [N] 16-byte per-vertex records (lf_forest.cu grs_load)
-    uint32_t* grs_spl;     // splitter bitmap
     int4* grs_meet;        // [2N] meet records per (vertex, slot)
     uint64_t* grs_meetk;
     int2* grs_mstop;       // [2N] per walk
