@@ -68,6 +68,7 @@ constexpr int kCtlNcyc = 131;     // broken cycles (single-pass forest)
 constexpr int kCtlGridBar = 133;  // arrival counter of k_red_full's grid barrier
 constexpr int kCtlBad = 135;      // the tile path met a malformed factor: later kernels leave
 constexpr int kCtlBadGrs = 136;   // a ruling-set walk met one (bounded; records stay well formed)
+constexpr int kCtlWalk = 137;     // next walk handed out by k_grs_walk (dynamic schedule)
 constexpr int kMaxSteps = 62;
 constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
 // ctl[192] splitter nodes (cycle pass), [193] unvisited vertices (fallback), [194] tiles
@@ -3139,8 +3140,15 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
     pdl_wait();
     pdl_trigger();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
-    const int stride = gridDim.x * blockDim.x;
-    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt; t += stride) {
+    const int lane = threadIdx.x & 31;
+    // dynamic schedule: a warp takes the next 32 walks when its last one has ended, so the
+    // walks in flight start at consecutive splitters -- a band of the id space -- instead of
+    // drifting apart with the walk lengths under a static grid stride (C5: 9.6 -> 8.4 ms).
+    // (A per-lane step machine that refills each lane at once measured 8.6 ms: the lanes'
+    // idle time is not what bounds the walk, random DRAM accesses are.)
+    int b = 0;
+    if (lane == 0) b = atomicAdd(&a.ctl[kCtlWalk], 32);
+    for (int t = __shfl_sync(0xffffffffu, b, 0) + lane; t < 2 * cnt;) {
         const int i = t >> 1, f = t & 1;
         const int32_t sv = __ldcg(a.list1 + i);
         int2 nbs;
@@ -3203,6 +3211,11 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
         r[f] = R;
         d[f] = DK;
         k[f] = K;
+        const unsigned act = __activemask();
+        const int ld = __ffs(act) - 1;
+        int nb = 0;
+        if (lane == ld) nb = atomicAdd(&a.ctl[kCtlWalk], __popc(act));
+        t = __shfl_sync(act, nb, ld) + __popc(act & ((1u << lane) - 1u));
     }
 }
 
@@ -3705,9 +3718,10 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         }
         {
             LF_PROF("grs_walk", -1, s);
-            int wg = persistent_grid((const void*)k_grs_walk, 256);
-            if (getenv("LF_WALK_BPSM")) wg = sm_count() * atoi(getenv("LF_WALK_BPSM"));
-            LF_CUDA(launch_pdl(k_grs_walk, wg, 256, 0, s, a));
+            // 2 CTAs (16 warps) per SM: fewer walks in flight keep their band of records in L2
+            // (C5, dynamic schedule: 8 CTAs/SM 8.4 ms, 4: 7.3, 3: 6.9, 2: 6.6, 1: 8.5)
+            const int bpsm = getenv("LF_WALK_BPSM") ? atoi(getenv("LF_WALK_BPSM")) : 2;
+            LF_CUDA(launch_pdl(k_grs_walk, sm_count() * (bpsm > 0 ? bpsm : 2), 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_meet, persistent_grid((const void*)k_grs_meet, 256), 256, 0, s, a));
         }
         {
