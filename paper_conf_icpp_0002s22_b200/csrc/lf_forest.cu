@@ -3071,11 +3071,10 @@ constexpr int kPackV = 8;
 __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
     LF_TL(g_tl_forest, 5);
     __shared__ int wsum[8];
-    __shared__ int bbase;
     pdl_wait();
     pdl_trigger();
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const int64_t chunk = (int64_t)blockDim.x * kPackV;
+    const int64_t chunk = (int64_t)blockDim.x * kPackV;  // 2048 (k_grs_list's chunk)
     for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < a.N; c0 += (int64_t)gridDim.x * chunk) {
         unsigned m[kPackV];
         int mine = 0;
@@ -3100,24 +3099,52 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
         }
         if (lane == 0) wsum[wid] = mine;
         __syncthreads();
-        if (threadIdx.x == 0) {
+        if (threadIdx.x == 0) {  // the chunk's splitter count; k_tile_prefix + k_grs_list list them
             int t = 0;
-            for (int q = 0; q < (int)(blockDim.x >> 5); q++) { const int x = wsum[q]; wsum[q] = t; t += x; }
-            bbase = t ? atomicAdd(&a.ctl[kCtlCnt1], t) : 0;
+            for (int q = 0; q < (int)(blockDim.x >> 5); q++) t += wsum[q];
+            a.tsum[c0 / chunk] = t;
         }
-        __syncthreads();
-        int pos = bbase + wsum[wid];
+        __syncthreads();  // wsum reused
+    }
+}
+
+// The splitter list in id order: warp per 2048-vertex chunk (its 64 bitmap words as the pack
+// left them: splitters only), at the chunk's exclusive prefix.  In id order, the walks that
+// k_grs_walk hands out one after the other start at neighbouring splitters: the band of the
+// id space they cover is what L2 holds (an atomic list order jittered over ~9 planes).
+__global__ void __launch_bounds__(256) k_grs_list(ForestArgs a) {
+    LF_TL(g_tl_forest, 14);
+    pdl_wait();
+    pdl_trigger();
+    const int lane = threadIdx.x & 31;
+    const int64_t chunks = (a.N + 2047) / 2048, words = (a.N + 31) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; c < chunks; c += nw) {
+        const int base = __ldcg(a.tsum + c);
+        const int64_t w0 = c * 64 + 2 * lane;
+        uint32_t m0 = w0 < words ? __ldcg(a.grs_bits + w0) : 0u;
+        uint32_t m1 = w0 + 1 < words ? __ldcg(a.grs_bits + w0 + 1) : 0u;
+        const int cnt = __popc(m0) + __popc(m1);
+        int incl = cnt;
 #pragma unroll
-        for (int k = 0; k < kPackV; k++) {
-            const int64_t v = c0 + threadIdx.x + (int64_t)k * blockDim.x;
-            if ((m[k] >> lane) & 1u) {
-                const int p = pos + __popc(m[k] & ((1u << lane) - 1u));
-                a.list1[p] = (int32_t)v;
-                a.bidx1[v] = p;
-            }
-            pos += __popc(m[k]);
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
         }
-        __syncthreads();  // wsum / bbase reused
+        int pos = base + incl - cnt;
+        while (m0) {
+            const int32_t v = (int32_t)(w0 * 32 + __ffs(m0) - 1);
+            m0 &= m0 - 1u;
+            a.list1[pos] = v;
+            a.bidx1[v] = pos++;
+        }
+        while (m1) {
+            const int32_t v = (int32_t)((w0 + 1) * 32 + __ffs(m1) - 1);
+            m1 &= m1 - 1u;
+            a.list1[pos] = v;
+            a.bidx1[v] = pos++;
+        }
+        if (c == chunks - 1 && lane == 31) a.ctl[kCtlCnt1] = base + incl;
     }
 }
 
@@ -3715,6 +3742,10 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         {
             LF_PROF("grs_pack", -1, s);
             LF_CUDA(launch_pdl(k_grs_pack, persistent_grid((const void*)k_grs_pack, 256), 256, 0, s, a));
+            const int chunks = (int)((N + 2047) / 2048);
+            LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, chunks, (const int*)w.ctl,
+                               (unsigned long long*)nullptr, 1));
+            LF_CUDA(launch_pdl(k_grs_list, persistent_grid((const void*)k_grs_list, 256), 256, 0, s, a));
         }
         {
             LF_PROF("grs_walk", -1, s);
