@@ -69,6 +69,12 @@ constexpr int kCtlGridBar = 133;  // arrival counter of k_red_full's grid barrie
 constexpr int kCtlBad = 135;      // the tile path met a malformed factor: later kernels leave
 constexpr int kCtlBadGrs = 136;   // a ruling-set walk met one (bounded; records stay well formed)
 constexpr int kCtlWalk = 137;     // next walk handed out by k_grs_walk (dynamic schedule)
+constexpr int kCtlCycMax = 138;   // longest splitter-free cycle (lf_forest_stats)
+constexpr int kCycStripes = 32;   // counters of the splitter-free cycles (k_grs_cycfind),
+constexpr int kCtlCycS = 256;     //   ctl[256 + 32 s]: one 128-byte line each (atomics on one
+constexpr int kCtlCycStride = 32; //   line queue behind each other in its L2 slice)
+constexpr int kCtlInts = 256 + kCycStripes * kCtlCycStride;
+constexpr int kCtlCand = 139;     // candidates of k_grs_cyccand (list2)
 constexpr int kMaxSteps = 62;
 constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
 // ctl[192] splitter nodes (cycle pass), [193] unvisited vertices (fallback), [194] tiles
@@ -927,7 +933,6 @@ struct ForestArgs {
     const float2* pi2_val;
     const float* diag;
     int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
-    int grs_dbg;           // diagnostics (LF_GRS_DBG): 1 skip the r-side stores, 2 skip the window gathers
     int4* grs_meet;        // [2N] per (vertex, slot): the partial window of the walk that stopped
     uint64_t* grs_meetk;   //   there looking along that slot: (item, R, DK, 0) and K
     int2* grs_mstop;       // [2 cnt] (last, next) of a walk that met its partner, (-1, -1) final
@@ -2896,7 +2901,7 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.list2 = c.take<int32_t>(n);
     t.len = c.take<int32_t>(n);
     t.off = c.take<int32_t>(n);
-    t.ctl = c.take<int>(256);
+    t.ctl = c.take<int>(kCtlInts);
     t.kraw = c.take<ulonglong2>(n);
     t.ekb = c.take<ulonglong2>(n);
     t.cq = c.take<int2>(n);
@@ -2916,9 +2921,9 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.grs_meetk = c.take<uint64_t>(2 * ng);
     t.grs_mstop = c.take<int2>(2 * ng);
     t.grs_bits = c.take<uint32_t>(ng / 32 + 1);
-    t.grs_cyc = c.take<int4>(ng / 3 + 1);
-    t.grs_cyck = c.take<uint64_t>(ng / 3 + 1);
-    t.grs_desc = c.take<int4>(2 * ng);  // splitters + splitter-free cycles <= N (a cycle has >= 3 vertices)
+    t.grs_cyc = c.take<int4>(ng / 3 + 1 + kCycStripes);  // kCycStripes * grs_cyc_cap(N)
+    t.grs_cyck = c.take<uint64_t>(ng / 3 + 1 + kCycStripes);
+    t.grs_desc = c.take<int4>(2 * (ng + ng / 3 + 1 + kCycStripes));  // splitters + the cycle index space
     t.scan_tmp_bytes = scan_temp_bytes(N);
     t.scan_tmp = c.take<char>(t.scan_tmp_bytes);
     if (w) *w = t;
@@ -2945,7 +2950,7 @@ static int coop_launch(K kernel, int block, ForestArgs& a, cudaStream_t s, size_
 __global__ void k_ctl_zero(int* ctl) {
     pdl_trigger();
     pdl_wait();
-    ctl[threadIdx.x] = 0;
+    for (int i = threadIdx.x; i < kCtlInts; i += blockDim.x) ctl[i] = 0;
 }
 
 static int forest_prepare() {
@@ -3042,7 +3047,14 @@ static cudaError_t launch_red_full(const ForestArgs& a, cudaStream_t s) {
 #define LF_GRS_SHIFT 24  // hashed splitter density 2^-(32 - 24) = 1/256 (C5: 1/16..1/256 measured, sparse wins)
 #endif
 constexpr int kGrsShift = LF_GRS_SHIFT;
-constexpr int kCtlCyc = 134;      // splitter-free cycles recorded by k_grs_cycfind
+// splitter-free cycles recorded by k_grs_cycfind: kCycStripes counters (a single one was
+// the contended atomic that dominated the kernel, ~840 k cycles on C5), cycle c = stripe *
+// grs_cyc_cap(N) + its rank in the stripe
+__host__ __device__ __forceinline__ int64_t grs_cyc_cap(int64_t N) { return (N / 3 + 1) / kCycStripes + 1; }
+__device__ __forceinline__ bool grs_cyc_valid(const ForestArgs& a, int64_t c) {
+    const int64_t cap = grs_cyc_cap(a.N), s = c / cap;
+    return c >= 0 && s < kCycStripes && c - s * cap < (int64_t)__ldcg(&a.ctl[kCtlCycS + kCtlCycStride * s]);
+}
 
 __device__ __forceinline__ bool grs_hashed(const ForestArgs& a, int32_t v) {
     return (((uint32_t)v * 0x9E3779B1u) >> a.grs_shift) == 0u;
@@ -3215,7 +3227,7 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
                 R++;
                 if (spl) { tgt = cur; break; }
                 const int fs = nbc.x == prev ? 1 : 0;  // the slot away from prev
-                if (!(a.grs_dbg & 8)) grs_claim(a, cur, t, R, fs);  // cur's |w| half was read above
+                grs_claim(a, cur, t, R, fs);           // cur's |w| half was read above
                 const int32_t nxt = fs ? nbc.y : nbc.x;
                 if (R > a.N || (uint32_t)nxt >= (uint32_t)a.N) {  // a malformed factor: end the segment
                     atomicOr(&a.ctl[kCtlBadGrs], 1);                // as if at a path end
@@ -3390,88 +3402,126 @@ __device__ __forceinline__ uint64_t grs_prio(int32_t v) {
 // vertices no walk visited lie on cycles without a splitter: the lowest-priority vertex of
 // each walks it (slot 0 ahead), records the weakest edge (first occurrence, reading c9)
 // and writes the path length at the path-ID vertex
+// Vertices no walk claimed lie on cycles without a splitter (C5: ~840 k cycles, 3.7% of the
+// vertices, the longest ~200).  Only a vertex whose priority is below both neighbours' can
+// be its cycle's lowest: k_grs_cyccand lists those (one pass over the visit bitmap, one
+// atomic per warp), k_grs_cycfind walks from each of them, dynamically scheduled.
+__global__ void __launch_bounds__(256) k_grs_cyccand(ForestArgs a) {
+    LF_TL(g_tl_forest, 15);
+    pdl_wait();
+    pdl_trigger();
+    const int lane = threadIdx.x & 31;
+    const int64_t words = (a.N + 31) >> 5;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t w0 = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); w0 < words; w0 += stride) {
+        const int64_t wi = w0 + lane;
+        uint32_t m = 0;
+        if (wi < words) {
+            m = ~__ldcg(a.grs_bits + wi);
+            if ((wi + 1) * 32 > a.N) m &= (1u << (a.N - wi * 32)) - 1u;
+        }
+        uint32_t cm = 0;  // candidates among the unclaimed bits
+        for (uint32_t q = m; q;) {
+            const int bit = __ffs(q) - 1;
+            q &= q - 1u;
+            const int32_t v = (int32_t)(wi * 32 + bit);
+            const int4 r = __ldcg(a.grs_rec + (int64_t)v);
+            const bool ok = (uint32_t)r.x < (uint32_t)a.N && (uint32_t)r.y < (uint32_t)a.N;
+            const uint64_t pv = grs_prio(v);
+            if (!ok || (pv < grs_prio(r.x) && pv < grs_prio(r.y))) cm |= 1u << bit;  // malformed: let the walk flag it
+        }
+        const int n = __popc(cm);
+        int incl = n;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+        }
+        int base = 0;
+        if (lane == 31 && incl) base = atomicAdd(&a.ctl[kCtlCand], incl);
+        base = __shfl_sync(0xffffffffu, base, 31);
+        int pos = base + incl - n;
+        while (cm) {
+            const int bit = __ffs(cm) - 1;
+            cm &= cm - 1u;
+            a.list2[pos++] = (int32_t)(wi * 32 + bit);
+        }
+    }
+}
+
+__device__ __forceinline__ void grs_cyc_walk(const ForestArgs& a, int32_t v, int cnt) {
+    int2 nbv;
+    float2 wv;
+    grs_load(a, v, nbv, wv);
+    const uint64_t pv = grs_prio(v);
+    // one walk around the cycle from v (slot 0 ahead) folds the window and gives up at
+    // the first lower-priority vertex: only the lowest one completes it (the critical
+    // path of a long splitter-free cycle is this walk plus the claim walk below)
+    uint64_t K = KEY_INF;
+    int32_t DK = 0, R = 0;
+    int32_t prev = v, cur = v;
+    int2 nbc = nbv;
+    float2 wc = wv;
+    int fs = 0;
+    bool lowest = true;
+    do {
+        const int32_t nxt = fs ? nbc.y : nbc.x;
+        const float wn = fs ? wc.y : wc.x;
+        if ((uint32_t)nxt >= (uint32_t)a.N || R > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); lowest = false; break; }
+        if (grs_prio(nxt) < pv) { lowest = false; break; }
+        int2 nbn;
+        float2 wnx;
+        grs_load(a, nxt, nbn, wnx);
+        const uint64_t k = edge_key(cur, nxt, wn, cur < nxt ? nbc : nbn);
+        if (k < K) { K = k; DK = 2 * R + (cur < nxt ? 1 : 0); }
+        R++;
+        prev = cur;
+        cur = nxt;
+        nbc = nbn;
+        wc = wnx;
+        fs = nbc.x == prev ? 1 : 0;
+    } while (cur != v);
+    if (!lowest) return;
+    if (cur != v) return;  // the walk was stopped (a malformed factor)
+    const int stripe = (int)((v >> 5) & (kCycStripes - 1));
+    const int64_t cap = grs_cyc_cap(a.N);
+    const int local = atomicAdd(&a.ctl[kCtlCycS + kCtlCycStride * stripe], 1);
+    if (local >= cap) { atomicOr(&a.ctl[kCtlBadGrs], 1); return; }  // overlapping "cycles"
+    const int c = (int)(stripe * cap + local);
+    a.grs_cyc[c] = make_int4(v, DK, R, 0);
+    a.grs_cyck[c] = K;
+    const int32_t lk = key_min_end(K);
+    if (K == KEY_INF || lk < 0 || (int64_t)lk >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); return; }
+    a.len[lk] = R;
+    // claim the cycle's records as walk 2 cnt + c from v (slot 0 ahead) for k_grs_emit
+    const int tc = 2 * cnt + c;
+    prev = v;
+    cur = v;
+    nbc = nbv;
+    fs = 0;
+    int32_t d = 0;
+    do {
+        grs_claim(a, cur, tc, d, fs);
+        atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
+        const int32_t nxt = fs ? nbc.y : nbc.x;
+        const int4 rn = __ldcg(a.grs_rec + (int64_t)nxt);
+        prev = cur;
+        cur = nxt;
+        nbc = make_int2(rn.x, rn.y);
+        fs = nbc.x == prev ? 1 : 0;
+        d++;
+    } while (cur != v);
+}
+
 __global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
     LF_TL(g_tl_forest, 8);
     pdl_wait();
     pdl_trigger();
-    const int64_t words = (a.N + 31) >> 5;
-    for (int64_t wi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; wi < words;
-         wi += (int64_t)gridDim.x * blockDim.x) {
-        uint32_t m = ~__ldcg(a.grs_bits + wi);
-        if ((wi + 1) * 32 > a.N) m &= (1u << (a.N - wi * 32)) - 1u;
-        while (m) {
-            const int bit = __ffs(m) - 1;
-            m &= m - 1u;
-            const int32_t v = (int32_t)(wi * 32 + bit);
-            int2 nbv;
-            float2 wv;
-            grs_load(a, v, nbv, wv);
-            const uint64_t pv = grs_prio(v);
-            bool lowest = true;
-            {
-                int32_t prev = v, cur = nbv.x;
-                for (int64_t guard = 0; cur != v; guard++) {
-                    if ((uint32_t)cur >= (uint32_t)a.N || guard > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); lowest = false; break; }
-                    if (grs_prio(cur) < pv) { lowest = false; break; }
-                    int2 nb;
-                    float2 w;
-                    grs_load(a, cur, nb, w);
-                    const int32_t nxt = nb.x == prev ? nb.y : nb.x;
-                    prev = cur;
-                    cur = nxt;
-                }
-            }
-            if (!lowest) continue;
-            uint64_t K = KEY_INF;
-            int32_t DK = 0, R = 0;
-            int32_t prev = v, cur = v;
-            int2 nbc = nbv;
-            float2 wc = wv;
-            int fs = 0;
-            do {
-                const int32_t nxt = fs ? nbc.y : nbc.x;
-                const float wn = fs ? wc.y : wc.x;
-                if (nxt < 0 || R > a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); break; }
-                int2 nbn;
-                float2 wnx;
-                grs_load(a, nxt, nbn, wnx);
-                const uint64_t k = edge_key(cur, nxt, wn, cur < nxt ? nbc : nbn);
-                if (k < K) { K = k; DK = 2 * R + (cur < nxt ? 1 : 0); }
-                R++;
-                prev = cur;
-                cur = nxt;
-                nbc = nbn;
-                wc = wnx;
-                fs = nbc.x == prev ? 1 : 0;
-            } while (cur != v);
-            if (cur != v) continue;  // the walk was stopped (a malformed factor)
-            const int c = atomicAdd(&a.ctl[kCtlCyc], 1);
-            if ((int64_t)c > a.N / 3) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }  // overlapping "cycles"
-            a.grs_cyc[c] = make_int4(v, DK, R, 0);
-            a.grs_cyck[c] = K;
-            const int32_t lk = key_min_end(K);
-            if (K == KEY_INF || lk < 0 || (int64_t)lk >= a.N) { atomicOr(&a.ctl[kCtlBadGrs], 1); continue; }
-            a.len[lk] = R;
-            // claim the cycle's records as walk 2 cnt + c from v (slot 0 ahead) for k_grs_emit
-            const int tc = 2 * __ldcg(&a.ctl[kCtlCnt1]) + c;
-            prev = v;
-            cur = v;
-            nbc = nbv;
-            fs = 0;
-            int32_t d = 0;
-            do {
-                grs_claim(a, cur, tc, d, fs);
-                atomicOr(a.grs_bits + (cur >> 5), 1u << (cur & 31));
-                const int32_t nxt = fs ? nbc.y : nbc.x;
-                const int4 rn = __ldcg(a.grs_rec + (int64_t)nxt);
-                prev = cur;
-                cur = nxt;
-                nbc = make_int2(rn.x, rn.y);
-                fs = nbc.x == prev ? 1 : 0;
-                d++;
-            } while (cur != v);
-        }
-    }
+    const int ncand = __ldcg(&a.ctl[kCtlCand]);
+    const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
+    // a static stride (a dynamic schedule's counter was one more hot line: 1.8 vs 1.4 ms)
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x)
+        grs_cyc_walk(a, __ldcg(a.list2 + i), cnt);
 }
 
 // tile-local exclusive prefix of the path lengths (the tail of k_lf_full2)
@@ -3514,14 +3564,17 @@ __global__ void __launch_bounds__(256) k_grs_desc(ForestArgs a) {
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     // descriptors fit [N]: splitters and splitter-free cycles (>= 3 vertices each) are
     // disjoint on a valid factor; a malformed one is cut off (its vertices flag it in the emit)
-    const int ncl = (int)min(min((int64_t)__ldcg(&a.ctl[kCtlCyc]), a.N / 3 + 1), a.N - cnt);
-    for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < cnt + ncl; j += gridDim.x * blockDim.x) {
+    const int64_t ncl = kCycStripes * grs_cyc_cap(a.N);  // the cycle index space (striped)
+    int lmax = 0;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < cnt + ncl; j += (int64_t)gridDim.x * blockDim.x) {
         GrsWin W;
         if (j < cnt) {
-            W = grs_window(a, j, 0);
+            W = grs_window(a, (int)j, 0);
         } else {
-            const int c = j - cnt;
+            const int64_t c = j - cnt;
+            if (!grs_cyc_valid(a, c)) continue;
             const int4 cr = __ldcg(a.grs_cyc + c);
+            lmax = max(lmax, cr.z);
             W.cyc = true;
             W.ks = __ldcg(a.grs_cyck + c);
             W.pf = cr.y >> 1;
@@ -3548,6 +3601,9 @@ __global__ void __launch_bounds__(256) k_grs_desc(ForestArgs a) {
         a.grs_desc[2 * (int64_t)j] = h0;
         a.grs_desc[2 * (int64_t)j + 1] = h1;
     }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) lmax = max(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));
+    if ((threadIdx.x & 31) == 0 && lmax) atomicMax(&a.ctl[kCtlCycMax], lmax);  // lf_forest_stats
 }
 
 // Every vertex's outputs in one coalesced pass over the vertices: its claim (walk t, d,
@@ -3562,10 +3618,8 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
     LF_TL(g_tl_forest, 10);
     pdl_wait();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
-    const int ncl = (int)min(min((int64_t)__ldcg(&a.ctl[kCtlCyc]), a.N / 3 + 1), a.N - cnt);  // as k_grs_desc
+
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    uint64_t pol = 0;
-    if (a.grs_dbg & 4) asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
     int ncyc = 0;
     bool bad = false;
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += stride) {
@@ -3581,7 +3635,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             d = (int32_t)((uint32_t)rc.w >> 1);
             fs = rc.w & 1;
             if (t >= 0 && t < 2 * cnt) { j = t >> 1; f = t & 1; }
-            else if (t >= 2 * cnt && t - 2 * cnt < ncl) j = cnt + (t - 2 * cnt);
+            else if (t >= 2 * cnt && grs_cyc_valid(a, t - 2 * cnt)) j = cnt + (t - 2 * cnt);
         }  // else no walk claimed it: a malformed factor
         int4 h0 = make_int4(kDescBad, 0, 0, 0), h1;
         if (j >= 0) {
@@ -3610,7 +3664,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
                 o = grs_vertex((int32_t)v, nb, fs, d, W);
             }
         }
-        const int32_t r = (a.grs_dbg & 2) ? (int32_t)v : h0.y + o.p - 1;
+        const int32_t r = h0.y + o.p - 1;
         if ((h0.x & kDescBad) || r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {
             bad = true;
             __stcs(a.path_id + v, -1);
@@ -3624,7 +3678,6 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
         __stcs(a.iperm + v, r);
         __stcs(a.forest + v, o.f);
         ncyc += o.ncyc;
-        if (a.grs_dbg & 1) continue;
         int4 q4 = make_int4((int32_t)v, 0, 0, 0);
         if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
             const float2 q = __ldcs(a.pi2_val + v);
@@ -3634,12 +3687,7 @@ __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
             q4.z = __float_as_int(__ldcs(a.diag + v));
             q4.w = ss < 0 ? 0 : __float_as_int(ss ? q.y : q.x);
         }
-        if (a.grs_dbg & 4) {
-            asm volatile("st.global.L2::cache_hint.v4.s32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(a.grs_rout + r),
-                         "r"(q4.x), "r"(q4.y), "r"(q4.z), "r"(q4.w), "l"(pol) : "memory");
-        } else {
-            a.grs_rout[r] = q4;
-        }
+        a.grs_rout[r] = q4;
     }
     if (bad) atomicOr(&a.ctl[kCtlBadGrs], 1);
 #pragma unroll
@@ -3723,9 +3771,9 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
     if (use_grs(N)) {
         a.list1 = w.list1;
         a.grs_rec = w.grs_rec;
+        a.list2 = w.list2;  // k_grs_cyccand's candidates
         a.grs_shift = getenv("LF_GRS_SHIFT") ? atoi(getenv("LF_GRS_SHIFT")) : kGrsShift;
         if (a.grs_shift < 20 || a.grs_shift > 31) a.grs_shift = kGrsShift;
-        a.grs_dbg = getenv("LF_GRS_DBG") ? atoi(getenv("LF_GRS_DBG")) : 0;
         a.grs_bits = w.grs_bits;
         a.grs_cyc = w.grs_cyc;
         a.grs_cyck = w.grs_cyck;
@@ -3762,6 +3810,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         {
             LF_PROF("grs_len", -1, s);
             LF_CUDA(launch_pdl(k_grs_len, persistent_grid((const void*)k_grs_len, 256), 256, 0, s, a));
+            LF_CUDA(launch_pdl(k_grs_cyccand, persistent_grid((const void*)k_grs_cyccand, 256), 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_cycfind, persistent_grid((const void*)k_grs_cycfind, 256), 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_lenscan, tiles, ET, 0, s, a));
             LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, tiles, (const int*)w.ctl,
@@ -3815,7 +3864,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
 }
 
 int forest_stats(const ForestWs& w, int32_t* out, int cap) {
-    int h[256];
+    int h[kCtlInts];
     LF_CUDA(cudaMemcpy(h, w.ctl, sizeof(h), cudaMemcpyDeviceToHost));
     // [0] boundary vertices cycle pass, [1] rank pass, [2] reduced steps cycle, [3] rank,
     // [4] splitter nodes cycle pass, [5] unvisited, [6] fallback tiles, [7] nodes rank pass,
@@ -3825,9 +3874,11 @@ int forest_stats(const ForestWs& w, int32_t* out, int cap) {
         if (h[kCtlRed1 + i]) steps1 = i + 2;
         if (h[kCtlRed2 + i]) steps2 = i + 2;
     }
-    int v[10] = {h[kCtlCnt1], h[kCtlCnt2], steps1, steps2, h[kCtlStat], h[kCtlStat + 1], h[kCtlStat + 2],
-                 h[kCtlStat + 3], h[kCtlStat + 4], h[kCtlBad] | h[kCtlBadGrs]};
-    for (int i = 0; i < cap && i < 10; i++) out[i] = v[i];
+    // [10] splitter-free cycles of the ruling-set path, [11] the longest of them
+    int v[12] = {h[kCtlCnt1], h[kCtlCnt2], steps1, steps2, h[kCtlStat], h[kCtlStat + 1], h[kCtlStat + 2],
+                 h[kCtlStat + 3], h[kCtlStat + 4], h[kCtlBad] | h[kCtlBadGrs], 0, h[kCtlCycMax]};
+    for (int q = 0; q < kCycStripes; q++) v[10] += h[kCtlCycS + kCtlCycStride * q];
+    for (int i = 0; i < cap && i < 12; i++) out[i] = v[i];
     // [16..31]: per-phase cycle sums (units of 1024 cycles; LF_PHASE_TIMING builds only)
     const unsigned long long* ph = reinterpret_cast<const unsigned long long*>(h + 208);
     for (int i = 0; i < 8 && 16 + i < cap; i++) out[16 + i] = (int)(ph[i] >> 10);
@@ -4058,7 +4109,7 @@ int forest_part_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* 
     const int64_t lo = pc.lo, hi = pc.hi, n_own = hi - lo;
     int rc = forest_prepare();
     if (rc) return rc;
-    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * 256, s));
+    LF_CUDA(cudaMemsetAsync(w.ctl, 0, sizeof(int) * kCtlInts, s));
     LF_CUDA(cudaMemsetAsync(pc.tot, 0, sizeof(int64_t) * (pc.G + 2), s));
     ForestArgs a;
     memset(&a, 0, sizeof(a));

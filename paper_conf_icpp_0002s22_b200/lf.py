@@ -352,7 +352,8 @@ def profile_collect(cap: int = 4096):
 
 FOREST_STATS = ("boundary_cycle_pass", "boundary_rank_pass", "reduced_steps_cycle",
                 "reduced_steps_rank", "splitters_cycle_pass", "unvisited", "fallback_tiles",
-                "splitters_rank_pass", "max_node_scan_steps", "malformed_input")
+                "splitters_rank_pass", "max_node_scan_steps", "malformed_input",
+                "splitter_free_cycles", "longest_splitter_free_cycle")
 
 
 def forest_stats(N, ws):
