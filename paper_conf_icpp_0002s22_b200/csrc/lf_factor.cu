@@ -798,6 +798,26 @@ __device__ __forceinline__ void store_slots(T* __restrict__ p, const T (&o)[NN])
 // fresh round pi is empty and the proposals are already in key order, so the confirmed
 // ones are copied in place order without a merge.
 #ifndef LF_M0ROWS
+// one worklist atomic per CTA: the warps' counts (warp-uniform tot) are combined in shared
+// memory (a per-warp atomic put ~10^6 atomics on one counter per C5 round: its L2 line
+// became the bottleneck of the mutual kernels); returns the warp's base position
+__device__ __forceinline__ int block_append_base(int tot, int32_t* counter) {
+    __shared__ int s_w[32];
+    __shared__ int s_base;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    if (lane == 0) s_w[wid] = tot;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int t = 0;
+        for (int q = 0; q < (int)(blockDim.x >> 5); q++) { const int x = s_w[q]; s_w[q] = t; t += x; }
+        s_base = t ? atomicAdd(counter, t) : 0;
+    }
+    __syncthreads();
+    const int b = s_base + s_w[wid];
+    __syncthreads();  // s_w / s_base are reused by the next call
+    return b;
+}
+
 #define LF_M0ROWS 4
 #endif
 constexpr int kMutual0Rows = LF_M0ROWS;  // rows per thread of k_mutual0 (loads in flight)
@@ -873,14 +893,12 @@ __global__ void __launch_bounds__(256) k_mutual0(MutualArgs a) {
             }
             keepb[b] = keep;
         }
-        if (a.wl_next) {  // one worklist atomic per warp for all MB row batches
+        if (a.wl_next) {  // one worklist atomic per CTA for all MB row batches
             unsigned m[MB];
             int tot = 0;
 #pragma unroll
             for (int b = 0; b < MB; b++) { m[b] = __ballot_sync(0xffffffffu, keepb[b]); tot += __popc(m[b]); }
-            int32_t basepos = 0;
-            if (lane == 0 && tot) basepos = atomicAdd(a.wl_next_count, tot);
-            basepos = __shfl_sync(0xffffffffu, basepos, 0);
+            int32_t basepos = block_append_base(tot, a.wl_next_count);
 #pragma unroll
             for (int b = 0; b < MB; b++) {
                 const int64_t r = c0 + threadIdx.x + (int64_t)b * blockDim.x;
@@ -1739,14 +1757,12 @@ __device__ __forceinline__ void rows_mutual(const RowsArgs& a, int k, bool last)
             }
             if (ns != st[b]) a.state[v] = (uint8_t)ns;
         }
-        if (!last) {  // one worklist atomic per warp for all MB row batches
+        if (!last) {  // one worklist atomic per CTA for all MB row batches
             unsigned m[MB];
             int tot = 0;
 #pragma unroll
             for (int b = 0; b < MB; b++) { m[b] = __ballot_sync(0xffffffffu, keepb[b]); tot += __popc(m[b]); }
-            int32_t basepos = 0;
-            if (lane == 0 && tot) basepos = atomicAdd(cn, tot);
-            basepos = __shfl_sync(0xffffffffu, basepos, 0);
+            int32_t basepos = block_append_base(tot, cn);
 #pragma unroll
             for (int b = 0; b < MB; b++) {
                 if (keepb[b]) wn[basepos + __popc(m[b] & ((1u << lane) - 1u))] = vv[b];
