@@ -13,10 +13,12 @@
 //     boundary vertex; k_red_full scans that reduced list (one cluster through DSMEM, or
 //     the whole grid, cooperative launch); k_lf_full2 expands; k_tile_prefix + k_perm_tri
 //     write the permutation and the tridiagonal copy;
-//   global ruling set (paths that leave every tile: C4, C5) -- k_grs_pack,
-//     k_grs_walk (splitter-to-splitter walks), k_red_full on the splitter list, k_grs_len /
-//     k_grs_cycfind / k_grs_lenscan (path offsets), k_grs_emit (one more walk per segment
-//     writing perm and a/b/c sequentially at the new index) and k_grs_out.
+//   global ruling set (paths that leave every tile: C4, C5) -- k_grs_pack +
+//     k_grs_list (16-byte records, splitter list in id order), k_grs_walk + k_grs_meet
+//     (splitter-to-splitter walks that claim every vertex with its walk and distance),
+//     k_red_full on the splitter list, k_grs_len / k_grs_cyccand / k_grs_cycfind /
+//     k_grs_lenscan (path offsets, splitter-free cycles), k_grs_desc (walk descriptors),
+//     k_grs_emit (one coalesced pass over the vertices) and k_grs_split.
 //
 // The row-partitioned multi-GPU path (forest_part_run) still uses the older two-pass
 // kernels k_lf_local1/2/3 + k_red_scan: its exit-record exchange is built on them.
@@ -3017,28 +3019,16 @@ static cudaError_t launch_red_full(const ForestArgs& a, cudaStream_t s) {
 // Global ruling set (GRS) -- the single-pass window scan without the tile level, for
 // graphs whose paths leave every tile (C5's 27-point snakes: 96% of the vertices are tile
 // boundary vertices, so the reduced graph is nearly the whole graph and pointer jumping
-// over it costs ~20 full passes).  DESIGN.md §4.3a.  Random accesses dominate, so every
-// kernel is organised to touch as few 32-byte sectors per vertex as possible:
-//   1. k_grs_pack: one coalesced pass packs each vertex's factor slots, |w|, signed values
-//      and diagonal into one 32-byte record (one sector per visit later); splitters = path
-//      ends (fewer than two factor neighbours) and a hashed 1/64 of the others, listed in
-//      list1/bidx1 and pre-set in a visit bitmap (L2-resident: N/8 bytes); len := 0.
-//   2. k_grs_walk: from every splitter in each direction, a sequential walk through the
-//      non-splitters to the next splitter folds the full window (R, K, DK) of the segment:
-//      the reduced records (cq, cq_r, cq_k, cq_dk) of the splitter list; walked vertices are
-//      marked in the bitmap.
+// over it costs ~20 full passes).  DESIGN.md §5.5:
+//   1. k_grs_pack / k_grs_list: a 16-byte record per vertex (slots, |w|), splitters = path
+//      ends and a hashed 1/256 of the rest, the visit bitmap, the splitter list in id order.
+//   2. k_grs_walk / k_grs_meet: the two walks of every segment fold its full window and
+//      meet in the middle; each claims the vertices it visits with (walk, distance, slot).
 //   3. k_red_full on the splitter list (the reduced scan of the tile path, unchanged).
-//   4. k_grs_len: every splitter knows its path's ends and length, or its cycle's weakest
-//      edge (K, DK both ways, L = p_f + p_b + 1): the path length at the path-ID vertex.
-//      k_grs_cycfind: vertices left unmarked lie on cycles without a splitter; the
-//      lowest-priority vertex of each walks it and records it.
-//   5. k_grs_lenscan + k_tile_prefix: the exclusive prefix of the path lengths in id order.
-//   6. k_grs_emit: every segment is walked once more (by its smaller-id splitter; the
-//      splitter-free cycles by their recorded vertex).  A vertex at distance d from the
-//      splitter derives path id, position, forest slots from d and the splitter's final
-//      windows (paths: both ends; cycles: the weakest edge ahead / behind); its new index
-//      r = prefix(l) + p - 1 is consecutive along the walk, so perm, a, b, c are written
-//      sequentially, and only iperm, path_id, pos, forest are scattered.
+//   4. k_grs_len, k_grs_cyccand / k_grs_cycfind (cycles without a splitter), k_grs_lenscan
+//      + k_tile_prefix: path lengths at the path-ID vertices and their exclusive prefix.
+//   5. k_grs_desc: one descriptor per walk; k_grs_emit: every output of a vertex from its
+//      claim and its walk's descriptor in one coalesced pass; k_grs_split.
 // Every output equals the tile path's (and the oracle's) bit for bit: the windows fold the
 // same edge keys in the same walk order, and the readings c9/c11/c12/c14/c15 are applied by
 // the same cycle_finish / path rules as k_lf_full2 / k_perm_tri.

@@ -39,6 +39,7 @@ PROF = {"k_propose_stream": "propose[0]", "k_propose_long_blk": "propose_long", 
         "k_rows_mutual_k": "rows_mutual", "k_grs_pack": "grs_pack", "k_grs_walk": "grs_walk",
         "k_red_full": "red_scan", "k_grs_meet": "grs_walk", "k_grs_len": "grs_len", "k_grs_cycfind": "grs_len", "k_grs_lenscan": "grs_len",
         "k_tile_prefix": "grs_len", "k_grs_emit": "grs_emit_tri", "k_grs_split": "grs_split_tri", "k_ctl_zero": "ctl_zero",
+        "k_grs_list": "grs_pack", "k_grs_cyccand": "grs_len", "k_grs_desc": "grs_desc",
         "k_lf_full1": "lf_tile", "k_lf_full2": "lf_expand", "k_perm_tri": "perm_tridiag"}
 tot = sum(x["gpu__time_duration.sum"] for x in step)
 agg = {}
