@@ -1,7 +1,8 @@
 """Seeded synthetic input generators shared by the oracle tests and the CUDA path.
 
 This module holds NONE of the method's arithmetic (no proposal, no confirmation,
-no scan): it only builds symmetric sparse matrices in CSR form whose graphs are
+no scan): it only builds sparse matrices in CSR form (symmetric, and for SURVEY.md §8(f)
+f3 general non-symmetric ones) whose graphs are
 shaped like the paper's workloads (Table 3 and the ANISO
 stencils), following the recipes of SURVEY.md §8(d) "Concrete synthetic inputs".
 Both `oracle/` and the product path consume its output; neither is imported here.
@@ -26,6 +27,8 @@ from .graphs import (  # noqa: F401
     grid3d_27pt_big,
     grid27_nnz,
     random_graph,
+    directed_hash_u,
+    nonsymmetric,
     config,
     CONFIG_NAMES,
 )

@@ -452,6 +452,41 @@ def random_graph(N, E, seed=0, ties=False, diag="rowsum", shuffle_cols_seed=None
                           meta={"seed": seed, "ties": ties}, shuffle_cols_seed=shuffle_cols_seed)
 
 
+def directed_hash_u(i, j, N, seed):
+    """u in [0,1) on a 24-bit grid for the ORDERED pair (i, j) (input generation only)."""
+    i = np.asarray(i, dtype=np.uint64)
+    j = np.asarray(j, dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        x = np.uint64(seed) ^ np.uint64(0xA5A5A5A5) ^ ((i * np.uint64(N) + j) * GOLDEN)
+    return (splitmix64(x) >> np.uint64(40)).astype(np.float64) * (2.0 ** -24)
+
+
+def nonsymmetric(base, seed=7, drop=0.15, zeros=0.02, ties=False):
+    """A general (non-symmetric) matrix on the pattern of `base` (PAPER.md
+    L231, L315): every off-diagonal directed entry (i,j) of base is dropped with probability
+    `drop`, stored as an explicit zero with probability `zeros`, else gets its own value
+    a_ij = -(0.5 + u_ij) from a hash of the ORDERED pair (so a_ij != a_ji); `ties` rounds
+    the values to multiples of 1/4 (many equal |a_ij| + |a_ji|).  The diagonal of base is
+    kept.  Columns stay ascending within rows."""
+    N = base.N
+    rows = np.repeat(np.arange(N, dtype=np.int64), np.diff(base.rowptr))
+    col = base.col.astype(np.int64)
+    off = rows != col
+    u = directed_hash_u(rows, col, N, seed)
+    r2 = directed_hash_u(col, rows, N, seed + 1)  # an independent draw for the drop / zero tests
+    keep = ~off | (r2 >= drop)
+    val = np.where(off, -(0.5 + u), base.val.astype(np.float64))
+    if ties:
+        val = np.where(off, -np.round((0.5 + u) * 4.0) / 4.0, val)
+    val = np.where(off & (r2 >= drop) & (r2 < drop + zeros), 0.0, val).astype(np.float32)
+    rows, col, val = rows[keep], col[keep].astype(np.int32), val[keep]
+    counts = np.bincount(rows, minlength=N).astype(np.int64)
+    rowptr = np.zeros(N + 1, dtype=np.int64)
+    np.cumsum(counts, out=rowptr[1:])
+    return CSR(N=int(N), rowptr=rowptr, col=col, val=val, name=f"nonsym_{base.name}",
+               meta={"seed": seed, "drop": drop, "zeros": zeros, "base": base.name})
+
+
 CONFIG_NAMES = ("C1", "C2", "C3", "C4", "C5")
 
 

@@ -192,6 +192,56 @@ def run_pipeline(A, n=2, M=5, m=5, k_m=0, p=0.5, seed=0):
     return out
 
 
+class _SymCSR:
+    """A CSR triple with the attributes the oracle functions read."""
+
+    def __init__(self, N, rowptr, col, val):
+        self.N, self.rowptr, self.col, self.val = int(N), rowptr, col, val
+
+
+def symmetrize(A):
+    """S = A' + A'^T for a general A (§4, §5.1; reading f3-1):
+    A' = |A| - diag|A|; the entries of S are the union of the off-diagonal patterns of A and
+    A^T, s_ij = fl32(|a_ij| + |a_ji|) with a missing entry counted as 0; rows ascending.
+    The definition written out with numpy: the directed entries and their transposes, sorted
+    by (row, col) (library sort), equal keys added in float32."""
+    rp, col, val = _csr(A)
+    N = A.N
+    rows = np.repeat(np.arange(N, dtype=np.int64), np.diff(rp))
+    off = rows != col
+    i, j = rows[off], col[off].astype(np.int64)
+    w = np.abs(val[off]).astype(np.float32)
+    key = np.concatenate([i * N + j, j * N + i])
+    x = np.concatenate([w, w])
+    order = np.argsort(key, kind="stable")
+    key, x = key[order], x[order]
+    first = np.ones(key.size, dtype=bool)
+    first[1:] = key[1:] != key[:-1]
+    starts = np.flatnonzero(first)
+    s_val = x[starts].copy()
+    pair = np.flatnonzero(~first)  # the second entry of a key (at most two: no duplicates in A)
+    s_val[np.searchsorted(starts, pair, side="right") - 1] = (x[pair - 1] + x[pair]).astype(np.float32)
+    uk = key[starts]
+    s_rows = uk // N
+    s_col = (uk % N).astype(np.int32)
+    s_rp = np.zeros(N + 1, dtype=np.int64)
+    np.cumsum(np.bincount(s_rows, minlength=N), out=s_rp[1:])
+    return _SymCSR(N, s_rp, s_col, s_val.astype(np.float32))
+
+
+def run_pipeline_general(A, M=5, m=5, k_m=0, p=0.5, seed=0):
+    """The hot path on a general A: [0,2]-factor and linear forest of
+    S = A' + A'^T, tridiagonal coefficients from A itself (lfo_tridiag reads row perm[r] of
+    A, so a coupling A does not store is 0)."""
+    S = symmetrize(A)
+    pi, pw, rounds, _, _ = factor(S, 2, M, m, k_m, p, seed)
+    out = dict(S=S, pi=pi, pi_w=pw, rounds=rounds)
+    lf = linear_forest(pi, pw)
+    out.update(lf)
+    out["a"], out["b"], out["c"] = tridiag(A, lf["forest"], lf["perm"])
+    return out
+
+
 def tri_solve(a, b, c, x):
     """Apply the tridiagonal preconditioner: y = T^{-1} x, fp64.
 

@@ -27,6 +27,7 @@ EXPORTS = (
     "lf_comm_destroy", "lf_part_create", "lf_part_destroy", "lf_part_info", "lf_part_factor",
     "lf_part_export", "lf_part_linear_forest", "lf_part_forest_export", "lf_part_tridiag",
     "lf_tri_solve_workspace_size", "lf_tri_solve",
+    "lf_symmetrize_workspace_size", "lf_symmetrize", "lf_orig_coeffs",
 )
 
 
@@ -90,6 +91,12 @@ def load(path: str = LIB_PATH):
     L.lf_tri_solve_workspace_size.restype = C.c_size_t
     L.lf_tri_solve.argtypes = [I64, P, P, P, P, P, P, C.c_size_t, P]
     L.lf_tri_solve.restype = C.c_int
+    L.lf_symmetrize_workspace_size.argtypes = [I64, I64]
+    L.lf_symmetrize_workspace_size.restype = C.c_size_t
+    L.lf_symmetrize.argtypes = [P, P, P, P, P, P, C.c_size_t, P]
+    L.lf_symmetrize.restype = C.c_int
+    L.lf_orig_coeffs.argtypes = [P, I32, P, P, P, P]
+    L.lf_orig_coeffs.restype = C.c_int
     L.lf_profile_enable.argtypes = [I32]
     L.lf_profile_collect.argtypes = [P, I32, P, I32]
     L.lf_last_error.restype = C.c_char_p
@@ -237,6 +244,53 @@ def linear_forest_tridiag(pi2, pi2_w, pi2_val, diag, *, ws=None, out=None, n_cyc
                                       _ptr(out["b"]), _ptr(out["c"]), _ptr(out["n_cycles"]), _ptr(buf),
                                       nb, _stream()))
     return out
+
+
+def symmetrize(rowptr, col, val, *, ws=None):
+    """lf_symmetrize: S = A' + A'^T of a (possibly non-symmetric) device CSR -> (rowptr, col,
+    val) of S, trimmed to its stored entries (one device-to-host read of the count)."""
+    torch = _torch()
+    L = load()
+    N = rowptr.numel() - 1
+    nnz = col.numel()
+    dev = rowptr.device
+    s_rp = torch.empty(N + 1, dtype=torch.int64, device=dev)
+    s_col = torch.empty(max(2 * nnz, 1), dtype=torch.int32, device=dev)
+    s_val = torch.empty(max(2 * nnz, 1), dtype=torch.float32, device=dev)
+    s_nnz = torch.zeros(1, dtype=torch.int64, device=dev)
+    A = _csr_desc(rowptr, col, val)
+    nb = L.lf_symmetrize_workspace_size(N, nnz)
+    if nnz and not nb:
+        raise LFError("symmetrize: nnz must be < 2^30")
+    buf = (ws or _ws).get(nb)
+    _check(L.lf_symmetrize(C.byref(A), _ptr(s_rp), _ptr(s_col), _ptr(s_val), _ptr(s_nnz), _ptr(buf), nb,
+                           _stream()))
+    m = int(s_nnz.item())
+    return s_rp, s_col[:m], s_val[:m]
+
+
+def orig_coeffs(rowptr, col, val, pi, *, out=None):
+    """lf_orig_coeffs: (pi_val [N, n], diag [N]) of the ORIGINAL A on the factor slots pi."""
+    torch = _torch()
+    L = load()
+    N, n = pi.shape
+    if out is None:
+        out = (torch.empty((N, n), dtype=torch.float32, device=pi.device),
+               torch.empty(N, dtype=torch.float32, device=pi.device))
+    A = _csr_desc(rowptr, col, val)
+    _check(L.lf_orig_coeffs(C.byref(A), n, _ptr(pi), _ptr(out[0]), _ptr(out[1]), _stream()))
+    return out
+
+
+def general_pipeline(rowptr, col, val, *, M=5, m=5, k_m=0, p=0.5, seed=0, ws=None):
+    """The hot path on a general (non-symmetric) A: the [0,2]-factor and
+    the linear forest of S = A' + A'^T, the tridiagonal coefficients from A itself."""
+    S = symmetrize(rowptr, col, val, ws=ws)
+    fac = factor(*S, 2, M=M, m=m, k_m=k_m, p=p, seed=seed, want_val=False, want_diag=False, ws=ws)
+    pi_val, diag = orig_coeffs(rowptr, col, val, fac["pi"])
+    fac["pi_val"], fac["diag"] = pi_val, diag
+    lf = linear_forest_tridiag(fac["pi"], fac["pi_w"], pi_val, diag, ws=ws)
+    return S, fac, lf
 
 
 @dataclass

@@ -122,3 +122,19 @@ def test_validate_arguments_rejected_before_launch(lib):
     assert L.lf_validate_factor(10, 2, None, C.c_void_p(0x10000), 256, None) == -1
     assert L.lf_validate_factor(0, 2, None, None, 0, None) == 0
     assert L.lf_validate_factor(10, 2, C.c_void_p(0x1000), C.c_void_p(0x10000), 128, None) == -2
+
+
+def test_general_input_calls_reject_bad_arguments(lib):
+    from paper_conf_icpp_0002s22_b200 import lf
+
+    A = lf.CSRDesc(10, 4, 1, 1, 1)
+    assert lib.lf_symmetrize(C.byref(A), None, None, None, None, None, 0, None) == -1
+    assert b"NULL" in lib.lf_last_error()
+    big = lf.CSRDesc(10, 1 << 30, 1, 1, 1)
+    assert lib.lf_symmetrize(C.byref(big), 1, 1, 1, 1, None, 0, None) == -1
+    assert lib.lf_symmetrize_workspace_size(10, 1 << 30) == 0
+    assert lib.lf_symmetrize_workspace_size(10, 100) > 0
+    assert lib.lf_orig_coeffs(C.byref(A), 5, 1, 1, 1, None) == -1
+    assert lib.lf_orig_coeffs(C.byref(A), 2, None, None, None, None) == -1
+    ok = lf.CSRDesc(10, 4, 1, 1, 1)
+    assert lib.lf_symmetrize(C.byref(ok), 1, 1, 1, 1, None, 0, None) == -2  # no workspace
