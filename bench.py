@@ -48,7 +48,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C5")
-    ap.add_argument("--extra", default="C2,C2n1,C2n3,C2n4,C3,C4",
+    ap.add_argument("--extra", default="C2,C2n1,C2n3,C2n4,C3,C4,G3",
                     help="other configs measured in the same run ('' for none)")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -249,6 +249,38 @@ def make_graph(torch, name):
     A = lfgen.config(name)
     return {"name": name, "N": A.N, "Z": A.nnz, "E": A.n_edges, "rp": torch.from_numpy(A.rowptr).cuda(),
             "col": torch.from_numpy(A.col).cuda(), "val": torch.from_numpy(A.val).cuda()}
+
+
+def measure_general(torch, lf, name, steps, warmup, flush):
+    """SURVEY.md §8(f) f3 on a general input: G<k> = lfgen.nonsymmetric(C<k>); a step is
+    lf_symmetrize + lf_factor(S) + lf_orig_coeffs + lf_linear_forest_tridiag (one host read
+    of nnz(S) inside, to size S).  Medges/s over the undirected edges of S."""
+    import lfgen
+
+    A = lfgen.nonsymmetric(lfgen.config("C" + name[1:]), seed=7)
+    rp, col, val = (torch.from_numpy(x).cuda() for x in (A.rowptr, A.col, A.val))
+    ws = lf.Workspace()
+    S, _, _ = lf.general_pipeline(rp, col, val, ws=ws)
+    E = S[1].numel() // 2
+    stream = torch.cuda.current_stream()
+    for _ in range(warmup):
+        lf.general_pipeline(rp, col, val, ws=ws)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for _ in range(steps):
+        flush.zero_()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        lf.general_pipeline(rp, col, val, ws=ws)
+        ev1.record(stream)
+        ev1.synchronize()
+        ts.append(ev0.elapsed_time(ev1))
+    t = sorted(ts)[len(ts) // 2]
+    return {"name": name, "N": A.N, "Z": int(A.rowptr[-1]), "E_S": int(E), "n": 2,
+            "scope": "symmetrize + factor(S) + original coefficients + linear forest + perm + tridiag",
+            "input": f"lfgen.nonsymmetric(C{name[1:]}, seed=7): 15% of the directed entries dropped, "
+                     "2% explicit zeros, a_ij != a_ji",
+            "ms_per_step": round(t, 4), "Medges_per_s": round(E / (t * 1e-3) / 1e6, 1)}
 
 
 # ---------------------------------------------------------------------------
@@ -674,6 +706,10 @@ def main():
 
     extras = {}
     for cfg in [c for c in args.extra.split(",") if c]:
+        if cfg.startswith("G"):  # a general (non-symmetric) input, SURVEY.md §8(f) f3
+            extras[cfg] = measure_general(torch, lf, cfg, max(5, args.steps // 2), 3, flush)
+            torch.cuda.empty_cache()
+            continue
         name, n = (cfg.split("n")[0], int(cfg.split("n")[1])) if "n" in cfg else (cfg, 2)
         g = make_graph(torch, name)
         r = measure(torch, lf, g, n, max(5, args.steps // 2), 3, flush, use_graph=not args.no_graph)

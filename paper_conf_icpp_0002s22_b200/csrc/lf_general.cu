@@ -10,7 +10,7 @@
 //   lf_orig_coeffs  the signed coefficients of the ORIGINAL A on the factor's slots and its
 //                   diagonal (pi_val[v n + s] = a_{v, pi[v n + s]}, 0 if A does not store the
 //                   entry; diag[v] = a_vv): the input of lf_tridiag / lf_linear_forest_tridiag.
-// B200 design: S is built by one radix sort of the 2 nnz directed entries keyed (row, col)
+// B200 design: S is built by one radix sort of the 2 nnz directed entries keyed row n + col
 // -- every entry (i,j) contributes (i,j) and (j,i) -- and one reduce-by-key that adds the
 // (at most two) |values| of a key; fl32 addition of two operands is commutative, so the sum
 // does not depend on which of the two the sort puts first.  Diagonal entries get the
@@ -40,8 +40,8 @@ __global__ void k_sym_keys(int64_t n, const int64_t* __restrict__ rowptr, const 
             const int64_t j = col[e];
             const float w = fabsf(val[e]);  // A' = |A| (L231)
             const bool d = j == i;           // - diag|A|
-            keys[2 * e] = d ? kDiagKey : ((uint64_t)i << 32) | (uint64_t)j;
-            keys[2 * e + 1] = d ? kDiagKey : ((uint64_t)j << 32) | (uint64_t)i;
+            keys[2 * e] = d ? kDiagKey : (uint64_t)i * (uint64_t)n + (uint64_t)j;  // (row, col) as i n + j:
+            keys[2 * e + 1] = d ? kDiagKey : (uint64_t)j * (uint64_t)n + (uint64_t)i;  // fewer radix passes
             vals[2 * e] = w;
             vals[2 * e + 1] = w;
         }
@@ -61,14 +61,14 @@ __global__ void k_sym_rows(int64_t n, const uint64_t* __restrict__ ukeys, const 
     }
     for (int64_t r = t0; r < m; r += stride) {
         const uint64_t k = ukeys[r];
-        const int64_t i = (int64_t)(k >> 32);
-        s_col[r] = (int32_t)(k & 0xffffffffu);
+        const int64_t i = (int64_t)(k / (uint64_t)n);
+        s_col[r] = (int32_t)(k - (uint64_t)i * (uint64_t)n);
         // rows prev+1 .. i start at r (prev = the row of run r-1, -1 before the first run)
-        const int64_t prev = r > 0 ? (int64_t)(ukeys[r - 1] >> 32) : -1;
+        const int64_t prev = r > 0 ? (int64_t)(ukeys[r - 1] / (uint64_t)n) : -1;
         for (int64_t q = prev + 1; q <= i; q++) s_rowptr[q] = r;
     }
     // rows after the last run's row
-    const int64_t last = m > 0 ? (int64_t)(ukeys[m - 1] >> 32) : -1;
+    const int64_t last = m > 0 ? (int64_t)(ukeys[m - 1] / (uint64_t)n) : -1;
     for (int64_t q = last + 1 + t0; q < n; q += stride) s_rowptr[q] = m;
 }
 
@@ -171,7 +171,10 @@ extern "C" int lf_symmetrize(const lf_csr_t* A, int64_t* s_rowptr, int32_t* s_co
     k_sym_keys<<<grid, 256, 0, s>>>(n, A->rowptr, A->col, A->val, w.k0, w.v0);
     LF_CUDA(cudaGetLastError());
     size_t tb = w.tmp_bytes;
-    LF_CUDA(cub::DeviceRadixSort::SortPairs(w.tmp, tb, w.k0, w.k1, w.v0, w.v1, (int)m, 0, 64, s));
+    // keys below n^2 - 1 (the diagonal key, all ones, still sorts last on these bits)
+    int end_bit = 1;
+    while (end_bit < 64 && ((uint64_t)1 << end_bit) < (uint64_t)n * (uint64_t)n) end_bit++;
+    LF_CUDA(cub::DeviceRadixSort::SortPairs(w.tmp, tb, w.k0, w.k1, w.v0, w.v1, (int)m, 0, end_bit, s));
     tb = w.tmp_bytes;
     LF_CUDA(cub::DeviceReduce::ReduceByKey(w.tmp, tb, w.k1, w.uk, w.v1, s_val, w.nruns, cub::Sum(), (int)m, s));
     k_sym_rows<<<persistent_grid((const void*)k_sym_rows, 256), 256, 0, s>>>(n, w.uk, w.nruns, s_col, s_rowptr, s_nnz);

@@ -46,6 +46,7 @@ CASES = {
     "c1_ties": lambda: lfgen.nonsymmetric(lfgen.grid2d_5pt(48, seed=1), seed=12, ties=True, zeros=0.1),
     "g27": lambda: lfgen.nonsymmetric(lfgen.grid3d_27pt(24, seed=5), seed=13, drop=0.3),
     "c4": lambda: lfgen.nonsymmetric(lfgen.chung_lu(20000, seed=4), seed=14),
+    "g3": lambda: lfgen.nonsymmetric(lfgen.config("C3"), seed=7),  # bench.py's G3 input
     "rand_shuf": lambda: _shuffled_rows(lfgen.nonsymmetric(lfgen.random_graph(3000, 9000, seed=3), seed=15), 7),
 }
 
