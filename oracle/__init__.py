@@ -242,6 +242,84 @@ def run_pipeline_general(A, M=5, m=5, k_m=0, p=0.5, seed=0):
     return out
 
 
+def coarsen(A, mu):
+    """The coarse graph of AlgTriBlockPrecond (§6; readings f1-1..f1-3):
+    every matched pair of the [0,1]-factor mu is one coarse vertex (leader = its smaller id),
+    every unmatched vertex one more (with a ghost partner); coarse vertices numbered in leader
+    order; coarse weight w(P,Q) = sum of |a_ij| over i in P, j in Q (fp64, one rounding to
+    fp32), no coarse diagonal.  Returns (cid [N], members [Nc, 2] (-1 = ghost), CSR)."""
+    rp, col, val = _csr(A)
+    N = A.N
+    mu = np.asarray(mu, dtype=np.int64).reshape(-1)
+    v = np.arange(N, dtype=np.int64)
+    lead = (mu < 0) | (v < mu)
+    pre = np.cumsum(lead) - lead  # exclusive prefix of the leaders
+    cid = np.where(lead, pre, pre[np.maximum(mu, 0)]).astype(np.int32)
+    Nc = int(lead.sum())
+    members = np.full((Nc, 2), -1, dtype=np.int32)
+    members[pre[lead], 0] = v[lead]
+    members[pre[lead], 1] = mu[lead]
+    rows = np.repeat(v, np.diff(rp))
+    ci, cj = cid[rows].astype(np.int64), cid[col].astype(np.int64)
+    off = ci != cj
+    sums = {}
+    for a, b, w in zip(ci[off], cj[off], np.abs(val[off]).astype(np.float64)):
+        sums[(a, b)] = sums.get((a, b), 0.0) + w
+    keys = sorted(sums)
+    c_rows = np.array([k[0] for k in keys], dtype=np.int64)
+    c_col = np.array([k[1] for k in keys], dtype=np.int32)
+    c_val = np.array([sums[k] for k in keys], dtype=np.float64).astype(np.float32)
+    c_rp = np.zeros(Nc + 1, dtype=np.int64)
+    np.cumsum(np.bincount(c_rows, minlength=Nc), out=c_rp[1:])
+    return cid, members, _SymCSR(Nc, c_rp, c_col, c_val)
+
+
+def block_tridiag(A, members, cforest, cperm):
+    """The 2x2 block tridiagonal system (§6) in the coarse forest's order:
+    block row R = coarse vertex P = cperm[R] with fine rows members[P] (-1 = ghost):
+    D = the pair's own 2x2 block of A (a ghost row is (0, 1)), L / U = the blocks of A coupling
+    P to cperm[R-1] / cperm[R+1] if that is a coarse forest edge, else 0.  Row-major blocks."""
+    rp, col, val = _csr(A)
+    ent = {}
+    for i in range(A.N):
+        for e in range(rp[i], rp[i + 1]):
+            ent[(i, int(col[e]))] = val[e]
+
+    def a(i, j):
+        return ent.get((int(i), int(j)), np.float32(0)) if i >= 0 and j >= 0 else np.float32(0)
+
+    Nc = members.shape[0]
+    cf = np.asarray(cforest).reshape(-1, 2)
+    D = np.zeros((Nc, 4), np.float32)
+    L = np.zeros((Nc, 4), np.float32)
+    U = np.zeros((Nc, 4), np.float32)
+    fperm = np.zeros((Nc, 2), np.int32)
+    for R in range(Nc):
+        P = int(cperm[R])
+        p0, p1 = members[P]
+        fperm[R] = (p0, p1)
+        D[R] = (a(p0, p0), a(p0, p1), a(p1, p0), a(p1, p1))
+        if p1 < 0:
+            D[R, 3] = 1.0
+        for Q, out in ((cperm[R - 1] if R > 0 else -1, L), (cperm[R + 1] if R + 1 < Nc else -1, U)):
+            if Q >= 0 and Q in cf[P]:
+                q0, q1 = members[Q]
+                out[R] = (a(p0, q0), a(p0, q1), a(p1, q0), a(p1, q1))
+    return D, L, U, fperm
+
+
+def run_block_pipeline(A, M=5, m=5, k_m=0, p=0.5, seed=0):
+    """AlgTriBlockPrecond on the CPU: [0,1]-factor -> coarse graph -> [0,2]-factor + linear
+    forest on it -> 2x2 block tridiagonal system (§6)."""
+    mu, _, _, _, _ = factor(A, 1, M, m, k_m, p, seed)
+    cid, members, C = coarsen(A, mu)
+    cpi, cpw, _, _, _ = factor(C, 2, M, m, k_m, p, seed)
+    clf = linear_forest(cpi, cpw)
+    D, L, U, fperm = block_tridiag(A, members, clf["forest"], clf["perm"])
+    return dict(mu=np.asarray(mu).reshape(-1), cid=cid, members=members, C=C, cpi=cpi, cforest=clf["forest"],
+                cperm=clf["perm"], D=D, L=L, U=U, fperm=fperm)
+
+
 def tri_solve(a, b, c, x):
     """Apply the tridiagonal preconditioner: y = T^{-1} x, fp64.
 

@@ -28,6 +28,7 @@ EXPORTS = (
     "lf_part_export", "lf_part_linear_forest", "lf_part_forest_export", "lf_part_tridiag",
     "lf_tri_solve_workspace_size", "lf_tri_solve",
     "lf_symmetrize_workspace_size", "lf_symmetrize", "lf_orig_coeffs",
+    "lf_coarsen_workspace_size", "lf_coarsen", "lf_block_tridiag",
 )
 
 
@@ -97,6 +98,12 @@ def load(path: str = LIB_PATH):
     L.lf_symmetrize.restype = C.c_int
     L.lf_orig_coeffs.argtypes = [P, I32, P, P, P, P]
     L.lf_orig_coeffs.restype = C.c_int
+    L.lf_coarsen_workspace_size.argtypes = [I64, I64]
+    L.lf_coarsen_workspace_size.restype = C.c_size_t
+    L.lf_coarsen.argtypes = [P, P, P, P, P, P, P, P, P, C.c_size_t, P]
+    L.lf_coarsen.restype = C.c_int
+    L.lf_block_tridiag.argtypes = [P, I64, P, P, P, P, P, P, P, P]
+    L.lf_block_tridiag.restype = C.c_int
     L.lf_profile_enable.argtypes = [I32]
     L.lf_profile_collect.argtypes = [P, I32, P, I32]
     L.lf_last_error.restype = C.c_char_p
@@ -291,6 +298,55 @@ def general_pipeline(rowptr, col, val, *, M=5, m=5, k_m=0, p=0.5, seed=0, ws=Non
     fac["pi_val"], fac["diag"] = pi_val, diag
     lf = linear_forest_tridiag(fac["pi"], fac["pi_w"], pi_val, diag, ws=ws)
     return S, fac, lf
+
+
+def coarsen(rowptr, col, val, mu, *, ws=None):
+    """lf_coarsen: the coarse graph of the matched pairs of mu ([N] or [N,1]) ->
+    (cid [N], members [Nc, 2], (c_rowptr, c_col, c_val)) trimmed (one host read of Nc, nnz)."""
+    torch = _torch()
+    L = load()
+    N = rowptr.numel() - 1
+    nnz = col.numel()
+    dev = rowptr.device
+    cid = torch.empty(max(N, 1), dtype=torch.int32, device=dev)
+    members = torch.empty((max(N, 1), 2), dtype=torch.int32, device=dev)
+    c_rp = torch.empty(N + 1, dtype=torch.int64, device=dev)
+    c_col = torch.empty(max(nnz, 1), dtype=torch.int32, device=dev)
+    c_val = torch.empty(max(nnz, 1), dtype=torch.float32, device=dev)
+    info = torch.zeros(2, dtype=torch.int64, device=dev)
+    A = _csr_desc(rowptr, col, val)
+    nb = L.lf_coarsen_workspace_size(N, nnz)
+    buf = (ws or _ws).get(nb)
+    _check(L.lf_coarsen(C.byref(A), _ptr(mu.contiguous()), _ptr(cid), _ptr(members), _ptr(c_rp), _ptr(c_col),
+                        _ptr(c_val), _ptr(info), _ptr(buf), nb, _stream()))
+    nc, mc = (int(x) for x in info.tolist())
+    return cid[:N], members[:nc], (c_rp[:nc + 1], c_col[:mc], c_val[:mc])
+
+
+def block_tridiag(rowptr, col, val, members, cforest, cperm):
+    """lf_block_tridiag -> (D, L, U) [Nc, 4] row-major 2x2 blocks, fperm [Nc, 2] (-1 ghost)."""
+    torch = _torch()
+    Lb = load()
+    nc = members.shape[0]
+    dev = members.device
+    D, Lo, U = (torch.empty((max(nc, 1), 4), dtype=torch.float32, device=dev) for _ in range(3))
+    fperm = torch.empty((max(nc, 1), 2), dtype=torch.int32, device=dev)
+    A = _csr_desc(rowptr, col, val)
+    _check(Lb.lf_block_tridiag(C.byref(A), nc, _ptr(members.contiguous()), _ptr(cforest.contiguous()),
+                               _ptr(cperm.contiguous()), _ptr(D), _ptr(Lo), _ptr(U), _ptr(fperm), _stream()))
+    return D[:nc], Lo[:nc], U[:nc], fperm[:nc]
+
+
+def block_pipeline(rowptr, col, val, *, M=5, m=5, k_m=0, p=0.5, seed=0, ws=None):
+    """AlgTriBlockPrecond (§6): [0,1]-factor, coarse graph of the matched pairs,
+    [0,2]-factor + linear forest on it, the 2x2 block tridiagonal system."""
+    mu = factor(rowptr, col, val, 1, M=M, m=m, k_m=k_m, p=p, seed=seed, want_val=False, want_diag=False, ws=ws)["pi"]
+    cid, members, Cg = coarsen(rowptr, col, val, mu, ws=ws)
+    cf = factor(*Cg, 2, M=M, m=m, k_m=k_m, p=p, seed=seed, want_val=False, want_diag=False, ws=ws)
+    clf = linear_forest(cf["pi"], cf["pi_w"], ws=ws)
+    D, Lo, U, fperm = block_tridiag(rowptr, col, val, members, clf["forest"], clf["perm"])
+    return dict(mu=mu, cid=cid, members=members, coarse=Cg, cpi=cf["pi"], cforest=clf["forest"],
+                cperm=clf["perm"], D=D, L=Lo, U=U, fperm=fperm)
 
 
 @dataclass
