@@ -48,7 +48,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C5")
-    ap.add_argument("--extra", default="C2,C2n1,C2n3,C2n4,C3,C4,G3",
+    ap.add_argument("--extra", default="C2,C2n1,C2n3,C2n4,C3,C4,G3,B3",
                     help="other configs measured in the same run ('' for none)")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -281,6 +281,36 @@ def measure_general(torch, lf, name, steps, warmup, flush):
             "input": f"lfgen.nonsymmetric(C{name[1:]}, seed=7): 15% of the directed entries dropped, "
                      "2% explicit zeros, a_ij != a_ji",
             "ms_per_step": round(t, 4), "Medges_per_s": round(E / (t * 1e-3) / 1e6, 1)}
+
+
+def measure_block(torch, lf, name, steps, warmup, flush):
+    """SURVEY.md §8(f) f1 AlgTriBlockPrecond on C<k>: a step is the [0,1]-factor, lf_coarsen,
+    the [0,2]-factor + linear forest of the coarse graph and lf_block_tridiag (two host reads
+    inside: the coarse sizes).  Medges/s over the fine graph's edges."""
+    import lfgen
+
+    A = lfgen.config("C" + name[1:])
+    rp, col, val = (torch.from_numpy(x).cuda() for x in (A.rowptr, A.col, A.val))
+    ws = lf.Workspace()
+    g = lf.block_pipeline(rp, col, val, ws=ws)
+    nc = int(g["members"].shape[0])
+    stream = torch.cuda.current_stream()
+    for _ in range(warmup):
+        lf.block_pipeline(rp, col, val, ws=ws)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for _ in range(steps):
+        flush.zero_()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        lf.block_pipeline(rp, col, val, ws=ws)
+        ev1.record(stream)
+        ev1.synchronize()
+        ts.append(ev0.elapsed_time(ev1))
+    t = sorted(ts)[len(ts) // 2]
+    return {"name": name, "N": A.N, "E": A.n_edges, "coarse_N": nc,
+            "scope": "[0,1]-factor + coarse graph + coarse [0,2]-factor + coarse linear forest + 2x2 blocks",
+            "ms_per_step": round(t, 4), "Medges_per_s": round(A.n_edges / (t * 1e-3) / 1e6, 1)}
 
 
 # ---------------------------------------------------------------------------
@@ -708,6 +738,10 @@ def main():
     for cfg in [c for c in args.extra.split(",") if c]:
         if cfg.startswith("G"):  # a general (non-symmetric) input, SURVEY.md §8(f) f3
             extras[cfg] = measure_general(torch, lf, cfg, max(5, args.steps // 2), 3, flush)
+            torch.cuda.empty_cache()
+            continue
+        if cfg.startswith("B"):  # AlgTriBlockPrecond construction, SURVEY.md §8(f) f1
+            extras[cfg] = measure_block(torch, lf, cfg, max(5, args.steps // 2), 3, flush)
             torch.cuda.empty_cache()
             continue
         name, n = (cfg.split("n")[0], int(cfg.split("n")[1])) if "n" in cfg else (cfg, 2)
