@@ -3606,80 +3606,127 @@ __global__ void __launch_bounds__(256) k_grs_desc(ForestArgs a) {
 // (r xor 1) has been swept -- one or two planes later on C5 -- while four separate 4-byte
 // stores per vertex left most sectors partial in L2 and paid a DRAM read-modify-write each
 // (14.3 vs 6.6 ms).  k_grs_split copies the records out to the four arrays.
+// one vertex of the emit: its claim (walk j's descriptor h0/h1, direction f, distance d,
+// forward slot fs) -> outputs; pv / dg: its signed slot values and diagonal
+__device__ __forceinline__ void grs_emit_one(const ForestArgs& a, int64_t v, int2 nb, int f, int32_t d, int fs,
+                                             int4 h0, int4 h1, float2 pv, float dg, int& ncyc, bool& bad) {
+    GrsOut o;
+    if (!(h0.x & kDescBad)) {
+        if (!(h0.x & 1)) {  // a path
+            const int32_t sg = f ? -h1.x : h1.x;
+            o.l = h0.z;
+            o.p = h0.w + sg * d;
+            o.dir = sg > 0 ? fs ^ 1 : fs;
+            o.f = nb;
+            o.rs = -1;
+            o.ncyc = 0;
+        } else {
+            GrsWin W;
+            W.cyc = true;
+            W.ks = (uint64_t)(uint32_t)h1.x | ((uint64_t)(uint32_t)h1.y << 32);
+            const int bf = (h0.x >> 1) & 1, bb = (h0.x >> 2) & 1;
+            W.pf = f ? h0.w : h0.z;
+            W.pb = f ? h0.z : h0.w;
+            W.bf = f ? bb : bf;
+            W.bb = f ? bf : bb;
+            o = grs_vertex((int32_t)v, nb, fs, d, W);
+        }
+    }
+    const int32_t r = h0.y + o.p - 1;
+    if ((h0.x & kDescBad) || r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {
+        bad = true;
+        __stcs(a.path_id + v, -1);
+        __stcs(a.pos + v, -1);
+        __stcs(a.iperm + v, -1);
+        __stcs(a.forest + v, make_int2(-1, -1));
+        return;
+    }
+    __stcs(a.path_id + v, o.l);
+    __stcs(a.pos + v, o.p);
+    __stcs(a.iperm + v, r);
+    __stcs(a.forest + v, o.f);
+    ncyc += o.ncyc;
+    int4 q4 = make_int4((int32_t)v, 0, 0, 0);
+    if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
+        const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
+        const int ss = ((o.dir ^ 1) != o.rs && (o.dir ? nb.x : nb.y) >= 0) ? (o.dir ^ 1) : -1;
+        q4.y = ps < 0 ? 0 : __float_as_int(ps ? pv.y : pv.x);
+        q4.z = __float_as_int(dg);
+        q4.w = ss < 0 ? 0 : __float_as_int(ss ? pv.y : pv.x);
+    }
+    a.grs_rout[r] = q4;
+}
+
+// Every vertex's outputs in one coalesced pass over the vertices: its claim (walk t, d,
+// fslot) selects the descriptor of walk t, from which d gives path id, position, forest
+// slots and r = prefix(l) + p - 1 (grs_vertex's rules; cycles through grs_vertex itself).
+// path_id, pos, iperm, forest are written in vertex order; (perm, a, b, c) go to r as one
+// 16-byte record: the 32-byte sector of r-space is complete once the path neighbour
+// (r xor 1) has been swept -- one or two planes later on C5 -- while four separate 4-byte
+// stores per vertex left most sectors partial in L2 and paid a DRAM read-modify-write each
+// (14.3 vs 6.6 ms).  k_grs_split copies the records out to the four arrays.  A thread may
+// take kEmitB vertices (a grid stride apart) per pass with all their loads issued first:
+// measured on C5, 1 -> 3.17 ms, 2 -> 3.88, 4 -> 3.27 (the wider sweep costs the r-records'
+// L2 locality what the extra loads in flight gain).
+#ifndef LF_EMIT_B
+#define LF_EMIT_B 1
+#endif
+constexpr int kEmitB = LF_EMIT_B;
 __global__ void __launch_bounds__(256) k_grs_emit(ForestArgs a) {
     LF_TL(g_tl_forest, 10);
     pdl_wait();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
-
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     int ncyc = 0;
     bool bad = false;
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.N; v += stride) {
-        const int4 rc = __ldcs(a.grs_rec + v);
-        const int2 nb = make_int2(rc.x, rc.y);
-        const uint32_t bit = 1u << (v & 31);
-        int32_t d = 0;
-        int fs = 0, f = 0, j = -1;
-        if (grs_splitter(a, (int32_t)v, nb)) {  // a splitter: d = 0 on its slot-0 window
-            j = __ldcg(a.bidx1 + v);
-        } else if (__ldcg(a.grs_bits + (v >> 5)) & bit) {  // claimed by walk t
-            const int t = rc.z;
-            d = (int32_t)((uint32_t)rc.w >> 1);
-            fs = rc.w & 1;
-            if (t >= 0 && t < 2 * cnt) { j = t >> 1; f = t & 1; }
-            else if (t >= 2 * cnt && grs_cyc_valid(a, t - 2 * cnt)) j = cnt + (t - 2 * cnt);
-        }  // else no walk claimed it: a malformed factor
-        int4 h0 = make_int4(kDescBad, 0, 0, 0), h1;
-        if (j >= 0) {
-            h0 = __ldcg(a.grs_desc + 2 * (int64_t)j);
-            h1 = __ldcg(a.grs_desc + 2 * (int64_t)j + 1);
+    for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < a.N; v0 += kEmitB * stride) {
+        int4 rc[kEmitB], h0[kEmitB], h1[kEmitB];
+        int j[kEmitB], f[kEmitB], fs[kEmitB];
+        int32_t d[kEmitB];
+        float2 pv[kEmitB];
+        float dg[kEmitB];
+#pragma unroll
+        for (int u = 0; u < kEmitB; u++) {
+            const int64_t v = v0 + u * stride;
+            rc[u] = v < a.N ? __ldcs(a.grs_rec + v) : make_int4(-1, -1, 0, 0);
+            pv[u] = (a.ta && v < a.N) ? __ldcs(a.pi2_val + v) : make_float2(0.f, 0.f);
+            dg[u] = (a.ta && v < a.N) ? __ldcs(a.diag + v) : 0.f;
         }
-        GrsOut o;
-        if (!(h0.x & kDescBad)) {
-            if (!(h0.x & 1)) {  // a path
-                const int32_t sg = f ? -h1.x : h1.x;
-                o.l = h0.z;
-                o.p = h0.w + sg * d;
-                o.dir = sg > 0 ? fs ^ 1 : fs;
-                o.f = nb;
-                o.rs = -1;
-                o.ncyc = 0;
-            } else {
-                GrsWin W;
-                W.cyc = true;
-                W.ks = (uint64_t)(uint32_t)h1.x | ((uint64_t)(uint32_t)h1.y << 32);
-                const int bf = (h0.x >> 1) & 1, bb = (h0.x >> 2) & 1;
-                W.pf = f ? h0.w : h0.z;
-                W.pb = f ? h0.z : h0.w;
-                W.bf = f ? bb : bf;
-                W.bb = f ? bf : bb;
-                o = grs_vertex((int32_t)v, nb, fs, d, W);
+#pragma unroll
+        for (int u = 0; u < kEmitB; u++) {
+            const int64_t v = v0 + u * stride;
+            j[u] = -1;
+            f[u] = 0;
+            d[u] = 0;
+            fs[u] = 0;
+            if (v >= a.N) continue;
+            const int2 nb = make_int2(rc[u].x, rc[u].y);
+            if (grs_splitter(a, (int32_t)v, nb)) {  // a splitter: d = 0 on its slot-0 window
+                j[u] = __ldcg(a.bidx1 + v);
+            } else if (__ldcg(a.grs_bits + (v >> 5)) & (1u << (v & 31))) {  // claimed by walk t
+                const int t = rc[u].z;
+                d[u] = (int32_t)((uint32_t)rc[u].w >> 1);
+                fs[u] = rc[u].w & 1;
+                if (t >= 0 && t < 2 * cnt) { j[u] = t >> 1; f[u] = t & 1; }
+                else if (t >= 2 * cnt && grs_cyc_valid(a, t - 2 * cnt)) j[u] = cnt + (t - 2 * cnt);
+            }  // else no walk claimed it: a malformed factor
+        }
+#pragma unroll
+        for (int u = 0; u < kEmitB; u++) {
+            h0[u] = make_int4(kDescBad, 0, 0, 0);
+            h1[u] = make_int4(0, 0, 0, 0);
+            if (j[u] >= 0) {
+                h0[u] = __ldcg(a.grs_desc + 2 * (int64_t)j[u]);
+                h1[u] = __ldcg(a.grs_desc + 2 * (int64_t)j[u] + 1);
             }
         }
-        const int32_t r = h0.y + o.p - 1;
-        if ((h0.x & kDescBad) || r < 0 || (int64_t)r >= a.N || o.l < 0 || (int64_t)o.l >= a.N) {
-            bad = true;
-            __stcs(a.path_id + v, -1);
-            __stcs(a.pos + v, -1);
-            __stcs(a.iperm + v, -1);
-            __stcs(a.forest + v, make_int2(-1, -1));
-            continue;
+#pragma unroll
+        for (int u = 0; u < kEmitB; u++) {
+            const int64_t v = v0 + u * stride;
+            if (v < a.N)
+                grs_emit_one(a, v, make_int2(rc[u].x, rc[u].y), f[u], d[u], fs[u], h0[u], h1[u], pv[u], dg[u],
+                             ncyc, bad);
         }
-        __stcs(a.path_id + v, o.l);
-        __stcs(a.pos + v, o.p);
-        __stcs(a.iperm + v, r);
-        __stcs(a.forest + v, o.f);
-        ncyc += o.ncyc;
-        int4 q4 = make_int4((int32_t)v, 0, 0, 0);
-        if (a.ta) {  // the forest neighbour toward the path-id end is perm[r-1] (reading c15)
-            const float2 q = __ldcs(a.pi2_val + v);
-            const int ps = (o.dir != o.rs && (o.dir ? nb.y : nb.x) >= 0) ? o.dir : -1;
-            const int ss = ((o.dir ^ 1) != o.rs && (o.dir ? nb.x : nb.y) >= 0) ? (o.dir ^ 1) : -1;
-            q4.y = ps < 0 ? 0 : __float_as_int(ps ? q.y : q.x);
-            q4.z = __float_as_int(__ldcs(a.diag + v));
-            q4.w = ss < 0 ? 0 : __float_as_int(ss ? q.y : q.x);
-        }
-        a.grs_rout[r] = q4;
     }
     if (bad) atomicOr(&a.ctl[kCtlBadGrs], 1);
 #pragma unroll

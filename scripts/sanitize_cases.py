@@ -1,7 +1,8 @@
 """Small cases for compute-sanitizer runs (memcheck / racecheck / synccheck / initcheck):
 the single-GPU pipeline in both forest modes (tile path, global ruling set) and both round
 modes (cached, rows), factors n = 1..4, the row-partitioned path through the loopback
-exchange (G = 3), and lf_tri_solve -- every result still compared with the oracle."""
+exchange (G = 3), general inputs (f3), the block preconditioner (f1) and lf_tri_solve -- every
+result still compared with the oracle."""
 import os
 import sys
 
@@ -71,6 +72,25 @@ for name, A in graphs[:2]:
         p.close()
     comm.close()
     print("ok partitioned loopback", name, flush=True)
+for name, base in graphs[:3]:  # general inputs in both forest modes
+    A = lfgen.nonsymmetric(base, seed=5)
+    o = oracle.run_pipeline_general(A)
+    for forest in ("tile", "grs"):
+        os.environ["LF_FOREST"] = forest
+        _, fac, lfo = lf.general_pipeline(*dev(A))
+        torch.cuda.synchronize()
+        assert np.array_equal(lfo["perm"].cpu().numpy(), o["perm"]), (name, forest)
+        assert np.array_equal(lfo["a"].cpu().numpy().view(np.uint32), o["a"].view(np.uint32)), (name, forest)
+    os.environ.pop("LF_FOREST", None)
+    print("ok general", name, flush=True)
+for name, A in graphs[:3]:  # AlgTriBlockPrecond
+    o = oracle.run_block_pipeline(A)
+    g = lf.block_pipeline(*dev(A))
+    torch.cuda.synchronize()
+    assert np.array_equal(g["fperm"].cpu().numpy(), o["fperm"]), name
+    for k in ("D", "L", "U"):
+        assert np.array_equal(g[k].cpu().numpy().view(np.uint32), o[k].view(np.uint32)), (name, k)
+    print("ok block", name, flush=True)
 A = lfgen.config("C1")
 P = check_pipeline(A, "C1")
 x = np.random.default_rng(0).standard_normal(A.N).astype(np.float32)
