@@ -3836,9 +3836,11 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
         }
         {
             LF_PROF("grs_walk", -1, s);
-            // 2 CTAs (16 warps) per SM: fewer walks in flight keep their band of records in L2
-            // (C5, dynamic schedule: 8 CTAs/SM 8.4 ms, 4: 7.3, 3: 6.9, 2: 6.6, 1: 8.5)
-            const int bpsm = getenv("LF_WALK_BPSM") ? atoi(getenv("LF_WALK_BPSM")) : 2;
+            // large graphs: 2 CTAs (16 warps) per SM -- fewer walks in flight keep their band of
+            // records in L2 (C5, dynamic schedule: 8 CTAs/SM 8.4 ms, 4: 7.3, 3: 6.9, 2: 6.6,
+            // 1: 8.5); graphs whose records fit L2 anyway want the latency hiding (C4: 8 CTAs/SM)
+            const int bpsm_def = N >= ((int64_t)1 << 25) ? 2 : 8;
+            const int bpsm = getenv("LF_WALK_BPSM") ? atoi(getenv("LF_WALK_BPSM")) : bpsm_def;
             LF_CUDA(launch_pdl(k_grs_walk, sm_count() * (bpsm > 0 ? bpsm : 2), 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_meet, persistent_grid((const void*)k_grs_meet, 256), 256, 0, s, a));
         }
