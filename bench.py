@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Benchmark of the hot path: [0,2]-factor (M=5) + linear forest + permutation + tridiag.
 
-Contract (DESIGN.md §7): `python bench.py --gpus N --steps K --warmup W` prints ONE JSON
+Contract (DESIGN.md §8): `python bench.py --gpus N --steps K --warmup W` prints ONE JSON
 line on rank 0.  A step is one pass of the whole hot path over one synthetic graph resident
 in HBM; `value` is whole-job Medges/s (undirected edges E / step time).  Device time with
 CUDA events per step, L2 flushed between steps, max over ranks.
@@ -142,7 +142,7 @@ class Clocks:
 
 
 # ---------------------------------------------------------------------------
-# byte model (DESIGN.md §5; SURVEY.md §8(d))
+# byte model (DESIGN.md §9; SURVEY.md §8(d))
 # ---------------------------------------------------------------------------
 
 def survey_bytes(N, n, live_rows, live_nnz, with_lf=True):
@@ -156,7 +156,7 @@ def survey_bytes(N, n, live_rows, live_nnz, with_lf=True):
 
 
 def kernel_bytes(name, N, Z, n, live_rows, live_nnz, rows_ran=False):
-    """Algorithmic HBM bytes of one launch (DESIGN.md §5): what the method must move.
+    """Algorithmic HBM bytes of one launch (DESIGN.md §9): what the method must move.
     Rounds 1..M-1 run in ONE of two kernels (rows_ran: the rows mode did, the cached mode
     only raised its bail flag); their bytes go to that one."""
     base = name.split("[")[0]
@@ -501,7 +501,7 @@ def run_reference(args):
 def run_multi(args, ws, rank, local):
     """C5 row-partitioned over `ws` ranks: rank r generates and owns the z-planes
     [512 r / ws, 512 (r+1) / ws) and runs the partitioned factor (NCCL halo exchange), the
-    boundary-end-list linear forest and the tridiagonal extraction (DESIGN.md §8)."""
+    boundary-end-list linear forest and the tridiagonal extraction (DESIGN.md §10)."""
     import torch
     import torch.distributed as tdist
 

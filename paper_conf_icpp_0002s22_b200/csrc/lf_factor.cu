@@ -1,6 +1,6 @@
 // lf_factor.cu -- weighted [0,n]-factor, Algorithm 2 of PAPER.md (L93-L128, §3.2, §4.1).
 //
-// B200 design (DESIGN.md §4):
+// B200 design (DESIGN.md §5.1-§5.3):
 //  * one `propose` kernel per round (Alg. 2 L14-L22, the generalized SpMV of §4.1): G
 //    lanes per CSR row stream col/val with read-only loads, each lane keeps a sorted
 //    register top-n of 64-bit keys, a shuffle butterfly merges the G lists.  The key
@@ -9,7 +9,7 @@
 //    pi canonical, writes the next round's state byte (degree + charge, L8-L12) and
 //    appends still-live rows to the next worklist.  Rows whose charge-free candidate
 //    set became empty are retired: they provably never propose or receive a proposal
-//    again (DESIGN.md §4.2), so later rounds only touch live rows.
+//    again (DESIGN.md §5.2), so later rounds only touch live rows.
 //  * no host synchronisation: round count, worklist sizes and the maximality flags
 //    (L23-L25) stay on the device; the launch chain is fixed and graph-capturable.
 #include <cooperative_groups.h>
@@ -373,7 +373,7 @@ __global__ void LF_TILE_BOUNDS k_propose_tile(ProposeArgs a) {
 // ---------------------------------------------------------------------------
 // Round 0 as a pipelined stream: persistent CTAs walk their tiles while cp.async (LDGSTS)
 // copies the next tile's col/val range and the row pointers of the one after into the
-// other shared-memory stage, so HBM reads overlap the row scans (DESIGN.md §4.1).
+// other shared-memory stage, so HBM reads overlap the row scans (DESIGN.md §5.1).
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ void cp16(void* smem, const void* gmem) {
     const unsigned d = (unsigned)__cvta_generic_to_shared(smem);
@@ -974,7 +974,7 @@ struct FusedArgs {
 // Cached mode of rounds 1..M-1: every CTA owns a fixed slice of the round-1 worklist L1
 // (the rows mutual(0) kept) and keeps those rows -- state, confirmed keys and their CSR
 // entries as keys -- in shared memory for all rounds.  Rows outside L1 never propose
-// again and are never proposed to (DESIGN.md §4.2), so the slices cover every row the
+// again and are never proposed to (DESIGN.md §5.2), so the slices cover every row the
 // rounds touch.  Per round only two gathers remain: the state bytes of the entries'
 // targets (before propose, L15/L17) and the partners' proposals (before mutual, L27),
 // each one L2 level with every load of a CTA in flight together, instead of the

@@ -479,7 +479,7 @@ __device__ __forceinline__ void node_scan(TileSmem& s, int C, int* stats) {
     }
 }
 
-// Block-local ranking (DESIGN.md §4.3).  Same outputs as tile_scan, O(1) work per vertex:
+// Block-local ranking (DESIGN.md §5.4).  Same outputs as tile_scan, O(1) work per vertex:
 //  0. runs: maximal intervals of consecutive vertex ids linked in the factor (an x-line of
 //     a natural-order grid) are found with block-wide scans and contracted -- each end's
 //     slot into the run becomes a virtual link to the other end (weight = run length - 1,
@@ -1667,7 +1667,7 @@ __global__ void __launch_bounds__(256) k_perm_tri(int64_t N, const int32_t* __re
 }
 
 // ===========================================================================
-// Single-pass linear forest (DESIGN.md §4.3).  Every scan level carries the FULL window
+// Single-pass linear forest (DESIGN.md §5.4).  Every scan level carries the FULL window
 // of a vertex in one direction instead of one quantity per pass:
 //   pointer | R = edges covered | K = minimum edge key | DK = 2 * (distance to the near
 //   endpoint of that minimum edge) + [the near endpoint is the edge's min-id endpoint].
@@ -1882,7 +1882,7 @@ __device__ __forceinline__ void node_scan_full(TileSmemF& s, int C, int nt, int*
     }
 }
 
-// Block-local ranking with full windows (same phases as tile_rank, DESIGN.md §4.3).
+// Block-local ranking with full windows (same phases as tile_rank, DESIGN.md §5.4).
 // ek: real slot keys of the own vertices.  On return o[k] holds the vertex's result.
 __device__ void tile_rank_full(TileSmemF& s, int32_t b0, const ulonglong2 (&ek)[VPT], VRes (&o)[VPT],
                                int* stats) {
@@ -2803,7 +2803,7 @@ __global__ void __launch_bounds__(ET, LF_EMINB) k_lf_full2(ForestArgs a) {
             continue;
         }
         // on a cycle through other tiles (both terminals continue): is its weakest edge
-        // inside this vertex's segment?  (reading c9, DESIGN.md §4.3)
+        // inside this vertex's segment?  (reading c9, DESIGN.md §5.4)
         int2 c;
         if (st[k].kseg == ks) {
             const int delta = st[k].dseg >> 1, bt = st[k].dseg & 1;

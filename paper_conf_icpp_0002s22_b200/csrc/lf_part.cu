@@ -1,4 +1,4 @@
-// lf_part.cu -- the factor rounds row-partitioned across GPUs (SURVEY.md §8(e), DESIGN.md §8).
+// lf_part.cu -- the factor rounds row-partitioned across GPUs (SURVEY.md §8(e), DESIGN.md §10).
 //
 // Each GPU owns a contiguous row range [lo, hi) of A (global column ids).  Setup relabels
 // the columns into a local id space

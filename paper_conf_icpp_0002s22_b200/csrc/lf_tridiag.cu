@@ -4,7 +4,7 @@
 // The paper converts A to COO and scatters one thread per stored entry, checking forest
 // membership (L297).  Here the signed forest coefficients and the diagonal were captured
 // by lf_factor while it streamed the rows (pi_val, diag), so the pass is one thread per
-// vertex over O(N) bytes and never re-reads the CSR (DESIGN.md §4.4).
+// vertex over O(N) bytes and never re-reads the CSR (DESIGN.md §1).
 #include <cuda_runtime.h>
 
 #include <cstdint>

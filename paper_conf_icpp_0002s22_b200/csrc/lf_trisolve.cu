@@ -8,7 +8,7 @@
 // device flag (TriCtl::seq, set by the partition path's checks) makes one of them exit:
 //   - partition path (diagonally dominant T; k_part_pass1 / k_part_chain / k_part_pass2,
 //     below): fixed 32-row chunks, a reduced system of two unknowns per chunk swept per
-//     chain of coupled chunks, then one more pass per chunk (DESIGN.md §4.6);
+//     chain of coupled chunks, then one more pass per chunk (DESIGN.md §7);
 //   - sequential path (any other T): k_seg_solve, one thread per segment (found by a
 //     grid-stride scan of the rows), Gaussian elimination with scaled partial pivoting
 //     (the pivoting strategy of [21]; reading f2-1) streaming down the segment
@@ -92,7 +92,7 @@ __global__ void __launch_bounds__(128) k_seg_solve(int64_t N, const float* __res
 }
 
 // ---------------------------------------------------------------------------------------
-// Partition path (diagonally dominant T, DESIGN.md §4.6): fixed chunks of PK rows, one
+// Partition path (diagonally dominant T, DESIGN.md §7): fixed chunks of PK rows, one
 // thread per chunk, PB chunks per block staged through shared memory with coalesced loads.
 //   pass 1: each chunk solves T_j z = rhs for rhs = x_j, -a[s] e_1, -c[e] e_K (Thomas,
 //           no pivoting: stable under diagonal dominance) and keeps the first and last

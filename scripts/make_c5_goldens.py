@@ -7,7 +7,7 @@ size, and it would take it several minutes, so this script (which calls ONLY lfg
 oracle/) runs the oracle once here and stores sha256 digests of every output, plus a few
 thousand sampled values for diagnosis, in tests/golden/c5_<n>_n2.json.  The GPU test
 (tests/test_gpu_c5.py) regenerates the graph on the device, runs the CUDA path and compares
-digests -- bit-exact parity at full size (DESIGN.md §6).  No value here comes from the
+digests -- bit-exact parity at full size (DESIGN.md §2.1).  No value here comes from the
 CUDA path.
 
     python scripts/make_c5_goldens.py            # n = 512 (~45 GB RAM, ~30 min)

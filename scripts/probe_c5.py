@@ -1,5 +1,5 @@
 """Per-kernel times of the hot path on the C5 recipe (n^3 27-pt, device generator) under
-several environment settings (diagnostics for DESIGN.md §4; not a bench number).
+several environment settings (diagnostics for DESIGN.md §5 and §8; not a bench number).
 usage: python scripts/probe_c5.py [n] 'ENV=a,ENV2=b' 'ENV=c' ..."""
 import json
 import os

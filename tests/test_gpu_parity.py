@@ -1,6 +1,6 @@
 """CUDA path (through the C ABI) vs the CPU oracle, element by element, bit-exact.
 
-Parity bar: factor edges, |w|, signed values, diagonal, live-row counters,
+Parity bar (DESIGN.md §3 reading c18): factor edges, |w|, signed values, diagonal, live-row counters,
 round count, forest, path IDs, positions, perm/iperm and a/b/c are integer or copied fp32
 data, so every comparison is exact equality (no tolerance).
 """
@@ -152,7 +152,7 @@ SMALL_ZEROS = [
     ("c5_small_zeros", lambda: with_zeros(lfgen.grid3d_27pt(12), frac=0.3)),
     ("random_zeros_shuffled", lambda: with_zeros(lfgen.random_graph(2000, 7000, seed=2, shuffle_cols_seed=4))),
 ]
-FOREST_MODES = ["tile", "grs"]  # DESIGN.md §4.3 tile path / §4.3a global ruling set
+FOREST_MODES = ["tile", "grs"]  # DESIGN.md §5.4 tile path / §5.5 global ruling set
 
 
 @pytest.mark.parametrize("forest", FOREST_MODES)
@@ -269,7 +269,7 @@ def test_factor_unaligned_inputs(torch_cuda, lfm, oracle_mod):
 
 @pytest.mark.parametrize("cfg", ["C2", "C3"])
 def test_repeated_runs_cached_and_uncached_rounds(torch_cuda, lfm, oracle_mod, monkeypatch, cfg):
-    """Rounds 1..M-1 in both modes (shared-memory cached / global worklists, DESIGN.md §4.2),
+    """Rounds 1..M-1 in both modes (shared-memory cached / global worklists, DESIGN.md §5.3),
     five back-to-back runs each on one workspace without a host sync in between: every run
     equals the oracle-checked first one (catches races that a single run can miss)."""
     torch = torch_cuda

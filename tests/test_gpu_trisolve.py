@@ -1,7 +1,7 @@
 """lf_tri_solve (applying the tridiagonal preconditioner, PAPER.md
 L37, L447, ref. [21]) through the C ABI vs oracle.tri_solve (fp64 banded LU).
 
-Tolerance (DESIGN.md §4.5, readings f2-3 and f2-5): the kernel computes in fp32 (L301), the oracle in fp64, so
+Tolerance (DESIGN.md §7, readings f2-3 and f2-5): the kernel computes in fp32 (L301), the oracle in fp64, so
 results agree up to rounding, not bit for bit.  Two bars, both derived from fp32
 Gaussian elimination with partial pivoting on a tridiagonal system (growth factor <= 2):
   backward error  per independent block B (split where a[r] = c[r-1] = 0):
