@@ -1408,7 +1408,7 @@ __device__ __forceinline__ void write_prop(const RowsArgs& a, int32_t v, int deg
 #endif
 constexpr int kRowsBud = LF_ROWS_BUD;  // staged entries per warp (640: 3 CTAs of 8 warps per SM)
 constexpr int kRowsWarps = LF_ROWS_T / 32;
-template <int BUD>
+template <int BUD, int NQ = 4>
 struct RowsWarpSmemT {
     int32_t col[BUD];
     uint32_t val[BUD];
@@ -1416,22 +1416,28 @@ struct RowsWarpSmemT {
     int64_t qrs[64];      // queue of live rows: CSR start
     int32_t qv[64];       //   vertex
     int32_t qlen[64];     //   entries
-    int32_t qp[64][4];    //   confirmed slots
+    int32_t qp[64][NQ];   //   confirmed slots
     uint8_t qst[64];      //   state byte
 };
 using RowsWarpSmem = RowsWarpSmemT<kRowsBud>;
 struct RowsSmem {
     RowsWarpSmem w[kRowsWarps];
 };
-// the per-round propose kernel of large graphs: 4 warps per CTA, whole 32-row batches
-constexpr int kRowsBudK = 1024, kRowsTK = 128;
+// the per-round propose kernel of large graphs: 4 warps per CTA, whole 32-row batches; the
+// queue keeps n confirmed slots per row, so that 4 CTAs (16 warps) fit an SM for n <= 2
+// (with 4 slots: 3 CTAs, 12 warps)
+#ifndef LF_ROWSK_BUD
+#define LF_ROWSK_BUD 1024
+#endif
+constexpr int kRowsBudK = LF_ROWSK_BUD, kRowsTK = 128;
+template <int NN>
 struct RowsSmemK {
-    RowsWarpSmemT<kRowsBudK> w[kRowsTK / 32];
+    RowsWarpSmemT<kRowsBudK, NN> w[kRowsTK / 32];
 };
 
 // one batch: the longest prefix of the queue whose aligned ranges fit; returns its size
-template <int NN, int BUD>
-__device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmemT<BUD>& S, int qcnt, bool charging,
+template <int NN, int BUD, int NQ>
+__device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmemT<BUD, NQ>& S, int qcnt, bool charging,
                                           bool bulk_ok, int64_t nnz, unsigned long long& my_live,
                                           unsigned long long& my_nnz, int& my_prop) {
     const int lane = threadIdx.x & 31;
@@ -1532,8 +1538,8 @@ __device__ __forceinline__ int rows_batch(const RowsArgs& a, RowsWarpSmemT<BUD>&
     return nb;
 }
 
-template <int NN, int G, int BUD>
-__device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool charging, RowsWarpSmemT<BUD>& S) {
+template <int NN, int G, int BUD, int NQ = 4>
+__device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool charging, RowsWarpSmemT<BUD, NQ>& S) {
     const int lane = threadIdx.x & 31;
     const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -1584,9 +1590,9 @@ __device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool char
         }
         qcnt += __popc(m);
         __syncwarp();
-        while (qcnt >= 32) qcnt -= rows_batch<NN, BUD>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
+        while (qcnt >= 32) qcnt -= rows_batch<NN, BUD, NQ>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
     }
-    while (qcnt > 0) qcnt -= rows_batch<NN, BUD>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
+    while (qcnt > 0) qcnt -= rows_batch<NN, BUD, NQ>(a, S, qcnt, charging, bulk_ok, nnz, my_live, my_nnz, my_prop);
 #pragma unroll
     for (int off = 16; off >= 1; off >>= 1) {
         my_live += __shfl_xor_sync(0xffffffffu, my_live, off);
@@ -1871,11 +1877,11 @@ template <int NN>
 __global__ void __launch_bounds__(kRowsTK) k_rows_propose_k(RowsArgs a) {
     LF_TL(g_tl_factor, 5);
     extern __shared__ __align__(16) unsigned char rows_smem_k[];
-    auto& S = reinterpret_cast<RowsSmemK*>(rows_smem_k)->w[threadIdx.x >> 5];
+    auto& S = reinterpret_cast<RowsSmemK<NN>*>(rows_smem_k)->w[threadIdx.x >> 5];
     pdl_wait();
     pdl_trigger();
     if (a.bail && *(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
-    rows_propose<NN, 1, kRowsBudK>(a, a.only_k, (a.only_k % a.m) != a.k_m, S);
+    rows_propose<NN, 1, kRowsBudK, NN>(a, a.only_k, (a.only_k % a.m) != a.k_m, S);
 }
 template <int NN>
 __global__ void __launch_bounds__(256) k_rows_long_k(RowsArgs a) {
@@ -2105,7 +2111,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
         static bool pattr = false;
         if (!pattr) {
             LF_CUDA(cudaFuncSetAttribute((const void*)k_rows_propose_k<NN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)sizeof(RowsSmemK)));
+                                         (int)sizeof(RowsSmemK<NN>)));
             pattr = true;
         }
     }
@@ -2156,8 +2162,8 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             } else if (rows_part) {
                 pr.only_k = k;
                 LF_CUDA(launch_pdl(k_rows_propose_k<NN>,
-                                   persistent_grid((const void*)k_rows_propose_k<NN>, kRowsTK, sizeof(RowsSmemK)),
-                                   kRowsTK, sizeof(RowsSmemK), s, pr));
+                                   persistent_grid((const void*)k_rows_propose_k<NN>, kRowsTK, sizeof(RowsSmemK<NN>)),
+                                   kRowsTK, sizeof(RowsSmemK<NN>), s, pr));
             } else {
                 pa.defer_len = 32 * G;
                 launch_propose<NN>(G, pa, grid_p, s);
@@ -2362,7 +2368,7 @@ static int factor_impl(const lf_csr_t* A, const lf_factor_opts_t* o, int32_t* pi
             const bool split = sp ? strcmp(sp, "0") != 0 : N >= ((int64_t)1 << 22);
             if (split) {
                 const void* kp = (const void*)k_rows_propose_k<NN>;
-                const int psm = (int)sizeof(RowsSmemK);
+                const int psm = (int)sizeof(RowsSmemK<NN>);
                 static bool pattr = false;
                 if (!pattr) {
                     LF_CUDA(cudaFuncSetAttribute(kp, cudaFuncAttributeMaxDynamicSharedMemorySize, psm));
