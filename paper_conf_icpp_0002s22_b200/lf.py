@@ -253,11 +253,28 @@ def linear_forest_tridiag(pi2, pi2_w, pi2_val, diag, *, ws=None, out=None, n_cyc
     return out
 
 
+def _check_csr(name, rowptr, col, val):
+    """raw pointers cross the ABI: dtype, device, contiguity and lengths are checked here"""
+    torch = _torch()
+    for nm, t, dt in (("rowptr", rowptr, torch.int64), ("col", col, torch.int32), ("val", val, torch.float32)):
+        if not (t.is_cuda and t.dtype == dt and t.is_contiguous() and t.dim() == 1):
+            raise LFError(f"{name}: {nm} must be a contiguous 1-D {dt} CUDA tensor")
+    if col.numel() != val.numel():
+        raise LFError(f"{name}: col and val lengths differ")
+
+
+def _check_i32(name, nm, t, numel):
+    torch = _torch()
+    if not (t.is_cuda and t.dtype == torch.int32 and t.is_contiguous() and t.numel() == numel):
+        raise LFError(f"{name}: {nm} must be a contiguous int32 CUDA tensor of {numel} elements")
+
+
 def symmetrize(rowptr, col, val, *, ws=None):
     """lf_symmetrize: S = A' + A'^T of a (possibly non-symmetric) device CSR -> (rowptr, col,
     val) of S, trimmed to its stored entries (one device-to-host read of the count)."""
     torch = _torch()
     L = load()
+    _check_csr("symmetrize", rowptr, col, val)
     N = rowptr.numel() - 1
     nnz = col.numel()
     dev = rowptr.device
@@ -280,7 +297,11 @@ def orig_coeffs(rowptr, col, val, pi, *, out=None):
     """lf_orig_coeffs: (pi_val [N, n], diag [N]) of the ORIGINAL A on the factor slots pi."""
     torch = _torch()
     L = load()
+    _check_csr("orig_coeffs", rowptr, col, val)
     N, n = pi.shape
+    if rowptr.numel() != N + 1:
+        raise LFError("orig_coeffs: pi must have one row per vertex of A")
+    _check_i32("orig_coeffs", "pi", pi, N * n)
     if out is None:
         out = (torch.empty((N, n), dtype=torch.float32, device=pi.device),
                torch.empty(N, dtype=torch.float32, device=pi.device))
@@ -305,8 +326,10 @@ def coarsen(rowptr, col, val, mu, *, ws=None):
     (cid [N], members [Nc, 2], (c_rowptr, c_col, c_val)) trimmed (one host read of Nc, nnz)."""
     torch = _torch()
     L = load()
+    _check_csr("coarsen", rowptr, col, val)
     N = rowptr.numel() - 1
     nnz = col.numel()
+    _check_i32("coarsen", "mu", mu, N)
     dev = rowptr.device
     cid = torch.empty(max(N, 1), dtype=torch.int32, device=dev)
     members = torch.empty((max(N, 1), 2), dtype=torch.int32, device=dev)
@@ -327,7 +350,11 @@ def block_tridiag(rowptr, col, val, members, cforest, cperm):
     """lf_block_tridiag -> (D, L, U) [Nc, 4] row-major 2x2 blocks, fperm [Nc, 2] (-1 ghost)."""
     torch = _torch()
     Lb = load()
+    _check_csr("block_tridiag", rowptr, col, val)
     nc = members.shape[0]
+    _check_i32("block_tridiag", "members", members, 2 * nc)
+    _check_i32("block_tridiag", "cforest", cforest, 2 * nc)
+    _check_i32("block_tridiag", "cperm", cperm, nc)
     dev = members.device
     D, Lo, U = (torch.empty((max(nc, 1), 4), dtype=torch.float32, device=dev) for _ in range(3))
     fperm = torch.empty((max(nc, 1), 2), dtype=torch.int32, device=dev)
