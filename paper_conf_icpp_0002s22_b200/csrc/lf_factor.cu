@@ -475,7 +475,10 @@ __global__ void __launch_bounds__(T) k_propose_stream(ProposeArgs a) {
     constexpr int R = T / G;
     extern __shared__ __align__(16) unsigned char sraw[];
     StreamSmem<SE>& S = *reinterpret_cast<StreamSmem<SE>*>(sraw);
-    pdl_trigger();  // the long-row pass may launch and wait meanwhile
+    // small graphs: the long-row pass may launch and wait meanwhile (hides its launch); large
+    // ones trigger at exit -- early-launched dependents sharing the SMs with this persistent
+    // kernel cost more than the launch they hide (C5 graph replay 54.0 vs 45.1 ms without)
+    if (a.N < ((int64_t)1 << 22)) pdl_trigger();
     const int tid = threadIdx.x;
     const int64_t ntiles = (a.N + R - 1) / R;
     const int64_t t0 = blockIdx.x;
@@ -1882,14 +1885,12 @@ __global__ void __launch_bounds__(kRowsTK) k_rows_propose_k(RowsArgs a) {
     extern __shared__ __align__(16) unsigned char rows_smem_k[];
     auto& S = reinterpret_cast<RowsSmemK<NN>*>(rows_smem_k)->w[threadIdx.x >> 5];
     pdl_wait();
-    pdl_trigger();
     if (a.bail && *(volatile const int32_t*)a.bail == 0) return;  // the cached mode ran the rounds
     rows_propose<NN, 1, kRowsBudK, NN>(a, a.only_k, (a.only_k % a.m) != a.k_m, S);
 }
 template <int NN>
 __global__ void __launch_bounds__(256) k_rows_long_k(RowsArgs a) {
     pdl_wait();
-    pdl_trigger();
     if (a.bail && *(volatile const int32_t*)a.bail == 0) return;
     if (*(volatile int32_t*)&a.long_count[a.only_k] > 0) rows_long<NN>(a, a.only_k, (a.only_k % a.m) != a.k_m);
 }
@@ -1897,7 +1898,6 @@ template <int NN>
 __global__ void __launch_bounds__(256) k_rows_mutual_k(RowsArgs a) {
     LF_TL(g_tl_factor, 6);
     pdl_wait();
-    pdl_trigger();
     if (a.bail && *(volatile const int32_t*)a.bail == 0) return;
     const int k = a.only_k;
     const bool last = k == a.M - 1;

@@ -3074,7 +3074,6 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
     LF_TL(g_tl_forest, 5);
     __shared__ int wsum[8];
     pdl_wait();
-    pdl_trigger();
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int64_t chunk = (int64_t)blockDim.x * kPackV;  // 2048 (k_grs_list's chunk)
     for (int64_t c0 = (int64_t)blockIdx.x * chunk; c0 < a.N; c0 += (int64_t)gridDim.x * chunk) {
@@ -3117,7 +3116,6 @@ __global__ void __launch_bounds__(256) k_grs_pack(ForestArgs a) {
 __global__ void __launch_bounds__(256) k_grs_list(ForestArgs a) {
     LF_TL(g_tl_forest, 14);
     pdl_wait();
-    pdl_trigger();
     const int lane = threadIdx.x & 31;
     const int64_t chunks = (a.N + 2047) / 2048, words = (a.N + 31) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -3167,7 +3165,6 @@ __device__ __forceinline__ void walk_leave(const ForestArgs& a, int t, int32_t l
 __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
     LF_TL(g_tl_forest, 6);
     pdl_wait();
-    pdl_trigger();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     const int lane = threadIdx.x & 31;
     // dynamic schedule: a warp takes the next 32 walks when its last one has ended, so the
@@ -3255,7 +3252,6 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
 __global__ void __launch_bounds__(256) k_grs_meet(ForestArgs a) {
     LF_TL(g_tl_forest, 12);
     pdl_wait();
-    pdl_trigger();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt; t += gridDim.x * blockDim.x) {
         const int2 st = __ldcg(a.grs_mstop + t);
@@ -3373,7 +3369,6 @@ __device__ __forceinline__ GrsOut grs_vertex(int32_t x, int2 nb, int fslot, int3
 __global__ void __launch_bounds__(256) k_grs_len(ForestArgs a) {
     LF_TL(g_tl_forest, 7);
     pdl_wait();
-    pdl_trigger();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
         const GrsWin W = grs_window(a, i, 0);
@@ -3401,7 +3396,6 @@ __device__ __forceinline__ uint64_t grs_prio(int32_t v) {
 __global__ void __launch_bounds__(256) k_grs_cyccand(ForestArgs a) {
     LF_TL(g_tl_forest, 15);
     pdl_wait();
-    pdl_trigger();
     const int lane = threadIdx.x & 31;
     const int64_t words = (a.N + 31) >> 5;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -3508,7 +3502,6 @@ __device__ __forceinline__ void grs_cyc_walk(const ForestArgs& a, int32_t v, int
 __global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
     LF_TL(g_tl_forest, 8);
     pdl_wait();
-    pdl_trigger();
     const int ncand = __ldcg(&a.ctl[kCtlCand]);
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     // a static stride (a dynamic schedule's counter was one more hot line: 1.8 vs 1.4 ms)
@@ -3521,7 +3514,6 @@ __global__ void __launch_bounds__(ET) k_grs_lenscan(ForestArgs a) {
     LF_TL(g_tl_forest, 9);
     __shared__ int sh[32 * EV];
     pdl_wait();
-    pdl_trigger();
     const int64_t b0 = a.lo + (int64_t)blockIdx.x * LB;
     int lens[EV], e[EV], tot[EV];
 #pragma unroll
@@ -3552,7 +3544,6 @@ constexpr int kDescBad = 8;
 __global__ void __launch_bounds__(256) k_grs_desc(ForestArgs a) {
     LF_TL(g_tl_forest, 13);
     pdl_wait();
-    pdl_trigger();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     // descriptors fit [N]: splitters and splitter-free cycles (>= 3 vertices each) are
     // disjoint on a valid factor; a malformed one is cut off (its vertices flag it in the emit)
