@@ -1895,7 +1895,13 @@ __global__ void __launch_bounds__(256) k_rows_long_k(RowsArgs a) {
     if (*(volatile int32_t*)&a.long_count[a.only_k] > 0) rows_long<NN>(a, a.only_k, (a.only_k % a.m) != a.k_m);
 }
 template <int NN>
-__global__ void __launch_bounds__(256) k_rows_mutual_k(RowsArgs a) {
+#ifndef LF_RMUT_MINB
+#define LF_RMUT_MINB 1
+#endif
+#ifndef LF_RMUT_MB
+#define LF_RMUT_MB 2  // rows in flight per thread (C5 rounds 1-4: 2 -> 6.86 ms, 4 -> 7.09 ms)
+#endif
+__global__ void __launch_bounds__(256, LF_RMUT_MINB) k_rows_mutual_k(RowsArgs a) {
     LF_TL(g_tl_factor, 6);
     pdl_wait();
     if (a.bail && *(volatile const int32_t*)a.bail == 0) return;
@@ -1903,7 +1909,7 @@ __global__ void __launch_bounds__(256) k_rows_mutual_k(RowsArgs a) {
     const bool last = k == a.M - 1;
     if (last && blockIdx.x == 0 && (a.rounds || a.live))
         finalize_body(a.flags, a.M, a.m, a.k_m, a.rounds, a.live_part, a.live);
-    rows_mutual<NN, 4>(a, k, last);
+    rows_mutual<NN, LF_RMUT_MB>(a, k, last);
 }
 
 // state of round 0 when round 0 is charged (k_m != 0): degree 0 + charge(v, 0)
