@@ -382,9 +382,12 @@ def measure(torch, lf, g, n, steps, warmup, flush, use_graph=True):
         step(prof=True)
         torch.cuda.synchronize()
         recs = lf.profile_collect()
-        # one record per stage; the perm stage launches k_tile_prefix + k_perm_tri, and every
-        # lf_linear_forest call starts with the (unrecorded) control-block kernel k_ctl_zero
-        launches = sum(2 if nm in ("perm", "perm_tridiag") else 1 for nm, _ in recs) + (1 if n == 2 else 0)
+        # one record per profiled group; groups of several kernels: perm (k_tile_prefix +
+        # k_perm_tri), grs_pack (pack, k_tile_prefix, list), grs_walk (walk, meet), grs_len
+        # (len, cyccand, cycfind, lenscan, k_tile_prefix); every lf_linear_forest call starts
+        # with the (unrecorded) control-block kernel k_ctl_zero
+        mult = {"perm": 2, "perm_tridiag": 2, "grs_pack": 3, "grs_walk": 2, "grs_len": 5}
+        launches = sum(mult.get(nm, 1) for nm, _ in recs) + (1 if n == 2 else 0)
         for nm, ms in recs:
             kern.setdefault(nm, []).append(ms)
     t = sorted(step_ms)[len(step_ms) // 2]
