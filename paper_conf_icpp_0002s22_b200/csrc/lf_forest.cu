@@ -3547,24 +3547,7 @@ __global__ void __launch_bounds__(256) k_grs_desc(ForestArgs a) {
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     // descriptors fit [N]: splitters and splitter-free cycles (>= 3 vertices each) are
     // disjoint on a valid factor; a malformed one is cut off (its vertices flag it in the emit)
-    const int64_t ncl = kCycStripes * grs_cyc_cap(a.N);  // the cycle index space (striped)
-    int lmax = 0;
-    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < cnt + ncl; j += (int64_t)gridDim.x * blockDim.x) {
-        GrsWin W;
-        if (j < cnt) {
-            W = grs_window(a, (int)j, 0);
-        } else {
-            const int64_t c = j - cnt;
-            if (!grs_cyc_valid(a, c)) continue;
-            const int4 cr = __ldcg(a.grs_cyc + c);
-            lmax = max(lmax, cr.z);
-            W.cyc = true;
-            W.ks = __ldcg(a.grs_cyck + c);
-            W.pf = cr.y >> 1;
-            W.bf = cr.y & 1;
-            W.pb = cr.z - W.pf - 1;
-            W.bb = W.bf ^ 1;  // the far endpoint of the weakest edge
-        }
+    auto put = [&](int64_t j, const GrsWin& W) {
         int32_t L;
         const int32_t l = grs_path_id(W, L);
         int4 h0, h1 = make_int4(0, 0, 0, 0);
@@ -3581,8 +3564,29 @@ __global__ void __launch_bounds__(256) k_grs_desc(ForestArgs a) {
                 h1 = make_int4(back ? 1 : -1, 0, 0, 0);
             }
         }
-        a.grs_desc[2 * (int64_t)j] = h0;
-        a.grs_desc[2 * (int64_t)j + 1] = h1;
+        a.grs_desc[2 * j] = h0;
+        a.grs_desc[2 * j + 1] = h1;
+    };
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x, t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (int64_t j = t0; j < cnt; j += stride) put(j, grs_window(a, (int)j, 0));
+    // the splitter-free cycles: the filled part of every stripe of the cycle index space
+    const int64_t cap = grs_cyc_cap(a.N);
+    int lmax = 0;
+    for (int sidx = 0; sidx < kCycStripes; sidx++) {
+        const int64_t ns = min((int64_t)__ldcg(&a.ctl[kCtlCycS + kCtlCycStride * sidx]), cap);
+        for (int64_t q = t0; q < ns; q += stride) {
+            const int64_t c = sidx * cap + q;
+            const int4 cr = __ldcg(a.grs_cyc + c);
+            lmax = max(lmax, cr.z);
+            GrsWin W;
+            W.cyc = true;
+            W.ks = __ldcg(a.grs_cyck + c);
+            W.pf = cr.y >> 1;
+            W.bf = cr.y & 1;
+            W.pb = cr.z - W.pf - 1;
+            W.bb = W.bf ^ 1;  // the far endpoint of the weakest edge
+            put(cnt + c, W);
+        }
     }
 #pragma unroll
     for (int o = 16; o; o >>= 1) lmax = max(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));
