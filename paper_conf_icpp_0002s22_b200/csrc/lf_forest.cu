@@ -3510,26 +3510,51 @@ __global__ void __launch_bounds__(256) k_grs_cycfind(ForestArgs a) {
 }
 
 // tile-local exclusive prefix of the path lengths (the tail of k_lf_full2)
-__global__ void __launch_bounds__(ET) k_grs_lenscan(ForestArgs a) {
+// LB / 8 threads per tile, 8 consecutive lengths each (two 16-byte loads): a serial local
+// scan, one warp scan and one scan of the warp totals (a per-element block scan spent ~60
+// instructions per vertex: the C5 len group 1.41 -> 1.24 ms)
+constexpr int kLsT = LB / 8;
+__global__ void __launch_bounds__(kLsT) k_grs_lenscan(ForestArgs a) {
     LF_TL(g_tl_forest, 9);
-    __shared__ int sh[32 * EV];
+    __shared__ int wsum[kLsT / 32];
     pdl_wait();
     const int64_t b0 = a.lo + (int64_t)blockIdx.x * LB;
-    int lens[EV], e[EV], tot[EV];
+    const int64_t g0 = b0 + 8 * (int64_t)threadIdx.x;
+    int x[8];
+    if (g0 + 8 <= a.hi && ((((uintptr_t)(a.len + g0)) & 15) == 0)) {
+        const int4 u = __ldcs(reinterpret_cast<const int4*>(a.len + g0));
+        const int4 w = __ldcs(reinterpret_cast<const int4*>(a.len + g0) + 1);
+        x[0] = u.x; x[1] = u.y; x[2] = u.z; x[3] = u.w; x[4] = w.x; x[5] = w.y; x[6] = w.z; x[7] = w.w;
+    } else {
 #pragma unroll
-    for (int k = 0; k < EV; k++) {
-        const int64_t g = b0 + threadIdx.x + k * ET;
-        lens[k] = g < a.hi ? __ldcg(a.len + g) : 0;
+        for (int k = 0; k < 8; k++) x[k] = g0 + k < a.hi ? __ldcg(a.len + g0 + k) : 0;
     }
-    block_scan_sum_excl_v<EV>(lens, sh, e, tot);
-    int carry = 0;
+    int t = 0;
 #pragma unroll
-    for (int k = 0; k < EV; k++) {
-        const int64_t gk = b0 + threadIdx.x + k * ET;
-        if (gk < a.hi && lens[k]) a.off[gk] = carry + e[k];
-        carry += tot[k];
+    for (int k = 0; k < 8; k++) t += x[k];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int inc = t;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
     }
-    if (threadIdx.x == 0) a.tsum[blockIdx.x] = carry;
+    if (lane == 31) wsum[w] = inc;
+    __syncthreads();
+    int before = 0, total = 0;
+#pragma unroll
+    for (int q = 0; q < kLsT / 32; q++) {
+        const int ws = wsum[q];
+        before += q < w ? ws : 0;
+        total += ws;
+    }
+    int run = before + inc - t;  // exclusive prefix of this thread's first value in the tile
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+        if (x[k] && g0 + k < a.hi) a.off[g0 + k] = run;
+        run += x[k];
+    }
+    if (threadIdx.x == 0) a.tsum[blockIdx.x] = total;
 }
 
 // Walk descriptors: one 32-byte record per splitter j < cnt (its walks t = 2j + f) and per
@@ -3848,7 +3873,7 @@ int forest_run(int64_t N, const int32_t* pi2, const float* pi2_w, int32_t* fores
             LF_CUDA(launch_pdl(k_grs_len, persistent_grid((const void*)k_grs_len, 256), 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_cyccand, persistent_grid((const void*)k_grs_cyccand, 256), 256, 0, s, a));
             LF_CUDA(launch_pdl(k_grs_cycfind, persistent_grid((const void*)k_grs_cycfind, 256), 256, 0, s, a));
-            LF_CUDA(launch_pdl(k_grs_lenscan, tiles, ET, 0, s, a));
+            LF_CUDA(launch_pdl(k_grs_lenscan, tiles, kLsT, 0, s, a));
             LF_CUDA(launch_pdl(k_tile_prefix, 1, kPrefT, 0, s, w.tsum, tiles, (const int*)w.ctl,
                                (unsigned long long*)n_cycles, 1));
         }
