@@ -3396,11 +3396,15 @@ __device__ __forceinline__ uint64_t grs_prio(int32_t v) {
 __global__ void __launch_bounds__(256) k_grs_cyccand(ForestArgs a) {
     LF_TL(g_tl_forest, 15);
     pdl_wait();
-    const int lane = threadIdx.x & 31;
+    __shared__ int s_w[8];
+    __shared__ int s_base;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int64_t words = (a.N + 31) >> 5;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t w0 = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); w0 < words; w0 += stride) {
-        const int64_t wi = w0 + lane;
+    // block-uniform loop: one list atomic per CTA and pass (a per-warp atomic put ~10^5 on one
+    // control line, the hot spot of §5.5)
+    for (int64_t b0 = (int64_t)blockIdx.x * blockDim.x; b0 < words; b0 += stride) {
+        const int64_t wi = b0 + threadIdx.x;
         uint32_t m = 0;
         if (wi < words) {
             m = ~__ldcg(a.grs_bits + wi);
@@ -3423,10 +3427,16 @@ __global__ void __launch_bounds__(256) k_grs_cyccand(ForestArgs a) {
             const int y = __shfl_up_sync(0xffffffffu, incl, o);
             if (lane >= o) incl += y;
         }
-        int base = 0;
-        if (lane == 31 && incl) base = atomicAdd(&a.ctl[kCtlCand], incl);
-        base = __shfl_sync(0xffffffffu, base, 31);
-        int pos = base + incl - n;
+        if (lane == 31) s_w[wid] = incl;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int tsum = 0;
+            for (int q = 0; q < (int)(blockDim.x >> 5); q++) { const int x = s_w[q]; s_w[q] = tsum; tsum += x; }
+            s_base = tsum ? atomicAdd(&a.ctl[kCtlCand], tsum) : 0;
+        }
+        __syncthreads();
+        int pos = s_base + s_w[wid] + incl - n;
+        __syncthreads();  // s_w / s_base are reused by the next pass
         while (cm) {
             const int bit = __ffs(cm) - 1;
             cm &= cm - 1u;
