@@ -3162,6 +3162,9 @@ __device__ __forceinline__ void walk_leave(const ForestArgs& a, int t, int32_t l
     a.grs_meetk[2 * (int64_t)last + slot] = K;
 }
 
+#ifndef LF_WALK_PAIR
+#define LF_WALK_PAIR 2
+#endif
 __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
     LF_TL(g_tl_forest, 6);
     pdl_wait();
@@ -3174,9 +3177,13 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
     // ones that are done take their next walks together (__activemask) without waiting for
     // the rest of the warp.  (A full-warp grab of 32 walks after all lanes are done measured
     // 11.5 ms, 4 x 32 at a time 7.7 ms, this one 6.0 ms.)
+    // LF_WALK_PAIR: a lane takes both walks of a splitter (t, t + 1) per grab -- half the
+    // atomics on the schedule counter, whose single address bounded the walk (C5: 1 walk
+    // per grab 6.0 ms, 2 walks 5.4 ms, 4 walks 5.6 ms)
     int b = 0;
-    if (lane == 0) b = atomicAdd(&a.ctl[kCtlWalk], 32);
-    for (int t = __shfl_sync(0xffffffffu, b, 0) + lane; t < 2 * cnt;) {
+    if (lane == 0) b = atomicAdd(&a.ctl[kCtlWalk], 32 * LF_WALK_PAIR);
+    int spare = LF_WALK_PAIR - 1;
+    for (int t = __shfl_sync(0xffffffffu, b, 0) + LF_WALK_PAIR * lane; t < 2 * cnt;) {
         const int i = t >> 1, f = t & 1;
         const int32_t sv = __ldcg(a.list1 + i);
         int2 nbs;
@@ -3239,11 +3246,17 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
         r[f] = R;
         d[f] = DK;
         k[f] = K;
+        if (spare > 0) {  // the other walk of the same grab
+            spare--;
+            t++;
+            continue;
+        }
         const unsigned act = __activemask();
         const int ld = __ffs(act) - 1;
         int nb = 0;
-        if (lane == ld) nb = atomicAdd(&a.ctl[kCtlWalk], __popc(act));
-        t = __shfl_sync(act, nb, ld) + __popc(act & ((1u << lane) - 1u));
+        if (lane == ld) nb = atomicAdd(&a.ctl[kCtlWalk], LF_WALK_PAIR * __popc(act));
+        t = __shfl_sync(act, nb, ld) + LF_WALK_PAIR * __popc(act & ((1u << lane) - 1u));
+        spare = LF_WALK_PAIR - 1;
     }
 }
 
