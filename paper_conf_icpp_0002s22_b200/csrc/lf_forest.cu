@@ -72,10 +72,15 @@ constexpr int kCtlBad = 135;      // the tile path met a malformed factor: later
 constexpr int kCtlBadGrs = 136;   // a ruling-set walk met one (bounded; records stay well formed)
 constexpr int kCtlWalk = 137;     // next walk handed out by k_grs_walk (dynamic schedule)
 constexpr int kCtlCycMax = 138;   // longest splitter-free cycle (lf_forest_stats)
+#ifndef LF_WALK_CTRS
+#define LF_WALK_CTRS 4
+#endif
 constexpr int kCycStripes = 32;   // counters of the splitter-free cycles (k_grs_cycfind),
 constexpr int kCtlCycS = 256;     //   ctl[256 + 32 s]: one 128-byte line each (atomics on one
 constexpr int kCtlCycStride = 32; //   line queue behind each other in its L2 slice)
-constexpr int kCtlInts = 256 + kCycStripes * kCtlCycStride;
+constexpr int kWalkCtrs = LF_WALK_CTRS;  // schedule counters of k_grs_walk, one line each
+constexpr int kCtlWalkC = 256 + kCycStripes * kCtlCycStride;
+constexpr int kCtlInts = kCtlWalkC + 4 * kCtlCycStride;
 constexpr int kCtlCand = 139;     // candidates of k_grs_cyccand (list2)
 constexpr int kMaxSteps = 62;
 constexpr int kCtlStat = 192;     // ctl[192..]: diagnostics (lf_forest_stats)
@@ -3180,10 +3185,20 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
     // LF_WALK_PAIR: a lane takes both walks of a splitter (t, t + 1) per grab -- half the
     // atomics on the schedule counter, whose single address bounded the walk (C5: 1 walk
     // per grab 6.0 ms, 2 walks 5.4 ms, 4 walks 5.6 ms)
+    // kWalkCtrs counters (one 128-byte line each) hand out interleaved chunks of 2048 walks:
+    // counter c's n-th walk is walk (n / 2048 * kWalkCtrs + c) * 2048 + n % 2048, so the
+    // counters advance together and the walks in flight stay one band
+    int* ctr = a.ctl + kCtlWalkC + kCtlCycStride * (int)(blockIdx.x % kWalkCtrs);
+    const int cidx = (int)(blockIdx.x % kWalkCtrs);
+    auto walk_of = [&](int u) -> int {
+        const int64_t w = ((int64_t)(u >> 11) * kWalkCtrs + cidx) * 2048 + (u & 2047);
+        return w < 2 * (int64_t)cnt ? (int)w : INT_MAX;
+    };
     int b = 0;
-    if (lane == 0) b = atomicAdd(&a.ctl[kCtlWalk], 32 * LF_WALK_PAIR);
+    if (lane == 0) b = atomicAdd(ctr, 32 * LF_WALK_PAIR);
+    int u = __shfl_sync(0xffffffffu, b, 0) + LF_WALK_PAIR * lane;
     int spare = LF_WALK_PAIR - 1;
-    for (int t = __shfl_sync(0xffffffffu, b, 0) + LF_WALK_PAIR * lane; t < 2 * cnt;) {
+    for (int t = walk_of(u); t < 2 * cnt;) {
         const int i = t >> 1, f = t & 1;
         const int32_t sv = __ldcg(a.list1 + i);
         int2 nbs;
@@ -3248,14 +3263,15 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
         k[f] = K;
         if (spare > 0) {  // the other walk of the same grab
             spare--;
-            t++;
+            t = walk_of(++u);
             continue;
         }
         const unsigned act = __activemask();
         const int ld = __ffs(act) - 1;
         int nb = 0;
-        if (lane == ld) nb = atomicAdd(&a.ctl[kCtlWalk], LF_WALK_PAIR * __popc(act));
-        t = __shfl_sync(act, nb, ld) + LF_WALK_PAIR * __popc(act & ((1u << lane) - 1u));
+        if (lane == ld) nb = atomicAdd(ctr, LF_WALK_PAIR * __popc(act));
+        u = __shfl_sync(act, nb, ld) + LF_WALK_PAIR * __popc(act & ((1u << lane) - 1u));
+        t = walk_of(u);
         spare = LF_WALK_PAIR - 1;
     }
 }
