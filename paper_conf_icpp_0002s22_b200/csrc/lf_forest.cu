@@ -70,7 +70,6 @@ constexpr int kCtlNcyc = 131;     // broken cycles (single-pass forest)
 constexpr int kCtlGridBar = 133;  // arrival counter of k_red_full's grid barrier
 constexpr int kCtlBad = 135;      // the tile path met a malformed factor: later kernels leave
 constexpr int kCtlBadGrs = 136;   // a ruling-set walk met one (bounded; records stay well formed)
-constexpr int kCtlWalk = 137;     // next walk handed out by k_grs_walk (dynamic schedule)
 constexpr int kCtlCycMax = 138;   // longest splitter-free cycle (lf_forest_stats)
 #ifndef LF_WALK_CTRS
 #define LF_WALK_CTRS 4
