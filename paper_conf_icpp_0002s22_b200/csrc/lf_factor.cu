@@ -1556,23 +1556,43 @@ __device__ __forceinline__ void rows_propose(const RowsArgs& a, int k, bool char
     unsigned long long my_live = 0, my_nnz = 0;
     int my_prop = 0;
     int qcnt = 0;
-    int64_t i0 = wg * 32;
-    int32_t vn = (i0 + lane < cnt) ? __ldcg(wl + i0 + lane) : -1;
-    for (; i0 < cnt; i0 += nw * 32) {
-        const int32_t v = vn;
-        const int64_t i1 = i0 + nw * 32;
-        vn = (i1 + lane < cnt) ? __ldcg(wl + i1 + lane) : -1;  // the next entries, in flight
-        const bool valid = v >= 0;
-        uint32_t st = 0;
-        int64_t rs = 0, re = 0;
-        int32_t p[NN];
-        if (valid) {  // live: deg < n, so pi's unused slots hold -1
+    // a two-deep software pipeline over the worklist: the next 32 rows' state, row extent and
+    // confirmed slots are loaded while this iteration's batches run (the loads only block at
+    // the loop's back edge), and the ids after them are in flight as well
+    auto fetch = [&](int32_t v, uint32_t& st, int64_t& rs, int64_t& re, int32_t (&p)[NN]) {
+        st = 0;
+        rs = re = 0;
+#pragma unroll
+        for (int s2 = 0; s2 < NN; s2++) p[s2] = -1;
+        if (v >= 0) {  // live: deg < n, so pi's unused slots hold -1
             st = __ldcg(a.state + v);
             rs = __ldg(a.rowptr + (v - a.row_base));
             re = __ldg(a.rowptr + (v - a.row_base) + 1);
 #pragma unroll
             for (int s2 = 0; s2 < NN; s2++) p[s2] = __ldcg(a.pi + (int64_t)v * NN + s2);
         }
+    };
+    int64_t i0 = wg * 32;
+    int32_t vc = (i0 + lane < cnt) ? __ldcg(wl + i0 + lane) : -1;
+    int32_t vn = (i0 + nw * 32 + lane < cnt) ? __ldcg(wl + i0 + nw * 32 + lane) : -1;
+    uint32_t stc;
+    int64_t rsc, rec;
+    int32_t pc[NN];
+    fetch(vc, stc, rsc, rec, pc);
+    for (; i0 < cnt; i0 += nw * 32) {
+        const int32_t v = vc;
+        const bool valid = v >= 0;
+        const uint32_t st = stc;
+        const int64_t rs = rsc, re = rec;
+        int32_t p[NN];
+#pragma unroll
+        for (int s2 = 0; s2 < NN; s2++) p[s2] = pc[s2];
+        // the next iteration's rows (ids already here) and the ids after them
+        const int64_t i2 = i0 + 2 * nw * 32;
+        const int32_t vnn = (i2 + lane < cnt) ? __ldcg(wl + i2 + lane) : -1;
+        fetch(vn, stc, rsc, rec, pc);
+        vc = vn;
+        vn = vnn;
         const bool lng = valid && (re - rs) > a.defer_len;
         {   // long rows: a CTA per row after the barrier
             const unsigned m = __ballot_sync(0xffffffffu, lng);
