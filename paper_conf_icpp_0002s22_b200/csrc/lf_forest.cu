@@ -941,7 +941,7 @@ struct ForestArgs {
     int grs_shift;         // hashed splitter density 2^-(32 - grs_shift)
     int4* grs_meet;        // [2N] per (vertex, slot): the partial window of the walk that stopped
     uint64_t* grs_meetk;   //   there looking along that slot: (item, R, DK, 0) and K
-    int2* grs_mstop;       // [2 cnt] (last, next) of a walk that met its partner, (-1, -1) final
+    int4* grs_mstop;       // [2 cnt] (last, next | slot << 31, stop key) of a walk that met its partner; x = -1: final
     int4* grs_rout;        // [N] (perm, a, b, c) at the new index (the meet records' storage, free by then)
     int4* grs_desc;        // [2 (cnt + cycles)] walk descriptors (k_grs_desc); cnt + cycles <= N
 };
@@ -2925,7 +2925,7 @@ size_t forest_ws_carve(Carve& c, int64_t N, ForestWs* w, bool with_grs) {
     t.grs_rec = c.take<int4>(ng);  // one 16-byte record per vertex
     t.grs_meet = c.take<int4>(2 * ng);
     t.grs_meetk = c.take<uint64_t>(2 * ng);
-    t.grs_mstop = c.take<int2>(2 * ng);
+    t.grs_mstop = c.take<int4>(2 * ng);
     t.grs_bits = c.take<uint32_t>(ng / 32 + 1);
     t.grs_cyc = c.take<int4>(ng / 3 + 1 + kCycStripes);  // kCycStripes * grs_cyc_cap(N)
     t.grs_cyck = c.take<uint64_t>(ng / 3 + 1 + kCycStripes);
@@ -3206,7 +3206,7 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
         const int32_t x = f ? nbs.y : nbs.x;
         int32_t tgt, R = 0, DK = 0;
         uint64_t K = KEY_INF;
-        int2 stop = make_int2(-1, -1);
+        int4 stop = make_int4(-1, -1, 0, 0);
         if (x < 0) {
             tgt = -(sv + 1);  // a path end: marker
         } else {
@@ -3225,9 +3225,14 @@ __global__ void __launch_bounds__(256) k_grs_walk(ForestArgs a) {
                 float2 wc;
                 grs_load(a, cur, nbc, wc);
                 const bool spl = hs || nbc.x < 0 || nbc.y < 0;  // a path end's bit was set by the pack
-                if (!spl && ((old >> (cur & 31)) & 1u)) {  // the partner's: met (its record is not used)
+                if (!spl && ((old >> (cur & 31)) & 1u)) {  // the partner's: met (only its slots are used)
                     walk_leave(a, t, prev, sp, R, K, DK);
-                    stop = make_int2(prev, cur);
+                    // the stop edge's key and cur's slot toward prev, for k_grs_meet (cur's
+                    // slots are intact: a claim overwrites the |w| half only)
+                    const uint64_t ks = edge_key(prev, cur, wpc, prev < cur ? nbp : nbc);
+                    const uint32_t sn = nbc.x == prev ? 0u : 1u;
+                    stop = make_int4(prev, (int32_t)((uint32_t)cur | (sn << 31)), (int32_t)(uint32_t)ks,
+                                     (int32_t)(uint32_t)(ks >> 32));
                     tgt = cur;
                     break;
                 }
@@ -3282,15 +3287,13 @@ __global__ void __launch_bounds__(256) k_grs_meet(ForestArgs a) {
     pdl_wait();
     const int cnt = __ldcg(&a.ctl[kCtlCnt1]);
     for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 2 * cnt; t += gridDim.x * blockDim.x) {
-        const int2 st = __ldcg(a.grs_mstop + t);
+        const int4 st = __ldcg(a.grs_mstop + t);
         if (st.x < 0) continue;
         const int i = t >> 1, f = t & 1;
-        const int32_t last = st.x, nxt = st.y;
-        // both records were claimed (their |w| half overwritten): the factor arrays themselves
-        const int2 nbl = __ldg(a.pi2 + last), nbn = __ldg(a.pi2 + nxt);
-        const float2 wl = __ldg(a.pi2_w + last), wn = __ldg(a.pi2_w + nxt);
-        const int sl = nbl.x == nxt ? 0 : 1;   // last's slot toward nxt
-        const int sn = nbn.x == last ? 0 : 1;  // nxt's slot toward last: the partner's key
+        // the walk left (last, nxt, nxt's slot toward last, the stop edge's key)
+        const int32_t last = st.x, nxt = (int32_t)((uint32_t)st.y & 0x7FFFFFFFu);
+        const int sn = (int)((uint32_t)st.y >> 31);
+        const uint64_t kstop = (uint64_t)(uint32_t)st.z | ((uint64_t)(uint32_t)st.w << 32);
         const int4 pm = __ldcg(a.grs_meet + 2 * (int64_t)nxt + sn);
         const uint64_t pk = __ldcg(a.grs_meetk + 2 * (int64_t)nxt + sn);
         int32_t* q = reinterpret_cast<int32_t*>(a.cq + i);
@@ -3304,7 +3307,7 @@ __global__ void __launch_bounds__(256) k_grs_meet(ForestArgs a) {
             q[f] = -(__ldcg(a.list1 + i) + 1);
             continue;
         }
-        win_append(R, K, DK, 1, edge_key(last, nxt, sl ? wl.y : wl.x, last < nxt ? nbl : nbn), last < nxt ? 1 : 0);
+        win_append(R, K, DK, 1, kstop, last < nxt ? 1 : 0);
         win_append(R, K, DK, pm.y, pk, pk == KEY_INF ? 0 : 2 * pm.y - 1 - pm.z);
         q[f] = __ldcg(a.list1 + (pm.x >> 1));
         r[f] = R;

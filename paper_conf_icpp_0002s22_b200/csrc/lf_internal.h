@@ -141,7 +141,7 @@ struct ForestWs {
     int4* grs_rec;         // [N] 16-byte per-vertex records (lf_forest.cu grs_load)
     int4* grs_meet;        // [2N] meet records per (vertex, slot)
     uint64_t* grs_meetk;
-    int2* grs_mstop;       // [2N] per walk
+    int4* grs_mstop;       // [2N] per walk
     uint32_t* grs_bits;    // [N/32 + 1] splitter or visited by a walk
     int4* grs_cyc;         // [N/3 + 1] (lowest vertex, DK, L, 0) of a cycle without splitters
     uint64_t* grs_cyck;    // [N/3 + 1] its weakest key
